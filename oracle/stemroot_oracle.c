@@ -1,0 +1,566 @@
+/*
+ * stemroot_oracle.c -- TEST INFRASTRUCTURE ONLY (see stemroot_oracle.h).
+ *
+ * A plain, slow, single-threaded implementation of the STEM+ROOT sampling
+ * plan, in the order of PAPER.md §3 and the normative algorithm recorded in
+ * DESIGN.md §3 ("Readings").  Build: gcc -O2 -std=c11 -ffp-contract=off.
+ * Every fp64 expression is written in the order DESIGN.md fixes, and
+ * -ffp-contract=off keeps gcc from fusing a*b+c into an FMA.
+ *
+ * It shares no code with the CUDA library.  Nothing in the product path may
+ * load this file.
+ */
+#include "stemroot_oracle.h"
+
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+typedef unsigned __int128 u128;
+typedef __int128 i128;
+
+/* ------------------------------------------------------------------------ */
+/* Exact integer helpers                                                     */
+/* ------------------------------------------------------------------------ */
+
+/* Correctly rounded conversion of a 128-bit unsigned integer to double.
+ * gcc's (double)(unsigned __int128) is exact-then-round-to-nearest. */
+static double rn128(u128 v) { return (double)v; }
+static double rn64(uint64_t v) { return (double)v; }
+
+double or_u128_to_double(uint64_t lo, uint64_t hi) {
+    return rn128(((u128)hi << 64) | lo);
+}
+
+/* schoolbook multiply of little-endian 64-bit limb arrays: out[na+nb] */
+static void limb_mul(const uint64_t *a, int na, const uint64_t *b, int nb, uint64_t *out) {
+    for (int i = 0; i < na + nb; i++) out[i] = 0;
+    for (int i = 0; i < na; i++) {
+        uint64_t carry = 0;
+        for (int j = 0; j < nb; j++) {
+            u128 cur = (u128)a[i] * b[j] + out[i + j] + carry;
+            out[i + j] = (uint64_t)cur;
+            carry = (uint64_t)(cur >> 64);
+        }
+        out[i + nb] = carry;
+    }
+}
+
+/* compare little-endian limb arrays of equal length: -1, 0, +1 */
+static int limb_cmp(const uint64_t *a, const uint64_t *b, int n) {
+    for (int i = n - 1; i >= 0; i--) {
+        if (a[i] != b[i]) return a[i] < b[i] ? -1 : 1;
+    }
+    return 0;
+}
+
+/* Split-score comparison for the 2-means cut (R5):
+ * score(k) = D_k^2 / p_k with D_k = n*S_L(k) - S*k, p_k = k*(n-k).
+ * Compare D_a^2 * p_b against D_b^2 * p_a exactly (|D| < 2^96, p < 2^64:
+ * both products < 2^256).  Returns -1/0/+1 for score_a <,=,> score_b. */
+static int score_cmp(u128 absDa, uint64_t pa, u128 absDb, uint64_t pb) {
+    uint64_t da[2] = {(uint64_t)absDa, (uint64_t)(absDa >> 64)};
+    uint64_t db[2] = {(uint64_t)absDb, (uint64_t)(absDb >> 64)};
+    uint64_t da2[4], db2[4], lhs[5], rhs[5];
+    limb_mul(da, 2, da, 2, da2);
+    limb_mul(db, 2, db, 2, db2);
+    limb_mul(da2, 4, &pb, 1, lhs);
+    limb_mul(db2, 4, &pa, 1, rhs);
+    return limb_cmp(lhs, rhs, 5);
+}
+
+/* ------------------------------------------------------------------------ */
+/* Exact sum of non-negative doubles (R12)                          */
+/* A fixed-point accumulator of 32-bit digits; value = acc * 2^-OR_FIX_LSB.   */
+/* ------------------------------------------------------------------------ */
+#define OR_FIX_LSB 1100            /* covers every positive double's LSB (>= 2^-1074) */
+#define OR_FIX_DIGITS 72           /* 72*32 = 2304 bits: 2^-1100 .. 2^1204            */
+
+typedef struct { uint32_t d[OR_FIX_DIGITS]; } fixacc;
+
+static void fix_add(fixacc *acc, double x) {
+    if (!(x > 0.0)) return;                 /* zero contributes nothing */
+    int e;
+    double fr = frexp(x, &e);               /* x = fr * 2^e, fr in [0.5,1) */
+    uint64_t mant = (uint64_t)ldexp(fr, 53);/* exact 53-bit integer       */
+    int shift = e - 53 + OR_FIX_LSB;        /* x = mant * 2^(e-53)        */
+    /* add mant << shift, 32 bits at a time, propagating carries */
+    int digit = shift / 32, off = shift % 32;
+    u128 v = (u128)mant << off;             /* at most 53+31 = 84 bits    */
+    uint64_t carry = 0;
+    for (int i = digit; i < OR_FIX_DIGITS; i++) {
+        uint64_t add = (uint64_t)(v & 0xffffffffu);
+        v >>= 32;
+        uint64_t s = (uint64_t)acc->d[i] + add + carry;
+        acc->d[i] = (uint32_t)s;
+        carry = s >> 32;
+        if (v == 0 && carry == 0) break;
+    }
+}
+
+/* round-to-nearest-even of the accumulator to double */
+static double fix_round(const fixacc *acc) {
+    int top = -1;
+    for (int i = OR_FIX_DIGITS - 1; i >= 0; i--) if (acc->d[i]) { top = i; break; }
+    if (top < 0) return 0.0;
+    int msb = top * 32 + (31 - __builtin_clz(acc->d[top]));   /* bit index of MSB */
+    /* collect bits [msb-63, msb] into a 64-bit word, sticky-OR the rest */
+    int lo_bit = msb - 63;
+    uint64_t word = 0;
+    int sticky = 0;
+    for (int b = msb; b >= 0; b--) {
+        int bit = (acc->d[b / 32] >> (b % 32)) & 1;
+        if (b >= lo_bit) word = (word << 1) | (uint64_t)bit;
+        else if (bit) { sticky = 1; break; }
+    }
+    if (lo_bit < 0) lo_bit = 0;   /* fewer than 64 significant bits: word is exact */
+    word |= (uint64_t)sticky;   /* 11 guard bits below the 53 kept: sticky is enough */
+    return ldexp(rn64(word), lo_bit - OR_FIX_LSB);
+}
+
+double or_exact_sum(const double *x, uint64_t n) {
+    fixacc *acc = calloc(1, sizeof(fixacc));
+    if (!acc) return NAN;
+    for (uint64_t i = 0; i < n; i++) fix_add(acc, x[i]);
+    double r = fix_round(acc);
+    free(acc);
+    return r;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Philox4x32-10 (Random123), used for sampling with replacement    */
+/* ------------------------------------------------------------------------ */
+void or_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out[4]) {
+    uint32_t x0 = ctr[0], x1 = ctr[1], x2 = ctr[2], x3 = ctr[3];
+    uint32_t k0 = key[0], k1 = key[1];
+    for (int round = 0; round < 10; round++) {
+        uint64_t p0 = (uint64_t)0xD2511F53u * x0;
+        uint64_t p1 = (uint64_t)0xCD9E8D57u * x2;
+        uint32_t y0 = (uint32_t)(p1 >> 32) ^ x1 ^ k0;
+        uint32_t y1 = (uint32_t)p1;
+        uint32_t y2 = (uint32_t)(p0 >> 32) ^ x3 ^ k1;
+        uint32_t y3 = (uint32_t)p0;
+        x0 = y0; x1 = y1; x2 = y2; x3 = y3;
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+    out[0] = x0; out[1] = x1; out[2] = x2; out[3] = x3;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Inverse normal: AS241 (Wichura 1988) PPND16                               */
+/* ------------------------------------------------------------------------ */
+static double ppnd16(double p) {
+    double q = p - 0.5, r, val;
+    if (fabs(q) <= 0.425) {
+        r = 0.180625 - q * q;
+        val = q * (((((((2.5090809287301226727e+3 * r + 3.3430575583588128105e+4) * r +
+                        6.7265770927008700853e+4) * r + 4.5921953931549871457e+4) * r +
+                      1.3731693765509461125e+4) * r + 1.9715909503065514427e+3) * r +
+                    1.3314166789178437745e+2) * r + 3.3871328727963666080e0) /
+              (((((((5.2264952788528545610e+3 * r + 2.8729085735721942674e+4) * r +
+                    3.9307895800092710610e+4) * r + 2.1213794301586595867e+4) * r +
+                  5.3941960214247511077e+3) * r + 6.8718700749205790830e+2) * r +
+                4.2313330701600911252e+1) * r + 1.0);
+        return val;
+    }
+    r = (q < 0) ? p : 1.0 - p;
+    r = sqrt(-log(r));
+    if (r <= 5.0) {
+        r -= 1.6;
+        val = (((((((7.74545014278341407640e-4 * r + 2.27238449892691845833e-2) * r +
+                    2.41780725177450611770e-1) * r + 1.27045825245236838258e0) * r +
+                  3.64784832476320460504e0) * r + 5.76949722146069140550e0) * r +
+                4.63033784615654529590e0) * r + 1.42343711074968357734e0) /
+              (((((((1.05075007164441684324e-9 * r + 5.47593808499534494600e-4) * r +
+                    1.51986665636164571966e-2) * r + 1.48103976427480074590e-1) * r +
+                  6.89767334985100004550e-1) * r + 1.67638483018380384940e0) * r +
+                2.05319162663775882187e0) * r + 1.0);
+    } else {
+        r -= 5.0;
+        val = (((((((2.01033439929228813265e-7 * r + 2.71155556874348757815e-5) * r +
+                    1.24266094738807843860e-3) * r + 2.65321895265761230930e-2) * r +
+                  2.96560571828504891230e-1) * r + 1.78482653991729133580e0) * r +
+                5.46378491116411436990e0) * r + 6.65790464350110377720e0) /
+              (((((((2.04426310338993978564e-15 * r + 1.42151175831644588870e-7) * r +
+                    1.84631831751005468180e-5) * r + 7.86869131145613259100e-4) * r +
+                  1.48753612908506148525e-2) * r + 1.36929880922735805310e-1) * r +
+                5.99832206555887937690e-1) * r + 1.0);
+    }
+    return (q < 0.0) ? -val : val;
+}
+
+/* Two-sided z for confidence 1 - alpha: z = Phi^-1(1 - alpha/2). */
+double or_z_from_conf(double conf) {
+    if (!(conf > 0.0 && conf < 1.0)) return NAN;
+    return ppnd16(1.0 - (1.0 - conf) / 2.0);
+}
+
+/* ------------------------------------------------------------------------ */
+/* Cluster moments over a sorted range (n, S = sum t, Q = sum t^2)           */
+/* ------------------------------------------------------------------------ */
+typedef struct { uint64_t n, S; u128 Q; } moments;
+
+static moments range_moments(const uint32_t *t, uint64_t lo, uint64_t hi) {
+    moments m = {hi - lo, 0, 0};
+    for (uint64_t i = lo; i < hi; i++) {
+        m.S += t[i];
+        m.Q += (u128)t[i] * t[i];
+    }
+    return m;
+}
+
+/* V = n*Q - S^2 = n^2 sigma^2 (population sigma, R3) */
+static u128 moments_V(moments m) { return (u128)m.n * m.Q - (u128)m.S * m.S; }
+
+/* ------------------------------------------------------------------------ */
+/* ROOT sub-clustering: exact optimal 1-D 2-means (R5)        */
+/* ------------------------------------------------------------------------ */
+/* Cut k in [1, n-1] places t[lo..lo+k) left, t[lo+k..hi) right.  Only cuts
+ * between distinct values are candidates.  Maximises D^2/(k(n-k)) exactly;
+ * ties go to the smallest k.  Returns 0 when no candidate exists. */
+static uint64_t best_cut(const uint32_t *t, uint64_t lo, uint64_t hi, uint64_t S) {
+    uint64_t n = hi - lo, best_k = 0, best_p = 0;
+    u128 best_absD = 0;
+    uint64_t SL = 0;
+    for (uint64_t k = 1; k < n; k++) {
+        SL += t[lo + k - 1];
+        if (!(t[lo + k - 1] < t[lo + k])) continue;
+        i128 D = (i128)((u128)n * SL) - (i128)((u128)S * k);
+        u128 absD = D < 0 ? (u128)(-D) : (u128)D;
+        uint64_t p = k * (n - k);
+        if (best_k == 0 || score_cmp(absD, p, best_absD, best_p) > 0) {
+            best_k = k; best_absD = absD; best_p = p;
+        }
+    }
+    return best_k;
+}
+
+uint64_t or_best_cut(const uint32_t *t_sorted, uint64_t n) {
+    if (n < 2) return 0;
+    moments m = range_moments(t_sorted, 0, n);
+    return best_cut(t_sorted, 0, n, m.S);
+}
+
+/* ------------------------------------------------------------------------ */
+/* STEM sample sizes                                                          */
+/* ------------------------------------------------------------------------ */
+/* Eq. 3 in the fixed order of R9: x = (rn(V)/(rn(S)*rn(S))) * k2,
+ * k2 = (z/eps)^2, m = ceil(x), clamped to >= 1 when clamp. */
+static double eq3_m(u128 V, uint64_t S, double k2, int clamp) {
+    if (V == 0) return clamp ? 1.0 : 0.0;
+    double x = (rn128(V) / (rn64(S) * rn64(S))) * k2;
+    double m = ceil(x);
+    if (clamp && m < 1.0) m = 1.0;
+    return m;
+}
+
+double or_eq3_m(uint64_t n, uint64_t S, uint64_t Q_lo, uint64_t Q_hi, double eps, double z, int clamp) {
+    moments m = {n, S, ((u128)Q_hi << 64) | Q_lo};
+    double q = z / eps;
+    return eq3_m(moments_V(m), S, q * q, clamp);
+}
+
+/* Eq. 6 with the numerator of the derivation (reading R1):
+ * m_i = ceil( (sum_j sqrt(a_j b_j)) / c * sqrt(b_i / a_i) ),
+ * a_i = mu_i, b_i = V_i, c = (eps * T / z)^2. */
+static double eq6_one(double g, double mu, double V, int clamp) {
+    if (V == 0.0) return clamp ? 1.0 : 0.0;
+    double m = ceil(g * sqrt(V / mu));
+    if (clamp && m < 1.0) m = 1.0;
+    return m;
+}
+
+void or_eq6_m(uint32_t k, const double *mu, const double *V, double T, double eps, double z, double *m_out) {
+    double w = (eps * T) / z;
+    double c = w * w;
+    double *terms = calloc(k ? k : 1, sizeof(double));
+    for (uint32_t i = 0; i < k; i++) terms[i] = sqrt(mu[i] * V[i]);
+    double ssum = or_exact_sum(terms, k);
+    free(terms);
+    double g = ssum / c;
+    for (uint32_t i = 0; i < k; i++) m_out[i] = eq6_one(g, mu[i], V[i], 1);
+}
+
+/* ------------------------------------------------------------------------ */
+/* ROOT decision (Eq. 7 vs Eq. 8; readings R6-R9)                */
+/* ------------------------------------------------------------------------ */
+typedef struct { double tau_old, tau_new; uint64_t cut; int split; } decision;
+
+static decision root_decide(const uint32_t *t, uint64_t lo, uint64_t hi, double eps, double z,
+                            double k2, int clamp) {
+    decision d = {0.0, 0.0, 0, 0};
+    uint64_t n = hi - lo;
+    if (n < 2 || t[lo] == t[hi - 1]) return d;              /* R5: leaf */
+    moments all = range_moments(t, lo, hi);
+    uint64_t k = best_cut(t, lo, hi, all.S);
+    d.cut = k;
+    /* Eq. 7: tau_old = m * Xbar with m from Eq. 3 */
+    double mu = rn64(all.S) / rn64(all.n);
+    double m_old = eq3_m(moments_V(all), all.S, k2, clamp);
+    d.tau_old = m_old * mu;
+    /* Eq. 8: tau_new = sum_i m_i Xbar_i with m_i from Eq. 6 over {L, R} */
+    moments L = range_moments(t, lo, lo + k), R = range_moments(t, lo + k, hi);
+    u128 VL = moments_V(L), VR = moments_V(R);
+    double muL = rn64(L.S) / rn64(L.n), muR = rn64(R.S) / rn64(R.n);
+    double w = (eps * rn64(all.S)) / z;
+    double c = w * w;
+    double ssum = sqrt(muL * rn128(VL)) + sqrt(muR * rn128(VR));
+    double g = ssum / c;
+    double mL = eq6_one(g, muL, rn128(VL), clamp);
+    double mR = eq6_one(g, muR, rn128(VR), clamp);
+    d.tau_new = mL * muL + mR * muR;
+    d.split = d.tau_new < d.tau_old;                        /* strict */
+    return d;
+}
+
+int or_root_decide(const uint32_t *t_sorted, uint64_t n, double eps, double z, int clamp,
+                   double *tau_old, double *tau_new, uint64_t *cut) {
+    double q = z / eps;
+    decision d = root_decide(t_sorted, 0, n, eps, z, q * q, clamp);
+    if (tau_old) *tau_old = d.tau_old;
+    if (tau_new) *tau_new = d.tau_new;
+    if (cut) *cut = d.cut;
+    return d.split;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Whole plan                                                                 */
+/* ------------------------------------------------------------------------ */
+typedef struct { uint32_t kid, t, row; } trow;
+
+static int trow_cmp(const void *a, const void *b) {
+    const trow *x = a, *y = b;
+    if (x->kid != y->kid) return x->kid < y->kid ? -1 : 1;
+    if (x->t != y->t) return x->t < y->t ? -1 : 1;
+    if (x->row != y->row) return x->row < y->row ? -1 : 1;
+    return 0;
+}
+
+typedef struct { uint32_t kid; uint64_t lo, hi; } leaf;
+typedef struct { leaf *v; uint64_t n, cap; } leafvec;
+
+static int leaf_push(leafvec *lv, leaf x) {
+    if (lv->n == lv->cap) {
+        uint64_t nc = lv->cap ? lv->cap * 2 : 1024;
+        leaf *nv = realloc(lv->v, nc * sizeof(leaf));
+        if (!nv) return -1;
+        lv->v = nv; lv->cap = nc;
+    }
+    lv->v[lv->n++] = x;
+    return 0;
+}
+
+typedef struct { uint64_t lo, hi; uint32_t depth; } work_item;
+typedef struct { work_item *v; uint64_t n, cap; } workvec;
+
+static int work_push(workvec *wv, uint64_t lo, uint64_t hi, uint32_t depth) {
+    if (wv->n == wv->cap) {
+        uint64_t nc = wv->cap ? wv->cap * 2 : 256;
+        work_item *nv = realloc(wv->v, nc * sizeof(work_item));
+        if (!nv) return -1;
+        wv->v = nv; wv->cap = nc;
+    }
+    work_item w = {lo, hi, depth};
+    wv->v[wv->n++] = w;
+    return 0;
+}
+
+void or_plan_free(or_plan *p) {
+    if (!p) return;
+    free(p->kernel_id); free(p->ordinal); free(p->lo_ns); free(p->hi_ns);
+    free(p->n); free(p->sum_ns); free(p->m); free(p->mean_ns); free(p->std_ns);
+    free(p->census); free(p->sample_row); free(p->sample_cluster); free(p->sample_weight);
+    free(p->est_metric);
+    free(p);
+}
+
+int or_plan_build(uint64_t n, uint32_t n_kernels, const uint32_t *kernel_id,
+                  const uint32_t *exec_ns, uint32_t n_metrics, const double *metrics,
+                  double eps, const or_opts *opts, or_plan **out) {
+    if (!out) return OR_E_INVAL;
+    *out = NULL;
+    if (!opts || !kernel_id || !exec_ns || n == 0) return OR_E_INVAL;
+    if (!(eps > 0.0 && eps < 1.0) || !(opts->z > 0.0) || !isfinite(opts->z)) return OR_E_INVAL;
+    if (n_metrics > 64 || (n_metrics > 0 && !metrics)) return OR_E_INVAL;
+    if (opts->scope < 0 || opts->scope > 2) return OR_E_INVAL;
+    if (n >= ((uint64_t)1 << 32)) return OR_E_RANGE;
+    for (uint64_t i = 0; i < n; i++) if (kernel_id[i] >= n_kernels) return OR_E_RANGE;
+
+    const double z = opts->z;
+    const double q = z / eps;
+    const double k2 = q * q;
+    const int clamp = opts->clamp_in_split ? 1 : 0;
+    int status = OR_OK;
+
+    /* Step 1: group by kernel: stable sort by (kernel_id, t), row breaks ties */
+    trow *rows = malloc(n * sizeof(trow));
+    uint32_t *t = malloc(n * sizeof(uint32_t));
+    uint32_t *row_of = malloc(n * sizeof(uint32_t));
+    leafvec leaves = {0, 0, 0};
+    workvec work = {0, 0, 0};
+    u128 *V = NULL;
+    double *mu = NULL, *mreal = NULL, *terms = NULL;
+    or_plan *p = calloc(1, sizeof(or_plan));
+    if (!rows || !t || !row_of || !p) { status = OR_E_NOMEM; goto fail; }
+    for (uint64_t i = 0; i < n; i++) {
+        rows[i].kid = kernel_id[i]; rows[i].t = exec_ns[i]; rows[i].row = (uint32_t)i;
+    }
+    qsort(rows, n, sizeof(trow), trow_cmp);
+    for (uint64_t i = 0; i < n; i++) { t[i] = rows[i].t; row_of[i] = rows[i].row; }
+
+    /* Step 2: ROOT on each group, depth-first, left before right,
+     * so leaves come out in canonical (kernel_id, lo) order. */
+    uint32_t max_depth = 0;
+    for (uint64_t g0 = 0; g0 < n;) {
+        uint64_t g1 = g0;
+        while (g1 < n && rows[g1].kid == rows[g0].kid) g1++;
+        uint32_t kid = rows[g0].kid;
+        if (work_push(&work, g0, g1, 0)) { status = OR_E_NOMEM; goto fail; }
+        while (work.n > 0) {
+            work_item w = work.v[--work.n];
+            if (w.depth > max_depth) max_depth = w.depth;
+            decision d = {0.0, 0.0, 0, 0};
+            if (opts->root) d = root_decide(t, w.lo, w.hi, eps, z, k2, clamp);
+            if (d.split) {
+                /* push right then left: the left child is visited first */
+                if (work_push(&work, w.lo + d.cut, w.hi, w.depth + 1) ||
+                    work_push(&work, w.lo, w.lo + d.cut, w.depth + 1)) { status = OR_E_NOMEM; goto fail; }
+            } else {
+                leaf lf = {kid, w.lo, w.hi};
+                if (leaf_push(&leaves, lf)) { status = OR_E_NOMEM; goto fail; }
+            }
+        }
+        g0 = g1;
+    }
+    p->max_depth = max_depth;
+
+    /* Leaf statistics (Fig. 6) */
+    uint64_t L = leaves.n;
+    p->n_clusters = L;
+    p->kernel_id = malloc(L * 4); p->ordinal = malloc(L * 4);
+    p->lo_ns = malloc(L * 4); p->hi_ns = malloc(L * 4);
+    p->n = malloc(L * 8); p->sum_ns = malloc(L * 8); p->m = malloc(L * 8);
+    p->mean_ns = malloc(L * 8); p->std_ns = malloc(L * 8); p->census = calloc(L, 1);
+    V = malloc(L * sizeof(u128));
+    mu = malloc(L * 8); mreal = malloc(L * 8); terms = malloc(L * 8);
+    if (!p->kernel_id || !p->ordinal || !p->lo_ns || !p->hi_ns || !p->n || !p->sum_ns ||
+        !p->m || !p->mean_ns || !p->std_ns || !p->census || !V || !mu || !mreal || !terms) {
+        status = OR_E_NOMEM; goto fail_leaves;
+    }
+    uint64_t T = 0;
+    for (uint64_t i = 0; i < L; i++) {
+        leaf lf = leaves.v[i];
+        moments m = range_moments(t, lf.lo, lf.hi);
+        p->kernel_id[i] = lf.kid;
+        p->ordinal[i] = (i > 0 && leaves.v[i - 1].kid == lf.kid) ? p->ordinal[i - 1] + 1 : 0;
+        p->lo_ns[i] = t[lf.lo];
+        p->hi_ns[i] = t[lf.hi - 1];
+        p->n[i] = m.n;
+        p->sum_ns[i] = m.S;
+        V[i] = moments_V(m);
+        mu[i] = rn64(m.S) / rn64(m.n);
+        p->mean_ns[i] = mu[i];
+        p->std_ns[i] = sqrt(rn128(V[i])) / rn64(m.n);
+        T += m.S;
+    }
+
+    /* Step 3: STEM sample sizes (Eq. 6 corrected, P:L169 + P:L464; R1, R10, R11) */
+    if (opts->scope == 2) {
+        for (uint64_t i = 0; i < L; i++) mreal[i] = eq3_m(V[i], p->sum_ns[i], k2, 1);
+        p->ssum = NAN;
+    } else {
+        /* scope 0: one set = all leaves; scope 1: one set per kernel */
+        uint64_t a = 0;
+        while (a < L) {
+            uint64_t b = a;
+            if (opts->scope == 0) b = L;
+            else while (b < L && p->kernel_id[b] == p->kernel_id[a]) b++;
+            uint64_t Tset = 0;
+            for (uint64_t i = a; i < b; i++) {
+                Tset += p->sum_ns[i];
+                terms[i - a] = sqrt(mu[i] * rn128(V[i]));
+            }
+            double ssum = or_exact_sum(terms, b - a);
+            double w = (eps * rn64(Tset)) / z;
+            double c = w * w;
+            double g = ssum / c;
+            for (uint64_t i = a; i < b; i++) mreal[i] = eq6_one(g, mu[i], rn128(V[i]), 1);
+            if (opts->scope == 0) p->ssum = ssum;
+            a = b;
+        }
+        if (opts->scope == 1) p->ssum = NAN;
+    }
+    uint64_t total_m = 0;
+    for (uint64_t i = 0; i < L; i++) {
+        double mi = mreal[i];
+        if (opts->census_cap && mi >= rn64(p->n[i])) { mi = rn64(p->n[i]); p->census[i] = 1; }
+        if (!(mi < 4294967296.0)) { status = OR_E_LIMIT; goto fail_leaves; }
+        p->m[i] = (uint64_t)mi;
+        total_m += p->m[i];
+        if (total_m >= ((uint64_t)1 << 32)) { status = OR_E_LIMIT; goto fail_leaves; }
+    }
+
+    /* Step 4: random sampling with replacement (R14) */
+    p->n_samples = total_m;
+    p->sample_row = malloc((total_m ? total_m : 1) * 4);
+    p->sample_cluster = malloc((total_m ? total_m : 1) * 4);
+    p->sample_weight = malloc((total_m ? total_m : 1) * 8);
+    p->n_metrics = n_metrics;
+    p->est_metric = calloc(n_metrics ? n_metrics : 1, 8);
+    if (!p->sample_row || !p->sample_cluster || !p->sample_weight || !p->est_metric) {
+        status = OR_E_NOMEM; goto fail_leaves;
+    }
+    const uint32_t key[2] = {(uint32_t)opts->seed, (uint32_t)(opts->seed >> 32)};
+    uint64_t s = 0;
+    u128 sum_q = 0;
+    double sum_frac = 0.0, sum_var = 0.0;
+    for (uint64_t i = 0; i < L; i++) {
+        leaf lf = leaves.v[i];
+        uint64_t ni = p->n[i], mi = p->m[i];
+        uint64_t U = 0;
+        double wgt = rn64(ni) / rn64(mi);
+        for (uint64_t j = 0; j < mi; j++) {
+            uint64_t pos;
+            if (p->census[i]) {
+                pos = lf.lo + j;
+            } else {
+                uint32_t ctr[4] = {(uint32_t)(j >> 1), p->ordinal[i], p->kernel_id[i], 0x53544D31u};
+                uint32_t x[4];
+                or_philox4x32_10(ctr, key, x);
+                uint64_t r = (j & 1) ? (((uint64_t)x[3] << 32) | x[2]) : (((uint64_t)x[1] << 32) | x[0]);
+                pos = lf.lo + (uint64_t)(((u128)r * ni) >> 64);
+            }
+            p->sample_row[s] = row_of[pos];
+            p->sample_cluster[s] = (uint32_t)i;
+            p->sample_weight[s] = wgt;
+            U += t[pos];
+            for (uint32_t c = 0; c < n_metrics; c++)
+                p->est_metric[c] += wgt * metrics[(uint64_t)c * n + row_of[pos]];
+            s++;
+        }
+        /* Step 5: extrapolation: t_i = N_i * mean of samples */
+        u128 num = (u128)ni * U;
+        sum_q += num / mi;
+        sum_frac += rn128(num % mi) / rn64(mi);
+        sum_var += rn128(V[i]) / rn64(mi);
+    }
+    p->est_total_ns = rn128(sum_q) + sum_frac;
+    p->true_total_ns = T;
+    /* predicted bound, Eq. 5 / Eq. 12: z * sqrt(sum V_i/m_i) / T */
+    p->bound = (T == 0) ? 0.0 : z * sqrt(sum_var) / rn64(T);
+    p->eps = eps;
+    p->z = z;
+
+    free(V); free(mu); free(mreal); free(terms);
+    free(work.v); free(leaves.v); free(rows); free(t); free(row_of);
+    *out = p;
+    return OR_OK;
+
+fail_leaves:
+    free(V); free(mu); free(mreal); free(terms);
+fail:
+    free(work.v); free(leaves.v); free(rows); free(t); free(row_of);
+    or_plan_free(p);
+    return status;
+}

@@ -1,0 +1,362 @@
+"""Pins for the oracle (oracle/stemroot_oracle.c) against things other than itself:
+hand-computed vectors from PAPER.md's formulas (tests/golden/*.json, each with
+its citation), closed forms, brute force on tiny inputs, library routines
+(math.fsum, Python's int->float, mpmath/scipy quantiles, Random123 KAT),
+invariants (Theorem 3.1, partition, census exactness) and Monte-Carlo
+coverage of the stated bound.  No GPU needed."""
+import itertools
+import math
+import random
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import oracle as O
+
+Z95 = 1.959963984540054  # scipy.stats.norm.ppf(0.975)
+
+
+# ----------------------------------------------------------------- Eq. 3 (P1)
+def test_eq3_hand_vectors(golden):
+    g = golden("eq3_hand.json")
+    for c in g["cases"]:
+        t = c["t"]
+        n, S, Q = len(t), sum(t), sum(x * x for x in t)
+        assert O.eq3_m(n, S, Q, c["eps"], c["z"]) == c["m"], c
+
+
+def test_eq3_matches_textbook_form():
+    # Eq. 3 is the textbook CLT sample size ceil((z*CoV/eps)^2) with population sigma.
+    rng = random.Random(7)
+    agree = 0
+    for _ in range(500):
+        t = [rng.randint(1, 10_000) for _ in range(rng.randint(2, 40))]
+        n, S, Q = len(t), sum(t), sum(x * x for x in t)
+        mu = S / n
+        sigma = math.sqrt(sum((x - mu) ** 2 for x in t) / n)
+        x = (1.96 * sigma / (mu * 0.05)) ** 2
+        m = O.eq3_m(n, S, Q, 0.05, 1.96)
+        assert abs(m - max(1, math.ceil(x))) <= 1
+        agree += m == max(1, math.ceil(x))
+    assert agree >= 495
+
+
+# ----------------------------------------------------------------- Eq. 6 (P2, P2b, P2c, P3)
+def test_eq6_hand_vectors(golden):
+    g = golden("eq6_hand.json")
+    for c in g["cases"]:
+        m = O.eq6_m(c["mu"], c["V"], c["T"], c["eps"], c["z"])
+        assert list(m) == c["m"], c
+        w = c["eps"] * c["T"] / c["z"]
+        assert w * w == pytest.approx(c["c"], rel=1e-15)
+        if "tau_joint" in c:
+            tau = sum(mi * a for mi, a in zip(m, c["mu"]))
+            assert tau == c["tau_joint"] <= c["tau_indep"]
+
+
+def test_eq6_printed_numerator_violates_bound():
+    # Reading R1: with the printed sqrt(sum a_j b_j) numerator the constraint Eq. 5 fails.
+    a, b, T = [2.0, 12.0], [6.0, 6.0], 42.0
+    c = (0.05 * T / 1.96) ** 2
+    printed = [math.sqrt(sum(x * y for x, y in zip(a, b))) / c * math.sqrt(bi / ai) for ai, bi in zip(a, b)]
+    derived = [sum(math.sqrt(x * y) for x, y in zip(a, b)) / c * math.sqrt(bi / ai) for ai, bi in zip(a, b)]
+    assert sum(bi / mi for bi, mi in zip(b, printed)) > c * 1.3
+    assert sum(bi / mi for bi, mi in zip(b, derived)) == pytest.approx(c, rel=1e-12)
+    m = O.eq6_m(a, b, T, 0.05, 1.96)
+    assert sum(bi / mi for bi, mi in zip(b, m)) <= c
+
+
+def test_eq6_single_cluster_reduces_to_eq3():
+    # P2b: for k = 1, (sqrt(ab)/c)*sqrt(b/a) = b/c = (z sigma/(eps mu))^2 -- Eq. 6 == Eq. 3.
+    rng = random.Random(11)
+    same = 0
+    for _ in range(400):
+        t = [rng.randint(1, 5000) for _ in range(rng.randint(2, 30))]
+        n, S, Q = len(t), sum(t), sum(x * x for x in t)
+        V = n * Q - S * S
+        if V == 0:
+            continue
+        m6 = O.eq6_m([S / n], [float(V)], S, 0.05, 1.96)[0]
+        m3 = O.eq3_m(n, S, Q, 0.05, 1.96)
+        assert abs(m6 - m3) <= 1
+        same += m6 == m3
+    assert same >= 390
+
+
+def test_eq6_kkt_conditions():
+    # App. 9.1: stationarity m*^2 a_i / b_i equal across i, Eq. 5 tight at m*,
+    # and the ceiled solution stays feasible.
+    rng = np.random.default_rng(3)
+    for _ in range(200):
+        k = int(rng.integers(2, 8))
+        a = rng.uniform(1, 1000, k)
+        b = rng.uniform(1, 1e6, k) * a
+        T = float(a.sum() * rng.uniform(5, 50))
+        eps, z = 0.05, 1.96
+        c = (eps * T / z) ** 2
+        mstar = np.sqrt(a * b).sum() / c * np.sqrt(b / a)
+        lam = mstar ** 2 * a / b
+        assert np.allclose(lam, lam[0], rtol=1e-12)
+        assert (b / mstar).sum() == pytest.approx(c, rel=1e-12)
+        m = O.eq6_m(a, b, T, eps, z)
+        assert np.all(m == np.maximum(1, np.ceil(mstar)))
+        assert (b / m).sum() <= c * (1 + 1e-12)
+
+
+def test_eq6_integer_brute_force():
+    # P2c: tau* <= tau_int_opt <= tau(ceil m*) < tau* + sum a_i ("minor sub-optimality").
+    rng = random.Random(5)
+    for _ in range(60):
+        k = rng.randint(1, 3)
+        a = [rng.randint(1, 20) for _ in range(k)]
+        b = [rng.randint(1, 400) for _ in range(k)]
+        T = sum(a) * rng.randint(2, 6)
+        eps, z = 0.25, 1.0
+        c = (eps * T / z) ** 2
+        mstar = [sum(math.sqrt(x * y) for x, y in zip(a, b)) / c * math.sqrt(bi / ai) for ai, bi in zip(a, b)]
+        tau_star = sum(m * x for m, x in zip(mstar, a))
+        m = O.eq6_m(a, b, T, eps, z)
+        tau_ceil = sum(mi * x for mi, x in zip(m, a))
+        assert sum(bi / mi for bi, mi in zip(b, m)) <= c * (1 + 1e-12)
+        hi = int(max(m)) + 2
+        best = min(sum(mi * x for mi, x in zip(ms, a))
+                   for ms in itertools.product(range(1, hi + 1), repeat=k)
+                   if sum(Fraction(bi) / mi for bi, mi in zip(b, ms)) <= Fraction(c))
+        assert tau_star - 1e-9 <= best <= tau_ceil + 1e-9
+        assert tau_ceil < tau_star + sum(a) + 1e-9 or max(mstar) < 1
+
+
+# ----------------------------------------------------------------- 2-means split (P4, P4b)
+def _sse(vals):
+    if not vals:
+        return Fraction(0)
+    mu = Fraction(sum(vals), len(vals))
+    return sum((Fraction(v) - mu) ** 2 for v in vals)
+
+
+def test_split_is_optimal_two_means_brute_force():
+    rng = random.Random(17)
+    for _ in range(600):
+        n = rng.randint(2, 10)
+        t = sorted(rng.choice([rng.randint(0, 6), rng.randint(0, 60)]) for _ in range(n))
+        k = O.best_cut(t)
+        if t[0] == t[-1]:
+            assert k == 0
+            continue
+        assert 1 <= k < n and t[k - 1] < t[k]
+        best = min(_sse([t[i] for i in range(n) if mask >> i & 1]) + _sse([t[i] for i in range(n) if not mask >> i & 1])
+                   for mask in range(1, 2 ** n - 1))
+        assert _sse(t[:k]) + _sse(t[k:]) == best
+        # smallest k among the optimal distinct-value cuts
+        first = min(j for j in range(1, n) if t[j - 1] < t[j] and _sse(t[:j]) + _sse(t[j:]) == best)
+        assert k == first
+
+
+def test_split_exact_tie(golden):
+    for c in golden("split_tie.json")["cases"]:
+        t = [c["s"] * x for x in c["base"]]
+        assert O.best_cut(t) == c["cut"]
+
+
+# ----------------------------------------------------------------- ROOT trees (P5, P5b)
+def test_root_worked_trees(golden):
+    g = golden("root_trees.json")
+    for tr in g["trees"]:
+        split, to, tn, cut = O.root_decide(tr["t"], tr["eps"], tr["z"])
+        r = tr["root"]
+        assert (split, to, tn, cut) == (r["split"], r["tau_old"], r["tau_new"], r["cut"])
+        for seed in (0, 1, 12345):
+            p = O.plan([0] * len(tr["t"]), tr["t"], 1, eps=tr["eps"], z=tr["z"], seed=seed)
+            assert [[int(a), int(b)] for a, b in zip(p["lo_ns"], p["hi_ns"])] == tr["leaves_lo_hi"]
+            assert list(p["m"]) == tr["m"]
+            assert p["est_total_ns"] == tr["est"] and p["bound"] == tr["bound"]
+    for st in g["subtrees"]:
+        split, to, tn, cut = O.root_decide(st["t"], st["eps"], st["z"])
+        assert (split, to, tn, cut) == (st["split"], st["tau_old"], st["tau_new"], st["cut"])
+
+
+def test_stem_only_two_kernels(golden):
+    c = golden("eq6_hand.json")["cases"][1]
+    p = O.plan([0, 0, 0, 0, 1, 1, 1, 1], [10, 20, 30, 40, 100, 100, 100, 300], 2, eps=0.05, z=1.96, root=0)
+    assert list(p["m"]) == c["m"]
+    assert p["ssum"] == pytest.approx(c["ssum"], rel=1e-15)
+    # bound = z sqrt(sum V/m)/T (Eq. 5 at the realised m), below eps
+    b = 1.96 * math.sqrt(2000 / 126 + 120000 / 397) / 700
+    assert p["bound"] == pytest.approx(b, rel=1e-14) and p["bound"] <= 0.05
+
+
+# ----------------------------------------------------------------- primitives
+def test_philox_kat(golden):
+    for c in golden("philox_kat.json")["cases"]:
+        out = O.philox4x32_10([int(x, 16) for x in c["ctr"]], [int(x, 16) for x in c["key"]])
+        assert out == [int(x, 16) for x in c["out"]]
+
+
+def test_z_from_conf_against_mpmath_and_scipy():
+    import mpmath
+    from scipy.stats import norm
+    mpmath.mp.dps = 40
+    for conf in (0.5, 0.8, 0.9, 0.95, 0.975, 0.99, 0.999, 0.999999, 1 - 1e-12):
+        p = 1 - (1 - conf) / 2
+        ref = float(mpmath.sqrt(2) * mpmath.erfinv(2 * mpmath.mpf(p) - 1))
+        z = O.z_from_conf(conf)
+        assert abs(z - ref) <= 4 * math.ulp(ref), (conf, z, ref)
+        assert z == pytest.approx(norm.ppf(p), rel=1e-14)
+    assert math.isnan(O.z_from_conf(1.0)) and math.isnan(O.z_from_conf(0.0))
+
+
+def test_u128_to_double_rounding():
+    rng = random.Random(23)
+    cases = [0, 1, 2 ** 53 + 1, 2 ** 64 - 1, 2 ** 64, 2 ** 64 + 2 ** 11, 2 ** 128 - 1,
+             (2 ** 53 + 1) << 70, ((2 ** 53 + 1) << 70) + 1, (2 ** 54 + 2) << 60, ((2 ** 54 + 2) << 60) + 1]
+    for _ in range(20000):
+        bits = rng.randint(1, 128)
+        v = rng.getrandbits(bits)
+        if rng.random() < 0.3:  # near-tie patterns: 1 bit beyond the mantissa, maybe sticky
+            top = max(bits - 54, 0)
+            v = (v >> top << top) | (1 << max(top - 1, 0)) if top else v
+        cases.append(v)
+    for v in cases:
+        assert O.u128_to_double(v) == float(v), v  # Python int->float is correctly rounded
+
+
+def test_exact_sum_against_fsum():
+    rng = np.random.default_rng(29)
+    for _ in range(50):
+        n = int(rng.integers(0, 3000))
+        x = np.exp(rng.uniform(-11, 55, n))  # the KKT terms live in [2^-16, 2^80)
+        x[rng.random(n) < 0.05] = 0.0
+        assert O.exact_sum(x) == math.fsum(x)
+    # cancellation-free but order-sensitive case: naive summation differs, exact does not
+    x = np.array([2.0 ** 80] + [1.0] * 5000 + [2.0 ** -16] * 7)
+    assert O.exact_sum(x) == math.fsum(x) == O.exact_sum(x[::-1])
+
+
+# ----------------------------------------------------------------- invariants (P6, P7, P8)
+def _random_trace(rng, n, k, max_t=2 ** 20):
+    kid = rng.integers(0, k, n).astype(np.uint32)
+    centers = rng.integers(1000, max_t, (k, 3))
+    peak = rng.integers(0, 3, n)
+    t = (centers[kid, peak] * rng.lognormal(0, 0.05, n)).astype(np.uint64)
+    return kid, np.minimum(t, 2 ** 32 - 1).astype(np.uint32)
+
+
+@pytest.mark.parametrize("scope", [0, 1, 2])
+@pytest.mark.parametrize("eps", [0.01, 0.05, 0.2])
+def test_plan_invariants(scope, eps):
+    rng = np.random.default_rng(int(eps * 1000) + scope)
+    kid, t = _random_trace(rng, 4000, 7)
+    p = O.plan(kid, t, 7, eps=eps, z=Z95, seed=3, scope=scope)
+    L = len(p["n"])
+    # partition: leaves cover each group, sum n = N, no time value split across two leaves
+    assert int(p["n"].sum()) == len(t)
+    assert p["true_total_ns"] == int(t.astype(np.uint64).sum())
+    for k in range(7):
+        idx = np.nonzero(p["kernel_id"] == k)[0]
+        sel = np.sort(t[kid == k])
+        assert list(p["ordinal"][idx]) == list(range(len(idx)))
+        assert np.all(p["hi_ns"][idx][:-1] < p["lo_ns"][idx][1:])
+        assert p["lo_ns"][idx][0] == sel[0] and p["hi_ns"][idx][-1] == sel[-1]
+        for i in idx:
+            mem = sel[(sel >= p["lo_ns"][i]) & (sel <= p["hi_ns"][i])]
+            assert len(mem) == p["n"][i] and int(mem.astype(np.uint64).sum()) == p["sum_ns"][i]
+    assert np.all(np.diff(p["kernel_id"].astype(np.int64)) >= 0)
+    # bound: global scope obeys Eq. 5; per-kernel / per-leaf obey it by Theorem 3.1
+    assert p["bound"] <= eps
+    assert np.all(p["m"] >= 1)
+    # samples: ordered by cluster, each row belongs to its cluster, weight = n_i/m_i
+    assert len(p["sample_row"]) == int(p["m"].sum())
+    assert np.all(np.diff(p["sample_cluster"].astype(np.int64)) >= 0)
+    c = p["sample_cluster"]
+    rows = p["sample_row"]
+    assert np.all(kid[rows] == p["kernel_id"][c])
+    assert np.all((t[rows] >= p["lo_ns"][c]) & (t[rows] <= p["hi_ns"][c]))
+    assert np.allclose(p["sample_weight"], p["n"][c].astype(float) / p["m"][c])
+    assert L >= 7
+
+
+def test_leaves_invariant_to_row_order():
+    rng = np.random.default_rng(41)
+    kid, t = _random_trace(rng, 3000, 5)
+    a = O.plan(kid, t, 5)
+    perm = rng.permutation(len(t))
+    b = O.plan(kid[perm], t[perm], 5)
+    for key in ("kernel_id", "ordinal", "lo_ns", "hi_ns", "n", "sum_ns", "m"):
+        assert np.array_equal(a[key], b[key])
+
+
+def test_census_is_exact():
+    # P8: census_cap with a tiny eps takes every row once -> estimate == T exactly (north_star)
+    rng = np.random.default_rng(43)
+    kid, t = _random_trace(rng, 2000, 4)
+    met = np.vstack([t.astype(float), np.ones(len(t))])
+    p = O.plan(kid, t, 4, eps=1e-6, census_cap=1, root=0, metrics=met)
+    assert p["census"].all()
+    assert p["est_total_ns"] == float(p["true_total_ns"])
+    assert sorted(p["sample_row"]) == list(range(len(t)))
+    assert p["est_metric"][0] == pytest.approx(float(t.astype(np.float64).sum()), rel=1e-12)
+    assert p["est_metric"][1] == pytest.approx(len(t), rel=1e-12)
+    # with ROOT every leaf is either a census or constant (sigma = 0): still exact
+    p = O.plan(kid, t, 4, eps=1e-6, census_cap=1, metrics=met)
+    assert np.all((p["census"] == 1) | (p["lo_ns"] == p["hi_ns"]))
+    assert p["est_total_ns"] == float(p["true_total_ns"])
+
+
+def test_constant_and_singleton_kernels_are_exact():
+    kid = np.array([0, 0, 0, 1, 2, 2], np.uint32)
+    t = np.array([5, 5, 5, 9, 0, 0], np.uint32)
+    p = O.plan(kid, t, 3)
+    assert list(p["n"]) == [3, 1, 2] and list(p["m"]) == [1, 1, 1]
+    assert p["est_total_ns"] == 24.0 and p["bound"] == 0.0
+
+
+def test_error_codes():
+    with pytest.raises(O.OracleError) as e:
+        O.plan([0, 3], [1, 2], 3)
+    assert e.value.status == O.OR_E_RANGE
+    for eps in (0.0, 1.0, -1.0):
+        with pytest.raises(O.OracleError) as e:
+            O.plan([0], [1], 1, eps=eps)
+        assert e.value.status == O.OR_E_INVAL
+
+
+def test_literal_clamp_reading_differs_only_in_split_test():
+    # R7: clamp_in_split=0 uses literal ceilings (m may be 0 when sigma = 0) inside Eq. 7/8.
+    kid = np.zeros(20, np.uint32)
+    t = np.array([100] * 10 + [200] * 10, np.uint32)
+    for cl in (0, 1):
+        p = O.plan(kid, t, 1, clamp_in_split=cl, z=1.96)
+        assert list(p["n"]) == [10, 10] and list(p["m"]) == [1, 1]
+
+
+# ----------------------------------------------------------------- statistics (P9)
+def test_sample_positions_uniform():
+    # With replacement, uniform over the cluster: chi-square on a big cluster.
+    rng = np.random.default_rng(47)
+    t = rng.integers(1, 1000, 64).astype(np.uint32)
+    p = O.plan(np.zeros(64, np.uint32), t, 1, eps=0.002, root=0, seed=99)
+    rows = p["sample_row"]
+    assert len(rows) > 20000
+    counts = np.bincount(rows, minlength=64)
+    exp = len(rows) / 64
+    chi2 = ((counts - exp) ** 2 / exp).sum()
+    assert chi2 < 120  # 63 dof: p ~ 3e-5
+
+
+@pytest.mark.slow
+def test_monte_carlo_unbiased_and_coverage():
+    rng = np.random.default_rng(53)
+    kid, t = _random_trace(rng, 3000, 6)
+    # STEM only: m_i > 1, the CLT regime the paper models (Eq. 4/5)
+    R = 300
+    errs, cover = [], 0
+    for seed in range(R):
+        p = O.plan(kid, t, 6, eps=0.02, root=0, seed=seed)
+        T = p["true_total_ns"]
+        e = (p["est_total_ns"] - T) / T
+        errs.append(e)
+        cover += abs(e) <= p["bound"]
+    errs = np.array(errs)
+    assert abs(errs.mean()) < 4 * errs.std() / math.sqrt(R)
+    assert 0.89 <= cover / R <= 0.995
