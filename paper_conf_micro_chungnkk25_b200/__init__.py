@@ -1,0 +1,247 @@
+"""B200-native STEM+ROOT sampling-plan builder: thin Python binding.
+
+Argument marshalling only -- every step of the plan runs in the CUDA kernels
+of ``lib/libstemroot.so`` behind the C ABI declared in ``include/stemroot.h``
+(same function names).  There is no CPU path: if the library is missing or
+cannot find a GPU, every call raises.
+
+    import paper_conf_micro_chungnkk25_b200 as sr
+    ctx = sr.Context(0)
+    plan = ctx.plan(kernel_id, exec_ns, n_kernels, eps=0.05, conf=0.95)
+
+``kernel_id`` / ``exec_ns`` are uint32 data either as CUDA tensors (int32 or
+uint32 dtype, bytes reinterpreted) on the context's device, or as host numpy
+arrays (then the library copies them in).  PAPER.md citations: see
+include/stemroot.h.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_ROOT = os.path.dirname(_HERE)
+_CSRC = os.path.join(_HERE, "csrc")
+LIB_PATH = os.path.join(_HERE, "lib", "libstemroot.so")
+HEADER = os.path.join(_ROOT, "include", "stemroot.h")
+SOURCES = ["capi.cu", "sort.cu", "root.cu", "stem.cu"]
+NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "--fmad=false",
+              "--extended-lambda", "-Xcompiler", "-fPIC,-fvisibility=hidden", "-shared"]
+
+STEM_OK, STEM_E_INVAL, STEM_E_RANGE, STEM_E_NOMEM, STEM_E_CUDA, STEM_E_NCCL, STEM_E_LIMIT, STEM_E_STATE = \
+    0, -1, -2, -3, -4, -5, -6, -7
+
+
+def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile libstemroot.so for sm_100a in-tree (nvcc cross-compiles without a GPU)."""
+    srcs = [os.path.join(_CSRC, s) for s in SOURCES]
+    deps = srcs + [os.path.join(_CSRC, h) for h in os.listdir(_CSRC) if h.endswith((".cuh", ".h"))] + [HEADER]
+    if not force and os.path.exists(LIB_PATH) and os.path.getmtime(LIB_PATH) >= max(map(os.path.getmtime, deps)):
+        return LIB_PATH
+    os.makedirs(os.path.dirname(LIB_PATH), exist_ok=True)
+    cmd = ["nvcc"] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + ["-o", LIB_PATH] + srcs
+    subprocess.check_call(cmd, cwd=_CSRC)
+    return LIB_PATH
+
+
+# ------------------------------------------------------------------ ABI structs (mirror stemroot.h)
+class stem_trace(C.Structure):
+    _fields_ = [("n", C.c_uint64), ("n_kernels", C.c_uint32), ("kernel_id", C.c_void_p), ("exec_ns", C.c_void_p),
+                ("n_metrics", C.c_uint32), ("metrics", C.c_void_p), ("device", C.c_int)]
+
+
+class stem_opts(C.Structure):
+    _fields_ = [("seed", C.c_uint64), ("z", C.c_double), ("scope", C.c_int), ("root", C.c_int),
+                ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("stream", C.c_void_p)]
+
+
+class stem_cluster(C.Structure):
+    _fields_ = [("kernel_id", C.c_uint32), ("ordinal", C.c_uint32), ("lo_ns", C.c_uint32), ("hi_ns", C.c_uint32),
+                ("n", C.c_uint64), ("sum_ns", C.c_uint64), ("mean_ns", C.c_double), ("std_ns", C.c_double),
+                ("m", C.c_uint64), ("census", C.c_uint32), ("reserved", C.c_uint32)]
+
+
+CLUSTER_DTYPE = np.dtype([("kernel_id", "<u4"), ("ordinal", "<u4"), ("lo_ns", "<u4"), ("hi_ns", "<u4"),
+                          ("n", "<u8"), ("sum_ns", "<u8"), ("mean_ns", "<f8"), ("std_ns", "<f8"), ("m", "<u8"),
+                          ("census", "<u4"), ("reserved", "<u4")])
+assert CLUSTER_DTYPE.itemsize == C.sizeof(stem_cluster)
+
+
+class stem_plan(C.Structure):
+    _fields_ = [("n_clusters", C.c_uint64), ("clusters", C.POINTER(stem_cluster)), ("n_samples", C.c_uint64),
+                ("sample_row", C.POINTER(C.c_uint32)), ("sample_cluster", C.POINTER(C.c_uint32)),
+                ("sample_weight", C.POINTER(C.c_double)), ("est_total_ns", C.c_double),
+                ("true_total_ns", C.c_uint64), ("bound", C.c_double), ("eps", C.c_double), ("z", C.c_double),
+                ("n_metrics", C.c_uint32), ("est_metric", C.POINTER(C.c_double))]
+
+
+class stem_device_plan(C.Structure):
+    _fields_ = [("n_clusters", C.c_uint64), ("n_samples", C.c_uint64), ("clusters", C.c_void_p),
+                ("sample_row", C.c_void_p), ("sample_cluster", C.c_void_p), ("sample_weight", C.c_void_p),
+                ("est_total_ns", C.c_double), ("bound", C.c_double), ("eps", C.c_double), ("z", C.c_double),
+                ("true_total_ns", C.c_uint64), ("n_metrics", C.c_uint32), ("est_metric", C.POINTER(C.c_double))]
+
+
+class stem_stats(C.Structure):
+    _fields_ = [("key_bits", C.c_uint32), ("sort_passes", C.c_uint32), ("levels", C.c_uint32),
+                ("kernel_launches", C.c_uint32), ("active_rows", C.c_uint64), ("n_clusters", C.c_uint64),
+                ("n_samples", C.c_uint64), ("ssum", C.c_double)]
+
+
+EXPORTS = ["stem_default_opts", "stem_ctx_create", "stem_ctx_destroy", "stem_root_plan_ctx", "stem_root_plan",
+           "stem_ctx_device_plan", "stem_ctx_stats", "stem_plan_free", "stem_strerror", "stem_z_from_conf"]
+
+_lib = None
+
+
+def lib():
+    """Load libstemroot.so (raises if it was not built: there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} missing: run __graft_entry__.build() (no CPU fallback exists)")
+        L = C.CDLL(LIB_PATH)
+        P = C.POINTER
+        L.stem_default_opts.argtypes = [P(stem_opts)]
+        L.stem_ctx_create.argtypes = [C.c_int, P(C.c_void_p)]
+        L.stem_ctx_destroy.argtypes = [C.c_void_p]
+        L.stem_ctx_destroy.restype = None
+        L.stem_root_plan_ctx.argtypes = [C.c_void_p, P(stem_trace), C.c_double, C.c_double, P(stem_opts),
+                                         P(P(stem_plan))]
+        L.stem_root_plan.argtypes = [P(stem_trace), C.c_double, C.c_double, P(stem_opts), P(P(stem_plan))]
+        L.stem_ctx_device_plan.argtypes = [C.c_void_p, P(stem_device_plan)]
+        L.stem_ctx_stats.argtypes = [C.c_void_p, P(stem_stats)]
+        L.stem_plan_free.argtypes = [P(stem_plan)]
+        L.stem_plan_free.restype = None
+        L.stem_strerror.argtypes = [C.c_int]
+        L.stem_strerror.restype = C.c_char_p
+        L.stem_z_from_conf.argtypes = [C.c_double, P(C.c_double)]
+        _lib = L
+    return _lib
+
+
+class StemError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        super().__init__(f"{where}: {lib().stem_strerror(status).decode()} ({status})")
+        self.status = status
+
+
+def _check(st, where):
+    if st != STEM_OK:
+        raise StemError(st, where)
+
+
+def strerror(status: int) -> str:
+    return lib().stem_strerror(status).decode()
+
+
+def z_from_conf(conf: float) -> float:
+    z = C.c_double()
+    _check(lib().stem_z_from_conf(conf, C.byref(z)), "stem_z_from_conf")
+    return z.value
+
+
+def _arg(x, dtype):
+    """(pointer, device, keepalive) for a torch tensor or numpy array."""
+    try:
+        import torch
+        if isinstance(x, torch.Tensor):
+            if not x.is_contiguous():
+                raise ValueError("tensor must be contiguous")
+            return x.data_ptr(), (x.device.index if x.is_cuda else -1), x
+    except ImportError:
+        pass
+    a = np.ascontiguousarray(x).view(dtype) if np.asarray(x).dtype.itemsize == np.dtype(dtype).itemsize \
+        else np.ascontiguousarray(x, dtype=dtype)
+    return a.ctypes.data, -1, a
+
+
+def _plan_to_numpy(p: stem_plan) -> dict:
+    L, S = p.n_clusters, p.n_samples
+    cl = np.ctypeslib.as_array(C.cast(p.clusters, C.POINTER(C.c_uint8)), shape=(L * CLUSTER_DTYPE.itemsize,)) \
+        .view(CLUSTER_DTYPE).copy() if L else np.zeros(0, CLUSTER_DTYPE)
+
+    def arr(ptr, cnt, dt):
+        return np.ctypeslib.as_array(ptr, shape=(cnt,)).astype(dt, copy=True) if cnt else np.zeros(0, dt)
+    return dict(clusters=cl, sample_row=arr(p.sample_row, S, np.uint32),
+                sample_cluster=arr(p.sample_cluster, S, np.uint32), sample_weight=arr(p.sample_weight, S, np.float64),
+                est_total_ns=p.est_total_ns, true_total_ns=int(p.true_total_ns), bound=p.bound, eps=p.eps, z=p.z,
+                est_metric=arr(p.est_metric, p.n_metrics, np.float64))
+
+
+class Context:
+    """A stem_ctx: device workspace reused across plans (stem_ctx_create)."""
+
+    def __init__(self, device: int = 0):
+        self._h = C.c_void_p()
+        _check(lib().stem_ctx_create(device, C.byref(self._h)), "stem_ctx_create")
+        self.device = device
+
+    def close(self):
+        if self._h:
+            lib().stem_ctx_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def plan(self, kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, metrics=None,
+             seed: int = 0, z: float = 0.0, scope: int = 0, root: bool = True, clamp_in_split: bool = True,
+             census_cap: bool = False, stream=None, to_host: bool = True):
+        """stem_root_plan_ctx.  Returns the host plan as numpy arrays, or None when to_host=False
+        (the plan then stays on the device: see device_plan())."""
+        kp, kdev, k_keep = _arg(kernel_id, np.uint32)
+        tp, tdev, t_keep = _arg(exec_ns, np.uint32)
+        n = int(np.prod(getattr(k_keep, "shape", (0,))))
+        if kdev != tdev:
+            raise ValueError("kernel_id and exec_ns must live on the same device")
+        nm, mp, m_keep = 0, None, None
+        if metrics is not None:
+            mp, mdev, m_keep = _arg(metrics, np.float64)
+            if mdev != kdev:
+                raise ValueError("metrics must live with the trace")
+            nm = int(m_keep.shape[0]) if len(m_keep.shape) == 2 else 1
+        tr = stem_trace(n, n_kernels, kp, tp, nm, mp, kdev)
+        if stream is None and kdev >= 0:
+            import torch
+            stream = torch.cuda.current_stream(kdev).cuda_stream
+        o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
+                      stream or None)
+        out = C.POINTER(stem_plan)()
+        st = lib().stem_root_plan_ctx(self._h, C.byref(tr), eps, conf, C.byref(o),
+                                      C.byref(out) if to_host else None)
+        _check(st, "stem_root_plan_ctx")
+        del k_keep, t_keep, m_keep
+        if not to_host:
+            return None
+        res = _plan_to_numpy(out.contents)
+        lib().stem_plan_free(out)
+        return res
+
+    def device_plan(self) -> dict:
+        v = stem_device_plan()
+        _check(lib().stem_ctx_device_plan(self._h, C.byref(v)), "stem_ctx_device_plan")
+        return dict(n_clusters=v.n_clusters, n_samples=v.n_samples, clusters=v.clusters, sample_row=v.sample_row,
+                    sample_cluster=v.sample_cluster, sample_weight=v.sample_weight, est_total_ns=v.est_total_ns,
+                    bound=v.bound, eps=v.eps, z=v.z, true_total_ns=int(v.true_total_ns),
+                    est_metric=[v.est_metric[i] for i in range(v.n_metrics)])
+
+    def stats(self) -> dict:
+        s = stem_stats()
+        _check(lib().stem_ctx_stats(self._h, C.byref(s)), "stem_ctx_stats")
+        return {f: getattr(s, f) for f, _ in stem_stats._fields_}
+
+
+def plan(kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, device: int = 0, **kw):
+    """One-shot stem_root_plan through a temporary Context."""
+    ctx = Context(device)
+    try:
+        return ctx.plan(kernel_id, exec_ns, n_kernels, eps, conf, **kw)
+    finally:
+        ctx.close()

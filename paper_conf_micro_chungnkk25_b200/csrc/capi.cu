@@ -1,0 +1,329 @@
+// capi.cu -- the C ABI (include/stemroot.h): validation, workspace, stage
+// orchestration on one stream, host plan assembly.  All arithmetic of the
+// plan runs in the stage kernels (sort.cu, root.cu, stem.cu).
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+
+#include "internal.h"
+
+namespace sr {
+
+cudaError_t &last_cuda_error() {
+    static thread_local cudaError_t e = cudaSuccess;
+    return e;
+}
+
+int Ctx::ensure_all(uint64_t n, uint32_t K, uint32_t n_metrics) {
+    (void)n_metrics;
+    CKS(ensure(keys[0], cap_keys[0], sizeof(uint64_t) * n));
+    CKS(ensure(keys[1], cap_keys[1], sizeof(uint64_t) * n));
+    CKS(ensure(vals[0], cap_vals[0], sizeof(uint32_t) * n));
+    CKS(ensure(vals[1], cap_vals[1], sizeof(uint32_t) * n));
+    CKS(ensure(t_sorted, cap_ts, sizeof(uint32_t) * (n + 1)));
+    CKS(ensure(row_sorted, cap_rs, sizeof(uint32_t) * (n + 1)));
+    CKS(ensure(kid_count, cap_kc, sizeof(uint32_t) * ((uint64_t)K + 1)));
+    CKS(ensure(goff, cap_goff, sizeof(uint32_t) * ((uint64_t)K + 2)));
+    CKS(ensure(hist, cap_hist, sizeof(uint64_t) * 8 * 256));
+    CKS(ensure(scalars, cap_scalars, sizeof(DevScalars)));
+    CKS(ensure(scan_scratch, cap_scan, (scan_tiles((uint64_t)K + 2) + 1) * 32));
+    CKS(ensure(P1, cap_p1, sizeof(uint64_t) * (n + 1)));
+    CKS(ensure(P2, cap_p2, sizeof(u128) * (n + 1)));
+    CKS(ensure(flags, cap_flags, n + 16));
+    return STEM_OK;
+}
+
+template <class T>
+static void dfree(T *&p, size_t &cap) {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+}
+
+void Ctx::release() {
+    dfree(in_kid, cap_in_kid); dfree(in_t, cap_in_t); dfree(in_met, cap_in_met);
+    for (int i = 0; i < 2; i++) {
+        dfree(keys[i], cap_keys[i]); dfree(vals[i], cap_vals[i]);
+        dfree(f_lo[i], cap_flo[i]); dfree(f_hi[i], cap_fhi[i]); dfree(f_aoff[i], cap_faoff[i]);
+    }
+    dfree(t_sorted, cap_ts); dfree(row_sorted, cap_rs); dfree(kid_count, cap_kc); dfree(goff, cap_goff);
+    dfree(hist, cap_hist); dfree(sort_status, cap_status); dfree(scalars, cap_scalars);
+    dfree(scan_scratch, cap_scan); dfree(P1, cap_p1); dfree(P2, cap_p2);
+    dfree(cut, cap_cut); dfree(cnt_sz, cap_cntsz); dfree(split_part, cap_part); dfree(flags, cap_flags);
+    dfree(leaf_lo, cap_leaf_lo); dfree(leaf_m, cap_leaf_m); dfree(leaf_moff, cap_leaf_moff);
+    dfree(leaf_U, cap_leaf_U); dfree(leaf_census, cap_leaf_census); dfree(leaf_kid, cap_leaf_kid);
+    dfree(leaf_ord, cap_leaf_ord); dfree(fix_acc, cap_fix); dfree(kern_T, cap_kern_T); dfree(kern_g, cap_kern_g);
+    dfree(red_part, cap_red); dfree(out_clusters, cap_out_cl); dfree(out_row, cap_out_row);
+    dfree(out_cluster, cap_out_cluster); dfree(out_weight, cap_out_weight);
+}
+
+// z = Phi^-1(1 - q), q = (1-conf)/2: Acklam's rational initial guess for the
+// lower tail, refined by Halley steps on erfc (host; the oracle uses AS241).
+static double z_two_sided(double conf) {
+    const double q = 0.5 * (1.0 - conf);   // lower-tail probability, accurate for conf near 1
+    static const double a[] = {-3.969683028665376e+01, 2.209460984245205e+02, -2.759285104469687e+02,
+                               1.383577518672690e+02, -3.066479806614716e+01, 2.506628277459239e+00};
+    static const double b[] = {-5.447609879822406e+01, 1.615858368580409e+02, -1.556989798598866e+02,
+                               6.680131188771972e+01, -1.328068155288572e+01};
+    static const double c[] = {-7.784894002430293e-03, -3.223964580411365e-01, -2.400758277161838e+00,
+                               -2.549732539343734e+00, 4.374664141464968e+00, 2.938163982698783e+00};
+    static const double d[] = {7.784695709041462e-03, 3.224671290700398e-01, 2.445134137142996e+00,
+                               3.754408661907416e+00};
+    double x;
+    if (q < 0.02425) {
+        const double r = std::sqrt(-2.0 * std::log(q));
+        x = (((((c[0] * r + c[1]) * r + c[2]) * r + c[3]) * r + c[4]) * r + c[5]) /
+            ((((d[0] * r + d[1]) * r + d[2]) * r + d[3]) * r + 1.0);
+    } else {
+        const double u = q - 0.5, r = u * u;
+        x = (((((a[0] * r + a[1]) * r + a[2]) * r + a[3]) * r + a[4]) * r + a[5]) * u /
+            (((((b[0] * r + b[1]) * r + b[2]) * r + b[3]) * r + b[4]) * r + 1.0);
+    }
+    for (int it = 0; it < 2; it++) {   // Halley on F(x) = Phi(x) - q, x < 0
+        const double e = 0.5 * std::erfc(-x / std::sqrt(2.0)) - q;
+        const double u = e * std::sqrt(2.0 * M_PI) * std::exp(0.5 * x * x);
+        x = x - u / (1.0 + 0.5 * x * u);
+    }
+    return -x;
+}
+
+static int validate(const stem_trace *tr, double eps, double conf, const stem_opts &o) {
+    if (!tr) return STEM_E_INVAL;
+    if (!(eps > 0.0 && eps < 1.0)) return STEM_E_INVAL;
+    if (!(o.z > 0.0) && !(conf > 0.0 && conf < 1.0)) return STEM_E_INVAL;
+    if (o.z < 0.0 || std::isnan(o.z) || std::isinf(o.z)) return STEM_E_INVAL;
+    if (o.scope < 0 || o.scope > 2) return STEM_E_INVAL;
+    if (tr->n == 0 || !tr->kernel_id || !tr->exec_ns) return STEM_E_INVAL;
+    if (tr->n_metrics > 64 || (tr->n_metrics > 0 && !tr->metrics)) return STEM_E_INVAL;
+    if (tr->n >= (1ull << 32)) return STEM_E_RANGE;
+    if (tr->n_kernels == 0 || tr->n_kernels > (1u << 24)) return STEM_E_RANGE;
+    return STEM_OK;
+}
+
+static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const stem_opts &o) {
+    c.have_plan = false;
+    c.launches = 0;
+    c.stats = stem_stats{};
+    CKS(validate(tr, eps, conf, o));
+    CK(cudaSetDevice(c.device));
+    if (tr->device >= 0 && tr->device != c.device) return STEM_E_INVAL;
+    c.stream = (cudaStream_t)o.stream;
+    const uint64_t n = tr->n;
+    const uint32_t K = tr->n_kernels, nm = tr->n_metrics;
+    double z = o.z;
+    if (!(z > 0.0)) {
+        z = z_two_sided(conf);
+        if (!(z > 0.0) || std::isinf(z)) return STEM_E_INVAL;
+    }
+    const double q = z / eps;
+    const double k2 = q * q;
+    CKS(c.ensure_all(n, K, nm));
+    const uint32_t *kid = tr->kernel_id, *t = tr->exec_ns;
+    const double *met = tr->metrics;
+    if (tr->device < 0) {   // host trace: copy in on the stream
+        CKS(c.ensure(c.in_kid, c.cap_in_kid, sizeof(uint32_t) * n));
+        CKS(c.ensure(c.in_t, c.cap_in_t, sizeof(uint32_t) * n));
+        CK(cudaMemcpyAsync(c.in_kid, kid, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, c.stream));
+        CK(cudaMemcpyAsync(c.in_t, t, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, c.stream));
+        kid = c.in_kid;
+        t = c.in_t;
+        if (nm) {
+            CKS(c.ensure(c.in_met, c.cap_in_met, sizeof(double) * n * nm));
+            CK(cudaMemcpyAsync(c.in_met, met, sizeof(double) * n * nm, cudaMemcpyHostToDevice, c.stream));
+            met = c.in_met;
+        }
+    }
+    CKS(sort_trace(c, kid, t, n, K));                 // a1
+    CKS(prefix_moments(c, n));                        // a2
+    if (o.root) {
+        CKS(root_levels(c, n, K, eps, z, k2, o.clamp_in_split ? 1 : 0));   // a3, a4
+    } else {
+        CKS(stem_only_leaves(c, n, K));
+    }
+    CKS(leaves_and_plan(c, n, K, met, nm, eps, z, k2, o));   // a5 - a8
+    c.n = n;
+    c.K = K;
+    c.n_metrics = nm;
+    c.eps = eps;
+    c.z = z;
+    c.stats.kernel_launches = c.launches;
+    c.have_plan = true;
+    return STEM_OK;
+}
+
+static int to_host(Ctx &c, stem_plan **out) {
+    stem_plan *p = (stem_plan *)calloc(1, sizeof(stem_plan));
+    if (!p) return STEM_E_NOMEM;
+    const uint64_t L = c.n_leaves, S = c.n_samples;
+    p->n_clusters = L;
+    p->n_samples = S;
+    p->clusters = (stem_cluster *)malloc(sizeof(stem_cluster) * (L ? L : 1));
+    p->sample_row = (uint32_t *)malloc(sizeof(uint32_t) * (S ? S : 1));
+    p->sample_cluster = (uint32_t *)malloc(sizeof(uint32_t) * (S ? S : 1));
+    p->sample_weight = (double *)malloc(sizeof(double) * (S ? S : 1));
+    p->n_metrics = c.n_metrics;
+    p->est_metric = (double *)calloc(c.n_metrics ? c.n_metrics : 1, sizeof(double));
+    if (!p->clusters || !p->sample_row || !p->sample_cluster || !p->sample_weight || !p->est_metric) {
+        stem_plan_free(p);
+        return STEM_E_NOMEM;
+    }
+    cudaStream_t st = c.stream;
+    cudaError_t e = cudaSuccess;
+    if (L) e = cudaMemcpyAsync(p->clusters, c.out_clusters, sizeof(stem_cluster) * L, cudaMemcpyDeviceToHost, st);
+    if (S && e == cudaSuccess)
+        e = cudaMemcpyAsync(p->sample_row, c.out_row, sizeof(uint32_t) * S, cudaMemcpyDeviceToHost, st);
+    if (S && e == cudaSuccess)
+        e = cudaMemcpyAsync(p->sample_cluster, c.out_cluster, sizeof(uint32_t) * S, cudaMemcpyDeviceToHost, st);
+    if (S && e == cudaSuccess)
+        e = cudaMemcpyAsync(p->sample_weight, c.out_weight, sizeof(double) * S, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) {
+        last_cuda_error() = e;
+        stem_plan_free(p);
+        return STEM_E_CUDA;
+    }
+    p->est_total_ns = c.est_total;
+    p->true_total_ns = c.T;
+    p->bound = c.bound;
+    p->eps = c.eps;
+    p->z = c.z;
+    memcpy(p->est_metric, c.host_est_metric, sizeof(double) * c.n_metrics);
+    *out = p;
+    return STEM_OK;
+}
+
+}  // namespace sr
+
+struct stem_ctx {
+    sr::Ctx c;
+};
+
+extern "C" {
+
+int stem_default_opts(stem_opts *o) {
+    if (!o) return STEM_E_INVAL;
+    *o = stem_opts{};
+    o->seed = 0;
+    o->z = 0.0;
+    o->scope = 0;
+    o->root = 1;
+    o->clamp_in_split = 1;
+    o->census_cap = 0;
+    o->stream = nullptr;
+    return STEM_OK;
+}
+
+int stem_ctx_create(int device, stem_ctx **out) {
+    if (!out) return STEM_E_INVAL;
+    *out = nullptr;
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess) { sr::last_cuda_error() = e; return STEM_E_CUDA; }
+    if (device < 0 || device >= ndev) return STEM_E_INVAL;
+    stem_ctx *x = new (std::nothrow) stem_ctx();
+    if (!x) return STEM_E_NOMEM;
+    x->c.device = device;
+    e = cudaSetDevice(device);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&x->c.sms, cudaDevAttrMultiProcessorCount, device);
+    if (e != cudaSuccess) {
+        sr::last_cuda_error() = e;
+        delete x;
+        return STEM_E_CUDA;
+    }
+    *out = x;
+    return STEM_OK;
+}
+
+void stem_ctx_destroy(stem_ctx *ctx) {
+    if (!ctx) return;
+    cudaSetDevice(ctx->c.device);
+    ctx->c.release();
+    delete ctx;
+}
+
+int stem_root_plan_ctx(stem_ctx *ctx, const stem_trace *trace, double eps, double conf, const stem_opts *opts,
+                       stem_plan **out) {
+    if (out) *out = nullptr;
+    if (!ctx) return STEM_E_INVAL;
+    stem_opts o;
+    if (opts) o = *opts; else stem_default_opts(&o);
+    int s = sr::run_plan(ctx->c, trace, eps, conf, o);
+    if (s != STEM_OK) {
+        ctx->c.have_plan = false;
+        return s;
+    }
+    if (out) return sr::to_host(ctx->c, out);
+    return STEM_OK;
+}
+
+int stem_root_plan(const stem_trace *trace, double eps, double conf, const stem_opts *opts, stem_plan **out) {
+    if (out) *out = nullptr;
+    if (!trace || !out) return STEM_E_INVAL;
+    stem_ctx *ctx = nullptr;
+    int s = stem_ctx_create(trace->device >= 0 ? trace->device : 0, &ctx);
+    if (s != STEM_OK) return s;
+    s = stem_root_plan_ctx(ctx, trace, eps, conf, opts, out);
+    stem_ctx_destroy(ctx);
+    return s;
+}
+
+int stem_ctx_device_plan(const stem_ctx *ctx, stem_device_plan *v) {
+    if (!ctx || !v) return STEM_E_INVAL;
+    if (!ctx->c.have_plan) return STEM_E_STATE;
+    const sr::Ctx &c = ctx->c;
+    v->n_clusters = c.n_leaves;
+    v->n_samples = c.n_samples;
+    v->clusters = c.out_clusters;
+    v->sample_row = c.out_row;
+    v->sample_cluster = c.out_cluster;
+    v->sample_weight = c.out_weight;
+    v->est_total_ns = c.est_total;
+    v->bound = c.bound;
+    v->eps = c.eps;
+    v->z = c.z;
+    v->true_total_ns = c.T;
+    v->n_metrics = c.n_metrics;
+    v->est_metric = c.host_est_metric;
+    return STEM_OK;
+}
+
+int stem_ctx_stats(const stem_ctx *ctx, stem_stats *s) {
+    if (!ctx || !s) return STEM_E_INVAL;
+    *s = ctx->c.stats;
+    return STEM_OK;
+}
+
+void stem_plan_free(stem_plan *p) {
+    if (!p) return;
+    free(p->clusters);
+    free(p->sample_row);
+    free(p->sample_cluster);
+    free(p->sample_weight);
+    free(p->est_metric);
+    free(p);
+}
+
+const char *stem_strerror(int status) {
+    switch (status) {
+        case STEM_OK: return "ok";
+        case STEM_E_INVAL: return "invalid argument";
+        case STEM_E_RANGE: return "value out of range (n, n_kernels or a kernel_id)";
+        case STEM_E_NOMEM: return "out of memory";
+        case STEM_E_CUDA: return "CUDA error";
+        case STEM_E_NCCL: return "NCCL error";
+        case STEM_E_LIMIT: return "sample count limit (2^32) exceeded";
+        case STEM_E_STATE: return "no plan has been built on this context";
+        default: return "unknown status";
+    }
+}
+
+int stem_z_from_conf(double conf, double *z_out) {
+    if (!z_out) return STEM_E_INVAL;
+    *z_out = 0.0;
+    if (!(conf > 0.0 && conf < 1.0)) return STEM_E_INVAL;
+    *z_out = sr::z_two_sided(conf);
+    return STEM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,125 @@
+// internal.h -- host-side context and stage entry points of libstemroot.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/stemroot.h"
+#include "common.cuh"
+#include "scan.cuh"
+
+#define CK(x)                                              \
+    do {                                                   \
+        cudaError_t e_ = (x);                              \
+        if (e_ != cudaSuccess) {                           \
+            sr::last_cuda_error() = e_;                    \
+            return e_ == cudaErrorMemoryAllocation ? STEM_E_NOMEM : STEM_E_CUDA; \
+        }                                                  \
+    } while (0)
+
+#define CKS(x)                                             \
+    do {                                                   \
+        int s_ = (x);                                      \
+        if (s_ != STEM_OK) return s_;                      \
+    } while (0)
+
+namespace sr {
+
+cudaError_t &last_cuda_error();
+
+// Device-resident scalars of one plan call (one cudaMemcpy brings them home).
+struct DevScalars {
+    uint32_t max_t, err, tile_counter, pad0;
+    uint64_t scan_total64;        // generic scan total
+    uint64_t frontier_total;      // packed (count << 32 | rows) of the next frontier
+    uint64_t n_leaves;            // leaves after compaction
+    uint64_t total_m;             // sum of m_i
+    uint64_t sum_q;               // sum_i floor(n_i U_i / m_i)
+    uint64_t T;                   // exact total time
+    uint32_t limit_err, pad1;
+    double ssum;                  // RN(exact sum sqrt(mu V)) (global scope)
+    double g;                     // Ssum / c (global scope)
+    double est_frac, var_sum;     // sum rn(r_i)/m_i, sum rn(V_i)/m_i
+    alignas(16) uint64_t wide_total[4];   // total of a wide (struct) scan
+};
+
+constexpr int kFixDigits = 6;     // 6 x 32-bit digits in u64 lanes, LSB 2^-72
+constexpr int kFixLsb = 72;
+
+struct Ctx {
+    int device = 0;
+    int sms = 148;
+    cudaStream_t stream = nullptr;
+    uint32_t launches = 0;
+    int tbits = 0;
+    stem_stats stats{};
+
+    // ---- workspace (grow-only)
+    template <class T>
+    int ensure(T *&p, size_t &cap, size_t bytes) {
+        if (bytes <= cap) return STEM_OK;
+        if (p) cudaFree(p);
+        p = nullptr;
+        cap = 0;
+        size_t b = bytes + bytes / 8 + 256;
+        cudaError_t e = cudaMalloc((void **)&p, b);
+        if (e != cudaSuccess) { last_cuda_error() = e; p = nullptr; return STEM_E_NOMEM; }
+        cap = b;
+        return STEM_OK;
+    }
+    int ensure_all(uint64_t n, uint32_t K, uint32_t n_metrics);
+    void release();
+
+    // input copies when the trace is on the host
+    uint32_t *in_kid = nullptr, *in_t = nullptr; size_t cap_in_kid = 0, cap_in_t = 0;
+    double *in_met = nullptr; size_t cap_in_met = 0;
+    // sort
+    uint64_t *keys[2] = {nullptr, nullptr}; size_t cap_keys[2] = {0, 0};
+    uint32_t *vals[2] = {nullptr, nullptr}; size_t cap_vals[2] = {0, 0};
+    uint32_t *t_sorted = nullptr, *row_sorted = nullptr; size_t cap_ts = 0, cap_rs = 0;
+    uint32_t *kid_count = nullptr, *goff = nullptr; size_t cap_kc = 0, cap_goff = 0;
+    uint64_t *hist = nullptr; size_t cap_hist = 0;
+    void *sort_status = nullptr; size_t cap_status = 0;
+    DevScalars *scalars = nullptr; size_t cap_scalars = 0;
+    void *scan_scratch = nullptr; size_t cap_scan = 0;
+    // prefix moments (a2)
+    uint64_t *P1 = nullptr; size_t cap_p1 = 0;
+    u128 *P2 = nullptr; size_t cap_p2 = 0;
+    // ROOT frontier (a3/a4)
+    uint32_t *f_lo[2] = {nullptr, nullptr}, *f_hi[2] = {nullptr, nullptr}, *f_aoff[2] = {nullptr, nullptr};
+    size_t cap_flo[2] = {0, 0}, cap_fhi[2] = {0, 0}, cap_faoff[2] = {0, 0};
+    uint32_t *cut = nullptr; size_t cap_cut = 0;
+    uint64_t *cnt_sz = nullptr; size_t cap_cntsz = 0;
+    void *split_part = nullptr; size_t cap_part = 0;
+    uint8_t *flags = nullptr; size_t cap_flags = 0;
+    // leaves (a5/a6)
+    uint32_t *leaf_lo = nullptr; size_t cap_leaf_lo = 0;
+    uint64_t *leaf_m = nullptr, *leaf_moff = nullptr, *leaf_U = nullptr;
+    size_t cap_leaf_m = 0, cap_leaf_moff = 0, cap_leaf_U = 0;
+    uint8_t *leaf_census = nullptr; size_t cap_leaf_census = 0;
+    uint32_t *leaf_kid = nullptr, *leaf_ord = nullptr; size_t cap_leaf_kid = 0, cap_leaf_ord = 0;
+    uint64_t *fix_acc = nullptr; size_t cap_fix = 0;      // [K or 1][kFixDigits] lanes
+    uint64_t *kern_T = nullptr; size_t cap_kern_T = 0;    // per-kernel T (scope 1)
+    double *kern_g = nullptr; size_t cap_kern_g = 0;      // per-kernel g (scope 1)
+    double *red_part = nullptr; size_t cap_red = 0;       // deterministic block partials
+    // plan outputs (a7/a8)
+    stem_cluster *out_clusters = nullptr; size_t cap_out_cl = 0;
+    uint32_t *out_row = nullptr, *out_cluster = nullptr; size_t cap_out_row = 0, cap_out_cluster = 0;
+    double *out_weight = nullptr; size_t cap_out_weight = 0;
+    double host_est_metric[64];
+
+    // last plan
+    bool have_plan = false;
+    uint64_t n = 0, n_leaves = 0, n_samples = 0, T = 0;
+    uint32_t K = 0, n_metrics = 0;
+    double est_total = 0, bound = 0, eps = 0, z = 0;
+};
+
+// stages
+int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K);      // a1
+int prefix_moments(Ctx &c, uint64_t n);                                                        // a2
+int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp);   // a3, a4
+int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
+int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint32_t n_metrics, double eps,
+                    double z, double k2, const stem_opts &o);                                  // a5..a8
+
+}  // namespace sr

@@ -1,0 +1,436 @@
+// stem.cu -- steps a5-a8: leaf table, STEM sample sizes (Eq. 6 with the
+// corrected numerator, P:L169 + P:L464), Philox sampling with replacement
+// (P:L210), weighted-sum extrapolation and predicted bound (Eq. 5).
+#include "internal.h"
+
+namespace sr {
+
+constexpr int kThreads = 256;
+
+// ---------------------------------------------------------------- fixed point
+// term >= 2^-20 and < 2^100 (R12): value = mant * 2^(exp-1075);
+// in units of 2^-72 it is mant << (exp - 1003), spread over 32-bit digits.
+__device__ __forceinline__ void fix_digits(double d, uint32_t dig[3], int &q, bool &bad) {
+    dig[0] = dig[1] = dig[2] = 0;
+    q = 0;
+    if (!(d > 0.0)) return;
+    const uint64_t bits = (uint64_t)__double_as_longlong(d);
+    const int ex = (int)((bits >> 52) & 0x7FF);
+    const uint64_t mant = (bits & ((1ull << 52) - 1)) | (1ull << 52);
+    const int shift = ex - 1003;
+    if (shift < 0 || shift + 53 > 32 * kFixDigits) { bad = true; return; }
+    q = shift >> 5;
+    const u128 v = (u128)mant << (shift & 31);
+    dig[0] = (uint32_t)v;
+    dig[1] = (uint32_t)(v >> 32);
+    dig[2] = (uint32_t)(v >> 64);
+}
+
+// round-to-nearest of sum_j lane[j] 2^(32 j - 72)
+__device__ double fix_round(const uint64_t *lane) {
+    uint32_t d[kFixDigits + 2];
+    u128 carry = 0;
+    for (int j = 0; j < kFixDigits; j++) {
+        const u128 x = (u128)lane[j] + carry;
+        d[j] = (uint32_t)x;
+        carry = x >> 32;
+    }
+    d[kFixDigits] = (uint32_t)carry;
+    d[kFixDigits + 1] = (uint32_t)(carry >> 32);
+    int top = -1;
+    for (int j = kFixDigits + 1; j >= 0; j--)
+        if (d[j]) { top = j; break; }
+    if (top < 0) return 0.0;
+    const int msb = 32 * top + 31 - __clz(d[top]);
+    // gather the 64 bits [msb-63, msb]; sticky = any lower bit
+    uint64_t word = 0;
+    bool sticky = false;
+    const int lo_bit = msb - 63;
+    for (int b = msb; b >= 0 && b >= lo_bit; b--) word = (word << 1) | ((d[b >> 5] >> (b & 31)) & 1u);
+    for (int b = lo_bit - 1; b >= 0 && !sticky; b--) sticky = (d[b >> 5] >> (b & 31)) & 1u;
+    const int scale = (lo_bit > 0 ? lo_bit : 0) - kFixLsb;
+    if (sticky) word |= 1;
+    return __dmul_rn(__ull2double_rn(word), pow2(scale));
+}
+
+// ---------------------------------------------------------------- leaf table
+struct LeafArgs {
+    const uint32_t *leaf_lo, *goff, *t;
+    const uint64_t *P1;
+    const u128 *P2;
+    uint64_t L, n;
+    uint32_t K;
+    int scope;
+    uint32_t *leaf_kid, *leaf_ord;
+    uint64_t *fix_acc;   // [scope==1 ? K : 1][kFixDigits]
+    uint64_t *kern_T;    // scope 1
+    uint32_t *err;
+};
+
+struct LeafView {
+    uint32_t lo, hi;
+    uint64_t n, S;
+    u128 V;
+};
+
+__device__ __forceinline__ LeafView leaf_view(const uint32_t *leaf_lo, uint64_t L, uint64_t N, const uint64_t *P1,
+                                              const u128 *P2, uint64_t i) {
+    LeafView v;
+    v.lo = leaf_lo[i];
+    v.hi = (i + 1 < L) ? leaf_lo[i + 1] : (uint32_t)N;
+    v.n = v.hi - v.lo;
+    v.S = P1[v.hi] - P1[v.lo];
+    const u128 Q = P2[v.hi] - P2[v.lo];
+    v.V = (u128)v.n * Q - (u128)v.S * v.S;
+    return v;
+}
+
+__global__ void __launch_bounds__(kThreads) leaf_kkt_kernel(LeafArgs a) {
+    __shared__ unsigned long long s_acc[kFixDigits];
+    if (threadIdx.x < kFixDigits) s_acc[threadIdx.x] = 0;
+    __syncthreads();
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    bool bad = false;
+    if (i < a.L) {
+        const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.P1, a.P2, i);
+        const uint32_t g = (uint32_t)upper_bound(a.goff, (uint64_t)a.K + 1, v.lo) - 1;
+        const uint64_t first = lower_bound(a.leaf_lo, a.L, a.goff[g]);
+        a.leaf_kid[i] = g;
+        a.leaf_ord[i] = (uint32_t)(i - first);
+        if (a.scope != 2) {
+            const double mu = __ddiv_rn(rn64(v.S), rn64(v.n));
+            const double term = __dsqrt_rn(__dmul_rn(mu, rn128(v.V)));
+            uint32_t dig[3];
+            int q;
+            fix_digits(term, dig, q, bad);
+            if (a.scope == 0) {
+                for (int j = 0; j < 3; j++)
+                    if (dig[j]) atomicAdd(&s_acc[q + j], (unsigned long long)dig[j]);
+            } else {
+                for (int j = 0; j < 3; j++)
+                    if (dig[j]) atomicAdd((unsigned long long *)&a.fix_acc[(uint64_t)g * kFixDigits + q + j],
+                                          (unsigned long long)dig[j]);
+                atomicAdd((unsigned long long *)&a.kern_T[g], (unsigned long long)v.S);
+            }
+        }
+    }
+    if (bad) atomicOr(a.err, 2u);
+    __syncthreads();
+    if (a.scope == 0 && threadIdx.x < kFixDigits && s_acc[threadIdx.x])
+        atomicAdd((unsigned long long *)&a.fix_acc[threadIdx.x], s_acc[threadIdx.x]);
+}
+
+// g = Ssum / c with c = (eps T / z)^2 (R10, R11); global: one thread, per kernel: one per kernel
+__global__ void kkt_finalize_kernel(const uint64_t *fix_acc, const uint64_t *kern_T, const uint64_t *T,
+                                    uint32_t nsets, double eps, double z, double *g_out, double *ssum_out) {
+    const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= nsets) return;
+    const double ssum = fix_round(fix_acc + s * kFixDigits);
+    const uint64_t Ts = kern_T ? kern_T[s] : *T;
+    const double w = __ddiv_rn(__dmul_rn(eps, rn64(Ts)), z);
+    const double c = __dmul_rn(w, w);
+    g_out[s] = __ddiv_rn(ssum, c);
+    if (ssum_out) *ssum_out = ssum;
+}
+
+struct MArgs {
+    const uint32_t *leaf_lo, *leaf_kid;
+    const uint64_t *P1;
+    const u128 *P2;
+    uint64_t L, n;
+    int scope, census_cap;
+    double k2;
+    const double *g;     // [1] or [K]
+    uint64_t *m;
+    uint8_t *census;
+    uint32_t *limit_err;
+};
+
+__global__ void __launch_bounds__(kThreads) leaf_m_kernel(MArgs a) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= a.L) return;
+    const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.P1, a.P2, i);
+    double m;
+    if (v.V == 0) {
+        m = 1.0;
+    } else if (a.scope == 2) {   // Eq. 3 per leaf
+        const double dS = rn64(v.S);
+        m = ceil(__dmul_rn(__ddiv_rn(rn128(v.V), __dmul_rn(dS, dS)), a.k2));
+    } else {                     // Eq. 6, corrected numerator
+        const double mu = __ddiv_rn(rn64(v.S), rn64(v.n));
+        const double g = a.scope == 0 ? a.g[0] : a.g[a.leaf_kid[i]];
+        m = ceil(__dmul_rn(g, __dsqrt_rn(__ddiv_rn(rn128(v.V), mu))));
+    }
+    if (m < 1.0) m = 1.0;
+    uint8_t cen = 0;
+    if (a.census_cap && m >= rn64(v.n)) { m = rn64(v.n); cen = 1; }
+    if (!(m < 4294967296.0)) { atomicOr(a.limit_err, 1u); m = 1.0; }
+    a.m[i] = (uint64_t)m;
+    a.census[i] = cen;
+}
+
+// ---------------------------------------------------------------- a7: samples
+struct SampleArgs {
+    const uint32_t *leaf_lo, *leaf_kid, *leaf_ord;
+    const uint64_t *moff, *m;
+    const uint8_t *census;
+    const uint32_t *t, *row;
+    uint64_t L, n, S;
+    uint32_t key0, key1;
+    uint32_t *out_row, *out_cluster;
+    double *out_weight;
+    uint64_t *U;
+};
+
+__global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
+    const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= a.S) return;
+    const uint64_t i = upper_bound(a.moff, a.L, s) - 1;
+    const uint64_t j = s - a.moff[i];
+    const uint32_t lo = a.leaf_lo[i];
+    const uint32_t hi = (i + 1 < a.L) ? a.leaf_lo[i + 1] : (uint32_t)a.n;
+    const uint64_t n = hi - lo, m = a.m[i];
+    uint64_t pos;
+    if (a.census[i]) {
+        pos = lo + j;
+    } else {
+        const U4 x = philox4x32_10(U4{(uint32_t)(j >> 1), a.leaf_ord[i], a.leaf_kid[i], 0x53544D31u}, a.key0, a.key1);
+        const uint64_t r = (j & 1) ? (((uint64_t)x.w << 32) | x.z) : (((uint64_t)x.y << 32) | x.x);
+        pos = lo + __umul64hi(r, n);
+    }
+    a.out_row[s] = a.row[pos];
+    a.out_cluster[s] = (uint32_t)i;
+    a.out_weight[s] = __ddiv_rn(rn64(n), rn64(m));
+    atomicAdd((unsigned long long *)&a.U[i], (unsigned long long)a.t[pos]);
+}
+
+// ---------------------------------------------------------------- a8: estimate
+// deterministic block sum (fixed tree for a fixed launch shape)
+__device__ __forceinline__ double block_sum(double v, double *sm) {
+    for (int o = 16; o; o >>= 1) v = __dadd_rn(v, __shfl_xor_sync(0xffffffffu, v, o));
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    __syncthreads();
+    if (lane == 0) sm[w] = v;
+    __syncthreads();
+    double r = 0.0;
+    if (threadIdx.x == 0)
+        for (int k = 0; k < (int)(blockDim.x >> 5); k++) r = __dadd_rn(r, sm[k]);
+    return r;   // valid in thread 0
+}
+
+struct EstArgs {
+    const uint32_t *leaf_lo;
+    const uint64_t *P1;
+    const u128 *P2;
+    const uint64_t *m, *U;
+    uint64_t L, n;
+    uint64_t *sum_q;
+    double *part;   // [blocks][2]
+};
+
+__global__ void __launch_bounds__(kThreads) estimate_kernel(EstArgs a) {
+    __shared__ double sm[kThreads / 32];
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    double frac = 0.0, var = 0.0;
+    if (i < a.L) {
+        const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.P1, a.P2, i);
+        const uint64_t m = a.m[i];
+        const u128 num = (u128)v.n * a.U[i];
+        const uint64_t q = (uint64_t)(num / m), r = (uint64_t)(num % m);
+        atomicAdd((unsigned long long *)a.sum_q, (unsigned long long)q);
+        frac = __ddiv_rn(rn64(r), rn64(m));
+        var = __ddiv_rn(rn128(v.V), rn64(m));
+    }
+    const double f = block_sum(frac, sm);
+    const double vv = block_sum(var, sm);
+    if (threadIdx.x == 0) {
+        a.part[2 * blockIdx.x] = f;
+        a.part[2 * blockIdx.x + 1] = vv;
+    }
+}
+
+struct MetArgs {
+    const uint32_t *out_row;
+    const double *out_weight;
+    const double *metrics;
+    uint64_t n, S;
+    uint32_t nm;
+    double *part;   // [blocks][nm]
+};
+
+__global__ void __launch_bounds__(kThreads) metric_kernel(MetArgs a) {
+    __shared__ double sm[kThreads / 32];
+    const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    for (uint32_t c = 0; c < a.nm; c++) {
+        double v = 0.0;
+        if (s < a.S) v = __dmul_rn(a.out_weight[s], a.metrics[(uint64_t)c * a.n + a.out_row[s]]);
+        const double r = block_sum(v, sm);
+        if (threadIdx.x == 0) a.part[(uint64_t)blockIdx.x * a.nm + c] = r;
+    }
+}
+
+// sums block partials column by column in block order (deterministic)
+__global__ void reduce_cols_kernel(const double *part, uint64_t blocks, uint32_t cols, double *out) {
+    __shared__ double sm[kThreads / 32];
+    for (uint32_t c = 0; c < cols; c++) {
+        double v = 0.0;
+        for (uint64_t b = threadIdx.x; b < blocks; b += blockDim.x) v = __dadd_rn(v, part[b * cols + c]);
+        const double r = block_sum(v, sm);
+        if (threadIdx.x == 0) out[c] = r;
+    }
+}
+
+// est = rn(sum_i q_i) + sum_i rn(r_i)/m_i ; bound = z sqrt(sum_i V_i/m_i) / T  (R16, R17)
+__global__ void est_finalize_kernel(const uint64_t *sum_q, const double *red, const uint64_t *T, double z,
+                                    double *out) {
+    out[0] = __dadd_rn(rn64(*sum_q), red[0]);
+    out[1] = (*T == 0) ? 0.0 : __ddiv_rn(__dmul_rn(z, __dsqrt_rn(red[1])), rn64(*T));
+}
+
+__global__ void pack_kernel(const uint32_t *leaf_lo, const uint32_t *leaf_kid, const uint32_t *leaf_ord,
+                            const uint64_t *P1, const u128 *P2, const uint32_t *t, const uint64_t *m,
+                            const uint8_t *census, uint64_t L, uint64_t n, stem_cluster *out) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= L) return;
+    const LeafView v = leaf_view(leaf_lo, L, n, P1, P2, i);
+    stem_cluster c;
+    c.kernel_id = leaf_kid[i];
+    c.ordinal = leaf_ord[i];
+    c.lo_ns = t[v.lo];
+    c.hi_ns = t[v.hi - 1];
+    c.n = v.n;
+    c.sum_ns = v.S;
+    const double dn = rn64(v.n);
+    c.mean_ns = __ddiv_rn(rn64(v.S), dn);
+    c.std_ns = __ddiv_rn(__dsqrt_rn(rn128(v.V)), dn);
+    c.m = m[i];
+    c.census = census[i];
+    c.reserved = 0;
+    out[i] = c;
+}
+
+// ---------------------------------------------------------------- driver
+static unsigned blocks_for(uint64_t n) { return (unsigned)((n + kThreads - 1) / kThreads); }
+
+int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint32_t nm, double eps, double z,
+                    double k2, const stem_opts &o) {
+    cudaStream_t st = c.stream;
+    // a5: leaf starts = group starts U accepted cuts, in row order = canonical (kernel, lo) order
+    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(n) + 1) * sizeof(uint64_t)));
+    CKS(c.ensure(c.leaf_lo, c.cap_leaf_lo, sizeof(uint32_t) * (n + 1)));
+    {
+        const uint8_t *flags = c.flags;
+        uint32_t *leaf_lo = c.leaf_lo;
+        exclusive_scan<uint64_t>([flags] __device__(uint64_t i) -> uint64_t { return flags[i]; },
+                                 [leaf_lo] __device__(uint64_t i, uint64_t pre, uint64_t v) {
+                                     if (v) leaf_lo[pre] = (uint32_t)i;
+                                 },
+                                 n, (uint64_t *)c.scan_scratch, &c.scalars->n_leaves, st, &c.launches);
+        CK(cudaGetLastError());
+    }
+    uint64_t L = 0;
+    CK(cudaMemcpyAsync(&L, &c.scalars->n_leaves, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    c.n_leaves = L;
+    // per-leaf arrays (leaf_kid/ord live in the two halves of one allocation)
+    CKS(c.ensure(c.leaf_m, c.cap_leaf_m, sizeof(uint64_t) * (L + 1)));
+    CKS(c.ensure(c.leaf_moff, c.cap_leaf_moff, sizeof(uint64_t) * (L + 1)));
+    CKS(c.ensure(c.leaf_U, c.cap_leaf_U, sizeof(uint64_t) * (L + 1)));
+    CKS(c.ensure(c.leaf_census, c.cap_leaf_census, L + 1));
+    CKS(c.ensure(c.leaf_kid, c.cap_leaf_kid, sizeof(uint32_t) * (L + 1)));
+    CKS(c.ensure(c.leaf_ord, c.cap_leaf_ord, sizeof(uint32_t) * (L + 1)));
+    uint32_t *leaf_kid = c.leaf_kid, *leaf_ord = c.leaf_ord;
+    const uint32_t nsets = o.scope == 1 ? K : 1;
+    CKS(c.ensure(c.fix_acc, c.cap_fix, sizeof(uint64_t) * kFixDigits * nsets));
+    CKS(c.ensure(c.kern_T, c.cap_kern_T, sizeof(uint64_t) * nsets));
+    CKS(c.ensure(c.kern_g, c.cap_kern_g, sizeof(double) * nsets));
+    CK(cudaMemsetAsync(c.fix_acc, 0, sizeof(uint64_t) * kFixDigits * nsets, st));
+    CK(cudaMemsetAsync(c.kern_T, 0, sizeof(uint64_t) * nsets, st));
+    CK(cudaMemsetAsync(c.leaf_U, 0, sizeof(uint64_t) * (L + 1), st));
+
+    LeafArgs la{c.leaf_lo, c.goff, c.t_sorted, c.P1, c.P2, L, n, K, o.scope, leaf_kid, leaf_ord,
+                c.fix_acc, c.kern_T, &c.scalars->err};
+    leaf_kkt_kernel<<<blocks_for(L), kThreads, 0, st>>>(la);
+    c.launches++;
+    // T = P1[n] (exact total, a2)
+    if (o.scope == 0)
+        kkt_finalize_kernel<<<1, 32, 0, st>>>(c.fix_acc, nullptr, c.P1 + n, 1, eps, z, c.kern_g, &c.scalars->ssum);
+    else if (o.scope == 1)
+        kkt_finalize_kernel<<<blocks_for(K), kThreads, 0, st>>>(c.fix_acc, c.kern_T, nullptr, K, eps, z, c.kern_g,
+                                                               nullptr);
+    if (o.scope != 2) c.launches++;
+    MArgs ma{c.leaf_lo, leaf_kid, c.P1, c.P2, L, n, o.scope, o.census_cap, k2, c.kern_g, c.leaf_m,
+             c.leaf_census, &c.scalars->limit_err};
+    leaf_m_kernel<<<blocks_for(L), kThreads, 0, st>>>(ma);
+    c.launches++;
+    CK(cudaGetLastError());
+    {
+        const uint64_t *m = c.leaf_m;
+        uint64_t *moff = c.leaf_moff;
+        exclusive_scan<uint64_t>([m] __device__(uint64_t i) -> uint64_t { return m[i]; },
+                                 [moff] __device__(uint64_t i, uint64_t pre, uint64_t) { moff[i] = pre; }, L,
+                                 (uint64_t *)c.scan_scratch, &c.scalars->total_m, st, &c.launches);
+        CK(cudaGetLastError());
+    }
+    DevScalars hs;
+    CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (hs.err & 2) return STEM_E_CUDA;
+    if (hs.limit_err || hs.total_m >= (1ull << 32)) return STEM_E_LIMIT;
+    const uint64_t S = hs.total_m;
+    uint64_t T = 0;
+    CK(cudaMemcpy(&T, c.P1 + n, sizeof(uint64_t), cudaMemcpyDeviceToHost));
+    c.n_samples = S;
+    c.T = T;
+    c.stats.ssum = o.scope == 0 ? hs.ssum : 0.0;
+
+    // a7: samples
+    CKS(c.ensure(c.out_row, c.cap_out_row, sizeof(uint32_t) * (S + 1)));
+    CKS(c.ensure(c.out_cluster, c.cap_out_cluster, sizeof(uint32_t) * (S + 1)));
+    CKS(c.ensure(c.out_weight, c.cap_out_weight, sizeof(double) * (S + 1)));
+    SampleArgs sa{c.leaf_lo, leaf_kid, leaf_ord, c.leaf_moff, c.leaf_m, c.leaf_census, c.t_sorted, c.row_sorted,
+                  L, n, S, (uint32_t)o.seed, (uint32_t)(o.seed >> 32), c.out_row, c.out_cluster, c.out_weight,
+                  c.leaf_U};
+    if (S) sample_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa);
+    c.launches += S ? 1 : 0;
+    CK(cudaGetLastError());
+
+    // a8: estimate, bound, metrics (deterministic block partials)
+    const uint64_t eb = blocks_for(L), mb = blocks_for(S);
+    const uint64_t part_cols = 2 + (uint64_t)nm;
+    const uint64_t part_doubles = 2 * eb + mb * (nm ? nm : 1) + part_cols + 16;
+    CKS(c.ensure(c.red_part, c.cap_red, sizeof(double) * part_doubles));
+    double *part_est = c.red_part, *part_met = c.red_part + 2 * eb, *red_out = part_met + mb * (nm ? nm : 1);
+    CK(cudaMemsetAsync(&c.scalars->sum_q, 0, sizeof(uint64_t), st));
+    EstArgs ea{c.leaf_lo, c.P1, c.P2, c.leaf_m, c.leaf_U, L, n, &c.scalars->sum_q, part_est};
+    estimate_kernel<<<(unsigned)eb, kThreads, 0, st>>>(ea);
+    reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_est, eb, 2, red_out);
+    c.launches += 2;
+    if (nm && S) {
+        MetArgs ma2{c.out_row, c.out_weight, metrics, n, S, nm, part_met};
+        metric_kernel<<<(unsigned)mb, kThreads, 0, st>>>(ma2);
+        reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_met, mb, nm, red_out + 2);
+        c.launches += 2;
+    }
+    // a5 output records
+    CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
+    pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.P1, c.P2, c.t_sorted, c.leaf_m,
+                                                   c.leaf_census, L, n, c.out_clusters);
+    c.launches++;
+    CK(cudaGetLastError());
+    double *est_out = red_out + 2 + nm;
+    est_finalize_kernel<<<1, 1, 0, st>>>(&c.scalars->sum_q, red_out, c.P1 + n, z, est_out);
+    c.launches++;
+    CK(cudaGetLastError());
+    double red[2 + 64 + 2];
+    CK(cudaMemcpyAsync(red, red_out, sizeof(double) * (2 + nm + 2), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    c.est_total = red[2 + nm];
+    c.bound = red[2 + nm + 1];
+    for (uint32_t k = 0; k < nm; k++) c.host_est_metric[k] = S ? red[2 + k] : 0.0;
+    c.stats.n_clusters = L;
+    c.stats.n_samples = S;
+    return STEM_OK;
+}
+
+}  // namespace sr

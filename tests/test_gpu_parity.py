@@ -1,0 +1,191 @@
+"""CUDA path vs oracle, element by element, through the C ABI (needs a B200).
+
+Integer outputs (cluster boundaries, sizes, m_i, sample rows) bit-exact; fp64
+outputs within 1e-9 relative (north_star).  Inputs are seeded and synthetic
+(tracegen + small hand-made edge cases); the oracle never sees GPU output."""
+import numpy as np
+import pytest
+
+import oracle as O
+import tracegen as G
+from parity_util import Z95, assert_plans_equal
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def sr():
+    import paper_conf_micro_chungnkk25_b200 as m
+    m.build()
+    return m
+
+
+@pytest.fixture(scope="module")
+def ctx(sr):
+    c = sr.Context(0)
+    yield c
+    c.close()
+
+
+def _dev(a):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(a).view(np.int32)).cuda()
+
+
+def _both(ctx, kid, t, K, metrics=None, host=False, **kw):
+    kw.setdefault("z", Z95)
+    eps = kw.pop("eps", 0.05)
+    if host:
+        got = ctx.plan(kid, t, K, eps=eps, metrics=metrics, **kw)
+    else:
+        import torch
+        met = None if metrics is None else torch.from_numpy(np.ascontiguousarray(metrics)).cuda()
+        got = ctx.plan(_dev(kid), _dev(t), K, eps=eps, metrics=met, **kw)
+    ref = O.plan(kid, t, K, eps=eps, metrics=metrics, **kw)
+    return got, ref
+
+
+# ------------------------------------------------------------------ pinned worked examples
+def test_worked_trees(ctx, golden):
+    for tr in golden("root_trees.json")["trees"]:
+        t = np.array(tr["t"], np.uint32)
+        got, ref = _both(ctx, np.zeros(len(t), np.uint32), t, 1, eps=tr["eps"], z=tr["z"], seed=3)
+        assert_plans_equal(got, ref)
+        assert [[int(c["lo_ns"]), int(c["hi_ns"])] for c in got["clusters"]] == tr["leaves_lo_hi"]
+        assert got["est_total_ns"] == tr["est"]
+
+
+def test_exact_tie_split(ctx, golden):
+    for c in golden("split_tie.json")["cases"]:
+        t = np.array([c["s"] * x for x in c["base"]] * 3, np.uint32)
+        kid = np.repeat(np.arange(3, dtype=np.uint32), len(c["base"]))
+        t = np.concatenate([np.sort(t[kid == k]) for k in range(3)]).astype(np.uint32)
+        got, ref = _both(ctx, kid, t, 3, eps=0.05)
+        assert_plans_equal(got, ref)
+
+
+# ------------------------------------------------------------------ edge cases
+EDGE = {
+    "single_row": (np.array([0], np.uint32), np.array([5], np.uint32), 1),
+    "constant": (np.zeros(1000, np.uint32), np.full(1000, 77, np.uint32), 1),
+    "zeros": (np.zeros(50, np.uint32), np.zeros(50, np.uint32), 1),
+    "max_t": (np.zeros(4000, np.uint32), np.where(np.arange(4000) % 3 == 0, 2 ** 32 - 1, 2 ** 31).astype(np.uint32), 1),
+    "singletons_and_empty": (np.array([0, 2, 2, 5, 9, 9, 9], np.uint32), np.array([3, 1, 1, 8, 0, 4, 4], np.uint32), 12),
+    "two_values": (np.zeros(9000, np.uint32), (np.arange(9000) % 2 * 1000 + 10).astype(np.uint32), 1),
+    "decreasing": (np.zeros(3000, np.uint32), np.arange(3000, 0, -1).astype(np.uint32) * 1000, 1),
+    "one_off_short_call": (np.zeros(5000, np.uint32), np.r_[[100], np.full(4999, 150000)].astype(np.uint32), 1),
+}
+
+
+@pytest.mark.parametrize("name", sorted(EDGE))
+def test_edge_cases(ctx, name):
+    kid, t, K = EDGE[name]
+    for kw in ({}, {"root": False}, {"census_cap": True, "eps": 1e-4}):
+        got, ref = _both(ctx, kid, t, K, seed=11, **kw)
+        assert_plans_equal(got, ref)
+
+
+def test_errors(ctx, sr):
+    with pytest.raises(sr.StemError) as e:
+        ctx.plan(_dev(np.array([0, 4], np.uint32)), _dev(np.array([1, 2], np.uint32)), 4)
+    assert e.value.status == sr.STEM_E_RANGE
+    with pytest.raises(sr.StemError) as e:
+        ctx.plan(_dev(np.array([0], np.uint32)), _dev(np.array([1], np.uint32)), 1, eps=1.5)
+    assert e.value.status == sr.STEM_E_INVAL
+    # the context stays usable after an error
+    got, ref = _both(ctx, *EDGE["two_values"][:2], 1)
+    assert_plans_equal(got, ref)
+
+
+# ------------------------------------------------------------------ random traces, several tiles + ragged tail
+def _mixture(rng, n, K, peaks=3, spread=0.05, max_t=2 ** 24):
+    kid = (rng.zipf(1.3, n) - 1) % K
+    centers = rng.integers(500, max_t, (K, peaks))
+    p = rng.integers(0, peaks, n)
+    t = centers[kid, p] * rng.lognormal(0.0, spread, n)
+    return kid.astype(np.uint32), np.minimum(t, 2 ** 32 - 1).astype(np.uint32)
+
+
+@pytest.mark.parametrize("n,K", [(4097, 3), (20011, 17), (100003, 211), (250000, 1)])
+@pytest.mark.parametrize("eps", [0.01, 0.05, 0.25])
+def test_random_mixtures(ctx, n, K, eps):
+    rng = np.random.default_rng(n + K)
+    kid, t = _mixture(rng, n, K)
+    got, ref = _both(ctx, kid, t, K, eps=eps, seed=n)
+    assert_plans_equal(got, ref)
+
+
+@pytest.mark.parametrize("opts", [dict(scope=1), dict(scope=2), dict(root=False), dict(clamp_in_split=False),
+                                  dict(census_cap=True, eps=0.002), dict(seed=2 ** 63 + 12345)])
+def test_option_matrix(ctx, opts):
+    rng = np.random.default_rng(5)
+    kid, t = _mixture(rng, 60000, 40, peaks=4, spread=0.2)
+    got, ref = _both(ctx, kid, t, 40, **opts)
+    assert_plans_equal(got, ref)
+
+
+def test_host_pointers_and_metrics(ctx):
+    rng = np.random.default_rng(9)
+    kid, t = _mixture(rng, 30000, 25)
+    met = np.vstack([t * 1.5 + 3, rng.random(30000)])
+    got, ref = _both(ctx, kid, t, 25, metrics=met, host=True)
+    assert_plans_equal(got, ref, metrics=True)
+    got, ref = _both(ctx, kid, t, 25, metrics=met)
+    assert_plans_equal(got, ref, metrics=True)
+
+
+def test_determinism(ctx):
+    rng = np.random.default_rng(13)
+    kid, t = _mixture(rng, 200000, 64)
+    a = ctx.plan(_dev(kid), _dev(t), 64, z=Z95)
+    b = ctx.plan(_dev(kid), _dev(t), 64, z=Z95)
+    assert a["clusters"].tobytes() == b["clusters"].tobytes()
+    assert a["sample_row"].tobytes() == b["sample_row"].tobytes()
+    assert a["est_total_ns"] == b["est_total_ns"] and a["bound"] == b["bound"]
+
+
+def test_z_from_conf_matches_scipy(sr):
+    from scipy.stats import norm
+    for conf in (0.8, 0.9, 0.95, 0.99, 0.999999):
+        assert sr.z_from_conf(conf) == pytest.approx(norm.ppf(1 - (1 - conf) / 2), rel=1e-14)
+
+
+# ------------------------------------------------------------------ config-shaped traces (BASELINE configs)
+@pytest.mark.parametrize("name,n", [("C1", None), ("C2", None), ("C4", 2_000_000)])
+def test_configs(ctx, name, n):
+    sp = G.spec(name, n=n)
+    kid, t, _ = G.generate_np(sp)
+    got, ref = _both(ctx, kid, t, sp.n_kernels, eps=sp.eps, seed=1)
+    assert_plans_equal(got, ref)
+
+
+def test_config_c3_with_metrics(ctx):
+    sp = G.spec("C3", n=2_000_000)
+    kid, t, met = G.generate_np(sp)
+    got, ref = _both(ctx, kid, t, sp.n_kernels, metrics=met, eps=sp.eps, seed=2)
+    assert_plans_equal(got, ref, metrics=True)
+
+
+@pytest.mark.parametrize("eps", [0.01, 0.03, 0.1])
+def test_eps_sweep(ctx, eps):
+    sp = G.spec("C4", n=1_000_000)
+    kid, t, _ = G.generate_np(sp)
+    got, ref = _both(ctx, kid, t, sp.n_kernels, eps=eps, seed=4)
+    assert_plans_equal(got, ref)
+
+
+# ------------------------------------------------------------------ generator twin
+def test_tracegen_cuda_matches_numpy():
+    import torch
+    for name, n, row0 in (("C3", 300_000, 12_345_677), ("C2", 100_000, 0), ("C1", 10_000, 0)):
+        sp = G.spec(name)
+        ds = G.DeviceSpec(sp, "cuda:0")
+        k = torch.empty(n, dtype=torch.int32, device="cuda")
+        tt = torch.empty(n, dtype=torch.int32, device="cuda")
+        met = torch.empty((sp.n_metrics, n), dtype=torch.float64, device="cuda") if sp.n_metrics else None
+        G.generate_cuda(ds, k, tt, met, row0=row0, count=n)
+        kid, t, m = G.generate_np(sp, row0, n)
+        assert np.array_equal(k.cpu().numpy().view(np.uint32), kid)
+        assert np.array_equal(tt.cpu().numpy().view(np.uint32), t)
+        if sp.n_metrics:
+            assert np.array_equal(met.cpu().numpy(), m)
