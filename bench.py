@@ -1,0 +1,323 @@
+#!/usr/bin/env python
+"""Benchmark: trace rows/s to a STEM+ROOT sampling plan on B200 (BASELINE.json metric).
+
+One step = one full pass of the hot path (a1 group/sort, a2 prefix moments,
+a3/a4 ROOT levels, a5 leaf table, a6 STEM sizes, a7 Philox samples, a8
+estimate + bound) over one synthetic trace already resident in HBM, through
+the C ABI (stem_root_plan_ctx, plan left on the device).  Default workload:
+BASELINE config C5 (1e9 invocations, 10k kernel ids), the configuration the
+metric's 1/2/4/8-GPU figures are quoted on; it fits one B200.
+
+    python bench.py [--gpus N --steps K --warmup W] [--config C5 --n ROWS] [--impl reference]
+
+Prints ONE JSON line on rank 0.  See DESIGN.md §7 for every field.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "trace rows/sec to sampling plan"
+UNIT = "rows/s"
+WORKLOADS = {
+    "C1": "C1 tiny: 10k invocations, 20 kernel ids, bimodal Gaussian, eps 5%, 95% conf",
+    "C2": "C2 CASIO-shaped: 1M invocations, 500 kernel ids, unimodal/multimodal/gamma/lognormal mix",
+    "C3": "C3 LLM-inference-shaped: 20M invocations, 2k kernel ids, lognormal + multi-saturation, 12 metrics",
+    "C4": "C4 training-shaped: 100M invocations, 1k kernel ids, eps 5% (sweep 1-10% in tests)",
+    "C5": "C5: 1e9 invocations, 10k kernel ids, LLM mix, Zipf(1.1) call sites",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="C5")
+    ap.add_argument("--n", type=int, default=None, help="override rows")
+    ap.add_argument("--eps", type=float, default=None)
+    ap.add_argument("--conf", type=float, default=0.95)
+    ap.add_argument("--cpu-sample-rows", type=int, default=30_000_000)
+    ap.add_argument("--ref-sample-rows", type=int, default=8_000_000)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy kernel)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def load_ncu_traffic():
+    """Per-launch DRAM bytes of our kernels from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f)
+    return {}
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, dev):
+        self.dev = dev
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={self.dev}", f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"], stdout=self.f,
+                                      stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        self.p.wait()
+        self.f.flush()
+        rows = []
+        with open(self.f.name) as f:
+            for line in f:
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) >= 9:
+                    rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def dist_env():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+def run_reference(a):
+    """--impl reference: the oracle (plain single-threaded C, oracle/) as it stands, on the
+    host cores, on a bounded sample of the same workload; rank 0 only."""
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import numpy as np
+
+    import oracle
+    import tracegen
+    sp = tracegen.spec(a.config, n=a.n)
+    m = min(a.ref_sample_rows, sp.n)
+    kid, t, met = tracegen.generate_np(sp, 0, m)
+    eps = a.eps if a.eps is not None else sp.eps
+    z = 1.959963984540054
+    times = []
+    for i in range(a.warmup + a.steps):
+        t0 = time.perf_counter()
+        oracle.plan(kid, t, sp.n_kernels, eps=eps, z=z, seed=i, metrics=met)
+        dt = time.perf_counter() - t0
+        if i >= a.warmup:
+            times.append(dt)
+    tot = sum(times)
+    value = m * len(times) / tot
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
+        "ms_per_step": 1e3 * tot / len(times), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded)",
+        "impl": "reference",
+        "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n, "kernels": sp.n_kernels,
+                   "eps": eps, "conf": a.conf, "sample_rows": m},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": f"first {m} rows of {a.config} (oracle single-threaded C, -O2)"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "gpu_launches": 0,
+    }
+    print(json.dumps(line), flush=True)
+
+
+def run_ours(a):
+    import numpy as np
+    import torch
+
+    import paper_conf_micro_chungnkk25_b200 as sr
+    import tracegen
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    sp = tracegen.spec(a.config, n=a.n)
+    eps = a.eps if a.eps is not None else sp.eps
+    # rows of this rank: the whole trace at N=1; a row-range shard at N>1 (weak scaling of
+    # independent shard plans -- the kernel-id exchange is not in this build yet)
+    n_local = sp.n
+    row0 = 0
+    if world > 1:
+        row0 = rank * sp.n
+    ds = tracegen.DeviceSpec(sp, dev)
+    kid = torch.empty(n_local, dtype=torch.int32, device=dev)
+    tt = torch.empty(n_local, dtype=torch.int32, device=dev)
+    nm = sp.n_metrics
+    met = torch.empty((nm, n_local), dtype=torch.float64, device=dev) if nm else None
+    tracegen.generate_cuda(ds, kid, tt, met, row0=row0, count=n_local)
+    torch.cuda.synchronize()
+    del ds
+
+    ctx = sr.Context(local)
+    stream = torch.cuda.current_stream(dev)
+
+    def step(timing=False):
+        return ctx.plan(kid, tt, sp.n_kernels, eps=eps, conf=a.conf, metrics=met, seed=12345, to_host=False,
+                        stream=stream.cuda_stream)
+
+    for _ in range(a.warmup):
+        step()
+    torch.cuda.synchronize()
+    # timed region (device time, CUDA events on the plan's stream; per-stage events live)
+    ctx.enable_timing(True)
+    stages = {}
+    clocks = Clocks(local)
+    clocks.start()
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    launches = 0
+    for _ in range(a.steps):
+        step()
+        for s in ctx.stage_times():
+            g = stages.setdefault(s["name"], {"ms": 0.0, "bytes": 0, "launches": 0, "count": 0})
+            for k in ("ms", "bytes", "launches", "count"):
+                g[k] += s[k]
+        launches += ctx.stats()["kernel_launches"]
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    ck = clocks.stop()
+    ctx.enable_timing(False)
+    elapsed_ms = ev0.elapsed_time(ev1)
+    if world > 1:
+        tmax = torch.tensor([elapsed_ms], device=dev)
+        torch.distributed.all_reduce(tmax, op=torch.distributed.ReduceOp.MAX)
+        elapsed_ms = float(tmax.item())
+    st = ctx.stats()
+    dplan = ctx.device_plan()
+    ms_per_step = elapsed_ms / a.steps
+    value = (n_local * world) * a.steps / (elapsed_ms / 1e3)
+
+    # roofline of the dominant kernel (largest share of the step)
+    peak, peak_src = load_peaks()
+    dom = max(stages.items(), key=lambda kv: kv[1]["ms"])
+    per_launch_bytes = dom[1]["bytes"] / max(dom[1]["count"], 1)
+    per_launch_ms = dom[1]["ms"] / max(dom[1]["count"], 1)
+    achieved = per_launch_bytes / (per_launch_ms * 1e-3) / 1e9
+    traffic = load_ncu_traffic().get(a.config, {}).get(dom[0])
+    roofline = {"bound": "hbm", "kernel": dom[0], "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": per_launch_bytes, "ms_per_launch": per_launch_ms,
+                "share_of_step": dom[1]["ms"] / a.steps / ms_per_step}
+    all_bytes = sum(v["bytes"] for v in stages.values()) / a.steps
+    path = {"algorithmic_bytes_per_step": all_bytes,
+            "achieved_gbs_over_step": all_bytes / (ms_per_step * 1e-3) / 1e9}
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
+        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded, on device)",
+        "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": n_local * world,
+                   "kernels": sp.n_kernels, "eps": eps, "conf": a.conf, "metrics": nm,
+                   "parallelism": "single GPU" if world == 1 else f"{world} independent row shards",
+                   "l2": "inputs 8 B/row x rows >> 126 MB L2 (no flush needed)" if n_local >= 50_000_000
+                   else "inputs fit in L2: latency-bound workload",
+                   "sort_key_bits": st["key_bits"], "sort_passes": st["sort_passes"],
+                   "root_levels": st["levels"], "clusters": dplan["n_clusters"], "samples": dplan["n_samples"],
+                   "active_rows_over_levels": st["active_rows"]},
+        "clocks": ck,
+        "gpu_launches": launches,
+        "roofline": roofline,
+        "path": path,
+        "stages_ms_per_step": {k: v["ms"] / a.steps for k, v in sorted(stages.items(), key=lambda kv: -kv[1]["ms"])},
+    }
+
+    # e2e: same metric through the public API with HOST buffers (pinned), host plan out
+    if not a.no_e2e:
+        hk = torch.empty(n_local, dtype=torch.int32, pin_memory=True)
+        ht = torch.empty(n_local, dtype=torch.int32, pin_memory=True)
+        hk.copy_(kid)
+        ht.copy_(tt)
+        hm = None
+        if nm:
+            hm = torch.empty((nm, n_local), dtype=torch.float64, pin_memory=True)
+            hm.copy_(met)
+        torch.cuda.synchronize()
+        e2e_steps = max(1, min(a.steps, 3))
+        d2h = 0
+        p = ctx.plan(hk, ht, sp.n_kernels, eps=eps, conf=a.conf, metrics=hm, seed=12345, stream=stream.cuda_stream)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(e2e_steps):
+            p = ctx.plan(hk, ht, sp.n_kernels, eps=eps, conf=a.conf, metrics=hm, seed=12345,
+                         stream=stream.cuda_stream)
+        e2e_s = (time.perf_counter() - t0) / e2e_steps
+        d2h = p["clusters"].nbytes + p["sample_row"].nbytes + p["sample_cluster"].nbytes + \
+            p["sample_weight"].nbytes + 8 * (6 + nm)
+        line["e2e"] = {"value": n_local * world / e2e_s, "unit": UNIT,
+                       "h2d_bytes_per_step": n_local * (8 + 8 * nm), "d2h_bytes_per_step": int(d2h),
+                       "ms_per_step": e2e_s * 1e3, "steps": e2e_steps}
+        del hk, ht, hm
+
+    # cpu_baseline: the oracle as it stands, on a bounded sample of the same workload (rank 0, N=1)
+    if not a.no_cpu_baseline and rank == 0 and world == 1:
+        import oracle
+        m = min(a.cpu_sample_rows, n_local)
+        k_np = kid[:m].cpu().numpy().view(np.uint32)
+        t_np = tt[:m].cpu().numpy().view(np.uint32)
+        m_np = met[:, :m].cpu().numpy() if nm else None
+        t0 = time.perf_counter()
+        oracle.plan(k_np, t_np, sp.n_kernels, eps=eps, z=dplan["z"], seed=12345, metrics=m_np)
+        cs = time.perf_counter() - t0
+        line["cpu_baseline"] = {"value": m / cs, "unit": UNIT, "cores": 1, "kind": "oracle",
+                                "sample": f"first {m} rows of {a.config} ({cs:.1f} s, single-threaded C oracle)",
+                                "host_nproc": os.cpu_count()}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+def main():
+    a = parse()
+    if a.impl == "reference":
+        run_reference(a)
+    else:
+        run_ours(a)
+
+
+if __name__ == "__main__":
+    main()

@@ -140,6 +140,16 @@ typedef struct stem_stats {
     double   ssum;             /* RN(exact sum_i sqrt(mu_i V_i)) of the global KKT solve          */
 } stem_stats;
 
+/* Per-stage device time of the last plan (stem_ctx_enable_timing).  bytes is
+ * the stage's algorithmic HBM traffic as DESIGN.md §6 defines it. */
+typedef struct stem_stage_time {
+    char     name[24];         /* e.g. "sort_pass_mid", "root_split"                            */
+    double   ms;               /* summed CUDA-event time over the stage's occurrences            */
+    uint64_t bytes;            /* summed algorithmic bytes                                       */
+    uint32_t launches;         /* kernels launched by the stage                                  */
+    uint32_t count;            /* occurrences (passes, levels)                                    */
+} stem_stage_time;
+
 typedef struct stem_ctx stem_ctx;
 
 /* Fill *o with the defaults: seed 0, z 0, scope 0, root 1, clamp_in_split 1,
@@ -165,6 +175,12 @@ STEM_API int stem_root_plan(const stem_trace *trace, double eps, double conf, co
 
 STEM_API int stem_ctx_device_plan(const stem_ctx *ctx, stem_device_plan *view);
 STEM_API int stem_ctx_stats(const stem_ctx *ctx, stem_stats *stats);
+
+/* Bracket every stage of later plans on ctx with CUDA events (on = 1) or stop
+ * (on = 0).  stem_ctx_stage_times copies up to cap records of the last plan
+ * into out and the number available into *count. */
+STEM_API int stem_ctx_enable_timing(stem_ctx *ctx, int on);
+STEM_API int stem_ctx_stage_times(const stem_ctx *ctx, stem_stage_time *out, uint32_t cap, uint32_t *count);
 
 STEM_API void        stem_plan_free(stem_plan *p);  /* frees everything in the plan; NULL-safe */
 STEM_API const char *stem_strerror(int status);     /* static string, never NULL               */

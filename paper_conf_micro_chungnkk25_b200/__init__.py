@@ -91,8 +91,14 @@ class stem_stats(C.Structure):
                 ("n_samples", C.c_uint64), ("ssum", C.c_double)]
 
 
+class stem_stage_time(C.Structure):
+    _fields_ = [("name", C.c_char * 24), ("ms", C.c_double), ("bytes", C.c_uint64), ("launches", C.c_uint32),
+                ("count", C.c_uint32)]
+
+
 EXPORTS = ["stem_default_opts", "stem_ctx_create", "stem_ctx_destroy", "stem_root_plan_ctx", "stem_root_plan",
-           "stem_ctx_device_plan", "stem_ctx_stats", "stem_plan_free", "stem_strerror", "stem_z_from_conf"]
+           "stem_ctx_device_plan", "stem_ctx_stats", "stem_plan_free", "stem_strerror", "stem_z_from_conf",
+           "stem_ctx_enable_timing", "stem_ctx_stage_times"]
 
 _lib = None
 
@@ -119,6 +125,8 @@ def lib():
         L.stem_strerror.argtypes = [C.c_int]
         L.stem_strerror.restype = C.c_char_p
         L.stem_z_from_conf.argtypes = [C.c_double, P(C.c_double)]
+        L.stem_ctx_enable_timing.argtypes = [C.c_void_p, C.c_int]
+        L.stem_ctx_stage_times.argtypes = [C.c_void_p, P(stem_stage_time), C.c_uint32, P(C.c_uint32)]
         _lib = L
     return _lib
 
@@ -232,16 +240,45 @@ class Context:
                     bound=v.bound, eps=v.eps, z=v.z, true_total_ns=int(v.true_total_ns),
                     est_metric=[v.est_metric[i] for i in range(v.n_metrics)])
 
+    def enable_timing(self, on: bool = True):
+        _check(lib().stem_ctx_enable_timing(self._h, int(on)), "stem_ctx_enable_timing")
+
+    def stage_times(self) -> list:
+        cnt = C.c_uint32()
+        _check(lib().stem_ctx_stage_times(self._h, None, 0, C.byref(cnt)), "stem_ctx_stage_times")
+        arr = (stem_stage_time * max(cnt.value, 1))()
+        _check(lib().stem_ctx_stage_times(self._h, arr, cnt.value, C.byref(cnt)), "stem_ctx_stage_times")
+        return [dict(name=a.name.decode(), ms=a.ms, bytes=a.bytes, launches=a.launches, count=a.count)
+                for a in arr[:cnt.value]]
+
     def stats(self) -> dict:
         s = stem_stats()
         _check(lib().stem_ctx_stats(self._h, C.byref(s)), "stem_ctx_stats")
         return {f: getattr(s, f) for f, _ in stem_stats._fields_}
 
 
-def plan(kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, device: int = 0, **kw):
-    """One-shot stem_root_plan through a temporary Context."""
-    ctx = Context(device)
-    try:
-        return ctx.plan(kernel_id, exec_ns, n_kernels, eps, conf, **kw)
-    finally:
-        ctx.close()
+def plan(kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, metrics=None, seed: int = 0,
+         z: float = 0.0, scope: int = 0, root: bool = True, clamp_in_split: bool = True, census_cap: bool = False,
+         stream=None) -> dict:
+    """stem_root_plan: one-shot plan (temporary workspace), host plan out."""
+    kp, kdev, k_keep = _arg(kernel_id, np.uint32)
+    tp, tdev, t_keep = _arg(exec_ns, np.uint32)
+    if kdev != tdev:
+        raise ValueError("kernel_id and exec_ns must live on the same device")
+    n = int(np.prod(getattr(k_keep, "shape", (0,))))
+    nm, mp, m_keep = 0, None, None
+    if metrics is not None:
+        mp, _, m_keep = _arg(metrics, np.float64)
+        nm = int(m_keep.shape[0]) if len(m_keep.shape) == 2 else 1
+    if stream is None and kdev >= 0:
+        import torch
+        stream = torch.cuda.current_stream(kdev).cuda_stream
+    tr = stem_trace(n, n_kernels, kp, tp, nm, mp, kdev)
+    o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
+                  stream or None)
+    out = C.POINTER(stem_plan)()
+    _check(lib().stem_root_plan(C.byref(tr), eps, conf, C.byref(o), C.byref(out)), "stem_root_plan")
+    del k_keep, t_keep, m_keep
+    res = _plan_to_numpy(out.contents)
+    lib().stem_plan_free(out)
+    return res

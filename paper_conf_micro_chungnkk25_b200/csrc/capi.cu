@@ -105,6 +105,7 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
     c.have_plan = false;
     c.launches = 0;
     c.stats = stem_stats{};
+    c.timing.reset();
     CKS(validate(tr, eps, conf, o));
     CK(cudaSetDevice(c.device));
     if (tr->device >= 0 && tr->device != c.device) return STEM_E_INVAL;
@@ -148,6 +149,10 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
     c.eps = eps;
     c.z = z;
     c.stats.kernel_launches = c.launches;
+    if (c.timing.on) {
+        CK(cudaStreamSynchronize(c.stream));
+        c.timing.finish();
+    }
     c.have_plan = true;
     return STEM_OK;
 }
@@ -291,6 +296,27 @@ int stem_ctx_device_plan(const stem_ctx *ctx, stem_device_plan *v) {
 int stem_ctx_stats(const stem_ctx *ctx, stem_stats *s) {
     if (!ctx || !s) return STEM_E_INVAL;
     *s = ctx->c.stats;
+    return STEM_OK;
+}
+
+int stem_ctx_enable_timing(stem_ctx *ctx, int on) {
+    if (!ctx) return STEM_E_INVAL;
+    ctx->c.timing.on = on != 0;
+    return STEM_OK;
+}
+
+int stem_ctx_stage_times(const stem_ctx *ctx, stem_stage_time *out, uint32_t cap, uint32_t *count) {
+    if (!ctx || !count || (cap && !out)) return STEM_E_INVAL;
+    const auto &agg = ctx->c.timing.agg;
+    *count = (uint32_t)agg.size();
+    for (uint32_t i = 0; i < cap && i < agg.size(); i++) {
+        memset(&out[i], 0, sizeof(stem_stage_time));
+        strncpy(out[i].name, agg[i].name, sizeof(out[i].name) - 1);
+        out[i].ms = agg[i].ms;
+        out[i].bytes = agg[i].bytes;
+        out[i].launches = agg[i].launches;
+        out[i].count = agg[i].count;
+    }
     return STEM_OK;
 }
 

@@ -1,6 +1,8 @@
 // internal.h -- host-side context and stage entry points of libstemroot.
 #pragma once
 #include <cstdint>
+#include <cstring>
+#include <vector>
 #include <cuda_runtime.h>
 
 #include "../../include/stemroot.h"
@@ -45,6 +47,45 @@ struct DevScalars {
 constexpr int kFixDigits = 6;     // 6 x 32-bit digits in u64 lanes, LSB 2^-72
 constexpr int kFixLsb = 72;
 
+// Optional per-stage CUDA-event timing (stem_ctx_enable_timing): each stage
+// brackets its launches with two events on the plan's stream.
+struct StageAgg {
+    const char *name;
+    double ms;
+    uint64_t bytes;       // algorithmic bytes, summed over occurrences
+    uint32_t launches, count;
+};
+
+struct Timing {
+    bool on = false;
+    struct Pending { const char *name; cudaEvent_t a, b; uint64_t bytes; uint32_t launches; };
+    std::vector<cudaEvent_t> pool;
+    size_t used = 0;
+    std::vector<Pending> pend;
+    std::vector<StageAgg> agg;
+    cudaEvent_t get() {
+        if (used == pool.size()) {
+            cudaEvent_t e;
+            cudaEventCreate(&e);
+            pool.push_back(e);
+        }
+        return pool[used++];
+    }
+    void reset() { used = 0; pend.clear(); agg.clear(); }
+    void finish() {   // stream already synchronised
+        for (auto &p : pend) {
+            float ms = 0.f;
+            cudaEventElapsedTime(&ms, p.a, p.b);
+            StageAgg *g = nullptr;
+            for (auto &x : agg) if (!strcmp(x.name, p.name)) g = &x;
+            if (!g) { agg.push_back(StageAgg{p.name, 0.0, 0, 0, 0}); g = &agg.back(); }
+            g->ms += ms; g->bytes += p.bytes; g->launches += p.launches; g->count++;
+        }
+        pend.clear();
+    }
+    ~Timing() { for (auto e : pool) cudaEventDestroy(e); }
+};
+
 struct Ctx {
     int device = 0;
     int sms = 148;
@@ -52,6 +93,22 @@ struct Ctx {
     uint32_t launches = 0;
     int tbits = 0;
     stem_stats stats{};
+    Timing timing;
+    // stage bracket: returns an index to pass to stage_end (or -1 when timing is off)
+    int stage_begin(const char *name) {
+        if (!timing.on) return -1;
+        cudaEvent_t a = timing.get(), b = timing.get();
+        cudaEventRecord(a, stream);
+        timing.pend.push_back(Timing::Pending{name, a, b, 0, launches});
+        return (int)timing.pend.size() - 1;
+    }
+    void stage_end(int tok, uint64_t bytes) {
+        if (tok < 0) return;
+        auto &p = timing.pend[tok];
+        cudaEventRecord(p.b, stream);
+        p.bytes = bytes;
+        p.launches = launches - p.launches;
+    }
 
     // ---- workspace (grow-only)
     template <class T>

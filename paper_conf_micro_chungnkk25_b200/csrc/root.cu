@@ -33,6 +33,7 @@ int prefix_moments(Ctx &c, uint64_t n) {
     uint64_t *P1 = c.P1;
     u128 *P2 = c.P2;
     CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(n + 1) + 1) * sizeof(SQ)));
+    const int tk = c.stage_begin("prefix_moments");
     exclusive_scan<SQ>(
         [t, n] __device__(uint64_t i) -> SQ {
             if (i >= n) return SQ{0, 0};
@@ -45,6 +46,7 @@ int prefix_moments(Ctx &c, uint64_t n) {
         },
         n + 1, (SQ *)c.scan_scratch, (SQ *)c.scalars->wide_total,
         c.stream, &c.launches);
+    c.stage_end(tk, 4 * n + 24 * (n + 1));
     CK(cudaGetLastError());
     return STEM_OK;
 }
@@ -314,14 +316,20 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CKS(c.ensure(c.f_lo[nxt], c.cap_flo[nxt], sizeof(uint32_t) * 2 * C));
         CKS(c.ensure(c.f_hi[nxt], c.cap_fhi[nxt], sizeof(uint32_t) * 2 * C));
         CKS(c.ensure(c.f_aoff[nxt], c.cap_faoff[nxt], sizeof(uint32_t) * 2 * C));
+        const int tk_s = c.stage_begin("root_split");
         split_kernel<<<(unsigned)ntiles, kSplitThreads, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], (uint32_t)C, A,
                                                                 c.P1, c.cut, (Part *)c.split_part);
         fixup_kernel<<<(unsigned)((C * 32 + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur],
                                                                        (uint32_t)C, (const Part *)c.split_part, c.cut);
+        c.launches += 2;
+        c.stage_end(tk_s, 8 * A + 4 * C * 3);
+        const int tk_d = c.stage_begin("root_decide");
         DecideArgs da{c.f_lo[cur], c.f_hi[cur], c.cut, (uint32_t)C, c.P1, c.P2, c.t_sorted, c.flags, c.cnt_sz,
                       eps, z, k2, clamp};
         decide_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(da);
-        c.launches += 3;
+        c.launches += 1;
+        c.stage_end(tk_d, 96 * C);
+        const int tk_c = c.stage_begin("root_compact");
         CK(cudaGetLastError());
         const uint32_t *flo = c.f_lo[cur], *fhi = c.f_hi[cur], *fcut = c.cut, *t = c.t_sorted;
         const uint64_t *cs = c.cnt_sz;
@@ -341,6 +349,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                 }
             },
             C, (uint64_t *)c.scan_scratch, &c.scalars->frontier_total, st, &c.launches);
+        c.stage_end(tk_c, 8 * C + 24 * C);
         CK(cudaGetLastError());
         CKS(read_frontier_total(c, C, A));
         cur = nxt;

@@ -256,9 +256,11 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
     if (sm_bytes > 48 * 1024)
         CK(cudaFuncSetAttribute(prepass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_bytes));
     const int blocks = c.sms * (smem_kid && K > 8192 ? 2 : 4);
+    const int tk_pre = c.stage_begin("prepass");
     prepass_kernel<<<blocks, 256, sm_bytes, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.hist,
                                                   &c.scalars->max_t, &c.scalars->err);
     c.launches++;
+    c.stage_end(tk_pre, 8 * n);
     CK(cudaGetLastError());
     DevScalars hs;
     CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
@@ -302,6 +304,10 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
         a.row_out = c.row_sorted;
         const size_t smem = kSortTile * (sizeof(uint64_t) + sizeof(uint32_t)) +
                             sizeof(uint32_t) * kRadix * (kSortWarps + (first ? 7 : 0));
+        const char *sname = (first && last) ? "sort_pass_only" : first ? "sort_pass_first"
+                            : last ? "sort_pass_last" : "sort_pass_mid";
+        const uint64_t sbytes = n * ((first ? 8 : 12) + (last ? 8 : 12));
+        const int tk = c.stage_begin(sname);
         int rc;
         if (first && last) rc = launch_pass<true, true>(a, ntiles, smem, st);
         else if (first) rc = launch_pass<true, false>(a, ntiles, smem, st);
@@ -309,17 +315,20 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
         else rc = launch_pass<false, false>(a, ntiles, smem, st);
         CKS(rc);
         c.launches++;
+        c.stage_end(tk, sbytes);
         CK(cudaGetLastError());
-        uint64_t *tk = kin; kin = kout; kout = tk;
+        uint64_t *tkk = kin; kin = kout; kout = tkk;
         uint32_t *tv = vin; vin = vout; vout = tv;
     }
     // group offsets: goff = exclusive scan of kernel counts
     const uint32_t *cnt = c.kid_count;
     uint32_t *goff = c.goff;
+    const int tk_g = c.stage_begin("group_offsets");
     exclusive_scan<uint64_t>(
         [cnt, K] __device__(uint64_t i) -> uint64_t { return i < K ? (uint64_t)cnt[i] : 0; },
         [goff] __device__(uint64_t i, uint64_t pre, uint64_t) { goff[i] = (uint32_t)pre; },
         (uint64_t)K + 1, (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
+    c.stage_end(tk_g, 8 * ((uint64_t)K + 1));
     CK(cudaGetLastError());
     return STEM_OK;
 }

@@ -318,6 +318,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     // a5: leaf starts = group starts U accepted cuts, in row order = canonical (kernel, lo) order
     CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(n) + 1) * sizeof(uint64_t)));
     CKS(c.ensure(c.leaf_lo, c.cap_leaf_lo, sizeof(uint32_t) * (n + 1)));
+    const int tk_leaf = c.stage_begin("leaf_table");
     {
         const uint8_t *flags = c.flags;
         uint32_t *leaf_lo = c.leaf_lo;
@@ -328,6 +329,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
                                  n, (uint64_t *)c.scan_scratch, &c.scalars->n_leaves, st, &c.launches);
         CK(cudaGetLastError());
     }
+    c.stage_end(tk_leaf, n);
     uint64_t L = 0;
     CK(cudaMemcpyAsync(&L, &c.scalars->n_leaves, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -348,6 +350,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CK(cudaMemsetAsync(c.kern_T, 0, sizeof(uint64_t) * nsets, st));
     CK(cudaMemsetAsync(c.leaf_U, 0, sizeof(uint64_t) * (L + 1), st));
 
+    const int tk_kkt = c.stage_begin("stem_sizes");
     LeafArgs la{c.leaf_lo, c.goff, c.t_sorted, c.P1, c.P2, L, n, K, o.scope, leaf_kid, leaf_ord,
                 c.fix_acc, c.kern_T, &c.scalars->err};
     leaf_kkt_kernel<<<blocks_for(L), kThreads, 0, st>>>(la);
@@ -372,6 +375,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
                                  (uint64_t *)c.scan_scratch, &c.scalars->total_m, st, &c.launches);
         CK(cudaGetLastError());
     }
+    c.stage_end(tk_kkt, 64 * L);
     DevScalars hs;
     CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -391,8 +395,10 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     SampleArgs sa{c.leaf_lo, leaf_kid, leaf_ord, c.leaf_moff, c.leaf_m, c.leaf_census, c.t_sorted, c.row_sorted,
                   L, n, S, (uint32_t)o.seed, (uint32_t)(o.seed >> 32), c.out_row, c.out_cluster, c.out_weight,
                   c.leaf_U};
+    const int tk_smp = c.stage_begin("samples");
     if (S) sample_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa);
     c.launches += S ? 1 : 0;
+    c.stage_end(tk_smp, 40 * S);
     CK(cudaGetLastError());
 
     // a8: estimate, bound, metrics (deterministic block partials)
@@ -402,6 +408,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CKS(c.ensure(c.red_part, c.cap_red, sizeof(double) * part_doubles));
     double *part_est = c.red_part, *part_met = c.red_part + 2 * eb, *red_out = part_met + mb * (nm ? nm : 1);
     CK(cudaMemsetAsync(&c.scalars->sum_q, 0, sizeof(uint64_t), st));
+    const int tk_est = c.stage_begin("estimate");
     EstArgs ea{c.leaf_lo, c.P1, c.P2, c.leaf_m, c.leaf_U, L, n, &c.scalars->sum_q, part_est};
     estimate_kernel<<<(unsigned)eb, kThreads, 0, st>>>(ea);
     reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_est, eb, 2, red_out);
@@ -412,11 +419,14 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_met, mb, nm, red_out + 2);
         c.launches += 2;
     }
+    c.stage_end(tk_est, 56 * L + 12 * S * nm);
     // a5 output records
     CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
+    const int tk_pack = c.stage_begin("pack");
     pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.P1, c.P2, c.t_sorted, c.leaf_m,
                                                    c.leaf_census, L, n, c.out_clusters);
     c.launches++;
+    c.stage_end(tk_pack, 88 * L);
     CK(cudaGetLastError());
     double *est_out = red_out + 2 + nm;
     est_finalize_kernel<<<1, 1, 0, st>>>(&c.scalars->sum_q, red_out, c.P1 + n, z, est_out);

@@ -147,7 +147,7 @@ def test_determinism(ctx):
 def test_z_from_conf_matches_scipy(sr):
     from scipy.stats import norm
     for conf in (0.8, 0.9, 0.95, 0.99, 0.999999):
-        assert sr.z_from_conf(conf) == pytest.approx(norm.ppf(1 - (1 - conf) / 2), rel=1e-14)
+        assert sr.z_from_conf(conf) == pytest.approx(norm.isf((1 - conf) / 2), rel=1e-14)
 
 
 # ------------------------------------------------------------------ config-shaped traces (BASELINE configs)
