@@ -28,8 +28,8 @@ int Ctx::ensure_all(uint64_t n, uint32_t K, uint32_t n_metrics) {
     CKS(ensure(hist, cap_hist, sizeof(uint64_t) * 8 * 256));
     CKS(ensure(scalars, cap_scalars, sizeof(DevScalars)));
     CKS(ensure(scan_scratch, cap_scan, (scan_tiles((uint64_t)K + 2) + 1) * 32));
-    CKS(ensure(P1, cap_p1, sizeof(uint64_t) * (n + 1)));
-    CKS(ensure(P2, cap_p2, sizeof(u128) * (n + 1)));
+    CKS(ensure(PS1, cap_ps1, sizeof(uint64_t) * (n / kChunk + 2)));
+    CKS(ensure(PS2, cap_ps2, sizeof(u128) * (n / kChunk + 2)));
     CKS(ensure(flags, cap_flags, n + 16));
     return STEM_OK;
 }
@@ -46,11 +46,12 @@ void Ctx::release() {
     for (int i = 0; i < 2; i++) {
         dfree(keys[i], cap_keys[i]); dfree(vals[i], cap_vals[i]);
         dfree(f_lo[i], cap_flo[i]); dfree(f_hi[i], cap_fhi[i]); dfree(f_aoff[i], cap_faoff[i]);
+        dfree(f_S[i], cap_fS[i]); dfree(f_Q[i], cap_fQ[i]);
     }
     dfree(t_sorted, cap_ts); dfree(row_sorted, cap_rs); dfree(kid_count, cap_kc); dfree(goff, cap_goff);
     dfree(hist, cap_hist); dfree(sort_status, cap_status); dfree(scalars, cap_scalars);
-    dfree(scan_scratch, cap_scan); dfree(P1, cap_p1); dfree(P2, cap_p2);
-    dfree(cut, cap_cut); dfree(cnt_sz, cap_cntsz); dfree(split_part, cap_part); dfree(flags, cap_flags);
+    dfree(scan_scratch, cap_scan); dfree(PS1, cap_ps1); dfree(PS2, cap_ps2); dfree(chunk_sq, cap_chunk_sq);
+    dfree(cut, cap_cut); dfree(cut_SL, cap_cut_SL); dfree(cut_QL, cap_cut_QL); dfree(tile_map, cap_tile_map); dfree(cnt_sz, cap_cntsz); dfree(split_part, cap_part); dfree(flags, cap_flags);
     dfree(leaf_lo, cap_leaf_lo); dfree(leaf_m, cap_leaf_m); dfree(leaf_moff, cap_leaf_moff);
     dfree(leaf_U, cap_leaf_U); dfree(leaf_census, cap_leaf_census); dfree(leaf_kid, cap_leaf_kid);
     dfree(leaf_ord, cap_leaf_ord); dfree(fix_acc, cap_fix); dfree(kern_T, cap_kern_T); dfree(kern_g, cap_kern_g);

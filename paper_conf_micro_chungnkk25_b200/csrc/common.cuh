@@ -78,22 +78,29 @@ __device__ __forceinline__ int cmp256(const U256 &a, const U256 &b) {
 
 // ---------------------------------------------------------------- split candidates
 // Candidate cut k of a cluster: score = D^2 / p, D = n*S_L - S*k (< 0 for a
-// valid cut of sorted data), p = k (n - k).  f is the fp64 filter value.
+// valid cut of sorted data, |D| < 2^96), p = k (n - k).  f is the fp64
+// filter value; SL = S_L(k) travels with the candidate to the decision.
 struct Cand {
     double f;
-    u128 absD;
+    uint64_t dlo;   // |D| bits 0..63
     uint64_t p;
-    uint32_t k;  // 0 = no candidate
+    uint64_t SL;
+    uint32_t dhi;   // |D| bits 64..95
+    uint32_t k;     // 0 = no candidate
 };
 
 __device__ __forceinline__ Cand no_cand() {
     Cand c;
     c.f = 0.0;
-    c.absD = 0;
+    c.dlo = 0;
     c.p = 0;
+    c.SL = 0;
+    c.dhi = 0;
     c.k = 0;
     return c;
 }
+
+__device__ __forceinline__ u128 cand_absD(const Cand &c) { return ((u128)c.dhi << 64) | c.dlo; }
 
 // Exact strict total order (R5): larger score first, ties -> smaller k.
 // The fp64 filter decides only when the scores differ by > 2^-40 relative;
@@ -104,7 +111,7 @@ __device__ __forceinline__ bool better(const Cand &a, const Cand &b) {
     const double tol = 1.0 + 0x1p-40;
     if (a.f > __dmul_rn(b.f, tol)) return true;
     if (b.f > __dmul_rn(a.f, tol)) return false;
-    const int c = cmp256(sq_times(a.absD, b.p), sq_times(b.absD, a.p));
+    const int c = cmp256(sq_times(cand_absD(a), b.p), sq_times(cand_absD(b), a.p));
     if (c != 0) return c > 0;
     return a.k < b.k;
 }
@@ -112,12 +119,38 @@ __device__ __forceinline__ bool better(const Cand &a, const Cand &b) {
 __device__ __forceinline__ Cand make_cand(uint64_t n, uint64_t S, uint64_t SL, uint32_t k) {
     Cand c;
     const u128 a = (u128)n * SL, b = (u128)S * k;
-    c.absD = a > b ? a - b : b - a;
+    const u128 d = a > b ? a - b : b - a;
+    c.dlo = (uint64_t)d;
+    c.dhi = (uint32_t)(d >> 64);
     c.p = (uint64_t)k * (n - k);
-    const double dD = rn128(c.absD);
+    c.SL = SL;
+    const double dD = rn128(d);
     c.f = __ddiv_rn(__dmul_rn(dD, dD), rn64(c.p));
     c.k = k;
     return c;
+}
+
+// ---------------------------------------------------------------- sampled prefix moments
+// PS1[j] = sum_{i < 32 j} t[i] (u64), PS2[j] = sum_{i < 32 j} t[i]^2 (u128).
+// Prefix at any row x = chunk prefix + at most 31 loads of t.
+constexpr int kChunkLog = 5;
+constexpr uint64_t kChunk = 1ull << kChunkLog;
+
+__device__ __forceinline__ uint64_t pref1(const uint64_t *PS1, const uint32_t *t, uint64_t x) {
+    uint64_t s = PS1[x >> kChunkLog];
+    for (uint64_t i = x & ~(kChunk - 1); i < x; i++) s += t[i];
+    return s;
+}
+
+__device__ __forceinline__ void pref12(const uint64_t *PS1, const u128 *PS2, const uint32_t *t, uint64_t x,
+                                       uint64_t &s, u128 &q) {
+    s = PS1[x >> kChunkLog];
+    q = PS2[x >> kChunkLog];
+    for (uint64_t i = x & ~(kChunk - 1); i < x; i++) {
+        const uint64_t v = t[i];
+        s += v;
+        q += (u128)(v * v);
+    }
 }
 
 // ---------------------------------------------------------------- Philox4x32-10

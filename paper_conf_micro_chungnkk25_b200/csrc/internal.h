@@ -138,13 +138,19 @@ struct Ctx {
     void *sort_status = nullptr; size_t cap_status = 0;
     DevScalars *scalars = nullptr; size_t cap_scalars = 0;
     void *scan_scratch = nullptr; size_t cap_scan = 0;
-    // prefix moments (a2)
-    uint64_t *P1 = nullptr; size_t cap_p1 = 0;
-    u128 *P2 = nullptr; size_t cap_p2 = 0;
+    // sampled prefix moments (a2): PS1/PS2 every kChunk rows
+    uint64_t *PS1 = nullptr; size_t cap_ps1 = 0;
+    u128 *PS2 = nullptr; size_t cap_ps2 = 0;
+    void *chunk_sq = nullptr; size_t cap_chunk_sq = 0;
     // ROOT frontier (a3/a4)
     uint32_t *f_lo[2] = {nullptr, nullptr}, *f_hi[2] = {nullptr, nullptr}, *f_aoff[2] = {nullptr, nullptr};
     size_t cap_flo[2] = {0, 0}, cap_fhi[2] = {0, 0}, cap_faoff[2] = {0, 0};
+    uint64_t *f_S[2] = {nullptr, nullptr}; size_t cap_fS[2] = {0, 0};
+    u128 *f_Q[2] = {nullptr, nullptr}; size_t cap_fQ[2] = {0, 0};
     uint32_t *cut = nullptr; size_t cap_cut = 0;
+    uint64_t *cut_SL = nullptr; size_t cap_cut_SL = 0;
+    u128 *cut_QL = nullptr; size_t cap_cut_QL = 0;
+    uint32_t *tile_map = nullptr; size_t cap_tile_map = 0;
     uint64_t *cnt_sz = nullptr; size_t cap_cntsz = 0;
     void *split_part = nullptr; size_t cap_part = 0;
     uint8_t *flags = nullptr; size_t cap_flags = 0;

@@ -1,23 +1,27 @@
-// root.cu -- steps a2-a4: exact prefix moments of the grouped times and the
-// level-synchronous ROOT clustering (§3.4, Fig. 6).
+// root.cu -- steps a2-a4: sampled exact prefix moments of the grouped times
+// and the level-synchronous ROOT clustering (§3.4, Fig. 6).
 //
 // Every level processes the whole frontier (all kernels' active clusters at
 // once) as one segmented operation over the concatenated active rows:
-//   split_kernel   tiles of 2048 active rows; each candidate cut k of a
-//                  cluster [lo,hi) is scored exactly from P1 (D = n S_L - S k,
-//                  score D^2/(k(n-k)), R5); thread-, then block-level segmented
-//                  argmax; clusters inside a tile finish here.
-//   fixup_kernel   one warp per cluster spanning several tiles: argmax of the
-//                  per-tile partials.
-//   decide_kernel  Eq. 7 vs Eq. 8 per cluster (R6-R9) in the fixed fp64 order.
-//   scan + apply   compacts the non-trivial children into the next frontier.
+//   tile_map_kernel  first/last frontier cluster of every 2048-row tile
+//   split_kernel     stages the tile's t in shared memory (coalesced), block
+//                    scan of t gives S_L for every candidate cut k, scored
+//                    exactly (D = n S_L - S k, score D^2/(k(n-k)), R5);
+//                    thread- then block-level segmented argmax; clusters
+//                    inside a tile finish here
+//   fixup_kernel     one warp per cluster spanning several tiles
+//   decide_kernel    Eq. 7 vs Eq. 8 per cluster (R6-R9) in the fixed fp64 order
+//   scan + apply     compacts the non-trivial children into the next frontier
+// Cluster totals (S exact u64, Q exact u128) travel with the frontier; only
+// Q_L at the chosen cut is read from the sampled prefix arrays.
 #include "internal.h"
 
 namespace sr {
 
 constexpr int kSplitThreads = 256;
 constexpr int kSplitItems = 8;
-constexpr uint64_t kSplitTile = (uint64_t)kSplitThreads * kSplitItems;
+constexpr int kTile = kSplitThreads * kSplitItems;      // 2048 active rows
+constexpr int kMaxTileClusters = kTile / 2 + 2;         // frontier clusters have >= 2 rows
 constexpr uint32_t kNone = 0xFFFFFFFFu;
 
 struct SQ {
@@ -27,26 +31,44 @@ struct SQ {
 __host__ __device__ __forceinline__ SQ operator+(const SQ &a, const SQ &b) { return SQ{a.s + b.s, a.q + b.q}; }
 __host__ __device__ __forceinline__ SQ operator-(const SQ &a, const SQ &b) { return SQ{a.s - b.s, a.q - b.q}; }
 
-// ---------------------------------------------------------------- a2: P1, P2
+// ---------------------------------------------------------------- a2: sampled P1, P2
+__global__ void __launch_bounds__(256) chunk_sums_kernel(const uint32_t *__restrict__ t, uint64_t n, uint64_t nchunks,
+                                                         SQ *__restrict__ out) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t warps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t j = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < nchunks; j += warps) {
+        const uint64_t i = j * kChunk + lane;
+        const uint64_t v = i < n ? t[i] : 0;
+        uint64_t s = v, qlo = v * v, qhi = 0;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            s += __shfl_xor_sync(0xffffffffu, s, o);
+            const uint64_t ol = __shfl_xor_sync(0xffffffffu, qlo, o), oh = __shfl_xor_sync(0xffffffffu, qhi, o);
+            const uint64_t nl = qlo + ol;
+            qhi += oh + (nl < qlo);
+            qlo = nl;
+        }
+        if (lane == 0) out[j] = SQ{s, ((u128)qhi << 64) | qlo};
+    }
+}
+
 int prefix_moments(Ctx &c, uint64_t n) {
-    const uint32_t *t = c.t_sorted;
-    uint64_t *P1 = c.P1;
-    u128 *P2 = c.P2;
-    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(n + 1) + 1) * sizeof(SQ)));
+    const uint64_t nchunks = (n + kChunk - 1) / kChunk;
+    CKS(c.ensure(c.chunk_sq, c.cap_chunk_sq, sizeof(SQ) * (nchunks + 1)));
+    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(nchunks + 1) + 1) * sizeof(SQ)));
     const int tk = c.stage_begin("prefix_moments");
-    exclusive_scan<SQ>(
-        [t, n] __device__(uint64_t i) -> SQ {
-            if (i >= n) return SQ{0, 0};
-            const uint64_t x = t[i];
-            return SQ{x, (u128)(x * x)};
-        },
-        [P1, P2] __device__(uint64_t i, SQ pre, SQ) {
-            P1[i] = pre.s;
-            P2[i] = pre.q;
-        },
-        n + 1, (SQ *)c.scan_scratch, (SQ *)c.scalars->wide_total,
-        c.stream, &c.launches);
-    c.stage_end(tk, 4 * n + 24 * (n + 1));
+    SQ *cs = (SQ *)c.chunk_sq;
+    chunk_sums_kernel<<<c.sms * 8, 256, 0, c.stream>>>(c.t_sorted, n, nchunks, cs);
+    c.launches++;
+    uint64_t *PS1 = c.PS1;
+    u128 *PS2 = c.PS2;
+    exclusive_scan<SQ>([cs, nchunks] __device__(uint64_t j) -> SQ { return j < nchunks ? cs[j] : SQ{0, 0}; },
+                       [PS1, PS2] __device__(uint64_t j, SQ pre, SQ) {
+                           PS1[j] = pre.s;
+                           PS2[j] = pre.q;
+                       },
+                       nchunks + 1, (SQ *)c.scan_scratch, (SQ *)c.scalars->wide_total, c.stream, &c.launches);
+    c.stage_end(tk, 4 * n + 24 * (nchunks + 1));
     CK(cudaGetLastError());
     return STEM_OK;
 }
@@ -61,64 +83,186 @@ __device__ __forceinline__ bool nontrivial(const uint32_t *t, uint32_t lo, uint3
     return hi - lo >= 2 && t[lo] != t[hi - 1];
 }
 
-__global__ void __launch_bounds__(kSplitThreads)
-split_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, const uint32_t *__restrict__ aoff,
-             uint32_t C, uint64_t A, const uint64_t *__restrict__ P1, uint32_t *__restrict__ cut,
-             Part *__restrict__ part) {
-    __shared__ uint32_t s_c[2 * kSplitThreads];
-    __shared__ Cand s_v[2 * kSplitThreads];
-    const int tid = threadIdx.x;
-    const uint64_t tile_start = (uint64_t)blockIdx.x * kSplitTile;
-    const uint64_t tile_end = min(tile_start + kSplitTile, A);
-    const uint64_t a0 = tile_start + (uint64_t)tid * kSplitItems;
-    const uint64_t a_end = min(a0 + kSplitItems, tile_end);
+__global__ void tile_map_kernel(const uint32_t *__restrict__ aoff, uint32_t C, uint64_t A, uint64_t ntiles,
+                                uint32_t *__restrict__ first, uint32_t *__restrict__ last) {
+    const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (j >= ntiles) return;
+    const uint64_t ts = j * kTile, te = min(ts + kTile, A);
+    first[j] = (uint32_t)upper_bound(aoff, C, (uint32_t)ts) - 1;
+    last[j] = (uint32_t)upper_bound(aoff, C, (uint32_t)(te - 1)) - 1;
+}
 
+struct SplitArgs {
+    const uint32_t *f_lo, *f_hi, *aoff, *tile_first, *tile_last;
+    const uint64_t *f_S;
+    const uint64_t *PS1;
+    const uint32_t *t;
+    uint64_t A;
+    uint32_t *cut;
+    uint64_t *cut_SL;
+    Part *part;
+};
+
+__host__ __device__ constexpr int padx(int i) { return i + (i >> 3); }   // conflict-free blocked u32 reads
+
+struct SplitSmem {
+    Cand v[2 * kSplitThreads];                 // block segmented argmax entries
+    uint64_t S[kMaxTileClusters], base[kMaxTileClusters];
+    uint64_t red[kSplitThreads / 32 + 1];
+    uint64_t carry;
+    uint32_t t[padx(kTile + 1) + 1];           // t[padx(p + 1)] = t at tile position p; t[0] = halo
+    uint32_t ao[kMaxTileClusters], lo[kMaxTileClusters], n[kMaxTileClusters];
+    uint32_t wmax[kSplitThreads / 32];
+    uint32_t cc[2 * kSplitThreads];
+    uint16_t cid[kTile];                       // tile-relative cluster of every position
+};
+
+__global__ void __launch_bounds__(kSplitThreads) split_kernel(SplitArgs a) {
+    extern __shared__ __align__(16) unsigned char s_dyn[];
+    SplitSmem &sm = *reinterpret_cast<SplitSmem *>(s_dyn);
+    uint32_t *s_t = sm.t;
+    uint16_t *s_cid = sm.cid;
+    uint32_t *s_ao = sm.ao, *s_lo = sm.lo, *s_n = sm.n, *s_wmax = sm.wmax, *s_cc = sm.cc;
+    uint64_t *s_S = sm.S, *s_base = sm.base, *s_red = sm.red;
+    Cand *s_v = sm.v;
+    uint64_t &s_carry = sm.carry;
+
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint64_t ts = (uint64_t)blockIdx.x * kTile;
+    const uint64_t te = min(ts + kTile, a.A);
+    const int nt = (int)(te - ts);
+    const uint32_t c0 = a.tile_first[blockIdx.x];
+    const int nc = (int)(a.tile_last[blockIdx.x] - c0) + 1;
+
+    // cluster table of the tile
+    for (int i = tid; i < nc; i += kSplitThreads) {
+        const uint32_t c = c0 + i, lo = a.f_lo[c];
+        s_ao[i] = a.aoff[c];
+        s_lo[i] = lo;
+        s_n[i] = a.f_hi[c] - lo;
+        s_S[i] = a.f_S[c];
+    }
+    for (int p = tid; p < kTile; p += kSplitThreads) s_cid[p] = 0;
+    __syncthreads();
+    for (int i = tid + 1; i < nc; i += kSplitThreads) s_cid[s_ao[i] - ts] = (uint16_t)i;   // cluster heads
+    // carry into the first cluster when it began before this tile: sum of t over [lo, row(ts))
+    if (w == 0) {
+        uint64_t carry = 0;
+        if (s_ao[0] < ts) {
+            const uint64_t lo = s_lo[0], r = lo + (ts - s_ao[0]);
+            // pref1(r) - pref1(lo); the partial chunk sums are spread over the warp
+            uint64_t part = 0;
+            const uint64_t rb = r & ~(kChunk - 1), lb = lo & ~(kChunk - 1);
+            if (rb + lane < r) part += a.t[rb + lane];
+            if (lb + lane < lo) part -= a.t[lb + lane];
+            for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+            carry = a.PS1[r >> kChunkLog] - a.PS1[lo >> kChunkLog] + part;
+        }
+        if (lane == 0) s_carry = carry;
+    }
+    __syncthreads();
+    // running max over positions (heads carry increasing ids): blocked, 8 per thread
+    {
+        uint32_t run = 0;
+#pragma unroll
+        for (int j = 0; j < kSplitItems; j++) run = max(run, (uint32_t)s_cid[tid * kSplitItems + j]);
+        uint32_t incl = run;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl = max(incl, v);
+        }
+        if (lane == 31) s_wmax[w] = incl;
+        uint32_t pre = __shfl_up_sync(0xffffffffu, incl, 1);
+        if (lane == 0) pre = 0;
+        __syncthreads();
+        for (int ww = 0; ww < w; ww++) pre = max(pre, s_wmax[ww]);
+        uint32_t r = pre;
+#pragma unroll
+        for (int j = 0; j < kSplitItems; j++) {
+            r = max(r, (uint32_t)s_cid[tid * kSplitItems + j]);
+            s_cid[tid * kSplitItems + j] = (uint16_t)r;
+        }
+    }
+    __syncthreads();
+    // coalesced load of t for the tile (striped), plus the halo row before position 0
+    for (int idx = tid; idx <= nt; idx += kSplitThreads) {
+        uint32_t v = 0;
+        if (idx == 0) {
+            if (s_ao[0] < ts) v = a.t[s_lo[0] + (ts - s_ao[0]) - 1];
+        } else {
+            const int p = idx - 1, ci = s_cid[p];
+            v = a.t[s_lo[ci] + (ts + p - s_ao[ci])];
+        }
+        s_t[padx(idx)] = v;
+    }
+    __syncthreads();
+    // block exclusive scan of t over positions -> S_L of every candidate
+    const int p0 = tid * kSplitItems;
+    uint64_t mysum = 0;
+#pragma unroll
+    for (int j = 0; j < kSplitItems; j++)
+        if (p0 + j < nt) mysum += s_t[padx(p0 + j + 1)];
+    uint64_t tot;
+    const uint64_t excl = block_excl_scan<uint64_t, kSplitThreads>(mysum, s_red, &tot);
+    {
+        uint64_t run = excl;
+        for (int j = 0; j < kSplitItems && p0 + j < nt; j++) {
+            const int p = p0 + j, ci = s_cid[p];
+            if (s_ao[ci] == ts + p) s_base[ci] = run;          // cluster starts inside the tile
+            run += s_t[padx(p + 1)];
+        }
+        if (tid == 0 && s_ao[0] < ts) s_base[0] = (uint64_t)0 - s_carry;   // S_L = run + carry (mod 2^64)
+    }
+    __syncthreads();
+
+    // candidates, thread-local segmented argmax
     uint32_t head_c = kNone, tail_c = kNone;
     Cand head_b = no_cand(), tail_b = no_cand();
-    if (a0 < tile_end) {
-        uint32_t c = (uint32_t)upper_bound(aoff, C, (uint32_t)a0) - 1;
-        uint32_t lo = f_lo[c], hi = f_hi[c];
-        uint64_t ao = aoff[c], ae = ao + (hi - lo);
-        uint64_t p1lo = P1[lo], S = P1[hi] - p1lo;
-        uint64_t seg_start = a0;
+    if (p0 < nt) {
+        const int pend = min(p0 + kSplitItems, nt);
+        int ci = s_cid[p0];
+        uint64_t ao = s_ao[ci], ae = ao + s_n[ci];
+        int seg_start = p0;
         Cand best = no_cand();
-        auto flush = [&](uint64_t seg_end) {
-            if (ao >= a0 && ae <= a_end) {
-                cut[c] = best.k;                       // whole cluster inside this thread
-            } else if (seg_start == a0) {
-                head_c = c; head_b = best;
+        uint64_t run = excl;
+        auto flush = [&]() {
+            if (ao >= ts + p0 && ae <= ts + pend) {
+                a.cut[c0 + ci] = best.k;                      // whole cluster inside this thread
+                a.cut_SL[c0 + ci] = best.SL;
+            } else if (seg_start == p0) {
+                head_c = ci; head_b = best;
             } else {
-                tail_c = c; tail_b = best;
+                tail_c = ci; tail_b = best;
             }
         };
-        for (uint64_t a = a0; a < a_end; a++) {
-            if (a >= ae) {
-                flush(a);
-                c++;
-                lo = f_lo[c]; hi = f_hi[c];
-                ao = aoff[c]; ae = ao + (hi - lo);
-                p1lo = P1[lo]; S = P1[hi] - p1lo;
-                seg_start = a;
+        uint32_t tprev = s_t[padx(p0)];
+        for (int p = p0; p < pend; p++) {
+            const int cj = s_cid[p];
+            if (cj != ci) {
+                flush();
+                ci = cj;
+                ao = s_ao[ci];
+                ae = ao + s_n[ci];
+                seg_start = p;
                 best = no_cand();
             }
-            const uint32_t k = (uint32_t)(a - ao);
-            if (k >= 1) {
-                const uint64_t i = lo + k;
-                const uint64_t pm = P1[i - 1], p0 = P1[i], pp = P1[i + 1];
-                if (p0 - pm < pp - p0) {               // t[i-1] < t[i]: cut between distinct values
-                    const Cand cd = make_cand(hi - lo, S, p0 - p1lo, k);
-                    if (better(cd, best)) best = cd;
-                }
+            const uint32_t tc = s_t[padx(p + 1)];
+            const uint32_t k = (uint32_t)(ts + p - ao);
+            if (k >= 1 && tprev < tc) {                       // cut between distinct values only
+                const Cand cd = make_cand(s_n[ci], s_S[ci], run - s_base[ci], k);
+                if (better(cd, best)) best = cd;
             }
+            run += tc;
+            tprev = tc;
         }
-        flush(a_end);
-        if (head_c != kNone && tail_c == kNone) { tail_c = head_c; tail_b = head_b; }  // idempotent duplicate
+        flush();
+        if (head_c != kNone && tail_c == kNone) { tail_c = head_c; tail_b = head_b; }   // idempotent duplicate
     }
-    // block-level segmented argmax (Hillis-Steele over 2 entries per thread;
-    // runs of one cluster are contiguous, so "same id d entries back" = same run)
-    s_c[2 * tid] = head_c;
+    // block-level segmented argmax (Hillis-Steele; a cluster's entries are contiguous)
+    s_cc[2 * tid] = head_c;
     s_v[2 * tid] = head_b;
-    s_c[2 * tid + 1] = tail_c;
+    s_cc[2 * tid + 1] = tail_c;
     s_v[2 * tid + 1] = tail_b;
     __syncthreads();
     for (int d = 1; d < 2 * kSplitThreads; d <<= 1) {
@@ -127,9 +271,9 @@ split_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_h
 #pragma unroll
         for (int h = 0; h < 2; h++) {
             const int e = 2 * tid + h;
-            const uint32_t ce = s_c[e];
+            const uint32_t ce = s_cc[e];
             upd[h] = false;
-            if (ce != kNone && e >= d && s_c[e - d] == ce) {
+            if (ce != kNone && e >= d && s_cc[e - d] == ce) {
                 const Cand o = s_v[e - d];
                 nv[h] = s_v[e];
                 if (better(o, nv[h])) { nv[h] = o; upd[h] = true; }
@@ -144,15 +288,16 @@ split_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_h
 #pragma unroll
     for (int h = 0; h < 2; h++) {
         const int e = 2 * tid + h;
-        const uint32_t ce = s_c[e];
+        const uint32_t ce = s_cc[e];
         if (ce == kNone) continue;
-        if (e + 1 < 2 * kSplitThreads && s_c[e + 1] == ce) continue;   // not the run's last entry
-        const uint64_t ao = aoff[ce], ae = ao + (f_hi[ce] - f_lo[ce]);
-        if (ao >= tile_start && ae <= tile_end) {
-            cut[ce] = s_v[e].k;
+        if (e + 1 < 2 * kSplitThreads && s_cc[e + 1] == ce) continue;   // not the run's last entry
+        const uint64_t ao = s_ao[ce], ae = ao + s_n[ce];
+        if (ao >= ts && ae <= te) {
+            a.cut[c0 + ce] = s_v[e].k;
+            a.cut_SL[c0 + ce] = s_v[e].SL;
         } else {
-            const int slot = (ao <= tile_start) ? 0 : 1;   // first cluster of the tile -> slot 0
-            part[2 * (uint64_t)blockIdx.x + slot] = Part{s_v[e], ce};
+            const int slot = (ao <= ts) ? 0 : 1;   // first cluster of the tile -> slot 0
+            a.part[2 * (uint64_t)blockIdx.x + slot] = Part{s_v[e], c0 + ce};
         }
     }
 }
@@ -160,26 +305,26 @@ split_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_h
 __device__ __forceinline__ Cand shfl_cand(const Cand &a, int src) {
     Cand r;
     r.f = __shfl_sync(0xffffffffu, a.f, src);
-    const uint64_t lo = __shfl_sync(0xffffffffu, (uint64_t)a.absD, src);
-    const uint64_t hi = __shfl_sync(0xffffffffu, (uint64_t)(a.absD >> 64), src);
-    r.absD = ((u128)hi << 64) | lo;
+    r.dlo = __shfl_sync(0xffffffffu, a.dlo, src);
     r.p = __shfl_sync(0xffffffffu, a.p, src);
+    r.SL = __shfl_sync(0xffffffffu, a.SL, src);
+    r.dhi = __shfl_sync(0xffffffffu, a.dhi, src);
     r.k = __shfl_sync(0xffffffffu, a.k, src);
     return r;
 }
 
 __global__ void __launch_bounds__(256)
 fixup_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, const uint32_t *__restrict__ aoff,
-             uint32_t C, const Part *__restrict__ part, uint32_t *__restrict__ cut) {
+             uint32_t C, const Part *__restrict__ part, uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
     const uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (c >= C) return;
     const uint64_t ao = aoff[c], ae = ao + (f_hi[c] - f_lo[c]);
-    const uint64_t j0 = ao / kSplitTile, j1 = (ae - 1) / kSplitTile;
+    const uint64_t j0 = ao / kTile, j1 = (ae - 1) / kTile;
     if (j0 == j1) return;
     Cand best = no_cand();
     for (uint64_t j = j0 + lane; j <= j1; j += 32) {
-        const int slot = (j == j0 && ao != j0 * kSplitTile) ? 1 : 0;
+        const int slot = (j == j0 && ao != j0 * kTile) ? 1 : 0;
         const Cand v = part[2 * j + slot].cand;
         if (better(v, best)) best = v;
     }
@@ -188,18 +333,24 @@ fixup_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_h
         const Cand v = shfl_cand(best, lane ^ o);
         if (better(v, best)) best = v;
     }
-    if (lane == 0) cut[c] = best.k;
+    if (lane == 0) {
+        cut[c] = best.k;
+        cut_SL[c] = best.SL;
+    }
 }
 
 // ---------------------------------------------------------------- a4: decide
 struct DecideArgs {
     const uint32_t *f_lo, *f_hi, *cut;
+    const uint64_t *f_S, *cut_SL;
+    const u128 *f_Q;
     uint32_t C;
-    const uint64_t *P1;
-    const u128 *P2;
+    const uint64_t *PS1;
+    const u128 *PS2;
     const uint32_t *t;
     uint8_t *flags;
     uint64_t *cnt_sz;
+    u128 *cut_QL;
     double eps, z, k2;
     int clamp;
 };
@@ -225,8 +376,13 @@ __global__ void __launch_bounds__(256) decide_kernel(DecideArgs a) {
     const uint32_t lo = a.f_lo[c], hi = a.f_hi[c], k = a.cut[c];
     const uint32_t mid = lo + k;
     const uint64_t n = hi - lo, nL = k, nR = n - k;
-    const uint64_t S = a.P1[hi] - a.P1[lo], SL = a.P1[mid] - a.P1[lo], SR = S - SL;
-    const u128 Q = a.P2[hi] - a.P2[lo], QL = a.P2[mid] - a.P2[lo], QR = Q - QL;
+    const uint64_t S = a.f_S[c], SL = a.cut_SL[c], SR = S - SL;
+    const u128 Q = a.f_Q[c];
+    uint64_t s_lo, s_mid;
+    u128 q_lo, q_mid;
+    pref12(a.PS1, a.PS2, a.t, lo, s_lo, q_lo);
+    pref12(a.PS1, a.PS2, a.t, mid, s_mid, q_mid);
+    const u128 QL = q_mid - q_lo, QR = Q - QL;
     const u128 V = (u128)n * Q - (u128)S * S;
     const u128 VL = (u128)nL * QL - (u128)SL * SL, VR = (u128)nR * QR - (u128)SR * SR;
     // Eq. 7: tau_old = m * Xbar, m from Eq. 3
@@ -247,6 +403,7 @@ __global__ void __launch_bounds__(256) decide_kernel(DecideArgs a) {
         const bool ntL = nontrivial(a.t, lo, mid), ntR = nontrivial(a.t, mid, hi);
         cs = ((uint64_t)(ntL + ntR) << 32) | (uint64_t)((ntL ? nL : 0) + (ntR ? nR : 0));
     }
+    a.cut_QL[c] = QL;
     a.cnt_sz[c] = cs;
 }
 
@@ -273,30 +430,49 @@ int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K) {
     return STEM_OK;
 }
 
+static int ensure_frontier(Ctx &c, int b, uint64_t cap) {
+    CKS(c.ensure(c.f_lo[b], c.cap_flo[b], sizeof(uint32_t) * cap));
+    CKS(c.ensure(c.f_hi[b], c.cap_fhi[b], sizeof(uint32_t) * cap));
+    CKS(c.ensure(c.f_aoff[b], c.cap_faoff[b], sizeof(uint32_t) * cap));
+    CKS(c.ensure(c.f_S[b], c.cap_fS[b], sizeof(uint64_t) * cap));
+    CKS(c.ensure(c.f_Q[b], c.cap_fQ[b], sizeof(u128) * cap));
+    return STEM_OK;
+}
+
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp) {
     cudaStream_t st = c.stream;
     CKS(stem_only_leaves(c, n, K));
-    // initial frontier: non-trivial kernel groups, in kernel order
+    // initial frontier: non-trivial kernel groups, in kernel order, with exact S and Q
     {
-        CKS(c.ensure(c.f_lo[0], c.cap_flo[0], sizeof(uint32_t) * ((uint64_t)K + 1)));
-        CKS(c.ensure(c.f_hi[0], c.cap_fhi[0], sizeof(uint32_t) * ((uint64_t)K + 1)));
-        CKS(c.ensure(c.f_aoff[0], c.cap_faoff[0], sizeof(uint32_t) * ((uint64_t)K + 1)));
+        CKS(ensure_frontier(c, 0, (uint64_t)K + 1));
         CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(K) + 1) * sizeof(uint64_t)));
         const uint32_t *goff = c.goff, *t = c.t_sorted;
+        const uint64_t *PS1 = c.PS1;
+        const u128 *PS2 = c.PS2;
         uint32_t *nlo = c.f_lo[0], *nhi = c.f_hi[0], *nao = c.f_aoff[0];
+        uint64_t *nS = c.f_S[0];
+        u128 *nQ = c.f_Q[0];
+        const int tk = c.stage_begin("root_init");
         exclusive_scan<uint64_t>(
             [goff, t] __device__(uint64_t g) -> uint64_t {
                 const uint32_t lo = goff[g], hi = goff[g + 1];
                 return nontrivial(t, lo, hi) ? ((1ull << 32) | (hi - lo)) : 0ull;
             },
-            [nlo, nhi, nao, goff] __device__(uint64_t g, uint64_t pre, uint64_t v) {
+            [nlo, nhi, nao, nS, nQ, goff, t, PS1, PS2] __device__(uint64_t g, uint64_t pre, uint64_t v) {
                 if (!v) return;
-                const uint32_t idx = (uint32_t)(pre >> 32);
-                nlo[idx] = goff[g];
-                nhi[idx] = goff[g + 1];
+                const uint32_t idx = (uint32_t)(pre >> 32), lo = goff[g], hi = goff[g + 1];
+                uint64_t s0, s1;
+                u128 q0, q1;
+                pref12(PS1, PS2, t, lo, s0, q0);
+                pref12(PS1, PS2, t, hi, s1, q1);
+                nlo[idx] = lo;
+                nhi[idx] = hi;
                 nao[idx] = (uint32_t)pre;
+                nS[idx] = s1 - s0;
+                nQ[idx] = q1 - q0;
             },
             (uint64_t)K, (uint64_t *)c.scan_scratch, &c.scalars->frontier_total, st, &c.launches);
+        c.stage_end(tk, 64 * (uint64_t)K);
         CK(cudaGetLastError());
     }
     uint64_t C = 0, A = 0;
@@ -306,50 +482,63 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
     while (C > 0) {
         levels++;
         c.stats.active_rows += A;
-        const uint64_t ntiles = (A + kSplitTile - 1) / kSplitTile;
+        const uint64_t ntiles = (A + kTile - 1) / kTile;
         CKS(c.ensure(c.cut, c.cap_cut, sizeof(uint32_t) * C));
+        CKS(c.ensure(c.cut_SL, c.cap_cut_SL, sizeof(uint64_t) * C));
+        CKS(c.ensure(c.cut_QL, c.cap_cut_QL, sizeof(u128) * C));
         CKS(c.ensure(c.cnt_sz, c.cap_cntsz, sizeof(uint64_t) * C));
         CKS(c.ensure(c.split_part, c.cap_part, sizeof(Part) * 2 * ntiles));
+        CKS(c.ensure(c.tile_map, c.cap_tile_map, sizeof(uint32_t) * 2 * ntiles));
         CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(C) + 1) * sizeof(uint64_t)));
         const int nxt = cur ^ 1;
-        // children are at most 2 per cluster
-        CKS(c.ensure(c.f_lo[nxt], c.cap_flo[nxt], sizeof(uint32_t) * 2 * C));
-        CKS(c.ensure(c.f_hi[nxt], c.cap_fhi[nxt], sizeof(uint32_t) * 2 * C));
-        CKS(c.ensure(c.f_aoff[nxt], c.cap_faoff[nxt], sizeof(uint32_t) * 2 * C));
+        CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
         const int tk_s = c.stage_begin("root_split");
-        split_kernel<<<(unsigned)ntiles, kSplitThreads, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], (uint32_t)C, A,
-                                                                c.P1, c.cut, (Part *)c.split_part);
+        uint32_t *tfirst = c.tile_map, *tlast = c.tile_map + ntiles;
+        tile_map_kernel<<<(unsigned)((ntiles + 255) / 256), 256, 0, st>>>(c.f_aoff[cur], (uint32_t)C, A, ntiles,
+                                                                          tfirst, tlast);
+        SplitArgs sa{c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], tfirst, tlast, c.f_S[cur], c.PS1, c.t_sorted, A,
+                     c.cut, c.cut_SL, (Part *)c.split_part};
+        CK(cudaFuncSetAttribute(split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SplitSmem)));
+        split_kernel<<<(unsigned)ntiles, kSplitThreads, sizeof(SplitSmem), st>>>(sa);
         fixup_kernel<<<(unsigned)((C * 32 + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur],
-                                                                       (uint32_t)C, (const Part *)c.split_part, c.cut);
-        c.launches += 2;
-        c.stage_end(tk_s, 8 * A + 4 * C * 3);
+                                                                       (uint32_t)C, (const Part *)c.split_part, c.cut,
+                                                                       c.cut_SL);
+        c.launches += 3;
+        c.stage_end(tk_s, 4 * A + 8 * ntiles + 20 * C);
+        CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");
-        DecideArgs da{c.f_lo[cur], c.f_hi[cur], c.cut, (uint32_t)C, c.P1, c.P2, c.t_sorted, c.flags, c.cnt_sz,
-                      eps, z, k2, clamp};
+        DecideArgs da{c.f_lo[cur], c.f_hi[cur], c.cut, c.f_S[cur], c.cut_SL, c.f_Q[cur], (uint32_t)C, c.PS1, c.PS2,
+                      c.t_sorted, c.flags, c.cnt_sz, c.cut_QL, eps, z, k2, clamp};
         decide_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(da);
         c.launches += 1;
         c.stage_end(tk_d, 96 * C);
-        const int tk_c = c.stage_begin("root_compact");
         CK(cudaGetLastError());
+        const int tk_c = c.stage_begin("root_compact");
         const uint32_t *flo = c.f_lo[cur], *fhi = c.f_hi[cur], *fcut = c.cut, *t = c.t_sorted;
-        const uint64_t *cs = c.cnt_sz;
+        const uint64_t *cs = c.cnt_sz, *fS = c.f_S[cur], *cSL = c.cut_SL;
+        const u128 *fQ = c.f_Q[cur], *cQL = c.cut_QL;
         uint32_t *nlo = c.f_lo[nxt], *nhi = c.f_hi[nxt], *nao = c.f_aoff[nxt];
+        uint64_t *nS = c.f_S[nxt];
+        u128 *nQ = c.f_Q[nxt];
         exclusive_scan<uint64_t>(
             [cs] __device__(uint64_t i) -> uint64_t { return cs[i]; },
-            [flo, fhi, fcut, t, nlo, nhi, nao] __device__(uint64_t i, uint64_t pre, uint64_t v) {
+            [flo, fhi, fcut, t, fS, cSL, fQ, cQL, nlo, nhi, nao, nS, nQ] __device__(uint64_t i, uint64_t pre,
+                                                                                   uint64_t v) {
                 if (!v) return;
                 uint32_t idx = (uint32_t)(pre >> 32), off = (uint32_t)pre;
                 const uint32_t lo = flo[i], hi = fhi[i], mid = lo + fcut[i];
                 if (nontrivial(t, lo, mid)) {
                     nlo[idx] = lo; nhi[idx] = mid; nao[idx] = off;
+                    nS[idx] = cSL[i]; nQ[idx] = cQL[i];
                     idx++; off += mid - lo;
                 }
                 if (nontrivial(t, mid, hi)) {
                     nlo[idx] = mid; nhi[idx] = hi; nao[idx] = off;
+                    nS[idx] = fS[i] - cSL[i]; nQ[idx] = fQ[i] - cQL[i];
                 }
             },
             C, (uint64_t *)c.scan_scratch, &c.scalars->frontier_total, st, &c.launches);
-        c.stage_end(tk_c, 8 * C + 24 * C);
+        c.stage_end(tk_c, 48 * C);
         CK(cudaGetLastError());
         CKS(read_frontier_total(c, C, A));
         cur = nxt;

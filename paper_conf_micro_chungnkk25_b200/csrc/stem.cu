@@ -56,8 +56,8 @@ __device__ double fix_round(const uint64_t *lane) {
 // ---------------------------------------------------------------- leaf table
 struct LeafArgs {
     const uint32_t *leaf_lo, *goff, *t;
-    const uint64_t *P1;
-    const u128 *P2;
+    const uint64_t *PS1;
+    const u128 *PS2;
     uint64_t L, n;
     uint32_t K;
     int scope;
@@ -73,16 +73,25 @@ struct LeafView {
     u128 V;
 };
 
-__device__ __forceinline__ LeafView leaf_view(const uint32_t *leaf_lo, uint64_t L, uint64_t N, const uint64_t *P1,
-                                              const u128 *P2, uint64_t i) {
+__device__ __forceinline__ LeafView leaf_view(const uint32_t *leaf_lo, uint64_t L, uint64_t N, const uint64_t *PS1,
+                                              const u128 *PS2, const uint32_t *t, uint64_t i) {
     LeafView v;
     v.lo = leaf_lo[i];
     v.hi = (i + 1 < L) ? leaf_lo[i + 1] : (uint32_t)N;
     v.n = v.hi - v.lo;
-    v.S = P1[v.hi] - P1[v.lo];
-    const u128 Q = P2[v.hi] - P2[v.lo];
+    uint64_t s0, s1;
+    u128 q0, q1;
+    pref12(PS1, PS2, t, v.lo, s0, q0);
+    pref12(PS1, PS2, t, v.hi, s1, q1);
+    v.S = s1 - s0;
+    const u128 Q = q1 - q0;
     v.V = (u128)v.n * Q - (u128)v.S * v.S;
     return v;
+}
+
+// T = sum of all t (exact), from the sampled prefix
+__global__ void total_kernel(const uint64_t *PS1, const uint32_t *t, uint64_t n, uint64_t *T) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) *T = pref1(PS1, t, n);
 }
 
 __global__ void __launch_bounds__(kThreads) leaf_kkt_kernel(LeafArgs a) {
@@ -92,7 +101,7 @@ __global__ void __launch_bounds__(kThreads) leaf_kkt_kernel(LeafArgs a) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     bool bad = false;
     if (i < a.L) {
-        const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.P1, a.P2, i);
+        const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.PS1, a.PS2, a.t, i);
         const uint32_t g = (uint32_t)upper_bound(a.goff, (uint64_t)a.K + 1, v.lo) - 1;
         const uint64_t first = lower_bound(a.leaf_lo, a.L, a.goff[g]);
         a.leaf_kid[i] = g;
@@ -134,9 +143,9 @@ __global__ void kkt_finalize_kernel(const uint64_t *fix_acc, const uint64_t *ker
 }
 
 struct MArgs {
-    const uint32_t *leaf_lo, *leaf_kid;
-    const uint64_t *P1;
-    const u128 *P2;
+    const uint32_t *leaf_lo, *leaf_kid, *t;
+    const uint64_t *PS1;
+    const u128 *PS2;
     uint64_t L, n;
     int scope, census_cap;
     double k2;
@@ -149,7 +158,7 @@ struct MArgs {
 __global__ void __launch_bounds__(kThreads) leaf_m_kernel(MArgs a) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= a.L) return;
-    const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.P1, a.P2, i);
+    const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.PS1, a.PS2, a.t, i);
     double m;
     if (v.V == 0) {
         m = 1.0;
@@ -219,9 +228,9 @@ __device__ __forceinline__ double block_sum(double v, double *sm) {
 }
 
 struct EstArgs {
-    const uint32_t *leaf_lo;
-    const uint64_t *P1;
-    const u128 *P2;
+    const uint32_t *leaf_lo, *t;
+    const uint64_t *PS1;
+    const u128 *PS2;
     const uint64_t *m, *U;
     uint64_t L, n;
     uint64_t *sum_q;
@@ -233,7 +242,7 @@ __global__ void __launch_bounds__(kThreads) estimate_kernel(EstArgs a) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     double frac = 0.0, var = 0.0;
     if (i < a.L) {
-        const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.P1, a.P2, i);
+        const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.PS1, a.PS2, a.t, i);
         const uint64_t m = a.m[i];
         const u128 num = (u128)v.n * a.U[i];
         const uint64_t q = (uint64_t)(num / m), r = (uint64_t)(num % m);
@@ -288,11 +297,11 @@ __global__ void est_finalize_kernel(const uint64_t *sum_q, const double *red, co
 }
 
 __global__ void pack_kernel(const uint32_t *leaf_lo, const uint32_t *leaf_kid, const uint32_t *leaf_ord,
-                            const uint64_t *P1, const u128 *P2, const uint32_t *t, const uint64_t *m,
+                            const uint64_t *PS1, const u128 *PS2, const uint32_t *t, const uint64_t *m,
                             const uint8_t *census, uint64_t L, uint64_t n, stem_cluster *out) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= L) return;
-    const LeafView v = leaf_view(leaf_lo, L, n, P1, P2, i);
+    const LeafView v = leaf_view(leaf_lo, L, n, PS1, PS2, t, i);
     stem_cluster c;
     c.kernel_id = leaf_kid[i];
     c.ordinal = leaf_ord[i];
@@ -351,18 +360,20 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CK(cudaMemsetAsync(c.leaf_U, 0, sizeof(uint64_t) * (L + 1), st));
 
     const int tk_kkt = c.stage_begin("stem_sizes");
-    LeafArgs la{c.leaf_lo, c.goff, c.t_sorted, c.P1, c.P2, L, n, K, o.scope, leaf_kid, leaf_ord,
+    total_kernel<<<1, 32, 0, st>>>(c.PS1, c.t_sorted, n, &c.scalars->T);
+    c.launches++;
+    LeafArgs la{c.leaf_lo, c.goff, c.t_sorted, c.PS1, c.PS2, L, n, K, o.scope, leaf_kid, leaf_ord,
                 c.fix_acc, c.kern_T, &c.scalars->err};
     leaf_kkt_kernel<<<blocks_for(L), kThreads, 0, st>>>(la);
     c.launches++;
-    // T = P1[n] (exact total, a2)
+    // g per set (T = total_kernel above, exact)
     if (o.scope == 0)
-        kkt_finalize_kernel<<<1, 32, 0, st>>>(c.fix_acc, nullptr, c.P1 + n, 1, eps, z, c.kern_g, &c.scalars->ssum);
+        kkt_finalize_kernel<<<1, 32, 0, st>>>(c.fix_acc, nullptr, &c.scalars->T, 1, eps, z, c.kern_g, &c.scalars->ssum);
     else if (o.scope == 1)
         kkt_finalize_kernel<<<blocks_for(K), kThreads, 0, st>>>(c.fix_acc, c.kern_T, nullptr, K, eps, z, c.kern_g,
                                                                nullptr);
     if (o.scope != 2) c.launches++;
-    MArgs ma{c.leaf_lo, leaf_kid, c.P1, c.P2, L, n, o.scope, o.census_cap, k2, c.kern_g, c.leaf_m,
+    MArgs ma{c.leaf_lo, leaf_kid, c.t_sorted, c.PS1, c.PS2, L, n, o.scope, o.census_cap, k2, c.kern_g, c.leaf_m,
              c.leaf_census, &c.scalars->limit_err};
     leaf_m_kernel<<<blocks_for(L), kThreads, 0, st>>>(ma);
     c.launches++;
@@ -382,8 +393,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     if (hs.err & 2) return STEM_E_CUDA;
     if (hs.limit_err || hs.total_m >= (1ull << 32)) return STEM_E_LIMIT;
     const uint64_t S = hs.total_m;
-    uint64_t T = 0;
-    CK(cudaMemcpy(&T, c.P1 + n, sizeof(uint64_t), cudaMemcpyDeviceToHost));
+    const uint64_t T = hs.T;
     c.n_samples = S;
     c.T = T;
     c.stats.ssum = o.scope == 0 ? hs.ssum : 0.0;
@@ -409,7 +419,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     double *part_est = c.red_part, *part_met = c.red_part + 2 * eb, *red_out = part_met + mb * (nm ? nm : 1);
     CK(cudaMemsetAsync(&c.scalars->sum_q, 0, sizeof(uint64_t), st));
     const int tk_est = c.stage_begin("estimate");
-    EstArgs ea{c.leaf_lo, c.P1, c.P2, c.leaf_m, c.leaf_U, L, n, &c.scalars->sum_q, part_est};
+    EstArgs ea{c.leaf_lo, c.t_sorted, c.PS1, c.PS2, c.leaf_m, c.leaf_U, L, n, &c.scalars->sum_q, part_est};
     estimate_kernel<<<(unsigned)eb, kThreads, 0, st>>>(ea);
     reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_est, eb, 2, red_out);
     c.launches += 2;
@@ -423,13 +433,13 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     // a5 output records
     CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
     const int tk_pack = c.stage_begin("pack");
-    pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.P1, c.P2, c.t_sorted, c.leaf_m,
+    pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.PS1, c.PS2, c.t_sorted, c.leaf_m,
                                                    c.leaf_census, L, n, c.out_clusters);
     c.launches++;
     c.stage_end(tk_pack, 88 * L);
     CK(cudaGetLastError());
     double *est_out = red_out + 2 + nm;
-    est_finalize_kernel<<<1, 1, 0, st>>>(&c.scalars->sum_q, red_out, c.P1 + n, z, est_out);
+    est_finalize_kernel<<<1, 1, 0, st>>>(&c.scalars->sum_q, red_out, &c.scalars->T, z, est_out);
     c.launches++;
     CK(cudaGetLastError());
     double red[2 + 64 + 2];
