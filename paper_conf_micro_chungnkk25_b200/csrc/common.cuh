@@ -77,11 +77,11 @@ __device__ __forceinline__ int cmp256(const U256 &a, const U256 &b) {
 }
 
 // ---------------------------------------------------------------- split candidates
-// Candidate cut k of a cluster: score = D^2 / p, D = n*S_L - S*k (< 0 for a
-// valid cut of sorted data, |D| < 2^96), p = k (n - k).  f is the fp64
-// filter value; SL = S_L(k) travels with the candidate to the decision.
+// Candidate cut k of a cluster: score = D^2 / p, D = n*S_L - S*k (<= 0 for
+// sorted data, |D| < 2^96), p = k (n - k).  x = fp64 |D|^2 is the filter
+// value (relative error < 2^-50); SL = S_L(k) travels to the decision.
 struct Cand {
-    double f;
+    double x;       // ~ |D|^2
     uint64_t dlo;   // |D| bits 0..63
     uint64_t p;
     uint64_t SL;
@@ -91,7 +91,7 @@ struct Cand {
 
 __device__ __forceinline__ Cand no_cand() {
     Cand c;
-    c.f = 0.0;
+    c.x = 0.0;
     c.dlo = 0;
     c.p = 0;
     c.SL = 0;
@@ -102,32 +102,29 @@ __device__ __forceinline__ Cand no_cand() {
 
 __device__ __forceinline__ u128 cand_absD(const Cand &c) { return ((u128)c.dhi << 64) | c.dlo; }
 
+// fp64 approximation of |D| = hi:lo (hi < 2^32), relative error <= 2^-52
+__device__ __forceinline__ double approx_d(uint32_t hi, uint64_t lo) {
+    return __fma_rn(__uint2double_rn(hi), 0x1p64, __ull2double_rn(lo));
+}
+
+// Exact comparison D_a^2 p_b vs D_b^2 p_a (both < 2^256): -1, 0, +1
+__device__ __forceinline__ int exact_cmp(const Cand &a, const Cand &b) {
+    return cmp256(sq_times(cand_absD(a), b.p), sq_times(cand_absD(b), a.p));
+}
+
 // Exact strict total order (R5): larger score first, ties -> smaller k.
-// The fp64 filter decides only when the scores differ by > 2^-40 relative;
-// its own error is < 2^-50, so the order equals the exact one.
+// x_a * p_b vs x_b * p_a in fp64 (each side within 2^-49 relative) decides
+// only when they differ by more than 2^-40; otherwise the 256-bit products do.
 __device__ __forceinline__ bool better(const Cand &a, const Cand &b) {
     if (a.k == 0) return false;
     if (b.k == 0) return true;
+    const double L = __dmul_rn(a.x, __ull2double_rn(b.p)), R = __dmul_rn(b.x, __ull2double_rn(a.p));
     const double tol = 1.0 + 0x1p-40;
-    if (a.f > __dmul_rn(b.f, tol)) return true;
-    if (b.f > __dmul_rn(a.f, tol)) return false;
-    const int c = cmp256(sq_times(cand_absD(a), b.p), sq_times(cand_absD(b), a.p));
+    if (L > __dmul_rn(R, tol)) return true;
+    if (R > __dmul_rn(L, tol)) return false;
+    const int c = exact_cmp(a, b);
     if (c != 0) return c > 0;
     return a.k < b.k;
-}
-
-__device__ __forceinline__ Cand make_cand(uint64_t n, uint64_t S, uint64_t SL, uint32_t k) {
-    Cand c;
-    const u128 a = (u128)n * SL, b = (u128)S * k;
-    const u128 d = a > b ? a - b : b - a;
-    c.dlo = (uint64_t)d;
-    c.dhi = (uint32_t)(d >> 64);
-    c.p = (uint64_t)k * (n - k);
-    c.SL = SL;
-    const double dD = rn128(d);
-    c.f = __ddiv_rn(__dmul_rn(dD, dD), rn64(c.p));
-    c.k = k;
-    return c;
 }
 
 // ---------------------------------------------------------------- sampled prefix moments

@@ -106,26 +106,41 @@ struct SplitArgs {
 __host__ __device__ constexpr int padx(int i) { return i + (i >> 3); }   // conflict-free blocked u32 reads
 
 struct SplitSmem {
-    Cand v[2 * kSplitThreads];                 // block segmented argmax entries
     uint64_t S[kMaxTileClusters], base[kMaxTileClusters];
     uint64_t red[kSplitThreads / 32 + 1];
     uint64_t carry;
+    Cand wtot[kSplitThreads / 32];             // per-warp inclusive (flag, best) of the run scan
+    uint32_t wflag[kSplitThreads / 32];
     uint32_t t[padx(kTile + 1) + 1];           // t[padx(p + 1)] = t at tile position p; t[0] = halo
     uint32_t ao[kMaxTileClusters], lo[kMaxTileClusters], n[kMaxTileClusters];
     uint32_t wmax[kSplitThreads / 32];
-    uint32_t cc[2 * kSplitThreads];
     uint16_t cid[kTile];                       // tile-relative cluster of every position
 };
 
-__global__ void __launch_bounds__(kSplitThreads) split_kernel(SplitArgs a) {
+__device__ __forceinline__ Cand shfl_cand_up(const Cand &a, int d) {
+    Cand r;
+    r.x = __shfl_up_sync(0xffffffffu, a.x, d);
+    r.dlo = __shfl_up_sync(0xffffffffu, a.dlo, d);
+    r.p = __shfl_up_sync(0xffffffffu, a.p, d);
+    r.SL = __shfl_up_sync(0xffffffffu, a.SL, d);
+    r.dhi = __shfl_up_sync(0xffffffffu, a.dhi, d);
+    r.k = __shfl_up_sync(0xffffffffu, a.k, d);
+    return r;
+}
+
+// run-scan operator over threads: (f1,v1) + (f2,v2) = (f1|f2, f2 ? v2 : best(v1,v2))
+__device__ __forceinline__ void run_combine(uint32_t fp, const Cand &vp, uint32_t &f, Cand &v) {
+    if (!f && better(vp, v)) v = vp;
+    f |= fp;
+}
+
+__global__ void __launch_bounds__(kSplitThreads, 3) split_kernel(SplitArgs a) {
     extern __shared__ __align__(16) unsigned char s_dyn[];
     SplitSmem &sm = *reinterpret_cast<SplitSmem *>(s_dyn);
     uint32_t *s_t = sm.t;
     uint16_t *s_cid = sm.cid;
-    uint32_t *s_ao = sm.ao, *s_lo = sm.lo, *s_n = sm.n, *s_wmax = sm.wmax, *s_cc = sm.cc;
-    uint64_t *s_S = sm.S, *s_base = sm.base, *s_red = sm.red;
-    Cand *s_v = sm.v;
-    uint64_t &s_carry = sm.carry;
+    uint32_t *s_ao = sm.ao, *s_lo = sm.lo, *s_n = sm.n;
+    uint64_t *s_S = sm.S, *s_base = sm.base;
 
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const uint64_t ts = (uint64_t)blockIdx.x * kTile;
@@ -150,15 +165,14 @@ __global__ void __launch_bounds__(kSplitThreads) split_kernel(SplitArgs a) {
         uint64_t carry = 0;
         if (s_ao[0] < ts) {
             const uint64_t lo = s_lo[0], r = lo + (ts - s_ao[0]);
-            // pref1(r) - pref1(lo); the partial chunk sums are spread over the warp
-            uint64_t part = 0;
+            uint64_t part = 0;   // pref1(r) - pref1(lo); the partial chunk sums spread over the warp
             const uint64_t rb = r & ~(kChunk - 1), lb = lo & ~(kChunk - 1);
             if (rb + lane < r) part += a.t[rb + lane];
             if (lb + lane < lo) part -= a.t[lb + lane];
             for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
             carry = a.PS1[r >> kChunkLog] - a.PS1[lo >> kChunkLog] + part;
         }
-        if (lane == 0) s_carry = carry;
+        if (lane == 0) sm.carry = carry;
     }
     __syncthreads();
     // running max over positions (heads carry increasing ids): blocked, 8 per thread
@@ -172,11 +186,11 @@ __global__ void __launch_bounds__(kSplitThreads) split_kernel(SplitArgs a) {
             const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
             if (lane >= o) incl = max(incl, v);
         }
-        if (lane == 31) s_wmax[w] = incl;
+        if (lane == 31) sm.wmax[w] = incl;
         uint32_t pre = __shfl_up_sync(0xffffffffu, incl, 1);
         if (lane == 0) pre = 0;
         __syncthreads();
-        for (int ww = 0; ww < w; ww++) pre = max(pre, s_wmax[ww]);
+        for (int ww = 0; ww < w; ww++) pre = max(pre, sm.wmax[ww]);
         uint32_t r = pre;
 #pragma unroll
         for (int j = 0; j < kSplitItems; j++) {
@@ -197,114 +211,157 @@ __global__ void __launch_bounds__(kSplitThreads) split_kernel(SplitArgs a) {
         s_t[padx(idx)] = v;
     }
     __syncthreads();
-    // block exclusive scan of t over positions -> S_L of every candidate
+    // block exclusive scan of t over positions -> S_L at every thread's first position
     const int p0 = tid * kSplitItems;
+    const int pend = min(p0 + kSplitItems, nt);
     uint64_t mysum = 0;
 #pragma unroll
     for (int j = 0; j < kSplitItems; j++)
         if (p0 + j < nt) mysum += s_t[padx(p0 + j + 1)];
     uint64_t tot;
-    const uint64_t excl = block_excl_scan<uint64_t, kSplitThreads>(mysum, s_red, &tot);
+    const uint64_t excl = block_excl_scan<uint64_t, kSplitThreads>(mysum, sm.red, &tot);
     {
         uint64_t run = excl;
-        for (int j = 0; j < kSplitItems && p0 + j < nt; j++) {
-            const int p = p0 + j, ci = s_cid[p];
+        for (int p = p0; p < pend; p++) {
+            const int ci = s_cid[p];
             if (s_ao[ci] == ts + p) s_base[ci] = run;          // cluster starts inside the tile
             run += s_t[padx(p + 1)];
         }
-        if (tid == 0 && s_ao[0] < ts) s_base[0] = (uint64_t)0 - s_carry;   // S_L = run + carry (mod 2^64)
+        if (tid == 0 && s_ao[0] < ts) s_base[0] = (uint64_t)0 - sm.carry;   // S_L = run + carry (mod 2^64)
     }
     __syncthreads();
 
-    // candidates, thread-local segmented argmax
-    uint32_t head_c = kNone, tail_c = kNone;
-    Cand head_b = no_cand(), tail_b = no_cand();
+    // ---- candidates: thread-local segmented argmax with exact incremental D
+    int head_ci = -1;                   // first segment when incomplete
+    Cand head_b = no_cand();
+    bool head_before = false;           // its cluster started before this thread
+    uint32_t out_f = 1;                 // run-scan element: 1 = the carried run starts here / no carry
+    Cand out_v = no_cand();
+    int out_ci = -1;                    // cluster carried out of this thread (extends beyond it)
     if (p0 < nt) {
-        const int pend = min(p0 + kSplitItems, nt);
         int ci = s_cid[p0];
-        uint64_t ao = s_ao[ci], ae = ao + s_n[ci];
+        uint64_t n = s_n[ci], S = s_S[ci], ao = s_ao[ci];
+        uint32_t k = (uint32_t)(ts + p0 - ao);
+        uint64_t SL = excl - s_base[ci];
+        i128 D = (i128)((u128)n * SL) - (i128)((u128)S * k);
         int seg_start = p0;
         Cand best = no_cand();
-        uint64_t run = excl;
-        auto flush = [&]() {
-            if (ao >= ts + p0 && ae <= ts + pend) {
+        double best_dp = 0.0;
+        auto flush = [&](int seg_end) {
+            const bool before = ao < ts + p0, after = ao + n > ts + pend;
+            if (!before && !after) {
                 a.cut[c0 + ci] = best.k;                      // whole cluster inside this thread
                 a.cut_SL[c0 + ci] = best.SL;
-            } else if (seg_start == p0) {
-                head_c = ci; head_b = best;
-            } else {
-                tail_c = ci; tail_b = best;
+                return;
             }
+            if (seg_start == p0) { head_ci = ci; head_b = best; head_before = before; }
+            if (seg_end == pend && after) { out_ci = ci; out_v = best; out_f = before ? 0u : 1u; }
         };
         uint32_t tprev = s_t[padx(p0)];
         for (int p = p0; p < pend; p++) {
             const int cj = s_cid[p];
             if (cj != ci) {
-                flush();
+                flush(p);
                 ci = cj;
+                n = s_n[ci];
+                S = s_S[ci];
                 ao = s_ao[ci];
-                ae = ao + s_n[ci];
+                k = 0;
+                SL = 0;
+                D = 0;
                 seg_start = p;
                 best = no_cand();
             }
             const uint32_t tc = s_t[padx(p + 1)];
-            const uint32_t k = (uint32_t)(ts + p - ao);
             if (k >= 1 && tprev < tc) {                       // cut between distinct values only
-                const Cand cd = make_cand(s_n[ci], s_S[ci], run - s_base[ci], k);
-                if (better(cd, best)) best = cd;
+                const u128 ad = (u128)(-D);
+                const uint32_t dhi = (uint32_t)(ad >> 64);
+                const uint64_t dlo = (uint64_t)ad;
+                const double dD = approx_d(dhi, dlo);
+                const double x = __dmul_rn(dD, dD);
+                const double dp = __dmul_rn(__uint2double_rn(k), __uint2double_rn((uint32_t)(n - k)));
+                bool take = best.k == 0;
+                if (!take) {
+                    const double L = __dmul_rn(x, best_dp), R = __dmul_rn(best.x, dp);
+                    const double tol = 1.0 + 0x1p-40;
+                    if (L > __dmul_rn(R, tol)) {
+                        take = true;
+                    } else if (!(R > __dmul_rn(L, tol))) {    // near tie: exact 256-bit products
+                        Cand cd;
+                        cd.dlo = dlo; cd.dhi = dhi; cd.p = (uint64_t)k * (n - k);
+                        take = exact_cmp(cd, best) > 0;       // equal -> keep the smaller k
+                    }
+                }
+                if (take) {
+                    best.x = x; best.dlo = dlo; best.dhi = dhi; best.p = (uint64_t)k * (n - k);
+                    best.SL = SL; best.k = k;
+                    best_dp = dp;
+                }
             }
-            run += tc;
+            D += (i128)(uint64_t)(n * tc) - (i128)S;         // D_{k+1} = D_k + n t_k - S
+            SL += tc;
+            k++;
             tprev = tc;
         }
-        flush();
-        if (head_c != kNone && tail_c == kNone) { tail_c = head_c; tail_b = head_b; }   // idempotent duplicate
+        flush(pend);
     }
-    // block-level segmented argmax (Hillis-Steele; a cluster's entries are contiguous)
-    s_cc[2 * tid] = head_c;
-    s_v[2 * tid] = head_b;
-    s_cc[2 * tid + 1] = tail_c;
-    s_v[2 * tid + 1] = tail_b;
+    // ---- block run-scan over threads: element (out_f, out_v)
+    uint32_t f = out_f;
+    Cand v = out_v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const Cand ov = shfl_cand_up(v, o);
+        const uint32_t of = __shfl_up_sync(0xffffffffu, f, o);
+        if (lane >= o) run_combine(of, ov, f, v);
+    }
+    if (lane == 31) { sm.wtot[w] = v; sm.wflag[w] = f; }
+    const Cand wprev = shfl_cand_up(v, 1);
+    const uint32_t fprev = __shfl_up_sync(0xffffffffu, f, 1);
     __syncthreads();
-    for (int d = 1; d < 2 * kSplitThreads; d <<= 1) {
-        Cand nv[2];
-        bool upd[2];
-#pragma unroll
-        for (int h = 0; h < 2; h++) {
-            const int e = 2 * tid + h;
-            const uint32_t ce = s_cc[e];
-            upd[h] = false;
-            if (ce != kNone && e >= d && s_cc[e - d] == ce) {
-                const Cand o = s_v[e - d];
-                nv[h] = s_v[e];
-                if (better(o, nv[h])) { nv[h] = o; upd[h] = true; }
-            }
-        }
-        __syncthreads();
-#pragma unroll
-        for (int h = 0; h < 2; h++)
-            if (upd[h]) s_v[2 * tid + h] = nv[h];
-        __syncthreads();
+    uint32_t cf = 0;                    // combination of the previous warps' totals
+    Cand cv = no_cand();
+    for (int ww = 0; ww < w; ww++) {
+        uint32_t ff = sm.wflag[ww];
+        Cand vv = sm.wtot[ww];
+        run_combine(cf, cv, ff, vv);
+        cf = ff;
+        cv = vv;
     }
-#pragma unroll
-    for (int h = 0; h < 2; h++) {
-        const int e = 2 * tid + h;
-        const uint32_t ce = s_cc[e];
-        if (ce == kNone) continue;
-        if (e + 1 < 2 * kSplitThreads && s_cc[e + 1] == ce) continue;   // not the run's last entry
-        const uint64_t ao = s_ao[ce], ae = ao + s_n[ce];
-        if (ao >= ts && ae <= te) {
-            a.cut[c0 + ce] = s_v[e].k;
-            a.cut_SL[c0 + ce] = s_v[e].SL;
+    uint32_t ef = cf;                   // exclusive element at this thread
+    Cand ev = cv;
+    if (lane > 0) {
+        uint32_t ff = fprev;
+        Cand vv = wprev;
+        run_combine(cf, cv, ff, vv);
+        ef = ff;
+        ev = vv;
+    }
+    uint32_t inf = f;                   // inclusive element at this thread
+    Cand iv = v;
+    run_combine(cf, cv, inf, iv);
+    (void)ef;
+    // a head that started before this thread and ends inside it closes its run
+    if (head_ci >= 0 && head_before && out_ci != head_ci) {
+        Cand fin = head_b;
+        if (better(ev, fin)) fin = ev;
+        const uint64_t ao = s_ao[head_ci];
+        if (ao >= ts) {
+            a.cut[c0 + head_ci] = fin.k;
+            a.cut_SL[c0 + head_ci] = fin.SL;
         } else {
-            const int slot = (ao <= ts) ? 0 : 1;   // first cluster of the tile -> slot 0
-            a.part[2 * (uint64_t)blockIdx.x + slot] = Part{s_v[e], c0 + ce};
+            a.part[2 * (uint64_t)blockIdx.x] = Part{fin, c0 + head_ci};
         }
+    }
+    // the run carried out of the tile's last thread continues into the next tile
+    if (p0 < nt && pend == nt && out_ci >= 0) {
+        const uint64_t ao = s_ao[out_ci];
+        a.part[2 * (uint64_t)blockIdx.x + (ao <= ts ? 0 : 1)] = Part{iv, c0 + out_ci};
     }
 }
 
 __device__ __forceinline__ Cand shfl_cand(const Cand &a, int src) {
     Cand r;
-    r.f = __shfl_sync(0xffffffffu, a.f, src);
+    r.x = __shfl_sync(0xffffffffu, a.x, src);
     r.dlo = __shfl_sync(0xffffffffu, a.dlo, src);
     r.p = __shfl_sync(0xffffffffu, a.p, src);
     r.SL = __shfl_sync(0xffffffffu, a.SL, src);
