@@ -82,6 +82,7 @@ __device__ __forceinline__ int cmp256(const U256 &a, const U256 &b) {
 // value (relative error < 2^-50); SL = S_L(k) travels to the decision.
 struct Cand {
     double x;       // ~ |D|^2
+    double dp;      // ~ p
     uint64_t dlo;   // |D| bits 0..63
     uint64_t p;
     uint64_t SL;
@@ -92,6 +93,7 @@ struct Cand {
 __device__ __forceinline__ Cand no_cand() {
     Cand c;
     c.x = 0.0;
+    c.dp = 0.0;
     c.dlo = 0;
     c.p = 0;
     c.SL = 0;
@@ -113,12 +115,12 @@ __device__ __forceinline__ int exact_cmp(const Cand &a, const Cand &b) {
 }
 
 // Exact strict total order (R5): larger score first, ties -> smaller k.
-// x_a * p_b vs x_b * p_a in fp64 (each side within 2^-49 relative) decides
+// x_a * dp_b vs x_b * dp_a in fp64 (each side within 2^-49 relative) decides
 // only when they differ by more than 2^-40; otherwise the 256-bit products do.
 __device__ __forceinline__ bool better(const Cand &a, const Cand &b) {
     if (a.k == 0) return false;
     if (b.k == 0) return true;
-    const double L = __dmul_rn(a.x, __ull2double_rn(b.p)), R = __dmul_rn(b.x, __ull2double_rn(a.p));
+    const double L = __dmul_rn(a.x, b.dp), R = __dmul_rn(b.x, a.dp);
     const double tol = 1.0 + 0x1p-40;
     if (L > __dmul_rn(R, tol)) return true;
     if (R > __dmul_rn(L, tol)) return false;

@@ -19,8 +19,8 @@
 namespace sr {
 
 constexpr int kSplitThreads = 256;
-constexpr int kSplitItems = 8;
-constexpr int kTile = kSplitThreads * kSplitItems;      // 2048 active rows
+constexpr int kSplitItems = 16;
+constexpr int kTile = kSplitThreads * kSplitItems;      // 4096 active rows
 constexpr int kMaxTileClusters = kTile / 2 + 2;         // frontier clusters have >= 2 rows
 constexpr uint32_t kNone = 0xFFFFFFFFu;
 
@@ -83,17 +83,69 @@ __device__ __forceinline__ bool nontrivial(const uint32_t *t, uint32_t lo, uint3
     return hi - lo >= 2 && t[lo] != t[hi - 1];
 }
 
+// first/last frontier cluster of every tile; tiles inside one cluster go to
+// the fast list, the others to the general list (order is irrelevant).
 __global__ void tile_map_kernel(const uint32_t *__restrict__ aoff, uint32_t C, uint64_t A, uint64_t ntiles,
-                                uint32_t *__restrict__ first, uint32_t *__restrict__ last) {
+                                uint32_t *__restrict__ first, uint32_t *__restrict__ last,
+                                uint32_t *__restrict__ fast_list, uint32_t *__restrict__ gen_list,
+                                uint32_t *__restrict__ counts) {
     const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (j >= ntiles) return;
     const uint64_t ts = j * kTile, te = min(ts + kTile, A);
-    first[j] = (uint32_t)upper_bound(aoff, C, (uint32_t)ts) - 1;
-    last[j] = (uint32_t)upper_bound(aoff, C, (uint32_t)(te - 1)) - 1;
+    const uint32_t f = (uint32_t)upper_bound(aoff, C, (uint32_t)ts) - 1;
+    const uint32_t l = (uint32_t)upper_bound(aoff, C, (uint32_t)(te - 1)) - 1;
+    first[j] = f;
+    last[j] = l;
+    if (f == l) fast_list[atomicAdd(&counts[0], 1u)] = (uint32_t)j;
+    else gen_list[atomicAdd(&counts[1], 1u)] = (uint32_t)j;
+}
+
+// Evaluate the valid cut k (t[k-1] < t[k]) with its exact D = n S_L - S k <= 0.
+__device__ __forceinline__ void eval_cut(i128 D, uint32_t k, uint64_t n, uint64_t SL, Cand &best) {
+    const u128 ad = (u128)(-D);
+    const uint32_t dhi = (uint32_t)(ad >> 64);
+    const uint64_t dlo = (uint64_t)ad;
+    const double dD = approx_d(dhi, dlo);
+    const double x = __dmul_rn(dD, dD);
+    const double dp = __dmul_rn(__uint2double_rn(k), __uint2double_rn((uint32_t)(n - k)));
+    bool take = best.k == 0;
+    if (!take) {
+        const double L = __dmul_rn(x, best.dp), R = __dmul_rn(best.x, dp);
+        const double tol = 1.0 + 0x1p-40;
+        if (L > __dmul_rn(R, tol)) {
+            take = true;
+        } else if (!(R > __dmul_rn(L, tol))) {            // near tie: exact 256-bit products
+            Cand cd;
+            cd.dlo = dlo;
+            cd.dhi = dhi;
+            cd.p = (uint64_t)k * (n - k);
+            take = exact_cmp(cd, best) > 0;               // equal -> keep the smaller k
+        }
+    }
+    if (take) {
+        best.x = x;
+        best.dp = dp;
+        best.dlo = dlo;
+        best.dhi = dhi;
+        best.p = (uint64_t)k * (n - k);
+        best.SL = SL;
+        best.k = k;
+    }
+}
+
+// sum of t over [lo, r): pref1(r) - pref1(lo) with the partial chunks spread over a warp
+__device__ __forceinline__ uint64_t warp_range_sum(const uint64_t *PS1, const uint32_t *t, uint64_t lo, uint64_t r) {
+    const int lane = threadIdx.x & 31;
+    uint64_t part = 0;
+    const uint64_t rb = r & ~(kChunk - 1), lb = lo & ~(kChunk - 1);
+    if (rb + lane < r) part += t[rb + lane];
+    if (lb + lane < lo) part -= t[lb + lane];
+    for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+    return PS1[r >> kChunkLog] - PS1[lo >> kChunkLog] + part;
 }
 
 struct SplitArgs {
-    const uint32_t *f_lo, *f_hi, *aoff, *tile_first, *tile_last;
+    const uint32_t *f_lo, *f_hi, *aoff, *tile_first, *tile_last, *list;
     const uint64_t *f_S;
     const uint64_t *PS1;
     const uint32_t *t;
@@ -120,6 +172,7 @@ struct SplitSmem {
 __device__ __forceinline__ Cand shfl_cand_up(const Cand &a, int d) {
     Cand r;
     r.x = __shfl_up_sync(0xffffffffu, a.x, d);
+    r.dp = __shfl_up_sync(0xffffffffu, a.dp, d);
     r.dlo = __shfl_up_sync(0xffffffffu, a.dlo, d);
     r.p = __shfl_up_sync(0xffffffffu, a.p, d);
     r.SL = __shfl_up_sync(0xffffffffu, a.SL, d);
@@ -134,7 +187,7 @@ __device__ __forceinline__ void run_combine(uint32_t fp, const Cand &vp, uint32_
     f |= fp;
 }
 
-__global__ void __launch_bounds__(kSplitThreads, 3) split_kernel(SplitArgs a) {
+__global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
     extern __shared__ __align__(16) unsigned char s_dyn[];
     SplitSmem &sm = *reinterpret_cast<SplitSmem *>(s_dyn);
     uint32_t *s_t = sm.t;
@@ -143,11 +196,12 @@ __global__ void __launch_bounds__(kSplitThreads, 3) split_kernel(SplitArgs a) {
     uint64_t *s_S = sm.S, *s_base = sm.base;
 
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const uint64_t ts = (uint64_t)blockIdx.x * kTile;
+    const uint32_t tile = a.list[blockIdx.x];
+    const uint64_t ts = (uint64_t)tile * kTile;
     const uint64_t te = min(ts + kTile, a.A);
     const int nt = (int)(te - ts);
-    const uint32_t c0 = a.tile_first[blockIdx.x];
-    const int nc = (int)(a.tile_last[blockIdx.x] - c0) + 1;
+    const uint32_t c0 = a.tile_first[tile];
+    const int nc = (int)(a.tile_last[tile] - c0) + 1;
 
     // cluster table of the tile
     for (int i = tid; i < nc; i += kSplitThreads) {
@@ -163,15 +217,7 @@ __global__ void __launch_bounds__(kSplitThreads, 3) split_kernel(SplitArgs a) {
     // carry into the first cluster when it began before this tile: sum of t over [lo, row(ts))
     if (w == 0) {
         uint64_t carry = 0;
-        if (s_ao[0] < ts) {
-            const uint64_t lo = s_lo[0], r = lo + (ts - s_ao[0]);
-            uint64_t part = 0;   // pref1(r) - pref1(lo); the partial chunk sums spread over the warp
-            const uint64_t rb = r & ~(kChunk - 1), lb = lo & ~(kChunk - 1);
-            if (rb + lane < r) part += a.t[rb + lane];
-            if (lb + lane < lo) part -= a.t[lb + lane];
-            for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
-            carry = a.PS1[r >> kChunkLog] - a.PS1[lo >> kChunkLog] + part;
-        }
+        if (s_ao[0] < ts) carry = warp_range_sum(a.PS1, a.t, s_lo[0], s_lo[0] + (ts - s_ao[0]));
         if (lane == 0) sm.carry = carry;
     }
     __syncthreads();
@@ -246,7 +292,6 @@ __global__ void __launch_bounds__(kSplitThreads, 3) split_kernel(SplitArgs a) {
         i128 D = (i128)((u128)n * SL) - (i128)((u128)S * k);
         int seg_start = p0;
         Cand best = no_cand();
-        double best_dp = 0.0;
         auto flush = [&](int seg_end) {
             const bool before = ao < ts + p0, after = ao + n > ts + pend;
             if (!before && !after) {
@@ -273,31 +318,7 @@ __global__ void __launch_bounds__(kSplitThreads, 3) split_kernel(SplitArgs a) {
                 best = no_cand();
             }
             const uint32_t tc = s_t[padx(p + 1)];
-            if (k >= 1 && tprev < tc) {                       // cut between distinct values only
-                const u128 ad = (u128)(-D);
-                const uint32_t dhi = (uint32_t)(ad >> 64);
-                const uint64_t dlo = (uint64_t)ad;
-                const double dD = approx_d(dhi, dlo);
-                const double x = __dmul_rn(dD, dD);
-                const double dp = __dmul_rn(__uint2double_rn(k), __uint2double_rn((uint32_t)(n - k)));
-                bool take = best.k == 0;
-                if (!take) {
-                    const double L = __dmul_rn(x, best_dp), R = __dmul_rn(best.x, dp);
-                    const double tol = 1.0 + 0x1p-40;
-                    if (L > __dmul_rn(R, tol)) {
-                        take = true;
-                    } else if (!(R > __dmul_rn(L, tol))) {    // near tie: exact 256-bit products
-                        Cand cd;
-                        cd.dlo = dlo; cd.dhi = dhi; cd.p = (uint64_t)k * (n - k);
-                        take = exact_cmp(cd, best) > 0;       // equal -> keep the smaller k
-                    }
-                }
-                if (take) {
-                    best.x = x; best.dlo = dlo; best.dhi = dhi; best.p = (uint64_t)k * (n - k);
-                    best.SL = SL; best.k = k;
-                    best_dp = dp;
-                }
-            }
+            if (k >= 1 && tprev < tc) eval_cut(D, k, n, SL, best);   // cut between distinct values only
             D += (i128)(uint64_t)(n * tc) - (i128)S;         // D_{k+1} = D_k + n t_k - S
             SL += tc;
             k++;
@@ -349,19 +370,99 @@ __global__ void __launch_bounds__(kSplitThreads, 3) split_kernel(SplitArgs a) {
             a.cut[c0 + head_ci] = fin.k;
             a.cut_SL[c0 + head_ci] = fin.SL;
         } else {
-            a.part[2 * (uint64_t)blockIdx.x] = Part{fin, c0 + head_ci};
+            a.part[2 * (uint64_t)tile] = Part{fin, c0 + head_ci};
         }
     }
     // the run carried out of the tile's last thread continues into the next tile
     if (p0 < nt && pend == nt && out_ci >= 0) {
         const uint64_t ao = s_ao[out_ci];
-        a.part[2 * (uint64_t)blockIdx.x + (ao <= ts ? 0 : 1)] = Part{iv, c0 + out_ci};
+        a.part[2 * (uint64_t)tile + (ao <= ts ? 0 : 1)] = Part{iv, c0 + out_ci};
+    }
+}
+
+// Tiles that lie inside one cluster (most tiles while clusters are large):
+// no cluster table, no segmentation, plain block argmax.
+struct FastSmem {
+    Cand wbest[kSplitThreads / 32];
+    uint64_t red[kSplitThreads / 32 + 1];
+    uint64_t carry;
+    uint32_t t[padx(kTile + 1) + 1];
+};
+
+__device__ __forceinline__ Cand shfl_cand_xor(const Cand &a, int m) {
+    Cand r;
+    r.x = __shfl_xor_sync(0xffffffffu, a.x, m);
+    r.dp = __shfl_xor_sync(0xffffffffu, a.dp, m);
+    r.dlo = __shfl_xor_sync(0xffffffffu, a.dlo, m);
+    r.p = __shfl_xor_sync(0xffffffffu, a.p, m);
+    r.SL = __shfl_xor_sync(0xffffffffu, a.SL, m);
+    r.dhi = __shfl_xor_sync(0xffffffffu, a.dhi, m);
+    r.k = __shfl_xor_sync(0xffffffffu, a.k, m);
+    return r;
+}
+
+__global__ void __launch_bounds__(kSplitThreads) split_fast_kernel(SplitArgs a) {
+    __shared__ FastSmem sm;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint32_t tile = a.list[blockIdx.x];
+    const uint64_t ts = (uint64_t)tile * kTile;
+    const uint64_t te = min(ts + kTile, a.A);
+    const int nt = (int)(te - ts);
+    const uint32_t c = a.tile_first[tile];
+    const uint64_t lo = a.f_lo[c], n = a.f_hi[c] - lo, S = a.f_S[c], ao = a.aoff[c];
+    const uint64_t row0 = lo + (ts - ao);              // the tile lies inside [lo, hi)
+    if (w == 0) {
+        const uint64_t carry = row0 > lo ? warp_range_sum(a.PS1, a.t, lo, row0) : 0;
+        if (lane == 0) sm.carry = carry;
+    }
+    for (int idx = tid; idx <= nt; idx += kSplitThreads)
+        sm.t[padx(idx)] = idx ? a.t[row0 + idx - 1] : (row0 > lo ? a.t[row0 - 1] : 0u);
+    __syncthreads();
+    const int p0 = tid * kSplitItems, pend = min(p0 + kSplitItems, nt);
+    uint64_t mysum = 0;
+#pragma unroll
+    for (int j = 0; j < kSplitItems; j++)
+        if (p0 + j < nt) mysum += sm.t[padx(p0 + j + 1)];
+    uint64_t tot;
+    const uint64_t excl = block_excl_scan<uint64_t, kSplitThreads>(mysum, sm.red, &tot);
+    Cand best = no_cand();
+    if (p0 < nt) {
+        uint64_t SL = sm.carry + excl;
+        uint32_t k = (uint32_t)(ts - ao + p0);
+        i128 D = (i128)((u128)n * SL) - (i128)((u128)S * k);
+        uint32_t tprev = sm.t[padx(p0)];
+        for (int p = p0; p < pend; p++) {
+            const uint32_t tc = sm.t[padx(p + 1)];
+            if (k >= 1 && tprev < tc) eval_cut(D, k, n, SL, best);
+            D += (i128)(uint64_t)(n * tc) - (i128)S;
+            SL += tc;
+            k++;
+            tprev = tc;
+        }
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const Cand v = shfl_cand_xor(best, o);
+        if (better(v, best)) best = v;
+    }
+    if (lane == 0) sm.wbest[w] = best;
+    __syncthreads();
+    if (tid == 0) {
+        for (int ww = 1; ww < kSplitThreads / 32; ww++)
+            if (better(sm.wbest[ww], best)) best = sm.wbest[ww];
+        if (ao >= ts && ao + n <= te) {
+            a.cut[c] = best.k;
+            a.cut_SL[c] = best.SL;
+        } else {
+            a.part[2 * (uint64_t)tile] = Part{best, c};   // ao <= ts: slot 0
+        }
     }
 }
 
 __device__ __forceinline__ Cand shfl_cand(const Cand &a, int src) {
     Cand r;
     r.x = __shfl_sync(0xffffffffu, a.x, src);
+    r.dp = __shfl_sync(0xffffffffu, a.dp, src);
     r.dlo = __shfl_sync(0xffffffffu, a.dlo, src);
     r.p = __shfl_sync(0xffffffffu, a.p, src);
     r.SL = __shfl_sync(0xffffffffu, a.SL, src);
@@ -545,22 +646,32 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CKS(c.ensure(c.cut_QL, c.cap_cut_QL, sizeof(u128) * C));
         CKS(c.ensure(c.cnt_sz, c.cap_cntsz, sizeof(uint64_t) * C));
         CKS(c.ensure(c.split_part, c.cap_part, sizeof(Part) * 2 * ntiles));
-        CKS(c.ensure(c.tile_map, c.cap_tile_map, sizeof(uint32_t) * 2 * ntiles));
+        CKS(c.ensure(c.tile_map, c.cap_tile_map, sizeof(uint32_t) * 4 * ntiles));
         CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(C) + 1) * sizeof(uint64_t)));
         const int nxt = cur ^ 1;
         CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
         const int tk_s = c.stage_begin("root_split");
         uint32_t *tfirst = c.tile_map, *tlast = c.tile_map + ntiles;
+        uint32_t *fast_list = c.tile_map + 2 * ntiles, *gen_list = c.tile_map + 3 * ntiles;
+        CK(cudaMemsetAsync(c.scalars->tile_counts, 0, sizeof(uint32_t) * 2, st));
         tile_map_kernel<<<(unsigned)((ntiles + 255) / 256), 256, 0, st>>>(c.f_aoff[cur], (uint32_t)C, A, ntiles,
-                                                                          tfirst, tlast);
-        SplitArgs sa{c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], tfirst, tlast, c.f_S[cur], c.PS1, c.t_sorted, A,
-                     c.cut, c.cut_SL, (Part *)c.split_part};
-        CK(cudaFuncSetAttribute(split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SplitSmem)));
-        split_kernel<<<(unsigned)ntiles, kSplitThreads, sizeof(SplitSmem), st>>>(sa);
+                                                                          tfirst, tlast, fast_list, gen_list,
+                                                                          c.scalars->tile_counts);
+        uint32_t counts[2];
+        CK(cudaMemcpyAsync(counts, c.scalars->tile_counts, sizeof(counts), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        SplitArgs sa{c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], tfirst, tlast, fast_list, c.f_S[cur], c.PS1,
+                     c.t_sorted, A, c.cut, c.cut_SL, (Part *)c.split_part};
+        if (counts[0]) split_fast_kernel<<<counts[0], kSplitThreads, 0, st>>>(sa);
+        if (counts[1]) {
+            sa.list = gen_list;
+            CK(cudaFuncSetAttribute(split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SplitSmem)));
+            split_kernel<<<counts[1], kSplitThreads, sizeof(SplitSmem), st>>>(sa);
+        }
         fixup_kernel<<<(unsigned)((C * 32 + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur],
                                                                        (uint32_t)C, (const Part *)c.split_part, c.cut,
                                                                        c.cut_SL);
-        c.launches += 3;
+        c.launches += 2 + (counts[0] ? 1 : 0) + (counts[1] ? 1 : 0);
         c.stage_end(tk_s, 4 * A + 8 * ntiles + 20 * C);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");
