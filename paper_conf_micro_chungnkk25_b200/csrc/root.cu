@@ -32,23 +32,48 @@ __host__ __device__ __forceinline__ SQ operator+(const SQ &a, const SQ &b) { ret
 __host__ __device__ __forceinline__ SQ operator-(const SQ &a, const SQ &b) { return SQ{a.s - b.s, a.q - b.q}; }
 
 // ---------------------------------------------------------------- a2: sampled P1, P2
+// Sums of t and t^2 over every 32-row chunk.  Eight lanes cover one chunk with
+// one uint4 each, so one warp load is 512 contiguous bytes; four loads are in
+// flight per lane.
 __global__ void __launch_bounds__(256) chunk_sums_kernel(const uint32_t *__restrict__ t, uint64_t n, uint64_t nchunks,
                                                          SQ *__restrict__ out) {
-    const int lane = threadIdx.x & 31;
-    const uint64_t warps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    for (uint64_t j = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < nchunks; j += warps) {
-        const uint64_t i = j * kChunk + lane;
-        const uint64_t v = i < n ? t[i] : 0;
-        uint64_t s = v, qlo = v * v, qhi = 0;
+    constexpr int kUnroll = 4;
+    const int lane = threadIdx.x & 31, sub = lane & 7, grp = lane >> 3;
+    const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const bool vec = (reinterpret_cast<uintptr_t>(t) & 15) == 0;
+    for (uint64_t base = warp * 4 * kUnroll; base < nchunks; base += nwarps * 4 * kUnroll) {
+        uint4 v[kUnroll];
 #pragma unroll
-        for (int o = 16; o; o >>= 1) {
-            s += __shfl_xor_sync(0xffffffffu, s, o);
-            const uint64_t ol = __shfl_xor_sync(0xffffffffu, qlo, o), oh = __shfl_xor_sync(0xffffffffu, qhi, o);
-            const uint64_t nl = qlo + ol;
-            qhi += oh + (nl < qlo);
-            qlo = nl;
+        for (int u = 0; u < kUnroll; u++) {
+            const uint64_t j = base + u * 4 + grp;
+            const uint64_t i = j * kChunk + sub * 4;
+            if (vec && i + 3 < n) {
+                v[u] = __ldg(reinterpret_cast<const uint4 *>(t + i));
+            } else {
+                v[u].x = i < n ? t[i] : 0;
+                v[u].y = i + 1 < n ? t[i + 1] : 0;
+                v[u].z = i + 2 < n ? t[i + 2] : 0;
+                v[u].w = i + 3 < n ? t[i + 3] : 0;
+            }
         }
-        if (lane == 0) out[j] = SQ{s, ((u128)qhi << 64) | qlo};
+#pragma unroll
+        for (int u = 0; u < kUnroll; u++) {
+            const uint64_t x0 = v[u].x, x1 = v[u].y, x2 = v[u].z, x3 = v[u].w;
+            uint64_t s = x0 + x1 + x2 + x3;
+            u128 q = (u128)(x0 * x0) + (x1 * x1) + (u128)(x2 * x2) + (x3 * x3);
+            uint64_t qlo = (uint64_t)q, qhi = (uint64_t)(q >> 64);
+#pragma unroll
+            for (int o = 4; o; o >>= 1) {
+                s += __shfl_xor_sync(0xffffffffu, s, o);
+                const uint64_t ol = __shfl_xor_sync(0xffffffffu, qlo, o), oh = __shfl_xor_sync(0xffffffffu, qhi, o);
+                const uint64_t nl = qlo + ol;
+                qhi += oh + (nl < qlo);
+                qlo = nl;
+            }
+            const uint64_t j = base + u * 4 + grp;
+            if (sub == 0 && j < nchunks) out[j] = SQ{s, ((u128)qhi << 64) | qlo};
+        }
     }
 }
 

@@ -18,11 +18,11 @@ constexpr uint64_t kFlagA = 1ull << 62, kFlagP = 2ull << 62, kValMask = (1ull <<
 // ---------------------------------------------------------------- pre-pass
 __global__ void __launch_bounds__(256) prepass_kernel(const uint32_t *__restrict__ kid, const uint32_t *__restrict__ t,
                                                       uint64_t n, uint32_t K, int smem_kid_hist,
-                                                      uint32_t *__restrict__ kid_count, uint64_t *__restrict__ hist0,
+                                                      uint32_t *__restrict__ kid_count, uint64_t *__restrict__ hist_t,
                                                       uint32_t *__restrict__ max_t, uint32_t *__restrict__ err) {
-    extern __shared__ uint32_t sh[];   // [256] digit-0 hist, then [K] kernel hist when privatized
-    uint32_t *h0 = sh, *hk = sh + kRadix;
-    for (int i = threadIdx.x; i < kRadix; i += blockDim.x) h0[i] = 0;
+    extern __shared__ uint32_t sh[];   // [4][256] histograms of the 4 bytes of t, then [K] kernel hist
+    uint32_t *h0 = sh, *hk = sh + 4 * kRadix;
+    for (int i = threadIdx.x; i < 4 * kRadix; i += blockDim.x) h0[i] = 0;
     if (smem_kid_hist)
         for (uint32_t i = threadIdx.x; i < K; i += blockDim.x) hk[i] = 0;
     __syncthreads();
@@ -33,6 +33,9 @@ __global__ void __launch_bounds__(256) prepass_kernel(const uint32_t *__restrict
     auto one = [&](uint32_t k, uint32_t x) {
         mx = max(mx, x);
         atomicAdd(&h0[x & 0xFF], 1u);
+        atomicAdd(&h0[kRadix + ((x >> 8) & 0xFF)], 1u);
+        atomicAdd(&h0[2 * kRadix + ((x >> 16) & 0xFF)], 1u);
+        atomicAdd(&h0[3 * kRadix + (x >> 24)], 1u);
         if (k >= K) { bad = 1; return; }
         if (smem_kid_hist) atomicAdd(&hk[k], 1u); else atomicAdd(&kid_count[k], 1u);
     };
@@ -58,11 +61,20 @@ __global__ void __launch_bounds__(256) prepass_kernel(const uint32_t *__restrict
         if (bad) atomicOr(err, 1u);
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < kRadix; i += blockDim.x)
-        if (h0[i]) atomicAdd((unsigned long long *)&hist0[i], (unsigned long long)h0[i]);
+    for (int i = threadIdx.x; i < 4 * kRadix; i += blockDim.x)
+        if (h0[i]) atomicAdd((unsigned long long *)&hist_t[i], (unsigned long long)h0[i]);
     if (smem_kid_hist)
         for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
             if (hk[i]) atomicAdd(&kid_count[i], hk[i]);
+}
+
+// histograms of the kernel-id bytes of the aligned key, from the kernel-id counts
+__global__ void kid_digit_hist_kernel(const uint32_t *__restrict__ kid_count, uint32_t K, int nbytes,
+                                      uint64_t *__restrict__ hist) {
+    const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (g >= K || kid_count[g] == 0) return;
+    for (int b = 0; b < nbytes; b++)
+        atomicAdd((unsigned long long *)&hist[b * kRadix + ((g >> (8 * b)) & 0xFF)], (unsigned long long)kid_count[g]);
 }
 
 // ---------------------------------------------------------------- one-sweep pass
@@ -75,6 +87,7 @@ struct PassArgs {
     uint32_t *t_out, *row_out;          // LAST
     uint64_t n;
     int shift, tbits, npasses;
+    int first_hist;                     // FIRST: accumulate the later digits' histograms here
     const uint64_t *hist;               // [npasses][256] global digit counts
     uint64_t *hist_all;                 // FIRST: accumulates digits 1..npasses-1
     uint64_t *status;                   // [ntiles][256]
@@ -82,7 +95,7 @@ struct PassArgs {
 };
 
 template <bool FIRST, bool LAST>
-__global__ void __launch_bounds__(kSortThreads) onesweep_kernel(PassArgs a) {
+__global__ void __launch_bounds__(kSortThreads, 3) onesweep_kernel(PassArgs a) {
     extern __shared__ __align__(16) unsigned char s_dyn[];
     uint64_t *s_keys = reinterpret_cast<uint64_t *>(s_dyn);                        // [kSortTile]
     uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + kSortTile);           // [kSortTile]
@@ -95,7 +108,7 @@ __global__ void __launch_bounds__(kSortThreads) onesweep_kernel(PassArgs a) {
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     if (tid == 0) s_tile = atomicAdd(a.tile_counter, 1u);
     for (int i = tid; i < kSortWarps * kRadix; i += kSortThreads) (&s_whist[0][0])[i] = 0;
-    if (FIRST)
+    if (FIRST && a.first_hist)
         for (int i = tid; i < 7 * kRadix; i += kSortThreads) (&s_hlater[0][0])[i] = 0;
     __syncthreads();
     const uint32_t tile = s_tile;
@@ -122,7 +135,7 @@ __global__ void __launch_bounds__(kSortThreads) onesweep_kernel(PassArgs a) {
             val[j] = 0;
         }
     }
-    if (FIRST) {   // histograms of the later digits (each key seen exactly once here)
+    if (FIRST && a.first_hist) {   // histograms of the later digits (each key seen exactly once here)
 #pragma unroll
         for (int j = 0; j < kSortItems; j++) {
             const uint64_t i = wbase + (uint64_t)j * 32 + lane;
@@ -202,7 +215,7 @@ __global__ void __launch_bounds__(kSortThreads) onesweep_kernel(PassArgs a) {
         s_delta[d] = g_excl + s_delta[d] - c_excl;   // global position - local position
         if (d == kRadix - 1) s_lstart[kRadix] = c_excl + cnt;
     }
-    if (FIRST) {
+    if (FIRST && a.first_hist) {
         for (int p = 1; p < a.npasses; p++) {
             const uint32_t h = s_hlater[p - 1][d];
             if (h) atomicAdd((unsigned long long *)&a.hist_all[p * kRadix + d], (unsigned long long)h);
@@ -241,6 +254,7 @@ __global__ void __launch_bounds__(kSortThreads) onesweep_kernel(PassArgs a) {
 template <bool FIRST, bool LAST>
 static int launch_pass(const PassArgs &a, uint64_t ntiles, size_t smem, cudaStream_t st) {
     CK(cudaFuncSetAttribute(onesweep_kernel<FIRST, LAST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    CK(cudaFuncSetAttribute(onesweep_kernel<FIRST, LAST>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     onesweep_kernel<FIRST, LAST><<<(unsigned)ntiles, kSortThreads, smem, st>>>(a);
     return STEM_OK;
 }
@@ -249,15 +263,16 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
     cudaStream_t st = c.stream;
     // pre-pass
     CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * (K + 1), st));
-    CK(cudaMemsetAsync(c.hist, 0, sizeof(uint64_t) * 8 * kRadix, st));
+    CK(cudaMemsetAsync(c.hist, 0, sizeof(uint64_t) * 12 * kRadix, st));
     CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
+    uint64_t *hist_t = c.hist + 8 * kRadix;   // [4][256] bytes of t (pre-pass)
     const int smem_kid = (K <= 40000) ? 1 : 0;
-    const size_t sm_bytes = sizeof(uint32_t) * (kRadix + (smem_kid ? K : 0));
+    const size_t sm_bytes = sizeof(uint32_t) * (4 * kRadix + (smem_kid ? K : 0));
     if (sm_bytes > 48 * 1024)
         CK(cudaFuncSetAttribute(prepass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_bytes));
     const int blocks = c.sms * (smem_kid && K > 8192 ? 2 : 4);
     const int tk_pre = c.stage_begin("prepass");
-    prepass_kernel<<<blocks, 256, sm_bytes, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.hist,
+    prepass_kernel<<<blocks, 256, sm_bytes, st>>>(kid, t, n, K, smem_kid, c.kid_count, hist_t,
                                                   &c.scalars->max_t, &c.scalars->err);
     c.launches++;
     c.stage_end(tk_pre, 8 * n);
@@ -268,12 +283,29 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
     if (hs.err) return STEM_E_RANGE;
     int kbits = 0;
     while (kbits < 32 && ((uint64_t)1 << kbits) < (uint64_t)K) kbits++;
-    int tbits = 0;
-    while (tbits < 32 && ((uint64_t)1 << tbits) <= (uint64_t)hs.max_t) tbits++;
-    if (tbits < 8) tbits = 8;
-    const int bits = kbits + tbits;
-    const int npasses = (bits + 7) / 8;
-    c.stats.key_bits = bits;
+    int tb = 0;
+    while (tb < 32 && ((uint64_t)1 << tb) <= (uint64_t)hs.max_t) tb++;
+    if (tb < 8) tb = 8;
+    // key = kernel_id << tbits | t.  Aligned layout (tbits a multiple of 8): every digit is a
+    // byte of t or of kernel_id, all histograms come from the pre-pass.  Packed layout (tbits
+    // exact) saves a pass in some traces; its later-digit histograms are built by pass 0.
+    const int tb8 = (tb + 7) & ~7;
+    const int passes_aligned = tb8 / 8 + (kbits + 7) / 8;
+    const int passes_packed = (kbits + tb + 7) / 8;
+    const bool aligned = passes_aligned <= passes_packed;
+    const int tbits = aligned ? tb8 : tb;
+    const int npasses = aligned ? passes_aligned : passes_packed;
+    if (aligned) {
+        CK(cudaMemcpyAsync(c.hist, hist_t, sizeof(uint64_t) * kRadix * (tb8 / 8), cudaMemcpyDeviceToDevice, st));
+        if (kbits) {
+            kid_digit_hist_kernel<<<(unsigned)((K + 255) / 256), 256, 0, st>>>(c.kid_count, K, (kbits + 7) / 8,
+                                                                              c.hist + kRadix * (tb8 / 8));
+            c.launches++;
+        }
+    } else {
+        CK(cudaMemcpyAsync(c.hist, hist_t, sizeof(uint64_t) * kRadix, cudaMemcpyDeviceToDevice, st));
+    }
+    c.stats.key_bits = kbits + tbits;
     c.stats.sort_passes = npasses;
     c.tbits = tbits;
 
@@ -283,6 +315,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
     a.n = n;
     a.tbits = tbits;
     a.npasses = npasses;
+    a.first_hist = aligned ? 0 : 1;
     a.hist = c.hist;
     a.hist_all = c.hist;
     a.status = (uint64_t *)c.sort_status;
@@ -303,7 +336,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
         a.t_out = c.t_sorted;
         a.row_out = c.row_sorted;
         const size_t smem = kSortTile * (sizeof(uint64_t) + sizeof(uint32_t)) +
-                            sizeof(uint32_t) * kRadix * (kSortWarps + (first ? 7 : 0));
+                            sizeof(uint32_t) * kRadix * (kSortWarps + (first && !aligned ? 7 : 0));
         const char *sname = (first && last) ? "sort_pass_only" : first ? "sort_pass_first"
                             : last ? "sort_pass_last" : "sort_pass_mid";
         const uint64_t sbytes = n * ((first ? 8 : 12) + (last ? 8 : 12));
