@@ -4,15 +4,13 @@
 // their global digit offsets by decoupled look-back.  The pre-pass validates
 // kernel ids, finds max t, histograms kernel ids (group sizes) and digit 0;
 // pass 0 histograms all later digits, so no extra histogram pass is needed.
+#include <cstdlib>
+
 #include "internal.h"
 
 namespace sr {
 
-constexpr int kSortThreads = 256;   // = radix: thread d owns digit d in the block phases
-constexpr int kSortItems = 16;
-constexpr int kSortTile = kSortThreads * kSortItems;   // 4096 keys
 constexpr int kRadix = 256;
-constexpr int kSortWarps = kSortThreads / 32;
 constexpr uint64_t kFlagA = 1ull << 62, kFlagP = 2ull << 62, kValMask = (1ull << 62) - 1;
 
 // ---------------------------------------------------------------- pre-pass
@@ -94,41 +92,49 @@ struct PassArgs {
     uint32_t *tile_counter;
 };
 
-template <bool FIRST, bool LAST>
-__global__ void __launch_bounds__(kSortThreads, 3) onesweep_kernel(PassArgs a) {
+// One LSD pass over 8-bit digit (key >> shift) & 0xFF.  NT threads, IT keys per
+// thread, tile = NT*IT keys.  Keys are loaded warp-striped (coalesced), ranked
+// in element order by warp-level multi-split (match.any), the tile's digit
+// counts are published and the global offsets found by decoupled look-back
+// (thread d < 256 owns digit d), then keys are staged in shared memory in
+// tile-sorted order and written out in digit runs (coalesced).
+template <int NT, int IT, bool FIRST, bool LAST>
+__global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : 3)) onesweep_kernel(PassArgs a) {
+    constexpr int NW = NT / 32, TILE = NT * IT;
     extern __shared__ __align__(16) unsigned char s_dyn[];
-    uint64_t *s_keys = reinterpret_cast<uint64_t *>(s_dyn);                        // [kSortTile]
-    uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + kSortTile);           // [kSortTile]
-    uint32_t (*s_whist)[kRadix] = reinterpret_cast<uint32_t (*)[kRadix]>(s_vals + kSortTile);  // [warps][radix]
-    uint32_t (*s_hlater)[kRadix] = s_whist + kSortWarps;                            // FIRST: [7][radix]
+    uint64_t *s_keys = reinterpret_cast<uint64_t *>(s_dyn);                          // [TILE]
+    uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + TILE);                  // [TILE]
+    uint16_t (*s_whist)[kRadix] = reinterpret_cast<uint16_t (*)[kRadix]>(s_vals + TILE);   // [NW][radix]
+    uint32_t (*s_hlater)[kRadix] = reinterpret_cast<uint32_t (*)[kRadix]>(s_whist + NW);   // FIRST: [7][radix]
     __shared__ uint64_t s_delta[kRadix];
     __shared__ uint32_t s_lstart[kRadix + 1];
+    __shared__ uint64_t s_gw[8];
+    __shared__ uint32_t s_cw[8];
     __shared__ uint32_t s_tile;
 
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     if (tid == 0) s_tile = atomicAdd(a.tile_counter, 1u);
-    for (int i = tid; i < kSortWarps * kRadix; i += kSortThreads) (&s_whist[0][0])[i] = 0;
+    for (int i = tid; i < NW * kRadix / 2; i += NT) reinterpret_cast<uint32_t *>(&s_whist[0][0])[i] = 0;
     if (FIRST && a.first_hist)
-        for (int i = tid; i < 7 * kRadix; i += kSortThreads) (&s_hlater[0][0])[i] = 0;
+        for (int i = tid; i < 7 * kRadix; i += NT) (&s_hlater[0][0])[i] = 0;
     __syncthreads();
     const uint32_t tile = s_tile;
-    const uint64_t tile_base = (uint64_t)tile * kSortTile;
-    const uint64_t wbase = tile_base + (uint64_t)w * (32 * kSortItems);
+    const uint64_t wbase = (uint64_t)tile * TILE + (uint64_t)w * (32 * IT);
     const uint64_t tmask = (a.tbits >= 64) ? ~0ull : ((1ull << a.tbits) - 1);
 
     // load (warp-striped: item j of lane l is element wbase + 32 j + l)
-    uint64_t key[kSortItems];
-    uint32_t val[kSortItems];
+    uint64_t key[IT];
+    uint32_t val[IT];
 #pragma unroll
-    for (int j = 0; j < kSortItems; j++) {
+    for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         if (i < a.n) {
             if (FIRST) {
                 key[j] = ((uint64_t)__ldg(a.kid_in + i) << a.tbits) | (uint64_t)__ldg(a.t_in + i);
                 val[j] = (uint32_t)i;
             } else {
-                key[j] = a.keys_in[i];
-                val[j] = a.vals_in[i];
+                key[j] = __ldcs(a.keys_in + i);
+                val[j] = __ldcs(a.vals_in + i);
             }
         } else {
             key[j] = ~0ull;
@@ -137,7 +143,7 @@ __global__ void __launch_bounds__(kSortThreads, 3) onesweep_kernel(PassArgs a) {
     }
     if (FIRST && a.first_hist) {   // histograms of the later digits (each key seen exactly once here)
 #pragma unroll
-        for (int j = 0; j < kSortItems; j++) {
+        for (int j = 0; j < IT; j++) {
             const uint64_t i = wbase + (uint64_t)j * 32 + lane;
             if (i < a.n)
                 for (int p = 1; p < a.npasses; p++) atomicAdd(&s_hlater[p - 1][(key[j] >> (8 * p)) & 0xFF], 1u);
@@ -145,9 +151,9 @@ __global__ void __launch_bounds__(kSortThreads, 3) onesweep_kernel(PassArgs a) {
     }
 
     // warp-level multi-split ranking, in element order
-    uint32_t rank[kSortItems];
+    uint32_t rank[IT];
 #pragma unroll
-    for (int j = 0; j < kSortItems; j++) {
+    for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         const bool valid = i < a.n;
         const uint32_t vmask = __ballot_sync(0xffffffffu, valid);
@@ -158,74 +164,70 @@ __global__ void __launch_bounds__(kSortThreads, 3) onesweep_kernel(PassArgs a) {
             const uint32_t below = __popc(peers & ((1u << lane) - 1));
             rank[j] = base + below;
             __syncwarp(vmask);
-            if (below == 0) s_whist[w][d] = base + __popc(peers);
+            if (below == 0) s_whist[w][d] = (uint16_t)(base + __popc(peers));
         }
         __syncwarp();
     }
     __syncthreads();
 
-    // per digit: exclusive offsets over warps and tile count
+    // digit phase (threads d < 256): warp offsets, tile count, look-back
     const int d = tid;
     uint32_t cnt = 0;
+    uint64_t excl = 0, gcount = 0, g_incl = 0;
+    uint32_t c_incl = 0;
+    if (d < kRadix) {
 #pragma unroll
-    for (int ww = 0; ww < kSortWarps; ww++) {
-        const uint32_t c = s_whist[ww][d];
-        s_whist[ww][d] = cnt;
-        cnt += c;
-    }
-    // decoupled look-back on digit d
-    uint64_t *st = a.status + (uint64_t)tile * kRadix + d;
-    if (tile == 0) {
-        __stcg(st, kFlagP | cnt);
-    } else {
-        __stcg(st, kFlagA | cnt);
-        uint64_t excl = 0;
-        int64_t j = (int64_t)tile - 1;
-        while (true) {
-            const uint64_t s = *(volatile uint64_t *)(a.status + (uint64_t)j * kRadix + d);
-            if (s & kFlagP) { excl += s & kValMask; break; }
-            if (s & kFlagA) { excl += s & kValMask; j--; continue; }
+        for (int ww = 0; ww < NW; ww++) {
+            const uint32_t c = s_whist[ww][d];
+            s_whist[ww][d] = (uint16_t)cnt;
+            cnt += c;
         }
-        __stcg(st, kFlagP | (excl + cnt));
-        s_delta[d] = excl;  // temporarily the tile's exclusive prefix within digit d
-    }
-    if (tile == 0) s_delta[d] = 0;
-    // global bucket base for digit d (exclusive scan of the pass histogram)
-    const int pass = a.shift / 8;
-    const uint64_t gcount = a.hist[pass * kRadix + d];
-    // block exclusive scan over digits of (gcount) and of (cnt)
-    {
-        uint64_t g_incl = gcount;
-        uint32_t c_incl = cnt;
+        uint64_t *st = a.status + (uint64_t)tile * kRadix + d;
+        if (tile == 0) {
+            __stcg(st, kFlagP | cnt);
+        } else {
+            __stcg(st, kFlagA | cnt);
+            int64_t j = (int64_t)tile - 1;
+            while (true) {
+                const uint64_t sv = *(volatile uint64_t *)(a.status + (uint64_t)j * kRadix + d);
+                if (sv & kFlagP) { excl += sv & kValMask; break; }
+                if (sv & kFlagA) { excl += sv & kValMask; j--; }
+            }
+            __stcg(st, kFlagP | (excl + cnt));
+        }
+        gcount = a.hist[(a.shift / 8) * kRadix + d];
+        g_incl = gcount;
+        c_incl = cnt;
+#pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             const uint64_t gv = __shfl_up_sync(0xffffffffu, g_incl, o);
             const uint32_t cv = __shfl_up_sync(0xffffffffu, c_incl, o);
             if (lane >= o) { g_incl += gv; c_incl += cv; }
         }
-        __shared__ uint64_t s_gw[kSortWarps];
-        __shared__ uint32_t s_cw[kSortWarps];
         if (lane == 31) { s_gw[w] = g_incl; s_cw[w] = c_incl; }
-        __syncthreads();
+    }
+    __syncthreads();
+    if (d < kRadix) {
         uint64_t goff = 0;
         uint32_t coff = 0;
         for (int ww = 0; ww < w; ww++) { goff += s_gw[ww]; coff += s_cw[ww]; }
         const uint64_t g_excl = goff + g_incl - gcount;
         const uint32_t c_excl = coff + c_incl - cnt;
         s_lstart[d] = c_excl;
-        s_delta[d] = g_excl + s_delta[d] - c_excl;   // global position - local position
+        s_delta[d] = g_excl + excl - c_excl;   // global position - local position
         if (d == kRadix - 1) s_lstart[kRadix] = c_excl + cnt;
-    }
-    if (FIRST && a.first_hist) {
-        for (int p = 1; p < a.npasses; p++) {
-            const uint32_t h = s_hlater[p - 1][d];
-            if (h) atomicAdd((unsigned long long *)&a.hist_all[p * kRadix + d], (unsigned long long)h);
+        if (FIRST && a.first_hist) {
+            for (int p = 1; p < a.npasses; p++) {
+                const uint32_t h = s_hlater[p - 1][d];
+                if (h) atomicAdd((unsigned long long *)&a.hist_all[p * kRadix + d], (unsigned long long)h);
+            }
         }
     }
     __syncthreads();
 
     // scatter into shared memory in tile-sorted order
 #pragma unroll
-    for (int j = 0; j < kSortItems; j++) {
+    for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         if (i < a.n) {
             const uint32_t dd = (uint32_t)(key[j] >> a.shift) & 0xFF;
@@ -236,27 +238,64 @@ __global__ void __launch_bounds__(kSortThreads, 3) onesweep_kernel(PassArgs a) {
     }
     __syncthreads();
     const uint32_t nvalid = s_lstart[kRadix];
-    for (uint32_t i = tid; i < nvalid; i += kSortThreads) {
+#pragma unroll 4
+    for (uint32_t i = tid; i < nvalid; i += NT) {
         const uint64_t k = s_keys[i];
         const uint32_t dd = (uint32_t)(k >> a.shift) & 0xFF;
         const uint64_t gp = s_delta[dd] + i;
         if (LAST) {
-            a.t_out[gp] = (uint32_t)(k & tmask);
-            a.row_out[gp] = s_vals[i];
+            __stcs(a.t_out + gp, (uint32_t)(k & tmask));
+            __stcs(a.row_out + gp, s_vals[i]);
         } else {
-            a.keys_out[gp] = k;
-            a.vals_out[gp] = s_vals[i];
+            __stcs(a.keys_out + gp, k);
+            __stcs(a.vals_out + gp, s_vals[i]);
         }
     }
 }
 
 // ---------------------------------------------------------------- host driver
-template <bool FIRST, bool LAST>
-static int launch_pass(const PassArgs &a, uint64_t ntiles, size_t smem, cudaStream_t st) {
-    CK(cudaFuncSetAttribute(onesweep_kernel<FIRST, LAST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    CK(cudaFuncSetAttribute(onesweep_kernel<FIRST, LAST>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-    onesweep_kernel<FIRST, LAST><<<(unsigned)ntiles, kSortThreads, smem, st>>>(a);
+template <int NT, int IT, bool FIRST, bool LAST>
+static int launch_pass(const PassArgs &a, uint64_t ntiles, bool first_hist, cudaStream_t st) {
+    const size_t smem = (size_t)NT * IT * (sizeof(uint64_t) + sizeof(uint32_t)) + sizeof(uint16_t) * kRadix * (NT / 32) +
+                        (FIRST && first_hist ? sizeof(uint32_t) * 7 * kRadix : 0);
+    CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)smem));
+    CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                            100));
+    onesweep_kernel<NT, IT, FIRST, LAST><<<(unsigned)ntiles, NT, smem, st>>>(a);
     return STEM_OK;
+}
+
+template <int NT, int IT>
+static int launch_pass_cfg(const PassArgs &a, bool first, bool last, bool first_hist, cudaStream_t st) {
+    const uint64_t ntiles = (a.n + (uint64_t)NT * IT - 1) / ((uint64_t)NT * IT);
+    if (first && last) return launch_pass<NT, IT, true, true>(a, ntiles, first_hist, st);
+    if (first) return launch_pass<NT, IT, true, false>(a, ntiles, first_hist, st);
+    if (last) return launch_pass<NT, IT, false, true>(a, ntiles, first_hist, st);
+    return launch_pass<NT, IT, false, false>(a, ntiles, first_hist, st);
+}
+
+// tile configurations (threads, keys per thread); STEMROOT_SORT_CFG selects one for experiments
+struct SortCfg { int nt, it; };
+static const SortCfg kSortCfgs[] = {{256, 16}, {512, 8}, {384, 12}, {512, 12}};
+
+static int sort_cfg() {
+    static int cfg = -1;
+    if (cfg < 0) {
+        const char *e = getenv("STEMROOT_SORT_CFG");
+        cfg = e ? atoi(e) : 1;
+        if (cfg < 0 || cfg > 3) cfg = 1;
+    }
+    return cfg;
+}
+
+static int launch_sort_pass(const PassArgs &a, bool first, bool last, bool first_hist, cudaStream_t st) {
+    switch (sort_cfg()) {
+        case 0: return launch_pass_cfg<256, 16>(a, first, last, first_hist, st);
+        case 2: return launch_pass_cfg<384, 12>(a, first, last, first_hist, st);
+        case 3: return launch_pass_cfg<512, 12>(a, first, last, first_hist, st);
+        default: return launch_pass_cfg<512, 8>(a, first, last, first_hist, st);
+    }
 }
 
 int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K) {
@@ -309,8 +348,9 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
     c.stats.sort_passes = npasses;
     c.tbits = tbits;
 
-    const uint64_t ntiles = (n + kSortTile - 1) / kSortTile;
-    c.ensure(c.sort_status, c.cap_status, ntiles * kRadix * sizeof(uint64_t));
+    const SortCfg cfg = kSortCfgs[sort_cfg()];
+    const uint64_t ntiles = (n + (uint64_t)cfg.nt * cfg.it - 1) / ((uint64_t)cfg.nt * cfg.it);
+    CKS(c.ensure(c.sort_status, c.cap_status, ntiles * kRadix * sizeof(uint64_t)));
     PassArgs a{};
     a.n = n;
     a.tbits = tbits;
@@ -335,18 +375,11 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
         a.vals_out = vout;
         a.t_out = c.t_sorted;
         a.row_out = c.row_sorted;
-        const size_t smem = kSortTile * (sizeof(uint64_t) + sizeof(uint32_t)) +
-                            sizeof(uint32_t) * kRadix * (kSortWarps + (first && !aligned ? 7 : 0));
         const char *sname = (first && last) ? "sort_pass_only" : first ? "sort_pass_first"
                             : last ? "sort_pass_last" : "sort_pass_mid";
         const uint64_t sbytes = n * ((first ? 8 : 12) + (last ? 8 : 12));
         const int tk = c.stage_begin(sname);
-        int rc;
-        if (first && last) rc = launch_pass<true, true>(a, ntiles, smem, st);
-        else if (first) rc = launch_pass<true, false>(a, ntiles, smem, st);
-        else if (last) rc = launch_pass<false, true>(a, ntiles, smem, st);
-        else rc = launch_pass<false, false>(a, ntiles, smem, st);
-        CKS(rc);
+        CKS(launch_sort_pass(a, first, last, !aligned, st));
         c.launches++;
         c.stage_end(tk, sbytes);
         CK(cudaGetLastError());
