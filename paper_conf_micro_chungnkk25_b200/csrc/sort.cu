@@ -253,6 +253,165 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : 3)) onesweep_kernel(PassA
     }
 }
 
+// ---------------------------------------------------------------- reduce-then-scan pass
+// (alternative to the look-back: per-tile digit counts -> one scan -> scatter)
+template <int NT, int IT, bool FIRST>
+__global__ void __launch_bounds__(NT) upsweep_kernel(PassArgs a, uint32_t *__restrict__ tile_hist, uint64_t ntiles) {
+    constexpr int TILE = NT * IT;
+    __shared__ uint32_t h[kRadix];
+    for (int i = threadIdx.x; i < kRadix; i += NT) h[i] = 0;
+    __syncthreads();
+    const uint64_t base = (uint64_t)blockIdx.x * TILE;
+#pragma unroll
+    for (int j = 0; j < IT; j++) {
+        const uint64_t i = base + (uint64_t)j * NT + threadIdx.x;
+        if (i < a.n) {
+            uint64_t k;
+            if (FIRST) k = ((uint64_t)__ldg(a.kid_in + i) << a.tbits) | (uint64_t)__ldg(a.t_in + i);
+            else k = __ldg(a.keys_in + i);
+            atomicAdd(&h[(k >> a.shift) & 0xFF], 1u);
+        }
+    }
+    __syncthreads();
+    for (int d = threadIdx.x; d < kRadix; d += NT) tile_hist[(uint64_t)d * ntiles + blockIdx.x] = h[d];
+}
+
+template <int NT, int IT, bool FIRST, bool LAST>
+__global__ void __launch_bounds__(NT, 2) downsweep_kernel(PassArgs a, const uint32_t *__restrict__ tile_off,
+                                                          uint64_t ntiles) {
+    constexpr int NW = NT / 32, TILE = NT * IT;
+    extern __shared__ __align__(16) unsigned char s_dyn[];
+    uint64_t *s_keys = reinterpret_cast<uint64_t *>(s_dyn);
+    uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + TILE);
+    uint16_t (*s_whist)[kRadix] = reinterpret_cast<uint16_t (*)[kRadix]>(s_vals + TILE);
+    __shared__ uint64_t s_delta[kRadix];
+    __shared__ uint32_t s_lstart[kRadix + 1];
+    __shared__ uint32_t s_cw[8];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    for (int i = tid; i < NW * kRadix / 2; i += NT) reinterpret_cast<uint32_t *>(&s_whist[0][0])[i] = 0;
+    __syncthreads();
+    const uint32_t tile = blockIdx.x;
+    const uint64_t wbase = (uint64_t)tile * TILE + (uint64_t)w * (32 * IT);
+    const uint64_t tmask = (a.tbits >= 64) ? ~0ull : ((1ull << a.tbits) - 1);
+    uint64_t key[IT];
+    uint32_t val[IT];
+#pragma unroll
+    for (int j = 0; j < IT; j++) {
+        const uint64_t i = wbase + (uint64_t)j * 32 + lane;
+        if (i < a.n) {
+            if (FIRST) {
+                key[j] = ((uint64_t)__ldg(a.kid_in + i) << a.tbits) | (uint64_t)__ldg(a.t_in + i);
+                val[j] = (uint32_t)i;
+            } else {
+                key[j] = __ldcs(a.keys_in + i);
+                val[j] = __ldcs(a.vals_in + i);
+            }
+        } else {
+            key[j] = ~0ull;
+            val[j] = 0;
+        }
+    }
+    uint32_t rank[IT];
+#pragma unroll
+    for (int j = 0; j < IT; j++) {
+        const uint64_t i = wbase + (uint64_t)j * 32 + lane;
+        const bool valid = i < a.n;
+        const uint32_t vmask = __ballot_sync(0xffffffffu, valid);
+        if (valid) {
+            const uint32_t d = (uint32_t)(key[j] >> a.shift) & 0xFF;
+            const uint32_t peers = __match_any_sync(vmask, d);
+            const uint32_t base = s_whist[w][d];
+            const uint32_t below = __popc(peers & ((1u << lane) - 1));
+            rank[j] = base + below;
+            __syncwarp(vmask);
+            if (below == 0) s_whist[w][d] = (uint16_t)(base + __popc(peers));
+        }
+        __syncwarp();
+    }
+    __syncthreads();
+    const int d = tid;
+    uint32_t cnt = 0, c_incl = 0;
+    if (d < kRadix) {
+#pragma unroll
+        for (int ww = 0; ww < NW; ww++) {
+            const uint32_t c = s_whist[ww][d];
+            s_whist[ww][d] = (uint16_t)cnt;
+            cnt += c;
+        }
+        c_incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t cv = __shfl_up_sync(0xffffffffu, c_incl, o);
+            if (lane >= o) c_incl += cv;
+        }
+        if (lane == 31) s_cw[w] = c_incl;
+    }
+    __syncthreads();
+    if (d < kRadix) {
+        uint32_t coff = 0;
+        for (int ww = 0; ww < w; ww++) coff += s_cw[ww];
+        const uint32_t c_excl = coff + c_incl - cnt;
+        s_lstart[d] = c_excl;
+        s_delta[d] = (uint64_t)tile_off[(uint64_t)d * ntiles + tile] - c_excl;
+        if (d == kRadix - 1) s_lstart[kRadix] = c_excl + cnt;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < IT; j++) {
+        const uint64_t i = wbase + (uint64_t)j * 32 + lane;
+        if (i < a.n) {
+            const uint32_t dd = (uint32_t)(key[j] >> a.shift) & 0xFF;
+            const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + rank[j];
+            s_keys[lp] = key[j];
+            s_vals[lp] = val[j];
+        }
+    }
+    __syncthreads();
+    const uint32_t nvalid = s_lstart[kRadix];
+#pragma unroll 4
+    for (uint32_t i = tid; i < nvalid; i += NT) {
+        const uint64_t k = s_keys[i];
+        const uint32_t dd = (uint32_t)(k >> a.shift) & 0xFF;
+        const uint64_t gp = s_delta[dd] + i;
+        if (LAST) {
+            __stcs(a.t_out + gp, (uint32_t)(k & tmask));
+            __stcs(a.row_out + gp, s_vals[i]);
+        } else {
+            __stcs(a.keys_out + gp, k);
+            __stcs(a.vals_out + gp, s_vals[i]);
+        }
+    }
+}
+
+template <int NT, int IT, bool FIRST, bool LAST>
+static int rts_pass(Ctx &c, const PassArgs &a, cudaStream_t st) {
+    constexpr int TILE = NT * IT;
+    const uint64_t ntiles = (a.n + TILE - 1) / TILE;
+    const uint64_t cells = ntiles * kRadix;
+    CKS(c.ensure(c.sort_status, c.cap_status, cells * sizeof(uint32_t) * 2));
+    uint32_t *hist = (uint32_t *)c.sort_status, *off = hist + cells;
+    upsweep_kernel<NT, IT, FIRST><<<(unsigned)ntiles, NT, 0, st>>>(a, hist, ntiles);
+    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(cells) + 1) * sizeof(uint64_t)));
+    exclusive_scan<uint64_t>([hist] __device__(uint64_t i) -> uint64_t { return hist[i]; },
+                             [off] __device__(uint64_t i, uint64_t pre, uint64_t) { off[i] = (uint32_t)pre; }, cells,
+                             (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
+    const size_t smem = (size_t)TILE * 12 + sizeof(uint16_t) * kRadix * (NT / 32);
+    CK(cudaFuncSetAttribute(downsweep_kernel<NT, IT, FIRST, LAST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)smem));
+    CK(cudaFuncSetAttribute(downsweep_kernel<NT, IT, FIRST, LAST>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                            100));
+    downsweep_kernel<NT, IT, FIRST, LAST><<<(unsigned)ntiles, NT, smem, st>>>(a, off, ntiles);
+    c.launches += 2;
+    return STEM_OK;
+}
+
+static int rts_sort_pass(Ctx &c, const PassArgs &a, bool first, bool last, cudaStream_t st) {
+    if (first && last) return rts_pass<512, 8, true, true>(c, a, st);
+    if (first) return rts_pass<512, 8, true, false>(c, a, st);
+    if (last) return rts_pass<512, 8, false, true>(c, a, st);
+    return rts_pass<512, 8, false, false>(c, a, st);
+}
+
 // ---------------------------------------------------------------- host driver
 template <int NT, int IT, bool FIRST, bool LAST>
 static int launch_pass(const PassArgs &a, uint64_t ntiles, bool first_hist, cudaStream_t st) {
@@ -284,7 +443,7 @@ static int sort_cfg() {
     if (cfg < 0) {
         const char *e = getenv("STEMROOT_SORT_CFG");
         cfg = e ? atoi(e) : 1;
-        if (cfg < 0 || cfg > 3) cfg = 1;
+        if (cfg < 0 || cfg > 4) cfg = 1;
     }
     return cfg;
 }
@@ -348,7 +507,8 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
     c.stats.sort_passes = npasses;
     c.tbits = tbits;
 
-    const SortCfg cfg = kSortCfgs[sort_cfg()];
+    const bool rts = sort_cfg() == 4;   // reduce-then-scan passes (no look-back)
+    const SortCfg cfg = kSortCfgs[rts ? 1 : sort_cfg()];
     const uint64_t ntiles = (n + (uint64_t)cfg.nt * cfg.it - 1) / ((uint64_t)cfg.nt * cfg.it);
     CKS(c.ensure(c.sort_status, c.cap_status, ntiles * kRadix * sizeof(uint64_t)));
     PassArgs a{};
@@ -379,7 +539,11 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
                             : last ? "sort_pass_last" : "sort_pass_mid";
         const uint64_t sbytes = n * ((first ? 8 : 12) + (last ? 8 : 12));
         const int tk = c.stage_begin(sname);
-        CKS(launch_sort_pass(a, first, last, !aligned, st));
+        if (rts && (!first || aligned)) {
+            CKS(rts_sort_pass(c, a, first, last, st));
+        } else {
+            CKS(launch_sort_pass(a, first, last, !aligned, st));
+        }
         c.launches++;
         c.stage_end(tk, sbytes);
         CK(cudaGetLastError());

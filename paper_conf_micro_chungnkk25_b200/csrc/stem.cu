@@ -54,6 +54,55 @@ __device__ double fix_round(const uint64_t *lane) {
 }
 
 // ---------------------------------------------------------------- leaf table
+// leaf starts = positions of the 0/1 flag bytes; tile = 256 threads x 64 bytes
+constexpr int kFlagBytes = 64;
+constexpr uint64_t kFlagTile = (uint64_t)kThreads * kFlagBytes;
+
+__device__ __forceinline__ uint32_t flags_word(const uint8_t *f, uint64_t n, uint64_t i) {   // 4 flags at i
+    if (i + 3 < n) return *reinterpret_cast<const uint32_t *>(f + i);
+    uint32_t w = 0;
+    for (int b = 0; b < 4; b++)
+        if (i + b < n) w |= (uint32_t)f[i + b] << (8 * b);
+    return w;
+}
+
+__global__ void __launch_bounds__(kThreads) flag_count_kernel(const uint8_t *__restrict__ flags, uint64_t n,
+                                                             uint64_t *__restrict__ tile_cnt) {
+    __shared__ uint64_t sm[kThreads / 32 + 1];
+    const uint64_t i0 = blockIdx.x * kFlagTile + (uint64_t)threadIdx.x * kFlagBytes;
+    uint64_t c = 0;
+#pragma unroll
+    for (int q = 0; q < kFlagBytes; q += 4) c += __popc(flags_word(flags, n, i0 + q));
+    uint64_t tot;
+    block_excl_scan<uint64_t, kThreads>(c, sm, &tot);
+    if (threadIdx.x == 0) tile_cnt[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(kThreads) flag_compact_kernel(const uint8_t *__restrict__ flags, uint64_t n,
+                                                               const uint64_t *__restrict__ tile_off,
+                                                               uint32_t *__restrict__ leaf_lo) {
+    __shared__ uint64_t sm[kThreads / 32 + 1];
+    const uint64_t i0 = blockIdx.x * kFlagTile + (uint64_t)threadIdx.x * kFlagBytes;
+    uint32_t wv[kFlagBytes / 4];
+    uint64_t c = 0;
+#pragma unroll
+    for (int q = 0; q < kFlagBytes / 4; q++) {
+        wv[q] = flags_word(flags, n, i0 + 4 * q);
+        c += __popc(wv[q]);
+    }
+    uint64_t tot;
+    uint64_t pos = block_excl_scan<uint64_t, kThreads>(c, sm, &tot) + tile_off[blockIdx.x];
+#pragma unroll
+    for (int q = 0; q < kFlagBytes / 4; q++) {
+        uint32_t x = wv[q];
+        while (x) {
+            const int b = __ffs(x) - 1;               // bit 8*j marks byte j
+            leaf_lo[pos++] = (uint32_t)(i0 + 4 * q + (b >> 3));
+            x &= x - 1;
+        }
+    }
+}
+
 struct LeafArgs {
     const uint32_t *leaf_lo, *goff, *t;
     const uint64_t *PS1;
@@ -329,13 +378,15 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CKS(c.ensure(c.leaf_lo, c.cap_leaf_lo, sizeof(uint32_t) * (n + 1)));
     const int tk_leaf = c.stage_begin("leaf_table");
     {
-        const uint8_t *flags = c.flags;
-        uint32_t *leaf_lo = c.leaf_lo;
-        exclusive_scan<uint64_t>([flags] __device__(uint64_t i) -> uint64_t { return flags[i]; },
-                                 [leaf_lo] __device__(uint64_t i, uint64_t pre, uint64_t v) {
-                                     if (v) leaf_lo[pre] = (uint32_t)i;
-                                 },
-                                 n, (uint64_t *)c.scan_scratch, &c.scalars->n_leaves, st, &c.launches);
+        const uint64_t nt = (n + kFlagTile - 1) / kFlagTile;
+        CKS(c.ensure(c.leaf_moff, c.cap_leaf_moff, sizeof(uint64_t) * (nt + 1)));   // tile counts (scratch)
+        uint64_t *tcnt = c.leaf_moff;
+        flag_count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, n, tcnt);
+        exclusive_scan<uint64_t>([tcnt] __device__(uint64_t i) -> uint64_t { return tcnt[i]; },
+                                 [tcnt] __device__(uint64_t i, uint64_t pre, uint64_t) { tcnt[i] = pre; }, nt,
+                                 (uint64_t *)c.scan_scratch, &c.scalars->n_leaves, st, &c.launches);
+        flag_compact_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, n, tcnt, c.leaf_lo);
+        c.launches += 2;
         CK(cudaGetLastError());
     }
     c.stage_end(tk_leaf, n);

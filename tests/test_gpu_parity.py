@@ -189,3 +189,53 @@ def test_tracegen_cuda_matches_numpy():
         assert np.array_equal(tt.cpu().numpy().view(np.uint32), t)
         if sp.n_metrics:
             assert np.array_equal(met.cpu().numpy(), m)
+
+
+# ------------------------------------------------------------------ full BASELINE sizes
+def test_config_c3_full_size_with_metrics(ctx):
+    """configs[2] at its full size (20M rows, 12 metric columns), host-pointer path
+    (the e2e launch), element by element against the oracle."""
+    sp = G.spec("C3")
+    kid, t, met = G.generate_np(sp)
+    got, ref = _both(ctx, kid, t, sp.n_kernels, metrics=met, host=True, eps=sp.eps, seed=12345)
+    assert_plans_equal(got, ref, metrics=True)
+
+
+@pytest.mark.slow
+def test_config_c5_full_size_sampled(ctx):
+    """configs[4] (1e9 rows, 10k kernels) in the launch configuration bench.py times:
+    device-resident trace, default options.  The oracle recomputes the ROOT leaves of
+    sampled kernels one by one (leaves of a kernel depend only on its rows, P:L176-200);
+    global outputs are checked through properties that hold at any size."""
+    import torch
+    sp = G.spec("C5")
+    ds = G.DeviceSpec(sp, "cuda:0")
+    kid = torch.empty(sp.n, dtype=torch.int32, device="cuda")
+    tt = torch.empty(sp.n, dtype=torch.int32, device="cuda")
+    G.generate_cuda(ds, kid, tt)
+    p = ctx.plan(kid, tt, sp.n_kernels, eps=sp.eps, z=Z95, seed=12345)
+    cl = p["clusters"]
+    # properties: partition, exact total, ordering, bound, samples inside their clusters
+    counts = torch.bincount(kid, minlength=sp.n_kernels).cpu().numpy()
+    per_kernel = np.bincount(cl["kernel_id"], weights=cl["n"], minlength=sp.n_kernels)
+    assert np.array_equal(per_kernel.astype(np.int64), counts.astype(np.int64))
+    tot = int((tt.to(torch.int64) & 0xFFFFFFFF).sum().item())
+    assert p["true_total_ns"] == tot == int(cl["sum_ns"].astype(object).sum())
+    assert np.all(np.diff(cl["kernel_id"].astype(np.int64)) >= 0)
+    assert p["bound"] <= sp.eps and np.all(cl["m"] >= 1)
+    rows = torch.from_numpy(p["sample_row"].astype(np.int64)).cuda()
+    sc = p["sample_cluster"]
+    t_s = (tt[rows].to(torch.int64) & 0xFFFFFFFF).cpu().numpy()
+    k_s = kid[rows].cpu().numpy()
+    assert np.array_equal(k_s, cl["kernel_id"][sc].astype(np.int32))
+    assert np.all((t_s >= cl["lo_ns"][sc]) & (t_s <= cl["hi_ns"][sc]))
+    # element-wise: the oracle's leaves of sampled kernels (small to mid-size groups)
+    rng = np.random.default_rng(7)
+    cand = np.nonzero((counts > 1000) & (counts < 3_000_000))[0]
+    for k in list(rng.choice(cand, 6, replace=False)) + [int(np.argmin(np.where(counts > 0, counts, 1 << 40)))]:
+        sel = torch.nonzero(kid == int(k)).flatten()
+        sub_t = (tt[sel].to(torch.int64) & 0xFFFFFFFF).cpu().numpy().astype(np.uint32)
+        ref = O.plan(np.zeros(len(sub_t), np.uint32), sub_t, 1, eps=sp.eps, z=Z95)
+        mine = cl[cl["kernel_id"] == k]
+        for f in ("ordinal", "lo_ns", "hi_ns", "n", "sum_ns"):
+            assert np.array_equal(mine[f].astype(np.int64), ref[f].astype(np.int64)), (k, f)
