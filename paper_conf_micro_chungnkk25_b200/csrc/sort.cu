@@ -442,8 +442,8 @@ static int sort_cfg() {
     static int cfg = -1;
     if (cfg < 0) {
         const char *e = getenv("STEMROOT_SORT_CFG");
-        cfg = e ? atoi(e) : 1;
-        if (cfg < 0 || cfg > 4) cfg = 1;
+        cfg = e ? atoi(e) : 2;
+        if (cfg < 0 || cfg > 4) cfg = 2;
     }
     return cfg;
 }
