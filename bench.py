@@ -170,12 +170,18 @@ def run_ours(a):
         dist.init_process_group("nccl", device_id=dev)
     sp = tracegen.spec(a.config, n=a.n)
     eps = a.eps if a.eps is not None else sp.eps
-    # rows of this rank: the whole trace at N=1; a row-range shard at N>1 (weak scaling of
-    # independent shard plans -- the kernel-id exchange is not in this build yet)
-    n_local = sp.n
-    row0 = 0
+    # rows of this rank: the whole trace at N=1; at N>1 the contiguous row shard
+    # [r N/W, (r+1) N/W) of the same global trace (strong scaling); stem_root_plan_dist
+    # exchanges rows by kernel id over NCCL and gathers the plan on rank 0
+    row0 = sp.n * rank // world
+    n_local = sp.n * (rank + 1) // world - row0
+    comm = None
     if world > 1:
-        row0 = rank * sp.n
+        uid = torch.zeros(128, dtype=torch.uint8, device=dev)
+        if rank == 0:
+            uid.copy_(torch.frombuffer(bytearray(sr.nccl_unique_id()), dtype=torch.uint8))
+        torch.distributed.broadcast(uid, 0)
+        comm = sr.Comm.nccl(bytes(uid.cpu().numpy()), rank, world, local)
     ds = tracegen.DeviceSpec(sp, dev)
     kid = torch.empty(n_local, dtype=torch.int32, device=dev)
     tt = torch.empty(n_local, dtype=torch.int32, device=dev)
@@ -189,6 +195,9 @@ def run_ours(a):
     stream = torch.cuda.current_stream(dev)
 
     def step(timing=False):
+        if comm is not None:
+            return ctx.plan_dist(comm, kid, tt, sp.n_kernels, row0, eps=eps, conf=a.conf, metrics=met, seed=12345,
+                                 to_host=False, stream=stream.cuda_stream)
         return ctx.plan(kid, tt, sp.n_kernels, eps=eps, conf=a.conf, metrics=met, seed=12345, to_host=False,
                         stream=stream.cuda_stream)
 
@@ -228,7 +237,7 @@ def run_ours(a):
     st = ctx.stats()
     dplan = ctx.device_plan()
     ms_per_step = elapsed_ms / a.steps
-    value = (n_local * world) * a.steps / (elapsed_ms / 1e3)
+    value = sp.n * a.steps / (elapsed_ms / 1e3)
 
     # roofline of the dominant kernel (largest share of the step)
     peak, peak_src = load_peaks()
@@ -247,11 +256,12 @@ def run_ours(a):
 
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
-        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
         "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded, on device)",
-        "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": n_local * world,
+        "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n,
                    "kernels": sp.n_kernels, "eps": eps, "conf": a.conf, "metrics": nm,
-                   "parallelism": "single GPU" if world == 1 else f"{world} independent row shards",
+                   "parallelism": "single GPU" if world == 1 else
+                   f"{world} GPUs: row shards, NCCL all-to-all by kernel id, exact allreduce",
                    "l2": "inputs 8 B/row x rows >> 126 MB L2 (no flush needed)" if n_local >= 50_000_000
                    else "inputs fit in L2: latency-bound workload",
                    "sort_key_bits": st["key_bits"], "sort_passes": st["sort_passes"],
@@ -277,16 +287,27 @@ def run_ours(a):
         torch.cuda.synchronize()
         e2e_steps = max(1, min(a.steps, 3))
         d2h = 0
-        p = ctx.plan(hk, ht, sp.n_kernels, eps=eps, conf=a.conf, metrics=hm, seed=12345, stream=stream.cuda_stream)
+        def e2e_step():
+            if comm is not None:
+                return ctx.plan_dist(comm, hk, ht, sp.n_kernels, row0, eps=eps, conf=a.conf, metrics=hm,
+                                     seed=12345, stream=stream.cuda_stream)
+            return ctx.plan(hk, ht, sp.n_kernels, eps=eps, conf=a.conf, metrics=hm, seed=12345,
+                            stream=stream.cuda_stream)
+        p = e2e_step()
         torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
         t0 = time.perf_counter()
         for _ in range(e2e_steps):
-            p = ctx.plan(hk, ht, sp.n_kernels, eps=eps, conf=a.conf, metrics=hm, seed=12345,
-                         stream=stream.cuda_stream)
+            p = e2e_step()
         e2e_s = (time.perf_counter() - t0) / e2e_steps
-        d2h = p["clusters"].nbytes + p["sample_row"].nbytes + p["sample_cluster"].nbytes + \
+        if world > 1:
+            tm = torch.tensor([e2e_s], device=dev, dtype=torch.float64)
+            torch.distributed.all_reduce(tm, op=torch.distributed.ReduceOp.MAX)
+            e2e_s = float(tm.item())
+        d2h = 0 if p is None else p["clusters"].nbytes + p["sample_row"].nbytes + p["sample_cluster"].nbytes + \
             p["sample_weight"].nbytes + 8 * (6 + nm)
-        line["e2e"] = {"value": n_local * world / e2e_s, "unit": UNIT,
+        line["e2e"] = {"value": sp.n / e2e_s, "unit": UNIT,
                        "h2d_bytes_per_step": n_local * (8 + 8 * nm), "d2h_bytes_per_step": int(d2h),
                        "ms_per_step": e2e_s * 1e3, "steps": e2e_steps}
         del hk, ht, hm
@@ -307,6 +328,8 @@ def run_ours(a):
     if rank == 0:
         print(json.dumps(line), flush=True)
     ctx.close()
+    if comm is not None:
+        comm.close()
     if world > 1:
         torch.distributed.destroy_process_group()
 

@@ -185,6 +185,35 @@ STEM_API int stem_ctx_stage_times(const stem_ctx *ctx, stem_stage_time *out, uin
 STEM_API void        stem_plan_free(stem_plan *p);  /* frees everything in the plan; NULL-safe */
 STEM_API const char *stem_strerror(int status);     /* static string, never NULL               */
 
+/* ---- multi-GPU (one process or thread per GPU) ---------------------------
+ * The trace is sharded by contiguous row ranges: rank r holds rows
+ * [global_row_base_r, global_row_base_r + local_shard->n) (shards in rank
+ * order, no gaps).  stem_root_plan_dist exchanges rows so that every rank
+ * owns whole kernel groups (contiguous kernel-id ranges of ~N/world rows,
+ * stem_owner_ranges), runs steps a1-a5 locally, reduces T and the exact KKT
+ * sum as integers across ranks, samples locally, and gathers the plan on rank
+ * 0 (*out is set on rank 0 only; other ranks get NULL).  The plan is
+ * identical to stem_root_plan on the unsharded trace for every world size
+ * (integers bit-exact, fp64 sums within 1e-9 relative).  All ranks must call
+ * it collectively with the same eps, conf, opts and n_kernels. */
+typedef struct stem_comm stem_comm;
+
+/* 128 opaque bytes created by one rank and shared with all (e.g. broadcast
+ * through torch.distributed); STEM_E_NCCL if libnccl.so.2 cannot be loaded. */
+STEM_API int  stem_comm_nccl_unique_id(void *id_out);
+/* NCCL communicator over NVLink/NVSwitch for (rank, world) on CUDA device. */
+STEM_API int  stem_comm_init_nccl(const void *id, int rank, int world, int device, stem_comm **out);
+/* world communicators sharing one device, to be driven by world host threads
+ * (in-process test and emulation of the multi-rank logic on one GPU). */
+STEM_API int  stem_comm_init_loopback(int world, int device, stem_comm **comms);
+STEM_API void stem_comm_destroy(stem_comm *comm);   /* NULL-safe */
+/* bounds[r] = first kernel id owned by rank r (bounds[world] = n_kernels):
+ * the smallest k with (sum_{j<k} counts[j]) * world >= r * sum(counts).  Host only. */
+STEM_API int  stem_owner_ranges(const uint64_t *counts, uint32_t n_kernels, int world, uint32_t *bounds);
+STEM_API int  stem_root_plan_dist(stem_ctx *ctx, stem_comm *comm, const stem_trace *local_shard,
+                                  uint64_t global_row_base, double eps, double conf, const stem_opts *opts,
+                                  stem_plan **out);
+
 /* z = Phi^-1(1 - (1-conf)/2), conf in (0,1); host computation. */
 STEM_API int stem_z_from_conf(double conf, double *z_out);
 

@@ -27,12 +27,25 @@ _ROOT = os.path.dirname(_HERE)
 _CSRC = os.path.join(_HERE, "csrc")
 LIB_PATH = os.path.join(_HERE, "lib", "libstemroot.so")
 HEADER = os.path.join(_ROOT, "include", "stemroot.h")
-SOURCES = ["capi.cu", "sort.cu", "root.cu", "stem.cu"]
+SOURCES = ["capi.cu", "sort.cu", "root.cu", "stem.cu", "dist.cu"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "--fmad=false",
               "--extended-lambda", "-Xcompiler", "-fPIC,-fvisibility=hidden", "-shared"]
 
 STEM_OK, STEM_E_INVAL, STEM_E_RANGE, STEM_E_NOMEM, STEM_E_CUDA, STEM_E_NCCL, STEM_E_LIMIT, STEM_E_STATE = \
     0, -1, -2, -3, -4, -5, -6, -7
+
+
+def _nccl_include():
+    import glob
+    import sys
+    for sp in sys.path:
+        hit = glob.glob(os.path.join(sp, "nvidia", "nccl", "include", "nccl.h"))
+        if hit:
+            return os.path.dirname(hit[0])
+    for p in ("/usr/include", "/usr/local/cuda/include"):
+        if os.path.exists(os.path.join(p, "nccl.h")):
+            return p
+    raise RuntimeError("nccl.h not found (the NCCL headers are needed to build dist.cu)")
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
@@ -42,7 +55,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and os.path.exists(LIB_PATH) and os.path.getmtime(LIB_PATH) >= max(map(os.path.getmtime, deps)):
         return LIB_PATH
     os.makedirs(os.path.dirname(LIB_PATH), exist_ok=True)
-    cmd = ["nvcc"] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + ["-o", LIB_PATH] + srcs
+    cmd = ["nvcc"] + NVCC_FLAGS + ["-I", _nccl_include()] + (["-Xptxas", "-v"] if verbose else []) + \
+        ["-o", LIB_PATH] + srcs + ["-ldl"]
     subprocess.check_call(cmd, cwd=_CSRC)
     return LIB_PATH
 
@@ -98,7 +112,8 @@ class stem_stage_time(C.Structure):
 
 EXPORTS = ["stem_default_opts", "stem_ctx_create", "stem_ctx_destroy", "stem_root_plan_ctx", "stem_root_plan",
            "stem_ctx_device_plan", "stem_ctx_stats", "stem_plan_free", "stem_strerror", "stem_z_from_conf",
-           "stem_ctx_enable_timing", "stem_ctx_stage_times"]
+           "stem_ctx_enable_timing", "stem_ctx_stage_times", "stem_comm_nccl_unique_id", "stem_comm_init_nccl",
+           "stem_comm_init_loopback", "stem_comm_destroy", "stem_owner_ranges", "stem_root_plan_dist"]
 
 _lib = None
 
@@ -127,6 +142,14 @@ def lib():
         L.stem_z_from_conf.argtypes = [C.c_double, P(C.c_double)]
         L.stem_ctx_enable_timing.argtypes = [C.c_void_p, C.c_int]
         L.stem_ctx_stage_times.argtypes = [C.c_void_p, P(stem_stage_time), C.c_uint32, P(C.c_uint32)]
+        L.stem_comm_nccl_unique_id.argtypes = [C.c_void_p]
+        L.stem_comm_init_nccl.argtypes = [C.c_void_p, C.c_int, C.c_int, C.c_int, P(C.c_void_p)]
+        L.stem_comm_init_loopback.argtypes = [C.c_int, C.c_int, P(C.c_void_p)]
+        L.stem_comm_destroy.argtypes = [C.c_void_p]
+        L.stem_comm_destroy.restype = None
+        L.stem_owner_ranges.argtypes = [P(C.c_uint64), C.c_uint32, C.c_int, P(C.c_uint32)]
+        L.stem_root_plan_dist.argtypes = [C.c_void_p, C.c_void_p, P(stem_trace), C.c_uint64, C.c_double,
+                                          C.c_double, P(stem_opts), P(P(stem_plan))]
         _lib = L
     return _lib
 
@@ -180,6 +203,52 @@ def _plan_to_numpy(p: stem_plan) -> dict:
                 est_metric=arr(p.est_metric, p.n_metrics, np.float64))
 
 
+def owner_ranges(counts, world: int) -> np.ndarray:
+    """stem_owner_ranges: first kernel id of every rank's contiguous range (+ n_kernels)."""
+    c = np.ascontiguousarray(counts, dtype=np.uint64)
+    b = np.zeros(world + 1, np.uint32)
+    _check(lib().stem_owner_ranges(c.ctypes.data_as(C.POINTER(C.c_uint64)), len(c), world,
+                                   b.ctypes.data_as(C.POINTER(C.c_uint32))), "stem_owner_ranges")
+    return b
+
+
+def nccl_unique_id() -> bytes:
+    buf = (C.c_uint8 * 128)()
+    _check(lib().stem_comm_nccl_unique_id(buf), "stem_comm_nccl_unique_id")
+    return bytes(buf)
+
+
+class Comm:
+    """A stem_comm: NCCL (one process per GPU) or one member of a loopback group."""
+
+    def __init__(self, handle, rank, world):
+        self._h, self.rank, self.world = handle, rank, world
+
+    @staticmethod
+    def nccl(unique_id: bytes, rank: int, world: int, device: int) -> "Comm":
+        h = C.c_void_p()
+        buf = (C.c_uint8 * 128).from_buffer_copy(unique_id)
+        _check(lib().stem_comm_init_nccl(buf, rank, world, device, C.byref(h)), "stem_comm_init_nccl")
+        return Comm(h, rank, world)
+
+    @staticmethod
+    def loopback(world: int, device: int = 0) -> list:
+        arr = (C.c_void_p * world)()
+        _check(lib().stem_comm_init_loopback(world, device, arr), "stem_comm_init_loopback")
+        return [Comm(C.c_void_p(arr[r]), r, world) for r in range(world)]
+
+    def close(self):
+        if self._h:
+            lib().stem_comm_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 class Context:
     """A stem_ctx: device workspace reused across plans (stem_ctx_create)."""
 
@@ -227,6 +296,34 @@ class Context:
         _check(st, "stem_root_plan_ctx")
         del k_keep, t_keep, m_keep
         if not to_host:
+            return None
+        res = _plan_to_numpy(out.contents)
+        lib().stem_plan_free(out)
+        return res
+
+    def plan_dist(self, comm: "Comm", kernel_id, exec_ns, n_kernels: int, global_row_base: int, eps: float = 0.05,
+                  conf: float = 0.95, metrics=None, seed: int = 0, z: float = 0.0, scope: int = 0, root: bool = True,
+                  clamp_in_split: bool = True, census_cap: bool = False, stream=None, to_host: bool = True):
+        """stem_root_plan_dist (collective).  Returns the global plan on rank 0, None elsewhere."""
+        kp, kdev, k_keep = _arg(kernel_id, np.uint32)
+        tp, tdev, t_keep = _arg(exec_ns, np.uint32)
+        n = int(np.prod(getattr(k_keep, "shape", (0,))))
+        nm, mp, m_keep = 0, None, None
+        if metrics is not None:
+            mp, _, m_keep = _arg(metrics, np.float64)
+            nm = int(m_keep.shape[0]) if len(m_keep.shape) == 2 else 1
+        if stream is None and kdev >= 0:
+            import torch
+            stream = torch.cuda.current_stream(kdev).cuda_stream
+        tr = stem_trace(n, n_kernels, kp if n else None, tp if n else None, nm, mp if n else None, kdev)
+        o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
+                      stream or None)
+        out = C.POINTER(stem_plan)()
+        st = lib().stem_root_plan_dist(self._h, comm._h, C.byref(tr), global_row_base, eps, conf, C.byref(o),
+                                       C.byref(out) if to_host else None)
+        _check(st, "stem_root_plan_dist")
+        del k_keep, t_keep, m_keep
+        if not to_host or not out:
             return None
         res = _plan_to_numpy(out.contents)
         lib().stem_plan_free(out)

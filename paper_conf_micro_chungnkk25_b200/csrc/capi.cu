@@ -57,6 +57,11 @@ void Ctx::release() {
     dfree(leaf_ord, cap_leaf_ord); dfree(fix_acc, cap_fix); dfree(kern_T, cap_kern_T); dfree(kern_g, cap_kern_g);
     dfree(red_part, cap_red); dfree(out_clusters, cap_out_cl); dfree(out_row, cap_out_row);
     dfree(out_cluster, cap_out_cluster); dfree(out_weight, cap_out_weight);
+    dfree(part_cnt, cap_part_cnt); dfree(dist_cnt, cap_dist_cnt);
+    for (int i = 0; i < 3; i++) { dfree(xfer_u32[i], cap_xfer_u32[i]); dfree(recv_u32[i], cap_recv_u32[i]); }
+    dfree(xfer_f64, cap_xfer_f64); dfree(xfer_f64b, cap_xfer_f64b); dfree(red_part2, cap_red2);
+    dfree(g_clusters, cap_g_clusters); dfree(g_row, cap_g_row); dfree(g_cluster, cap_g_cluster);
+    dfree(g_weight, cap_g_weight);
 }
 
 // z = Phi^-1(1 - q), q = (1-conf)/2: Acklam's rational initial guess for the
@@ -136,7 +141,7 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
             met = c.in_met;
         }
     }
-    CKS(sort_trace(c, kid, t, n, K));                 // a1
+    CKS(sort_trace(c, kid, t, nullptr, n, K));        // a1
     CKS(prefix_moments(c, n));                        // a2
     if (o.root) {
         CKS(root_levels(c, n, K, eps, z, k2, o.clamp_in_split ? 1 : 0));   // a3, a4
@@ -205,6 +210,8 @@ struct stem_ctx {
     sr::Ctx c;
 };
 
+sr::Comm *stem_comm_impl(stem_comm *c);   // dist.cu
+
 extern "C" {
 
 int stem_default_opts(stem_opts *o) {
@@ -260,6 +267,49 @@ int stem_root_plan_ctx(stem_ctx *ctx, const stem_trace *trace, double eps, doubl
         return s;
     }
     if (out) return sr::to_host(ctx->c, out);
+    return STEM_OK;
+}
+
+int stem_root_plan_dist(stem_ctx *ctx, stem_comm *comm, const stem_trace *local_shard, uint64_t global_row_base,
+                        double eps, double conf, const stem_opts *opts, stem_plan **out) {
+    if (out) *out = nullptr;
+    sr::Comm *cm = stem_comm_impl(comm);
+    if (!ctx || !cm || !local_shard) return STEM_E_INVAL;
+    stem_opts o;
+    if (opts) o = *opts; else stem_default_opts(&o);
+    sr::Ctx &c = ctx->c;
+    c.have_plan = false;
+    c.launches = 0;
+    c.stats = stem_stats{};
+    c.timing.reset();
+    const stem_trace *tr = local_shard;
+    // validation identical on every rank (a local shard may be empty)
+    if (!(eps > 0.0 && eps < 1.0) || (!(o.z > 0.0) && !(conf > 0.0 && conf < 1.0)) || o.z < 0.0 ||
+        std::isnan(o.z) || std::isinf(o.z) || o.scope < 0 || o.scope > 2 || tr->n_metrics > 64 ||
+        (tr->n && (!tr->kernel_id || !tr->exec_ns)) || (tr->n && tr->n_metrics && !tr->metrics))
+        return STEM_E_INVAL;
+    if (tr->n >= (1ull << 32)) return STEM_E_RANGE;
+    if (tr->n_kernels == 0 || tr->n_kernels > (1u << 24)) return STEM_E_RANGE;
+    if (cudaSetDevice(c.device) != cudaSuccess) return STEM_E_CUDA;
+    if (tr->device >= 0 && tr->device != c.device) return STEM_E_INVAL;
+    c.stream = (cudaStream_t)o.stream;
+    double z = o.z;
+    if (!(z > 0.0)) z = sr::z_two_sided(conf);
+    c.z = z;
+    c.eps = eps;
+    c.comm = cm;
+    int s = sr::run_plan_dist(c, *cm, tr, global_row_base, eps, conf, o);
+    c.comm = nullptr;
+    c.kid_base = 0;
+    if (s != STEM_OK) return s;
+    c.n_metrics = tr->n_metrics;
+    c.stats.kernel_launches = c.launches;
+    if (c.timing.on) {
+        if (cudaStreamSynchronize(c.stream) != cudaSuccess) return STEM_E_CUDA;
+        c.timing.finish();
+    }
+    c.have_plan = true;
+    if (out && sr::comm_rank(cm) == 0) return sr::to_host(c, out);
     return STEM_OK;
 }
 

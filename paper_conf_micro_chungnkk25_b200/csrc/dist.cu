@@ -1,0 +1,672 @@
+// dist.cu -- multi-GPU plan: one process (or thread) per GPU,
+// trace rows sharded by row range.  The path shards naturally by kernel id:
+// ROOT decisions depend only on a cluster's own rows, so after
+// one all-to-all that gives every rank whole kernel groups, everything is
+// local except the two global KKT scalars (T and Ssum, reduced EXACTLY as
+// integers) and the final estimate sums.  Kernel ranges are contiguous and
+// rows arrive in global row order, so leaves, ordinals, Philox counters and
+// sample rows are identical for every GPU count.
+//
+// Collectives go through class Comm: NCCL (dlopen'ed libnccl.so.2, device
+// buffers over NVLink/NVSwitch) or a loopback group of threads sharing one
+// GPU (single-GPU tests of the multi-rank logic).
+#include <dlfcn.h>
+
+#include <condition_variable>
+#include <cstring>
+#include <memory>
+#include <mutex>
+#include <vector>
+
+#include "internal.h"
+#include "nccl.h"
+
+namespace sr {
+
+// ---------------------------------------------------------------- communicators
+class Comm {
+  public:
+    int rank = 0, world = 1, device = 0;
+    virtual ~Comm() {}
+    // in-place sum over ranks of a device buffer (u64 or f64)
+    virtual int allreduce(void *buf, size_t count, bool f64, cudaStream_t st) = 0;
+    // host arrays: all[r * count + i] = rank r's mine[i]
+    virtual int allgather_host(const uint64_t *mine, size_t count, uint64_t *all, cudaStream_t st) = 0;
+    // device buffers; counts/displacements are host arrays of `world` elements (units of elem bytes)
+    virtual int alltoallv(const void *send, const uint64_t *scnt, const uint64_t *sdsp, void *recv,
+                          const uint64_t *rcnt, const uint64_t *rdsp, size_t elem, cudaStream_t st) = 0;
+};
+
+struct NcclApi {
+    bool ok = false;
+    ncclResult_t (*getUniqueId)(ncclUniqueId *) = nullptr;
+    ncclResult_t (*commInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*allReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                              cudaStream_t) = nullptr;
+    ncclResult_t (*allGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*send)(const void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*groupStart)() = nullptr;
+    ncclResult_t (*groupEnd)() = nullptr;
+};
+
+static NcclApi &nccl() {
+    static NcclApi api = [] {
+        NcclApi a;
+        void *h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) return a;
+        a.getUniqueId = (decltype(a.getUniqueId))dlsym(h, "ncclGetUniqueId");
+        a.commInitRank = (decltype(a.commInitRank))dlsym(h, "ncclCommInitRank");
+        a.commDestroy = (decltype(a.commDestroy))dlsym(h, "ncclCommDestroy");
+        a.allReduce = (decltype(a.allReduce))dlsym(h, "ncclAllReduce");
+        a.allGather = (decltype(a.allGather))dlsym(h, "ncclAllGather");
+        a.send = (decltype(a.send))dlsym(h, "ncclSend");
+        a.recv = (decltype(a.recv))dlsym(h, "ncclRecv");
+        a.groupStart = (decltype(a.groupStart))dlsym(h, "ncclGroupStart");
+        a.groupEnd = (decltype(a.groupEnd))dlsym(h, "ncclGroupEnd");
+        a.ok = a.getUniqueId && a.commInitRank && a.commDestroy && a.allReduce && a.allGather && a.send &&
+               a.recv && a.groupStart && a.groupEnd;
+        return a;
+    }();
+    return api;
+}
+
+#define NK(x)                                      \
+    do {                                           \
+        if ((x) != ncclSuccess) return STEM_E_NCCL; \
+    } while (0)
+
+class NcclComm : public Comm {
+  public:
+    ncclComm_t comm = nullptr;
+    uint64_t *stage = nullptr;
+    size_t stage_cap = 0;
+    ~NcclComm() override {
+        if (comm) nccl().commDestroy(comm);
+        if (stage) cudaFree(stage);
+    }
+    int allreduce(void *buf, size_t count, bool f64, cudaStream_t st) override {
+        NK(nccl().allReduce(buf, buf, count, f64 ? ncclFloat64 : ncclUint64, ncclSum, comm, st));
+        return STEM_OK;
+    }
+    int allgather_host(const uint64_t *mine, size_t count, uint64_t *all, cudaStream_t st) override {
+        const size_t need = count * (world + 1) * sizeof(uint64_t);
+        if (need > stage_cap) {
+            if (stage) cudaFree(stage);
+            stage = nullptr;
+            CK(cudaMalloc((void **)&stage, need));
+            stage_cap = need;
+        }
+        uint64_t *send = stage + count * world;
+        CK(cudaMemcpyAsync(send, mine, count * sizeof(uint64_t), cudaMemcpyHostToDevice, st));
+        NK(nccl().allGather(send, stage, count, ncclUint64, comm, st));
+        CK(cudaMemcpyAsync(all, stage, count * world * sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        return STEM_OK;
+    }
+    int alltoallv(const void *send, const uint64_t *scnt, const uint64_t *sdsp, void *recv, const uint64_t *rcnt,
+                  const uint64_t *rdsp, size_t elem, cudaStream_t st) override {
+        NK(nccl().groupStart());
+        for (int p = 0; p < world; p++) {
+            if (scnt[p])
+                NK(nccl().send((const char *)send + sdsp[p] * elem, scnt[p] * elem, ncclUint8, p, comm, st));
+            if (rcnt[p]) NK(nccl().recv((char *)recv + rdsp[p] * elem, rcnt[p] * elem, ncclUint8, p, comm, st));
+        }
+        NK(nccl().groupEnd());
+        return STEM_OK;
+    }
+};
+
+// Loopback: `world` threads on one GPU, rendezvous on a host barrier, data moved
+// by device-to-device copies / a summing kernel.
+struct LoopGroup {
+    int world;
+    std::mutex m;
+    std::condition_variable cv;
+    int arrived = 0;
+    uint64_t gen = 0;
+    std::vector<const void *> ptr;
+    std::vector<const uint64_t *> h0, h1;
+    explicit LoopGroup(int w) : world(w), ptr(w), h0(w), h1(w) {}
+    void barrier() {
+        std::unique_lock<std::mutex> l(m);
+        const uint64_t g = gen;
+        if (++arrived == world) {
+            arrived = 0;
+            gen++;
+            cv.notify_all();
+        } else {
+            cv.wait(l, [&] { return gen != g; });
+        }
+    }
+};
+
+constexpr int kMaxWorld = 64;
+struct PtrSet { const void *p[kMaxWorld]; };
+
+__global__ void sum_buffers_kernel(PtrSet ps, int world, size_t count, bool f64, void *out) {
+    const size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= count) return;
+    if (f64) {
+        double s = 0.0;
+        for (int r = 0; r < world; r++) s = __dadd_rn(s, ((const double *)ps.p[r])[i]);   // fixed rank order
+        ((double *)out)[i] = s;
+    } else {
+        uint64_t s = 0;
+        for (int r = 0; r < world; r++) s += ((const uint64_t *)ps.p[r])[i];
+        ((uint64_t *)out)[i] = s;
+    }
+}
+
+class LoopComm : public Comm {
+  public:
+    std::shared_ptr<LoopGroup> g;
+    void *tmp = nullptr;
+    size_t tmp_cap = 0;
+    ~LoopComm() override {
+        if (tmp) cudaFree(tmp);
+    }
+    int allreduce(void *buf, size_t count, bool f64, cudaStream_t st) override {
+        if (count * 8 > tmp_cap) {
+            if (tmp) cudaFree(tmp);
+            tmp = nullptr;
+            CK(cudaMalloc(&tmp, count * 8));
+            tmp_cap = count * 8;
+        }
+        CK(cudaStreamSynchronize(st));
+        g->ptr[rank] = buf;
+        g->barrier();
+        PtrSet ps{};
+        for (int r = 0; r < world; r++) ps.p[r] = g->ptr[r];
+        if (count) sum_buffers_kernel<<<(unsigned)((count + 255) / 256), 256, 0, st>>>(ps, world, count, f64, tmp);
+        cudaError_t e = cudaStreamSynchronize(st);
+        g->barrier();   // every rank has read every buffer
+        if (e != cudaSuccess) return STEM_E_CUDA;
+        CK(cudaMemcpyAsync(buf, tmp, count * 8, cudaMemcpyDeviceToDevice, st));
+        CK(cudaStreamSynchronize(st));
+        return STEM_OK;
+    }
+    int allgather_host(const uint64_t *mine, size_t count, uint64_t *all, cudaStream_t) override {
+        g->h0[rank] = mine;
+        g->barrier();
+        for (int r = 0; r < world; r++) memcpy(all + (size_t)r * count, g->h0[r], count * sizeof(uint64_t));
+        g->barrier();
+        return STEM_OK;
+    }
+    int alltoallv(const void *send, const uint64_t *scnt, const uint64_t *sdsp, void *recv, const uint64_t *rcnt,
+                  const uint64_t *rdsp, size_t elem, cudaStream_t st) override {
+        (void)rcnt;
+        CK(cudaStreamSynchronize(st));
+        g->ptr[rank] = send;
+        g->h0[rank] = scnt;
+        g->h1[rank] = sdsp;
+        g->barrier();
+        cudaError_t e = cudaSuccess;
+        for (int r = 0; r < world && e == cudaSuccess; r++) {
+            const uint64_t cnt = g->h0[r][rank];
+            if (cnt)
+                e = cudaMemcpyAsync((char *)recv + rdsp[r] * elem, (const char *)g->ptr[r] + g->h1[r][rank] * elem,
+                                    cnt * elem, cudaMemcpyDeviceToDevice, st);
+        }
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        g->barrier();   // senders may reuse their buffers
+        if (e != cudaSuccess) return STEM_E_CUDA;
+        return STEM_OK;
+    }
+};
+
+int comm_rank(const Comm *c) { return c->rank; }
+int dist_allreduce_u64(Ctx &c, uint64_t *buf, size_t count) { return c.comm->allreduce(buf, count, false, c.stream); }
+int dist_allreduce_f64(Ctx &c, double *buf, size_t count) { return c.comm->allreduce(buf, count, true, c.stream); }
+
+// ---------------------------------------------------------------- owner ranges
+// bounds[r] = smallest k with sum_{j<k} counts[j] * world >= r * total: contiguous kernel-id
+// ranges holding ~total/world rows each (a kernel is never split).
+void owner_ranges(const uint64_t *counts, uint32_t K, int world, uint32_t *bounds) {
+    u128 total = 0;
+    for (uint32_t k = 0; k < K; k++) total += counts[k];
+    bounds[0] = 0;
+    int r = 1;
+    u128 cum = 0;
+    for (uint32_t k = 0; k < K && r < world; k++) {
+        while (r < world && cum * (u128)world >= (u128)r * total) bounds[r++] = k;
+        cum += counts[k];
+    }
+    while (r < world) bounds[r++] = K;
+    bounds[world] = K;
+}
+
+// ---------------------------------------------------------------- stable partition by destination
+constexpr int kPartThreads = 256, kPartItems = 16;
+constexpr uint64_t kPartTile = (uint64_t)kPartThreads * kPartItems;
+
+struct PartArgs {
+    const uint32_t *key;            // destination key (kernel id or global row)
+    uint64_t key_add;               // key value = key[i] + key_add (key == NULL: key_add + i)
+    uint64_t bounds[kMaxWorld + 1]; // dest = #{r in 1..world-1 : bounds[r] <= key}
+    int world;
+    uint64_t n;
+    const uint32_t *in0, *in1;      // payload u32 columns (NULL = skip)
+    uint64_t in2_add;               // third u32 column = in2_add + i (the global row), if out2
+    const double *inw;              // payload f64 column
+    uint32_t *out0, *out1, *out2;
+    double *outw;
+};
+
+__device__ __forceinline__ int part_dest(const PartArgs &a, uint64_t i) {
+    const uint64_t k = a.key ? (uint64_t)a.key[i] + a.key_add : a.key_add + i;
+    int d = 0;
+    for (int r = 1; r < a.world; r++) d += a.bounds[r] <= k;
+    return d;
+}
+
+__global__ void __launch_bounds__(kPartThreads) part_count_kernel(PartArgs a, uint64_t ntiles, uint64_t *cnt) {
+    __shared__ uint32_t h[kMaxWorld];
+    for (int i = threadIdx.x; i < a.world; i += kPartThreads) h[i] = 0;
+    __syncthreads();
+    const uint64_t base = blockIdx.x * kPartTile;
+    for (int j = 0; j < kPartItems; j++) {
+        const uint64_t i = base + (uint64_t)j * kPartThreads + threadIdx.x;
+        if (i < a.n) atomicAdd(&h[part_dest(a, i)], 1u);
+    }
+    __syncthreads();
+    for (int d = threadIdx.x; d < a.world; d += kPartThreads) cnt[(uint64_t)d * ntiles + blockIdx.x] = h[d];
+}
+
+// stable: element order within each destination is preserved (warp-striped ranking)
+__global__ void __launch_bounds__(kPartThreads) part_scatter_kernel(PartArgs a, uint64_t ntiles, const uint64_t *off) {
+    constexpr int NW = kPartThreads / 32;
+    __shared__ uint32_t wh[NW][kMaxWorld];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    for (int i = tid; i < NW * kMaxWorld; i += kPartThreads) (&wh[0][0])[i] = 0;
+    __syncthreads();
+    const uint64_t wbase = blockIdx.x * kPartTile + (uint64_t)w * 32 * kPartItems;
+    int dst[kPartItems];
+    uint32_t rank[kPartItems];
+    for (int j = 0; j < kPartItems; j++) {
+        const uint64_t i = wbase + (uint64_t)j * 32 + lane;
+        const bool valid = i < a.n;
+        const uint32_t vmask = __ballot_sync(0xffffffffu, valid);
+        dst[j] = 0;
+        rank[j] = 0;
+        if (valid) {
+            const int d = part_dest(a, i);
+            const uint32_t peers = __match_any_sync(vmask, d);
+            const uint32_t base = wh[w][d];
+            const uint32_t below = __popc(peers & ((1u << lane) - 1));
+            dst[j] = d;
+            rank[j] = base + below;
+            __syncwarp(vmask);
+            if (below == 0) wh[w][d] = base + __popc(peers);
+        }
+        __syncwarp();
+    }
+    __syncthreads();
+    if (tid < a.world) {   // exclusive offsets over warps, per destination
+        uint32_t run = 0;
+        for (int ww = 0; ww < NW; ww++) {
+            const uint32_t c = wh[ww][tid];
+            wh[ww][tid] = run;
+            run += c;
+        }
+    }
+    __syncthreads();
+    for (int j = 0; j < kPartItems; j++) {
+        const uint64_t i = wbase + (uint64_t)j * 32 + lane;
+        if (i >= a.n) continue;
+        const int d = dst[j];
+        const uint64_t pos = off[(uint64_t)d * ntiles + blockIdx.x] + wh[w][d] + rank[j];
+        if (a.out0) a.out0[pos] = a.in0[i];
+        if (a.out1) a.out1[pos] = a.in1[i];
+        if (a.out2) a.out2[pos] = (uint32_t)(a.in2_add + i);
+        if (a.outw) a.outw[pos] = a.inw[i];
+    }
+}
+
+__global__ void part_displs_kernel(const uint64_t *off, uint64_t ntiles, int world, uint64_t *displs) {
+    const int d = threadIdx.x;
+    if (d <= world) displs[d] = off[(uint64_t)d * ntiles];
+}
+
+// Runs the partition; host scnt/sdsp get per-destination counts and displacements.
+static int partition(Ctx &c, PartArgs &a, uint64_t *scnt, uint64_t *sdsp) {
+    cudaStream_t st = c.stream;
+    const int W = a.world;
+    if (a.n == 0) {
+        for (int d = 0; d < W; d++) scnt[d] = sdsp[d] = 0;
+        return STEM_OK;
+    }
+    const uint64_t ntiles = (a.n + kPartTile - 1) / kPartTile;
+    const uint64_t cells = (uint64_t)W * ntiles;
+    CKS(c.ensure(c.part_cnt, c.cap_part_cnt, sizeof(uint64_t) * (cells + 1 + kMaxWorld + 1)));
+    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(cells + 1) + 1) * sizeof(uint64_t)));
+    uint64_t *cnt = c.part_cnt, *displs = c.part_cnt + cells + 1;
+    part_count_kernel<<<(unsigned)ntiles, kPartThreads, 0, st>>>(a, ntiles, cnt);
+    exclusive_scan<uint64_t>([cnt, cells] __device__(uint64_t i) -> uint64_t { return i < cells ? cnt[i] : 0; },
+                             [cnt] __device__(uint64_t i, uint64_t pre, uint64_t) { cnt[i] = pre; }, cells + 1,
+                             (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
+    part_scatter_kernel<<<(unsigned)ntiles, kPartThreads, 0, st>>>(a, ntiles, cnt);
+    part_displs_kernel<<<1, kMaxWorld + 1, 0, st>>>(cnt, ntiles, W, displs);
+    c.launches += 3;
+    CK(cudaGetLastError());
+    uint64_t h[kMaxWorld + 1];
+    CK(cudaMemcpyAsync(h, displs, sizeof(uint64_t) * (W + 1), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    for (int d = 0; d < W; d++) {
+        sdsp[d] = h[d];
+        scnt[d] = h[d + 1] - h[d];
+    }
+    return STEM_OK;
+}
+
+// receive layout from everyone's send counts: rcnt[s] = counts s sends to me
+static int exchange_counts(Ctx &c, const uint64_t *scnt, uint64_t *rcnt, uint64_t *rdsp, uint64_t &total) {
+    const int W = c.comm->world, me = c.comm->rank;
+    std::vector<uint64_t> all((size_t)W * W);
+    CKS(c.comm->allgather_host(scnt, W, all.data(), c.stream));
+    total = 0;
+    for (int s = 0; s < W; s++) {
+        rcnt[s] = all[(size_t)s * W + me];
+        rdsp[s] = total;
+        total += rcnt[s];
+    }
+    return STEM_OK;
+}
+
+// ---------------------------------------------------------------- metric estimates across ranks
+__global__ void __launch_bounds__(256) metric_req_kernel(const uint32_t *rows, const double *w, uint64_t cnt,
+                                                         uint64_t row_base, const double *metrics, uint64_t n_local,
+                                                         uint32_t nm, double *part) {
+    __shared__ double sm[8];
+    const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    for (uint32_t cc = 0; cc < nm; cc++) {
+        double v = 0.0;
+        if (s < cnt) v = __dmul_rn(w[s], metrics[(uint64_t)cc * n_local + (rows[s] - row_base)]);
+        for (int o = 16; o; o >>= 1) v = __dadd_rn(v, __shfl_xor_sync(0xffffffffu, v, o));
+        __syncthreads();
+        if ((threadIdx.x & 31) == 0) sm[threadIdx.x >> 5] = v;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double r = 0.0;
+            for (int k = 0; k < 8; k++) r = __dadd_rn(r, sm[k]);
+            part[(uint64_t)blockIdx.x * nm + cc] = r;
+        }
+    }
+}
+
+__global__ void cols_sum_kernel(const double *part, uint64_t blocks, uint32_t cols, double *out) {
+    const uint32_t cc = threadIdx.x;
+    if (cc >= cols) return;
+    double r = 0.0;
+    for (uint64_t b = 0; b < blocks; b++) r = __dadd_rn(r, part[b * cols + cc]);
+    out[cc] = r;
+}
+
+// sum over samples of weight * metric[row]: each request goes to the rank holding the row
+int dist_metric_sums(Ctx &c, const double *metrics_local, uint32_t nm, uint64_t S, double *out) {
+    cudaStream_t st = c.stream;
+    const int W = c.comm->world;
+    PartArgs a{};
+    a.key = c.out_row;
+    a.key_add = 0;
+    for (int r = 0; r <= W; r++) a.bounds[r] = c.row_bases[r];
+    a.world = W;
+    a.n = S;
+    a.in0 = c.out_row;
+    a.inw = c.out_weight;
+    CKS(c.ensure(c.xfer_u32[0], c.cap_xfer_u32[0], sizeof(uint32_t) * (S + 1)));
+    CKS(c.ensure(c.xfer_f64, c.cap_xfer_f64, sizeof(double) * (S + 1)));
+    a.out0 = c.xfer_u32[0];
+    a.outw = c.xfer_f64;
+    uint64_t scnt[kMaxWorld], sdsp[kMaxWorld], rcnt[kMaxWorld], rdsp[kMaxWorld], R = 0;
+    CKS(partition(c, a, scnt, sdsp));
+    CKS(exchange_counts(c, scnt, rcnt, rdsp, R));
+    CKS(c.ensure(c.xfer_u32[1], c.cap_xfer_u32[1], sizeof(uint32_t) * (R + 1)));
+    CKS(c.ensure(c.xfer_f64b, c.cap_xfer_f64b, sizeof(double) * (R + 1)));
+    CKS(c.comm->alltoallv(c.xfer_u32[0], scnt, sdsp, c.xfer_u32[1], rcnt, rdsp, sizeof(uint32_t), st));
+    CKS(c.comm->alltoallv(c.xfer_f64, scnt, sdsp, c.xfer_f64b, rcnt, rdsp, sizeof(double), st));
+    const uint64_t blocks = (R + 255) / 256;
+    CKS(c.ensure(c.red_part2, c.cap_red2, sizeof(double) * (blocks * nm + nm + 1)));
+    if (R) {
+        metric_req_kernel<<<(unsigned)blocks, 256, 0, st>>>(c.xfer_u32[1], c.xfer_f64b, R, c.row_bases[c.comm->rank],
+                                                            metrics_local, c.n_local_rows, nm, c.red_part2);
+        c.launches++;
+    }
+    cols_sum_kernel<<<1, 64, 0, st>>>(c.red_part2, blocks, nm, out);
+    c.launches++;
+    CK(cudaGetLastError());
+    return c.comm->allreduce(out, nm, true, st);
+}
+
+// ---------------------------------------------------------------- the distributed plan
+__global__ void kid_counts_u64_kernel(const uint32_t *cnt32, uint32_t K, const uint32_t *err, uint64_t *out) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < K) out[i] = cnt32[i];
+    if (i == K) out[K] = *err ? 1 : 0;
+}
+
+__global__ void sub_kernel_u32(uint32_t *x, uint64_t n, uint32_t v) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) x[i] -= v;
+}
+
+__global__ void add_kernel_u32(uint32_t *x, uint64_t n, uint32_t v) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) x[i] += v;
+}
+
+int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K);   // sort.cu
+
+int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
+                  const stem_opts &o) {
+    const int W = comm.world, me = comm.rank;
+    const uint64_t n = tr->n;
+    const uint32_t K = tr->n_kernels, nm = tr->n_metrics;
+    cudaStream_t st = c.stream;
+    const uint32_t *kid = tr->kernel_id, *t = tr->exec_ns;
+    const double *met = tr->metrics;
+    if (tr->device < 0 && n) {   // host shard: copy in on the stream
+        CKS(c.ensure(c.in_kid, c.cap_in_kid, sizeof(uint32_t) * n));
+        CKS(c.ensure(c.in_t, c.cap_in_t, sizeof(uint32_t) * n));
+        CK(cudaMemcpyAsync(c.in_kid, kid, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(c.in_t, t, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
+        kid = c.in_kid;
+        t = c.in_t;
+        if (nm) {
+            CKS(c.ensure(c.in_met, c.cap_in_met, sizeof(double) * n * nm));
+            CK(cudaMemcpyAsync(c.in_met, met, sizeof(double) * n * nm, cudaMemcpyHostToDevice, st));
+            met = c.in_met;
+        }
+    }
+    // row shards of every rank (metric requests are routed by row)
+    {
+        uint64_t mine[2] = {row_base, n};
+        std::vector<uint64_t> all(2 * (size_t)W);
+        CKS(comm.allgather_host(mine, 2, all.data(), st));
+        for (int r = 0; r < W; r++) {
+            c.row_bases[r] = all[2 * r];
+            if (r > 0 && all[2 * r] != all[2 * (r - 1)] + all[2 * (r - 1) + 1]) return STEM_E_INVAL;   // contiguous
+        }
+        c.row_bases[W] = all[2 * (W - 1)] + all[2 * (W - 1) + 1];
+        if (c.row_bases[W] >= (1ull << 32)) return STEM_E_RANGE;
+        c.n_local_rows = n;
+    }
+    // 1. global kernel histogram (+ range errors) -> owner ranges
+    CKS(c.ensure(c.kid_count, c.cap_kc, sizeof(uint32_t) * ((uint64_t)K + 1)));
+    CKS(c.ensure(c.dist_cnt, c.cap_dist_cnt, sizeof(uint64_t) * ((uint64_t)K + 2)));
+    CKS(c.ensure(c.scalars, c.cap_scalars, sizeof(DevScalars)));
+    CKS(c.ensure(c.hist, c.cap_hist, sizeof(uint64_t) * 12 * 256));
+    CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
+    CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
+    const int tk_x = c.stage_begin("dist_exchange");
+    if (n) CKS(histogram_kernels(c, kid, t, n, K));
+    kid_counts_u64_kernel<<<(unsigned)((K + 256) / 256), 256, 0, st>>>(c.kid_count, K, &c.scalars->err, c.dist_cnt);
+    c.launches++;
+    CKS(comm.allreduce(c.dist_cnt, (size_t)K + 1, false, st));
+    std::vector<uint64_t> gcnt((size_t)K + 1);
+    CK(cudaMemcpyAsync(gcnt.data(), c.dist_cnt, sizeof(uint64_t) * ((uint64_t)K + 1), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (gcnt[K]) return STEM_E_RANGE;
+    std::vector<uint32_t> bounds(W + 1);
+    owner_ranges(gcnt.data(), K, W, bounds.data());
+    const uint32_t kb = bounds[me], ke = bounds[me + 1];
+    // 2. all-to-all keyed on kernel id: (kernel_id, t, global row) to the owner of the kernel
+    PartArgs pa{};
+    pa.key = kid;
+    for (int r = 0; r <= W; r++) pa.bounds[r] = bounds[r];
+    pa.world = W;
+    pa.n = n;
+    pa.in0 = kid;
+    pa.in1 = t;
+    pa.in2_add = row_base;
+    for (int i = 0; i < 3; i++) CKS(c.ensure(c.xfer_u32[i], c.cap_xfer_u32[i], sizeof(uint32_t) * (n + 1)));
+    pa.out0 = c.xfer_u32[0];
+    pa.out1 = c.xfer_u32[1];
+    pa.out2 = c.xfer_u32[2];
+    uint64_t scnt[kMaxWorld], sdsp[kMaxWorld], rcnt[kMaxWorld], rdsp[kMaxWorld], R = 0;
+    CKS(partition(c, pa, scnt, sdsp));
+    CKS(exchange_counts(c, scnt, rcnt, rdsp, R));
+    if (R >= (1ull << 32)) return STEM_E_RANGE;
+    for (int i = 0; i < 3; i++) CKS(c.ensure(c.recv_u32[i], c.cap_recv_u32[i], sizeof(uint32_t) * (R + 1)));
+    for (int i = 0; i < 3; i++)
+        CKS(comm.alltoallv(c.xfer_u32[i], scnt, sdsp, c.recv_u32[i], rcnt, rdsp, sizeof(uint32_t), st));
+    c.stage_end(tk_x, 24 * n + 12 * R);
+    // 3. the local pipeline on my kernel range (kernel ids rebased to 0)
+    const uint32_t KL = ke - kb;
+    c.kid_base = kb;
+    if (R) {
+        sub_kernel_u32<<<(unsigned)((R + 255) / 256), 256, 0, st>>>(c.recv_u32[0], R, kb);
+        c.launches++;
+        CKS(c.ensure_all(R, KL, nm));
+        CKS(sort_trace(c, c.recv_u32[0], c.recv_u32[1], c.recv_u32[2], R, KL));
+        CKS(prefix_moments(c, R));
+        if (o.root) {
+            CKS(root_levels(c, R, KL, eps, c.z, c.z / eps * (c.z / eps), o.clamp_in_split ? 1 : 0));
+        } else {
+            CKS(stem_only_leaves(c, R, KL));
+        }
+    }
+    const double q = c.z / eps;
+    CKS(leaves_and_plan(c, R, KL, met, nm, eps, c.z, q * q, o));
+    (void)conf;
+    // 4. gather the plan on rank 0, canonical order = rank order (kernel ranges ascend)
+    uint64_t mine[2] = {c.n_leaves, c.n_samples};
+    std::vector<uint64_t> all(2 * (size_t)W);
+    CKS(comm.allgather_host(mine, 2, all.data(), st));
+    uint64_t Lg = 0, Sg = 0, Loff = 0;
+    for (int r = 0; r < W; r++) {
+        if (r == me) Loff = Lg;
+        Lg += all[2 * r];
+        Sg += all[2 * r + 1];
+    }
+    if (c.n_samples && Loff) {
+        add_kernel_u32<<<(unsigned)((c.n_samples + 255) / 256), 256, 0, st>>>(c.out_cluster, c.n_samples,
+                                                                             (uint32_t)Loff);
+        c.launches++;
+    }
+    std::vector<uint64_t> s_c(W, 0), s_d(W, 0), r_c(W, 0), r_d(W, 0);
+    auto gather = [&](void *src, void *&dst, size_t &cap, size_t elem, int which) -> int {
+        s_c[0] = all[2 * me + which];
+        if (me == 0) {
+            uint64_t off = 0;
+            for (int r = 0; r < W; r++) {
+                r_c[r] = all[2 * r + which];
+                r_d[r] = off;
+                off += r_c[r];
+            }
+            CKS(c.ensure(dst, cap, elem * (off + 1)));
+        }
+        return comm.alltoallv(src, s_c.data(), s_d.data(), dst, r_c.data(), r_d.data(), elem, st);
+    };
+    CKS(gather(c.out_clusters, c.g_clusters, c.cap_g_clusters, sizeof(stem_cluster), 0));
+    CKS(gather(c.out_row, c.g_row, c.cap_g_row, sizeof(uint32_t), 1));
+    CKS(gather(c.out_cluster, c.g_cluster, c.cap_g_cluster, sizeof(uint32_t), 1));
+    CKS(gather(c.out_weight, c.g_weight, c.cap_g_weight, sizeof(double), 1));
+    CK(cudaStreamSynchronize(st));
+    if (me == 0) {   // the global plan becomes this ctx's output
+        std::swap(c.out_clusters, *(stem_cluster **)&c.g_clusters);
+        std::swap(c.cap_out_cl, c.cap_g_clusters);
+        std::swap(c.out_row, *(uint32_t **)&c.g_row);
+        std::swap(c.cap_out_row, c.cap_g_row);
+        std::swap(c.out_cluster, *(uint32_t **)&c.g_cluster);
+        std::swap(c.cap_out_cluster, c.cap_g_cluster);
+        std::swap(c.out_weight, *(double **)&c.g_weight);
+        std::swap(c.cap_out_weight, c.cap_g_weight);
+    }
+    c.n_leaves = Lg;
+    c.n_samples = Sg;
+    c.stats.n_clusters = Lg;
+    c.stats.n_samples = Sg;
+    return STEM_OK;
+}
+
+}  // namespace sr
+
+// ---------------------------------------------------------------- C ABI
+struct stem_comm {
+    std::unique_ptr<sr::Comm> c;
+};
+
+extern "C" {
+
+int stem_comm_nccl_unique_id(void *id_out) {
+    if (!id_out) return STEM_E_INVAL;
+    if (!sr::nccl().ok) return STEM_E_NCCL;
+    ncclUniqueId id;
+    if (sr::nccl().getUniqueId(&id) != ncclSuccess) return STEM_E_NCCL;
+    memcpy(id_out, &id, sizeof(id));
+    return STEM_OK;
+}
+
+int stem_comm_init_nccl(const void *id, int rank, int world, int device, stem_comm **out) {
+    if (!out) return STEM_E_INVAL;
+    *out = nullptr;
+    if (!id || world < 1 || world > sr::kMaxWorld || rank < 0 || rank >= world || device < 0) return STEM_E_INVAL;
+    if (!sr::nccl().ok) return STEM_E_NCCL;
+    if (cudaSetDevice(device) != cudaSuccess) return STEM_E_CUDA;
+    auto nc = std::make_unique<sr::NcclComm>();
+    nc->rank = rank;
+    nc->world = world;
+    nc->device = device;
+    ncclUniqueId uid;
+    memcpy(&uid, id, sizeof(uid));
+    if (sr::nccl().commInitRank(&nc->comm, world, uid, rank) != ncclSuccess) {
+        nc->comm = nullptr;
+        return STEM_E_NCCL;
+    }
+    stem_comm *x = new (std::nothrow) stem_comm();
+    if (!x) return STEM_E_NOMEM;
+    x->c = std::move(nc);
+    *out = x;
+    return STEM_OK;
+}
+
+int stem_comm_init_loopback(int world, int device, stem_comm **comms) {
+    if (!comms || world < 1 || world > sr::kMaxWorld || device < 0) return STEM_E_INVAL;
+    auto g = std::make_shared<sr::LoopGroup>(world);
+    for (int r = 0; r < world; r++) {
+        auto lc = std::make_unique<sr::LoopComm>();
+        lc->rank = r;
+        lc->world = world;
+        lc->device = device;
+        lc->g = g;
+        comms[r] = new stem_comm();
+        comms[r]->c = std::move(lc);
+    }
+    return STEM_OK;
+}
+
+void stem_comm_destroy(stem_comm *c) { delete c; }
+
+int stem_owner_ranges(const uint64_t *counts, uint32_t n_kernels, int world, uint32_t *bounds) {
+    if (!counts || !bounds || world < 1 || world > sr::kMaxWorld || n_kernels == 0) return STEM_E_INVAL;
+    sr::owner_ranges(counts, n_kernels, world, bounds);
+    return STEM_OK;
+}
+
+}  // extern "C"
+
+// the dist entry point lives with the ctx in capi.cu; this accessor bridges the opaque handle
+sr::Comm *stem_comm_impl(stem_comm *c) { return c ? c->c.get() : nullptr; }

@@ -44,6 +44,7 @@ struct DevScalars {
     double g;                     // Ssum / c (global scope)
     double est_frac, var_sum;     // sum rn(r_i)/m_i, sum rn(V_i)/m_i
     alignas(16) uint64_t wide_total[4];   // total of a wide (struct) scan
+    uint64_t red7[8];                     // multi-GPU reduction staging
 };
 
 constexpr int kFixDigits = 6;     // 6 x 32-bit digits in u64 lanes, LSB 2^-72
@@ -88,8 +89,12 @@ struct Timing {
     ~Timing() { for (auto e : pool) cudaEventDestroy(e); }
 };
 
+class Comm;   // dist.cu: multi-GPU collectives (NCCL or in-process loopback)
+
 struct Ctx {
     int device = 0;
+    Comm *comm = nullptr;          // non-NULL inside stem_root_plan_dist
+    uint32_t kid_base = 0;         // global id of local kernel 0 (dist: first owned kernel)
     int sms = 148;
     cudaStream_t stream = nullptr;
     uint32_t launches = 0;
@@ -171,19 +176,41 @@ struct Ctx {
     uint32_t *out_row = nullptr, *out_cluster = nullptr; size_t cap_out_row = 0, cap_out_cluster = 0;
     double *out_weight = nullptr; size_t cap_out_weight = 0;
     double host_est_metric[64];
+    // multi-GPU (dist.cu)
+    uint64_t *part_cnt = nullptr; size_t cap_part_cnt = 0;
+    uint64_t *dist_cnt = nullptr; size_t cap_dist_cnt = 0;
+    uint32_t *xfer_u32[3] = {nullptr, nullptr, nullptr}; size_t cap_xfer_u32[3] = {0, 0, 0};
+    uint32_t *recv_u32[3] = {nullptr, nullptr, nullptr}; size_t cap_recv_u32[3] = {0, 0, 0};
+    double *xfer_f64 = nullptr, *xfer_f64b = nullptr; size_t cap_xfer_f64 = 0, cap_xfer_f64b = 0;
+    double *red_part2 = nullptr; size_t cap_red2 = 0;
+    void *g_clusters = nullptr, *g_row = nullptr, *g_cluster = nullptr, *g_weight = nullptr;
+    size_t cap_g_clusters = 0, cap_g_row = 0, cap_g_cluster = 0, cap_g_weight = 0;
+    uint64_t row_bases[65] = {0};
+    uint64_t n_local_rows = 0;
 
     // last plan
     bool have_plan = false;
     uint64_t n = 0, n_leaves = 0, n_samples = 0, T = 0;
+    uint64_t n_samples_global = 0;
     uint32_t K = 0, n_metrics = 0;
     double est_total = 0, bound = 0, eps = 0, z = 0;
 };
 
+// multi-GPU collectives on c.comm (dist.cu); device buffers, in place, sums
+int comm_rank(const Comm *c);
+int dist_allreduce_u64(Ctx &c, uint64_t *buf, size_t count);
+int dist_allreduce_f64(Ctx &c, double *buf, size_t count);
+int dist_metric_sums(Ctx &c, const double *metrics_local, uint32_t nm, uint64_t S, double *out);
+
 // stages
-int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K);      // a1
+int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *row_in, uint64_t n,
+               uint32_t K);                                                                    // a1
 int prefix_moments(Ctx &c, uint64_t n);                                                        // a2
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp);   // a3, a4
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
+int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K);   // pre-pass only
+int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
+                  const stem_opts &o);
 int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint32_t n_metrics, double eps,
                     double z, double k2, const stem_opts &o);                                  // a5..a8
 

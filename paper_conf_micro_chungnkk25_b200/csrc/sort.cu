@@ -78,6 +78,7 @@ __global__ void kid_digit_hist_kernel(const uint32_t *__restrict__ kid_count, ui
 // ---------------------------------------------------------------- one-sweep pass
 struct PassArgs {
     const uint32_t *kid_in, *t_in;      // FIRST: trace columns
+    const uint32_t *row_in;             // FIRST: row payload (NULL = the row index)
     const uint64_t *keys_in;            // !FIRST
     const uint32_t *vals_in;            // !FIRST
     uint64_t *keys_out;                 // !LAST
@@ -131,7 +132,7 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : 3)) onesweep_kernel(PassA
         if (i < a.n) {
             if (FIRST) {
                 key[j] = ((uint64_t)__ldg(a.kid_in + i) << a.tbits) | (uint64_t)__ldg(a.t_in + i);
-                val[j] = (uint32_t)i;
+                val[j] = a.row_in ? __ldg(a.row_in + i) : (uint32_t)i;
             } else {
                 key[j] = __ldcs(a.keys_in + i);
                 val[j] = __ldcs(a.vals_in + i);
@@ -301,7 +302,7 @@ __global__ void __launch_bounds__(NT, 2) downsweep_kernel(PassArgs a, const uint
         if (i < a.n) {
             if (FIRST) {
                 key[j] = ((uint64_t)__ldg(a.kid_in + i) << a.tbits) | (uint64_t)__ldg(a.t_in + i);
-                val[j] = (uint32_t)i;
+                val[j] = a.row_in ? __ldg(a.row_in + i) : (uint32_t)i;
             } else {
                 key[j] = __ldcs(a.keys_in + i);
                 val[j] = __ldcs(a.vals_in + i);
@@ -457,7 +458,22 @@ static int launch_sort_pass(const PassArgs &a, bool first, bool last, bool first
     }
 }
 
-int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K) {
+// the pre-pass alone (kernel-id counts, range check, max t): multi-GPU histogram
+int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K) {
+    cudaStream_t st = c.stream;
+    CK(cudaMemsetAsync(c.hist, 0, sizeof(uint64_t) * 12 * kRadix, st));
+    const int smem_kid = (K <= 40000) ? 1 : 0;
+    const size_t sm_bytes = sizeof(uint32_t) * (4 * kRadix + (smem_kid ? K : 0));
+    if (sm_bytes > 48 * 1024)
+        CK(cudaFuncSetAttribute(prepass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_bytes));
+    prepass_kernel<<<c.sms * 2, 256, sm_bytes, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.hist + 8 * kRadix,
+                                                     &c.scalars->max_t, &c.scalars->err);
+    c.launches++;
+    CK(cudaGetLastError());
+    return STEM_OK;
+}
+
+int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *row_in, uint64_t n, uint32_t K) {
     cudaStream_t st = c.stream;
     // pre-pass
     CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * (K + 1), st));
@@ -529,6 +545,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint3
         const bool first = p == 0, last = p == npasses - 1;
         a.kid_in = kid;
         a.t_in = t;
+        a.row_in = row_in;
         a.keys_in = kin;
         a.vals_in = vin;
         a.keys_out = kout;

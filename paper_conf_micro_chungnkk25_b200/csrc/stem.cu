@@ -234,7 +234,7 @@ struct SampleArgs {
     const uint8_t *census;
     const uint32_t *t, *row;
     uint64_t L, n, S;
-    uint32_t key0, key1;
+    uint32_t key0, key1, kid_base;
     uint32_t *out_row, *out_cluster;
     double *out_weight;
     uint64_t *U;
@@ -252,7 +252,8 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
     if (a.census[i]) {
         pos = lo + j;
     } else {
-        const U4 x = philox4x32_10(U4{(uint32_t)(j >> 1), a.leaf_ord[i], a.leaf_kid[i], 0x53544D31u}, a.key0, a.key1);
+        const U4 x = philox4x32_10(U4{(uint32_t)(j >> 1), a.leaf_ord[i], a.kid_base + a.leaf_kid[i], 0x53544D31u},
+                                   a.key0, a.key1);
         const uint64_t r = (j & 1) ? (((uint64_t)x.w << 32) | x.z) : (((uint64_t)x.y << 32) | x.x);
         pos = lo + __umul64hi(r, n);
     }
@@ -347,12 +348,12 @@ __global__ void est_finalize_kernel(const uint64_t *sum_q, const double *red, co
 
 __global__ void pack_kernel(const uint32_t *leaf_lo, const uint32_t *leaf_kid, const uint32_t *leaf_ord,
                             const uint64_t *PS1, const u128 *PS2, const uint32_t *t, const uint64_t *m,
-                            const uint8_t *census, uint64_t L, uint64_t n, stem_cluster *out) {
+                            const uint8_t *census, uint64_t L, uint64_t n, uint32_t kid_base, stem_cluster *out) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= L) return;
     const LeafView v = leaf_view(leaf_lo, L, n, PS1, PS2, t, i);
     stem_cluster c;
-    c.kernel_id = leaf_kid[i];
+    c.kernel_id = kid_base + leaf_kid[i];
     c.ordinal = leaf_ord[i];
     c.lo_ns = t[v.lo];
     c.hi_ns = t[v.hi - 1];
@@ -381,11 +382,11 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         const uint64_t nt = (n + kFlagTile - 1) / kFlagTile;
         CKS(c.ensure(c.leaf_moff, c.cap_leaf_moff, sizeof(uint64_t) * (nt + 1)));   // tile counts (scratch)
         uint64_t *tcnt = c.leaf_moff;
-        flag_count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, n, tcnt);
+        if (nt) flag_count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, n, tcnt);
         exclusive_scan<uint64_t>([tcnt] __device__(uint64_t i) -> uint64_t { return tcnt[i]; },
                                  [tcnt] __device__(uint64_t i, uint64_t pre, uint64_t) { tcnt[i] = pre; }, nt,
                                  (uint64_t *)c.scan_scratch, &c.scalars->n_leaves, st, &c.launches);
-        flag_compact_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, n, tcnt, c.leaf_lo);
+        if (nt) flag_compact_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, n, tcnt, c.leaf_lo);
         c.launches += 2;
         CK(cudaGetLastError());
     }
@@ -411,22 +412,35 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CK(cudaMemsetAsync(c.leaf_U, 0, sizeof(uint64_t) * (L + 1), st));
 
     const int tk_kkt = c.stage_begin("stem_sizes");
-    total_kernel<<<1, 32, 0, st>>>(c.PS1, c.t_sorted, n, &c.scalars->T);
-    c.launches++;
+    if (n) {
+        total_kernel<<<1, 32, 0, st>>>(c.PS1, c.t_sorted, n, &c.scalars->T);
+        c.launches++;
+    } else {
+        CK(cudaMemsetAsync(&c.scalars->T, 0, sizeof(uint64_t), st));
+    }
     LeafArgs la{c.leaf_lo, c.goff, c.t_sorted, c.PS1, c.PS2, L, n, K, o.scope, leaf_kid, leaf_ord,
                 c.fix_acc, c.kern_T, &c.scalars->err};
-    leaf_kkt_kernel<<<blocks_for(L), kThreads, 0, st>>>(la);
+    if (L) leaf_kkt_kernel<<<blocks_for(L), kThreads, 0, st>>>(la);
     c.launches++;
+    if (c.comm) {   // multi-GPU: T and the exact Ssum digits are sums over every rank's leaves
+        uint64_t *r7 = c.scalars->red7;
+        CK(cudaMemcpyAsync(r7, &c.scalars->T, sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(r7 + 1, c.fix_acc, sizeof(uint64_t) * kFixDigits, cudaMemcpyDeviceToDevice, st));
+        CKS(dist_allreduce_u64(c, r7, o.scope == 0 ? 1 + kFixDigits : 1));
+        CK(cudaMemcpyAsync(&c.scalars->T, r7, sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
+        if (o.scope == 0)
+            CK(cudaMemcpyAsync(c.fix_acc, r7 + 1, sizeof(uint64_t) * kFixDigits, cudaMemcpyDeviceToDevice, st));
+    }
     // g per set (T = total_kernel above, exact)
     if (o.scope == 0)
         kkt_finalize_kernel<<<1, 32, 0, st>>>(c.fix_acc, nullptr, &c.scalars->T, 1, eps, z, c.kern_g, &c.scalars->ssum);
-    else if (o.scope == 1)
+    else if (o.scope == 1 && K)
         kkt_finalize_kernel<<<blocks_for(K), kThreads, 0, st>>>(c.fix_acc, c.kern_T, nullptr, K, eps, z, c.kern_g,
                                                                nullptr);
     if (o.scope != 2) c.launches++;
     MArgs ma{c.leaf_lo, leaf_kid, c.t_sorted, c.PS1, c.PS2, L, n, o.scope, o.census_cap, k2, c.kern_g, c.leaf_m,
              c.leaf_census, &c.scalars->limit_err};
-    leaf_m_kernel<<<blocks_for(L), kThreads, 0, st>>>(ma);
+    if (L) leaf_m_kernel<<<blocks_for(L), kThreads, 0, st>>>(ma);
     c.launches++;
     CK(cudaGetLastError());
     {
@@ -438,6 +452,19 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         CK(cudaGetLastError());
     }
     c.stage_end(tk_kkt, 64 * L);
+    uint64_t S_global = 0;
+    if (c.comm) {
+        uint64_t *r7 = c.scalars->red7;
+        CK(cudaMemcpyAsync(r7, &c.scalars->total_m, sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemsetAsync(r7 + 1, 0, sizeof(uint64_t), st));
+        CK(cudaMemcpyAsync(r7 + 1, &c.scalars->limit_err, sizeof(uint32_t), cudaMemcpyDeviceToDevice, st));
+        CKS(dist_allreduce_u64(c, r7, 2));
+        uint64_t h2[2];
+        CK(cudaMemcpyAsync(h2, r7, sizeof(h2), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        if (h2[1] || h2[0] >= (1ull << 32)) return STEM_E_LIMIT;
+        S_global = h2[0];
+    }
     DevScalars hs;
     CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -448,14 +475,15 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     c.n_samples = S;
     c.T = T;
     c.stats.ssum = o.scope == 0 ? hs.ssum : 0.0;
+    c.n_samples_global = c.comm ? S_global : S;
 
     // a7: samples
     CKS(c.ensure(c.out_row, c.cap_out_row, sizeof(uint32_t) * (S + 1)));
     CKS(c.ensure(c.out_cluster, c.cap_out_cluster, sizeof(uint32_t) * (S + 1)));
     CKS(c.ensure(c.out_weight, c.cap_out_weight, sizeof(double) * (S + 1)));
     SampleArgs sa{c.leaf_lo, leaf_kid, leaf_ord, c.leaf_moff, c.leaf_m, c.leaf_census, c.t_sorted, c.row_sorted,
-                  L, n, S, (uint32_t)o.seed, (uint32_t)(o.seed >> 32), c.out_row, c.out_cluster, c.out_weight,
-                  c.leaf_U};
+                  L, n, S, (uint32_t)o.seed, (uint32_t)(o.seed >> 32), c.kid_base, c.out_row, c.out_cluster,
+                  c.out_weight, c.leaf_U};
     const int tk_smp = c.stage_begin("samples");
     if (S) sample_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa);
     c.launches += S ? 1 : 0;
@@ -471,10 +499,14 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CK(cudaMemsetAsync(&c.scalars->sum_q, 0, sizeof(uint64_t), st));
     const int tk_est = c.stage_begin("estimate");
     EstArgs ea{c.leaf_lo, c.t_sorted, c.PS1, c.PS2, c.leaf_m, c.leaf_U, L, n, &c.scalars->sum_q, part_est};
-    estimate_kernel<<<(unsigned)eb, kThreads, 0, st>>>(ea);
+    if (eb) estimate_kernel<<<(unsigned)eb, kThreads, 0, st>>>(ea);
     reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_est, eb, 2, red_out);
     c.launches += 2;
-    if (nm && S) {
+    if (c.comm) {
+        CKS(dist_allreduce_u64(c, &c.scalars->sum_q, 1));
+        CKS(dist_allreduce_f64(c, red_out, 2));
+        if (nm) CKS(dist_metric_sums(c, metrics, nm, S, red_out + 2));
+    } else if (nm && S) {
         MetArgs ma2{c.out_row, c.out_weight, metrics, n, S, nm, part_met};
         metric_kernel<<<(unsigned)mb, kThreads, 0, st>>>(ma2);
         reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_met, mb, nm, red_out + 2);
@@ -484,8 +516,8 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     // a5 output records
     CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
     const int tk_pack = c.stage_begin("pack");
-    pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.PS1, c.PS2, c.t_sorted, c.leaf_m,
-                                                   c.leaf_census, L, n, c.out_clusters);
+    if (L) pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.PS1, c.PS2, c.t_sorted, c.leaf_m,
+                                                   c.leaf_census, L, n, c.kid_base, c.out_clusters);
     c.launches++;
     c.stage_end(tk_pack, 88 * L);
     CK(cudaGetLastError());
@@ -498,7 +530,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CK(cudaStreamSynchronize(st));
     c.est_total = red[2 + nm];
     c.bound = red[2 + nm + 1];
-    for (uint32_t k = 0; k < nm; k++) c.host_est_metric[k] = S ? red[2 + k] : 0.0;
+    for (uint32_t k = 0; k < nm; k++) c.host_est_metric[k] = (S || c.comm) ? red[2 + k] : 0.0;
     c.stats.n_clusters = L;
     c.stats.n_samples = S;
     return STEM_OK;

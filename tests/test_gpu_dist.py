@@ -1,0 +1,118 @@
+"""Multi-GPU path on one B200: world ranks emulated by threads
+sharing cuda:0 through the loopback communicator (the same C++ SPMD code the
+NCCL communicator drives), and a real one-rank NCCL communicator.  The
+gathered plan must equal the single-GPU plan: integers bit-exact, fp64 sums
+within 1e-9 relative (their summation order depends on the rank count)."""
+import threading
+
+import numpy as np
+import pytest
+
+import oracle as O
+import tracegen as G
+from parity_util import Z95, assert_plans_equal
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def sr():
+    import paper_conf_micro_chungnkk25_b200 as m
+    m.build()
+    return m
+
+
+def _dist_plan(sr, kid, t, K, world, metrics=None, **kw):
+    import torch
+    n = len(kid)
+    cuts = [n * r // world for r in range(world + 1)]
+    comms = sr.Comm.loopback(world, 0)
+    ctxs = [sr.Context(0) for _ in range(world)]
+    streams = [torch.cuda.Stream() for _ in range(world)]
+    shards = []
+    for r in range(world):
+        a, b = cuts[r], cuts[r + 1]
+        dk = torch.from_numpy(np.ascontiguousarray(kid[a:b]).view(np.int32)).cuda()
+        dt = torch.from_numpy(np.ascontiguousarray(t[a:b]).view(np.int32)).cuda()
+        dm = None if metrics is None else torch.from_numpy(np.ascontiguousarray(metrics[:, a:b])).cuda()
+        shards.append((dk, dt, dm))
+    torch.cuda.synchronize()
+    out, err = [None] * world, [None] * world
+
+    def run(r):
+        try:
+            dk, dt, dm = shards[r]
+            out[r] = ctxs[r].plan_dist(comms[r], dk, dt, K, cuts[r], metrics=dm, stream=streams[r].cuda_stream,
+                                       **kw)
+        except Exception as e:  # noqa: BLE001
+            err[r] = e
+    th = [threading.Thread(target=run, args=(r,)) for r in range(world)]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join(timeout=600)
+    for e in err:
+        if e is not None:
+            raise e
+    assert all(o is None for o in out[1:])
+    for c in ctxs:
+        c.close()
+    for c in comms:
+        c.close()
+    return out[0]
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4])
+def test_loopback_matches_single_gpu(sr, world):
+    sp = G.spec("C2", n=300_000)
+    kid, t, _ = G.generate_np(sp)
+    ref = O.plan(kid, t, sp.n_kernels, eps=0.05, z=Z95, seed=5)
+    got = _dist_plan(sr, kid, t, sp.n_kernels, world, eps=0.05, z=Z95, seed=5)
+    assert_plans_equal(got, ref)
+
+
+@pytest.mark.parametrize("opts", [dict(scope=1), dict(scope=2), dict(root=False), dict(census_cap=True, eps=0.003)])
+def test_loopback_options(sr, opts):
+    rng = np.random.default_rng(3)
+    n, K = 80_000, 37
+    kid = (rng.zipf(1.3, n) % K).astype(np.uint32)
+    t = (rng.integers(1, 5, K)[kid] * 10000 * rng.lognormal(0, 0.2, n)).astype(np.uint32)
+    kw = dict(z=Z95, seed=9)
+    kw.update(opts)
+    eps = kw.pop("eps", 0.05)
+    ref = O.plan(kid, t, K, eps=eps, **kw)
+    got = _dist_plan(sr, kid, t, K, 3, eps=eps, **kw)
+    assert_plans_equal(got, ref)
+
+
+def test_loopback_metrics_and_empty_ranks(sr):
+    sp = G.spec("C3", n=200_000)
+    kid, t, met = G.generate_np(sp)
+    ref = O.plan(kid, t, sp.n_kernels, eps=0.05, z=Z95, seed=1, metrics=met)
+    got = _dist_plan(sr, kid, t, sp.n_kernels, 4, metrics=met, eps=0.05, z=Z95, seed=1)
+    assert_plans_equal(got, ref, metrics=True)
+    # a single kernel: ranks 1.. own no kernels and receive no rows
+    kid1 = np.zeros(5000, np.uint32)
+    t1 = (np.arange(5000) % 7 * 1000 + 5).astype(np.uint32)
+    ref = O.plan(kid1, t1, 1, z=Z95)
+    got = _dist_plan(sr, kid1, t1, 1, 3, z=Z95)
+    assert_plans_equal(got, ref)
+
+
+def test_nccl_single_rank(sr):
+    import torch
+    sp = G.spec("C1")
+    kid, t, _ = G.generate_np(sp)
+    try:
+        uid = sr.nccl_unique_id()
+    except sr.StemError as e:
+        pytest.skip(f"NCCL unavailable: {e}")
+    comm = sr.Comm.nccl(uid, 0, 1, 0)
+    ctx = sr.Context(0)
+    dk = torch.from_numpy(kid.view(np.int32)).cuda()
+    dt = torch.from_numpy(t.view(np.int32)).cuda()
+    got = ctx.plan_dist(comm, dk, dt, sp.n_kernels, 0, z=Z95, seed=2)
+    ref = O.plan(kid, t, sp.n_kernels, z=Z95, seed=2)
+    assert_plans_equal(got, ref)
+    ctx.close()
+    comm.close()
