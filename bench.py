@@ -142,7 +142,7 @@ def run_reference(a):
     value = m * len(times) / tot
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
-        "ms_per_step": 1e3 * tot / len(times), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "ms_per_step": 1e3 * tot / len(times), "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
         "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded)",
         "impl": "reference",
         "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n, "kernels": sp.n_kernels,
@@ -308,7 +308,7 @@ def run_ours(a):
         d2h = 0 if p is None else p["clusters"].nbytes + p["sample_row"].nbytes + p["sample_cluster"].nbytes + \
             p["sample_weight"].nbytes + 8 * (6 + nm)
         line["e2e"] = {"value": sp.n / e2e_s, "unit": UNIT,
-                       "h2d_bytes_per_step": n_local * (8 + 8 * nm), "d2h_bytes_per_step": int(d2h),
+                       "h2d_bytes_per_step": sp.n * (8 + 8 * nm), "d2h_bytes_per_step": int(d2h),
                        "ms_per_step": e2e_s * 1e3, "steps": e2e_steps}
         del hk, ht, hm
 
