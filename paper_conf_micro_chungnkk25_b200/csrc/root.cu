@@ -125,9 +125,10 @@ __global__ void tile_map_kernel(const uint32_t *__restrict__ aoff, uint32_t C, u
     else gen_list[atomicAdd(&counts[1], 1u)] = (uint32_t)j;
 }
 
-// Evaluate the valid cut k (t[k-1] < t[k]) with its exact D = n S_L - S k <= 0.
-__device__ __forceinline__ void eval_cut(i128 D, uint32_t k, uint64_t n, uint64_t SL, Cand &best) {
-    const u128 ad = (u128)(-D);
+// Evaluate the valid cut k (t[k-1] < t[k]): |D| = S k - n S_L (D <= 0 for sorted
+// data) computed exactly here, only at distinct-value boundaries.
+__device__ __forceinline__ void eval_cut(uint32_t k, uint64_t n, uint64_t S, uint64_t SL, Cand &best) {
+    const u128 ad = (u128)S * k - (u128)n * SL;
     const uint32_t dhi = (uint32_t)(ad >> 64);
     const uint64_t dlo = (uint64_t)ad;
     const double dD = approx_d(dhi, dlo);
@@ -314,7 +315,6 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
         uint64_t n = s_n[ci], S = s_S[ci], ao = s_ao[ci];
         uint32_t k = (uint32_t)(ts + p0 - ao);
         uint64_t SL = excl - s_base[ci];
-        i128 D = (i128)((u128)n * SL) - (i128)((u128)S * k);
         int seg_start = p0;
         Cand best = no_cand();
         auto flush = [&](int seg_end) {
@@ -338,13 +338,11 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
                 ao = s_ao[ci];
                 k = 0;
                 SL = 0;
-                D = 0;
                 seg_start = p;
                 best = no_cand();
             }
             const uint32_t tc = s_t[padx(p + 1)];
-            if (k >= 1 && tprev < tc) eval_cut(D, k, n, SL, best);   // cut between distinct values only
-            D += (i128)(uint64_t)(n * tc) - (i128)S;         // D_{k+1} = D_k + n t_k - S
+            if (k >= 1 && tprev < tc) eval_cut(k, n, S, SL, best);   // cut between distinct values only
             SL += tc;
             k++;
             tprev = tc;
@@ -426,7 +424,7 @@ __device__ __forceinline__ Cand shfl_cand_xor(const Cand &a, int m) {
     return r;
 }
 
-__global__ void __launch_bounds__(kSplitThreads) split_fast_kernel(SplitArgs a) {
+__global__ void __launch_bounds__(kSplitThreads, 4) split_fast_kernel(SplitArgs a) {
     __shared__ FastSmem sm;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const uint32_t tile = a.list[blockIdx.x];
@@ -454,15 +452,16 @@ __global__ void __launch_bounds__(kSplitThreads) split_fast_kernel(SplitArgs a) 
     if (p0 < nt) {
         uint64_t SL = sm.carry + excl;
         uint32_t k = (uint32_t)(ts - ao + p0);
-        i128 D = (i128)((u128)n * SL) - (i128)((u128)S * k);
         uint32_t tprev = sm.t[padx(p0)];
-        for (int p = p0; p < pend; p++) {
-            const uint32_t tc = sm.t[padx(p + 1)];
-            if (k >= 1 && tprev < tc) eval_cut(D, k, n, SL, best);
-            D += (i128)(uint64_t)(n * tc) - (i128)S;
-            SL += tc;
-            k++;
-            tprev = tc;
+#pragma unroll
+        for (int j = 0; j < kSplitItems; j++) {
+            if (p0 + j < pend) {
+                const uint32_t tc = sm.t[padx(p0 + j + 1)];
+                if (k >= 1 && tprev < tc) eval_cut(k, n, S, SL, best);
+                SL += tc;
+                k++;
+                tprev = tc;
+            }
         }
     }
 #pragma unroll
