@@ -254,6 +254,252 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : 3)) onesweep_kernel(PassA
     }
 }
 
+// ---------------------------------------------------------------- persistent TMA pass
+// Same algorithm as onesweep_kernel, but persistent blocks with two smem tile
+// buffers: while tile i is ranked, looked back and scattered, the Tensor Memory
+// Accelerator (cp.async.bulk) streams tile i+1 into the other buffer.  The
+// buffer of tile i doubles as the scatter staging area once its keys sit in
+// registers.
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase) {
+    asm volatile(
+        "{\n .reg .pred p;\n WAIT_%=:\n"
+        " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(phase)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+constexpr int kTmaThreads = 512, kTmaItems = 8, kTmaTile = kTmaThreads * kTmaItems;   // 4096 keys
+
+// The TMA part of a tile covers its first (cnt & ~3) elements (whole 16-byte
+// units, never past the end of an array); the <= 3 tail elements are read
+// directly from global memory.
+__device__ __forceinline__ uint64_t tma_elems(const PassArgs &a, uint32_t tile) {
+    const uint64_t start = (uint64_t)tile * kTmaTile;
+    return min((uint64_t)kTmaTile, a.n - start) & ~3ull;
+}
+
+template <bool FIRST>
+__device__ __forceinline__ void tma_issue(const PassArgs &a, uint32_t tile, unsigned char *buf, uint64_t *bar) {
+    const uint64_t start = (uint64_t)tile * kTmaTile;
+    const uint32_t e = (uint32_t)tma_elems(a, tile);
+    if (FIRST) {
+        mbar_expect_tx(bar, 8 * e);
+        if (e) {
+            tma_load(buf, a.kid_in + start, 4 * e, bar);
+            tma_load(buf + kTmaTile * 8, a.t_in + start, 4 * e, bar);
+        }
+    } else {
+        mbar_expect_tx(bar, 12 * e);
+        if (e) {
+            tma_load(buf, a.keys_in + start, 8 * e, bar);
+            tma_load(buf + kTmaTile * 8, a.vals_in + start, 4 * e, bar);
+        }
+    }
+}
+
+template <bool FIRST, bool LAST>
+__global__ void __launch_bounds__(kTmaThreads, 2) onesweep_tma_kernel(PassArgs a, uint32_t ntiles) {
+    constexpr int NT = kTmaThreads, IT = kTmaItems, TILE = kTmaTile, NW = NT / 32;
+    constexpr int BUF = TILE * 12;                      // keys (8 B) then vals (4 B); FIRST: kid, t
+    extern __shared__ __align__(128) unsigned char s_dyn[];
+    unsigned char *bufs = s_dyn;                        // [2][BUF]
+    uint16_t (*s_whist)[kRadix] = reinterpret_cast<uint16_t (*)[kRadix]>(s_dyn + 2 * BUF);
+    __shared__ __align__(8) uint64_t s_bar[2];
+    __shared__ uint64_t s_delta[kRadix];
+    __shared__ uint32_t s_lstart[kRadix + 1];
+    __shared__ uint64_t s_gw[8];
+    __shared__ uint32_t s_cw[8];
+    __shared__ uint32_t s_next;
+
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint64_t tmask = (a.tbits >= 64) ? ~0ull : ((1ull << a.tbits) - 1);
+    if (tid == 0) {
+        mbar_init(&s_bar[0], 1);
+        mbar_init(&s_bar[1], 1);
+        fence_async_smem();
+        s_next = atomicAdd(a.tile_counter, 1u);
+    }
+    __syncthreads();
+    uint32_t tile = s_next;
+    if (tile >= ntiles) return;
+    if (tid == 0) tma_issue<FIRST>(a, tile, bufs, &s_bar[0]);
+    uint32_t phase[2] = {0, 0};
+    int cur = 0;
+    while (true) {
+        unsigned char *buf = bufs + cur * BUF;
+        for (int i = tid; i < NW * kRadix / 2; i += NT) reinterpret_cast<uint32_t *>(&s_whist[0][0])[i] = 0;
+        mbar_wait(&s_bar[cur], phase[cur]);
+        phase[cur] ^= 1;
+        // keys of this tile into registers (warp-striped)
+        const uint64_t tbase = (uint64_t)tile * TILE;
+        const uint64_t te = tma_elems(a, tile);
+        const int wb = w * 32 * IT;
+        uint64_t key[IT];
+        uint32_t val[IT];
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const int li = wb + j * 32 + lane;
+            const uint64_t i = tbase + li;
+            if (i < a.n) {
+                const bool sm = (uint64_t)li < te;
+                if (FIRST) {
+                    const uint32_t kk = sm ? reinterpret_cast<const uint32_t *>(buf)[li] : __ldg(a.kid_in + i);
+                    const uint32_t tv = sm ? reinterpret_cast<const uint32_t *>(buf + TILE * 8)[li] : __ldg(a.t_in + i);
+                    key[j] = ((uint64_t)kk << a.tbits) | tv;
+                    val[j] = a.row_in ? __ldg(a.row_in + i) : (uint32_t)i;
+                } else {
+                    key[j] = sm ? reinterpret_cast<const uint64_t *>(buf)[li] : a.keys_in[i];
+                    val[j] = sm ? reinterpret_cast<const uint32_t *>(buf + TILE * 8)[li] : a.vals_in[i];
+                }
+            } else {
+                key[j] = ~0ull;
+                val[j] = 0;
+            }
+        }
+        __syncthreads();   // buffer `cur` is free (becomes the staging area); whist zeroed
+        // prefetch the next tile into the other buffer
+        if (tid == 0) {
+            s_next = atomicAdd(a.tile_counter, 1u);
+            if (s_next < ntiles) {
+                fence_async_smem();
+                tma_issue<FIRST>(a, s_next, bufs + (cur ^ 1) * BUF, &s_bar[cur ^ 1]);
+            }
+        }
+        // warp-level multi-split ranking
+        uint32_t rank[IT];
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = tbase + wb + j * 32 + lane;
+            const bool valid = i < a.n;
+            const uint32_t vmask = __ballot_sync(0xffffffffu, valid);
+            if (valid) {
+                const uint32_t d = (uint32_t)(key[j] >> a.shift) & 0xFF;
+                const uint32_t peers = __match_any_sync(vmask, d);
+                const uint32_t base = s_whist[w][d];
+                const uint32_t below = __popc(peers & ((1u << lane) - 1));
+                rank[j] = base + below;
+                __syncwarp(vmask);
+                if (below == 0) s_whist[w][d] = (uint16_t)(base + __popc(peers));
+            }
+            __syncwarp();
+        }
+        __syncthreads();
+        const int d = tid;
+        uint32_t cnt = 0, c_incl = 0;
+        uint64_t excl = 0, gcount = 0, g_incl = 0;
+        if (d < kRadix) {
+#pragma unroll
+            for (int ww = 0; ww < NW; ww++) {
+                const uint32_t c = s_whist[ww][d];
+                s_whist[ww][d] = (uint16_t)cnt;
+                cnt += c;
+            }
+            uint64_t *st = a.status + (uint64_t)tile * kRadix + d;
+            if (tile == 0) {
+                __stcg(st, kFlagP | cnt);
+            } else {
+                __stcg(st, kFlagA | cnt);
+                int64_t j = (int64_t)tile - 1;
+                while (true) {
+                    const uint64_t sv = *(volatile uint64_t *)(a.status + (uint64_t)j * kRadix + d);
+                    if (sv & kFlagP) { excl += sv & kValMask; break; }
+                    if (sv & kFlagA) { excl += sv & kValMask; j--; }
+                }
+                __stcg(st, kFlagP | (excl + cnt));
+            }
+            gcount = a.hist[(a.shift / 8) * kRadix + d];
+            g_incl = gcount;
+            c_incl = cnt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint64_t gv = __shfl_up_sync(0xffffffffu, g_incl, o);
+                const uint32_t cv = __shfl_up_sync(0xffffffffu, c_incl, o);
+                if (lane >= o) { g_incl += gv; c_incl += cv; }
+            }
+            if (lane == 31) { s_gw[w] = g_incl; s_cw[w] = c_incl; }
+        }
+        __syncthreads();
+        if (d < kRadix) {
+            uint64_t goff = 0;
+            uint32_t coff = 0;
+            for (int ww = 0; ww < w; ww++) { goff += s_gw[ww]; coff += s_cw[ww]; }
+            const uint64_t g_excl = goff + g_incl - gcount;
+            const uint32_t c_excl = coff + c_incl - cnt;
+            s_lstart[d] = c_excl;
+            s_delta[d] = g_excl + excl - c_excl;
+            if (d == kRadix - 1) s_lstart[kRadix] = c_excl + cnt;
+        }
+        __syncthreads();
+        uint64_t *s_keys = reinterpret_cast<uint64_t *>(buf);
+        uint32_t *s_vals = reinterpret_cast<uint32_t *>(buf + TILE * 8);
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = tbase + wb + j * 32 + lane;
+            if (i < a.n) {
+                const uint32_t dd = (uint32_t)(key[j] >> a.shift) & 0xFF;
+                const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + rank[j];
+                s_keys[lp] = key[j];
+                s_vals[lp] = val[j];
+            }
+        }
+        __syncthreads();
+        const uint32_t nvalid = s_lstart[kRadix];
+#pragma unroll 4
+        for (uint32_t i = tid; i < nvalid; i += NT) {
+            const uint64_t k = s_keys[i];
+            const uint32_t dd = (uint32_t)(k >> a.shift) & 0xFF;
+            const uint64_t gp = s_delta[dd] + i;
+            if (LAST) {
+                __stcs(a.t_out + gp, (uint32_t)(k & tmask));
+                __stcs(a.row_out + gp, s_vals[i]);
+            } else {
+                __stcs(a.keys_out + gp, k);
+                __stcs(a.vals_out + gp, s_vals[i]);
+            }
+        }
+        const uint32_t nxt = s_next;
+        __syncthreads();   // staging reads done before this buffer is refilled next round
+        if (nxt >= ntiles) break;
+        tile = nxt;
+        cur ^= 1;
+    }
+}
+
+template <bool FIRST, bool LAST>
+static int launch_tma(const PassArgs &a, int sms, cudaStream_t st) {
+    const uint32_t ntiles = (uint32_t)((a.n + kTmaTile - 1) / kTmaTile);
+    const size_t smem = 2 * (size_t)kTmaTile * 12 + sizeof(uint16_t) * kRadix * (kTmaThreads / 32);
+    CK(cudaFuncSetAttribute(onesweep_tma_kernel<FIRST, LAST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)smem));
+    CK(cudaFuncSetAttribute(onesweep_tma_kernel<FIRST, LAST>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+    const uint32_t grid = min(ntiles, (uint32_t)sms * 2);
+    onesweep_tma_kernel<FIRST, LAST><<<grid, kTmaThreads, smem, st>>>(a, ntiles);
+    return STEM_OK;
+}
+
+static int tma_sort_pass(const PassArgs &a, bool first, bool last, int sms, cudaStream_t st) {
+    if (first && last) return launch_tma<true, true>(a, sms, st);
+    if (first) return launch_tma<true, false>(a, sms, st);
+    if (last) return launch_tma<false, true>(a, sms, st);
+    return launch_tma<false, false>(a, sms, st);
+}
+
 // ---------------------------------------------------------------- reduce-then-scan pass
 // (alternative to the look-back: per-tile digit counts -> one scan -> scatter)
 template <int NT, int IT, bool FIRST>
@@ -444,7 +690,7 @@ static int sort_cfg() {
     if (cfg < 0) {
         const char *e = getenv("STEMROOT_SORT_CFG");
         cfg = e ? atoi(e) : 2;
-        if (cfg < 0 || cfg > 4) cfg = 2;
+        if (cfg < 0 || cfg > 5) cfg = 2;
     }
     return cfg;
 }
@@ -524,7 +770,8 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     c.tbits = tbits;
 
     const bool rts = sort_cfg() == 4;   // reduce-then-scan passes (no look-back)
-    const SortCfg cfg = kSortCfgs[rts ? 1 : sort_cfg()];
+    const bool tma = sort_cfg() == 5;   // persistent blocks, TMA prefetch of the next tile
+    const SortCfg cfg = kSortCfgs[(rts || tma) ? 1 : sort_cfg()];
     const uint64_t ntiles = (n + (uint64_t)cfg.nt * cfg.it - 1) / ((uint64_t)cfg.nt * cfg.it);
     CKS(c.ensure(c.sort_status, c.cap_status, ntiles * kRadix * sizeof(uint64_t)));
     PassArgs a{};
@@ -558,6 +805,9 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         const int tk = c.stage_begin(sname);
         if (rts && (!first || aligned)) {
             CKS(rts_sort_pass(c, a, first, last, st));
+        } else if (tma && (!first || aligned) &&
+                   !(first && ((reinterpret_cast<uintptr_t>(kid) | reinterpret_cast<uintptr_t>(t)) & 15))) {
+            CKS(tma_sort_pass(a, first, last, c.sms, st));
         } else {
             CKS(launch_sort_pass(a, first, last, !aligned, st));
         }
