@@ -39,7 +39,7 @@ struct DevScalars {
     uint64_t T;                   // exact total time
     uint32_t limit_err, pad1;
     uint32_t tile_counts[2];      // fast / general split tiles of the current level
-    uint32_t pad2[2];
+    uint32_t big_count, pad2;     // clusters left to fixup_big_kernel
     double ssum;                  // RN(exact sum sqrt(mu V)) (global scope)
     double g;                     // Ssum / c (global scope)
     double est_frac, var_sum;     // sum rn(r_i)/m_i, sum rn(V_i)/m_i

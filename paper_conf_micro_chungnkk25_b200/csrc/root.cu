@@ -407,6 +407,7 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
 // no cluster table, no segmentation, plain block argmax.
 struct FastSmem {
     Cand wbest[kSplitThreads / 32];
+    double thr[kSplitThreads / 32];
     uint64_t red[kSplitThreads / 32 + 1];
     uint64_t carry;
     uint32_t t[padx(kTile + 1) + 1];
@@ -448,10 +449,52 @@ __global__ void __launch_bounds__(kSplitThreads, 4) split_fast_kernel(SplitArgs 
         if (p0 + j < nt) mysum += sm.t[padx(p0 + j + 1)];
     uint64_t tot;
     const uint64_t excl = block_excl_scan<uint64_t, kSplitThreads>(mysum, sm.red, &tot);
-    Cand best = no_cand();
+    // ---- exact-safe pruning.  |D_k| is concave in k for sorted t, so over this
+    // thread's cuts k0..k0+cnt-1:  |D_k| <= |D_k0| + (k-k0) max(0, S - n t_k0),
+    // and k(n-k) >= its value at an end.  A thread whose upper bound is below the
+    // score of a real candidate of the tile cannot hold the argmax (or a tie).
+    const uint64_t SL0 = sm.carry + excl;
+    const uint32_t k0 = (uint32_t)(ts - ao + p0);
+    double ub = 0.0, lb = 0.0;
     if (p0 < nt) {
-        uint64_t SL = sm.carry + excl;
-        uint32_t k = (uint32_t)(ts - ao + p0);
+        const int cnt = pend - p0;
+        const u128 ad0 = (u128)S * k0 - (u128)n * SL0;
+        const uint64_t nt0 = n * (uint64_t)sm.t[padx(p0 + 1)];
+        const double slope = S > nt0 ? __ull2double_rn(S - nt0) : 0.0;
+        const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
+        const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad0 >> 64), (uint64_t)ad0),
+                                               __dmul_rn(slope, (double)(cnt - 1))), up);
+        const uint64_t kf = max((uint64_t)k0, (uint64_t)1), kl = min((uint64_t)k0 + cnt - 1, n - 1);
+        if (kf <= kl) {
+            const double pmin = fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
+            ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
+        }
+        // one real candidate: the thread's first valid cut
+        uint64_t SLj = SL0;
+        uint32_t tprev = sm.t[padx(p0)];
+        for (int j = 0; j < cnt; j++) {
+            const uint32_t tc = sm.t[padx(p0 + j + 1)];
+            const uint32_t k = k0 + j;
+            if (k >= 1 && tprev < tc) {
+                const u128 ad = (u128)S * k - (u128)n * SLj;
+                const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
+                lb = __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)k, (double)(n - k))), dn);
+                break;
+            }
+            SLj += tc;
+            tprev = tc;
+        }
+    }
+    double thr = lb;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) thr = fmax(thr, __shfl_xor_sync(0xffffffffu, thr, o));
+    if (lane == 0) sm.thr[w] = thr;
+    __syncthreads();
+    for (int ww = 0; ww < kSplitThreads / 32; ww++) thr = fmax(thr, sm.thr[ww]);
+    Cand best = no_cand();
+    if (p0 < nt && ub >= thr) {
+        uint64_t SL = SL0;
+        uint32_t k = k0;
         uint32_t tprev = sm.t[padx(p0)];
 #pragma unroll
         for (int j = 0; j < kSplitItems; j++) {
@@ -495,15 +538,24 @@ __device__ __forceinline__ Cand shfl_cand(const Cand &a, int src) {
     return r;
 }
 
+// One warp per cluster spanning several tiles: argmax of its tile partials.
+// Clusters spanning more than kBigSpan tiles are left to fixup_big_kernel.
+constexpr uint64_t kBigSpan = 2048;
+
 __global__ void __launch_bounds__(256)
 fixup_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, const uint32_t *__restrict__ aoff,
-             uint32_t C, const Part *__restrict__ part, uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
+             uint32_t C, const Part *__restrict__ part, uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL,
+             uint32_t *__restrict__ big_list, uint32_t *__restrict__ big_count) {
     const uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (c >= C) return;
     const uint64_t ao = aoff[c], ae = ao + (f_hi[c] - f_lo[c]);
     const uint64_t j0 = ao / kTile, j1 = (ae - 1) / kTile;
     if (j0 == j1) return;
+    if (j1 - j0 > kBigSpan) {
+        if (lane == 0) big_list[atomicAdd(big_count, 1u)] = (uint32_t)c;
+        return;
+    }
     Cand best = no_cand();
     for (uint64_t j = j0 + lane; j <= j1; j += 32) {
         const int slot = (j == j0 && ao != j0 * kTile) ? 1 : 0;
@@ -516,6 +568,38 @@ fixup_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_h
         if (better(v, best)) best = v;
     }
     if (lane == 0) {
+        cut[c] = best.k;
+        cut_SL[c] = best.SL;
+    }
+}
+
+// one block per very large cluster
+__global__ void __launch_bounds__(256)
+fixup_big_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
+                 const uint32_t *__restrict__ aoff, const Part *__restrict__ part, const uint32_t *__restrict__ big_list,
+                 const uint32_t *__restrict__ big_count, uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
+    __shared__ Cand s_w[8];
+    if (blockIdx.x >= *big_count) return;
+    const uint32_t c = big_list[blockIdx.x];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const uint64_t ao = aoff[c], ae = ao + (f_hi[c] - f_lo[c]);
+    const uint64_t j0 = ao / kTile, j1 = (ae - 1) / kTile;
+    Cand best = no_cand();
+    for (uint64_t j = j0 + threadIdx.x; j <= j1; j += blockDim.x) {
+        const int slot = (j == j0 && ao != j0 * kTile) ? 1 : 0;
+        const Cand v = part[2 * j + slot].cand;
+        if (better(v, best)) best = v;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const Cand v = shfl_cand(best, lane ^ o);
+        if (better(v, best)) best = v;
+    }
+    if (lane == 0) s_w[w] = best;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int k = 1; k < 8; k++)
+            if (better(s_w[k], best)) best = s_w[k];
         cut[c] = best.k;
         cut_SL[c] = best.SL;
     }
@@ -670,7 +754,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CKS(c.ensure(c.cut_QL, c.cap_cut_QL, sizeof(u128) * C));
         CKS(c.ensure(c.cnt_sz, c.cap_cntsz, sizeof(uint64_t) * C));
         CKS(c.ensure(c.split_part, c.cap_part, sizeof(Part) * 2 * ntiles));
-        CKS(c.ensure(c.tile_map, c.cap_tile_map, sizeof(uint32_t) * 4 * ntiles));
+        CKS(c.ensure(c.tile_map, c.cap_tile_map, sizeof(uint32_t) * (4 * ntiles + 1024)));
         CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(C) + 1) * sizeof(uint64_t)));
         const int nxt = cur ^ 1;
         CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
@@ -692,10 +776,15 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             CK(cudaFuncSetAttribute(split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SplitSmem)));
             split_kernel<<<counts[1], kSplitThreads, sizeof(SplitSmem), st>>>(sa);
         }
+        uint32_t *big_list = c.tile_map + 4 * ntiles;   // <= A / (kTile * kBigSpan) + 1 <= 513 entries
+        CK(cudaMemsetAsync(&c.scalars->big_count, 0, sizeof(uint32_t), st));
+        const uint32_t max_big = (uint32_t)(A / ((uint64_t)kTile * kBigSpan) + 1);
         fixup_kernel<<<(unsigned)((C * 32 + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur],
                                                                        (uint32_t)C, (const Part *)c.split_part, c.cut,
-                                                                       c.cut_SL);
-        c.launches += 2 + (counts[0] ? 1 : 0) + (counts[1] ? 1 : 0);
+                                                                       c.cut_SL, big_list, &c.scalars->big_count);
+        fixup_big_kernel<<<max_big, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], (const Part *)c.split_part,
+                                                   big_list, &c.scalars->big_count, c.cut, c.cut_SL);
+        c.launches += 3 + (counts[0] ? 1 : 0) + (counts[1] ? 1 : 0);
         c.stage_end(tk_s, 4 * A + 8 * ntiles + 20 * C);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");
