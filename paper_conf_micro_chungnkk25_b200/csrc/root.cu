@@ -22,7 +22,8 @@ constexpr int kSplitThreads = 256;
 constexpr int kSplitItems = 16;
 constexpr int kTile = kSplitThreads * kSplitItems;      // 4096 active rows
 constexpr int kMaxTileClusters = kTile / 2 + 2;         // frontier clusters have >= 2 rows
-constexpr uint32_t kNone = 0xFFFFFFFFu;
+constexpr uint64_t kBig = 65536;                       // clusters this large take the chunk-bound path
+constexpr uint64_t kBigSeg = 65536;                    // rows per block on that path
 
 struct SQ {
     uint64_t s;
@@ -110,7 +111,8 @@ __device__ __forceinline__ bool nontrivial(const uint32_t *t, uint32_t lo, uint3
 
 // first/last frontier cluster of every tile; tiles inside one cluster go to
 // the fast list, the others to the general list (order is irrelevant).
-__global__ void tile_map_kernel(const uint32_t *__restrict__ aoff, uint32_t C, uint64_t A, uint64_t ntiles,
+__global__ void tile_map_kernel(const uint32_t *__restrict__ aoff, const uint32_t *__restrict__ f_lo,
+                                const uint32_t *__restrict__ f_hi, uint32_t C, uint64_t A, uint64_t ntiles,
                                 uint32_t *__restrict__ first, uint32_t *__restrict__ last,
                                 uint32_t *__restrict__ fast_list, uint32_t *__restrict__ gen_list,
                                 uint32_t *__restrict__ counts) {
@@ -121,6 +123,7 @@ __global__ void tile_map_kernel(const uint32_t *__restrict__ aoff, uint32_t C, u
     const uint32_t l = (uint32_t)upper_bound(aoff, C, (uint32_t)(te - 1)) - 1;
     first[j] = f;
     last[j] = l;
+    if (f == l && f_hi[f] - f_lo[f] >= kBig) return;   // inside a big cluster: chunk-bound path
     if (f == l) fast_list[atomicAdd(&counts[0], 1u)] = (uint32_t)j;
     else gen_list[atomicAdd(&counts[1], 1u)] = (uint32_t)j;
 }
@@ -342,7 +345,7 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
                 best = no_cand();
             }
             const uint32_t tc = s_t[padx(p + 1)];
-            if (k >= 1 && tprev < tc) eval_cut(k, n, S, SL, best);   // cut between distinct values only
+            if (k >= 1 && tprev < tc && n < kBig) eval_cut(k, n, S, SL, best);   // distinct values only
             SL += tc;
             k++;
             tprev = tc;
@@ -385,7 +388,7 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
     run_combine(cf, cv, inf, iv);
     (void)ef;
     // a head that started before this thread and ends inside it closes its run
-    if (head_ci >= 0 && head_before && out_ci != head_ci) {
+    if (head_ci >= 0 && head_before && out_ci != head_ci && s_n[head_ci] < kBig) {
         Cand fin = head_b;
         if (better(ev, fin)) fin = ev;
         const uint64_t ao = s_ao[head_ci];
@@ -397,7 +400,7 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
         }
     }
     // the run carried out of the tile's last thread continues into the next tile
-    if (p0 < nt && pend == nt && out_ci >= 0) {
+    if (p0 < nt && pend == nt && out_ci >= 0 && s_n[out_ci] < kBig) {
         const uint64_t ao = s_ao[out_ci];
         a.part[2 * (uint64_t)tile + (ao <= ts ? 0 : 1)] = Part{iv, c0 + out_ci};
     }
@@ -551,7 +554,7 @@ fixup_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_h
     if (c >= C) return;
     const uint64_t ao = aoff[c], ae = ao + (f_hi[c] - f_lo[c]);
     const uint64_t j0 = ao / kTile, j1 = (ae - 1) / kTile;
-    if (j0 == j1) return;
+    if (j0 == j1 || ae - ao >= kBig) return;
     if (j1 - j0 > kBigSpan) {
         if (lane == 0) big_list[atomicAdd(big_count, 1u)] = (uint32_t)c;
         return;
@@ -603,6 +606,176 @@ fixup_big_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__
         cut[c] = best.k;
         cut_SL[c] = best.SL;
     }
+}
+
+// ---------------------------------------------------------------- big clusters: chunk bounds
+// Clusters of >= kBig rows.  One block per kBigSeg rows.  For every 32-row chunk
+// (aligned to the sampled prefix PS1) the concavity bound of |D| gives an upper
+// bound of the chunk's scores from S_L at the chunk start (PS1, exact) and one
+// t value; a real candidate at every chunk start gives lower bounds.  Only
+// chunks whose bound reaches the best lower bound (of this block, or of the
+// whole cluster through an atomic max) are scanned row by row.  Exact: a pruned
+// chunk cannot hold a candidate scoring >= an existing one, so neither the
+// argmax nor a tie is lost.
+struct BigEntry {
+    uint32_t c, seg;
+};
+
+__global__ void big_entries_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, uint32_t C,
+                                   BigEntry *__restrict__ ent, uint32_t *__restrict__ first_ent,
+                                   uint32_t *__restrict__ count) {
+    const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= C) return;
+    const uint64_t n = f_hi[c] - f_lo[c];
+    if (n < kBig) return;
+    const uint32_t nb = (uint32_t)((n + kBigSeg - 1) / kBigSeg);
+    const uint32_t e0 = atomicAdd(count, nb);
+    for (uint32_t s = 0; s < nb; s++) ent[e0 + s] = BigEntry{(uint32_t)c, s};
+    first_ent[c] = e0;
+}
+
+struct BigArgs {
+    const BigEntry *ent;
+    const uint32_t *count;
+    const uint32_t *f_lo, *f_hi;
+    const uint64_t *f_S, *PS1;
+    const uint32_t *t;
+    unsigned long long *thr;   // per cluster: bits of the best lower bound so far
+    Cand *part;                // per entry
+};
+
+constexpr int kBigThreads = 256;
+constexpr int kBigChunks = (int)(kBigSeg / kChunk) + 2;
+
+__global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
+    __shared__ double s_ub[kBigChunks];
+    __shared__ uint64_t s_sl[kBigChunks];
+    __shared__ uint16_t s_list[kBigChunks];
+    __shared__ uint32_t s_nlist;
+    __shared__ double s_thr[kBigThreads / 32];
+    __shared__ Cand s_best[kBigThreads / 32];
+    __shared__ uint64_t s_base;
+    if (blockIdx.x >= *a.count) return;
+    const BigEntry e = a.ent[blockIdx.x];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint64_t lo = a.f_lo[e.c], hi = a.f_hi[e.c], n = hi - lo, S = a.f_S[e.c];
+    const uint64_t r0 = lo + (uint64_t)e.seg * kBigSeg, r1 = min(r0 + kBigSeg, hi);
+    if (w == 0) {   // pref1(lo) = PS1[lo/32] + partial chunk
+        uint64_t part = 0;
+        const uint64_t lb0 = lo & ~(kChunk - 1);
+        if (lb0 + lane < lo) part = a.t[lb0 + lane];
+        for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+        if (lane == 0) {
+            s_base = a.PS1[lo >> kChunkLog] + part;
+            s_nlist = 0;
+        }
+    }
+    __syncthreads();
+    const uint64_t q0 = r0 >> kChunkLog, q1 = (r1 - 1) >> kChunkLog;   // chunks touching [r0, r1)
+    const int nq = (int)(q1 - q0 + 1);
+    const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
+    double lbm = 0.0;
+    for (int i = tid; i < nq; i += kBigThreads) {
+        const uint64_t q = q0 + i;
+        const uint64_t ra = max(r0, q << kChunkLog), rb = min(r1, (q + 1) << kChunkLog);   // rows [ra, rb)
+        uint64_t pa;
+        if ((ra & (kChunk - 1)) == 0) {
+            pa = a.PS1[ra >> kChunkLog];
+        } else {   // only the block's first chunk can start unaligned
+            pa = a.PS1[ra >> kChunkLog];
+            for (uint64_t x = ra & ~(kChunk - 1); x < ra; x++) pa += a.t[x];
+        }
+        const uint64_t SL = pa - s_base;       // S_L at k_a = ra - lo (exact)
+        const uint32_t ka = (uint32_t)(ra - lo);
+        const uint32_t ta = a.t[ra];
+        s_sl[i] = SL;
+        const u128 ad = (u128)S * ka - (u128)n * SL;
+        const uint64_t nta = n * (uint64_t)ta;
+        const double slope = S > nta ? __ull2double_rn(S - nta) : 0.0;
+        const uint64_t cnt = rb - ra;
+        const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad >> 64), (uint64_t)ad),
+                                               __dmul_rn(slope, (double)(cnt - 1))), up);
+        const uint64_t kf = max((uint64_t)ka, (uint64_t)1), kl = min((uint64_t)ka + cnt - 1, n - 1);
+        double ub = 0.0;
+        if (kf <= kl) {
+            const double pmin = fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
+            ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
+        }
+        s_ub[i] = ub;
+        if (ka >= 1 && a.t[ra - 1] < ta) {      // the chunk start is a real candidate
+            const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
+            lbm = fmax(lbm, __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)ka, (double)(n - ka))), dn));
+        }
+    }
+    for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));
+    if (lane == 0) s_thr[w] = lbm;
+    __syncthreads();
+    if (tid == 0) {
+        double m = 0.0;
+        for (int k = 0; k < kBigThreads / 32; k++) m = fmax(m, s_thr[k]);
+        const unsigned long long prev = atomicMax(a.thr + e.c, (unsigned long long)__double_as_longlong(m));
+        s_thr[0] = fmax(m, __longlong_as_double((long long)prev));   // positive doubles order as integers
+    }
+    __syncthreads();
+    const double thr = s_thr[0];
+    for (int i = tid; i < nq; i += kBigThreads)
+        if (s_ub[i] >= thr && s_ub[i] > 0.0) s_list[atomicAdd(&s_nlist, 1u)] = (uint16_t)i;
+    __syncthreads();
+    // row-by-row scan of the surviving chunks: one warp per chunk, lane = row
+    Cand best = no_cand();
+    for (uint32_t li = w; li < s_nlist; li += kBigThreads / 32) {
+        const int i = s_list[li];
+        const uint64_t q = q0 + i;
+        const uint64_t ra = max(r0, q << kChunkLog), rb = min(r1, (q + 1) << kChunkLog);
+        const uint64_t row = ra + lane;
+        const bool in = row < rb;
+        const uint32_t tc = in ? a.t[row] : 0u;
+        const uint32_t tp = (in && row > lo) ? a.t[row - 1] : 0u;
+        uint64_t incl = tc;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += v;
+        }
+        const uint64_t SLr = s_sl[i] + incl - tc;
+        const uint32_t k = (uint32_t)(row - lo);
+        if (in && k >= 1 && tp < tc) eval_cut(k, n, S, SLr, best);
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const Cand v = shfl_cand_xor(best, o);
+        if (better(v, best)) best = v;
+    }
+    if (lane == 0) s_best[w] = best;
+    __syncthreads();
+    if (tid == 0) {
+        for (int k = 1; k < kBigThreads / 32; k++)
+            if (better(s_best[k], best)) best = s_best[k];
+        a.part[blockIdx.x] = best;
+    }
+}
+
+// one block per big cluster: argmax over its entries
+__global__ void big_reduce_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, uint32_t C,
+                                  const uint32_t *__restrict__ first_ent, const Cand *__restrict__ part,
+                                  uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
+  for (uint64_t c = blockIdx.x; c < C; c += gridDim.x) {
+    const uint64_t n = f_hi[c] - f_lo[c];
+    if (n < kBig) continue;
+    const uint32_t nb = (uint32_t)((n + kBigSeg - 1) / kBigSeg), e0 = first_ent[c];
+    Cand best = no_cand();
+    for (uint32_t s = threadIdx.x; s < nb; s += 32)
+        if (better(part[e0 + s], best)) best = part[e0 + s];
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const Cand v = shfl_cand_xor(best, o);
+        if (better(v, best)) best = v;
+    }
+    if (threadIdx.x == 0) {
+        cut[c] = best.k;
+        cut_SL[c] = best.SL;
+    }
+  }
 }
 
 // ---------------------------------------------------------------- a4: decide
@@ -762,9 +935,24 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         uint32_t *tfirst = c.tile_map, *tlast = c.tile_map + ntiles;
         uint32_t *fast_list = c.tile_map + 2 * ntiles, *gen_list = c.tile_map + 3 * ntiles;
         CK(cudaMemsetAsync(c.scalars->tile_counts, 0, sizeof(uint32_t) * 2, st));
-        tile_map_kernel<<<(unsigned)((ntiles + 255) / 256), 256, 0, st>>>(c.f_aoff[cur], (uint32_t)C, A, ntiles,
-                                                                          tfirst, tlast, fast_list, gen_list,
-                                                                          c.scalars->tile_counts);
+        tile_map_kernel<<<(unsigned)((ntiles + 255) / 256), 256, 0, st>>>(c.f_aoff[cur], c.f_lo[cur], c.f_hi[cur],
+                                                                          (uint32_t)C, A, ntiles, tfirst, tlast,
+                                                                          fast_list, gen_list, c.scalars->tile_counts);
+        // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
+        const uint64_t max_ent = A / kBigSeg + A / kBig + 1;
+        CKS(c.ensure(c.big_ent, c.cap_big_ent, sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (C + 1)));
+        CKS(c.ensure(c.big_part, c.cap_big_part, sizeof(Cand) * max_ent));
+        CKS(c.ensure(c.big_thr, c.cap_big_thr, sizeof(unsigned long long) * C));
+        BigEntry *ent = (BigEntry *)c.big_ent;
+        uint32_t *first_ent = (uint32_t *)(ent + max_ent);
+        CK(cudaMemsetAsync(&c.scalars->big_count, 0, sizeof(uint32_t), st));
+        CK(cudaMemsetAsync(c.big_thr, 0, sizeof(unsigned long long) * C, st));
+        big_entries_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, ent,
+                                                                       first_ent, &c.scalars->big_count);
+        BigArgs ba{ent, &c.scalars->big_count, c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.PS1, c.t_sorted,
+                   (unsigned long long *)c.big_thr, (Cand *)c.big_part};
+        big_split_kernel<<<(unsigned)max_ent, kBigThreads, 0, st>>>(ba);
+        c.launches += 2;
         uint32_t counts[2];
         CK(cudaMemcpyAsync(counts, c.scalars->tile_counts, sizeof(counts), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
@@ -777,13 +965,16 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             split_kernel<<<counts[1], kSplitThreads, sizeof(SplitSmem), st>>>(sa);
         }
         uint32_t *big_list = c.tile_map + 4 * ntiles;   // <= A / (kTile * kBigSpan) + 1 <= 513 entries
-        CK(cudaMemsetAsync(&c.scalars->big_count, 0, sizeof(uint32_t), st));
+        CK(cudaMemsetAsync(&c.scalars->big_count2, 0, sizeof(uint32_t), st));
         const uint32_t max_big = (uint32_t)(A / ((uint64_t)kTile * kBigSpan) + 1);
         fixup_kernel<<<(unsigned)((C * 32 + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur],
                                                                        (uint32_t)C, (const Part *)c.split_part, c.cut,
-                                                                       c.cut_SL, big_list, &c.scalars->big_count);
+                                                                       c.cut_SL, big_list, &c.scalars->big_count2);
         fixup_big_kernel<<<max_big, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], (const Part *)c.split_part,
-                                                   big_list, &c.scalars->big_count, c.cut, c.cut_SL);
+                                                   big_list, &c.scalars->big_count2, c.cut, c.cut_SL);
+        big_reduce_kernel<<<(unsigned)min(C, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, first_ent,
+                                                      (const Cand *)c.big_part, c.cut, c.cut_SL);
+        c.launches++;
         c.launches += 3 + (counts[0] ? 1 : 0) + (counts[1] ? 1 : 0);
         c.stage_end(tk_s, 4 * A + 8 * ntiles + 20 * C);
         CK(cudaGetLastError());

@@ -100,7 +100,7 @@ struct PassArgs {
 // (thread d < 256 owns digit d), then keys are staged in shared memory in
 // tile-sorted order and written out in digit runs (coalesced).
 template <int NT, int IT, bool FIRST, bool LAST>
-__global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : 3)) onesweep_kernel(PassArgs a) {
+__global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : NT >= 256 ? 4 : 8)) onesweep_kernel(PassArgs a) {
     constexpr int NW = NT / 32, TILE = NT * IT;
     extern __shared__ __align__(16) unsigned char s_dyn[];
     uint64_t *s_keys = reinterpret_cast<uint64_t *>(s_dyn);                          // [TILE]
@@ -683,14 +683,15 @@ static int launch_pass_cfg(const PassArgs &a, bool first, bool last, bool first_
 
 // tile configurations (threads, keys per thread); STEMROOT_SORT_CFG selects one for experiments
 struct SortCfg { int nt, it; };
-static const SortCfg kSortCfgs[] = {{256, 16}, {512, 8}, {384, 12}, {512, 12}};
+static const SortCfg kSortCfgs[] = {{256, 16}, {512, 8}, {384, 12}, {512, 12}, {512, 8}, {512, 8},
+                                    {256, 8}, {128, 16}, {256, 12}};
 
 static int sort_cfg() {
     static int cfg = -1;
     if (cfg < 0) {
         const char *e = getenv("STEMROOT_SORT_CFG");
         cfg = e ? atoi(e) : 2;
-        if (cfg < 0 || cfg > 5) cfg = 2;
+        if (cfg < 0 || cfg > 8) cfg = 2;
     }
     return cfg;
 }
@@ -700,6 +701,9 @@ static int launch_sort_pass(const PassArgs &a, bool first, bool last, bool first
         case 0: return launch_pass_cfg<256, 16>(a, first, last, first_hist, st);
         case 2: return launch_pass_cfg<384, 12>(a, first, last, first_hist, st);
         case 3: return launch_pass_cfg<512, 12>(a, first, last, first_hist, st);
+        case 6: return launch_pass_cfg<256, 8>(a, first, last, first_hist, st);
+        case 7: return launch_pass_cfg<128, 16>(a, first, last, first_hist, st);
+        case 8: return launch_pass_cfg<256, 12>(a, first, last, first_hist, st);
         default: return launch_pass_cfg<512, 8>(a, first, last, first_hist, st);
     }
 }

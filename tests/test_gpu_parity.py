@@ -239,3 +239,23 @@ def test_config_c5_full_size_sampled(ctx):
         mine = cl[cl["kernel_id"] == k]
         for f in ("ordinal", "lo_ns", "hi_ns", "n", "sum_ns"):
             assert np.array_equal(mine[f].astype(np.int64), ref[f].astype(np.int64)), (k, f)
+
+
+# ------------------------------------------------------------------ big clusters (chunk-bound path, >= 65536 rows)
+BIG = {
+    "distinct_ramp": lambda: np.arange(300_000, dtype=np.uint32) * 7 + 1000,
+    "two_values_outlier": lambda: np.r_[np.full(150_000, 5), np.full(120_000, 6), [4000]].astype(np.uint32),
+    "symmetric_tie": lambda: np.r_[np.full(70_000, 0), np.full(90_000, 10), np.full(70_000, 20)].astype(np.uint32),
+    "lognormal_wide": lambda: (np.random.default_rng(3).lognormal(12, 1.1, 500_000)).astype(np.uint32),
+    "near_constant": lambda: (3_000_000_000 + np.random.default_rng(4).integers(0, 3, 200_000)).astype(np.uint32),
+}
+
+
+@pytest.mark.parametrize("name", sorted(BIG))
+def test_big_clusters(ctx, name):
+    t = BIG[name]()
+    rng = np.random.default_rng(len(t))
+    perm = rng.permutation(len(t))
+    kid = np.zeros(len(t), np.uint32)
+    got, ref = _both(ctx, kid, t[perm], 1, eps=0.02, seed=4)
+    assert_plans_equal(got, ref)
