@@ -112,10 +112,12 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : NT >= 256
     __shared__ uint64_t s_gw[8];
     __shared__ uint32_t s_cw[8];
     __shared__ uint32_t s_tile;
+    __shared__ uint32_t s_cnt[kRadix];
 
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     if (tid == 0) s_tile = atomicAdd(a.tile_counter, 1u);
     for (int i = tid; i < NW * kRadix / 2; i += NT) reinterpret_cast<uint32_t *>(&s_whist[0][0])[i] = 0;
+    for (int i = tid; i < kRadix; i += NT) s_cnt[i] = 0;
     if (FIRST && a.first_hist)
         for (int i = tid; i < 7 * kRadix; i += NT) (&s_hlater[0][0])[i] = 0;
     __syncthreads();
@@ -151,6 +153,14 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : NT >= 256
         }
     }
 
+    // tile digit counts first, published at once (flag A) so that successors'
+    // look-backs do not wait for this tile's ranking
+#pragma unroll
+    for (int j = 0; j < IT; j++)
+        if (wbase + (uint64_t)j * 32 + lane < a.n) atomicAdd(&s_cnt[(uint32_t)(key[j] >> a.shift) & 0xFF], 1u);
+    __syncthreads();
+    if (tid < kRadix) __stcg(a.status + (uint64_t)tile * kRadix + tid, (tile == 0 ? kFlagP : kFlagA) | s_cnt[tid]);
+
     // warp-level multi-split ranking, in element order
     uint32_t rank[IT];
 #pragma unroll
@@ -184,10 +194,7 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : NT >= 256
             cnt += c;
         }
         uint64_t *st = a.status + (uint64_t)tile * kRadix + d;
-        if (tile == 0) {
-            __stcg(st, kFlagP | cnt);
-        } else {
-            __stcg(st, kFlagA | cnt);
+        if (tile != 0) {
             int64_t j = (int64_t)tile - 1;
             while (true) {
                 const uint64_t sv = *(volatile uint64_t *)(a.status + (uint64_t)j * kRadix + d);
