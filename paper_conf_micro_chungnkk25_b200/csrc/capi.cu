@@ -25,7 +25,7 @@ int Ctx::ensure_all(uint64_t n, uint32_t K, uint32_t n_metrics) {
     CKS(ensure(row_sorted, cap_rs, sizeof(uint32_t) * (n + 1)));
     CKS(ensure(kid_count, cap_kc, sizeof(uint32_t) * ((uint64_t)K + 1)));
     CKS(ensure(goff, cap_goff, sizeof(uint32_t) * ((uint64_t)K + 2)));
-    CKS(ensure(hist, cap_hist, sizeof(uint64_t) * 12 * 256));
+    CKS(ensure(hist, cap_hist, sizeof(uint64_t) * 12 * 512));
     CKS(ensure(scalars, cap_scalars, sizeof(DevScalars)));
     CKS(ensure(scan_scratch, cap_scan, (scan_tiles((uint64_t)K + 2) + 1) * 32));
     CKS(ensure(PS1, cap_ps1, sizeof(uint64_t) * (n / kChunk + 2)));

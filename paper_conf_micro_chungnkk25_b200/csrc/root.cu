@@ -14,6 +14,8 @@
 //   scan + apply     compacts the non-trivial children into the next frontier
 // Cluster totals (S exact u64, Q exact u128) travel with the frontier; only
 // Q_L at the chosen cut is read from the sampled prefix arrays.
+#include <cstdlib>
+
 #include "internal.h"
 
 namespace sr {
@@ -22,7 +24,17 @@ constexpr int kSplitThreads = 256;
 constexpr int kSplitItems = 16;
 constexpr int kTile = kSplitThreads * kSplitItems;      // 4096 active rows
 constexpr int kMaxTileClusters = kTile / 2 + 2;         // frontier clusters have >= 2 rows
-constexpr uint64_t kBig = 65536;                       // clusters this large take the chunk-bound path
+// clusters of >= big_rows() rows take the chunk-bound path (STEMROOT_BIG_ROWS overrides)
+__constant__ uint64_t c_big;
+static uint64_t big_rows() {
+    static uint64_t v = 0;
+    if (!v) {
+        const char *e = getenv("STEMROOT_BIG_ROWS");
+        v = e ? strtoull(e, nullptr, 10) : 65536;
+        if (v < 64) v = 64;
+    }
+    return v;
+}
 constexpr uint64_t kBigSeg = 65536;                    // rows per block on that path
 
 struct SQ {
@@ -123,7 +135,7 @@ __global__ void tile_map_kernel(const uint32_t *__restrict__ aoff, const uint32_
     const uint32_t l = (uint32_t)upper_bound(aoff, C, (uint32_t)(te - 1)) - 1;
     first[j] = f;
     last[j] = l;
-    if (f == l && f_hi[f] - f_lo[f] >= kBig) return;   // inside a big cluster: chunk-bound path
+    if (f == l && f_hi[f] - f_lo[f] >= c_big) return;   // inside a big cluster: chunk-bound path
     if (f == l) fast_list[atomicAdd(&counts[0], 1u)] = (uint32_t)j;
     else gen_list[atomicAdd(&counts[1], 1u)] = (uint32_t)j;
 }
@@ -345,7 +357,7 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
                 best = no_cand();
             }
             const uint32_t tc = s_t[padx(p + 1)];
-            if (k >= 1 && tprev < tc && n < kBig) eval_cut(k, n, S, SL, best);   // distinct values only
+            if (k >= 1 && tprev < tc && n < c_big) eval_cut(k, n, S, SL, best);   // distinct values only
             SL += tc;
             k++;
             tprev = tc;
@@ -388,7 +400,7 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
     run_combine(cf, cv, inf, iv);
     (void)ef;
     // a head that started before this thread and ends inside it closes its run
-    if (head_ci >= 0 && head_before && out_ci != head_ci && s_n[head_ci] < kBig) {
+    if (head_ci >= 0 && head_before && out_ci != head_ci && s_n[head_ci] < c_big) {
         Cand fin = head_b;
         if (better(ev, fin)) fin = ev;
         const uint64_t ao = s_ao[head_ci];
@@ -400,7 +412,7 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
         }
     }
     // the run carried out of the tile's last thread continues into the next tile
-    if (p0 < nt && pend == nt && out_ci >= 0 && s_n[out_ci] < kBig) {
+    if (p0 < nt && pend == nt && out_ci >= 0 && s_n[out_ci] < c_big) {
         const uint64_t ao = s_ao[out_ci];
         a.part[2 * (uint64_t)tile + (ao <= ts ? 0 : 1)] = Part{iv, c0 + out_ci};
     }
@@ -554,7 +566,7 @@ fixup_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_h
     if (c >= C) return;
     const uint64_t ao = aoff[c], ae = ao + (f_hi[c] - f_lo[c]);
     const uint64_t j0 = ao / kTile, j1 = (ae - 1) / kTile;
-    if (j0 == j1 || ae - ao >= kBig) return;
+    if (j0 == j1 || ae - ao >= c_big) return;
     if (j1 - j0 > kBigSpan) {
         if (lane == 0) big_list[atomicAdd(big_count, 1u)] = (uint32_t)c;
         return;
@@ -627,7 +639,7 @@ __global__ void big_entries_kernel(const uint32_t *__restrict__ f_lo, const uint
     const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= C) return;
     const uint64_t n = f_hi[c] - f_lo[c];
-    if (n < kBig) return;
+    if (n < c_big) return;
     const uint32_t nb = (uint32_t)((n + kBigSeg - 1) / kBigSeg);
     const uint32_t e0 = atomicAdd(count, nb);
     for (uint32_t s = 0; s < nb; s++) ent[e0 + s] = BigEntry{(uint32_t)c, s};
@@ -761,7 +773,7 @@ __global__ void big_reduce_kernel(const uint32_t *__restrict__ f_lo, const uint3
                                   uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
   for (uint64_t c = blockIdx.x; c < C; c += gridDim.x) {
     const uint64_t n = f_hi[c] - f_lo[c];
-    if (n < kBig) continue;
+    if (n < c_big) continue;
     const uint32_t nb = (uint32_t)((n + kBigSeg - 1) / kBigSeg), e0 = first_ent[c];
     Cand best = no_cand();
     for (uint32_t s = threadIdx.x; s < nb; s += 32)
@@ -880,6 +892,10 @@ static int ensure_frontier(Ctx &c, int b, uint64_t cap) {
 
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp) {
     cudaStream_t st = c.stream;
+    {
+        const uint64_t b = big_rows();
+        CK(cudaMemcpyToSymbolAsync(c_big, &b, sizeof(b), 0, cudaMemcpyHostToDevice, st));
+    }
     CKS(stem_only_leaves(c, n, K));
     // initial frontier: non-trivial kernel groups, in kernel order, with exact S and Q
     {
@@ -939,7 +955,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                                                                           (uint32_t)C, A, ntiles, tfirst, tlast,
                                                                           fast_list, gen_list, c.scalars->tile_counts);
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
-        const uint64_t max_ent = A / kBigSeg + A / kBig + 1;
+        const uint64_t max_ent = A / kBigSeg + A / big_rows() + 1;
         CKS(c.ensure(c.big_ent, c.cap_big_ent, sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (C + 1)));
         CKS(c.ensure(c.big_part, c.cap_big_part, sizeof(Cand) * max_ent));
         CKS(c.ensure(c.big_thr, c.cap_big_thr, sizeof(unsigned long long) * C));
