@@ -3,12 +3,13 @@
 // (Adinets & Merrill): every pass reads and writes the data once; tiles get
 // their global digit offsets by decoupled look-back.
 //
-// Digits are RB = 9 bits wide (512 buckets) and tbits is rounded up to a
-// multiple of RB, so every digit is a window of t or of kernel_id alone: the
-// pre-pass (one read of the trace) yields the histograms of every pass, and
-// the pass count is ceil(bits(max t)/9) + ceil(bits(K-1)/9) -- 5 for the C5
-// trace instead of 6 with bytes.  STEMROOT_SORT_RADIX=8 selects byte digits
-// (kept for comparison).
+// Digits are RB = 8 bits wide (256 buckets) and tbits is rounded up to a
+// multiple of RB, so every digit is a byte of t or of kernel_id alone: the
+// pre-pass (one read of the trace) yields the histograms of every pass; the
+// pass count is ceil(bits(max t)/8) + ceil(bits(K-1)/8) (6 for C5, whose
+// lognormal tails reach 2^32 ns).  STEMROOT_SORT_RADIX=9 selects 9-bit digits
+// (512 threads x 9 keys per tile): fewer passes on some traces, but each pass
+// measured ~20% slower on B200, so bytes are the default.
 #include <cstdlib>
 
 #include "internal.h"
@@ -24,7 +25,7 @@ static int radix_bits() {
     static int rb = 0;
     if (!rb) {
         const char *e = getenv("STEMROOT_SORT_RADIX");
-        rb = (e && atoi(e) == 8) ? 8 : 9;
+        rb = (e && atoi(e) == 9) ? 9 : 8;
     }
     return rb;
 }
