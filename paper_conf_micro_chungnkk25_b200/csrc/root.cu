@@ -769,9 +769,13 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
             ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
         }
         s_ub[i] = ub;
-        if (ka >= 1 && a.t[ra - 1] < ta) {      // the chunk start is a real candidate
-            const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
-            lbm = fmax(lbm, __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)ka, (double)(n - ka))), dn));
+        // a real candidate for the lower bound: the cut after the chunk's first row
+        // (t[ra], t[ra+1] share a sector with the value the bound already reads)
+        if (ra + 1 < rb && ta < a.t[ra + 1]) {
+            const uint32_t k1 = ka + 1;
+            const u128 ad1 = (u128)S * k1 - (u128)n * (SL + ta);
+            const double dD = approx_d((uint32_t)(ad1 >> 64), (uint64_t)ad1);
+            lbm = fmax(lbm, __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)k1, (double)(n - k1))), dn));
         }
     }
     for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));
