@@ -200,7 +200,6 @@ __host__ __device__ constexpr int padx(int i) { return i + (i >> 3); }   // conf
 
 struct SplitSmem {
     uint64_t S[kMaxTileClusters], base[kMaxTileClusters];
-    unsigned long long thr[kMaxTileClusters];  // per cluster: bits of the best lower bound in this tile
     uint64_t red[kSplitThreads / 32 + 1];
     uint64_t carry;
     Cand wtot[kSplitThreads / 32];             // per-warp inclusive (flag, best) of the run scan
@@ -252,7 +251,6 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
         s_lo[i] = lo;
         s_n[i] = a.f_hi[c] - lo;
         s_S[i] = a.f_S[c];
-        sm.thr[i] = 0ull;
     }
     for (int p = tid; p < kTile; p += kSplitThreads) s_cid[p] = 0;
     __syncthreads();
@@ -320,40 +318,6 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
     }
     __syncthreads();
 
-    // ---- exact-safe pruning (see split_fast_kernel): every thread segment posts the
-    // score of its first valid cut as a lower bound of its cluster; a segment whose
-    // concavity upper bound is below its cluster's best lower bound is skipped.
-    if (p0 < nt) {
-        int ci = -1;
-        uint64_t n = 0, S = 0, SL = 0;
-        uint32_t k = 0, tprev = s_t[padx(p0)];
-        bool found = false;
-        for (int p = p0; p < pend; p++) {
-            const int cj = s_cid[p];
-            if (cj != ci) {
-                ci = cj;
-                n = s_n[ci];
-                S = s_S[ci];
-                k = (uint32_t)(ts + p - s_ao[ci]);
-                SL = (p == p0) ? excl - s_base[ci] : 0;
-                found = false;
-            }
-            const uint32_t tc = s_t[padx(p + 1)];
-            if (!found && k >= 1 && tprev < tc && n < c_big) {
-                const u128 ad = (u128)S * k - (u128)n * SL;
-                const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
-                const double lb = __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)k, (double)(n - k))),
-                                            1.0 - 0x1p-44);
-                atomicMax(&sm.thr[ci], (unsigned long long)__double_as_longlong(lb));
-                found = true;
-            }
-            SL += tc;
-            k++;
-            tprev = tc;
-        }
-    }
-    __syncthreads();
-
     // ---- candidates: thread-local segmented argmax with exact incremental D
     int head_ci = -1;                   // first segment when incomplete
     Cand head_b = no_cand();
@@ -378,24 +342,6 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
             if (seg_start == p0) { head_ci = ci; head_b = best; head_before = before; }
             if (seg_end == pend && after) { out_ci = ci; out_v = best; out_f = before ? 0u : 1u; }
         };
-        // concavity upper bound of the segment starting at position p (cut k, prefix SL)
-        auto seg_live = [&](int p, uint32_t kk, uint64_t sl) -> bool {
-            if (n >= c_big) return false;
-            const int cnt = (int)min((uint64_t)pend, ao + n - ts) - p;
-            const u128 ad = (u128)S * kk - (u128)n * sl;
-            const uint64_t ntk = n * (uint64_t)s_t[padx(p + 1)];
-            const double slope = S > ntk ? __ull2double_rn(S - ntk) : 0.0;
-            const double up = 1.0 + 0x1p-44;
-            const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad >> 64), (uint64_t)ad),
-                                                   __dmul_rn(slope, (double)(cnt - 1))), up);
-            const uint64_t kf = max((uint64_t)kk, (uint64_t)1), kl = min((uint64_t)kk + cnt - 1, n - 1);
-            if (kf > kl) return false;
-            const double pmin =
-                fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
-            const double ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
-            return ub >= __longlong_as_double((long long)sm.thr[ci]);
-        };
-        bool live = seg_live(p0, k, SL);
         uint32_t tprev = s_t[padx(p0)];
         for (int p = p0; p < pend; p++) {
             const int cj = s_cid[p];
@@ -409,10 +355,9 @@ __global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
                 SL = 0;
                 seg_start = p;
                 best = no_cand();
-                live = seg_live(p, 0, 0);
             }
             const uint32_t tc = s_t[padx(p + 1)];
-            if (live && k >= 1 && tprev < tc) eval_cut(k, n, S, SL, best);   // distinct values only
+            if (k >= 1 && tprev < tc && n < c_big) eval_cut(k, n, S, SL, best);   // distinct values only
             SL += tc;
             k++;
             tprev = tc;
@@ -769,13 +714,9 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
             ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
         }
         s_ub[i] = ub;
-        // a real candidate for the lower bound: the cut after the chunk's first row
-        // (t[ra], t[ra+1] share a sector with the value the bound already reads)
-        if (ra + 1 < rb && ta < a.t[ra + 1]) {
-            const uint32_t k1 = ka + 1;
-            const u128 ad1 = (u128)S * k1 - (u128)n * (SL + ta);
-            const double dD = approx_d((uint32_t)(ad1 >> 64), (uint64_t)ad1);
-            lbm = fmax(lbm, __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)k1, (double)(n - k1))), dn));
+        if (ka >= 1 && a.t[ra - 1] < ta) {      // the chunk start is a real candidate
+            const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
+            lbm = fmax(lbm, __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)ka, (double)(n - ka))), dn));
         }
     }
     for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));

@@ -129,7 +129,8 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : 4)) onesw
     uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + TILE);                   // [TILE]
     uint16_t (*s_whist)[R] = reinterpret_cast<uint16_t (*)[R]>(s_vals + TILE);        // [NW][R]
     __shared__ uint64_t s_delta[R];
-    __shared__ uint32_t s_nvalid;
+    __shared__ uint32_t s_lstart[R + 1];
+    __shared__ uint32_t s_cnt[R];
     __shared__ uint64_t s_gw[NW];
     __shared__ uint32_t s_cw[NW];
     __shared__ uint32_t s_tile;
@@ -137,6 +138,7 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : 4)) onesw
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     if (tid == 0) s_tile = atomicAdd(a.tile_counter, 1u);
     for (int i = tid; i < NW * R / 2; i += NT) reinterpret_cast<uint32_t *>(&s_whist[0][0])[i] = 0;
+    for (int i = tid; i < R; i += NT) s_cnt[i] = 0;
     __syncthreads();
     const uint32_t tile = s_tile;
     const uint64_t wbase = (uint64_t)tile * TILE + (uint64_t)w * (32 * IT);
@@ -160,6 +162,14 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : 4)) onesw
             val[j] = 0;
         }
     }
+    // the tile's digit counts, published at once so that successors' look-backs
+    // do not wait for this tile's ranking
+#pragma unroll
+    for (int j = 0; j < IT; j++)
+        if (wbase + (uint64_t)j * 32 + lane < a.n) atomicAdd(&s_cnt[(uint32_t)(key[j] >> a.shift) & (R - 1)], 1u);
+    __syncthreads();
+    if (tid < R) __stcg(a.status + (uint64_t)tile * R + tid, (tile == 0 ? kFlagP : kFlagA) | s_cnt[tid]);
+
     // warp-level multi-split ranking, in element order
     uint32_t rank[IT];
 #pragma unroll
@@ -191,7 +201,6 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : 4)) onesw
             s_whist[ww][d] = (uint16_t)cnt;
             cnt += c;
         }
-        __stcg(a.status + (uint64_t)tile * R + d, (tile == 0 ? kFlagP : kFlagA) | cnt);
         if (tile != 0) {
             int64_t j = (int64_t)tile - 1;
             while (true) {
@@ -219,10 +228,9 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : 4)) onesw
         for (int ww = 0; ww < w; ww++) { goff += s_gw[ww]; coff += s_cw[ww]; }
         const uint64_t g_excl = goff + g_incl - gcount;
         const uint32_t c_excl = coff + c_incl - cnt;
+        s_lstart[d] = c_excl;
         s_delta[d] = g_excl + excl - c_excl;   // global position - local position
-        if (d == R - 1) s_nvalid = c_excl + cnt;
-#pragma unroll
-        for (int ww = 0; ww < NW; ww++) s_whist[ww][d] += (uint16_t)c_excl;   // warp base in tile order
+        if (d == R - 1) s_lstart[R] = c_excl + cnt;
     }
     __syncthreads();
 
@@ -232,13 +240,13 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : 4)) onesw
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         if (i < a.n) {
             const uint32_t dd = (uint32_t)(key[j] >> a.shift) & (R - 1);
-            const uint32_t lp = s_whist[w][dd] + rank[j];
+            const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + rank[j];
             s_keys[lp] = key[j];
             s_vals[lp] = val[j];
         }
     }
     __syncthreads();
-    const uint32_t nvalid = s_nvalid;
+    const uint32_t nvalid = s_lstart[R];
 #pragma unroll 4
     for (uint32_t i = tid; i < nvalid; i += NT) {
         const uint64_t k = s_keys[i];
