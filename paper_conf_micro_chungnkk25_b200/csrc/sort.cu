@@ -109,6 +109,7 @@ struct PassArgs {
     uint32_t *t_out, *row_out;          // LAST
     uint64_t n;
     int shift, tbits, pass;
+    int ballot_rank;                    // 1: equal-digit lanes by RB ballots instead of match.any
     const uint64_t *hist;               // [pass][kHistR] global digit counts
     uint64_t *status;                   // [ntiles][R]
     uint32_t *tile_counter;
@@ -179,7 +180,17 @@ __global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : 4)) onesw
         const uint32_t vmask = __ballot_sync(0xffffffffu, valid);
         if (valid) {
             const uint32_t d = (uint32_t)(key[j] >> a.shift) & (R - 1);
-            const uint32_t peers = __match_any_sync(vmask, d);
+            uint32_t peers;
+            if (a.ballot_rank) {   // lanes with an equal digit from RB ballots (no match.any)
+                peers = vmask;
+#pragma unroll
+                for (int b = 0; b < RB; b++) {
+                    const uint32_t bal = __ballot_sync(vmask, (d >> b) & 1u);
+                    peers &= ((d >> b) & 1u) ? bal : ~bal;
+                }
+            } else {
+                peers = __match_any_sync(vmask, d);
+            }
             const uint32_t base = s_whist[w][d];
             const uint32_t below = __popc(peers & ((1u << lane) - 1));
             rank[j] = base + below;
@@ -354,6 +365,10 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     a.hist = c.hist;
     a.status = (uint64_t *)c.sort_status;
     a.tile_counter = &c.scalars->tile_counter;
+    {
+        const char *e = getenv("STEMROOT_SORT_RANK");
+        a.ballot_rank = (e && e[0] == 'b') ? 1 : 0;
+    }
     uint64_t *kin = c.keys[0], *kout = c.keys[1];
     uint32_t *vin = c.vals[0], *vout = c.vals[1];
     for (int p = 0; p < npasses; p++) {
