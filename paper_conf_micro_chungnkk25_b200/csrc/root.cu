@@ -2,16 +2,15 @@
 // and the level-synchronous ROOT clustering (§3.4, Fig. 6).
 //
 // Every level processes the whole frontier (all kernels' active clusters at
-// once) as one segmented operation over the concatenated active rows:
-//   tile_map_kernel  first/last frontier cluster of every 2048-row tile
-//   split_kernel     stages the tile's t in shared memory (coalesced), block
-//                    scan of t gives S_L for every candidate cut k, scored
-//                    exactly (D = n S_L - S k, score D^2/(k(n-k)), R5);
-//                    thread- then block-level segmented argmax; clusters
-//                    inside a tile finish here
-//   fixup_kernel     one warp per cluster spanning several tiles
-//   decide_kernel    Eq. 7 vs Eq. 8 per cluster (R6-R9) in the fixed fp64 order
-//   scan + apply     compacts the non-trivial children into the next frontier
+// once).  For each cluster the 2-means cut (R5) is the argmax over its cuts k
+// of D_k^2/(k(n-k)), D_k = n S_L(k) - S k, compared exactly:
+//   small_split_kernel  clusters < big_rows(): one warp per 1024-row range of
+//                       the frontier, 32 rows per step, exact-safe pruning
+//   big_split_kernel    clusters >= big_rows(): one block per 65536 rows,
+//                       chunk bounds from the sampled prefix, only chunks that
+//                       may hold the argmax are scanned; big_reduce_kernel
+//   decide_kernel       Eq. 7 vs Eq. 8 per cluster (R6-R9), fixed fp64 order
+//   scan + apply        compacts the non-trivial children into the next frontier
 // Cluster totals (S exact u64, Q exact u128) travel with the frontier; only
 // Q_L at the chosen cut is read from the sampled prefix arrays.
 #include <cstdlib>
@@ -20,10 +19,6 @@
 
 namespace sr {
 
-constexpr int kSplitThreads = 256;
-constexpr int kSplitItems = 16;
-constexpr int kTile = kSplitThreads * kSplitItems;      // 4096 active rows
-constexpr int kMaxTileClusters = kTile / 2 + 2;         // frontier clusters have >= 2 rows
 // clusters of >= big_rows() rows take the chunk-bound path (STEMROOT_BIG_ROWS overrides)
 __constant__ uint64_t c_big;
 static uint64_t big_rows() {
@@ -112,32 +107,8 @@ int prefix_moments(Ctx &c, uint64_t n) {
 }
 
 // ---------------------------------------------------------------- a3: split
-struct Part {
-    Cand cand;
-    uint32_t c;
-};
-
 __device__ __forceinline__ bool nontrivial(const uint32_t *t, uint32_t lo, uint32_t hi) {
     return hi - lo >= 2 && t[lo] != t[hi - 1];
-}
-
-// first/last frontier cluster of every tile; tiles inside one cluster go to
-// the fast list, the others to the general list (order is irrelevant).
-__global__ void tile_map_kernel(const uint32_t *__restrict__ aoff, const uint32_t *__restrict__ f_lo,
-                                const uint32_t *__restrict__ f_hi, uint32_t C, uint64_t A, uint64_t ntiles,
-                                uint32_t *__restrict__ first, uint32_t *__restrict__ last,
-                                uint32_t *__restrict__ fast_list, uint32_t *__restrict__ gen_list,
-                                uint32_t *__restrict__ counts) {
-    const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (j >= ntiles) return;
-    const uint64_t ts = j * kTile, te = min(ts + kTile, A);
-    const uint32_t f = (uint32_t)upper_bound(aoff, C, (uint32_t)ts) - 1;
-    const uint32_t l = (uint32_t)upper_bound(aoff, C, (uint32_t)(te - 1)) - 1;
-    first[j] = f;
-    last[j] = l;
-    if (f == l && f_hi[f] - f_lo[f] >= c_big) return;   // inside a big cluster: chunk-bound path
-    if (f == l) fast_list[atomicAdd(&counts[0], 1u)] = (uint32_t)j;
-    else gen_list[atomicAdd(&counts[1], 1u)] = (uint32_t)j;
 }
 
 // Evaluate the valid cut k (t[k-1] < t[k]): |D| = S k - n S_L (D <= 0 for sorted
@@ -174,260 +145,6 @@ __device__ __forceinline__ void eval_cut(uint32_t k, uint64_t n, uint64_t S, uin
     }
 }
 
-// sum of t over [lo, r): pref1(r) - pref1(lo) with the partial chunks spread over a warp
-__device__ __forceinline__ uint64_t warp_range_sum(const uint64_t *PS1, const uint32_t *t, uint64_t lo, uint64_t r) {
-    const int lane = threadIdx.x & 31;
-    uint64_t part = 0;
-    const uint64_t rb = r & ~(kChunk - 1), lb = lo & ~(kChunk - 1);
-    if (rb + lane < r) part += t[rb + lane];
-    if (lb + lane < lo) part -= t[lb + lane];
-    for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
-    return PS1[r >> kChunkLog] - PS1[lo >> kChunkLog] + part;
-}
-
-struct SplitArgs {
-    const uint32_t *f_lo, *f_hi, *aoff, *tile_first, *tile_last, *list;
-    const uint64_t *f_S;
-    const uint64_t *PS1;
-    const uint32_t *t;
-    uint64_t A;
-    uint32_t *cut;
-    uint64_t *cut_SL;
-    Part *part;
-};
-
-__host__ __device__ constexpr int padx(int i) { return i + (i >> 3); }   // conflict-free blocked u32 reads
-
-struct SplitSmem {
-    uint64_t S[kMaxTileClusters], base[kMaxTileClusters];
-    uint64_t red[kSplitThreads / 32 + 1];
-    uint64_t carry;
-    Cand wtot[kSplitThreads / 32];             // per-warp inclusive (flag, best) of the run scan
-    uint32_t wflag[kSplitThreads / 32];
-    uint32_t t[padx(kTile + 1) + 1];           // t[padx(p + 1)] = t at tile position p; t[0] = halo
-    uint32_t ao[kMaxTileClusters], lo[kMaxTileClusters], n[kMaxTileClusters];
-    uint32_t wmax[kSplitThreads / 32];
-    uint16_t cid[kTile];                       // tile-relative cluster of every position
-};
-
-__device__ __forceinline__ Cand shfl_cand_up(const Cand &a, int d) {
-    Cand r;
-    r.x = __shfl_up_sync(0xffffffffu, a.x, d);
-    r.dp = __shfl_up_sync(0xffffffffu, a.dp, d);
-    r.dlo = __shfl_up_sync(0xffffffffu, a.dlo, d);
-    r.p = __shfl_up_sync(0xffffffffu, a.p, d);
-    r.SL = __shfl_up_sync(0xffffffffu, a.SL, d);
-    r.dhi = __shfl_up_sync(0xffffffffu, a.dhi, d);
-    r.k = __shfl_up_sync(0xffffffffu, a.k, d);
-    return r;
-}
-
-// run-scan operator over threads: (f1,v1) + (f2,v2) = (f1|f2, f2 ? v2 : best(v1,v2))
-__device__ __forceinline__ void run_combine(uint32_t fp, const Cand &vp, uint32_t &f, Cand &v) {
-    if (!f && better(vp, v)) v = vp;
-    f |= fp;
-}
-
-__global__ void __launch_bounds__(kSplitThreads, 2) split_kernel(SplitArgs a) {
-    extern __shared__ __align__(16) unsigned char s_dyn[];
-    SplitSmem &sm = *reinterpret_cast<SplitSmem *>(s_dyn);
-    uint32_t *s_t = sm.t;
-    uint16_t *s_cid = sm.cid;
-    uint32_t *s_ao = sm.ao, *s_lo = sm.lo, *s_n = sm.n;
-    uint64_t *s_S = sm.S, *s_base = sm.base;
-
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const uint32_t tile = a.list[blockIdx.x];
-    const uint64_t ts = (uint64_t)tile * kTile;
-    const uint64_t te = min(ts + kTile, a.A);
-    const int nt = (int)(te - ts);
-    const uint32_t c0 = a.tile_first[tile];
-    const int nc = (int)(a.tile_last[tile] - c0) + 1;
-
-    // cluster table of the tile
-    for (int i = tid; i < nc; i += kSplitThreads) {
-        const uint32_t c = c0 + i, lo = a.f_lo[c];
-        s_ao[i] = a.aoff[c];
-        s_lo[i] = lo;
-        s_n[i] = a.f_hi[c] - lo;
-        s_S[i] = a.f_S[c];
-    }
-    for (int p = tid; p < kTile; p += kSplitThreads) s_cid[p] = 0;
-    __syncthreads();
-    for (int i = tid + 1; i < nc; i += kSplitThreads) s_cid[s_ao[i] - ts] = (uint16_t)i;   // cluster heads
-    // carry into the first cluster when it began before this tile: sum of t over [lo, row(ts))
-    if (w == 0) {
-        uint64_t carry = 0;
-        if (s_ao[0] < ts) carry = warp_range_sum(a.PS1, a.t, s_lo[0], s_lo[0] + (ts - s_ao[0]));
-        if (lane == 0) sm.carry = carry;
-    }
-    __syncthreads();
-    // running max over positions (heads carry increasing ids): blocked, 8 per thread
-    {
-        uint32_t run = 0;
-#pragma unroll
-        for (int j = 0; j < kSplitItems; j++) run = max(run, (uint32_t)s_cid[tid * kSplitItems + j]);
-        uint32_t incl = run;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl = max(incl, v);
-        }
-        if (lane == 31) sm.wmax[w] = incl;
-        uint32_t pre = __shfl_up_sync(0xffffffffu, incl, 1);
-        if (lane == 0) pre = 0;
-        __syncthreads();
-        for (int ww = 0; ww < w; ww++) pre = max(pre, sm.wmax[ww]);
-        uint32_t r = pre;
-#pragma unroll
-        for (int j = 0; j < kSplitItems; j++) {
-            r = max(r, (uint32_t)s_cid[tid * kSplitItems + j]);
-            s_cid[tid * kSplitItems + j] = (uint16_t)r;
-        }
-    }
-    __syncthreads();
-    // coalesced load of t for the tile (striped), plus the halo row before position 0
-    for (int idx = tid; idx <= nt; idx += kSplitThreads) {
-        uint32_t v = 0;
-        if (idx == 0) {
-            if (s_ao[0] < ts) v = a.t[s_lo[0] + (ts - s_ao[0]) - 1];
-        } else {
-            const int p = idx - 1, ci = s_cid[p];
-            v = a.t[s_lo[ci] + (ts + p - s_ao[ci])];
-        }
-        s_t[padx(idx)] = v;
-    }
-    __syncthreads();
-    // block exclusive scan of t over positions -> S_L at every thread's first position
-    const int p0 = tid * kSplitItems;
-    const int pend = min(p0 + kSplitItems, nt);
-    uint64_t mysum = 0;
-#pragma unroll
-    for (int j = 0; j < kSplitItems; j++)
-        if (p0 + j < nt) mysum += s_t[padx(p0 + j + 1)];
-    uint64_t tot;
-    const uint64_t excl = block_excl_scan<uint64_t, kSplitThreads>(mysum, sm.red, &tot);
-    {
-        uint64_t run = excl;
-        for (int p = p0; p < pend; p++) {
-            const int ci = s_cid[p];
-            if (s_ao[ci] == ts + p) s_base[ci] = run;          // cluster starts inside the tile
-            run += s_t[padx(p + 1)];
-        }
-        if (tid == 0 && s_ao[0] < ts) s_base[0] = (uint64_t)0 - sm.carry;   // S_L = run + carry (mod 2^64)
-    }
-    __syncthreads();
-
-    // ---- candidates: thread-local segmented argmax with exact incremental D
-    int head_ci = -1;                   // first segment when incomplete
-    Cand head_b = no_cand();
-    bool head_before = false;           // its cluster started before this thread
-    uint32_t out_f = 1;                 // run-scan element: 1 = the carried run starts here / no carry
-    Cand out_v = no_cand();
-    int out_ci = -1;                    // cluster carried out of this thread (extends beyond it)
-    if (p0 < nt) {
-        int ci = s_cid[p0];
-        uint64_t n = s_n[ci], S = s_S[ci], ao = s_ao[ci];
-        uint32_t k = (uint32_t)(ts + p0 - ao);
-        uint64_t SL = excl - s_base[ci];
-        int seg_start = p0;
-        Cand best = no_cand();
-        auto flush = [&](int seg_end) {
-            const bool before = ao < ts + p0, after = ao + n > ts + pend;
-            if (!before && !after) {
-                a.cut[c0 + ci] = best.k;                      // whole cluster inside this thread
-                a.cut_SL[c0 + ci] = best.SL;
-                return;
-            }
-            if (seg_start == p0) { head_ci = ci; head_b = best; head_before = before; }
-            if (seg_end == pend && after) { out_ci = ci; out_v = best; out_f = before ? 0u : 1u; }
-        };
-        uint32_t tprev = s_t[padx(p0)];
-        for (int p = p0; p < pend; p++) {
-            const int cj = s_cid[p];
-            if (cj != ci) {
-                flush(p);
-                ci = cj;
-                n = s_n[ci];
-                S = s_S[ci];
-                ao = s_ao[ci];
-                k = 0;
-                SL = 0;
-                seg_start = p;
-                best = no_cand();
-            }
-            const uint32_t tc = s_t[padx(p + 1)];
-            if (k >= 1 && tprev < tc && n < c_big) eval_cut(k, n, S, SL, best);   // distinct values only
-            SL += tc;
-            k++;
-            tprev = tc;
-        }
-        flush(pend);
-    }
-    // ---- block run-scan over threads: element (out_f, out_v)
-    uint32_t f = out_f;
-    Cand v = out_v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const Cand ov = shfl_cand_up(v, o);
-        const uint32_t of = __shfl_up_sync(0xffffffffu, f, o);
-        if (lane >= o) run_combine(of, ov, f, v);
-    }
-    if (lane == 31) { sm.wtot[w] = v; sm.wflag[w] = f; }
-    const Cand wprev = shfl_cand_up(v, 1);
-    const uint32_t fprev = __shfl_up_sync(0xffffffffu, f, 1);
-    __syncthreads();
-    uint32_t cf = 0;                    // combination of the previous warps' totals
-    Cand cv = no_cand();
-    for (int ww = 0; ww < w; ww++) {
-        uint32_t ff = sm.wflag[ww];
-        Cand vv = sm.wtot[ww];
-        run_combine(cf, cv, ff, vv);
-        cf = ff;
-        cv = vv;
-    }
-    uint32_t ef = cf;                   // exclusive element at this thread
-    Cand ev = cv;
-    if (lane > 0) {
-        uint32_t ff = fprev;
-        Cand vv = wprev;
-        run_combine(cf, cv, ff, vv);
-        ef = ff;
-        ev = vv;
-    }
-    uint32_t inf = f;                   // inclusive element at this thread
-    Cand iv = v;
-    run_combine(cf, cv, inf, iv);
-    (void)ef;
-    // a head that started before this thread and ends inside it closes its run
-    if (head_ci >= 0 && head_before && out_ci != head_ci && s_n[head_ci] < c_big) {
-        Cand fin = head_b;
-        if (better(ev, fin)) fin = ev;
-        const uint64_t ao = s_ao[head_ci];
-        if (ao >= ts) {
-            a.cut[c0 + head_ci] = fin.k;
-            a.cut_SL[c0 + head_ci] = fin.SL;
-        } else {
-            a.part[2 * (uint64_t)tile] = Part{fin, c0 + head_ci};
-        }
-    }
-    // the run carried out of the tile's last thread continues into the next tile
-    if (p0 < nt && pend == nt && out_ci >= 0 && s_n[out_ci] < c_big) {
-        const uint64_t ao = s_ao[out_ci];
-        a.part[2 * (uint64_t)tile + (ao <= ts ? 0 : 1)] = Part{iv, c0 + out_ci};
-    }
-}
-
-// Tiles that lie inside one cluster (most tiles while clusters are large):
-// no cluster table, no segmentation, plain block argmax.
-struct FastSmem {
-    Cand wbest[kSplitThreads / 32];
-    double thr[kSplitThreads / 32];
-    uint64_t red[kSplitThreads / 32 + 1];
-    uint64_t carry;
-    uint32_t t[padx(kTile + 1) + 1];
-};
-
 __device__ __forceinline__ Cand shfl_cand_xor(const Cand &a, int m) {
     Cand r;
     r.x = __shfl_xor_sync(0xffffffffu, a.x, m);
@@ -440,183 +157,81 @@ __device__ __forceinline__ Cand shfl_cand_xor(const Cand &a, int m) {
     return r;
 }
 
-__global__ void __launch_bounds__(kSplitThreads, 4) split_fast_kernel(SplitArgs a) {
-    __shared__ FastSmem sm;
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const uint32_t tile = a.list[blockIdx.x];
-    const uint64_t ts = (uint64_t)tile * kTile;
-    const uint64_t te = min(ts + kTile, a.A);
-    const int nt = (int)(te - ts);
-    const uint32_t c = a.tile_first[tile];
-    const uint64_t lo = a.f_lo[c], n = a.f_hi[c] - lo, S = a.f_S[c], ao = a.aoff[c];
-    const uint64_t row0 = lo + (ts - ao);              // the tile lies inside [lo, hi)
-    if (w == 0) {
-        const uint64_t carry = row0 > lo ? warp_range_sum(a.PS1, a.t, lo, row0) : 0;
-        if (lane == 0) sm.carry = carry;
-    }
-    for (int idx = tid; idx <= nt; idx += kSplitThreads)
-        sm.t[padx(idx)] = idx ? a.t[row0 + idx - 1] : (row0 > lo ? a.t[row0 - 1] : 0u);
-    __syncthreads();
-    const int p0 = tid * kSplitItems, pend = min(p0 + kSplitItems, nt);
-    uint64_t mysum = 0;
-#pragma unroll
-    for (int j = 0; j < kSplitItems; j++)
-        if (p0 + j < nt) mysum += sm.t[padx(p0 + j + 1)];
-    uint64_t tot;
-    const uint64_t excl = block_excl_scan<uint64_t, kSplitThreads>(mysum, sm.red, &tot);
-    // ---- exact-safe pruning.  |D_k| is concave in k for sorted t, so over this
-    // thread's cuts k0..k0+cnt-1:  |D_k| <= |D_k0| + (k-k0) max(0, S - n t_k0),
-    // and k(n-k) >= its value at an end.  A thread whose upper bound is below the
-    // score of a real candidate of the tile cannot hold the argmax (or a tie).
-    const uint64_t SL0 = sm.carry + excl;
-    const uint32_t k0 = (uint32_t)(ts - ao + p0);
-    double ub = 0.0, lb = 0.0;
-    if (p0 < nt) {
-        const int cnt = pend - p0;
-        const u128 ad0 = (u128)S * k0 - (u128)n * SL0;
-        const uint64_t nt0 = n * (uint64_t)sm.t[padx(p0 + 1)];
-        const double slope = S > nt0 ? __ull2double_rn(S - nt0) : 0.0;
-        const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
-        const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad0 >> 64), (uint64_t)ad0),
-                                               __dmul_rn(slope, (double)(cnt - 1))), up);
-        const uint64_t kf = max((uint64_t)k0, (uint64_t)1), kl = min((uint64_t)k0 + cnt - 1, n - 1);
-        if (kf <= kl) {
-            const double pmin = fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
-            ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
-        }
-        // one real candidate: the thread's first valid cut
-        uint64_t SLj = SL0;
-        uint32_t tprev = sm.t[padx(p0)];
-        for (int j = 0; j < cnt; j++) {
-            const uint32_t tc = sm.t[padx(p0 + j + 1)];
-            const uint32_t k = k0 + j;
-            if (k >= 1 && tprev < tc) {
-                const u128 ad = (u128)S * k - (u128)n * SLj;
-                const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
-                lb = __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)k, (double)(n - k))), dn);
-                break;
-            }
-            SLj += tc;
-            tprev = tc;
-        }
-    }
-    double thr = lb;
-#pragma unroll
-    for (int o = 16; o; o >>= 1) thr = fmax(thr, __shfl_xor_sync(0xffffffffu, thr, o));
-    if (lane == 0) sm.thr[w] = thr;
-    __syncthreads();
-    for (int ww = 0; ww < kSplitThreads / 32; ww++) thr = fmax(thr, sm.thr[ww]);
-    Cand best = no_cand();
-    if (p0 < nt && ub >= thr) {
-        uint64_t SL = SL0;
-        uint32_t k = k0;
-        uint32_t tprev = sm.t[padx(p0)];
-#pragma unroll
-        for (int j = 0; j < kSplitItems; j++) {
-            if (p0 + j < pend) {
-                const uint32_t tc = sm.t[padx(p0 + j + 1)];
-                if (k >= 1 && tprev < tc) eval_cut(k, n, S, SL, best);
-                SL += tc;
-                k++;
-                tprev = tc;
-            }
-        }
-    }
-#pragma unroll
-    for (int o = 16; o; o >>= 1) {
-        const Cand v = shfl_cand_xor(best, o);
-        if (better(v, best)) best = v;
-    }
-    if (lane == 0) sm.wbest[w] = best;
-    __syncthreads();
-    if (tid == 0) {
-        for (int ww = 1; ww < kSplitThreads / 32; ww++)
-            if (better(sm.wbest[ww], best)) best = sm.wbest[ww];
-        if (ao >= ts && ao + n <= te) {
-            a.cut[c] = best.k;
-            a.cut_SL[c] = best.SL;
-        } else {
-            a.part[2 * (uint64_t)tile] = Part{best, c};   // ao <= ts: slot 0
-        }
-    }
-}
+// ---------------------------------------------------------------- small clusters: a warp per range
+// Clusters of < big_rows() rows.  Warp g owns every cluster whose active offset
+// starts in [g*kSmallRange, (g+1)*kSmallRange) and scans it 32 rows at a time:
+// coalesced loads, a warp scan gives S_L, every valid cut is scored exactly
+// (eval_cut).  A 32-row chunk is skipped when the concavity bound of its cuts
+// is below the best candidate of the cluster so far (exact-safe, see
+// big_split_kernel).  No shared memory, no cross-warp reduction.
+constexpr uint64_t kSmallRange = 1024;
 
-__device__ __forceinline__ Cand shfl_cand(const Cand &a, int src) {
-    Cand r;
-    r.x = __shfl_sync(0xffffffffu, a.x, src);
-    r.dp = __shfl_sync(0xffffffffu, a.dp, src);
-    r.dlo = __shfl_sync(0xffffffffu, a.dlo, src);
-    r.p = __shfl_sync(0xffffffffu, a.p, src);
-    r.SL = __shfl_sync(0xffffffffu, a.SL, src);
-    r.dhi = __shfl_sync(0xffffffffu, a.dhi, src);
-    r.k = __shfl_sync(0xffffffffu, a.k, src);
-    return r;
-}
-
-// One warp per cluster spanning several tiles: argmax of its tile partials.
-// Clusters spanning more than kBigSpan tiles are left to fixup_big_kernel.
-constexpr uint64_t kBigSpan = 2048;
-
-__global__ void __launch_bounds__(256)
-fixup_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, const uint32_t *__restrict__ aoff,
-             uint32_t C, const Part *__restrict__ part, uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL,
-             uint32_t *__restrict__ big_list, uint32_t *__restrict__ big_count) {
-    const uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+__global__ void __launch_bounds__(256) small_split_kernel(const uint32_t *__restrict__ f_lo,
+                                                          const uint32_t *__restrict__ f_hi,
+                                                          const uint32_t *__restrict__ aoff,
+                                                          const uint64_t *__restrict__ f_S, uint32_t C, uint64_t A,
+                                                          const uint32_t *__restrict__ t, uint32_t *__restrict__ cut,
+                                                          uint64_t *__restrict__ cut_SL) {
+    const uint64_t g = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
-    if (c >= C) return;
-    const uint64_t ao = aoff[c], ae = ao + (f_hi[c] - f_lo[c]);
-    const uint64_t j0 = ao / kTile, j1 = (ae - 1) / kTile;
-    if (j0 == j1 || ae - ao >= c_big) return;
-    if (j1 - j0 > kBigSpan) {
-        if (lane == 0) big_list[atomicAdd(big_count, 1u)] = (uint32_t)c;
-        return;
-    }
-    Cand best = no_cand();
-    for (uint64_t j = j0 + lane; j <= j1; j += 32) {
-        const int slot = (j == j0 && ao != j0 * kTile) ? 1 : 0;
-        const Cand v = part[2 * j + slot].cand;
-        if (better(v, best)) best = v;
-    }
+    const uint64_t r0 = g * kSmallRange;
+    if (r0 >= A) return;
+    const uint64_t r1 = r0 + kSmallRange;
+    const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
+    for (uint32_t c = (uint32_t)lower_bound(aoff, C, (uint32_t)r0); c < C && aoff[c] < r1; c++) {
+        const uint64_t lo = f_lo[c], n = f_hi[c] - lo;
+        if (n >= c_big) continue;
+        const uint64_t S = f_S[c];
+        Cand best = no_cand();
+        double thr = 0.0;
+        uint64_t SLb = 0;
+        uint32_t tlast = 0;
+        for (uint64_t k0 = 0; k0 < n; k0 += 32) {
+            const uint64_t k = k0 + lane;
+            const bool in = k < n;
+            const uint32_t tc = in ? t[lo + k] : 0u;
+            uint32_t tp = __shfl_up_sync(0xffffffffu, tc, 1);
+            if (lane == 0) tp = tlast;
+            uint64_t incl = tc;
 #pragma unroll
-    for (int o = 16; o; o >>= 1) {
-        const Cand v = shfl_cand(best, lane ^ o);
-        if (better(v, best)) best = v;
-    }
-    if (lane == 0) {
-        cut[c] = best.k;
-        cut_SL[c] = best.SL;
-    }
-}
-
-// one block per very large cluster
-__global__ void __launch_bounds__(256)
-fixup_big_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
-                 const uint32_t *__restrict__ aoff, const Part *__restrict__ part, const uint32_t *__restrict__ big_list,
-                 const uint32_t *__restrict__ big_count, uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
-    __shared__ Cand s_w[8];
-    if (blockIdx.x >= *big_count) return;
-    const uint32_t c = big_list[blockIdx.x];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const uint64_t ao = aoff[c], ae = ao + (f_hi[c] - f_lo[c]);
-    const uint64_t j0 = ao / kTile, j1 = (ae - 1) / kTile;
-    Cand best = no_cand();
-    for (uint64_t j = j0 + threadIdx.x; j <= j1; j += blockDim.x) {
-        const int slot = (j == j0 && ao != j0 * kTile) ? 1 : 0;
-        const Cand v = part[2 * j + slot].cand;
-        if (better(v, best)) best = v;
-    }
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += v;
+            }
+            // upper bound of the chunk's scores from its first cut (warp-uniform)
+            const uint64_t cnt = min((uint64_t)32, n - k0);
+            const uint32_t t0 = __shfl_sync(0xffffffffu, tc, 0);
+            const u128 ad0 = (u128)S * k0 - (u128)n * SLb;
+            const uint64_t nt0 = n * (uint64_t)t0;
+            const double slope = S > nt0 ? __ull2double_rn(S - nt0) : 0.0;
+            const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad0 >> 64), (uint64_t)ad0),
+                                                   __dmul_rn(slope, (double)(cnt - 1))), up);
+            const uint64_t kf = max(k0, (uint64_t)1), kl = min(k0 + cnt - 1, n - 1);
+            double ub = 0.0;
+            if (kf <= kl) {
+                const double pmin =
+                    fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
+                ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
+            }
+            if (ub >= thr) {
+                if (in && k >= 1 && tp < tc) eval_cut((uint32_t)k, n, S, SLb + incl - tc, best);
+                double lb = best.k ? __dmul_rn(__ddiv_rn(best.x, best.dp), dn) : 0.0;
 #pragma unroll
-    for (int o = 16; o; o >>= 1) {
-        const Cand v = shfl_cand(best, lane ^ o);
-        if (better(v, best)) best = v;
-    }
-    if (lane == 0) s_w[w] = best;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int k = 1; k < 8; k++)
-            if (better(s_w[k], best)) best = s_w[k];
-        cut[c] = best.k;
-        cut_SL[c] = best.SL;
+                for (int o = 16; o; o >>= 1) lb = fmax(lb, __shfl_xor_sync(0xffffffffu, lb, o));
+                thr = fmax(thr, lb);
+            }
+            SLb += __shfl_sync(0xffffffffu, incl, 31);
+            tlast = __shfl_sync(0xffffffffu, tc, 31);
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            const Cand v = shfl_cand_xor(best, o);
+            if (better(v, best)) best = v;
+        }
+        if (lane == 0) {
+            cut[c] = best.k;
+            cut_SL[c] = best.SL;
+        }
     }
 }
 
@@ -937,23 +552,16 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
     while (C > 0) {
         levels++;
         c.stats.active_rows += A;
-        const uint64_t ntiles = (A + kTile - 1) / kTile;
         CKS(c.ensure(c.cut, c.cap_cut, sizeof(uint32_t) * C));
         CKS(c.ensure(c.cut_SL, c.cap_cut_SL, sizeof(uint64_t) * C));
         CKS(c.ensure(c.cut_QL, c.cap_cut_QL, sizeof(u128) * C));
         CKS(c.ensure(c.cnt_sz, c.cap_cntsz, sizeof(uint64_t) * C));
-        CKS(c.ensure(c.split_part, c.cap_part, sizeof(Part) * 2 * ntiles));
-        CKS(c.ensure(c.tile_map, c.cap_tile_map, sizeof(uint32_t) * (4 * ntiles + 1024)));
         CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(C) + 1) * sizeof(uint64_t)));
         const int nxt = cur ^ 1;
         CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
         const int tk_s = c.stage_begin("root_split");
-        uint32_t *tfirst = c.tile_map, *tlast = c.tile_map + ntiles;
-        uint32_t *fast_list = c.tile_map + 2 * ntiles, *gen_list = c.tile_map + 3 * ntiles;
-        CK(cudaMemsetAsync(c.scalars->tile_counts, 0, sizeof(uint32_t) * 2, st));
-        tile_map_kernel<<<(unsigned)((ntiles + 255) / 256), 256, 0, st>>>(c.f_aoff[cur], c.f_lo[cur], c.f_hi[cur],
-                                                                          (uint32_t)C, A, ntiles, tfirst, tlast,
-                                                                          fast_list, gen_list, c.scalars->tile_counts);
+        small_split_kernel<<<(unsigned)(((A + kSmallRange - 1) / kSmallRange * 32 + 255) / 256), 256, 0, st>>>(
+            c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], c.f_S[cur], (uint32_t)C, A, c.t_sorted, c.cut, c.cut_SL);
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
         const uint64_t max_ent = A / kBigSeg + A / big_rows() + 1;
         CKS(c.ensure(c.big_ent, c.cap_big_ent, sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (C + 1)));
@@ -969,30 +577,10 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                    (unsigned long long *)c.big_thr, (Cand *)c.big_part};
         big_split_kernel<<<(unsigned)max_ent, kBigThreads, 0, st>>>(ba);
         c.launches += 2;
-        uint32_t counts[2];
-        CK(cudaMemcpyAsync(counts, c.scalars->tile_counts, sizeof(counts), cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        SplitArgs sa{c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], tfirst, tlast, fast_list, c.f_S[cur], c.PS1,
-                     c.t_sorted, A, c.cut, c.cut_SL, (Part *)c.split_part};
-        if (counts[0]) split_fast_kernel<<<counts[0], kSplitThreads, 0, st>>>(sa);
-        if (counts[1]) {
-            sa.list = gen_list;
-            CK(cudaFuncSetAttribute(split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SplitSmem)));
-            split_kernel<<<counts[1], kSplitThreads, sizeof(SplitSmem), st>>>(sa);
-        }
-        uint32_t *big_list = c.tile_map + 4 * ntiles;   // <= A / (kTile * kBigSpan) + 1 <= 513 entries
-        CK(cudaMemsetAsync(&c.scalars->big_count2, 0, sizeof(uint32_t), st));
-        const uint32_t max_big = (uint32_t)(A / ((uint64_t)kTile * kBigSpan) + 1);
-        fixup_kernel<<<(unsigned)((C * 32 + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur],
-                                                                       (uint32_t)C, (const Part *)c.split_part, c.cut,
-                                                                       c.cut_SL, big_list, &c.scalars->big_count2);
-        fixup_big_kernel<<<max_big, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], (const Part *)c.split_part,
-                                                   big_list, &c.scalars->big_count2, c.cut, c.cut_SL);
         big_reduce_kernel<<<(unsigned)min(C, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, first_ent,
                                                       (const Cand *)c.big_part, c.cut, c.cut_SL);
-        c.launches++;
-        c.launches += 3 + (counts[0] ? 1 : 0) + (counts[1] ? 1 : 0);
-        c.stage_end(tk_s, 4 * A + 8 * ntiles + 20 * C);
+        c.launches += 2;
+        c.stage_end(tk_s, 4 * A + 20 * C);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");
         DecideArgs da{c.f_lo[cur], c.f_hi[cur], c.cut, c.f_S[cur], c.cut_SL, c.f_Q[cur], (uint32_t)C, c.PS1, c.PS2,
