@@ -25,7 +25,7 @@ static uint64_t big_rows() {
     static uint64_t v = 0;
     if (!v) {
         const char *e = getenv("STEMROOT_BIG_ROWS");
-        v = e ? strtoull(e, nullptr, 10) : 4096;
+        v = e ? strtoull(e, nullptr, 10) : 1024;
         if (v < 64) v = 64;
     }
     return v;
@@ -165,6 +165,7 @@ __device__ __forceinline__ Cand shfl_cand_xor(const Cand &a, int m) {
 // is below the best candidate of the cluster so far (exact-safe, see
 // big_split_kernel).  No shared memory, no cross-warp reduction.
 constexpr uint64_t kSmallRange = 1024;
+constexpr int kSmallQ = 4;   // 32-row chunks loaded per step
 
 __global__ void __launch_bounds__(256) small_split_kernel(const uint32_t *__restrict__ f_lo,
                                                           const uint32_t *__restrict__ f_hi,
@@ -186,42 +187,53 @@ __global__ void __launch_bounds__(256) small_split_kernel(const uint32_t *__rest
         double thr = 0.0;
         uint64_t SLb = 0;
         uint32_t tlast = 0;
-        for (uint64_t k0 = 0; k0 < n; k0 += 32) {
-            const uint64_t k = k0 + lane;
-            const bool in = k < n;
-            const uint32_t tc = in ? t[lo + k] : 0u;
-            uint32_t tp = __shfl_up_sync(0xffffffffu, tc, 1);
-            if (lane == 0) tp = tlast;
-            uint64_t incl = tc;
+        for (uint64_t kb = 0; kb < n; kb += 32 * kSmallQ) {
+            uint32_t tq[kSmallQ];   // kSmallQ chunks' loads in flight
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
-                if (lane >= o) incl += v;
+            for (int q = 0; q < kSmallQ; q++) {
+                const uint64_t k = kb + 32 * q + lane;
+                tq[q] = k < n ? t[lo + k] : 0u;
             }
-            // upper bound of the chunk's scores from its first cut (warp-uniform)
-            const uint64_t cnt = min((uint64_t)32, n - k0);
-            const uint32_t t0 = __shfl_sync(0xffffffffu, tc, 0);
-            const u128 ad0 = (u128)S * k0 - (u128)n * SLb;
-            const uint64_t nt0 = n * (uint64_t)t0;
-            const double slope = S > nt0 ? __ull2double_rn(S - nt0) : 0.0;
-            const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad0 >> 64), (uint64_t)ad0),
-                                                   __dmul_rn(slope, (double)(cnt - 1))), up);
-            const uint64_t kf = max(k0, (uint64_t)1), kl = min(k0 + cnt - 1, n - 1);
-            double ub = 0.0;
-            if (kf <= kl) {
-                const double pmin =
-                    fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
-                ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
-            }
-            if (ub >= thr) {
-                if (in && k >= 1 && tp < tc) eval_cut((uint32_t)k, n, S, SLb + incl - tc, best);
-                double lb = best.k ? __dmul_rn(__ddiv_rn(best.x, best.dp), dn) : 0.0;
 #pragma unroll
-                for (int o = 16; o; o >>= 1) lb = fmax(lb, __shfl_xor_sync(0xffffffffu, lb, o));
-                thr = fmax(thr, lb);
+            for (int q = 0; q < kSmallQ; q++) {
+                const uint64_t k0 = kb + 32 * q;
+                if (k0 >= n) break;
+                const uint64_t k = k0 + lane;
+                const bool in = k < n;
+                const uint32_t tc = tq[q];
+                uint32_t tp = __shfl_up_sync(0xffffffffu, tc, 1);
+                if (lane == 0) tp = tlast;
+                uint64_t incl = tc;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+                    if (lane >= o) incl += v;
+                }
+                // upper bound of the chunk's scores from its first cut (warp-uniform)
+                const uint64_t cnt = min((uint64_t)32, n - k0);
+                const uint32_t t0 = __shfl_sync(0xffffffffu, tc, 0);
+                const u128 ad0 = (u128)S * k0 - (u128)n * SLb;
+                const uint64_t nt0 = n * (uint64_t)t0;
+                const double slope = S > nt0 ? __ull2double_rn(S - nt0) : 0.0;
+                const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad0 >> 64), (uint64_t)ad0),
+                                                       __dmul_rn(slope, (double)(cnt - 1))), up);
+                const uint64_t kf = max(k0, (uint64_t)1), kl = min(k0 + cnt - 1, n - 1);
+                double ub = 0.0;
+                if (kf <= kl) {
+                    const double pmin =
+                        fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
+                    ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
+                }
+                if (ub >= thr) {
+                    if (in && k >= 1 && tp < tc) eval_cut((uint32_t)k, n, S, SLb + incl - tc, best);
+                    double lb = best.k ? __dmul_rn(__ddiv_rn(best.x, best.dp), dn) : 0.0;
+#pragma unroll
+                    for (int o = 16; o; o >>= 1) lb = fmax(lb, __shfl_xor_sync(0xffffffffu, lb, o));
+                    thr = fmax(thr, lb);
+                }
+                SLb += __shfl_sync(0xffffffffu, incl, 31);
+                tlast = __shfl_sync(0xffffffffu, tc, 31);
             }
-            SLb += __shfl_sync(0xffffffffu, incl, 31);
-            tlast = __shfl_sync(0xffffffffu, tc, 31);
         }
 #pragma unroll
         for (int o = 16; o; o >>= 1) {
