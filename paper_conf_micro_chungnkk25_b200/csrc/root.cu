@@ -25,7 +25,7 @@ static uint64_t big_rows() {
     static uint64_t v = 0;
     if (!v) {
         const char *e = getenv("STEMROOT_BIG_ROWS");
-        v = e ? strtoull(e, nullptr, 10) : 1024;
+        v = e ? strtoull(e, nullptr, 10) : 2048;
         if (v < 64) v = 64;
     }
     return v;
