@@ -122,7 +122,7 @@ struct PassArgs {
 // (thread d < R owns digit d), then keys are staged in shared memory in
 // tile-sorted order and written out in digit runs (coalesced).
 template <int NT, int IT, int RB, bool FIRST, bool LAST>
-__global__ void __launch_bounds__(NT, (NT >= 512 ? 2 : NT >= 384 ? 3 : 4)) onesweep_kernel(PassArgs a) {
+__global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesweep_kernel(PassArgs a) {
     constexpr int NW = NT / 32, TILE = NT * IT, R = 1 << RB;
     static_assert(NT >= R, "one thread per digit");
     extern __shared__ __align__(16) unsigned char s_dyn[];
@@ -295,11 +295,33 @@ static int launch_pass_cfg(const PassArgs &a, bool first, bool last, cudaStream_
 }
 
 // tile shapes: 9-bit digits need >= 512 threads (one per digit); 8-bit keep 384 x 12
-static uint64_t tile_keys(int rb) { return rb == 9 ? 512 * 9 : 384 * 12; }
+// 8-bit tile shapes (threads, keys per thread); STEMROOT_SORT_SHAPE picks one for experiments
+struct Shape { int nt, it; };
+static const Shape kShapes[] = {{384, 12}, {384, 10}, {320, 14}, {448, 10}, {256, 20}, {512, 9}};
+static int shape_idx() {
+    static int s = -1;
+    if (s < 0) {
+        const char *e = getenv("STEMROOT_SORT_SHAPE");
+        s = e ? atoi(e) : 0;
+        if (s < 0 || s > 5) s = 0;
+    }
+    return s;
+}
+
+static uint64_t tile_keys(int rb) {
+    return rb == 9 ? 512 * 9 : (uint64_t)kShapes[shape_idx()].nt * kShapes[shape_idx()].it;
+}
 
 static int launch_sort_pass(const PassArgs &a, int rb, bool first, bool last, cudaStream_t st) {
     if (rb == 9) return launch_pass_cfg<512, 9, 9>(a, first, last, st);
-    return launch_pass_cfg<384, 12, 8>(a, first, last, st);
+    switch (shape_idx()) {
+        case 1: return launch_pass_cfg<384, 10, 8>(a, first, last, st);
+        case 2: return launch_pass_cfg<320, 14, 8>(a, first, last, st);
+        case 3: return launch_pass_cfg<448, 10, 8>(a, first, last, st);
+        case 4: return launch_pass_cfg<256, 20, 8>(a, first, last, st);
+        case 5: return launch_pass_cfg<512, 9, 8>(a, first, last, st);
+        default: return launch_pass_cfg<384, 12, 8>(a, first, last, st);
+    }
 }
 
 template <int RB>
