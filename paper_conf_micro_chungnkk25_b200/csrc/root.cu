@@ -165,9 +165,8 @@ __device__ __forceinline__ Cand shfl_cand_xor(const Cand &a, int m) {
 // is below the best candidate of the cluster so far (exact-safe, see
 // big_split_kernel).  No shared memory, no cross-warp reduction.
 constexpr uint64_t kSmallRange = 1024;
-constexpr int kSmallQ = 4;   // 32-row chunks loaded per step
-
-__global__ void __launch_bounds__(256) small_split_kernel(const uint32_t *__restrict__ f_lo,
+template <int kSmallQ, int MINB>   // 32-row chunks loaded per step; min resident blocks
+__global__ void __launch_bounds__(256, MINB) small_split_kernel(const uint32_t *__restrict__ f_lo,
                                                           const uint32_t *__restrict__ f_hi,
                                                           const uint32_t *__restrict__ aoff,
                                                           const uint64_t *__restrict__ f_S, uint32_t C, uint64_t A,
@@ -572,8 +571,18 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         const int nxt = cur ^ 1;
         CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
         const int tk_s = c.stage_begin("root_split");
-        small_split_kernel<<<(unsigned)(((A + kSmallRange - 1) / kSmallRange * 32 + 255) / 256), 256, 0, st>>>(
-            c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], c.f_S[cur], (uint32_t)C, A, c.t_sorted, c.cut, c.cut_SL);
+        {
+            const unsigned g = (unsigned)(((A + kSmallRange - 1) / kSmallRange * 32 + 255) / 256);
+            static int cfg = -1;
+            if (cfg < 0) {
+                const char *e = getenv("STEMROOT_SMALL_CFG");
+                cfg = e ? atoi(e) : 0;
+            }
+            auto *kern = cfg == 1 ? small_split_kernel<4, 4> : cfg == 2 ? small_split_kernel<8, 3>
+                       : cfg == 3 ? small_split_kernel<2, 4> : small_split_kernel<4, 3>;
+            kern<<<g, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], c.f_S[cur], (uint32_t)C, A, c.t_sorted,
+                                    c.cut, c.cut_SL);
+        }
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
         const uint64_t max_ent = A / kBigSeg + A / big_rows() + 1;
         CKS(c.ensure(c.big_ent, c.cap_big_ent, sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (C + 1)));
