@@ -51,7 +51,7 @@ void Ctx::release() {
     dfree(t_sorted, cap_ts); dfree(row_sorted, cap_rs); dfree(kid_count, cap_kc); dfree(goff, cap_goff);
     dfree(hist, cap_hist); dfree(sort_status, cap_status); dfree(scalars, cap_scalars);
     dfree(scan_scratch, cap_scan); dfree(PS1, cap_ps1); dfree(PS2, cap_ps2); dfree(chunk_sq, cap_chunk_sq);
-    dfree(cut, cap_cut); dfree(cut_SL, cap_cut_SL); dfree(cut_QL, cap_cut_QL); dfree(tile_map, cap_tile_map); dfree(cnt_sz, cap_cntsz); dfree(split_part, cap_part); dfree(flags, cap_flags);
+    dfree(cut, cap_cut); dfree(cut_SL, cap_cut_SL); dfree(cut_QL, cap_cut_QL); dfree(cnt_sz, cap_cntsz); dfree(flags, cap_flags);
     dfree(leaf_lo, cap_leaf_lo); dfree(leaf_m, cap_leaf_m); dfree(leaf_moff, cap_leaf_moff);
     dfree(leaf_U, cap_leaf_U); dfree(leaf_census, cap_leaf_census); dfree(leaf_kid, cap_leaf_kid);
     dfree(leaf_ord, cap_leaf_ord); dfree(fix_acc, cap_fix); dfree(kern_T, cap_kern_T); dfree(kern_g, cap_kern_g);

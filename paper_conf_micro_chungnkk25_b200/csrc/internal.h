@@ -38,8 +38,7 @@ struct DevScalars {
     uint64_t sum_q;               // sum_i floor(n_i U_i / m_i)
     uint64_t T;                   // exact total time
     uint32_t limit_err, pad1;
-    uint32_t tile_counts[2];      // fast / general split tiles of the current level
-    uint32_t big_count, big_count2;   // big-cluster entries / clusters left to fixup_big_kernel
+    uint32_t big_count, pad2;     // big-cluster (cluster, segment) entries of the current level
     double ssum;                  // RN(exact sum sqrt(mu V)) (global scope)
     double g;                     // Ssum / c (global scope)
     double est_frac, var_sum;     // sum rn(r_i)/m_i, sum rn(V_i)/m_i
@@ -157,11 +156,9 @@ struct Ctx {
     uint32_t *cut = nullptr; size_t cap_cut = 0;
     uint64_t *cut_SL = nullptr; size_t cap_cut_SL = 0;
     u128 *cut_QL = nullptr; size_t cap_cut_QL = 0;
-    uint32_t *tile_map = nullptr; size_t cap_tile_map = 0;
     void *big_ent = nullptr, *big_part = nullptr, *big_thr = nullptr;
     size_t cap_big_ent = 0, cap_big_part = 0, cap_big_thr = 0;
     uint64_t *cnt_sz = nullptr; size_t cap_cntsz = 0;
-    void *split_part = nullptr; size_t cap_part = 0;
     uint8_t *flags = nullptr; size_t cap_flags = 0;
     // leaves (a5/a6)
     uint32_t *leaf_lo = nullptr; size_t cap_leaf_lo = 0;
