@@ -497,7 +497,8 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
     CKS(c.ensure(c.kid_count, c.cap_kc, sizeof(uint32_t) * ((uint64_t)K + 1)));
     CKS(c.ensure(c.dist_cnt, c.cap_dist_cnt, sizeof(uint64_t) * ((uint64_t)K + 2)));
     CKS(c.ensure(c.scalars, c.cap_scalars, sizeof(DevScalars)));
-    CKS(c.ensure(c.hist, c.cap_hist, sizeof(uint64_t) * 12 * 512));
+    CKS(c.ensure(c.kid_max, c.cap_kmax, sizeof(uint32_t) * ((uint64_t)K + 1)));
+    CKS(c.ensure(c.hist, c.cap_hist, sizeof(uint64_t) * 8 * 256));
     CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
     CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
     const int tk_x = c.stage_begin("dist_exchange");

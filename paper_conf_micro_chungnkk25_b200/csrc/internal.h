@@ -97,7 +97,6 @@ struct Ctx {
     int sms = 148;
     cudaStream_t stream = nullptr;
     uint32_t launches = 0;
-    int tbits = 0;
     stem_stats stats{};
     Timing timing;
     // stage bracket: returns an index to pass to stage_end (or -1 when timing is off)
@@ -140,6 +139,9 @@ struct Ctx {
     uint32_t *vals[2] = {nullptr, nullptr}; size_t cap_vals[2] = {0, 0};
     uint32_t *t_sorted = nullptr, *row_sorted = nullptr; size_t cap_ts = 0, cap_rs = 0;
     uint32_t *kid_count = nullptr, *goff = nullptr; size_t cap_kc = 0, cap_goff = 0;
+    uint32_t *kid_max = nullptr; size_t cap_kmax = 0;          // per-kernel max t
+    uint64_t *key_base = nullptr; size_t cap_kbase = 0;        // [K + 1] offset-key bases
+    uint32_t *kid_tab = nullptr; size_t cap_kid_tab = 0;       // key >> 16 -> kernel
     uint64_t *hist = nullptr; size_t cap_hist = 0;
     void *sort_status = nullptr; size_t cap_status = 0;
     DevScalars *scalars = nullptr; size_t cap_scalars = 0;

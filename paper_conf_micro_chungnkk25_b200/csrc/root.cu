@@ -579,7 +579,9 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                 cfg = e ? atoi(e) : 0;
             }
             auto *kern = cfg == 1 ? small_split_kernel<4, 4> : cfg == 2 ? small_split_kernel<8, 3>
-                       : cfg == 3 ? small_split_kernel<2, 4> : small_split_kernel<4, 3>;
+                       : cfg == 3 ? small_split_kernel<4, 3> : cfg == 4 ? small_split_kernel<1, 6>
+                       : cfg == 5 ? small_split_kernel<2, 6> : cfg == 6 ? small_split_kernel<1, 8>
+                       : cfg == 7 ? small_split_kernel<2, 5> : small_split_kernel<2, 4>;
             kern<<<g, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], c.f_S[cur], (uint32_t)C, A, c.t_sorted,
                                     c.cut, c.cut_SL);
         }
