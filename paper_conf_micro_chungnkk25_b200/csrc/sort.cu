@@ -99,6 +99,29 @@ __global__ void kid_table_kernel(const uint64_t *__restrict__ B, uint32_t K, uin
     tab[j] = (uint32_t)(upper_bound(B, (uint64_t)K + 1, j << kBaseShift) - 1);
 }
 
+// Ranking mode per pass from its digit histogram.  MATCH.ANY slows down as
+// the number of distinct digits among a warp's 32 keys approaches 32, while
+// 8 ballots cost the same for any digit mix.  Measured on B200 (C5, per pass
+// ms match/ballot: 14.2/12.0, 9.7/8.8, 8.5/8.6, 7.4/8.3, 7.3/8.6 at expected
+// distinct digits 30.1, 29.8, 26.1, 24.8, 9.9): ballots when E[distinct] >= 27.
+__global__ void rank_mode_kernel(const uint64_t *__restrict__ hist, int p0, int p1, uint64_t n,
+                                 uint32_t *__restrict__ mode) {
+    __shared__ double s_w[8];
+    for (int p = p0; p < p1; p++) {
+        const double q = (double)hist[p * kHistR + threadIdx.x] / (double)n;
+        double e = 1.0 - pow(1.0 - q, 32.0);
+        for (int o = 16; o; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
+        if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = e;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double tot = 0.0;
+            for (int i = 0; i < 8; i++) tot += s_w[i];
+            mode[p] = tot >= 27.0 ? 1u : 0u;
+        }
+        __syncthreads();
+    }
+}
+
 // ---------------------------------------------------------------- one-sweep pass
 struct PassArgs {
     const uint32_t *kid_in, *t_in;      // FIRST: trace columns
@@ -114,6 +137,8 @@ struct PassArgs {
     uint32_t K;
     int shift, pass;
     int nxh;                            // FIRST: key bytes 2 .. 2 + nxh - 1 histogrammed here
+    uint32_t pf;                        // tiles ahead to prefetch into L2 (0 = off)
+    const uint32_t *ballot;             // [pass] 1: equal-digit lanes by 8 ballots, 0: match.any
     uint64_t *hist;                     // [pass][kHistR] global digit counts
     uint64_t *status;                   // [ntiles][R]
     uint32_t *tile_counter;
@@ -150,6 +175,26 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
     __syncthreads();
     const uint32_t tile = s_tile;
     const uint64_t wbase = (uint64_t)tile * TILE + (uint64_t)w * (32 * IT);
+    // L2 prefetch of the tile that will be claimed pf tiles from now: its DRAM
+    // reads overlap this tile's ranking and look-back (tiles are claimed in order)
+    if (a.pf && tid < 2) {
+        const uint64_t pt = (uint64_t)tile + a.pf, p0 = pt * TILE;
+        if (p0 < a.n) {
+            const uint64_t cnt = min((uint64_t)TILE, a.n - p0);
+            const void *src;
+            uint32_t bytes;
+            if (FIRST) {
+                src = tid == 0 ? (const void *)(a.kid_in + p0) : (const void *)(a.t_in + p0);
+                bytes = (uint32_t)(cnt * 4);
+            } else {
+                src = tid == 0 ? (const void *)(a.keys_in + p0) : (const void *)(a.vals_in + p0);
+                bytes = (uint32_t)(cnt * (tid == 0 ? 8 : 4));
+            }
+            bytes &= ~15u;
+            if (bytes && (reinterpret_cast<uintptr_t>(src) & 15) == 0)
+                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+        }
+    }
 
     uint64_t key[IT];
     uint32_t val[IT];
@@ -187,6 +232,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
                 atomicAdd((unsigned long long *)&a.hist[(2 + x) * kHistR + tid], (unsigned long long)s_xh[x * R + tid]);
 
     // warp-level multi-split ranking, in element order
+    const uint32_t ballot = a.ballot[a.pass];
     uint32_t rank[IT];
 #pragma unroll
     for (int j = 0; j < IT; j++) {
@@ -195,7 +241,17 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
         const uint32_t vmask = __ballot_sync(0xffffffffu, valid);
         if (valid) {
             const uint32_t d = (uint32_t)(key[j] >> a.shift) & (R - 1);
-            const uint32_t peers = __match_any_sync(vmask, d);
+            uint32_t peers;
+            if (ballot) {
+                peers = vmask;
+#pragma unroll
+                for (int b = 0; b < kRB; b++) {
+                    const uint32_t bal = __ballot_sync(vmask, (d >> b) & 1u);
+                    peers &= ((d >> b) & 1u) ? bal : ~bal;
+                }
+            } else {
+                peers = __match_any_sync(vmask, d);
+            }
             const uint32_t base = s_whist[w][d];
             const uint32_t below = __popc(peers & ((1u << lane) - 1));
             rank[j] = base + below;
@@ -392,6 +448,29 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     a.B = B;
     a.tab = tab;
     a.nxh = npasses - 2;
+    {
+        static int pf = -1;
+        if (pf < 0) {
+            const char *e = getenv("STEMROOT_SORT_PF");
+            pf = e ? atoi(e) : 3 * c.sms;   // about one wave of resident tiles (measured best)
+        }
+        a.pf = (uint32_t)pf;
+    }
+    // ranking mode per pass (STEMROOT_SORT_RANK=match|ballot forces one)
+    static int rank_force = -2;
+    if (rank_force == -2) {
+        const char *e = getenv("STEMROOT_SORT_RANK");
+        rank_force = !e ? -1 : e[0] == 'b' ? 1 : e[0] == 'm' ? 0 : -1;
+    }
+    uint32_t *mode = c.sort_mode;
+    if (rank_force >= 0) {
+        CK(cudaMemsetAsync(mode, 0, sizeof(uint32_t) * kMaxPasses, st));
+        if (rank_force) CK(cudaMemsetAsync(mode, 1, sizeof(uint32_t) * kMaxPasses, st));   // nonzero bytes
+    } else {
+        rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 0, 2, n, mode);   // key bytes 0, 1: pre-pass histograms
+        c.launches++;
+    }
+    a.ballot = mode;
     a.hist = c.hist;
     a.status = (uint64_t *)c.sort_status;
     a.tile_counter = &c.scalars->tile_counter;
@@ -419,6 +498,10 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         c.launches++;
         c.stage_end(tk, sbytes);
         CK(cudaGetLastError());
+        if (first && rank_force < 0 && npasses > 2) {   // higher bytes: histogrammed by pass 0
+            rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 2, npasses, n, mode);
+            c.launches++;
+        }
         uint64_t *tkk = kin; kin = kout; kout = tkk;
         uint32_t *tv = vin; vin = vout; vout = tv;
     }
