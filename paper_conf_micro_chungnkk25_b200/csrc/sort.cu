@@ -150,7 +150,7 @@ struct PassArgs {
 // multi-split (match.any), global offsets found by decoupled look-back
 // (thread d < 256 owns digit d), then keys are staged in shared memory in
 // tile-sorted order and written out in digit runs (coalesced).
-template <int NT, int IT, bool FIRST, bool LAST>
+template <int NT, int IT, bool FIRST, bool LAST, bool FULL>
 __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesweep_kernel(PassArgs a) {
     constexpr int NW = NT / 32, TILE = NT * IT, R = kR;
     static_assert(NT >= R, "one thread per digit");
@@ -201,7 +201,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
 #pragma unroll
     for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
-        if (i < a.n) {
+        if (FULL || i < a.n) {
             if (FIRST) {
                 key[j] = __ldg(a.B + __ldg(a.kid_in + i)) + (uint64_t)__ldg(a.t_in + i);
                 val[j] = a.row_in ? __ldg(a.row_in + i) : (uint32_t)i;
@@ -218,7 +218,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
     // do not wait for this tile's ranking
 #pragma unroll
     for (int j = 0; j < IT; j++)
-        if (wbase + (uint64_t)j * 32 + lane < a.n) {
+        if (FULL || wbase + (uint64_t)j * 32 + lane < a.n) {
             atomicAdd(&s_cnt[(uint32_t)(key[j] >> a.shift) & (R - 1)], 1u);
             if (FIRST)
                 for (int x = 0; x < a.nxh; x++)
@@ -237,8 +237,8 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
 #pragma unroll
     for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
-        const bool valid = i < a.n;
-        const uint32_t vmask = __ballot_sync(0xffffffffu, valid);
+        const bool valid = FULL || i < a.n;
+        const uint32_t vmask = FULL ? 0xffffffffu : __ballot_sync(0xffffffffu, valid);
         if (valid) {
             const uint32_t d = (uint32_t)(key[j] >> a.shift) & (R - 1);
             uint32_t peers;
@@ -310,7 +310,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
 #pragma unroll
     for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
-        if (i < a.n) {
+        if (FULL || i < a.n) {
             const uint32_t dd = (uint32_t)(key[j] >> a.shift) & (R - 1);
             const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + rank[j];
             s_keys[lp] = key[j];
@@ -337,24 +337,42 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
 }
 
 // ---------------------------------------------------------------- host driver
+// full tiles in one launch (no bounds checks), the ragged last tile in a second
+// launch: its look-back finds every predecessor already inclusive
 template <int NT, int IT, bool FIRST, bool LAST>
-static int launch_pass(const PassArgs &a, cudaStream_t st) {
-    const uint64_t ntiles = (a.n + (uint64_t)NT * IT - 1) / ((uint64_t)NT * IT);
-    const size_t smem = (size_t)NT * IT * (sizeof(uint64_t) + sizeof(uint32_t)) + sizeof(uint16_t) * (NT / 32) * kR;
-    CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)smem));
-    CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                            100));
-    onesweep_kernel<NT, IT, FIRST, LAST><<<(unsigned)ntiles, NT, smem, st>>>(a);
+static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
+    constexpr uint64_t TILE = (uint64_t)NT * IT;
+    const uint64_t full = a.n / TILE, rag = a.n % TILE;
+    const size_t smem = (size_t)TILE * (sizeof(uint64_t) + sizeof(uint32_t)) + sizeof(uint16_t) * (NT / 32) * kR;
+    static bool attr = false;
+    if (!attr) {
+        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true>,
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true>,
+                                cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false>,
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false>,
+                                cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+        attr = true;
+    }
+    if (full) {
+        onesweep_kernel<NT, IT, FIRST, LAST, true><<<(unsigned)full, NT, smem, st>>>(a);
+        (*launches)++;
+    }
+    if (rag) {
+        onesweep_kernel<NT, IT, FIRST, LAST, false><<<1, NT, smem, st>>>(a);
+        (*launches)++;
+    }
     return STEM_OK;
 }
 
 template <int NT, int IT>
-static int launch_pass_cfg(const PassArgs &a, bool first, bool last, cudaStream_t st) {
-    if (first && last) return launch_pass<NT, IT, true, true>(a, st);
-    if (first) return launch_pass<NT, IT, true, false>(a, st);
-    if (last) return launch_pass<NT, IT, false, true>(a, st);
-    return launch_pass<NT, IT, false, false>(a, st);
+static int launch_pass_cfg(const PassArgs &a, bool first, bool last, cudaStream_t st, uint32_t *launches) {
+    if (first && last) return launch_pass<NT, IT, true, true>(a, st, launches);
+    if (first) return launch_pass<NT, IT, true, false>(a, st, launches);
+    if (last) return launch_pass<NT, IT, false, true>(a, st, launches);
+    return launch_pass<NT, IT, false, false>(a, st, launches);
 }
 
 // tile shapes (threads, keys per thread); STEMROOT_SORT_SHAPE picks one for
@@ -373,11 +391,11 @@ static int shape_idx() {
 
 static uint64_t tile_keys() { return (uint64_t)kShapes[shape_idx()].nt * kShapes[shape_idx()].it; }
 
-static int launch_sort_pass(const PassArgs &a, bool first, bool last, cudaStream_t st) {
+static int launch_sort_pass(const PassArgs &a, bool first, bool last, cudaStream_t st, uint32_t *launches) {
     switch (shape_idx()) {
-        case 1: return launch_pass_cfg<384, 10>(a, first, last, st);
-        case 2: return launch_pass_cfg<320, 14>(a, first, last, st);
-        default: return launch_pass_cfg<384, 12>(a, first, last, st);
+        case 1: return launch_pass_cfg<384, 10>(a, first, last, st, launches);
+        case 2: return launch_pass_cfg<320, 14>(a, first, last, st, launches);
+        default: return launch_pass_cfg<384, 12>(a, first, last, st, launches);
     }
 }
 
@@ -494,8 +512,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         const char *sname = first ? "sort_pass_first" : last ? "sort_pass_last" : "sort_pass_mid";
         const uint64_t sbytes = n * ((first ? 8 : 12) + (last ? 8 : 12));
         const int tk = c.stage_begin(sname);
-        CKS(launch_sort_pass(a, first, last, st));
-        c.launches++;
+        CKS(launch_sort_pass(a, first, last, st, &c.launches));
         c.stage_end(tk, sbytes);
         CK(cudaGetLastError());
         if (first && rank_force < 0 && npasses > 2) {   // higher bytes: histogrammed by pass 0
