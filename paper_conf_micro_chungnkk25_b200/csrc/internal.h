@@ -44,6 +44,8 @@ struct DevScalars {
     double est_frac, var_sum;     // sum rn(r_i)/m_i, sum rn(V_i)/m_i
     alignas(16) uint64_t wide_total[4];   // total of a wide (struct) scan
     uint64_t red7[8];                     // multi-GPU reduction staging
+    unsigned long long local_rows;        // rows scanned below the frontier (local subtrees)
+    uint32_t local_depth, pad3;           // deepest ROOT level reached by a local subtree
 };
 
 constexpr int kFixDigits = 6;     // 6 x 32-bit digits in u64 lanes, LSB 2^-72
@@ -150,6 +152,7 @@ struct Ctx {
     // sampled prefix moments (a2): PS1/PS2 every kChunk rows
     uint64_t *PS1 = nullptr; size_t cap_ps1 = 0;
     u128 *PS2 = nullptr; size_t cap_ps2 = 0;
+    uint32_t *TB = nullptr; size_t cap_TB = 0;            // chunk-boundary pairs (t[32j-1], t[32j])
     void *chunk_sq = nullptr; size_t cap_chunk_sq = 0;
     // ROOT frontier (a3/a4)
     uint32_t *f_lo[2] = {nullptr, nullptr}, *f_hi[2] = {nullptr, nullptr}, *f_aoff[2] = {nullptr, nullptr};

@@ -4,13 +4,17 @@
 // Every level processes the whole frontier (all kernels' active clusters at
 // once).  For each cluster the 2-means cut (R5) is the argmax over its cuts k
 // of D_k^2/(k(n-k)), D_k = n S_L(k) - S k, compared exactly:
-//   small_split_kernel  clusters < big_rows(): one warp per 1024-row range of
-//                       the frontier, 32 rows per step, exact-safe pruning
+//   local_root_kernel   clusters < big_rows(): one warp finishes the cluster's
+//                       whole ROOT subtree (cut, Eq. 7/8 decision, children)
+//                       depth first, rows re-read from L1/L2 instead of one
+//                       frontier pass per level
 //   big_split_kernel    clusters >= big_rows(): one block per 65536 rows,
 //                       chunk bounds from the sampled prefix, only chunks that
 //                       may hold the argmax are scanned; big_reduce_kernel
-//   decide_kernel       Eq. 7 vs Eq. 8 per cluster (R6-R9), fixed fp64 order
+//   decide_kernel       Eq. 7 vs Eq. 8 per big cluster (R6-R9), fixed fp64 order
 //   scan + apply        compacts the non-trivial children into the next frontier
+// The decision of a cluster depends on its rows alone, so the order in which
+// clusters are finished does not change the leaves (flags at the cut rows).
 // Cluster totals (S exact u64, Q exact u128) travel with the frontier; only
 // Q_L at the chosen cut is read from the sampled prefix arrays.
 #include <cstdlib>
@@ -30,7 +34,19 @@ static uint64_t big_rows() {
     }
     return v;
 }
-constexpr uint64_t kBigSeg = 65536;                    // rows per block on that path
+constexpr uint64_t kBigSeg = 65536;                    // rows per block on the big-cluster path
+// clusters of < local_rows() rows are finished by local_root_kernel
+// (STEMROOT_LOCAL_ROWS, default 0 = off: measured slower than the level loop
+// on C5)
+__constant__ uint64_t c_loc;
+static uint64_t local_rows() {
+    static uint64_t v = ~0ull;
+    if (v == ~0ull) {
+        const char *e = getenv("STEMROOT_LOCAL_ROWS");
+        v = e ? strtoull(e, nullptr, 10) : 0;
+    }
+    return v;
+}
 
 struct SQ {
     uint64_t s;
@@ -43,8 +59,10 @@ __host__ __device__ __forceinline__ SQ operator-(const SQ &a, const SQ &b) { ret
 // Sums of t and t^2 over every 32-row chunk.  Eight lanes cover one chunk with
 // one uint4 each, so one warp load is 512 contiguous bytes; four loads are in
 // flight per lane.
+// Also writes the chunk-boundary pairs TB[j] = (t[32 j - 1], t[32 j]) that the
+// split bounds read (8 B per chunk instead of two scattered sectors).
 __global__ void __launch_bounds__(256) chunk_sums_kernel(const uint32_t *__restrict__ t, uint64_t n, uint64_t nchunks,
-                                                         SQ *__restrict__ out) {
+                                                         SQ *__restrict__ out, uint32_t *__restrict__ TB) {
     constexpr int kUnroll = 4;
     const int lane = threadIdx.x & 31, sub = lane & 7, grp = lane >> 3;
     const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -80,7 +98,12 @@ __global__ void __launch_bounds__(256) chunk_sums_kernel(const uint32_t *__restr
                 qlo = nl;
             }
             const uint64_t j = base + u * 4 + grp;
-            if (sub == 0 && j < nchunks) out[j] = SQ{s, ((u128)qhi << 64) | qlo};
+            if (sub == 0 && j < nchunks) {
+                out[j] = SQ{s, ((u128)qhi << 64) | qlo};
+                TB[2 * j + 1] = v[u].x;                 // t[32 j]
+                if (j == 0) TB[0] = 0;
+            }
+            if (sub == 7 && j + 1 < nchunks) TB[2 * (j + 1)] = v[u].w;   // t[32 (j + 1) - 1]
         }
     }
 }
@@ -91,7 +114,8 @@ int prefix_moments(Ctx &c, uint64_t n) {
     CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(nchunks + 1) + 1) * sizeof(SQ)));
     const int tk = c.stage_begin("prefix_moments");
     SQ *cs = (SQ *)c.chunk_sq;
-    chunk_sums_kernel<<<c.sms * 8, 256, 0, c.stream>>>(c.t_sorted, n, nchunks, cs);
+    CKS(c.ensure(c.TB, c.cap_TB, sizeof(uint32_t) * 2 * (nchunks + 1)));
+    chunk_sums_kernel<<<c.sms * 8, 256, 0, c.stream>>>(c.t_sorted, n, nchunks, cs, c.TB);
     c.launches++;
     uint64_t *PS1 = c.PS1;
     u128 *PS2 = c.PS2;
@@ -157,88 +181,245 @@ __device__ __forceinline__ Cand shfl_cand_xor(const Cand &a, int m) {
     return r;
 }
 
-// ---------------------------------------------------------------- small clusters: a warp per range
-// Clusters of < big_rows() rows.  Warp g owns every cluster whose active offset
-// starts in [g*kSmallRange, (g+1)*kSmallRange) and scans it 32 rows at a time:
-// coalesced loads, a warp scan gives S_L, every valid cut is scored exactly
-// (eval_cut).  A 32-row chunk is skipped when the concavity bound of its cuts
-// is below the best candidate of the cluster so far (exact-safe, see
-// big_split_kernel).  No shared memory, no cross-warp reduction.
-constexpr uint64_t kSmallRange = 1024;
-template <int kSmallQ, int MINB>   // 32-row chunks loaded per step; min resident blocks
-__global__ void __launch_bounds__(256, MINB) small_split_kernel(const uint32_t *__restrict__ f_lo,
-                                                          const uint32_t *__restrict__ f_hi,
-                                                          const uint32_t *__restrict__ aoff,
-                                                          const uint64_t *__restrict__ f_S, uint32_t C, uint64_t A,
-                                                          const uint32_t *__restrict__ t, uint32_t *__restrict__ cut,
-                                                          uint64_t *__restrict__ cut_SL) {
-    const uint64_t g = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+// ---------------------------------------------------------------- warp argmax over one cluster
+// Best valid cut of t[lo, lo + n) (S = its sum), 32 rows per step: coalesced
+// loads, a warp scan gives S_L, every valid cut is scored exactly (eval_cut).
+// A 32-row chunk is skipped when the concavity bound of its cuts is below the
+// best candidate so far (exact-safe, see big_split_kernel).  Every lane
+// returns the same candidate.
+__device__ __forceinline__ Cand warp_scan_cut(const uint32_t *__restrict__ t, uint64_t lo, uint64_t n, uint64_t S) {
+    constexpr int kQ = 2;   // 32-row chunks loaded per step
     const int lane = threadIdx.x & 31;
-    const uint64_t r0 = g * kSmallRange;
-    if (r0 >= A) return;
-    const uint64_t r1 = r0 + kSmallRange;
     const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
-    for (uint32_t c = (uint32_t)lower_bound(aoff, C, (uint32_t)r0); c < C && aoff[c] < r1; c++) {
+    Cand best = no_cand();
+    double thr = 0.0;
+    uint64_t SLb = 0;
+    uint32_t tlast = 0;
+    for (uint64_t kb = 0; kb < n; kb += 32 * kQ) {
+        uint32_t tq[kQ];
+#pragma unroll
+        for (int q = 0; q < kQ; q++) {
+            const uint64_t k = kb + 32 * q + lane;
+            tq[q] = k < n ? t[lo + k] : 0u;
+        }
+#pragma unroll
+        for (int q = 0; q < kQ; q++) {
+            const uint64_t k0 = kb + 32 * q;
+            if (k0 >= n) break;
+            const uint64_t k = k0 + lane;
+            const bool in = k < n;
+            const uint32_t tc = tq[q];
+            uint32_t tp = __shfl_up_sync(0xffffffffu, tc, 1);
+            if (lane == 0) tp = tlast;
+            uint64_t incl = tc;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += v;
+            }
+            // upper bound of the chunk's scores from its first cut (warp-uniform)
+            const uint64_t cnt = min((uint64_t)32, n - k0);
+            const uint32_t t0 = __shfl_sync(0xffffffffu, tc, 0);
+            const u128 ad0 = (u128)S * k0 - (u128)n * SLb;
+            const uint64_t nt0 = n * (uint64_t)t0;
+            const double slope = S > nt0 ? __ull2double_rn(S - nt0) : 0.0;
+            const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad0 >> 64), (uint64_t)ad0),
+                                                   __dmul_rn(slope, (double)(cnt - 1))), up);
+            const uint64_t kf = max(k0, (uint64_t)1), kl = min(k0 + cnt - 1, n - 1);
+            double ub = 0.0;
+            if (kf <= kl) {
+                const double pmin =
+                    fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
+                ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
+            }
+            if (ub >= thr) {
+                if (in && k >= 1 && tp < tc) eval_cut((uint32_t)k, n, S, SLb + incl - tc, best);
+                double lb = best.k ? __dmul_rn(__ddiv_rn(best.x, best.dp), dn) : 0.0;
+#pragma unroll
+                for (int o = 16; o; o >>= 1) lb = fmax(lb, __shfl_xor_sync(0xffffffffu, lb, o));
+                thr = fmax(thr, lb);
+            }
+            SLb += __shfl_sync(0xffffffffu, incl, 31);
+            tlast = __shfl_sync(0xffffffffu, tc, 31);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const Cand v = shfl_cand_xor(best, o);
+        if (better(v, best)) best = v;
+    }
+    return best;
+}
+
+// lower bound of x / p (x, p > 0): fast reciprocal refined by one Newton step,
+// scaled down by 2^-30 to cover its error (a smaller lower bound only prunes less)
+__device__ __forceinline__ double div_lower(double x, double p) {
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(p));
+    r = __fma_rn(r, __fma_rn(-p, r, 1.0), r);
+    return __dmul_rn(__dmul_rn(x, r), 1.0 - 0x1p-30);
+}
+
+// Warp scan of the rows [ra, rb) of a cluster starting at lo (S_L at ra = SLa):
+// every valid cut is scored exactly into best.
+__device__ __forceinline__ void scan_chunk(const uint32_t *__restrict__ t, uint64_t lo, uint64_t n, uint64_t S,
+                                           uint64_t ra, uint64_t rb, uint64_t SLa, Cand &best) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t row = ra + lane;
+    const bool in = row < rb;
+    const uint32_t tc = in ? t[row] : 0u;
+    uint32_t tp = __shfl_up_sync(0xffffffffu, tc, 1);
+    if (lane == 0) tp = row > lo ? t[row - 1] : 0u;
+    uint64_t incl = tc;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += v;
+    }
+    const uint64_t k = row - lo;
+    if (in && k >= 1 && tp < tc) eval_cut((uint32_t)k, n, S, SLa + incl - tc, best);
+}
+
+// Best valid cut k with lo + k in [r0, r1) of the cluster [lo, lo + n) (sum S,
+// base = sum of t before lo), by chunk bounds: the rows are cut into 32-row
+// chunks aligned to the sampled prefix; lane i bounds chunk i from S_L at its
+// start (PS1, exact) and t there (TB), and scores the chunk start when it is a
+// valid cut (a real candidate: a lower bound of the argmax).  Only chunks
+// whose bound reaches the best lower bound are scanned row by row, and every
+// scored candidate raises that threshold.  With cthr != NULL the threshold is
+// shared with the other warps of the cluster (atomic max of the bits of a
+// positive double).  Exact: a pruned chunk cannot hold a candidate scoring >=
+// an existing one, so neither the argmax nor a tie is lost.  At most
+// 32 * kMaxRounds chunks; every lane returns the same candidate.
+constexpr int kMaxRounds = 3;
+__device__ __forceinline__ Cand warp_range_best(const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
+                                                const uint32_t *__restrict__ TB, uint64_t lo, uint64_t n, uint64_t S,
+                                                uint64_t base, uint64_t r0, uint64_t r1,
+                                                unsigned long long *cthr) {
+    const int lane = threadIdx.x & 31;
+    const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
+    const uint64_t q0 = r0 >> kChunkLog, nq = ((r1 - 1) >> kChunkLog) - q0 + 1;
+    double d2[kMaxRounds], pm[kMaxRounds];
+    uint64_t sla[kMaxRounds];
+    double lbm = 0.0;
+#pragma unroll
+    for (int r = 0; r < kMaxRounds; r++) {   // loads of every round in flight first
+        const uint64_t i = (uint64_t)r * 32 + lane;
+        sla[r] = 0;
+        pm[r] = 0.0;
+        d2[r] = 0.0;
+        if (i < nq) {
+            const uint64_t q = q0 + i;
+            sla[r] = PS1[q];
+            const uint2 tb = reinterpret_cast<const uint2 *>(TB)[q];
+            pm[r] = __longlong_as_double((long long)(((uint64_t)tb.y << 32) | tb.x));   // parked
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < kMaxRounds; r++) {
+        const uint64_t i = (uint64_t)r * 32 + lane;
+        if (i < nq) {
+            const uint64_t q = q0 + i;
+            const uint64_t ra = max(r0, q << kChunkLog), rb = min(r1, (q + 1) << kChunkLog);
+            const uint64_t pk = (uint64_t)__double_as_longlong(pm[r]);
+            uint32_t ta = (uint32_t)(pk >> 32), tprev = (uint32_t)pk;
+            uint64_t p = sla[r];
+            if (ra & (kChunk - 1)) {   // unaligned start (the range's first chunk)
+                for (uint64_t x = ra & ~(kChunk - 1); x < ra; x++) p += t[x];
+                ta = t[ra];
+                tprev = ra > lo ? t[ra - 1] : 0u;
+            }
+            const uint64_t SL = p - base;
+            sla[r] = SL;
+            const uint64_t ka = ra - lo, cnt = rb - ra;
+            const u128 ad = (u128)S * ka - (u128)n * SL;
+            const uint64_t nta = n * (uint64_t)ta;
+            const double slope = S > nta ? __ull2double_rn(S - nta) : 0.0;
+            const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
+            const double dub = __dmul_rn(__dadd_rn(dD, __dmul_rn(slope, (double)(cnt - 1))), up);
+            const uint64_t kf = max(ka, (uint64_t)1), kl = min(ka + cnt - 1, n - 1);
+            pm[r] = 0.0;
+            if (kf <= kl) {
+                pm[r] = fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
+                d2[r] = __dmul_rn(__dmul_rn(dub, dub), 1.0 + 0x1p-43);
+            }
+            if (ka >= 1 && tprev < ta)   // the chunk start is a real candidate
+                lbm = fmax(lbm, div_lower(__dmul_rn(dD, dD), __dmul_rn((double)ka, (double)(n - ka))));
+        }
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));
+    double thr = __dmul_rn(lbm, dn);
+    if (cthr) {
+        unsigned long long prev = 0;
+        if (lane == 0) prev = atomicMax(cthr, (unsigned long long)__double_as_longlong(thr));
+        prev = __shfl_sync(0xffffffffu, prev, 0);
+        thr = fmax(thr, __longlong_as_double((long long)prev));   // positive doubles order as integers
+    }
+    Cand best = no_cand();
+#pragma unroll
+    for (int r = 0; r < kMaxRounds; r++) {
+        // kept when d2 >= thr * pmin (d2 = RN(dub^2) (1 + 2^-43) covers the roundings)
+        uint32_t live = __ballot_sync(0xffffffffu, d2[r] > 0.0 && d2[r] >= __dmul_rn(thr, pm[r]));
+        while (live) {
+            const int src = __ffs(live) - 1;
+            live &= live - 1;
+            const double sd2 = __shfl_sync(0xffffffffu, d2[r], src), spm = __shfl_sync(0xffffffffu, pm[r], src);
+            if (sd2 < __dmul_rn(thr, spm)) continue;   // threshold raised meanwhile
+            const uint64_t q = q0 + (uint64_t)r * 32 + src;
+            const uint64_t SLa = __shfl_sync(0xffffffffu, sla[r], src);
+            scan_chunk(t, lo, n, S, max(r0, q << kChunkLog), min(r1, (q + 1) << kChunkLog), SLa, best);
+            double lb = best.k ? div_lower(best.x, best.dp) : 0.0;
+#pragma unroll
+            for (int o = 16; o; o >>= 1) lb = fmax(lb, __shfl_xor_sync(0xffffffffu, lb, o));
+            thr = fmax(thr, __dmul_rn(lb, dn));
+        }
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const Cand v = shfl_cand_xor(best, o);
+        if (better(v, best)) best = v;
+    }
+    return best;
+}
+
+// warp: sum of t before lo (pref1(lo) = PS1[lo / 32] + partial chunk)
+__device__ __forceinline__ uint64_t warp_pref1(const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
+                                               uint64_t lo) {
+    const int lane = threadIdx.x & 31;
+    uint64_t part = 0;
+    const uint64_t b0 = lo & ~(kChunk - 1);
+    if (b0 + lane < lo) part = t[b0 + lane];
+#pragma unroll
+    for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+    return part + PS1[lo >> kChunkLog];
+}
+
+// Best valid cut of a whole cluster: the plain scan for <= 64 rows, chunk bounds
+// up to 32 * kMaxRounds chunks, else the plain scan (only reached when
+// big_rows() is raised past kSeg).
+__device__ __forceinline__ Cand warp_best_cut(const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
+                                              const uint32_t *__restrict__ TB, uint64_t lo, uint64_t n, uint64_t S) {
+    const uint64_t nq = ((lo + n - 1) >> kChunkLog) - (lo >> kChunkLog) + 1;
+    if (n <= 64 || nq > 32 * kMaxRounds) return warp_scan_cut(t, lo, n, S);
+    return warp_range_best(t, PS1, TB, lo, n, S, warp_pref1(t, PS1, lo), lo, lo + n, nullptr);
+}
+
+// ---------------------------------------------------------------- mid clusters: a warp per cluster
+// Clusters of local_rows() .. big_rows() rows, one warp each (grid-stride).
+__global__ void __launch_bounds__(256, 4) small_split_kernel(const uint32_t *__restrict__ f_lo,
+                                                          const uint32_t *__restrict__ f_hi,
+                                                          const uint64_t *__restrict__ f_S, uint32_t C,
+                                                          const uint32_t *__restrict__ t,
+                                                          const uint64_t *__restrict__ PS1,
+                                                          const uint32_t *__restrict__ TB, uint32_t *__restrict__ cut,
+                                                          uint64_t *__restrict__ cut_SL) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
         const uint64_t lo = f_lo[c], n = f_hi[c] - lo;
-        if (n >= c_big) continue;
-        const uint64_t S = f_S[c];
-        Cand best = no_cand();
-        double thr = 0.0;
-        uint64_t SLb = 0;
-        uint32_t tlast = 0;
-        for (uint64_t kb = 0; kb < n; kb += 32 * kSmallQ) {
-            uint32_t tq[kSmallQ];   // kSmallQ chunks' loads in flight
-#pragma unroll
-            for (int q = 0; q < kSmallQ; q++) {
-                const uint64_t k = kb + 32 * q + lane;
-                tq[q] = k < n ? t[lo + k] : 0u;
-            }
-#pragma unroll
-            for (int q = 0; q < kSmallQ; q++) {
-                const uint64_t k0 = kb + 32 * q;
-                if (k0 >= n) break;
-                const uint64_t k = k0 + lane;
-                const bool in = k < n;
-                const uint32_t tc = tq[q];
-                uint32_t tp = __shfl_up_sync(0xffffffffu, tc, 1);
-                if (lane == 0) tp = tlast;
-                uint64_t incl = tc;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
-                    if (lane >= o) incl += v;
-                }
-                // upper bound of the chunk's scores from its first cut (warp-uniform)
-                const uint64_t cnt = min((uint64_t)32, n - k0);
-                const uint32_t t0 = __shfl_sync(0xffffffffu, tc, 0);
-                const u128 ad0 = (u128)S * k0 - (u128)n * SLb;
-                const uint64_t nt0 = n * (uint64_t)t0;
-                const double slope = S > nt0 ? __ull2double_rn(S - nt0) : 0.0;
-                const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad0 >> 64), (uint64_t)ad0),
-                                                       __dmul_rn(slope, (double)(cnt - 1))), up);
-                const uint64_t kf = max(k0, (uint64_t)1), kl = min(k0 + cnt - 1, n - 1);
-                double ub = 0.0;
-                if (kf <= kl) {
-                    const double pmin =
-                        fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
-                    ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
-                }
-                if (ub >= thr) {
-                    if (in && k >= 1 && tp < tc) eval_cut((uint32_t)k, n, S, SLb + incl - tc, best);
-                    double lb = best.k ? __dmul_rn(__ddiv_rn(best.x, best.dp), dn) : 0.0;
-#pragma unroll
-                    for (int o = 16; o; o >>= 1) lb = fmax(lb, __shfl_xor_sync(0xffffffffu, lb, o));
-                    thr = fmax(thr, lb);
-                }
-                SLb += __shfl_sync(0xffffffffu, incl, 31);
-                tlast = __shfl_sync(0xffffffffu, tc, 31);
-            }
-        }
-#pragma unroll
-        for (int o = 16; o; o >>= 1) {
-            const Cand v = shfl_cand_xor(best, o);
-            if (better(v, best)) best = v;
-        }
+        if (n < c_loc || n >= c_big) continue;
+        const Cand best = warp_best_cut(t, PS1, TB, lo, n, f_S[c]);
         if (lane == 0) {
             cut[c] = best.k;
             cut_SL[c] = best.SL;
@@ -278,6 +459,7 @@ struct BigArgs {
     const uint32_t *f_lo, *f_hi;
     const uint64_t *f_S, *PS1;
     const uint32_t *t;
+    const uint32_t *TB;        // chunk-boundary pairs (t[32 j - 1], t[32 j])
     unsigned long long *thr;   // per cluster: bits of the best lower bound so far
     Cand *part;                // per entry
 };
@@ -293,9 +475,11 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
     __shared__ double s_thr[kBigThreads / 32];
     __shared__ Cand s_best[kBigThreads / 32];
     __shared__ uint64_t s_base;
-    if (blockIdx.x >= *a.count) return;
-    const BigEntry e = a.ent[blockIdx.x];
+    const uint32_t n_ent = *a.count;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    for (uint32_t eb = blockIdx.x; eb < n_ent; eb += gridDim.x) {
+    __syncthreads();   // shared memory of the previous entry
+    const BigEntry e = a.ent[eb];
     const uint64_t lo = a.f_lo[e.c], hi = a.f_hi[e.c], n = hi - lo, S = a.f_S[e.c];
     const uint64_t r0 = lo + (uint64_t)e.seg * kBigSeg, r1 = min(r0 + kBigSeg, hi);
     if (w == 0) {   // pref1(lo) = PS1[lo/32] + partial chunk
@@ -325,7 +509,9 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
         }
         const uint64_t SL = pa - s_base;       // S_L at k_a = ra - lo (exact)
         const uint32_t ka = (uint32_t)(ra - lo);
-        const uint32_t ta = a.t[ra];
+        const bool al = (ra & (kChunk - 1)) == 0;
+        const uint2 tb = al ? reinterpret_cast<const uint2 *>(a.TB)[ra >> kChunkLog] : make_uint2(0u, 0u);
+        const uint32_t ta = al ? tb.y : a.t[ra];
         s_sl[i] = SL;
         const u128 ad = (u128)S * ka - (u128)n * SL;
         const uint64_t nta = n * (uint64_t)ta;
@@ -340,7 +526,7 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
             ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
         }
         s_ub[i] = ub;
-        if (ka >= 1 && a.t[ra - 1] < ta) {      // the chunk start is a real candidate
+        if (ka >= 1 && (al ? tb.x : a.t[ra - 1]) < ta) {   // the chunk start is a real candidate
             const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
             lbm = fmax(lbm, __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)ka, (double)(n - ka))), dn));
         }
@@ -389,7 +575,8 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
     if (tid == 0) {
         for (int k = 1; k < kBigThreads / 32; k++)
             if (better(s_best[k], best)) best = s_best[k];
-        a.part[blockIdx.x] = best;
+        a.part[eb] = best;
+    }
     }
 }
 
@@ -447,41 +634,170 @@ __device__ __forceinline__ double eq6_m(double g, double mu, double V, int clamp
     return m;
 }
 
-__global__ void __launch_bounds__(256) decide_kernel(DecideArgs a) {
-    const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= a.C) return;
-    const uint32_t lo = a.f_lo[c], hi = a.f_hi[c], k = a.cut[c];
-    const uint32_t mid = lo + k;
-    const uint64_t n = hi - lo, nL = k, nR = n - k;
-    const uint64_t S = a.f_S[c], SL = a.cut_SL[c], SR = S - SL;
-    const u128 Q = a.f_Q[c];
-    uint64_t s_lo, s_mid;
-    u128 q_lo, q_mid;
-    pref12(a.PS1, a.PS2, a.t, lo, s_lo, q_lo);
-    pref12(a.PS1, a.PS2, a.t, mid, s_mid, q_mid);
-    const u128 QL = q_mid - q_lo, QR = Q - QL;
+// Eq. 7 vs Eq. 8 for a cluster (n, S, Q) cut at k (k >= 1) with left sums
+// (SL, QL): true when the split lowers the sample cost (strict).
+__device__ __forceinline__ bool split_pays(uint64_t n, uint64_t S, u128 Q, uint64_t k, uint64_t SL, u128 QL,
+                                           double eps, double z, double k2, int clamp) {
+    const uint64_t nL = k, nR = n - k, SR = S - SL;
+    const u128 QR = Q - QL;
     const u128 V = (u128)n * Q - (u128)S * S;
     const u128 VL = (u128)nL * QL - (u128)SL * SL, VR = (u128)nR * QR - (u128)SR * SR;
     // Eq. 7: tau_old = m * Xbar, m from Eq. 3
     const double mu = __ddiv_rn(rn64(S), rn64(n));
-    const double tau_old = __dmul_rn(eq3_m(V, S, a.k2, a.clamp), mu);
+    const double tau_old = __dmul_rn(eq3_m(V, S, k2, clamp), mu);
     // Eq. 8 with Eq. 6 (corrected numerator) over {L, R}, c from the parent's total
     const double muL = __ddiv_rn(rn64(SL), rn64(nL)), muR = __ddiv_rn(rn64(SR), rn64(nR));
     const double dVL = rn128(VL), dVR = rn128(VR);
-    const double w = __ddiv_rn(__dmul_rn(a.eps, rn64(S)), a.z);
+    const double w = __ddiv_rn(__dmul_rn(eps, rn64(S)), z);
     const double cc = __dmul_rn(w, w);
     const double ssum = __dadd_rn(__dsqrt_rn(__dmul_rn(muL, dVL)), __dsqrt_rn(__dmul_rn(muR, dVR)));
     const double g = __ddiv_rn(ssum, cc);
-    const double mL = eq6_m(g, muL, dVL, a.clamp), mR = eq6_m(g, muR, dVR, a.clamp);
+    const double mL = eq6_m(g, muL, dVL, clamp), mR = eq6_m(g, muR, dVR, clamp);
     const double tau_new = __dadd_rn(__dmul_rn(mL, muL), __dmul_rn(mR, muR));
+    return tau_new < tau_old;
+}
+
+// clusters of >= local_rows() rows (the local kernel finishes the others)
+__global__ void __launch_bounds__(256) decide_kernel(DecideArgs a) {
+    const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= a.C) return;
+    const uint32_t lo = a.f_lo[c], hi = a.f_hi[c], k = a.cut[c];
+    const uint64_t n = hi - lo;
+    if (n < c_loc) {   // finished by local_root_kernel
+        a.cnt_sz[c] = 0;
+        return;
+    }
+    const uint32_t mid = lo + k;
+    const uint64_t nL = k, nR = n - k;
+    const uint64_t S = a.f_S[c], SL = a.cut_SL[c];
+    uint64_t s_lo, s_mid;
+    u128 q_lo, q_mid;
+    pref12(a.PS1, a.PS2, a.t, lo, s_lo, q_lo);
+    pref12(a.PS1, a.PS2, a.t, mid, s_mid, q_mid);
+    const u128 QL = q_mid - q_lo;
     uint64_t cs = 0;
-    if (k != 0 && tau_new < tau_old) {                  // strict
+    if (k != 0 && split_pays(n, S, a.f_Q[c], k, SL, QL, a.eps, a.z, a.k2, a.clamp)) {
         a.flags[mid] = 1;
         const bool ntL = nontrivial(a.t, lo, mid), ntR = nontrivial(a.t, mid, hi);
         cs = ((uint64_t)(ntL + ntR) << 32) | (uint64_t)((ntL ? nL : 0) + (ntR ? nR : 0));
     }
     a.cut_QL[c] = QL;
     a.cnt_sz[c] = cs;
+}
+
+// ---------------------------------------------------------------- local subtrees
+// One warp per frontier cluster of < local_rows() rows: cut (warp_best_cut),
+// decision (split_pays, Q_L from the sampled prefix), then the children,
+// depth first; the larger child waits on a per-warp stack and the smaller is
+// processed next, so the stack holds at most log2(local_rows()) nodes.  Writes
+// flags at the cuts; the cluster leaves the frontier.
+constexpr int kLocalStack = 24;
+struct LNode {
+    uint64_t S;
+    u128 Q;
+    uint32_t lo, hi, depth, pad;
+};
+
+struct LocalArgs {
+    const uint32_t *f_lo, *f_hi;
+    const uint64_t *f_S;
+    const u128 *f_Q;
+    uint32_t C, level;
+    const uint64_t *PS1;
+    const u128 *PS2;
+    const uint32_t *t, *TB;
+    uint8_t *flags;
+    double eps, z, k2;
+    int clamp;
+    unsigned long long *rows;   // stats: rows scanned
+    uint32_t *depth;            // stats: deepest level reached (1-based)
+    uint32_t *err;
+};
+
+// warp: sum of t^2 over [x & ~31, x) (the partial chunk of a sampled prefix), all lanes
+__device__ __forceinline__ u128 warp_partial_sq(const uint32_t *t, uint64_t x) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t b = x & ~(kChunk - 1);
+    uint64_t v = 0;
+    if (b + lane < x) {
+        const uint64_t tv = t[b + lane];
+        v = tv * tv;
+    }
+    u128 s = v;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const uint64_t lo_ = __shfl_xor_sync(0xffffffffu, (uint64_t)s, o);
+        const uint64_t hi_ = __shfl_xor_sync(0xffffffffu, (uint64_t)(s >> 64), o);
+        s += ((u128)hi_ << 64) | lo_;
+    }
+    return s;
+}
+
+__global__ void __launch_bounds__(256) local_root_kernel(LocalArgs a) {
+    __shared__ LNode s_stack[8][kLocalStack];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    uint64_t rows = 0;
+    uint32_t dmax = 0;
+    for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < a.C; c += nwarps) {
+        LNode cur;
+        cur.lo = a.f_lo[c];
+        cur.hi = a.f_hi[c];
+        if ((uint64_t)(cur.hi - cur.lo) >= c_loc) continue;
+        cur.S = a.f_S[c];
+        cur.Q = a.f_Q[c];
+        cur.depth = a.level;
+        int sp = 0;
+        while (true) {   // cur is non-trivial
+            const uint64_t n = cur.hi - cur.lo;
+            if (cur.depth > a.level) rows += n;   // the frontier level counts the root node
+            dmax = max(dmax, cur.depth + 1);
+            const Cand b = warp_best_cut(a.t, a.PS1, a.TB, cur.lo, n, cur.S);
+            bool have = false;
+            LNode nx;
+            if (b.k != 0) {
+                const uint32_t mid = cur.lo + b.k;
+                // Q_L = P2(mid) - P2(lo) from the sampled prefix (exact, mod 2^128)
+                const u128 QL = (a.PS2[mid >> kChunkLog] + warp_partial_sq(a.t, mid)) -
+                                (a.PS2[cur.lo >> kChunkLog] + warp_partial_sq(a.t, cur.lo));
+                if (split_pays(n, cur.S, cur.Q, b.k, b.SL, QL, a.eps, a.z, a.k2, a.clamp)) {
+                    if (lane == 0) a.flags[mid] = 1;
+                    LNode L{b.SL, QL, cur.lo, mid, cur.depth + 1, 0};
+                    LNode R{cur.S - b.SL, cur.Q - QL, mid, cur.hi, cur.depth + 1, 0};
+                    const bool ntL = nontrivial(a.t, cur.lo, mid), ntR = nontrivial(a.t, mid, cur.hi);
+                    if (ntL && ntR) {
+                        const bool lbig = (mid - cur.lo) >= (cur.hi - mid);
+                        if (sp == kLocalStack) {   // cannot happen: sizes halve along the stack
+                            if (lane == 0) atomicOr(a.err, 4u);
+                            break;
+                        }
+                        if (lane == 0) s_stack[w][sp] = lbig ? L : R;
+                        sp++;
+                        nx = lbig ? R : L;
+                        have = true;
+                    } else if (ntL) {
+                        nx = L;
+                        have = true;
+                    } else if (ntR) {
+                        nx = R;
+                        have = true;
+                    }
+                }
+            }
+            if (!have) {
+                if (sp == 0) break;
+                __syncwarp();
+                nx = s_stack[w][--sp];
+            }
+            __syncwarp();
+            cur = nx;
+        }
+    }
+    // stats (one atomic per warp)
+    if (lane == 0 && rows) {
+        atomicAdd(a.rows, (unsigned long long)rows);
+        atomicMax(a.depth, dmax);
+    }
 }
 
 // ---------------------------------------------------------------- frontier bookkeeping
@@ -521,6 +837,8 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
     {
         const uint64_t b = big_rows();
         CK(cudaMemcpyToSymbolAsync(c_big, &b, sizeof(b), 0, cudaMemcpyHostToDevice, st));
+        const uint64_t l = local_rows() < b ? local_rows() : b;
+        CK(cudaMemcpyToSymbolAsync(c_loc, &l, sizeof(l), 0, cudaMemcpyHostToDevice, st));
     }
     CKS(stem_only_leaves(c, n, K));
     // initial frontier: non-trivial kernel groups, in kernel order, with exact S and Q
@@ -570,20 +888,23 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(C) + 1) * sizeof(uint64_t)));
         const int nxt = cur ^ 1;
         CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
+        const int tk_l = c.stage_begin("root_local");
+        if (local_rows() > 0) {
+            LocalArgs la{c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], (uint32_t)C, levels - 1, c.PS1, c.PS2,
+                         c.t_sorted, c.TB, c.flags, eps, z, k2, clamp, &c.scalars->local_rows, &c.scalars->local_depth,
+                         &c.scalars->err};
+            const uint64_t blocks = (C + 7) / 8;
+            local_root_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 64), 256, 0, st>>>(la);
+            c.launches++;
+        }
+        c.stage_end(tk_l, 4 * A);
+        CK(cudaGetLastError());
         const int tk_s = c.stage_begin("root_split");
-        {
-            const unsigned g = (unsigned)(((A + kSmallRange - 1) / kSmallRange * 32 + 255) / 256);
-            static int cfg = -1;
-            if (cfg < 0) {
-                const char *e = getenv("STEMROOT_SMALL_CFG");
-                cfg = e ? atoi(e) : 0;
-            }
-            auto *kern = cfg == 1 ? small_split_kernel<4, 4> : cfg == 2 ? small_split_kernel<8, 3>
-                       : cfg == 3 ? small_split_kernel<4, 3> : cfg == 4 ? small_split_kernel<1, 6>
-                       : cfg == 5 ? small_split_kernel<2, 6> : cfg == 6 ? small_split_kernel<1, 8>
-                       : cfg == 7 ? small_split_kernel<2, 5> : small_split_kernel<2, 4>;
-            kern<<<g, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_aoff[cur], c.f_S[cur], (uint32_t)C, A, c.t_sorted,
-                                    c.cut, c.cut_SL);
+        if (local_rows() < big_rows()) {
+            const uint64_t blocks = (C + 7) / 8;
+            small_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, st>>>(
+                c.f_lo[cur], c.f_hi[cur], c.f_S[cur], (uint32_t)C, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
+            c.launches++;
         }
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
         const uint64_t max_ent = A / kBigSeg + A / big_rows() + 1;
@@ -596,9 +917,9 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CK(cudaMemsetAsync(c.big_thr, 0, sizeof(unsigned long long) * C, st));
         big_entries_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, ent,
                                                                        first_ent, &c.scalars->big_count);
-        BigArgs ba{ent, &c.scalars->big_count, c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.PS1, c.t_sorted,
+        BigArgs ba{ent, &c.scalars->big_count, c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.PS1, c.t_sorted, c.TB,
                    (unsigned long long *)c.big_thr, (Cand *)c.big_part};
-        big_split_kernel<<<(unsigned)max_ent, kBigThreads, 0, st>>>(ba);
+        big_split_kernel<<<(unsigned)min(max_ent, (uint64_t)c.sms * 8), kBigThreads, 0, st>>>(ba);
         c.launches += 2;
         big_reduce_kernel<<<(unsigned)min(C, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, first_ent,
                                                       (const Cand *)c.big_part, c.cut, c.cut_SL);
@@ -642,7 +963,12 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CKS(read_frontier_total(c, C, A));
         cur = nxt;
     }
-    c.stats.levels = levels;
+    DevScalars hs;
+    CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (hs.err & 4u) return STEM_E_CUDA;   // local stack overflow (unreachable)
+    c.stats.levels = levels > hs.local_depth ? levels : hs.local_depth;
+    c.stats.active_rows += hs.local_rows;
     return STEM_OK;
 }
 
