@@ -265,6 +265,7 @@ def run_ours(a):
                    "l2": "inputs 8 B/row x rows >> 126 MB L2 (no flush needed)" if n_local >= 50_000_000
                    else "inputs fit in L2: latency-bound workload",
                    "sort_key_bits": st["key_bits"], "sort_passes": st["sort_passes"],
+                   "sort_row_bits_in_key": st["pack_bits"], "ambiguous_samples": st["ambiguous_samples"],
                    "root_levels": st["levels"], "clusters": dplan["n_clusters"], "samples": dplan["n_samples"],
                    "active_rows_over_levels": st["active_rows"]},
         "clocks": ck,

@@ -138,6 +138,8 @@ typedef struct stem_stats {
     uint64_t active_rows;      /* sum over levels of rows in the ROOT frontier                   */
     uint64_t n_clusters, n_samples;
     double   ssum;             /* RN(exact sum_i sqrt(mu_i V_i)) of the global KKT solve          */
+    uint32_t pack_bits;        /* low row bits carried inside the sort key (0: row payload mode)  */
+    uint32_t ambiguous_samples;/* samples whose row needed the run scan (packed mode)            */
 } stem_stats;
 
 /* Per-stage device time of the last plan (stem_ctx_enable_timing).  bytes is

@@ -102,7 +102,8 @@ class stem_device_plan(C.Structure):
 class stem_stats(C.Structure):
     _fields_ = [("key_bits", C.c_uint32), ("sort_passes", C.c_uint32), ("levels", C.c_uint32),
                 ("kernel_launches", C.c_uint32), ("active_rows", C.c_uint64), ("n_clusters", C.c_uint64),
-                ("n_samples", C.c_uint64), ("ssum", C.c_double)]
+                ("n_samples", C.c_uint64), ("ssum", C.c_double), ("pack_bits", C.c_uint32),
+                ("ambiguous_samples", C.c_uint32)]
 
 
 class stem_stage_time(C.Structure):

@@ -146,7 +146,7 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
             met = c.in_met;
         }
     }
-    CKS(sort_trace(c, kid, t, nullptr, n, K));        // a1
+    CKS(sort_trace(c, kid, t, nullptr, n, K, !o.census_cap));   // a1
     CKS(prefix_moments(c, n));                        // a2
     if (o.root) {
         CKS(root_levels(c, n, K, eps, z, k2, o.clamp_in_split ? 1 : 0));   // a3, a4

@@ -45,8 +45,10 @@ struct DevScalars {
     alignas(16) uint64_t wide_total[4];   // total of a wide (struct) scan
     uint64_t red7[8];                     // multi-GPU reduction staging
     unsigned long long local_rows;        // rows scanned below the frontier (local subtrees)
-    uint32_t local_depth, pad3;           // deepest ROOT level reached by a local subtree
+    uint32_t local_depth, amb_count;      // deepest ROOT level of a local subtree; ambiguous samples
 };
+
+constexpr int kMaxCand = 64;     // packed sort: most candidate rows per sample (one u64 mask)
 
 constexpr int kFixDigits = 6;     // 6 x 32-bit digits in u64 lanes, LSB 2^-72
 constexpr int kFixLsb = 72;
@@ -140,6 +142,12 @@ struct Ctx {
     uint64_t *keys[2] = {nullptr, nullptr}; size_t cap_keys[2] = {0, 0};
     uint32_t *vals[2] = {nullptr, nullptr}; size_t cap_vals[2] = {0, 0};
     uint32_t *t_sorted = nullptr, *row_sorted = nullptr; size_t cap_ts = 0, cap_rs = 0;
+    // packed sort (sort.cu): row_sorted holds the low pack_s bits of the row;
+    // pack_h = candidate rows per sample (0: payload mode, row_sorted = rows)
+    int pack_s = 0;
+    uint32_t pack_h = 0;
+    const uint32_t *sort_kid = nullptr, *sort_t = nullptr, *sort_row_in = nullptr;
+    void *amb = nullptr; size_t cap_amb = 0;                   // ambiguous-sample entries
     uint32_t *kid_count = nullptr, *goff = nullptr; size_t cap_kc = 0, cap_goff = 0;
     uint32_t *kid_max = nullptr; size_t cap_kmax = 0;          // per-kernel max t
     uint64_t *key_base = nullptr; size_t cap_kbase = 0;        // [K + 1] offset-key bases
@@ -209,7 +217,7 @@ int dist_metric_sums(Ctx &c, const double *metrics_local, uint32_t nm, uint64_t 
 
 // stages
 int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *row_in, uint64_t n,
-               uint32_t K);                                                                    // a1
+               uint32_t K, bool allow_pack);                                                   // a1
 int prefix_moments(Ctx &c, uint64_t n);                                                        // a2
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp);   // a3, a4
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);

@@ -14,6 +14,14 @@
 // reads the keys.  The last pass recovers kid from key >> 16 through a table
 // (B[k] >> 16 .. B[k+1] >> 16 -> k), or by binary search over B when the
 // table would be large, and writes t = key - B[kid].
+//
+// Packed mode (no payload).  When the key needs `bits` bits, the u64 holds
+// (B[kid] + t) << s | (row mod 2^s), s = 64 - bits: the passes sort on the
+// digits at s + 8p and the low row bits ride along for free, so every pass
+// moves 8 B per row instead of 12.  Equal keys keep row order (stable LSD), so
+// the last pass writes t and the low row bits in (kid, t, row) order; the
+// sample stage recovers a full row from its low bits by checking the
+// ceil(n / 2^s) candidate rows against the trace (stem.cu, R14 unchanged).
 #include <cstdlib>
 
 #include "internal.h"
@@ -134,6 +142,8 @@ struct PassArgs {
     const uint64_t *B;                  // [K + 1] key base per kernel
     const uint32_t *tab;                // LAST: kid table (NULL: binary search over B)
     uint64_t n;
+    uint64_t lomask;                    // packed: low row bits kept in the key (2^ks - 1, <= 2^32 - 1)
+    int ks;                             // packed: key shift s (0 in payload mode)
     uint32_t K;
     int shift, pass;
     int nxh;                            // FIRST: key bytes 2 .. 2 + nxh - 1 histogrammed here
@@ -150,14 +160,14 @@ struct PassArgs {
 // multi-split (match.any), global offsets found by decoupled look-back
 // (thread d < 256 owns digit d), then keys are staged in shared memory in
 // tile-sorted order and written out in digit runs (coalesced).
-template <int NT, int IT, bool FIRST, bool LAST, bool FULL>
+template <int NT, int IT, bool FIRST, bool LAST, bool FULL, bool PK>
 __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesweep_kernel(PassArgs a) {
     constexpr int NW = NT / 32, TILE = NT * IT, R = kR;
     static_assert(NT >= R, "one thread per digit");
     extern __shared__ __align__(16) unsigned char s_dyn[];
     uint64_t *s_keys = reinterpret_cast<uint64_t *>(s_dyn);                           // [TILE]
-    uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + TILE);                   // [TILE]
-    uint16_t (*s_whist)[R] = reinterpret_cast<uint16_t (*)[R]>(s_vals + TILE);        // [NW][R]
+    uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + TILE);                   // [TILE] (!PK)
+    uint16_t (*s_whist)[R] = reinterpret_cast<uint16_t (*)[R]>(PK ? (void *)(s_keys + TILE) : (void *)(s_vals + TILE));
     __shared__ uint64_t s_delta[R];
     __shared__ uint32_t s_lstart[R + 1];
     __shared__ uint32_t s_cnt[R];
@@ -186,6 +196,9 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             if (FIRST) {
                 src = tid == 0 ? (const void *)(a.kid_in + p0) : (const void *)(a.t_in + p0);
                 bytes = (uint32_t)(cnt * 4);
+            } else if (PK) {
+                src = (const void *)(a.keys_in + p0 + (tid ? cnt / 2 : 0));
+                bytes = (uint32_t)(tid ? (cnt - cnt / 2) * 8 : (cnt / 2) * 8);
             } else {
                 src = tid == 0 ? (const void *)(a.keys_in + p0) : (const void *)(a.vals_in + p0);
                 bytes = (uint32_t)(cnt * (tid == 0 ? 8 : 4));
@@ -197,21 +210,26 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
     }
 
     uint64_t key[IT];
-    uint32_t val[IT];
+    uint32_t val[PK ? 1 : IT];
 #pragma unroll
     for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         if (FULL || i < a.n) {
             if (FIRST) {
-                key[j] = __ldg(a.B + __ldg(a.kid_in + i)) + (uint64_t)__ldg(a.t_in + i);
-                val[j] = a.row_in ? __ldg(a.row_in + i) : (uint32_t)i;
+                const uint64_t kk = __ldg(a.B + __ldg(a.kid_in + i)) + (uint64_t)__ldg(a.t_in + i);
+                if (PK) {
+                    key[j] = (kk << a.ks) | (i & a.lomask);
+                } else {
+                    key[j] = kk;
+                    val[PK ? 0 : j] = a.row_in ? __ldg(a.row_in + i) : (uint32_t)i;
+                }
             } else {
                 key[j] = __ldcs(a.keys_in + i);
-                val[j] = __ldcs(a.vals_in + i);
+                if (!PK) val[PK ? 0 : j] = __ldcs(a.vals_in + i);
             }
         } else {
             key[j] = ~0ull;
-            val[j] = 0;
+            if (!PK) val[PK ? 0 : j] = 0;
         }
     }
     // the tile's digit counts, published at once so that successors' look-backs
@@ -222,7 +240,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             atomicAdd(&s_cnt[(uint32_t)(key[j] >> a.shift) & (R - 1)], 1u);
             if (FIRST)
                 for (int x = 0; x < a.nxh; x++)
-                    atomicAdd(&s_xh[x * R + ((uint32_t)(key[j] >> (kBaseShift + kRB * x)) & (R - 1))], 1u);
+                    atomicAdd(&s_xh[x * R + ((uint32_t)(key[j] >> (a.ks + kBaseShift + kRB * x)) & (R - 1))], 1u);
         }
     __syncthreads();
     if (tid < R) __stcg(a.status + (uint64_t)tile * R + tid, (tile == 0 ? kFlagP : kFlagA) | s_cnt[tid]);
@@ -314,7 +332,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             const uint32_t dd = (uint32_t)(key[j] >> a.shift) & (R - 1);
             const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + rank[j];
             s_keys[lp] = key[j];
-            s_vals[lp] = val[j];
+            if (!PK) s_vals[lp] = val[PK ? 0 : j];
         }
     }
     __syncthreads();
@@ -325,13 +343,14 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
         const uint32_t dd = (uint32_t)(k >> a.shift) & (R - 1);
         const uint64_t gp = s_delta[dd] + i;
         if (LAST) {
-            const uint32_t g = a.tab ? __ldg(a.tab + (k >> kBaseShift))
-                                     : (uint32_t)(upper_bound(a.B, (uint64_t)a.K + 1, k) - 1);
-            __stcs(a.t_out + gp, (uint32_t)(k - __ldg(a.B + g)));
-            __stcs(a.row_out + gp, s_vals[i]);
+            const uint64_t kk = PK ? k >> a.ks : k;
+            const uint32_t g = a.tab ? __ldg(a.tab + (kk >> kBaseShift))
+                                     : (uint32_t)(upper_bound(a.B, (uint64_t)a.K + 1, kk) - 1);
+            __stcs(a.t_out + gp, (uint32_t)(kk - __ldg(a.B + g)));
+            __stcs(a.row_out + gp, PK ? (uint32_t)(k & a.lomask) : s_vals[i]);
         } else {
             __stcs(a.keys_out + gp, k);
-            __stcs(a.vals_out + gp, s_vals[i]);
+            if (!PK) __stcs(a.vals_out + gp, s_vals[i]);
         }
     }
 }
@@ -339,40 +358,46 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
 // ---------------------------------------------------------------- host driver
 // full tiles in one launch (no bounds checks), the ragged last tile in a second
 // launch: its look-back finds every predecessor already inclusive
-template <int NT, int IT, bool FIRST, bool LAST>
+template <int NT, int IT, bool FIRST, bool LAST, bool PK>
 static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
     constexpr uint64_t TILE = (uint64_t)NT * IT;
     const uint64_t full = a.n / TILE, rag = a.n % TILE;
-    const size_t smem = (size_t)TILE * (sizeof(uint64_t) + sizeof(uint32_t)) + sizeof(uint16_t) * (NT / 32) * kR;
+    const size_t smem = (size_t)TILE * (sizeof(uint64_t) + (PK ? 0 : sizeof(uint32_t))) + sizeof(uint16_t) * (NT / 32) * kR;
     static bool attr = false;
     if (!attr) {
-        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true>,
+        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true, PK>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true>,
+        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true, PK>,
                                 cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false>,
+        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false, PK>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false>,
+        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false, PK>,
                                 cudaFuncAttributePreferredSharedMemoryCarveout, 100));
         attr = true;
     }
     if (full) {
-        onesweep_kernel<NT, IT, FIRST, LAST, true><<<(unsigned)full, NT, smem, st>>>(a);
+        onesweep_kernel<NT, IT, FIRST, LAST, true, PK><<<(unsigned)full, NT, smem, st>>>(a);
         (*launches)++;
     }
     if (rag) {
-        onesweep_kernel<NT, IT, FIRST, LAST, false><<<1, NT, smem, st>>>(a);
+        onesweep_kernel<NT, IT, FIRST, LAST, false, PK><<<1, NT, smem, st>>>(a);
         (*launches)++;
     }
     return STEM_OK;
 }
 
+template <int NT, int IT, bool PK>
+static int launch_pass_pk(const PassArgs &a, bool first, bool last, cudaStream_t st, uint32_t *launches) {
+    if (first && last) return launch_pass<NT, IT, true, true, PK>(a, st, launches);
+    if (first) return launch_pass<NT, IT, true, false, PK>(a, st, launches);
+    if (last) return launch_pass<NT, IT, false, true, PK>(a, st, launches);
+    return launch_pass<NT, IT, false, false, PK>(a, st, launches);
+}
+
 template <int NT, int IT>
 static int launch_pass_cfg(const PassArgs &a, bool first, bool last, cudaStream_t st, uint32_t *launches) {
-    if (first && last) return launch_pass<NT, IT, true, true>(a, st, launches);
-    if (first) return launch_pass<NT, IT, true, false>(a, st, launches);
-    if (last) return launch_pass<NT, IT, false, true>(a, st, launches);
-    return launch_pass<NT, IT, false, false>(a, st, launches);
+    return a.ks ? launch_pass_pk<NT, IT, true>(a, first, last, st, launches)
+                : launch_pass_pk<NT, IT, false>(a, first, last, st, launches);
 }
 
 // tile shapes (threads, keys per thread); STEMROOT_SORT_SHAPE picks one for
@@ -419,7 +444,8 @@ int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n
     return STEM_OK;
 }
 
-int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *row_in, uint64_t n, uint32_t K) {
+int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *row_in, uint64_t n, uint32_t K,
+               bool allow_pack) {
     cudaStream_t st = c.stream;
     CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
     const int tk_pre = c.stage_begin("prepass");
@@ -447,6 +473,25 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     if (npasses > kMaxPasses) return STEM_E_RANGE;
     c.stats.key_bits = bits;
     c.stats.sort_passes = npasses;
+    // packed mode: s = 64 - bits low row bits in the key, at most kMaxCand
+    // candidate rows per sample (STEMROOT_SORT_PACK=0 forces the payload mode,
+    // STEMROOT_PACK_BITS=s a smaller s, for tests of the candidate path)
+    int ks = 64 - bits;
+    if (const char *e = getenv("STEMROOT_PACK_BITS")) {
+        const int f = atoi(e);
+        if (f > 0 && f < ks) ks = f;
+    }
+    uint64_t hcount = 1;
+    if (ks < 32) hcount = (n + (1ull << ks) - 1) >> ks;
+    if (const char *e = getenv("STEMROOT_SORT_PACK"))
+        if (e[0] == '0') allow_pack = false;
+    if (!allow_pack || ks <= 0 || hcount > (uint64_t)kMaxCand) ks = 0;
+    c.pack_s = ks;
+    c.pack_h = ks ? (uint32_t)hcount : 0;
+    c.sort_kid = kid;
+    c.sort_t = t;
+    c.sort_row_in = row_in;
+    c.stats.pack_bits = (uint32_t)ks;
 
     // kid table for the last pass
     const uint64_t entries = range >> kBaseShift;
@@ -466,6 +511,8 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     a.B = B;
     a.tab = tab;
     a.nxh = npasses - 2;
+    a.ks = ks;
+    a.lomask = ks ? (ks >= 32 ? 0xffffffffull : (1ull << ks) - 1) : 0;
     {
         static int pf = -1;
         if (pf < 0) {
@@ -497,7 +544,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     for (int p = 0; p < npasses; p++) {
         CK(cudaMemsetAsync(a.status, 0, ntiles * kR * sizeof(uint64_t), st));
         CK(cudaMemsetAsync(a.tile_counter, 0, sizeof(uint32_t), st));
-        a.shift = kRB * p;
+        a.shift = ks + kRB * p;
         a.pass = p;
         const bool first = p == 0, last = p == npasses - 1;
         a.kid_in = kid;
@@ -510,7 +557,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         a.t_out = c.t_sorted;
         a.row_out = c.row_sorted;
         const char *sname = first ? "sort_pass_first" : last ? "sort_pass_last" : "sort_pass_mid";
-        const uint64_t sbytes = n * ((first ? 8 : 12) + (last ? 8 : 12));
+        const uint64_t sbytes = n * ((first ? 8 : ks ? 8 : 12) + (last ? 8 : ks ? 8 : 12));
         const int tk = c.stage_begin(sname);
         CKS(launch_sort_pass(a, first, last, st, &c.launches));
         c.stage_end(tk, sbytes);

@@ -232,13 +232,31 @@ struct SampleArgs {
     const uint32_t *leaf_lo, *leaf_kid, *leaf_ord;
     const uint64_t *moff, *m;
     const uint8_t *census;
-    const uint32_t *t, *row;
+    const uint32_t *t, *row;             // t_sorted; row_sorted (payload) or low row bits (packed)
     uint64_t L, n, S;
     uint32_t key0, key1, kid_base;
     uint32_t *out_row, *out_cluster;
     double *out_weight;
     uint64_t *U;
+    // packed sort (sort.cu): the full row is one of pack_h candidates
+    // (h << pack_s) | lo; the sort's input columns tell which
+    int pack_s;
+    uint32_t pack_h;
+    const uint32_t *kid_in, *t_in, *row_in;   // sort input (row_in: local -> trace row, or NULL)
+    struct Amb *amb;
+    uint32_t *amb_count;
 };
+
+// a sample whose low row bits match more than one candidate row
+struct Amb {
+    uint64_t mask;      // candidates h that hold (kernel, t)
+    uint32_t s, leaf, pos, lo;
+    uint32_t a, b;      // counted range of the run (the shorter side of pos)
+    uint32_t side, q;   // side 0: [r0, pos), 1: (pos, r1); q = matches of lo in [a, b)
+};
+__device__ __forceinline__ uint32_t map_row(const SampleArgs &a, uint32_t r) {
+    return a.row_in ? __ldg(a.row_in + r) : r;
+}
 
 __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
     const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -257,10 +275,102 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
         const uint64_t r = (j & 1) ? (((uint64_t)x.w << 32) | x.z) : (((uint64_t)x.y << 32) | x.x);
         pos = lo + __umul64hi(r, n);
     }
-    a.out_row[s] = a.row[pos];
+    const uint32_t tv = a.t[pos];
+    if (a.pack_h == 0) {
+        a.out_row[s] = a.row[pos];
+    } else {
+        const uint32_t low = a.row[pos];
+        if (a.pack_h == 1) {
+            a.out_row[s] = map_row(a, low);
+        } else {
+            // rows with the same (kernel, t) are in ascending row order in the
+            // sorted run; the candidates (h << s) | low that hold (kernel, t)
+            const uint32_t k = a.leaf_kid[i];
+            uint64_t mask = 0;
+            for (uint32_t h = 0; h < a.pack_h; h++) {
+                const uint64_t r = ((uint64_t)h << a.pack_s) | low;
+                if (r < a.n && __ldg(a.kid_in + r) == k && __ldg(a.t_in + r) == tv) mask |= 1ull << h;
+            }
+            if (__popcll(mask) == 1) {
+                a.out_row[s] = map_row(a, (uint32_t)(((uint64_t)(__ffsll(mask) - 1) << a.pack_s) | low));
+            } else {   // resolved by resolve_kernel: which of the matches sits at pos
+                const uint32_t e = atomicAdd(a.amb_count, 1u);
+                a.amb[e] = Amb{mask, (uint32_t)s, (uint32_t)i, (uint32_t)pos, low};
+            }
+        }
+    }
     a.out_cluster[s] = (uint32_t)i;
     a.out_weight[s] = __ddiv_rn(rn64(n), rn64(m));
-    atomicAdd((unsigned long long *)&a.U[i], (unsigned long long)a.t[pos]);
+    atomicAdd((unsigned long long *)&a.U[i], (unsigned long long)tv);
+}
+
+// Ambiguous sample at pos in the run [r0, r1) of equal (kernel, t): the run
+// lists the matching rows in ascending order and the low bits of each element
+// are known, so the sample is the q-th (ascending) of its candidates, where q
+// counts the run's elements before pos with the same low bits (or, counting
+// the shorter side, M - 1 - the elements after pos).  Three steps: locate the
+// run and the side to count, count it in 64k-element chunks over the whole
+// grid, pick the candidate.
+constexpr uint32_t kAmbChunk = 1u << 16;
+
+__global__ void __launch_bounds__(kThreads) resolve_locate_kernel(SampleArgs a, uint32_t na, uint64_t *nch) {
+    const uint32_t e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= na) return;
+    Amb &en = a.amb[e];
+    const uint32_t tv = a.t[en.pos];
+    const uint32_t lo = a.leaf_lo[en.leaf];
+    const uint32_t hi = (en.leaf + 1 < a.L) ? a.leaf_lo[en.leaf + 1] : (uint32_t)a.n;
+    const uint32_t r0 = lo + (uint32_t)lower_bound(a.t + lo, (uint64_t)(en.pos - lo), tv);
+    const uint32_t r1 = en.pos + 1 + (uint32_t)upper_bound(a.t + en.pos + 1, (uint64_t)(hi - en.pos - 1), tv);
+    if (en.pos - r0 <= r1 - en.pos - 1) { en.a = r0; en.b = en.pos; en.side = 0; }
+    else { en.a = en.pos + 1; en.b = r1; en.side = 1; }
+    en.q = 0;
+    nch[e] = (en.b - en.a + kAmbChunk - 1) / kAmbChunk;
+}
+
+__global__ void __launch_bounds__(kThreads) resolve_count_kernel(SampleArgs a, uint32_t na, const uint64_t *choff,
+                                                                 const uint64_t *total) {
+    __shared__ uint32_t s_cnt[kThreads / 32];
+    const uint64_t nc = *total;
+    for (uint64_t c = blockIdx.x; c < nc; c += gridDim.x) {
+        const uint32_t e = (uint32_t)(upper_bound(choff, (uint64_t)na, c) - 1);
+        const Amb &en = a.amb[e];
+        const uint32_t x0 = en.a + (uint32_t)(c - choff[e]) * kAmbChunk;
+        const uint32_t x1 = min(en.b, x0 + kAmbChunk);
+        const uint32_t v = en.lo;
+        uint32_t q = 0;
+        const uint32_t v0 = min(x1, (x0 + 3) & ~3u), v1 = max(v0, x1 & ~3u);
+        for (uint32_t x = x0 + threadIdx.x; x < v0; x += blockDim.x) q += __ldcs(a.row + x) == v;
+        for (uint32_t x = v1 + threadIdx.x; x < x1; x += blockDim.x) q += __ldcs(a.row + x) == v;
+        const uint4 *p4 = reinterpret_cast<const uint4 *>(a.row + v0);
+        const uint32_t n4 = (v1 - v0) / 4;
+#pragma unroll 4
+        for (uint32_t x = threadIdx.x; x < n4; x += blockDim.x) {
+            const uint4 w = __ldcs(p4 + x);
+            q += (w.x == v) + (w.y == v) + (w.z == v) + (w.w == v);
+        }
+        for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+        if ((threadIdx.x & 31) == 0) s_cnt[threadIdx.x >> 5] = q;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint32_t qq = 0;
+            for (int w = 0; w < kThreads / 32; w++) qq += s_cnt[w];
+            if (qq) atomicAdd(&a.amb[e].q, qq);
+        }
+        __syncthreads();
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) resolve_final_kernel(SampleArgs a, uint32_t na) {
+    const uint32_t e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= na) return;
+    const Amb en = a.amb[e];
+    const uint32_t M = (uint32_t)__popcll(en.mask);
+    uint32_t idx = en.side ? M - 1 - en.q : en.q;
+    uint64_t mk = en.mask;
+    for (uint32_t b = 0; b < idx && mk; b++) mk &= mk - 1;   // drop the idx lowest matches
+    const uint32_t h = mk ? (uint32_t)(__ffsll(mk) - 1) : 0u;
+    a.out_row[en.s] = map_row(a, (uint32_t)(((uint64_t)h << a.pack_s) | en.lo));
 }
 
 // ---------------------------------------------------------------- a8: estimate
@@ -481,12 +591,33 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CKS(c.ensure(c.out_row, c.cap_out_row, sizeof(uint32_t) * (S + 1)));
     CKS(c.ensure(c.out_cluster, c.cap_out_cluster, sizeof(uint32_t) * (S + 1)));
     CKS(c.ensure(c.out_weight, c.cap_out_weight, sizeof(double) * (S + 1)));
+    // packed sort: ambiguous-sample entries, their chunk counts/offsets, scan scratch
+    const size_t amb_bytes = sizeof(Amb) * (S + 1), nch_bytes = sizeof(uint64_t) * (S + 1);
+    if (c.pack_h > 1) CKS(c.ensure(c.amb, c.cap_amb, amb_bytes + 2 * nch_bytes + (scan_tiles(S + 1) + 2) * 16));
     SampleArgs sa{c.leaf_lo, leaf_kid, leaf_ord, c.leaf_moff, c.leaf_m, c.leaf_census, c.t_sorted, c.row_sorted,
                   L, n, S, (uint32_t)o.seed, (uint32_t)(o.seed >> 32), c.kid_base, c.out_row, c.out_cluster,
-                  c.out_weight, c.leaf_U};
+                  c.out_weight, c.leaf_U, c.pack_s, c.pack_h, c.sort_kid, c.sort_t, c.sort_row_in,
+                  (Amb *)c.amb, &c.scalars->amb_count};
     const int tk_smp = c.stage_begin("samples");
+    CK(cudaMemsetAsync(&c.scalars->amb_count, 0, sizeof(uint32_t), st));
     if (S) sample_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa);
     c.launches += S ? 1 : 0;
+    uint32_t n_amb = 0;
+    if (S && c.pack_h > 1) {
+        CK(cudaMemcpyAsync(&n_amb, &c.scalars->amb_count, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+    }
+    if (n_amb) {
+        uint64_t *nch = (uint64_t *)((char *)c.amb + amb_bytes), *choff = nch + (S + 1), *scr = choff + (S + 1);
+        uint64_t *tot = &c.scalars->scan_total64;
+        resolve_locate_kernel<<<blocks_for(n_amb), kThreads, 0, st>>>(sa, n_amb, nch);
+        exclusive_scan<uint64_t>([nch] __device__(uint64_t i) -> uint64_t { return nch[i]; },
+                                 [choff] __device__(uint64_t i, uint64_t pre, uint64_t) { choff[i] = pre; },
+                                 (uint64_t)n_amb, scr, tot, st, &c.launches);
+        resolve_count_kernel<<<4 * c.sms, kThreads, 0, st>>>(sa, n_amb, choff, tot);
+        resolve_final_kernel<<<blocks_for(n_amb), kThreads, 0, st>>>(sa, n_amb);
+        c.launches += 3;
+    }
     c.stage_end(tk_smp, 40 * S);
     CK(cudaGetLastError());
 
@@ -533,6 +664,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     for (uint32_t k = 0; k < nm; k++) c.host_est_metric[k] = (S || c.comm) ? red[2 + k] : 0.0;
     c.stats.n_clusters = L;
     c.stats.n_samples = S;
+    c.stats.ambiguous_samples = n_amb;
     return STEM_OK;
 }
 

@@ -116,3 +116,16 @@ def test_nccl_single_rank(sr):
     assert_plans_equal(got, ref)
     ctx.close()
     comm.close()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_packed_sort_candidate_rows_dist(sr, monkeypatch, world):
+    """packed sort key with a forced small packing (many candidate rows per
+    sample) under the multi-GPU row mapping (local index -> global row)"""
+    monkeypatch.setenv("STEMROOT_PACK_BITS", "9")
+    rng = np.random.default_rng(world)
+    kid = rng.integers(0, 5, 30_011).astype(np.uint32)
+    t = (rng.integers(0, 4, 30_011) * 300 + 1000 + kid * 7).astype(np.uint32)
+    ref = O.plan(kid, t, 5, eps=0.002, z=Z95, seed=8)
+    got = _dist_plan(sr, kid, t, 5, world, eps=0.002, z=Z95, seed=8)
+    assert_plans_equal(got, ref)

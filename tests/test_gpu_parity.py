@@ -259,3 +259,34 @@ def test_big_clusters(ctx, name):
     kid = np.zeros(len(t), np.uint32)
     got, ref = _both(ctx, kid, t[perm], 1, eps=0.02, seed=4)
     assert_plans_equal(got, ref)
+
+
+# ------------------------------------------------------------------ sort modes (sort.cu): row payload vs packed key
+def _dup_heavy(n, K, seed):
+    """few distinct times per kernel: long runs of equal (kernel, t), the case
+    where a packed key's low row bits match several candidate rows"""
+    rng = np.random.default_rng(seed)
+    kid = rng.integers(0, K, n).astype(np.uint32)
+    base = rng.integers(1000, 50_000, K)
+    t = base[kid] + rng.integers(0, 6, n) * (base[kid] // 7)
+    return kid, t.astype(np.uint32)
+
+
+@pytest.mark.parametrize("mode", ["payload", "packed", "bits16", "bits12"])
+@pytest.mark.parametrize("eps", [0.002, 0.05])
+def test_sort_modes(ctx, monkeypatch, mode, eps):
+    """Every sort mode gives the oracle's plan bit for bit; the forced small
+    packings (4 and 49 candidate rows per sample) go through the ambiguous-run
+    resolution, which the default packing at these sizes never needs."""
+    if mode == "payload":
+        monkeypatch.setenv("STEMROOT_SORT_PACK", "0")
+    elif mode.startswith("bits"):
+        monkeypatch.setenv("STEMROOT_PACK_BITS", mode[4:])
+    kid, t = _dup_heavy(200_003, 7, 17)
+    got, ref = _both(ctx, kid, t, 7, eps=eps, seed=21)
+    assert_plans_equal(got, ref)
+    st = ctx.stats()
+    assert st["pack_bits"] == {"payload": 0, "bits16": 16, "bits12": 12}.get(mode, st["key_bits"] and 64 - st["key_bits"])
+    if mode.startswith("bits") and eps == 0.002:
+        assert st["ambiguous_samples"] > 0
+
