@@ -29,6 +29,7 @@ int Ctx::ensure_all(uint64_t n, uint32_t K, uint32_t n_metrics) {
     CKS(ensure(key_base, cap_kbase, sizeof(uint64_t) * ((uint64_t)K + 2)));
     CKS(ensure(hist, cap_hist, sizeof(uint64_t) * 8 * 256));
     CKS(ensure(sort_mode, cap_sort_mode, sizeof(uint32_t) * 8));
+    CKS(ensure(sort_gbase, cap_sort_gbase, sizeof(uint64_t) * 8 * 256));
     CKS(ensure(scalars, cap_scalars, sizeof(DevScalars)));
     CKS(ensure(scan_scratch, cap_scan, (scan_tiles((uint64_t)K + 2) + 1) * 32));
     CKS(ensure(PS1, cap_ps1, sizeof(uint64_t) * (n / kChunk + 2)));
@@ -52,7 +53,7 @@ void Ctx::release() {
         dfree(f_S[i], cap_fS[i]); dfree(f_Q[i], cap_fQ[i]);
     }
     dfree(t_sorted, cap_ts); dfree(row_sorted, cap_rs); dfree(kid_count, cap_kc); dfree(goff, cap_goff);
-    dfree(kid_max, cap_kmax); dfree(key_base, cap_kbase); dfree(kid_tab, cap_kid_tab); dfree(sort_mode, cap_sort_mode);
+    dfree(kid_max, cap_kmax); dfree(key_base, cap_kbase); dfree(kid_tab, cap_kid_tab); dfree(sort_mode, cap_sort_mode); dfree(sort_gbase, cap_sort_gbase);
     dfree(hist, cap_hist); dfree(sort_status, cap_status); dfree(scalars, cap_scalars);
     dfree(scan_scratch, cap_scan); dfree(PS1, cap_ps1); dfree(PS2, cap_ps2); dfree(TB, cap_TB); dfree(chunk_sq, cap_chunk_sq);
     dfree(cut, cap_cut); dfree(cut_SL, cap_cut_SL); dfree(cut_QL, cap_cut_QL); dfree(cnt_sz, cap_cntsz); dfree(flags, cap_flags);

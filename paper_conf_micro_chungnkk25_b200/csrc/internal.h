@@ -153,6 +153,7 @@ struct Ctx {
     uint64_t *key_base = nullptr; size_t cap_kbase = 0;        // [K + 1] offset-key bases
     uint32_t *kid_tab = nullptr; size_t cap_kid_tab = 0;       // key >> 16 -> kernel
     uint32_t *sort_mode = nullptr; size_t cap_sort_mode = 0;   // ranking mode per pass
+    uint64_t *sort_gbase = nullptr; size_t cap_sort_gbase = 0; // [pass][256] digit bases
     uint64_t *hist = nullptr; size_t cap_hist = 0;
     void *sort_status = nullptr; size_t cap_status = 0;
     DevScalars *scalars = nullptr; size_t cap_scalars = 0;

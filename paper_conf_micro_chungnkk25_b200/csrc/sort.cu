@@ -35,6 +35,7 @@ constexpr int kHistR = 256;                 // histogram row stride
 constexpr int kBaseShift = 16;              // B[k] is a multiple of 2^16
 constexpr int kMaxExtra = kMaxPasses - 2;   // digits histogrammed by the first pass
 constexpr uint64_t kMaxTable = 1ull << 27;  // kid-table entries (512 MB) before binary search
+constexpr int kLB = 4;                      // look-back: predecessor statuses read per round trip
 
 // ---------------------------------------------------------------- pre-pass
 // kernel-id counts (group sizes), per-kernel max t, kernel-id range check, max
@@ -107,24 +108,37 @@ __global__ void kid_table_kernel(const uint64_t *__restrict__ B, uint32_t K, uin
     tab[j] = (uint32_t)(upper_bound(B, (uint64_t)K + 1, j << kBaseShift) - 1);
 }
 
-// Ranking mode per pass from its digit histogram.  MATCH.ANY slows down as
-// the number of distinct digits among a warp's 32 keys approaches 32, while
-// 8 ballots cost the same for any digit mix.  Measured on B200 (C5, per pass
-// ms match/ballot: 14.2/12.0, 9.7/8.8, 8.5/8.6, 7.4/8.3, 7.3/8.6 at expected
-// distinct digits 30.1, 29.8, 26.1, 24.8, 9.9): ballots when E[distinct] >= 27.
-__global__ void rank_mode_kernel(const uint64_t *__restrict__ hist, int p0, int p1, uint64_t n,
-                                 uint32_t *__restrict__ mode) {
+// Per pass, from its digit histogram: the digit bases (exclusive scan) and
+// the ranking mode.  MATCH.ANY slows down as the number of distinct digits
+// among a warp's 32 keys approaches 32, while 8 ballots cost the same for any
+// digit mix.  Measured on B200 (C5, per pass ms match/ballot: 14.2/12.0,
+// 9.7/8.8, 8.5/8.6, 7.4/8.3, 7.3/8.6 at expected distinct digits 30.1, 29.8,
+// 26.1, 24.8, 9.9): ballots when E[distinct] >= 27.  force >= 0 fixes the mode.
+__global__ void rank_mode_kernel(const uint64_t *__restrict__ hist, int p0, int p1, uint64_t n, int force,
+                                 uint32_t *__restrict__ mode, uint64_t *__restrict__ gbase) {
     __shared__ double s_w[8];
+    __shared__ uint64_t s_c[8];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     for (int p = p0; p < p1; p++) {
-        const double q = (double)hist[p * kHistR + threadIdx.x] / (double)n;
+        const uint64_t h = hist[p * kHistR + threadIdx.x];
+        const double q = (double)h / (double)n;
         double e = 1.0 - pow(1.0 - q, 32.0);
         for (int o = 16; o; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
-        if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = e;
+        uint64_t inc = h;
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint64_t v = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += v;
+        }
+        if (lane == 0) s_w[w] = e;
+        if (lane == 31) s_c[w] = inc;
         __syncthreads();
+        uint64_t off = 0;
+        for (int k = 0; k < w; k++) off += s_c[k];
+        gbase[p * kHistR + threadIdx.x] = off + inc - h;
         if (threadIdx.x == 0) {
             double tot = 0.0;
             for (int i = 0; i < 8; i++) tot += s_w[i];
-            mode[p] = tot >= 27.0 ? 1u : 0u;
+            mode[p] = force >= 0 ? (uint32_t)force : tot >= 27.0 ? 1u : 0u;
         }
         __syncthreads();
     }
@@ -149,6 +163,7 @@ struct PassArgs {
     int nxh;                            // FIRST: key bytes 2 .. 2 + nxh - 1 histogrammed here
     uint32_t pf;                        // tiles ahead to prefetch into L2 (0 = off)
     const uint32_t *ballot;             // [pass] 1: equal-digit lanes by 8 ballots, 0: match.any
+    const uint64_t *gbase;              // [pass][kHistR] exclusive scan of the pass's digit counts
     uint64_t *hist;                     // [pass][kHistR] global digit counts
     uint64_t *status;                   // [ntiles][R]
     uint32_t *tile_counter;
@@ -171,7 +186,6 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
     __shared__ uint64_t s_delta[R];
     __shared__ uint32_t s_lstart[R + 1];
     __shared__ uint32_t s_cnt[R];
-    __shared__ uint64_t s_gw[NW];
     __shared__ uint32_t s_cw[NW];
     __shared__ uint32_t s_tile;
     __shared__ uint32_t s_xh[FIRST ? kMaxExtra * R : 1];
@@ -280,10 +294,9 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
     }
     __syncthreads();
 
-    // digit phase (threads d < R): warp offsets, look-back, global offsets
+    // local digit offsets (threads d < R): per-warp bases, tile-wide exclusive scan
     const int d = tid;
     uint32_t cnt = 0, c_incl = 0;
-    uint64_t excl = 0, gcount = 0, g_incl = 0;
     if (d < R) {
 #pragma unroll
         for (int ww = 0; ww < NW; ww++) {
@@ -291,40 +304,26 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             s_whist[ww][d] = (uint16_t)cnt;
             cnt += c;
         }
-        if (tile != 0) {
-            int64_t j = (int64_t)tile - 1;
-            while (true) {
-                const uint64_t sv = *(volatile uint64_t *)(a.status + (uint64_t)j * R + d);
-                if (sv & kFlagP) { excl += sv & kValMask; break; }
-                if (sv & kFlagA) { excl += sv & kValMask; j--; }
-            }
-            __stcg(a.status + (uint64_t)tile * R + d, kFlagP | (excl + cnt));
-        }
-        gcount = a.hist[a.pass * kHistR + d];
-        g_incl = gcount;
         c_incl = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
-            const uint64_t gv = __shfl_up_sync(0xffffffffu, g_incl, o);
             const uint32_t cv = __shfl_up_sync(0xffffffffu, c_incl, o);
-            if (lane >= o) { g_incl += gv; c_incl += cv; }
+            if (lane >= o) c_incl += cv;
         }
-        if (lane == 31) { s_gw[w] = g_incl; s_cw[w] = c_incl; }
+        if (lane == 31) s_cw[w] = c_incl;
     }
     __syncthreads();
     if (d < R) {
-        uint64_t goff = 0;
         uint32_t coff = 0;
-        for (int ww = 0; ww < w; ww++) { goff += s_gw[ww]; coff += s_cw[ww]; }
-        const uint64_t g_excl = goff + g_incl - gcount;
+        for (int ww = 0; ww < w; ww++) coff += s_cw[ww];
         const uint32_t c_excl = coff + c_incl - cnt;
         s_lstart[d] = c_excl;
-        s_delta[d] = g_excl + excl - c_excl;   // global position - local position
         if (d == R - 1) s_lstart[R] = c_excl + cnt;
     }
     __syncthreads();
 
-    // scatter into shared memory in tile-sorted order, then out in digit runs
+    // scatter into shared memory in tile-sorted order (needs only local
+    // offsets: predecessors keep publishing meanwhile)
 #pragma unroll
     for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
@@ -334,6 +333,32 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             s_keys[lp] = key[j];
             if (!PK) s_vals[lp] = val[PK ? 0 : j];
         }
+    }
+
+    // decoupled look-back (thread d < R owns digit d), kLB predecessors per
+    // round trip; global offset = pass digit base + predecessors' counts
+    if (d < R) {
+        uint64_t excl = 0;
+        if (tile != 0) {
+            int64_t j = (int64_t)tile - 1;
+            bool done = false;
+            while (!done) {
+                uint64_t sv[kLB];
+#pragma unroll
+                for (int q = 0; q < kLB; q++)
+                    sv[q] = (j - q >= 0) ? *(volatile uint64_t *)(a.status + (uint64_t)(j - q) * R + d) : (2ull << 62);
+#pragma unroll
+                for (int q = 0; q < kLB; q++) {
+                    if (done) break;
+                    const uint64_t v = sv[q];
+                    if (v & kFlagP) { excl += v & kValMask; done = true; }
+                    else if (v & kFlagA) { excl += v & kValMask; j--; }
+                    else break;   // not published yet: poll again from tile j
+                }
+            }
+            __stcg(a.status + (uint64_t)tile * R + d, kFlagP | (excl + cnt));
+        }
+        s_delta[d] = a.gbase[a.pass * kHistR + d] + excl - s_lstart[d];   // global position - local position
     }
     __syncthreads();
     const uint32_t nvalid = s_lstart[R];
@@ -528,14 +553,11 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         rank_force = !e ? -1 : e[0] == 'b' ? 1 : e[0] == 'm' ? 0 : -1;
     }
     uint32_t *mode = c.sort_mode;
-    if (rank_force >= 0) {
-        CK(cudaMemsetAsync(mode, 0, sizeof(uint32_t) * kMaxPasses, st));
-        if (rank_force) CK(cudaMemsetAsync(mode, 1, sizeof(uint32_t) * kMaxPasses, st));   // nonzero bytes
-    } else {
-        rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 0, 2, n, mode);   // key bytes 0, 1: pre-pass histograms
-        c.launches++;
-    }
+    uint64_t *gbase = c.sort_gbase;
+    rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 0, 2, n, rank_force, mode, gbase);   // key bytes 0, 1: pre-pass
+    c.launches++;
     a.ballot = mode;
+    a.gbase = gbase;
     a.hist = c.hist;
     a.status = (uint64_t *)c.sort_status;
     a.tile_counter = &c.scalars->tile_counter;
@@ -562,8 +584,8 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         CKS(launch_sort_pass(a, first, last, st, &c.launches));
         c.stage_end(tk, sbytes);
         CK(cudaGetLastError());
-        if (first && rank_force < 0 && npasses > 2) {   // higher bytes: histogrammed by pass 0
-            rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 2, npasses, n, mode);
+        if (first && npasses > 2) {   // higher bytes: histogrammed by pass 0
+            rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 2, npasses, n, rank_force, mode, gbase);
             c.launches++;
         }
         uint64_t *tkk = kin; kin = kout; kout = tkk;
