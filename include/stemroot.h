@@ -140,6 +140,8 @@ typedef struct stem_stats {
     double   ssum;             /* RN(exact sum_i sqrt(mu_i V_i)) of the global KKT solve          */
     uint32_t pack_bits;        /* low row bits carried inside the sort key (0: row payload mode)  */
     uint32_t ambiguous_samples;/* samples whose row needed the run scan (packed mode)            */
+    uint32_t coarse_bases;     /* 1: kernel key bases aligned to 2^24 (pass histograms from the pre-pass) */
+    uint32_t reserved0;
 } stem_stats;
 
 /* Per-stage device time of the last plan (stem_ctx_enable_timing).  bytes is

@@ -27,7 +27,8 @@ int Ctx::ensure_all(uint64_t n, uint32_t K, uint32_t n_metrics) {
     CKS(ensure(goff, cap_goff, sizeof(uint32_t) * ((uint64_t)K + 2)));
     CKS(ensure(kid_max, cap_kmax, sizeof(uint32_t) * ((uint64_t)K + 1)));
     CKS(ensure(key_base, cap_kbase, sizeof(uint64_t) * ((uint64_t)K + 2)));
-    CKS(ensure(hist, cap_hist, sizeof(uint64_t) * 8 * 256));
+    CKS(ensure(key_base_c, cap_kbase_c, sizeof(uint64_t) * ((uint64_t)K + 2)));
+    CKS(ensure(hist, cap_hist, sizeof(uint64_t) * 9 * 256));
     CKS(ensure(sort_mode, cap_sort_mode, sizeof(uint32_t) * 8));
     CKS(ensure(sort_gbase, cap_sort_gbase, sizeof(uint64_t) * 8 * 256));
     CKS(ensure(scalars, cap_scalars, sizeof(DevScalars)));
@@ -53,7 +54,7 @@ void Ctx::release() {
         dfree(f_S[i], cap_fS[i]); dfree(f_Q[i], cap_fQ[i]);
     }
     dfree(t_sorted, cap_ts); dfree(row_sorted, cap_rs); dfree(kid_count, cap_kc); dfree(goff, cap_goff);
-    dfree(kid_max, cap_kmax); dfree(key_base, cap_kbase); dfree(kid_tab, cap_kid_tab); dfree(sort_mode, cap_sort_mode); dfree(sort_gbase, cap_sort_gbase);
+    dfree(kid_max, cap_kmax); dfree(key_base, cap_kbase); dfree(key_base_c, cap_kbase_c); dfree(key_base_s, cap_kbase_s); dfree(tailh, cap_tailh); dfree(kid_tab, cap_kid_tab); dfree(sort_mode, cap_sort_mode); dfree(sort_gbase, cap_sort_gbase);
     dfree(hist, cap_hist); dfree(sort_status, cap_status); dfree(scalars, cap_scalars);
     dfree(scan_scratch, cap_scan); dfree(PS1, cap_ps1); dfree(PS2, cap_ps2); dfree(TB, cap_TB); dfree(chunk_sq, cap_chunk_sq);
     dfree(cut, cap_cut); dfree(cut_SL, cap_cut_SL); dfree(cut_QL, cap_cut_QL); dfree(cnt_sz, cap_cntsz); dfree(flags, cap_flags);

@@ -457,7 +457,6 @@ __global__ void add_kernel_u32(uint32_t *x, uint64_t n, uint32_t v) {
     if (i < n) x[i] += v;
 }
 
-int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K);   // sort.cu
 
 int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
                   const stem_opts &o) {
@@ -498,11 +497,11 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
     CKS(c.ensure(c.dist_cnt, c.cap_dist_cnt, sizeof(uint64_t) * ((uint64_t)K + 2)));
     CKS(c.ensure(c.scalars, c.cap_scalars, sizeof(DevScalars)));
     CKS(c.ensure(c.kid_max, c.cap_kmax, sizeof(uint32_t) * ((uint64_t)K + 1)));
-    CKS(c.ensure(c.hist, c.cap_hist, sizeof(uint64_t) * 8 * 256));
+    CKS(c.ensure(c.hist, c.cap_hist, sizeof(uint64_t) * 9 * 256));
     CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
     CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
     const int tk_x = c.stage_begin("dist_exchange");
-    if (n) CKS(histogram_kernels(c, kid, t, n, K));
+    if (n) CKS(histogram_kernels(c, kid, t, n, K, nullptr));
     kid_counts_u64_kernel<<<(unsigned)((K + 256) / 256), 256, 0, st>>>(c.kid_count, K, &c.scalars->err, c.dist_cnt);
     c.launches++;
     CKS(comm.allreduce(c.dist_cnt, (size_t)K + 1, false, st));

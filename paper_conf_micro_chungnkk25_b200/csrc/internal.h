@@ -32,6 +32,7 @@ cudaError_t &last_cuda_error();
 struct DevScalars {
     uint32_t max_t, err, tile_counter, pad0;
     uint64_t scan_total64;        // generic scan total
+    uint64_t scan_total64b;       // second scan total (coarse key bases)
     uint64_t frontier_total;      // packed (count << 32 | rows) of the next frontier
     uint64_t n_leaves;            // leaves after compaction
     uint64_t total_m;             // sum of m_i
@@ -151,6 +152,9 @@ struct Ctx {
     uint32_t *kid_count = nullptr, *goff = nullptr; size_t cap_kc = 0, cap_goff = 0;
     uint32_t *kid_max = nullptr; size_t cap_kmax = 0;          // per-kernel max t
     uint64_t *key_base = nullptr; size_t cap_kbase = 0;        // [K + 1] offset-key bases
+    uint64_t *key_base_c = nullptr; size_t cap_kbase_c = 0;    // [K + 1] coarse (2^24) bases
+    uint32_t *key_base_s = nullptr; size_t cap_kbase_s = 0;    // [K + 1] chosen bases >> shift
+    uint32_t *tailh = nullptr; size_t cap_tailh = 0;           // [K][256] rows per (kernel, t >> 24)
     uint32_t *kid_tab = nullptr; size_t cap_kid_tab = 0;       // key >> 16 -> kernel
     uint32_t *sort_mode = nullptr; size_t cap_sort_mode = 0;   // ranking mode per pass
     uint64_t *sort_gbase = nullptr; size_t cap_sort_gbase = 0; // [pass][256] digit bases
@@ -222,7 +226,8 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
 int prefix_moments(Ctx &c, uint64_t n);                                                        // a2
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp);   // a3, a4
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
-int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K);   // pre-pass only
+int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,
+                      uint32_t *tailh);   // pre-pass only
 int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
                   const stem_opts &o);
 int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint32_t n_metrics, double eps,

@@ -15,6 +15,12 @@
 // (B[k] >> 16 .. B[k+1] >> 16 -> k), or by binary search over B when the
 // table would be large, and writes t = key - B[kid].
 //
+// Coarse bases.  When rounding W[k] up to 2^24 instead costs no extra pass,
+// B[k] is a multiple of 2^24: key byte 2 is t byte 2, and key bits 24.. are
+// (B[k] >> 24) + (t >> 24), so every pass histogram comes from the pre-pass
+// (t bytes 0-2, and a per-kernel histogram of t >> 24 that only the rare rows
+// with t >= 2^24 touch) and the first pass does no extra counting.
+//
 // Packed mode (no payload).  When the key needs `bits` bits, the u64 holds
 // (B[kid] + t) << s | (row mod 2^s), s = 64 - bits: the passes sort on the
 // digits at s + 8p and the low row bits ride along for free, so every pass
@@ -36,18 +42,23 @@ constexpr int kBaseShift = 16;              // B[k] is a multiple of 2^16
 constexpr int kMaxExtra = kMaxPasses - 2;   // digits histogrammed by the first pass
 constexpr uint64_t kMaxTable = 1ull << 27;  // kid-table entries (512 MB) before binary search
 constexpr int kLB = 4;                      // look-back: predecessor statuses read per round trip
+constexpr int kCoarseShift = 24;            // coarse bases: B[k] a multiple of 2^24
+constexpr uint32_t kMaxTailK = 1u << 16;    // coarse bases need a [K][256] tail histogram
+constexpr int kHistT2 = kMaxPasses;         // hist row of t byte 2 (pre-pass)
 
 // ---------------------------------------------------------------- pre-pass
 // kernel-id counts (group sizes), per-kernel max t, kernel-id range check, max
-// t, and the histograms of t bytes 0 and 1 (= key bytes 0 and 1).
-__global__ void __launch_bounds__(256) prepass_kernel(const uint32_t *__restrict__ kid, const uint32_t *__restrict__ t,
+// t, the histograms of t bytes 0 and 1 (= key bytes 0 and 1) and 2 (row
+// kHistT2), and (tailh != NULL) the per-kernel histogram of t >> 24 >= 1.
+constexpr int kPreThreads = 1024;
+__global__ void __launch_bounds__(kPreThreads, 2) prepass_kernel(const uint32_t *__restrict__ kid, const uint32_t *__restrict__ t,
                                                       uint64_t n, uint32_t K, int smem_kid,
                                                       uint32_t *__restrict__ kid_count, uint32_t *__restrict__ kid_max,
                                                       uint64_t *__restrict__ hist, uint32_t *__restrict__ max_t,
-                                                      uint32_t *__restrict__ err) {
-    extern __shared__ uint32_t sh[];   // [2][256] byte histograms, then [K] counts, [K] max
-    uint32_t *h0 = sh, *hk = sh + 2 * kR, *hm = hk + (smem_kid ? K : 0);
-    for (int i = threadIdx.x; i < 2 * kR; i += blockDim.x) h0[i] = 0;
+                                                      uint32_t *__restrict__ err, uint32_t *__restrict__ tailh) {
+    extern __shared__ uint32_t sh[];   // [3][256] byte histograms, then [K] counts, [K] max
+    uint32_t *h0 = sh, *hk = sh + 3 * kR, *hm = hk + (smem_kid ? K : 0);
+    for (int i = threadIdx.x; i < 3 * kR; i += blockDim.x) h0[i] = 0;
     if (smem_kid)
         for (uint32_t i = threadIdx.x; i < 2 * K; i += blockDim.x) hk[i] = 0;
     __syncthreads();
@@ -59,10 +70,12 @@ __global__ void __launch_bounds__(256) prepass_kernel(const uint32_t *__restrict
         mx = max(mx, x);
         atomicAdd(&h0[x & (kR - 1)], 1u);
         atomicAdd(&h0[kR + ((x >> kRB) & (kR - 1))], 1u);
+        if ((x >> (2 * kRB)) & (kR - 1)) atomicAdd(&h0[2 * kR + ((x >> (2 * kRB)) & (kR - 1))], 1u);   // bin 0: n - rest
         if (k >= K) { bad = 1; return; }
+        if (tailh && (x >> kCoarseShift)) atomicAdd(&tailh[(uint64_t)k * kR + (x >> kCoarseShift)], 1u);
         if (smem_kid) {
             atomicAdd(&hk[k], 1u);
-            atomicMax(&hm[k], x);
+            if (x > hm[k]) atomicMax(&hm[k], x);   // a read first: most rows do not raise the max
         } else {
             atomicAdd(&kid_count[k], 1u);
             atomicMax(&kid_max[k], x);
@@ -70,7 +83,14 @@ __global__ void __launch_bounds__(256) prepass_kernel(const uint32_t *__restrict
     };
     const bool aligned = ((reinterpret_cast<uintptr_t>(kid) | reinterpret_cast<uintptr_t>(t)) & 15) == 0;
     if (aligned) {
-        for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
+        uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+        for (; i + stride < n4; i += 2 * stride) {   // two uint4 pairs in flight per thread
+            const uint4 a = __ldg(kid4 + i), b = __ldg(t4 + i);
+            const uint4 a2 = __ldg(kid4 + i + stride), b2 = __ldg(t4 + i + stride);
+            one(a.x, b.x); one(a.y, b.y); one(a.z, b.z); one(a.w, b.w);
+            one(a2.x, b2.x); one(a2.y, b2.y); one(a2.z, b2.z); one(a2.w, b2.w);
+        }
+        for (; i < n4; i += stride) {
             const uint4 a = __ldg(kid4 + i), b = __ldg(t4 + i);
             one(a.x, b.x); one(a.y, b.y); one(a.z, b.z); one(a.w, b.w);
         }
@@ -89,8 +109,8 @@ __global__ void __launch_bounds__(256) prepass_kernel(const uint32_t *__restrict
         if (bad) atomicOr(err, 1u);
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < 2 * kR; i += blockDim.x)
-        if (h0[i]) atomicAdd((unsigned long long *)&hist[(i >> kRB) * kHistR + (i & (kR - 1))],
+    for (int i = threadIdx.x; i < 3 * kR; i += blockDim.x)
+        if (h0[i]) atomicAdd((unsigned long long *)&hist[((i >> kRB) == 2 ? kHistT2 : (i >> kRB)) * kHistR + (i & (kR - 1))],
                              (unsigned long long)h0[i]);
     if (smem_kid)
         for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
@@ -100,12 +120,51 @@ __global__ void __launch_bounds__(256) prepass_kernel(const uint32_t *__restrict
             }
 }
 
-// kid-table entry j -> the kernel whose key range holds j << 16
-__global__ void kid_table_kernel(const uint64_t *__restrict__ B, uint32_t K, uint64_t entries,
+// kid-table entry j -> the kernel whose key range holds j << tsh
+__global__ void kid_table_kernel(const uint64_t *__restrict__ B, uint32_t K, uint64_t entries, int tsh,
                                  uint32_t *__restrict__ tab) {
     const uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (j >= entries) return;
-    tab[j] = (uint32_t)(upper_bound(B, (uint64_t)K + 1, j << kBaseShift) - 1);
+    tab[j] = (uint32_t)(upper_bound(B, (uint64_t)K + 1, j << tsh) - 1);
+}
+
+__global__ void base_shift_kernel(const uint64_t *__restrict__ B, uint64_t m, int tsh, uint32_t *__restrict__ Bs) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < m) Bs[i] = (uint32_t)(B[i] >> tsh);
+}
+
+// Coarse bases: histograms of key bytes 2 .. npasses-1 from the pre-pass.
+// Byte 2 is t byte 2; bits 24.. of kernel k's keys are (B[k] >> 24) + u for
+// its rows with t >> 24 = u.  One warp per kernel.
+__global__ void coarse_hist_kernel(const uint32_t *__restrict__ cnt, const uint32_t *__restrict__ tailh,
+                                   const uint64_t *__restrict__ B, uint32_t K, int npasses, uint64_t n,
+                                   uint64_t *__restrict__ hist) {
+    if (blockIdx.x == 0 && npasses > 2) {   // t byte 2; the pre-pass counts bins >= 1 only
+        __shared__ uint64_t s_part[8];
+        const uint64_t h = threadIdx.x ? hist[kHistT2 * kHistR + threadIdx.x] : 0;
+        uint64_t v = h;
+        for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if ((threadIdx.x & 31) == 0) s_part[threadIdx.x >> 5] = v;
+        __syncthreads();
+        uint64_t rest = 0;
+        for (int w = 0; w < 8; w++) rest += s_part[w];
+        hist[2 * kHistR + threadIdx.x] = threadIdx.x ? h : n - rest;
+    }
+    const uint32_t k = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+    if (k >= K || cnt[k] == 0) return;
+    const uint64_t v0 = B[k] >> kCoarseShift;
+    auto add = [&](uint64_t v, uint32_t c) {
+        for (int x = 3; x < npasses; x++)
+            atomicAdd((unsigned long long *)&hist[x * kHistR + ((v >> (kRB * (x - 3))) & (kR - 1))],
+                      (unsigned long long)c);
+    };
+    uint32_t tail = 0;
+    for (uint32_t u = 1 + lane; u < (uint32_t)kR; u += 32) {
+        const uint32_t c = tailh[(uint64_t)k * kR + u];
+        if (c) { tail += c; add(v0 + u, c); }
+    }
+    for (int o = 16; o; o >>= 1) tail += __shfl_xor_sync(0xffffffffu, tail, o);
+    if (lane == 0) add(v0, cnt[k] - tail);
 }
 
 // Per pass, from its digit histogram: the digit bases (exclusive scan) and
@@ -154,7 +213,9 @@ struct PassArgs {
     uint32_t *vals_out;                 // !LAST
     uint32_t *t_out, *row_out;          // LAST
     const uint64_t *B;                  // [K + 1] key base per kernel
+    const uint32_t *Bs;                 // [K + 1] B >> tsh (FIRST: a 4-byte gather that stays in L1)
     const uint32_t *tab;                // LAST: kid table (NULL: binary search over B)
+    int tsh;                            // B[k] is a multiple of 2^tsh; LAST: kid-table index = key >> tsh
     uint64_t n;
     uint64_t lomask;                    // packed: low row bits kept in the key (2^ks - 1, <= 2^32 - 1)
     int ks;                             // packed: key shift s (0 in payload mode)
@@ -230,7 +291,9 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         if (FULL || i < a.n) {
             if (FIRST) {
-                const uint64_t kk = __ldg(a.B + __ldg(a.kid_in + i)) + (uint64_t)__ldg(a.t_in + i);
+                const uint32_t kd = __ldg(a.kid_in + i);
+                const uint64_t kb = a.Bs ? (uint64_t)__ldg(a.Bs + kd) << a.tsh : __ldg(a.B + kd);
+                const uint64_t kk = kb + (uint64_t)__ldg(a.t_in + i);
                 if (PK) {
                     key[j] = (kk << a.ks) | (i & a.lomask);
                 } else {
@@ -369,7 +432,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
         const uint64_t gp = s_delta[dd] + i;
         if (LAST) {
             const uint64_t kk = PK ? k >> a.ks : k;
-            const uint32_t g = a.tab ? __ldg(a.tab + (kk >> kBaseShift))
+            const uint32_t g = a.tab ? __ldg(a.tab + (kk >> a.tsh))
                                      : (uint32_t)(upper_bound(a.B, (uint64_t)a.K + 1, kk) - 1);
             __stcs(a.t_out + gp, (uint32_t)(kk - __ldg(a.B + g)));
             __stcs(a.row_out + gp, PK ? (uint32_t)(k & a.lomask) : s_vals[i]);
@@ -392,12 +455,14 @@ static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
     if (!attr) {
         CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true, PK>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        // FIRST gathers B[kid]: keep L1 beside three blocks' shared memory
+        const int carve = FIRST ? (int)((3 * (smem + 12 * 1024) * 100 + 228 * 1024 - 1) / (228 * 1024)) : 100;
         CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true, PK>,
-                                cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+                                cudaFuncAttributePreferredSharedMemoryCarveout, carve > 100 ? 100 : carve));
         CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false, PK>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false, PK>,
-                                cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+                                cudaFuncAttributePreferredSharedMemoryCarveout, carve > 100 ? 100 : carve));
         attr = true;
     }
     if (full) {
@@ -451,19 +516,20 @@ static int launch_sort_pass(const PassArgs &a, bool first, bool last, cudaStream
 
 // the pre-pass alone (kernel-id counts and max t, range check): also the
 // multi-GPU histogram step.  Zeroes its outputs first.
-int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K) {
+int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K, uint32_t *tailh) {
     cudaStream_t st = c.stream;
-    CK(cudaMemsetAsync(c.hist, 0, sizeof(uint64_t) * kMaxPasses * kHistR, st));
+    CK(cudaMemsetAsync(c.hist, 0, sizeof(uint64_t) * (kMaxPasses + 1) * kHistR, st));
+    if (tailh) CK(cudaMemsetAsync(tailh, 0, sizeof(uint32_t) * kR * (uint64_t)K, st));
     CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
     CK(cudaMemsetAsync(c.kid_max, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
     const int smem_kid = (K <= 24000) ? 1 : 0;
-    const size_t sm_bytes = sizeof(uint32_t) * (2 * kR + (smem_kid ? 2 * (size_t)K : 0));
+    const size_t sm_bytes = sizeof(uint32_t) * (3 * kR + (smem_kid ? 2 * (size_t)K : 0));
     if (sm_bytes > 48 * 1024)
         CK(cudaFuncSetAttribute(prepass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_bytes));
     int per_sm = (int)((200 * 1024) / (sm_bytes + 1024));
-    per_sm = per_sm < 1 ? 1 : per_sm > 4 ? 4 : per_sm;
-    prepass_kernel<<<c.sms * per_sm, 256, sm_bytes, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.kid_max, c.hist,
-                                                          &c.scalars->max_t, &c.scalars->err);
+    per_sm = per_sm < 1 ? 1 : per_sm > 2 ? 2 : per_sm;
+    prepass_kernel<<<c.sms * per_sm, kPreThreads, sm_bytes, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.kid_max, c.hist,
+                                                          &c.scalars->max_t, &c.scalars->err, tailh);
     c.launches++;
     CK(cudaGetLastError());
     return STEM_OK;
@@ -474,28 +540,50 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     cudaStream_t st = c.stream;
     CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
     const int tk_pre = c.stage_begin("prepass");
-    CKS(histogram_kernels(c, kid, t, n, K));
-    // key bases B = exclusive scan of W[k] = roundup(max_t[k] + 1, 2^16) (0 if absent)
+    // coarse bases are possible when the [K][256] tail histogram is small
+    const bool coarse_ok = K <= kMaxTailK && !(getenv("STEMROOT_SORT_COARSE") && getenv("STEMROOT_SORT_COARSE")[0] == '0');
+    if (coarse_ok) CKS(c.ensure(c.tailh, c.cap_tailh, sizeof(uint32_t) * kR * (uint64_t)K));
+    CKS(histogram_kernels(c, kid, t, n, K, coarse_ok ? c.tailh : nullptr));
+    // key bases B = exclusive scan of W[k] = roundup(max_t[k] + 1, 2^16) (0 if
+    // absent); Bc the same with 2^24
     const uint32_t *cnt = c.kid_count, *kmax = c.kid_max;
-    uint64_t *B = c.key_base;
-    exclusive_scan<uint64_t>(
-        [cnt, kmax, K] __device__(uint64_t i) -> uint64_t {
-            if (i >= K || cnt[i] == 0) return 0;
-            return (((uint64_t)kmax[i] >> kBaseShift) + 1) << kBaseShift;
-        },
-        [B] __device__(uint64_t i, uint64_t pre, uint64_t) { B[i] = pre; },
-        (uint64_t)K + 1, (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
-    c.stage_end(tk_pre, 8 * n);
+    for (int v = 0; v < (coarse_ok ? 2 : 1); v++) {
+        uint64_t *Bv = v ? c.key_base_c : c.key_base;
+        const int sh = v ? kCoarseShift : kBaseShift;
+        exclusive_scan<uint64_t>(
+            [cnt, kmax, K, sh] __device__(uint64_t i) -> uint64_t {
+                if (i >= K || cnt[i] == 0) return 0;
+                return (((uint64_t)kmax[i] >> sh) + 1) << sh;
+            },
+            [Bv] __device__(uint64_t i, uint64_t pre, uint64_t) { Bv[i] = pre; }, (uint64_t)K + 1,
+            (uint64_t *)c.scan_scratch, v ? &c.scalars->scan_total64b : &c.scalars->scan_total64, st, &c.launches);
+    }
     DevScalars hs;
     CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     if (hs.err) return STEM_E_RANGE;
-    const uint64_t range = hs.scan_total64;     // keys lie in [0, range)
-    int bits = 0;
-    while (bits < 64 && (bits == 0 || (range - 1) >> bits)) bits++;
-    int npasses = (bits + kRB - 1) / kRB;
-    if (npasses < 2) npasses = 2;
+    auto nbits = [](uint64_t range) {   // keys lie in [0, range)
+        int b = 0;
+        while (b < 64 && (b == 0 || (range - 1) >> b)) b++;
+        return b;
+    };
+    auto npass = [](int b) { return b <= 16 ? 2 : (b + kRB - 1) / kRB; };
+    int bits = nbits(hs.scan_total64);
+    bool coarse = false;
+    if (coarse_ok && hs.scan_total64b && npass(nbits(hs.scan_total64b)) <= npass(bits)) {
+        coarse = true;
+        bits = nbits(hs.scan_total64b);
+    }
+    const uint64_t range = coarse ? hs.scan_total64b : hs.scan_total64;
+    const int npasses = npass(bits);
     if (npasses > kMaxPasses) return STEM_E_RANGE;
+    uint64_t *B = coarse ? c.key_base_c : c.key_base;
+    if (coarse) {
+        coarse_hist_kernel<<<(unsigned)((K + 7) / 8), kR, 0, st>>>(cnt, c.tailh, B, K, npasses, n, c.hist);
+        c.launches++;
+    }
+    c.stage_end(tk_pre, 8 * n);
+    c.stats.coarse_bases = coarse ? 1 : 0;
     c.stats.key_bits = bits;
     c.stats.sort_passes = npasses;
     // packed mode: s = 64 - bits low row bits in the key, at most kMaxCand
@@ -519,11 +607,12 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     c.stats.pack_bits = (uint32_t)ks;
 
     // kid table for the last pass
-    const uint64_t entries = range >> kBaseShift;
+    const int tsh = coarse ? kCoarseShift : kBaseShift;
+    const uint64_t entries = range >> tsh;
     const uint32_t *tab = nullptr;
     if (entries <= kMaxTable) {
         CKS(c.ensure(c.kid_tab, c.cap_kid_tab, sizeof(uint32_t) * (entries + 1)));
-        kid_table_kernel<<<(unsigned)((entries + 255) / 256), 256, 0, st>>>(B, K, entries, c.kid_tab);
+        kid_table_kernel<<<(unsigned)((entries + 255) / 256), 256, 0, st>>>(B, K, entries, tsh, c.kid_tab);
         c.launches++;
         tab = c.kid_tab;
     }
@@ -534,8 +623,16 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     a.n = n;
     a.K = K;
     a.B = B;
+    a.Bs = nullptr;
+    if ((range >> tsh) < (1ull << 32)) {   // bases >> tsh fit 32 bits
+        CKS(c.ensure(c.key_base_s, c.cap_kbase_s, sizeof(uint32_t) * ((uint64_t)K + 2)));
+        base_shift_kernel<<<(unsigned)((K + 256) / 256), 256, 0, st>>>(B, (uint64_t)K + 1, tsh, c.key_base_s);
+        c.launches++;
+        a.Bs = c.key_base_s;
+    }
     a.tab = tab;
-    a.nxh = npasses - 2;
+    a.nxh = coarse ? 0 : npasses - 2;
+    a.tsh = tsh;
     a.ks = ks;
     a.lomask = ks ? (ks >= 32 ? 0xffffffffull : (1ull << ks) - 1) : 0;
     {
@@ -546,12 +643,8 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         }
         a.pf = (uint32_t)pf;
     }
-    // ranking mode per pass (STEMROOT_SORT_RANK=match|ballot forces one)
-    static int rank_force = -2;
-    if (rank_force == -2) {
-        const char *e = getenv("STEMROOT_SORT_RANK");
-        rank_force = !e ? -1 : e[0] == 'b' ? 1 : e[0] == 'm' ? 0 : -1;
-    }
+    int rank_force = -1;   // STEMROOT_SORT_RANK=match|ballot forces one ranking mode
+    if (const char *e = getenv("STEMROOT_SORT_RANK")) rank_force = e[0] == 'b' ? 1 : e[0] == 'm' ? 0 : -1;
     uint32_t *mode = c.sort_mode;
     uint64_t *gbase = c.sort_gbase;
     rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 0, 2, n, rank_force, mode, gbase);   // key bytes 0, 1: pre-pass

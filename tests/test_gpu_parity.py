@@ -290,3 +290,33 @@ def test_sort_modes(ctx, monkeypatch, mode, eps):
     if mode.startswith("bits") and eps == 0.002:
         assert st["ambiguous_samples"] > 0
 
+
+
+@pytest.mark.parametrize("rank", ["match", "ballot"])
+@pytest.mark.parametrize("pack", ["0", "1"])
+def test_sort_ranking_modes(ctx, monkeypatch, rank, pack):
+    """each warp ranking method of the radix passes (match.any, 8 ballots)
+    in both key layouts gives the oracle's plan"""
+    monkeypatch.setenv("STEMROOT_SORT_RANK", rank)
+    monkeypatch.setenv("STEMROOT_SORT_PACK", pack)
+    rng = np.random.default_rng(99)
+    kid, t = _mixture(rng, 150_001, 300, peaks=3, spread=0.3)
+    got, ref = _both(ctx, kid, t, 300, eps=0.03, seed=5)
+    assert_plans_equal(got, ref)
+
+
+@pytest.mark.parametrize("coarse", ["0", "1"])
+@pytest.mark.parametrize("K", [3, 700])
+def test_key_bases_heavy_tails(ctx, sr, monkeypatch, coarse, K):
+    """fine (2^16) and coarse (2^24) kernel key bases; heavy tails put many
+    rows at t >= 2^24, which the coarse pass histograms take from the
+    per-kernel tail histogram of the pre-pass"""
+    monkeypatch.setenv("STEMROOT_SORT_COARSE", coarse)
+    rng = np.random.default_rng(K)
+    n = 300_007
+    kid = rng.integers(0, K, n).astype(np.uint32)
+    t = np.minimum(rng.lognormal(14 + (kid % 5), 1.6, n), 2 ** 32 - 1).astype(np.uint32)
+    t[::997] = 2 ** 32 - 1
+    got, ref = _both(ctx, kid, t, K, eps=0.05, seed=3)
+    assert_plans_equal(got, ref)
+    assert ctx.stats()["coarse_bases"] == (1 if coarse == "1" else 0)
