@@ -170,9 +170,9 @@ __global__ void coarse_hist_kernel(const uint32_t *__restrict__ cnt, const uint3
 // Per pass, from its digit histogram: the digit bases (exclusive scan) and
 // the ranking mode.  MATCH.ANY slows down as the number of distinct digits
 // among a warp's 32 keys approaches 32, while 8 ballots cost the same for any
-// digit mix.  Measured on B200 (C5, per pass ms match/ballot: 14.2/12.0,
-// 9.7/8.8, 8.5/8.6, 7.4/8.3, 7.3/8.6 at expected distinct digits 30.1, 29.8,
-// 26.1, 24.8, 9.9): ballots when E[distinct] >= 27.  force >= 0 fixes the mode.
+// digit mix.  Measured on B200 (C5, 5 passes; whole sort ms all-ballot /
+// all-match: first 6.8/9.4, mid 16.1/18.9, last (E[distinct] ~10) 5.8/5.3):
+// ballots when E[distinct] >= 16.  force >= 0 fixes the mode.
 __global__ void rank_mode_kernel(const uint64_t *__restrict__ hist, int p0, int p1, uint64_t n, int force,
                                  uint32_t *__restrict__ mode, uint64_t *__restrict__ gbase) {
     __shared__ double s_w[8];
@@ -197,10 +197,27 @@ __global__ void rank_mode_kernel(const uint64_t *__restrict__ hist, int p0, int 
         if (threadIdx.x == 0) {
             double tot = 0.0;
             for (int i = 0; i < 8; i++) tot += s_w[i];
-            mode[p] = force >= 0 ? (uint32_t)force : tot >= 27.0 ? 1u : 0u;
+            mode[p] = force >= 0 ? (uint32_t)force : tot >= 16.0 ? 1u : 0u;
         }
         __syncthreads();
     }
+}
+
+// Lanes of vmask whose 8-bit digit differs from this lane's d: one ballot per
+// bit, mismatches = ballot ^ (my bit ? ~0 : 0), OR-accumulated (4 SASS per bit).
+__device__ __forceinline__ uint32_t ballot_diff8(uint32_t d, uint32_t vmask) {
+    uint32_t diff;
+    asm("{\n\t.reg .pred p;\n\t.reg .b32 b, m, acc;\n\t"
+        "mov.b32 acc, 0;\n\t"
+#define SR_BAL_BIT(K) "and.b32 m, %1, " #K ";\n\tsetp.ne.u32 p, m, 0;\n\tvote.sync.ballot.b32 b, p, %2;\n\t" \
+                      "selp.b32 m, -1, 0, p;\n\txor.b32 b, b, m;\n\tor.b32 acc, acc, b;\n\t"
+        SR_BAL_BIT(1) SR_BAL_BIT(2) SR_BAL_BIT(4) SR_BAL_BIT(8) SR_BAL_BIT(16) SR_BAL_BIT(32) SR_BAL_BIT(64)
+        SR_BAL_BIT(128)
+#undef SR_BAL_BIT
+        "mov.b32 %0, acc;\n\t}"
+        : "=r"(diff)
+        : "r"(d), "r"(vmask));
+    return diff;
 }
 
 // ---------------------------------------------------------------- one-sweep pass
@@ -244,7 +261,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
     uint64_t *s_keys = reinterpret_cast<uint64_t *>(s_dyn);                           // [TILE]
     uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + TILE);                   // [TILE] (!PK)
     uint16_t (*s_whist)[R] = reinterpret_cast<uint16_t (*)[R]>(PK ? (void *)(s_keys + TILE) : (void *)(s_vals + TILE));
-    __shared__ uint64_t s_delta[R];
+    __shared__ uint32_t s_delta[R];   // global - local position, mod 2^32 (n < 2^32)
     __shared__ uint32_t s_lstart[R + 1];
     __shared__ uint32_t s_cnt[R];
     __shared__ uint32_t s_cw[NW];
@@ -338,12 +355,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             const uint32_t d = (uint32_t)(key[j] >> a.shift) & (R - 1);
             uint32_t peers;
             if (ballot) {
-                peers = vmask;
-#pragma unroll
-                for (int b = 0; b < kRB; b++) {
-                    const uint32_t bal = __ballot_sync(vmask, (d >> b) & 1u);
-                    peers &= ((d >> b) & 1u) ? bal : ~bal;
-                }
+                peers = vmask & ~ballot_diff8(d, vmask);
             } else {
                 peers = __match_any_sync(vmask, d);
             }
@@ -416,12 +428,12 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
                     const uint64_t v = sv[q];
                     if (v & kFlagP) { excl += v & kValMask; done = true; }
                     else if (v & kFlagA) { excl += v & kValMask; j--; }
-                    else break;   // not published yet: poll again from tile j
+                    else { __nanosleep(20); break; }   // not published yet: poll again from tile j
                 }
             }
             __stcg(a.status + (uint64_t)tile * R + d, kFlagP | (excl + cnt));
         }
-        s_delta[d] = a.gbase[a.pass * kHistR + d] + excl - s_lstart[d];   // global position - local position
+        s_delta[d] = (uint32_t)(a.gbase[a.pass * kHistR + d] + excl) - s_lstart[d];
     }
     __syncthreads();
     const uint32_t nvalid = s_lstart[R];
@@ -429,7 +441,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
     for (uint32_t i = tid; i < nvalid; i += NT) {
         const uint64_t k = s_keys[i];
         const uint32_t dd = (uint32_t)(k >> a.shift) & (R - 1);
-        const uint64_t gp = s_delta[dd] + i;
+        const uint32_t gp = s_delta[dd] + i;
         if (LAST) {
             const uint64_t kk = PK ? k >> a.ks : k;
             const uint32_t g = a.tab ? __ldg(a.tab + (kk >> a.tsh))
