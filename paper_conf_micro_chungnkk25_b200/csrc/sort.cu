@@ -171,10 +171,11 @@ __global__ void coarse_hist_kernel(const uint32_t *__restrict__ cnt, const uint3
 // the ranking mode.  MATCH.ANY slows down as the number of distinct digits
 // among a warp's 32 keys approaches 32, while 8 ballots cost the same for any
 // digit mix.  Measured on B200 (C5, 5 passes; whole sort ms all-ballot /
-// all-match: first 6.8/9.4, mid 16.1/18.9, last (E[distinct] ~10) 5.8/5.3):
-// ballots when E[distinct] >= 16.  force >= 0 fixes the mode.
+// all-match: first 6.8/9.4, mid 16.1/18.9, last 5.8/5.3; threshold 16/20/24:
+// last pass 5.09/5.09/4.76): ballots when E[distinct] >= 24.  force >= 0
+// fixes the mode.
 __global__ void rank_mode_kernel(const uint64_t *__restrict__ hist, int p0, int p1, uint64_t n, int force,
-                                 uint32_t *__restrict__ mode, uint64_t *__restrict__ gbase) {
+                                 double thr, uint32_t *__restrict__ mode, uint64_t *__restrict__ gbase) {
     __shared__ double s_w[8];
     __shared__ uint64_t s_c[8];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -197,7 +198,7 @@ __global__ void rank_mode_kernel(const uint64_t *__restrict__ hist, int p0, int 
         if (threadIdx.x == 0) {
             double tot = 0.0;
             for (int i = 0; i < 8; i++) tot += s_w[i];
-            mode[p] = force >= 0 ? (uint32_t)force : tot >= 16.0 ? 1u : 0u;
+            mode[p] = force >= 0 ? (uint32_t)force : tot >= thr ? 1u : 0u;
         }
         __syncthreads();
     }
@@ -503,15 +504,16 @@ static int launch_pass_cfg(const PassArgs &a, bool first, bool last, cudaStream_
 }
 
 // tile shapes (threads, keys per thread); STEMROOT_SORT_SHAPE picks one for
-// experiments.  384 x 12 measured fastest on B200 (profiles/README.md).
+// experiments.  256 x 20 (4 blocks/SM) measured fastest on B200 for packed keys
+// (C5 mid pass 5.07 ms vs 5.36 for 384 x 12, 5.09-5.29 for 256 x 16/24).
 struct Shape { int nt, it; };
-static const Shape kShapes[] = {{384, 12}, {384, 10}, {320, 14}};
+static const Shape kShapes[] = {{256, 20}, {384, 12}, {256, 24}, {256, 16}};
 static int shape_idx() {
     static int s = -1;
     if (s < 0) {
         const char *e = getenv("STEMROOT_SORT_SHAPE");
         s = e ? atoi(e) : 0;
-        if (s < 0 || s > 2) s = 0;
+        if (s < 0 || s > 3) s = 0;
     }
     return s;
 }
@@ -520,9 +522,10 @@ static uint64_t tile_keys() { return (uint64_t)kShapes[shape_idx()].nt * kShapes
 
 static int launch_sort_pass(const PassArgs &a, bool first, bool last, cudaStream_t st, uint32_t *launches) {
     switch (shape_idx()) {
-        case 1: return launch_pass_cfg<384, 10>(a, first, last, st, launches);
-        case 2: return launch_pass_cfg<320, 14>(a, first, last, st, launches);
-        default: return launch_pass_cfg<384, 12>(a, first, last, st, launches);
+        case 1: return launch_pass_cfg<384, 12>(a, first, last, st, launches);
+        case 2: return launch_pass_cfg<256, 24>(a, first, last, st, launches);
+        case 3: return launch_pass_cfg<256, 16>(a, first, last, st, launches);
+        default: return launch_pass_cfg<256, 20>(a, first, last, st, launches);
     }
 }
 
@@ -656,10 +659,12 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         a.pf = (uint32_t)pf;
     }
     int rank_force = -1;   // STEMROOT_SORT_RANK=match|ballot forces one ranking mode
+    double rank_thr = 24.0;   // STEMROOT_SORT_RANK_THR: ballots from this many expected distinct digits
+    if (const char *e = getenv("STEMROOT_SORT_RANK_THR")) rank_thr = atof(e);
     if (const char *e = getenv("STEMROOT_SORT_RANK")) rank_force = e[0] == 'b' ? 1 : e[0] == 'm' ? 0 : -1;
     uint32_t *mode = c.sort_mode;
     uint64_t *gbase = c.sort_gbase;
-    rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 0, 2, n, rank_force, mode, gbase);   // key bytes 0, 1: pre-pass
+    rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 0, 2, n, rank_force, rank_thr, mode, gbase);   // key bytes 0, 1: pre-pass
     c.launches++;
     a.ballot = mode;
     a.gbase = gbase;
@@ -690,7 +695,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         c.stage_end(tk, sbytes);
         CK(cudaGetLastError());
         if (first && npasses > 2) {   // higher bytes: histogrammed by pass 0
-            rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 2, npasses, n, rank_force, mode, gbase);
+            rank_mode_kernel<<<1, kR, 0, st>>>(c.hist, 2, npasses, n, rank_force, rank_thr, mode, gbase);
             c.launches++;
         }
         uint64_t *tkk = kin; kin = kout; kout = tkk;
