@@ -258,6 +258,7 @@ template <int NT, int IT, bool FIRST, bool LAST, bool FULL, bool PK>
 __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesweep_kernel(PassArgs a) {
     constexpr int NW = NT / 32, TILE = NT * IT, R = kR;
     static_assert(NT >= R, "one thread per digit");
+    static_assert(NT * IT <= 65536, "16-bit ranks");
     extern __shared__ __align__(16) unsigned char s_dyn[];
     uint64_t *s_keys = reinterpret_cast<uint64_t *>(s_dyn);                           // [TILE]
     uint32_t *s_vals = reinterpret_cast<uint32_t *>(s_keys + TILE);                   // [TILE] (!PK)
@@ -346,7 +347,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
 
     // warp-level multi-split ranking, in element order
     const uint32_t ballot = a.ballot[a.pass];
-    uint32_t rank[IT];
+    uint32_t rank2[(IT + 1) / 2];   // two 16-bit ranks per register (ranks < TILE <= 2^16)
 #pragma unroll
     for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
@@ -362,7 +363,8 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             }
             const uint32_t base = s_whist[w][d];
             const uint32_t below = __popc(peers & ((1u << lane) - 1));
-            rank[j] = base + below;
+            if (j & 1) rank2[j / 2] |= (base + below) << 16;
+            else rank2[j / 2] = base + below;
             __syncwarp(vmask);
             if (below == 0) s_whist[w][d] = (uint16_t)(base + __popc(peers));
         }
@@ -405,7 +407,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         if (FULL || i < a.n) {
             const uint32_t dd = (uint32_t)(key[j] >> a.shift) & (R - 1);
-            const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + rank[j];
+            const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + ((rank2[j / 2] >> (16 * (j & 1))) & 0xffffu);
             s_keys[lp] = key[j];
             if (!PK) s_vals[lp] = val[PK ? 0 : j];
         }

@@ -13,7 +13,12 @@ def main():
                                   stderr=subprocess.DEVNULL).decode()
     r = list(csv.reader(io.StringIO(out)))
     h = r[1]
-    rows = r[2:]
+    rows = []
+    for x in r[2:]:   # the first kernel's section only
+        if x and x[0].startswith("Kernel Name"):
+            break
+        if len(x) == len(h):
+            rows.append(x)
     ix = {k: i for i, k in enumerate(h)}
     S = ix["Warp Stall Sampling (All Samples)"]
     E = ix["Instructions Executed"]
