@@ -266,6 +266,7 @@ def run_ours(a):
                    else "inputs fit in L2: latency-bound workload",
                    "sort_key_bits": st["key_bits"], "sort_passes": st["sort_passes"],
                    "sort_row_bits_in_key": st["pack_bits"], "ambiguous_samples": st["ambiguous_samples"],
+                   "split_chunks": st["split_chunks"], "split_scanned": st["split_scanned"],
                    "root_levels": st["levels"], "clusters": dplan["n_clusters"], "samples": dplan["n_samples"],
                    "active_rows_over_levels": st["active_rows"]},
         "clocks": ck,

@@ -142,6 +142,8 @@ typedef struct stem_stats {
     uint32_t ambiguous_samples;/* samples whose row needed the run scan (packed mode)            */
     uint32_t coarse_bases;     /* 1: kernel key bases aligned to 2^24 (pass histograms from the pre-pass) */
     uint32_t reserved0;
+    uint64_t split_chunks;     /* 32-row chunks of big clusters bounded, summed over ROOT levels   */
+    uint64_t split_scanned;    /* of those, chunks scanned row by row (the rest pruned exactly)   */
 } stem_stats;
 
 /* Per-stage device time of the last plan (stem_ctx_enable_timing).  bytes is

@@ -103,7 +103,8 @@ class stem_stats(C.Structure):
     _fields_ = [("key_bits", C.c_uint32), ("sort_passes", C.c_uint32), ("levels", C.c_uint32),
                 ("kernel_launches", C.c_uint32), ("active_rows", C.c_uint64), ("n_clusters", C.c_uint64),
                 ("n_samples", C.c_uint64), ("ssum", C.c_double), ("pack_bits", C.c_uint32),
-                ("ambiguous_samples", C.c_uint32), ("coarse_bases", C.c_uint32), ("reserved0", C.c_uint32)]
+                ("ambiguous_samples", C.c_uint32), ("coarse_bases", C.c_uint32), ("reserved0", C.c_uint32),
+                ("split_chunks", C.c_uint64), ("split_scanned", C.c_uint64)]
 
 
 class stem_stage_time(C.Structure):

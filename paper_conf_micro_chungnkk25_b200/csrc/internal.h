@@ -46,6 +46,7 @@ struct DevScalars {
     alignas(16) uint64_t wide_total[4];   // total of a wide (struct) scan
     uint64_t red7[8];                     // multi-GPU reduction staging
     unsigned long long local_rows;        // rows scanned below the frontier (local subtrees)
+    unsigned long long split_chunks, split_scanned;   // big-cluster chunks bounded / scanned row by row
     uint32_t local_depth, amb_count;      // deepest ROOT level of a local subtree; ambiguous samples
 };
 

@@ -25,6 +25,7 @@ namespace sr {
 
 // clusters of >= big_rows() rows take the chunk-bound path (STEMROOT_BIG_ROWS overrides)
 __constant__ uint64_t c_big;
+__constant__ int c_bound2;   // 1: two-sided chunk bounds on the big path (STEMROOT_SPLIT_BOUND=1)
 static uint64_t big_rows() {
     static uint64_t v = 0;
     if (!v) {
@@ -260,6 +261,42 @@ __device__ __forceinline__ double div_lower(double x, double p) {
     return __dmul_rn(__dmul_rn(x, r), 1.0 - 0x1p-30);
 }
 
+// upper bound of x / p (x >= 0, p > 0): as div_lower, scaled up by 2^-30
+__device__ __forceinline__ double div_upper(double x, double p) {
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(p));
+    r = __fma_rn(r, __fma_rn(-p, r, 1.0), r);
+    return __dmul_rn(__dmul_rn(x, r), 1.0 + 0x1p-30);
+}
+
+// Upper bound of ad_k = S k - n S_L(k) (>= 0 for sorted rows) over the cuts
+// k in [ka, ka + cnt - 1] of one chunk, from A = ad_ka and the chunk's first
+// time ta.  ad is concave in k (its increments S - n t_j fall as t rises), so it
+// lies below the tangent at the chunk start (slope S - n ta) and, when the
+// exact E = ad at ka + cnt and the chunk's last time tl are known (has_e),
+// below the line through that point with slope S - n tl: the bound is the
+// value where the two lines cross.  fp64 with the roundings covered: every
+// term is nonnegative and within a few ulps of max(A, E), the crossing uses an
+// upward-rounded division, and the result gets 2^-46 max(A, E) of absolute
+// slack (the callers also scale it up).
+__device__ __forceinline__ double chunk_ad_bound(double A, uint64_t n, uint64_t S, uint32_t ta, uint64_t cnt,
+                                                 bool has_e, double E, uint32_t tl) {
+    const uint64_t nta = n * (uint64_t)ta;
+    if (S <= nta) return A;                                 // increments <= 0: the maximum is at ka
+    const double sa = __ull2double_rn(S - nta);
+    const double U1 = __dadd_rn(A, __dmul_rn(sa, (double)(cnt - 1)));   // tangent at the start
+    if (!has_e) return U1;
+    const double slack = __dmul_rn(fmax(A, E), 0x1p-46);
+    const uint64_t ntl = n * (uint64_t)tl;
+    if (S >= ntl) return fmin(U1, __dadd_rn(E, slack));      // increments >= 0: ad <= ad at ka + cnt
+    const double sb = __ull2double_rn(ntl - S);               // |last increment|
+    // A + sa x = E + sb (cnt - x) at x = (E - A + sb cnt) / (sa + sb)
+    const double num = __dadd_rn(__dsub_rn(E, A), __dmul_rn(sb, (double)cnt));
+    const double x = num > 0.0 ? div_upper(num, __dadd_rn(sa, sb)) : 0.0;
+    const double Uc = __dadd_rn(__dadd_rn(A, __dmul_rn(sa, x)), slack);
+    return fmin(U1, Uc);
+}
+
 // Warp scan of the rows [ra, rb) of a cluster starting at lo (S_L at ra = SLa):
 // every valid cut is scored exactly into best.
 __device__ __forceinline__ void scan_chunk(const uint32_t *__restrict__ t, uint64_t lo, uint64_t n, uint64_t S,
@@ -462,6 +499,7 @@ struct BigArgs {
     const uint32_t *TB;        // chunk-boundary pairs (t[32 j - 1], t[32 j])
     unsigned long long *thr;   // per cluster: bits of the best lower bound so far
     Cand *part;                // per entry
+    unsigned long long *n_chunks, *n_scanned;   // stats
 };
 
 constexpr int kBigThreads = 256;
@@ -514,11 +552,23 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
         const uint32_t ta = al ? tb.y : a.t[ra];
         s_sl[i] = SL;
         const u128 ad = (u128)S * ka - (u128)n * SL;
-        const uint64_t nta = n * (uint64_t)ta;
-        const double slope = S > nta ? __ull2double_rn(S - nta) : 0.0;
         const uint64_t cnt = rb - ra;
-        const double dub = __dmul_rn(__dadd_rn(approx_d((uint32_t)(ad >> 64), (uint64_t)ad),
-                                               __dmul_rn(slope, (double)(cnt - 1))), up);
+        bool has_e = false;
+        double E = 0.0;
+        uint32_t tl = 0;
+        if (c_bound2) {
+            if (rb == hi) {                          // ad = 0 at the cluster end
+                has_e = true;
+                tl = a.t[rb - 1];
+            } else if ((rb & (kChunk - 1)) == 0) {   // the next chunk's start (sampled prefix)
+                has_e = true;
+                const u128 ade = (u128)S * (rb - lo) - (u128)n * (a.PS1[rb >> kChunkLog] - s_base);
+                E = approx_d((uint32_t)(ade >> 64), (uint64_t)ade);
+                tl = reinterpret_cast<const uint2 *>(a.TB)[rb >> kChunkLog].x;
+            }
+        }
+        const double dub =
+            __dmul_rn(chunk_ad_bound(approx_d((uint32_t)(ad >> 64), (uint64_t)ad), n, S, ta, cnt, has_e, E, tl), up);
         const uint64_t kf = max((uint64_t)ka, (uint64_t)1), kl = min((uint64_t)ka + cnt - 1, n - 1);
         double ub = 0.0;
         if (kf <= kl) {
@@ -545,6 +595,10 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
     for (int i = tid; i < nq; i += kBigThreads)
         if (s_ub[i] >= thr && s_ub[i] > 0.0) s_list[atomicAdd(&s_nlist, 1u)] = (uint16_t)i;
     __syncthreads();
+    if (tid == 0) {   // stats: chunks bounded / scanned
+        atomicAdd(a.n_chunks, (unsigned long long)nq);
+        atomicAdd(a.n_scanned, (unsigned long long)s_nlist);
+    }
     // row-by-row scan of the surviving chunks: one warp per chunk, lane = row
     Cand best = no_cand();
     for (uint32_t li = w; li < s_nlist; li += kBigThreads / 32) {
@@ -839,6 +893,9 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CK(cudaMemcpyToSymbolAsync(c_big, &b, sizeof(b), 0, cudaMemcpyHostToDevice, st));
         const uint64_t l = local_rows() < b ? local_rows() : b;
         CK(cudaMemcpyToSymbolAsync(c_loc, &l, sizeof(l), 0, cudaMemcpyHostToDevice, st));
+        int b2 = 0;
+        if (const char *e = getenv("STEMROOT_SPLIT_BOUND")) b2 = atoi(e) ? 1 : 0;
+        CK(cudaMemcpyToSymbolAsync(c_bound2, &b2, sizeof(b2), 0, cudaMemcpyHostToDevice, st));
     }
     CKS(stem_only_leaves(c, n, K));
     // initial frontier: non-trivial kernel groups, in kernel order, with exact S and Q
@@ -918,7 +975,8 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         big_entries_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, ent,
                                                                        first_ent, &c.scalars->big_count);
         BigArgs ba{ent, &c.scalars->big_count, c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.PS1, c.t_sorted, c.TB,
-                   (unsigned long long *)c.big_thr, (Cand *)c.big_part};
+                   (unsigned long long *)c.big_thr, (Cand *)c.big_part, &c.scalars->split_chunks,
+                   &c.scalars->split_scanned};
         big_split_kernel<<<(unsigned)min(max_ent, (uint64_t)c.sms * 8), kBigThreads, 0, st>>>(ba);
         c.launches += 2;
         big_reduce_kernel<<<(unsigned)min(C, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, first_ent,
@@ -969,6 +1027,8 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
     if (hs.err & 4u) return STEM_E_CUDA;   // local stack overflow (unreachable)
     c.stats.levels = levels > hs.local_depth ? levels : hs.local_depth;
     c.stats.active_rows += hs.local_rows;
+    c.stats.split_chunks = hs.split_chunks;
+    c.stats.split_scanned = hs.split_scanned;
     return STEM_OK;
 }
 

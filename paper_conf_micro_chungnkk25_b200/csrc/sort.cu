@@ -241,6 +241,8 @@ struct PassArgs {
     int shift, pass;
     int nxh;                            // FIRST: key bytes 2 .. 2 + nxh - 1 histogrammed here
     uint32_t pf;                        // tiles ahead to prefetch into L2 (0 = off)
+    int late;                           // 1: publish the tile's digit counts after ranking
+    uint32_t nap;                       // look-back: ns to sleep before re-polling an unpublished status
     const uint32_t *ballot;             // [pass] 1: equal-digit lanes by 8 ballots, 0: match.any
     const uint64_t *gbase;              // [pass][kHistR] exclusive scan of the pass's digit counts
     uint64_t *hist;                     // [pass][kHistR] global digit counts
@@ -328,18 +330,22 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             if (!PK) val[PK ? 0 : j] = 0;
         }
     }
-    // the tile's digit counts, published at once so that successors' look-backs
-    // do not wait for this tile's ranking
+    // the tile's digit counts: either counted and published here, before
+    // ranking (successors' look-backs need not wait for it), or (a.late, the
+    // default: fewer instructions per key, measured faster) taken from the
+    // ranking's warp histograms and published after ranking
+    if (!a.late || (FIRST && a.nxh)) {
 #pragma unroll
-    for (int j = 0; j < IT; j++)
-        if (FULL || wbase + (uint64_t)j * 32 + lane < a.n) {
-            atomicAdd(&s_cnt[(uint32_t)(key[j] >> a.shift) & (R - 1)], 1u);
-            if (FIRST)
-                for (int x = 0; x < a.nxh; x++)
-                    atomicAdd(&s_xh[x * R + ((uint32_t)(key[j] >> (a.ks + kBaseShift + kRB * x)) & (R - 1))], 1u);
-        }
+        for (int j = 0; j < IT; j++)
+            if (FULL || wbase + (uint64_t)j * 32 + lane < a.n) {
+                if (!a.late) atomicAdd(&s_cnt[(uint32_t)(key[j] >> a.shift) & (R - 1)], 1u);
+                if (FIRST)
+                    for (int x = 0; x < a.nxh; x++)
+                        atomicAdd(&s_xh[x * R + ((uint32_t)(key[j] >> (a.ks + kBaseShift + kRB * x)) & (R - 1))], 1u);
+            }
+    }
     __syncthreads();
-    if (tid < R) __stcg(a.status + (uint64_t)tile * R + tid, (tile == 0 ? kFlagP : kFlagA) | s_cnt[tid]);
+    if (tid < R && !a.late) __stcg(a.status + (uint64_t)tile * R + tid, (tile == 0 ? kFlagP : kFlagA) | s_cnt[tid]);
     if (FIRST && tid < R)
         for (int x = 0; x < a.nxh; x++)
             if (s_xh[x * R + tid])
@@ -382,6 +388,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             s_whist[ww][d] = (uint16_t)cnt;
             cnt += c;
         }
+        if (a.late) __stcg(a.status + (uint64_t)tile * R + d, (tile == 0 ? kFlagP : kFlagA) | cnt);
         c_incl = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -431,7 +438,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
                     const uint64_t v = sv[q];
                     if (v & kFlagP) { excl += v & kValMask; done = true; }
                     else if (v & kFlagA) { excl += v & kValMask; j--; }
-                    else { __nanosleep(20); break; }   // not published yet: poll again from tile j
+                    else { if (a.nap) __nanosleep(a.nap); break; }   // not published yet: poll again from tile j
                 }
             }
             __stcg(a.status + (uint64_t)tile * R + d, kFlagP | (excl + cnt));
@@ -660,6 +667,12 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         }
         a.pf = (uint32_t)pf;
     }
+    a.nap = 20;
+    if (const char *e = getenv("STEMROOT_SORT_NAP")) a.nap = (uint32_t)atoi(e);
+    // publish the tile's counts after ranking (from the warp histograms): no
+    // separate counting of the keys (C5 mid pass 4.67 ms vs 4.94 counting first)
+    a.late = 1;
+    if (const char *e = getenv("STEMROOT_SORT_LATE")) a.late = atoi(e) ? 1 : 0;
     int rank_force = -1;   // STEMROOT_SORT_RANK=match|ballot forces one ranking mode
     double rank_thr = 24.0;   // STEMROOT_SORT_RANK_THR: ballots from this many expected distinct digits
     if (const char *e = getenv("STEMROOT_SORT_RANK_THR")) rank_thr = atof(e);
