@@ -35,7 +35,7 @@ int Ctx::ensure_all(uint64_t n, uint32_t K, uint32_t n_metrics) {
     CKS(ensure(scan_scratch, cap_scan, (scan_tiles((uint64_t)K + 2) + 1) * 32));
     CKS(ensure(PS1, cap_ps1, sizeof(uint64_t) * (n / kChunk + 2)));
     CKS(ensure(PS2, cap_ps2, sizeof(u128) * (n / kChunk + 2)));
-    CKS(ensure(flags, cap_flags, n + 16));
+    CKS(ensure(flags, cap_flags, sizeof(uint32_t) * (n / 32 + 4)));
     return STEM_OK;
 }
 

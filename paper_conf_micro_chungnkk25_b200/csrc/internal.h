@@ -179,7 +179,7 @@ struct Ctx {
     void *big_ent = nullptr, *big_part = nullptr, *big_thr = nullptr;
     size_t cap_big_ent = 0, cap_big_part = 0, cap_big_thr = 0;
     uint64_t *cnt_sz = nullptr; size_t cap_cntsz = 0;
-    uint8_t *flags = nullptr; size_t cap_flags = 0;
+    uint32_t *flags = nullptr; size_t cap_flags = 0;   // leaf-start bitmap: bit i & 31 of word i >> 5
     // leaves (a5/a6)
     uint32_t *leaf_lo = nullptr; size_t cap_leaf_lo = 0;
     uint64_t *leaf_m = nullptr, *leaf_moff = nullptr, *leaf_U = nullptr;

@@ -1,3 +1,4 @@
+#include <cstdio>
 // root.cu -- steps a2-a4: sampled exact prefix moments of the grouped times
 // and the level-synchronous ROOT clustering (§3.4, Fig. 6).
 //
@@ -40,6 +41,11 @@ constexpr uint64_t kBigSeg = 65536;                    // rows per block on the 
 // (STEMROOT_LOCAL_ROWS, default 0 = off: measured slower than the level loop
 // on C5)
 __constant__ uint64_t c_loc;
+static bool debug_levels() {
+    static int v = -1;
+    if (v < 0) v = getenv("STEMROOT_DEBUG_LEVELS") ? 1 : 0;
+    return v == 1;
+}
 static uint64_t local_rows() {
     static uint64_t v = ~0ull;
     if (v == ~0ull) {
@@ -57,75 +63,180 @@ __host__ __device__ __forceinline__ SQ operator+(const SQ &a, const SQ &b) { ret
 __host__ __device__ __forceinline__ SQ operator-(const SQ &a, const SQ &b) { return SQ{a.s - b.s, a.q - b.q}; }
 
 // ---------------------------------------------------------------- a2: sampled P1, P2
-// Sums of t and t^2 over every 32-row chunk.  Eight lanes cover one chunk with
-// one uint4 each, so one warp load is 512 contiguous bytes; four loads are in
-// flight per lane.
-// Also writes the chunk-boundary pairs TB[j] = (t[32 j - 1], t[32 j]) that the
-// split bounds read (8 B per chunk instead of two scattered sectors).
-__global__ void __launch_bounds__(256) chunk_sums_kernel(const uint32_t *__restrict__ t, uint64_t n, uint64_t nchunks,
-                                                         SQ *__restrict__ out, uint32_t *__restrict__ TB) {
-    constexpr int kUnroll = 4;
-    const int lane = threadIdx.x & 31, sub = lane & 7, grp = lane >> 3;
-    const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+// Three launches, each a coalesced stream (no look-back chain: a single-pass
+// decoupled look-back was measured slower, its tiles waiting on predecessors):
+//  1. pm_sums: a block per tile of kPmChunks 32-row chunks sums t and t^2 per
+//     chunk (eight lanes per chunk, one uint4 each, eight warp loads in
+//     flight), writes the chunk sums, the tile total and the chunk-boundary
+//     pairs TB[j] = (t[32 j - 1], t[32 j]) that the split bounds read;
+//  2. pm_tiles: one block scans the tile totals;
+//  3. pm_apply: a block per tile scans its chunk sums and writes PS1/PS2.
+// Element j of the scan is chunk j (zero for j >= nchunks), j in [0, nchunks].
+// Bytes: 4 per row + 24 + 24 + 24 (+ 8 TB) per chunk.
+constexpr int kPmThreads = 256, kPmChunks = 2 * kPmThreads;   // 16 384 rows per tile
+constexpr int kPmScanBlock = 1024;                                // tile totals per pm_tiles block
+struct SQ3 {   // chunk sums, 24 B
+    uint64_t s, lo, hi;
+};
+
+__device__ __forceinline__ void add128(uint64_t &lo, uint64_t &hi, uint64_t ol, uint64_t oh) {
+    const uint64_t nl = lo + ol;
+    hi += oh + (nl < lo);
+    lo = nl;
+}
+
+__global__ void __launch_bounds__(kPmThreads) pm_sums_kernel(const uint32_t *__restrict__ t, uint64_t n,
+                                                             uint64_t nchunks, SQ3 *__restrict__ csum,
+                                                             SQ *__restrict__ tile_tot, uint32_t *__restrict__ TB) {
+    __shared__ SQ s_part[kPmThreads / 32];
+    const int tid = threadIdx.x, lane = tid & 31, sub = lane & 3, grp = lane >> 2, w = tid >> 5;
+    const uint64_t c0 = (uint64_t)blockIdx.x * kPmChunks;
     const bool vec = (reinterpret_cast<uintptr_t>(t) & 15) == 0;
-    for (uint64_t base = warp * 4 * kUnroll; base < nchunks; base += nwarps * 4 * kUnroll) {
-        uint4 v[kUnroll];
+    // four lanes per chunk, two uint4 each (lane sub covers rows 8 sub .. 8 sub + 7
+    // of the chunk); eight chunks per warp step; kU steps of loads in flight
+    constexpr int kPerWarp = kPmChunks / (kPmThreads / 32), kU = 4;   // 64 chunks per warp
+    uint64_t as = 0, al = 0, ah = 0;
 #pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
-            const uint64_t j = base + u * 4 + grp;
-            const uint64_t i = j * kChunk + sub * 4;
-            if (vec && i + 3 < n) {
-                v[u] = __ldg(reinterpret_cast<const uint4 *>(t + i));
-            } else {
-                v[u].x = i < n ? t[i] : 0;
-                v[u].y = i + 1 < n ? t[i + 1] : 0;
-                v[u].z = i + 2 < n ? t[i + 2] : 0;
-                v[u].w = i + 3 < n ? t[i + 3] : 0;
+    for (int r = 0; r < kPerWarp / (8 * kU); r++) {
+        uint4 v[kU][2];
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+            const uint64_t j = c0 + w * kPerWarp + (r * kU + u) * 8 + grp;
+            const uint64_t i = j * kChunk + sub * 8;
+#pragma unroll
+            for (int h = 0; h < 2; h++) {
+                const uint64_t ih = i + 4 * h;
+                if (vec && ih + 3 < n) {
+                    v[u][h] = __ldcs(reinterpret_cast<const uint4 *>(t + ih));
+                } else {
+                    v[u][h].x = ih < n ? t[ih] : 0;
+                    v[u][h].y = ih + 1 < n ? t[ih + 1] : 0;
+                    v[u][h].z = ih + 2 < n ? t[ih + 2] : 0;
+                    v[u][h].w = ih + 3 < n ? t[ih + 3] : 0;
+                }
             }
         }
 #pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
-            const uint64_t x0 = v[u].x, x1 = v[u].y, x2 = v[u].z, x3 = v[u].w;
-            uint64_t s = x0 + x1 + x2 + x3;
-            u128 q = (u128)(x0 * x0) + (x1 * x1) + (u128)(x2 * x2) + (x3 * x3);
-            uint64_t qlo = (uint64_t)q, qhi = (uint64_t)(q >> 64);
+        for (int u = 0; u < kU; u++) {
+            uint64_t s = 0, qlo = 0, qhi = 0;
 #pragma unroll
-            for (int o = 4; o; o >>= 1) {
+            for (int h = 0; h < 2; h++) {
+                const uint64_t x0 = v[u][h].x, x1 = v[u][h].y, x2 = v[u][h].z, x3 = v[u][h].w;
+                s += x0 + x1 + x2 + x3;
+                const uint64_t a0 = x0 * x0, a1 = x1 * x1, a2 = x2 * x2, a3 = x3 * x3;
+                add128(qlo, qhi, a0, 0);
+                add128(qlo, qhi, a1, 0);
+                add128(qlo, qhi, a2, 0);
+                add128(qlo, qhi, a3, 0);
+            }
+#pragma unroll
+            for (int o = 2; o; o >>= 1) {
                 s += __shfl_xor_sync(0xffffffffu, s, o);
                 const uint64_t ol = __shfl_xor_sync(0xffffffffu, qlo, o), oh = __shfl_xor_sync(0xffffffffu, qhi, o);
-                const uint64_t nl = qlo + ol;
-                qhi += oh + (nl < qlo);
-                qlo = nl;
+                add128(qlo, qhi, ol, oh);
             }
-            const uint64_t j = base + u * 4 + grp;
-            if (sub == 0 && j < nchunks) {
-                out[j] = SQ{s, ((u128)qhi << 64) | qlo};
-                TB[2 * j + 1] = v[u].x;                 // t[32 j]
-                if (j == 0) TB[0] = 0;
+            const uint64_t j = c0 + w * kPerWarp + (r * kU + u) * 8 + grp;
+            if (sub == 0) {
+                as += s;
+                add128(al, ah, qlo, qhi);
+                if (j <= nchunks) csum[j] = SQ3{s, qlo, qhi};
+                if (j < nchunks) {
+                    TB[2 * j + 1] = v[u][0].x;                 // t[32 j]
+                    if (j == 0) TB[0] = 0;
+                }
             }
-            if (sub == 7 && j + 1 < nchunks) TB[2 * (j + 1)] = v[u].w;   // t[32 (j + 1) - 1]
+            if (sub == 3 && j + 1 < nchunks) TB[2 * (j + 1)] = v[u][1].w;   // t[32 (j + 1) - 1]
         }
+    }
+    // tile total (lanes sub != 0 hold zero)
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        as += __shfl_xor_sync(0xffffffffu, as, o);
+        const uint64_t ol = __shfl_xor_sync(0xffffffffu, al, o), oh = __shfl_xor_sync(0xffffffffu, ah, o);
+        add128(al, ah, ol, oh);
+    }
+    if (lane == 0) s_part[w] = SQ{as, ((u128)ah << 64) | al};
+    __syncthreads();
+    if (tid == 0) {
+        SQ tot{0, 0};
+        for (int k = 0; k < kPmThreads / 32; k++) tot = tot + s_part[k];
+        tile_tot[blockIdx.x] = tot;
+    }
+}
+
+// a block per kPmScanBlock tile totals: exclusive scan in place, the block's
+// total to btot[blockIdx]
+__global__ void __launch_bounds__(kPmScanBlock) pm_tiles_kernel(SQ *__restrict__ tile_tot, uint64_t ntiles,
+                                                                SQ *__restrict__ btot) {
+    __shared__ SQ sm[kPmScanBlock / 32 + 1];
+    const uint64_t i = (uint64_t)blockIdx.x * kPmScanBlock + threadIdx.x;
+    const SQ v = i < ntiles ? tile_tot[i] : SQ{0, 0};
+    SQ tot;
+    const SQ ex = block_excl_scan<SQ, kPmScanBlock>(v, sm, &tot);
+    if (i < ntiles) tile_tot[i] = ex;
+    if (threadIdx.x == 0) btot[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(kPmThreads) pm_apply_kernel(const SQ3 *__restrict__ csum, uint64_t nchunks,
+                                                              const SQ *__restrict__ tile_pre, const SQ *__restrict__ btot,
+                                                              uint64_t ntiles, uint64_t *__restrict__ PS1,
+                                                              u128 *__restrict__ PS2, uint64_t *__restrict__ total) {
+    __shared__ SQ s_scan[kPmThreads / 32 + 1];
+    __shared__ SQ s_base;
+    const int tid = threadIdx.x, lane = tid & 31;
+    if (tid < 32) {   // sum of the pm_tiles blocks before this tile's
+        const uint32_t nb = blockIdx.x / kPmScanBlock;
+        uint64_t bs = 0, bl = 0, bh = 0;
+        for (uint32_t k = lane; k < nb; k += 32) {
+            const SQ x = btot[k];
+            bs += x.s;
+            add128(bl, bh, (uint64_t)x.q, (uint64_t)(x.q >> 64));
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            bs += __shfl_xor_sync(0xffffffffu, bs, o);
+            const uint64_t ol = __shfl_xor_sync(0xffffffffu, bl, o), oh = __shfl_xor_sync(0xffffffffu, bh, o);
+            add128(bl, bh, ol, oh);
+        }
+        if (lane == 0) s_base = SQ{bs, ((u128)bh << 64) | bl} + tile_pre[blockIdx.x];
+    }
+    const uint64_t j0 = (uint64_t)blockIdx.x * kPmChunks + 2 * tid;
+    SQ e0{0, 0}, e1{0, 0};
+    if (j0 <= nchunks) { const SQ3 x = csum[j0]; e0 = SQ{x.s, ((u128)x.hi << 64) | x.lo}; }
+    if (j0 + 1 <= nchunks) { const SQ3 x = csum[j0 + 1]; e1 = SQ{x.s, ((u128)x.hi << 64) | x.lo}; }
+    SQ tot;
+    const SQ ex = block_excl_scan<SQ, kPmThreads>(e0 + e1, s_scan, &tot);   // (syncs: s_base visible)
+    const SQ p0 = s_base + ex, p1 = p0 + e0;
+    if (j0 + 1 <= nchunks) {
+        reinterpret_cast<ulonglong2 *>(PS1)[j0 >> 1] = make_ulonglong2(p0.s, p1.s);
+        PS2[j0] = p0.q;
+        PS2[j0 + 1] = p1.q;
+    } else if (j0 <= nchunks) {
+        PS1[j0] = p0.s;
+        PS2[j0] = p0.q;
+    }
+    if (tid == 0 && blockIdx.x + 1 == ntiles) {   // the tile holding element nchunks: grand total
+        const SQ g = s_base + tot;
+        total[0] = g.s;
+        total[1] = (uint64_t)g.q;
+        total[2] = (uint64_t)(g.q >> 64);
     }
 }
 
 int prefix_moments(Ctx &c, uint64_t n) {
     const uint64_t nchunks = (n + kChunk - 1) / kChunk;
-    CKS(c.ensure(c.chunk_sq, c.cap_chunk_sq, sizeof(SQ) * (nchunks + 1)));
-    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(nchunks + 1) + 1) * sizeof(SQ)));
-    const int tk = c.stage_begin("prefix_moments");
-    SQ *cs = (SQ *)c.chunk_sq;
+    const uint64_t ntiles = (nchunks + 1 + kPmChunks - 1) / kPmChunks;
+    const uint64_t nblk = (ntiles + kPmScanBlock - 1) / kPmScanBlock;
+    CKS(c.ensure(c.chunk_sq, c.cap_chunk_sq, sizeof(SQ3) * (ntiles * kPmChunks) + sizeof(SQ) * (ntiles + nblk + 1)));
     CKS(c.ensure(c.TB, c.cap_TB, sizeof(uint32_t) * 2 * (nchunks + 1)));
-    chunk_sums_kernel<<<c.sms * 8, 256, 0, c.stream>>>(c.t_sorted, n, nchunks, cs, c.TB);
-    c.launches++;
-    uint64_t *PS1 = c.PS1;
-    u128 *PS2 = c.PS2;
-    exclusive_scan<SQ>([cs, nchunks] __device__(uint64_t j) -> SQ { return j < nchunks ? cs[j] : SQ{0, 0}; },
-                       [PS1, PS2] __device__(uint64_t j, SQ pre, SQ) {
-                           PS1[j] = pre.s;
-                           PS2[j] = pre.q;
-                       },
-                       nchunks + 1, (SQ *)c.scan_scratch, (SQ *)c.scalars->wide_total, c.stream, &c.launches);
+    SQ3 *csum = (SQ3 *)c.chunk_sq;
+    SQ *ttot = (SQ *)(csum + ntiles * kPmChunks), *btot = ttot + ntiles;
+    const int tk = c.stage_begin("prefix_moments");
+    pm_sums_kernel<<<(unsigned)ntiles, kPmThreads, 0, c.stream>>>(c.t_sorted, n, nchunks, csum, ttot, c.TB);
+    pm_tiles_kernel<<<(unsigned)nblk, kPmScanBlock, 0, c.stream>>>(ttot, ntiles, btot);
+    pm_apply_kernel<<<(unsigned)ntiles, kPmThreads, 0, c.stream>>>(csum, nchunks, ttot, btot, ntiles, c.PS1, c.PS2,
+                                                                   c.scalars->wide_total);
+    c.launches += 3;
     c.stage_end(tk, 4 * n + 24 * (nchunks + 1));
     CK(cudaGetLastError());
     return STEM_OK;
@@ -504,9 +615,11 @@ struct BigArgs {
 
 constexpr int kBigThreads = 256;
 constexpr int kBigChunks = (int)(kBigSeg / kChunk) + 2;
+constexpr int kBigRounds = (kBigChunks + kBigThreads - 1) / kBigThreads;
 
-__global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
-    __shared__ double s_ub[kBigChunks];
+__global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
+    __shared__ double s_ub[kBigChunks];   // d2: the squared |D| bound of the chunk
+    __shared__ float s_pm[kBigChunks];    // min of k (n - k) over the chunk's cuts, rounded down (prunes less)
     __shared__ uint64_t s_sl[kBigChunks];
     __shared__ uint16_t s_list[kBigChunks];
     __shared__ uint32_t s_nlist;
@@ -535,20 +648,32 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
     const int nq = (int)(q1 - q0 + 1);
     const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
     double lbm = 0.0;
-    for (int i = tid; i < nq; i += kBigThreads) {
+    // every round's sampled-prefix and boundary loads in flight first
+    uint64_t pav[kBigRounds];
+    uint2 tbv[kBigRounds];
+#pragma unroll
+    for (int r = 0; r < kBigRounds; r++) {
+        const int i = tid + r * kBigThreads;
+        pav[r] = 0;
+        tbv[r] = make_uint2(0u, 0u);
+        if (i < nq) {
+            pav[r] = a.PS1[q0 + i];
+            tbv[r] = reinterpret_cast<const uint2 *>(a.TB)[q0 + i];
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < kBigRounds; r++) {
+        const int i = tid + r * kBigThreads;
+        if (i >= nq) break;
         const uint64_t q = q0 + i;
         const uint64_t ra = max(r0, q << kChunkLog), rb = min(r1, (q + 1) << kChunkLog);   // rows [ra, rb)
-        uint64_t pa;
-        if ((ra & (kChunk - 1)) == 0) {
-            pa = a.PS1[ra >> kChunkLog];
-        } else {   // only the block's first chunk can start unaligned
-            pa = a.PS1[ra >> kChunkLog];
+        uint64_t pa = pav[r];
+        const bool al = (ra & (kChunk - 1)) == 0;
+        if (!al)   // only the block's first chunk can start unaligned
             for (uint64_t x = ra & ~(kChunk - 1); x < ra; x++) pa += a.t[x];
-        }
         const uint64_t SL = pa - s_base;       // S_L at k_a = ra - lo (exact)
         const uint32_t ka = (uint32_t)(ra - lo);
-        const bool al = (ra & (kChunk - 1)) == 0;
-        const uint2 tb = al ? reinterpret_cast<const uint2 *>(a.TB)[ra >> kChunkLog] : make_uint2(0u, 0u);
+        const uint2 tb = al ? tbv[r] : make_uint2(0u, 0u);
         const uint32_t ta = al ? tb.y : a.t[ra];
         s_sl[i] = SL;
         const u128 ad = (u128)S * ka - (u128)n * SL;
@@ -570,15 +695,18 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
         const double dub =
             __dmul_rn(chunk_ad_bound(approx_d((uint32_t)(ad >> 64), (uint64_t)ad), n, S, ta, cnt, has_e, E, tl), up);
         const uint64_t kf = max((uint64_t)ka, (uint64_t)1), kl = min((uint64_t)ka + cnt - 1, n - 1);
-        double ub = 0.0;
+        // division-free: the chunk survives when d2 >= thr * pmin, d2 = RN(dub^2) (1 + 2^-43)
+        // covering the roundings (as warp_range_best)
+        double d2 = 0.0, pmin = 0.0;
         if (kf <= kl) {
-            const double pmin = fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
-            ub = __dmul_rn(__ddiv_rn(__dmul_rn(dub, dub), pmin), up);
+            pmin = fmin(__dmul_rn((double)kf, (double)(n - kf)), __dmul_rn((double)kl, (double)(n - kl)));
+            d2 = __dmul_rn(__dmul_rn(dub, dub), 1.0 + 0x1p-43);
         }
-        s_ub[i] = ub;
+        s_ub[i] = d2;
+        s_pm[i] = __double2float_rd(pmin);
         if (ka >= 1 && (al ? tb.x : a.t[ra - 1]) < ta) {   // the chunk start is a real candidate
             const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
-            lbm = fmax(lbm, __dmul_rn(__ddiv_rn(__dmul_rn(dD, dD), __dmul_rn((double)ka, (double)(n - ka))), dn));
+            lbm = fmax(lbm, div_lower(__dmul_rn(dD, dD), __dmul_rn((double)ka, (double)(n - ka))));
         }
     }
     for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));
@@ -591,33 +719,56 @@ __global__ void __launch_bounds__(kBigThreads) big_split_kernel(BigArgs a) {
         s_thr[0] = fmax(m, __longlong_as_double((long long)prev));   // positive doubles order as integers
     }
     __syncthreads();
-    const double thr = s_thr[0];
+    const double thr = __dmul_rn(s_thr[0], dn);
     for (int i = tid; i < nq; i += kBigThreads)
-        if (s_ub[i] >= thr && s_ub[i] > 0.0) s_list[atomicAdd(&s_nlist, 1u)] = (uint16_t)i;
+        if (s_ub[i] > 0.0 && s_ub[i] >= __dmul_rn(thr, (double)s_pm[i])) s_list[atomicAdd(&s_nlist, 1u)] = (uint16_t)i;
     __syncthreads();
     if (tid == 0) {   // stats: chunks bounded / scanned
         atomicAdd(a.n_chunks, (unsigned long long)nq);
         atomicAdd(a.n_scanned, (unsigned long long)s_nlist);
     }
-    // row-by-row scan of the surviving chunks: one warp per chunk, lane = row
+    // row-by-row scan of the surviving chunks: one warp per chunk, lane = row;
+    // kScanU chunks per warp step with their loads in flight first
+    constexpr int kScanU = 4, kNW = kBigThreads / 32;
     Cand best = no_cand();
-    for (uint32_t li = w; li < s_nlist; li += kBigThreads / 32) {
-        const int i = s_list[li];
-        const uint64_t q = q0 + i;
-        const uint64_t ra = max(r0, q << kChunkLog), rb = min(r1, (q + 1) << kChunkLog);
-        const uint64_t row = ra + lane;
-        const bool in = row < rb;
-        const uint32_t tc = in ? a.t[row] : 0u;
-        const uint32_t tp = (in && row > lo) ? a.t[row - 1] : 0u;
-        uint64_t incl = tc;
+    const uint32_t nlist = s_nlist;
+    for (uint32_t lb = w; lb < nlist; lb += kNW * kScanU) {
+        uint32_t tcv[kScanU], tpv[kScanU];
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += v;
+        for (int u = 0; u < kScanU; u++) {
+            const uint32_t li = lb + u * kNW;
+            tcv[u] = 0u;
+            tpv[u] = 0u;
+            if (li < nlist) {
+                const uint64_t q = q0 + s_list[li];
+                const uint64_t ra = max(r0, q << kChunkLog), rb = min(r1, (q + 1) << kChunkLog);
+                const uint64_t row = ra + lane;
+                if (row < rb) tcv[u] = a.t[row];
+                if (lane == 0 && row > lo) tpv[u] = a.t[row - 1];
+            }
         }
-        const uint64_t SLr = s_sl[i] + incl - tc;
-        const uint32_t k = (uint32_t)(row - lo);
-        if (in && k >= 1 && tp < tc) eval_cut(k, n, S, SLr, best);
+#pragma unroll
+        for (int u = 0; u < kScanU; u++) {
+            const uint32_t li = lb + u * kNW;
+            if (li >= nlist) break;
+            const int i = s_list[li];
+            const uint64_t q = q0 + i;
+            const uint64_t ra = max(r0, q << kChunkLog), rb = min(r1, (q + 1) << kChunkLog);
+            const uint64_t row = ra + lane;
+            const bool in = row < rb;
+            const uint32_t tc = tcv[u];
+            uint32_t tp = __shfl_up_sync(0xffffffffu, tc, 1);
+            if (lane == 0) tp = tpv[u];
+            uint64_t incl = tc;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += v;
+            }
+            const uint64_t SLr = s_sl[i] + incl - tc;
+            const uint32_t k = (uint32_t)(row - lo);
+            if (in && k >= 1 && tp < tc) eval_cut(k, n, S, SLr, best);
+        }
     }
 #pragma unroll
     for (int o = 16; o; o >>= 1) {
@@ -666,9 +817,11 @@ struct DecideArgs {
     const uint64_t *PS1;
     const u128 *PS2;
     const uint32_t *t;
-    uint8_t *flags;
-    uint64_t *cnt_sz;
-    u128 *cut_QL;
+    uint32_t *flags;   // leaf-start bitmap
+    uint32_t *nlo, *nhi;   // next frontier
+    uint64_t *nS;
+    u128 *nQ;
+    uint64_t *total;       // packed (count << 32 | rows) of the next frontier (zeroed before)
     double eps, z, k2;
     int clamp;
 };
@@ -711,32 +864,63 @@ __device__ __forceinline__ bool split_pays(uint64_t n, uint64_t S, u128 Q, uint6
     return tau_new < tau_old;
 }
 
-// clusters of >= local_rows() rows (the local kernel finishes the others)
+// clusters of >= local_rows() rows (the local kernel finishes the others).
+// Accepted cuts set their leaf-start bit, and the non-trivial children are
+// appended to the next frontier directly: a warp-aggregated atomicAdd on the
+// packed (count << 32 | rows) total gives each warp its slots.  The frontier
+// order is immaterial (leaves come from the bitmap, decisions from each
+// cluster's own rows), so no ordered compaction is needed.
 __global__ void __launch_bounds__(256) decide_kernel(DecideArgs a) {
     const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= a.C) return;
-    const uint32_t lo = a.f_lo[c], hi = a.f_hi[c], k = a.cut[c];
-    const uint64_t n = hi - lo;
-    if (n < c_loc) {   // finished by local_root_kernel
-        a.cnt_sz[c] = 0;
-        return;
+    const int lane = threadIdx.x & 31;
+    uint32_t lo = 0, hi = 0, mid = 0;
+    uint64_t S = 0, SL = 0;
+    u128 Q = 0, QL = 0;
+    bool ntL = false, ntR = false;
+    if (c < a.C) {
+        lo = a.f_lo[c];
+        hi = a.f_hi[c];
+        const uint32_t k = a.cut[c];
+        const uint64_t n = hi - lo;
+        if (n >= c_loc && k != 0) {   // n < c_loc: finished by local_root_kernel
+            mid = lo + k;
+            S = a.f_S[c];
+            SL = a.cut_SL[c];
+            Q = a.f_Q[c];
+            uint64_t s_lo, s_mid;
+            u128 q_lo, q_mid;
+            pref12(a.PS1, a.PS2, a.t, lo, s_lo, q_lo);
+            pref12(a.PS1, a.PS2, a.t, mid, s_mid, q_mid);
+            QL = q_mid - q_lo;
+            if (split_pays(n, S, Q, k, SL, QL, a.eps, a.z, a.k2, a.clamp)) {
+                atomicOr(&a.flags[mid >> 5], 1u << (mid & 31));
+                ntL = nontrivial(a.t, lo, mid);
+                ntR = nontrivial(a.t, mid, hi);
+            }
+        }
     }
-    const uint32_t mid = lo + k;
-    const uint64_t nL = k, nR = n - k;
-    const uint64_t S = a.f_S[c], SL = a.cut_SL[c];
-    uint64_t s_lo, s_mid;
-    u128 q_lo, q_mid;
-    pref12(a.PS1, a.PS2, a.t, lo, s_lo, q_lo);
-    pref12(a.PS1, a.PS2, a.t, mid, s_mid, q_mid);
-    const u128 QL = q_mid - q_lo;
-    uint64_t cs = 0;
-    if (k != 0 && split_pays(n, S, a.f_Q[c], k, SL, QL, a.eps, a.z, a.k2, a.clamp)) {
-        a.flags[mid] = 1;
-        const bool ntL = nontrivial(a.t, lo, mid), ntR = nontrivial(a.t, mid, hi);
-        cs = ((uint64_t)(ntL + ntR) << 32) | (uint64_t)((ntL ? nL : 0) + (ntR ? nR : 0));
+    // warp-aggregated append of (count << 32 | rows)
+    const uint64_t mine = ((uint64_t)(ntL + ntR) << 32) | (uint64_t)((ntL ? mid - lo : 0u) + (ntR ? hi - mid : 0u));
+    uint64_t incl = mine;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += v;
     }
-    a.cut_QL[c] = QL;
-    a.cnt_sz[c] = cs;
+    uint64_t base = 0;
+    const uint64_t wtot = __shfl_sync(0xffffffffu, incl, 31);
+    if (lane == 31 && wtot) base = atomicAdd((unsigned long long *)a.total, (unsigned long long)wtot);
+    base = __shfl_sync(0xffffffffu, base, 31);
+    uint32_t idx = (uint32_t)((base + incl - mine) >> 32);
+    if (ntL) {
+        a.nlo[idx] = lo; a.nhi[idx] = mid;
+        a.nS[idx] = SL; a.nQ[idx] = QL;
+        idx++;
+    }
+    if (ntR) {
+        a.nlo[idx] = mid; a.nhi[idx] = hi;
+        a.nS[idx] = S - SL; a.nQ[idx] = Q - QL;
+    }
 }
 
 // ---------------------------------------------------------------- local subtrees
@@ -760,7 +944,7 @@ struct LocalArgs {
     const uint64_t *PS1;
     const u128 *PS2;
     const uint32_t *t, *TB;
-    uint8_t *flags;
+    uint32_t *flags;   // leaf-start bitmap
     double eps, z, k2;
     int clamp;
     unsigned long long *rows;   // stats: rows scanned
@@ -815,7 +999,7 @@ __global__ void __launch_bounds__(256) local_root_kernel(LocalArgs a) {
                 const u128 QL = (a.PS2[mid >> kChunkLog] + warp_partial_sq(a.t, mid)) -
                                 (a.PS2[cur.lo >> kChunkLog] + warp_partial_sq(a.t, cur.lo));
                 if (split_pays(n, cur.S, cur.Q, b.k, b.SL, QL, a.eps, a.z, a.k2, a.clamp)) {
-                    if (lane == 0) a.flags[mid] = 1;
+                    if (lane == 0) atomicOr(&a.flags[mid >> 5], 1u << (mid & 31));
                     LNode L{b.SL, QL, cur.lo, mid, cur.depth + 1, 0};
                     LNode R{cur.S - b.SL, cur.Q - QL, mid, cur.hi, cur.depth + 1, 0};
                     const bool ntL = nontrivial(a.t, cur.lo, mid), ntR = nontrivial(a.t, mid, cur.hi);
@@ -855,9 +1039,9 @@ __global__ void __launch_bounds__(256) local_root_kernel(LocalArgs a) {
 }
 
 // ---------------------------------------------------------------- frontier bookkeeping
-__global__ void group_flags_kernel(const uint32_t *goff, uint32_t K, uint8_t *flags) {
+__global__ void group_flags_kernel(const uint32_t *goff, uint32_t K, uint32_t *flags) {
     const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (g < K && goff[g] < goff[g + 1]) flags[goff[g]] = 1;
+    if (g < K && goff[g] < goff[g + 1]) atomicOr(&flags[goff[g] >> 5], 1u << (goff[g] & 31));
 }
 
 static int read_frontier_total(Ctx &c, uint64_t &C, uint64_t &A) {
@@ -870,7 +1054,7 @@ static int read_frontier_total(Ctx &c, uint64_t &C, uint64_t &A) {
 }
 
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K) {
-    CK(cudaMemsetAsync(c.flags, 0, n + 1, c.stream));
+    CK(cudaMemsetAsync(c.flags, 0, sizeof(uint32_t) * (n / 32 + 1), c.stream));
     group_flags_kernel<<<(unsigned)((K + 255) / 256), 256, 0, c.stream>>>(c.goff, K, c.flags);
     c.launches++;
     CK(cudaGetLastError());
@@ -880,7 +1064,6 @@ int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K) {
 static int ensure_frontier(Ctx &c, int b, uint64_t cap) {
     CKS(c.ensure(c.f_lo[b], c.cap_flo[b], sizeof(uint32_t) * cap));
     CKS(c.ensure(c.f_hi[b], c.cap_fhi[b], sizeof(uint32_t) * cap));
-    CKS(c.ensure(c.f_aoff[b], c.cap_faoff[b], sizeof(uint32_t) * cap));
     CKS(c.ensure(c.f_S[b], c.cap_fS[b], sizeof(uint64_t) * cap));
     CKS(c.ensure(c.f_Q[b], c.cap_fQ[b], sizeof(u128) * cap));
     return STEM_OK;
@@ -905,7 +1088,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         const uint32_t *goff = c.goff, *t = c.t_sorted;
         const uint64_t *PS1 = c.PS1;
         const u128 *PS2 = c.PS2;
-        uint32_t *nlo = c.f_lo[0], *nhi = c.f_hi[0], *nao = c.f_aoff[0];
+        uint32_t *nlo = c.f_lo[0], *nhi = c.f_hi[0];
         uint64_t *nS = c.f_S[0];
         u128 *nQ = c.f_Q[0];
         const int tk = c.stage_begin("root_init");
@@ -914,7 +1097,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                 const uint32_t lo = goff[g], hi = goff[g + 1];
                 return nontrivial(t, lo, hi) ? ((1ull << 32) | (hi - lo)) : 0ull;
             },
-            [nlo, nhi, nao, nS, nQ, goff, t, PS1, PS2] __device__(uint64_t g, uint64_t pre, uint64_t v) {
+            [nlo, nhi, nS, nQ, goff, t, PS1, PS2] __device__(uint64_t g, uint64_t pre, uint64_t v) {
                 if (!v) return;
                 const uint32_t idx = (uint32_t)(pre >> 32), lo = goff[g], hi = goff[g + 1];
                 uint64_t s0, s1;
@@ -923,7 +1106,6 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                 pref12(PS1, PS2, t, hi, s1, q1);
                 nlo[idx] = lo;
                 nhi[idx] = hi;
-                nao[idx] = (uint32_t)pre;
                 nS[idx] = s1 - s0;
                 nQ[idx] = q1 - q0;
             },
@@ -940,8 +1122,6 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         c.stats.active_rows += A;
         CKS(c.ensure(c.cut, c.cap_cut, sizeof(uint32_t) * C));
         CKS(c.ensure(c.cut_SL, c.cap_cut_SL, sizeof(uint64_t) * C));
-        CKS(c.ensure(c.cut_QL, c.cap_cut_QL, sizeof(u128) * C));
-        CKS(c.ensure(c.cnt_sz, c.cap_cntsz, sizeof(uint64_t) * C));
         CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(C) + 1) * sizeof(uint64_t)));
         const int nxt = cur ^ 1;
         CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
@@ -985,39 +1165,21 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         c.stage_end(tk_s, 4 * A + 20 * C);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");
+        CK(cudaMemsetAsync(&c.scalars->frontier_total, 0, sizeof(uint64_t), st));
         DecideArgs da{c.f_lo[cur], c.f_hi[cur], c.cut, c.f_S[cur], c.cut_SL, c.f_Q[cur], (uint32_t)C, c.PS1, c.PS2,
-                      c.t_sorted, c.flags, c.cnt_sz, c.cut_QL, eps, z, k2, clamp};
+                      c.t_sorted, c.flags, c.f_lo[nxt], c.f_hi[nxt], c.f_S[nxt], c.f_Q[nxt],
+                      &c.scalars->frontier_total, eps, z, k2, clamp};
         decide_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(da);
         c.launches += 1;
         c.stage_end(tk_d, 96 * C);
         CK(cudaGetLastError());
-        const int tk_c = c.stage_begin("root_compact");
-        const uint32_t *flo = c.f_lo[cur], *fhi = c.f_hi[cur], *fcut = c.cut, *t = c.t_sorted;
-        const uint64_t *cs = c.cnt_sz, *fS = c.f_S[cur], *cSL = c.cut_SL;
-        const u128 *fQ = c.f_Q[cur], *cQL = c.cut_QL;
-        uint32_t *nlo = c.f_lo[nxt], *nhi = c.f_hi[nxt], *nao = c.f_aoff[nxt];
-        uint64_t *nS = c.f_S[nxt];
-        u128 *nQ = c.f_Q[nxt];
-        exclusive_scan<uint64_t>(
-            [cs] __device__(uint64_t i) -> uint64_t { return cs[i]; },
-            [flo, fhi, fcut, t, fS, cSL, fQ, cQL, nlo, nhi, nao, nS, nQ] __device__(uint64_t i, uint64_t pre,
-                                                                                   uint64_t v) {
-                if (!v) return;
-                uint32_t idx = (uint32_t)(pre >> 32), off = (uint32_t)pre;
-                const uint32_t lo = flo[i], hi = fhi[i], mid = lo + fcut[i];
-                if (nontrivial(t, lo, mid)) {
-                    nlo[idx] = lo; nhi[idx] = mid; nao[idx] = off;
-                    nS[idx] = cSL[i]; nQ[idx] = cQL[i];
-                    idx++; off += mid - lo;
-                }
-                if (nontrivial(t, mid, hi)) {
-                    nlo[idx] = mid; nhi[idx] = hi; nao[idx] = off;
-                    nS[idx] = fS[i] - cSL[i]; nQ[idx] = fQ[i] - cQL[i];
-                }
-            },
-            C, (uint64_t *)c.scan_scratch, &c.scalars->frontier_total, st, &c.launches);
-        c.stage_end(tk_c, 48 * C);
-        CK(cudaGetLastError());
+        if (debug_levels()) {   // STEMROOT_DEBUG_LEVELS=1: per-level frontier and big-path stats on stderr
+            DevScalars hs;
+            CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            fprintf(stderr, "level %u: clusters %llu rows %llu big_entries %u chunks %llu scanned %llu\n", levels,
+                    (unsigned long long)C, (unsigned long long)A, hs.big_count, hs.split_chunks, hs.split_scanned);
+        }
         CKS(read_frontier_total(c, C, A));
         cur = nxt;
     }

@@ -128,9 +128,12 @@ __global__ void kid_table_kernel(const uint64_t *__restrict__ B, uint32_t K, uin
     tab[j] = (uint32_t)(upper_bound(B, (uint64_t)K + 1, j << tsh) - 1);
 }
 
-__global__ void base_shift_kernel(const uint64_t *__restrict__ B, uint64_t m, int tsh, uint32_t *__restrict__ Bs) {
+__global__ void base_shift_kernel(const uint64_t *__restrict__ B, uint64_t m, int tsh, uint32_t *__restrict__ Bs,
+                                  uint16_t *__restrict__ Bs16) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i < m) Bs[i] = (uint32_t)(B[i] >> tsh);
+    if (i >= m) return;
+    if (Bs16) Bs16[i] = (uint16_t)(B[i] >> tsh);
+    else Bs[i] = (uint32_t)(B[i] >> tsh);
 }
 
 // Coarse bases: histograms of key bytes 2 .. npasses-1 from the pre-pass.
@@ -222,6 +225,13 @@ __device__ __forceinline__ uint32_t ballot_diff8(uint32_t d, uint32_t vmask) {
 }
 
 // ---------------------------------------------------------------- one-sweep pass
+// a streaming 4-byte load that does not allocate in L1
+__device__ __forceinline__ uint32_t ld_na(const uint32_t *p) {
+    uint32_t v;
+    asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(v) : "l"(p));   // read-only for the kernel
+    return v;
+}
+
 struct PassArgs {
     const uint32_t *kid_in, *t_in;      // FIRST: trace columns
     const uint32_t *row_in;             // FIRST: row payload (NULL = the row index)
@@ -232,6 +242,7 @@ struct PassArgs {
     uint32_t *t_out, *row_out;          // LAST
     const uint64_t *B;                  // [K + 1] key base per kernel
     const uint32_t *Bs;                 // [K + 1] B >> tsh (FIRST: a 4-byte gather that stays in L1)
+    const uint16_t *Bs16;               // [K + 1] B >> tsh when it fits 16 bits (a 2-byte gather: half the L1 room)
     const uint32_t *tab;                // LAST: kid table (NULL: binary search over B)
     int tsh;                            // B[k] is a multiple of 2^tsh; LAST: kid-table index = key >> tsh
     uint64_t n;
@@ -242,6 +253,7 @@ struct PassArgs {
     int nxh;                            // FIRST: key bytes 2 .. 2 + nxh - 1 histogrammed here
     uint32_t pf;                        // tiles ahead to prefetch into L2 (0 = off)
     int late;                           // 1: publish the tile's digit counts after ranking
+    int noalloc;                        // FIRST: stream kid / t past L1 (keeps the B[kid] table resident)
     uint32_t nap;                       // look-back: ns to sleep before re-polling an unpublished status
     const uint32_t *ballot;             // [pass] 1: equal-digit lanes by 8 ballots, 0: match.any
     const uint64_t *gbase;              // [pass][kHistR] exclusive scan of the pass's digit counts
@@ -312,9 +324,10 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         if (FULL || i < a.n) {
             if (FIRST) {
-                const uint32_t kd = __ldg(a.kid_in + i);
-                const uint64_t kb = a.Bs ? (uint64_t)__ldg(a.Bs + kd) << a.tsh : __ldg(a.B + kd);
-                const uint64_t kk = kb + (uint64_t)__ldg(a.t_in + i);
+                const uint32_t kd = a.noalloc ? ld_na(a.kid_in + i) : __ldg(a.kid_in + i);
+                const uint64_t kb = a.Bs16 ? (uint64_t)__ldg(a.Bs16 + kd) << a.tsh
+                                    : a.Bs ? (uint64_t)__ldg(a.Bs + kd) << a.tsh : __ldg(a.B + kd);
+                const uint64_t kk = kb + (uint64_t)(a.noalloc ? ld_na(a.t_in + i) : __ldg(a.t_in + i));
                 if (PK) {
                     key[j] = (kk << a.ks) | (i & a.lomask);
                 } else {
@@ -466,6 +479,18 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
 }
 
 // ---------------------------------------------------------------- host driver
+// resident blocks per SM the first pass leaves L1 room for (its B[kid] gather
+// table lives in L1); STEMROOT_FIRST_BLOCKS overrides
+static int first_blocks() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("STEMROOT_FIRST_BLOCKS");
+        v = e ? atoi(e) : 3;
+        if (v < 1 || v > 4) v = 3;
+    }
+    return v;
+}
+
 // full tiles in one launch (no bounds checks), the ragged last tile in a second
 // launch: its look-back finds every predecessor already inclusive
 template <int NT, int IT, bool FIRST, bool LAST, bool PK>
@@ -477,8 +502,8 @@ static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
     if (!attr) {
         CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true, PK>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        // FIRST gathers B[kid]: keep L1 beside three blocks' shared memory
-        const int carve = FIRST ? (int)((3 * (smem + 12 * 1024) * 100 + 228 * 1024 - 1) / (228 * 1024)) : 100;
+        // FIRST gathers B[kid]: keep L1 beside first_blocks() blocks' shared memory
+        const int carve = FIRST ? (int)((first_blocks() * (smem + 12 * 1024) * 100 + 228 * 1024 - 1) / (228 * 1024)) : 100;
         CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true, PK>,
                                 cudaFuncAttributePreferredSharedMemoryCarveout, carve > 100 ? 100 : carve));
         CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false, PK>,
@@ -648,11 +673,15 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     a.K = K;
     a.B = B;
     a.Bs = nullptr;
-    if ((range >> tsh) < (1ull << 32)) {   // bases >> tsh fit 32 bits
+    a.Bs16 = nullptr;
+    if ((range >> tsh) < (1ull << 32)) {   // bases >> tsh fit 32 (or 16) bits
+        const bool b16 = (range >> tsh) < (1ull << 16) && !(getenv("STEMROOT_SORT_BS16") && getenv("STEMROOT_SORT_BS16")[0] == '0');
         CKS(c.ensure(c.key_base_s, c.cap_kbase_s, sizeof(uint32_t) * ((uint64_t)K + 2)));
-        base_shift_kernel<<<(unsigned)((K + 256) / 256), 256, 0, st>>>(B, (uint64_t)K + 1, tsh, c.key_base_s);
+        base_shift_kernel<<<(unsigned)((K + 256) / 256), 256, 0, st>>>(B, (uint64_t)K + 1, tsh, b16 ? nullptr : c.key_base_s,
+                                                                       b16 ? (uint16_t *)c.key_base_s : nullptr);
         c.launches++;
-        a.Bs = c.key_base_s;
+        if (b16) a.Bs16 = (const uint16_t *)c.key_base_s;
+        else a.Bs = c.key_base_s;
     }
     a.tab = tab;
     a.nxh = coarse ? 0 : npasses - 2;
@@ -672,6 +701,8 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     // publish the tile's counts after ranking (from the warp histograms): no
     // separate counting of the keys (C5 mid pass 4.67 ms vs 4.94 counting first)
     a.late = 1;
+    a.noalloc = 1;
+    if (const char *e = getenv("STEMROOT_SORT_NOALLOC")) a.noalloc = atoi(e) ? 1 : 0;
     if (const char *e = getenv("STEMROOT_SORT_LATE")) a.late = atoi(e) ? 1 : 0;
     int rank_force = -1;   // STEMROOT_SORT_RANK=match|ballot forces one ranking mode
     double rank_thr = 24.0;   // STEMROOT_SORT_RANK_THR: ballots from this many expected distinct digits

@@ -54,50 +54,51 @@ __device__ double fix_round(const uint64_t *lane) {
 }
 
 // ---------------------------------------------------------------- leaf table
-// leaf starts = positions of the 0/1 flag bytes; tile = 256 threads x 64 bytes
-constexpr int kFlagBytes = 64;
-constexpr uint64_t kFlagTile = (uint64_t)kThreads * kFlagBytes;
+// leaf starts = the set bits of the leaf-start bitmap (bit i & 31 of word
+// i >> 5); tile = 256 threads x 8 words (65 536 rows), two uint4 per thread
+constexpr int kFlagWords = 8;
+constexpr uint64_t kFlagTileW = (uint64_t)kThreads * kFlagWords;
 
-__device__ __forceinline__ uint32_t flags_word(const uint8_t *f, uint64_t n, uint64_t i) {   // 4 flags at i
-    if (i + 3 < n) return *reinterpret_cast<const uint32_t *>(f + i);
-    uint32_t w = 0;
-    for (int b = 0; b < 4; b++)
-        if (i + b < n) w |= (uint32_t)f[i + b] << (8 * b);
-    return w;
+__device__ __forceinline__ void flag_words(const uint32_t *f, uint64_t nw, uint64_t w0, uint32_t (&wv)[kFlagWords]) {
+    if (w0 + kFlagWords <= nw) {
+        const uint4 a = __ldcs(reinterpret_cast<const uint4 *>(f + w0)), b = __ldcs(reinterpret_cast<const uint4 *>(f + w0 + 4));
+        wv[0] = a.x; wv[1] = a.y; wv[2] = a.z; wv[3] = a.w; wv[4] = b.x; wv[5] = b.y; wv[6] = b.z; wv[7] = b.w;
+    } else {
+#pragma unroll
+        for (int q = 0; q < kFlagWords; q++) wv[q] = w0 + q < nw ? f[w0 + q] : 0u;
+    }
 }
 
-__global__ void __launch_bounds__(kThreads) flag_count_kernel(const uint8_t *__restrict__ flags, uint64_t n,
+__global__ void __launch_bounds__(kThreads) flag_count_kernel(const uint32_t *__restrict__ flags, uint64_t nw,
                                                              uint64_t *__restrict__ tile_cnt) {
     __shared__ uint64_t sm[kThreads / 32 + 1];
-    const uint64_t i0 = blockIdx.x * kFlagTile + (uint64_t)threadIdx.x * kFlagBytes;
+    uint32_t wv[kFlagWords];
+    flag_words(flags, nw, blockIdx.x * kFlagTileW + (uint64_t)threadIdx.x * kFlagWords, wv);
     uint64_t c = 0;
 #pragma unroll
-    for (int q = 0; q < kFlagBytes; q += 4) c += __popc(flags_word(flags, n, i0 + q));
+    for (int q = 0; q < kFlagWords; q++) c += __popc(wv[q]);
     uint64_t tot;
     block_excl_scan<uint64_t, kThreads>(c, sm, &tot);
     if (threadIdx.x == 0) tile_cnt[blockIdx.x] = tot;
 }
 
-__global__ void __launch_bounds__(kThreads) flag_compact_kernel(const uint8_t *__restrict__ flags, uint64_t n,
+__global__ void __launch_bounds__(kThreads) flag_compact_kernel(const uint32_t *__restrict__ flags, uint64_t nw,
                                                                const uint64_t *__restrict__ tile_off,
                                                                uint32_t *__restrict__ leaf_lo) {
     __shared__ uint64_t sm[kThreads / 32 + 1];
-    const uint64_t i0 = blockIdx.x * kFlagTile + (uint64_t)threadIdx.x * kFlagBytes;
-    uint32_t wv[kFlagBytes / 4];
+    const uint64_t w0 = blockIdx.x * kFlagTileW + (uint64_t)threadIdx.x * kFlagWords;
+    uint32_t wv[kFlagWords];
+    flag_words(flags, nw, w0, wv);
     uint64_t c = 0;
 #pragma unroll
-    for (int q = 0; q < kFlagBytes / 4; q++) {
-        wv[q] = flags_word(flags, n, i0 + 4 * q);
-        c += __popc(wv[q]);
-    }
+    for (int q = 0; q < kFlagWords; q++) c += __popc(wv[q]);
     uint64_t tot;
     uint64_t pos = block_excl_scan<uint64_t, kThreads>(c, sm, &tot) + tile_off[blockIdx.x];
 #pragma unroll
-    for (int q = 0; q < kFlagBytes / 4; q++) {
+    for (int q = 0; q < kFlagWords; q++) {
         uint32_t x = wv[q];
         while (x) {
-            const int b = __ffs(x) - 1;               // bit 8*j marks byte j
-            leaf_lo[pos++] = (uint32_t)(i0 + 4 * q + (b >> 3));
+            leaf_lo[pos++] = (uint32_t)((w0 + q) * 32 + (uint32_t)(__ffs(x) - 1));
             x &= x - 1;
         }
     }
@@ -489,18 +490,18 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     CKS(c.ensure(c.leaf_lo, c.cap_leaf_lo, sizeof(uint32_t) * (n + 1)));
     const int tk_leaf = c.stage_begin("leaf_table");
     {
-        const uint64_t nt = (n + kFlagTile - 1) / kFlagTile;
+        const uint64_t nw = (n + 31) / 32, nt = (nw + kFlagTileW - 1) / kFlagTileW;   // bits >= n are never set
         CKS(c.ensure(c.leaf_moff, c.cap_leaf_moff, sizeof(uint64_t) * (nt + 1)));   // tile counts (scratch)
         uint64_t *tcnt = c.leaf_moff;
-        if (nt) flag_count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, n, tcnt);
+        if (nt) flag_count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, nw, tcnt);
         exclusive_scan<uint64_t>([tcnt] __device__(uint64_t i) -> uint64_t { return tcnt[i]; },
                                  [tcnt] __device__(uint64_t i, uint64_t pre, uint64_t) { tcnt[i] = pre; }, nt,
                                  (uint64_t *)c.scan_scratch, &c.scalars->n_leaves, st, &c.launches);
-        if (nt) flag_compact_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, n, tcnt, c.leaf_lo);
+        if (nt) flag_compact_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, nw, tcnt, c.leaf_lo);
         c.launches += 2;
         CK(cudaGetLastError());
     }
-    c.stage_end(tk_leaf, n);
+    c.stage_end(tk_leaf, 2 * 4 * (n / 32 + 1));
     uint64_t L = 0;
     CK(cudaMemcpyAsync(&L, &c.scalars->n_leaves, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));

@@ -1,6 +1,6 @@
 """Top SASS instructions of an ncu report by warp-stall samples, with their stall reasons.
 
-    python tools/sass_hot.py report.ncu-rep [N]"""
+    python tools/sass_hot.py report.ncu-rep [N] [kernel-regex]"""
 import csv
 import io
 import subprocess
@@ -9,7 +9,8 @@ import sys
 
 def main():
     rep, top = sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 30
-    out = subprocess.check_output(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+    filt = ["-k", "regex:" + sys.argv[3]] if len(sys.argv) > 3 else []
+    out = subprocess.check_output(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"] + filt,
                                   stderr=subprocess.DEVNULL).decode()
     r = list(csv.reader(io.StringIO(out)))
     h = r[1]
