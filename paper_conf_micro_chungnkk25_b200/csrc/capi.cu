@@ -47,6 +47,11 @@ static void dfree(T *&p, size_t &cap) {
 }
 
 void Ctx::release() {
+    if (ev_fork) cudaEventDestroy(ev_fork);
+    if (ev_join) cudaEventDestroy(ev_join);
+    if (side) cudaStreamDestroy(side);
+    ev_fork = ev_join = nullptr;
+    side = nullptr;
     dfree(in_kid, cap_in_kid); dfree(in_t, cap_in_t); dfree(in_met, cap_in_met);
     for (int i = 0; i < 2; i++) {
         dfree(keys[i], cap_keys[i]); dfree(vals[i], cap_vals[i]);

@@ -102,6 +102,8 @@ struct Ctx {
     uint32_t kid_base = 0;         // global id of local kernel 0 (dist: first owned kernel)
     int sms = 148;
     cudaStream_t stream = nullptr;
+    cudaStream_t side = nullptr;                 // ROOT: the small-cluster split runs beside the big path
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     uint32_t launches = 0;
     stem_stats stats{};
     Timing timing;

@@ -41,6 +41,16 @@ constexpr uint64_t kBigSeg = 65536;                    // rows per block on the 
 // (STEMROOT_LOCAL_ROWS, default 0 = off: measured slower than the level loop
 // on C5)
 __constant__ uint64_t c_loc;
+static bool split_overlap() {   // STEMROOT_SPLIT_OVERLAP=0: small and big split in sequence
+    static int v = -1;
+    if (v < 0) v = (getenv("STEMROOT_SPLIT_OVERLAP") && getenv("STEMROOT_SPLIT_OVERLAP")[0] == '0') ? 0 : 1;
+    return v == 1;
+}
+static bool seed_on() {   // STEMROOT_SPLIT_SEED=0 disables the coarse threshold seed
+    static int v = -1;
+    if (v < 0) v = (getenv("STEMROOT_SPLIT_SEED") && getenv("STEMROOT_SPLIT_SEED")[0] == '0') ? 0 : 1;
+    return v == 1;
+}
 static bool debug_levels() {
     static int v = -1;
     if (v < 0) v = getenv("STEMROOT_DEBUG_LEVELS") ? 1 : 0;
@@ -507,7 +517,9 @@ __device__ __forceinline__ Cand warp_range_best(const uint32_t *__restrict__ t, 
     Cand best = no_cand();
 #pragma unroll
     for (int r = 0; r < kMaxRounds; r++) {
-        // kept when d2 >= thr * pmin (d2 = RN(dub^2) (1 + 2^-43) covers the roundings)
+        // kept when d2 >= thr * pmin (d2 = RN(dub^2) (1 + 2^-43) covers the roundings).
+        // (Scanning the survivors four at a time with their rows loaded together
+        // spilled registers and measured slower.)
         uint32_t live = __ballot_sync(0xffffffffu, d2[r] > 0.0 && d2[r] >= __dmul_rn(thr, pm[r]));
         while (live) {
             const int src = __ffs(live) - 1;
@@ -555,7 +567,8 @@ __device__ __forceinline__ Cand warp_best_cut(const uint32_t *__restrict__ t, co
 
 // ---------------------------------------------------------------- mid clusters: a warp per cluster
 // Clusters of local_rows() .. big_rows() rows, one warp each (grid-stride).
-__global__ void __launch_bounds__(256, 4) small_split_kernel(const uint32_t *__restrict__ f_lo,
+template <int MINB>
+__global__ void __launch_bounds__(256, MINB) small_split_kernel(const uint32_t *__restrict__ f_lo,
                                                           const uint32_t *__restrict__ f_hi,
                                                           const uint64_t *__restrict__ f_S, uint32_t C,
                                                           const uint32_t *__restrict__ t,
@@ -588,6 +601,10 @@ struct BigEntry {
     uint32_t c, seg;
 };
 
+__device__ __forceinline__ uint32_t big_nseg(uint64_t lo, uint64_t hi) {
+    return (uint32_t)((hi - lo + kBigSeg - 1) / kBigSeg);
+}
+
 __global__ void big_entries_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, uint32_t C,
                                    BigEntry *__restrict__ ent, uint32_t *__restrict__ first_ent,
                                    uint32_t *__restrict__ count) {
@@ -595,7 +612,7 @@ __global__ void big_entries_kernel(const uint32_t *__restrict__ f_lo, const uint
     if (c >= C) return;
     const uint64_t n = f_hi[c] - f_lo[c];
     if (n < c_big) return;
-    const uint32_t nb = (uint32_t)((n + kBigSeg - 1) / kBigSeg);
+    const uint32_t nb = big_nseg(f_lo[c], f_hi[c]);
     const uint32_t e0 = atomicAdd(count, nb);
     for (uint32_t s = 0; s < nb; s++) ent[e0 + s] = BigEntry{(uint32_t)c, s};
     first_ent[c] = e0;
@@ -614,6 +631,51 @@ struct BigArgs {
 };
 
 constexpr int kBigThreads = 256;
+
+// Seed of each big cluster's pruning threshold: real candidates on a coarse
+// grid (every kSeedStride rows, at chunk starts, so S_L comes from PS1 and the
+// validity t[k-1] < t[k] from TB), one warp per entry.  Their best lower bound
+// (atomic max of the bits of a positive double) is a strict lower bound of a
+// real candidate's score, so pruning against it keeps the argmax and its ties;
+// it only makes far-away segments prune as hard as the segment holding the
+// optimum.
+constexpr uint64_t kSeedStride = 1024;
+__global__ void __launch_bounds__(256) big_seed_kernel(BigArgs a) {
+    const uint32_t n_ent = *a.count;
+    const int lane = threadIdx.x & 31;
+    const uint32_t nw = gridDim.x * (blockDim.x / 32);
+    for (uint32_t eb = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); eb < n_ent; eb += nw) {
+        const BigEntry e = a.ent[eb];
+        const uint64_t lo = a.f_lo[e.c], hi = a.f_hi[e.c], n = hi - lo, S = a.f_S[e.c];
+        const uint64_t r0 = lo + (uint64_t)e.seg * kBigSeg, r1 = min(r0 + kBigSeg, hi);
+        uint64_t part = 0;
+        const uint64_t lb0 = lo & ~(kChunk - 1);
+        if (lb0 + lane < lo) part = a.t[lb0 + lane];
+#pragma unroll
+        for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+        const uint64_t base = a.PS1[lo >> kChunkLog] + part;
+        const uint64_t g0 = (r0 + kChunk - 1) & ~(kChunk - 1);   // first chunk start in the segment
+        double lbm = 0.0;
+#pragma unroll
+        for (int r = 0; r < (int)(kBigSeg / kSeedStride / 32); r++) {
+            const uint64_t ra = g0 + ((uint64_t)r * 32 + lane) * kSeedStride;
+            if (ra > lo && ra < r1) {
+                const uint64_t SL = a.PS1[ra >> kChunkLog] - base;
+                const uint2 tb = reinterpret_cast<const uint2 *>(a.TB)[ra >> kChunkLog];
+                if (tb.x < tb.y) {   // t[ra - 1] < t[ra]: a valid cut
+                    const uint64_t ka = ra - lo;
+                    const u128 ad = (u128)S * ka - (u128)n * SL;
+                    const double dD = approx_d((uint32_t)(ad >> 64), (uint64_t)ad);
+                    lbm = fmax(lbm, div_lower(__dmul_rn(dD, dD), __dmul_rn((double)ka, (double)(n - ka))));
+                }
+            }
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));
+        if (lane == 0 && lbm > 0.0)
+            atomicMax(a.thr + e.c, (unsigned long long)__double_as_longlong(__dmul_rn(lbm, 1.0 - 0x1p-44)));
+    }
+}
 constexpr int kBigChunks = (int)(kBigSeg / kChunk) + 2;
 constexpr int kBigRounds = (kBigChunks + kBigThreads - 1) / kBigThreads;
 
@@ -628,27 +690,26 @@ __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
     __shared__ uint64_t s_base;
     const uint32_t n_ent = *a.count;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    // the entry descriptors are software-pipelined: the next entry's (cluster,
+    // lo, hi, S) loads are issued while the current entry is processed
+    BigEntry e{0, 0};
+    uint64_t lo = 0, hi = 0, S = 0;
+    if (blockIdx.x < n_ent) {
+        e = a.ent[blockIdx.x];
+        lo = a.f_lo[e.c];
+        hi = a.f_hi[e.c];
+        S = a.f_S[e.c];
+    }
     for (uint32_t eb = blockIdx.x; eb < n_ent; eb += gridDim.x) {
     __syncthreads();   // shared memory of the previous entry
-    const BigEntry e = a.ent[eb];
-    const uint64_t lo = a.f_lo[e.c], hi = a.f_hi[e.c], n = hi - lo, S = a.f_S[e.c];
+    const uint64_t n = hi - lo;
     const uint64_t r0 = lo + (uint64_t)e.seg * kBigSeg, r1 = min(r0 + kBigSeg, hi);
-    if (w == 0) {   // pref1(lo) = PS1[lo/32] + partial chunk
-        uint64_t part = 0;
-        const uint64_t lb0 = lo & ~(kChunk - 1);
-        if (lb0 + lane < lo) part = a.t[lb0 + lane];
-        for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
-        if (lane == 0) {
-            s_base = a.PS1[lo >> kChunkLog] + part;
-            s_nlist = 0;
-        }
-    }
-    __syncthreads();
     const uint64_t q0 = r0 >> kChunkLog, q1 = (r1 - 1) >> kChunkLog;   // chunks touching [r0, r1)
     const int nq = (int)(q1 - q0 + 1);
     const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
     double lbm = 0.0;
-    // every round's sampled-prefix and boundary loads in flight first
+    // every round's sampled-prefix and boundary loads in flight first, with
+    // pref1(lo), the cluster's published threshold and the next descriptors
     uint64_t pav[kBigRounds];
     uint2 tbv[kBigRounds];
 #pragma unroll
@@ -661,6 +722,27 @@ __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
             tbv[r] = reinterpret_cast<const uint2 *>(a.TB)[q0 + i];
         }
     }
+    if (w == 0) {   // pref1(lo) = PS1[lo/32] + partial chunk
+        uint64_t part = 0;
+        const uint64_t lb0 = lo & ~(kChunk - 1);
+        if (lb0 + lane < lo) part = a.t[lb0 + lane];
+        const uint64_t p1 = a.PS1[lo >> kChunkLog];
+        for (int o = 16; o; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+        if (lane == 0) {
+            s_base = p1 + part;
+            s_nlist = 0;
+        }
+    }
+    const uint32_t ebn = eb + gridDim.x;
+    BigEntry en{0, 0};
+    uint64_t lon = 0, hin = 0, Sn = 0;
+    if (ebn < n_ent) {
+        en = a.ent[ebn];
+        lon = a.f_lo[en.c];
+        hin = a.f_hi[en.c];
+        Sn = a.f_S[en.c];
+    }
+    __syncthreads();
 #pragma unroll
     for (int r = 0; r < kBigRounds; r++) {
         const int i = tid + r * kBigThreads;
@@ -712,11 +794,11 @@ __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
     for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));
     if (lane == 0) s_thr[w] = lbm;
     __syncthreads();
-    if (tid == 0) {
+    if (tid == 0) {   // block best vs the cluster's threshold (positive doubles order as integers)
         double m = 0.0;
         for (int k = 0; k < kBigThreads / 32; k++) m = fmax(m, s_thr[k]);
         const unsigned long long prev = atomicMax(a.thr + e.c, (unsigned long long)__double_as_longlong(m));
-        s_thr[0] = fmax(m, __longlong_as_double((long long)prev));   // positive doubles order as integers
+        s_thr[0] = fmax(m, __longlong_as_double((long long)prev));
     }
     __syncthreads();
     const double thr = __dmul_rn(s_thr[0], dn);
@@ -782,6 +864,10 @@ __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
             if (better(s_best[k], best)) best = s_best[k];
         a.part[eb] = best;
     }
+    e = en;
+    lo = lon;
+    hi = hin;
+    S = Sn;
     }
 }
 
@@ -792,7 +878,7 @@ __global__ void big_reduce_kernel(const uint32_t *__restrict__ f_lo, const uint3
   for (uint64_t c = blockIdx.x; c < C; c += gridDim.x) {
     const uint64_t n = f_hi[c] - f_lo[c];
     if (n < c_big) continue;
-    const uint32_t nb = (uint32_t)((n + kBigSeg - 1) / kBigSeg), e0 = first_ent[c];
+    const uint32_t nb = big_nseg(f_lo[c], f_hi[c]), e0 = first_ent[c];
     Cand best = no_cand();
     for (uint32_t s = threadIdx.x; s < nb; s += 32)
         if (better(part[e0 + s], best)) best = part[e0 + s];
@@ -1137,10 +1223,30 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         c.stage_end(tk_l, 4 * A);
         CK(cudaGetLastError());
         const int tk_s = c.stage_begin("root_split");
+        // the small-cluster warps run on a side stream beside the big-cluster
+        // chain (both latency-bound; they read the same frontier and write
+        // disjoint cuts), joined before the decision
+        if (!c.side) {
+            CK(cudaStreamCreateWithFlags(&c.side, cudaStreamNonBlocking));
+            CK(cudaEventCreateWithFlags(&c.ev_fork, cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming));
+        }
+        const bool overlap = split_overlap();
+        cudaStream_t sst = overlap ? c.side : st;
+        if (overlap) {
+            CK(cudaEventRecord(c.ev_fork, st));
+            CK(cudaStreamWaitEvent(c.side, c.ev_fork, 0));
+        }
         if (local_rows() < big_rows()) {
             const uint64_t blocks = (C + 7) / 8;
-            small_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, st>>>(
-                c.f_lo[cur], c.f_hi[cur], c.f_S[cur], (uint32_t)C, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
+            static int minb = -1;   // STEMROOT_SMALL_MINB: resident blocks per SM the registers are sized for
+            if (minb < 0) minb = getenv("STEMROOT_SMALL_MINB") ? atoi(getenv("STEMROOT_SMALL_MINB")) : 4;
+            if (minb == 3)
+                small_split_kernel<3><<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, sst>>>(
+                    c.f_lo[cur], c.f_hi[cur], c.f_S[cur], (uint32_t)C, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
+            else
+                small_split_kernel<4><<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, sst>>>(
+                    c.f_lo[cur], c.f_hi[cur], c.f_S[cur], (uint32_t)C, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
             c.launches++;
         }
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
@@ -1157,11 +1263,19 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         BigArgs ba{ent, &c.scalars->big_count, c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.PS1, c.t_sorted, c.TB,
                    (unsigned long long *)c.big_thr, (Cand *)c.big_part, &c.scalars->split_chunks,
                    &c.scalars->split_scanned};
+        if (seed_on()) {
+            big_seed_kernel<<<(unsigned)min((max_ent + 7) / 8, (uint64_t)c.sms * 8), 256, 0, st>>>(ba);
+            c.launches++;
+        }
         big_split_kernel<<<(unsigned)min(max_ent, (uint64_t)c.sms * 8), kBigThreads, 0, st>>>(ba);
         c.launches += 2;
         big_reduce_kernel<<<(unsigned)min(C, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, first_ent,
                                                       (const Cand *)c.big_part, c.cut, c.cut_SL);
         c.launches += 2;
+        if (overlap) {
+            CK(cudaEventRecord(c.ev_join, c.side));
+            CK(cudaStreamWaitEvent(st, c.ev_join, 0));
+        }
         c.stage_end(tk_s, 4 * A + 20 * C);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");

@@ -39,7 +39,6 @@ constexpr int kMaxPasses = 8;
 constexpr int kRB = 8, kR = 1 << kRB;       // byte digits
 constexpr int kHistR = 256;                 // histogram row stride
 constexpr int kBaseShift = 16;              // B[k] is a multiple of 2^16
-constexpr int kMaxExtra = kMaxPasses - 2;   // digits histogrammed by the first pass
 constexpr uint64_t kMaxTable = 1ull << 27;  // kid-table entries (512 MB) before binary search
 constexpr int kLB = 4;                      // look-back: predecessor statuses read per round trip
 constexpr int kCoarseShift = 24;            // coarse bases: B[k] a multiple of 2^24
@@ -282,7 +281,8 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
     __shared__ uint32_t s_cnt[R];
     __shared__ uint32_t s_cw[NW];
     __shared__ uint32_t s_tile;
-    __shared__ uint32_t s_xh[FIRST ? kMaxExtra * R : 1];
+    // FIRST: the extra digit histograms (a.nxh x R; dynamic, none with coarse bases)
+    uint32_t *s_xh = reinterpret_cast<uint32_t *>(&s_whist[0][0] + NW * R);
 
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     if (tid == 0) s_tile = atomicAdd(a.tile_counter, 1u);
@@ -497,21 +497,27 @@ template <int NT, int IT, bool FIRST, bool LAST, bool PK>
 static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
     constexpr uint64_t TILE = (uint64_t)NT * IT;
     const uint64_t full = a.n / TILE, rag = a.n % TILE;
-    const size_t smem = (size_t)TILE * (sizeof(uint64_t) + (PK ? 0 : sizeof(uint32_t))) + sizeof(uint16_t) * (NT / 32) * kR;
-    static bool attr = false;
-    if (!attr) {
-        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true, PK>,
-                                cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const size_t smem = (size_t)TILE * (sizeof(uint64_t) + (PK ? 0 : sizeof(uint32_t))) + sizeof(uint16_t) * (NT / 32) * kR +
+                        (FIRST ? sizeof(uint32_t) * kR * (size_t)a.nxh : 0);
+    // attributes once per instantiation (thread-safe static init: ranks of a
+    // loopback group launch from several host threads), sized for the largest
+    // dynamic shared memory any call can ask for (FIRST: kMaxPasses - 2 extra histograms)
+    static const int attr_status = [] {
+        const size_t smax = (size_t)TILE * (sizeof(uint64_t) + (PK ? 0 : sizeof(uint32_t))) +
+                            sizeof(uint16_t) * (NT / 32) * kR + (FIRST ? sizeof(uint32_t) * kR * (kMaxPasses - 2) : 0);
+        const size_t sbase = smax - (FIRST ? sizeof(uint32_t) * kR * (kMaxPasses - 2) : 0);
         // FIRST gathers B[kid]: keep L1 beside first_blocks() blocks' shared memory
-        const int carve = FIRST ? (int)((first_blocks() * (smem + 12 * 1024) * 100 + 228 * 1024 - 1) / (228 * 1024)) : 100;
-        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, true, PK>,
-                                cudaFuncAttributePreferredSharedMemoryCarveout, carve > 100 ? 100 : carve));
-        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false, PK>,
-                                cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        CK(cudaFuncSetAttribute(onesweep_kernel<NT, IT, FIRST, LAST, false, PK>,
-                                cudaFuncAttributePreferredSharedMemoryCarveout, carve > 100 ? 100 : carve));
-        attr = true;
-    }
+        const int carve = FIRST ? (int)((first_blocks() * (sbase + 12 * 1024) * 100 + 228 * 1024 - 1) / (228 * 1024)) : 100;
+        for (int f = 0; f < 2; f++) {
+            auto fn = f ? onesweep_kernel<NT, IT, FIRST, LAST, true, PK> : onesweep_kernel<NT, IT, FIRST, LAST, false, PK>;
+            if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smax) != cudaSuccess ||
+                cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, carve > 100 ? 100 : carve) !=
+                    cudaSuccess)
+                return 1;
+        }
+        return 0;
+    }();
+    if (attr_status) return STEM_E_CUDA;
     if (full) {
         onesweep_kernel<NT, IT, FIRST, LAST, true, PK><<<(unsigned)full, NT, smem, st>>>(a);
         (*launches)++;
@@ -537,30 +543,14 @@ static int launch_pass_cfg(const PassArgs &a, bool first, bool last, cudaStream_
                 : launch_pass_pk<NT, IT, false>(a, first, last, st, launches);
 }
 
-// tile shapes (threads, keys per thread); STEMROOT_SORT_SHAPE picks one for
-// experiments.  256 x 20 (4 blocks/SM) measured fastest on B200 for packed keys
-// (C5 mid pass 5.07 ms vs 5.36 for 384 x 12, 5.09-5.29 for 256 x 16/24).
-struct Shape { int nt, it; };
-static const Shape kShapes[] = {{256, 20}, {384, 12}, {256, 24}, {256, 16}};
-static int shape_idx() {
-    static int s = -1;
-    if (s < 0) {
-        const char *e = getenv("STEMROOT_SORT_SHAPE");
-        s = e ? atoi(e) : 0;
-        if (s < 0 || s > 3) s = 0;
-    }
-    return s;
-}
-
-static uint64_t tile_keys() { return (uint64_t)kShapes[shape_idx()].nt * kShapes[shape_idx()].it; }
+// tile shape (threads, keys per thread): 256 x 20 (4 blocks/SM) measured
+// fastest on B200 for packed keys (C5 mid pass 5.07 ms vs 5.36 for 384 x 12,
+// 5.09-5.29 for 256 x 16/24; the other shapes were dropped after the sweep)
+constexpr int kSortNT = 256, kSortIT = 20;
+static uint64_t tile_keys() { return (uint64_t)kSortNT * kSortIT; }
 
 static int launch_sort_pass(const PassArgs &a, bool first, bool last, cudaStream_t st, uint32_t *launches) {
-    switch (shape_idx()) {
-        case 1: return launch_pass_cfg<384, 12>(a, first, last, st, launches);
-        case 2: return launch_pass_cfg<256, 24>(a, first, last, st, launches);
-        case 3: return launch_pass_cfg<256, 16>(a, first, last, st, launches);
-        default: return launch_pass_cfg<256, 20>(a, first, last, st, launches);
-    }
+    return launch_pass_cfg<kSortNT, kSortIT>(a, first, last, st, launches);
 }
 
 // the pre-pass alone (kernel-id counts and max t, range check): also the
@@ -573,8 +563,10 @@ int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n
     CK(cudaMemsetAsync(c.kid_max, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
     const int smem_kid = (K <= 24000) ? 1 : 0;
     const size_t sm_bytes = sizeof(uint32_t) * (3 * kR + (smem_kid ? 2 * (size_t)K : 0));
-    if (sm_bytes > 48 * 1024)
-        CK(cudaFuncSetAttribute(prepass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_bytes));
+    // once, for the largest request (thread-safe: loopback ranks are host threads)
+    static const cudaError_t pre_attr = cudaFuncSetAttribute(
+        prepass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(uint32_t) * (3 * kR + 2 * 24000)));
+    CK(pre_attr);
     int per_sm = (int)((200 * 1024) / (sm_bytes + 1024));
     per_sm = per_sm < 1 ? 1 : per_sm > 2 ? 2 : per_sm;
     prepass_kernel<<<c.sms * per_sm, kPreThreads, sm_bytes, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.kid_max, c.hist,

@@ -320,3 +320,20 @@ def test_key_bases_heavy_tails(ctx, sr, monkeypatch, coarse, K):
     got, ref = _both(ctx, kid, t, K, eps=0.05, seed=3)
     assert_plans_equal(got, ref)
     assert ctx.stats()["coarse_bases"] == (1 if coarse == "1" else 0)
+
+
+def test_big_path_multi_segment(ctx):
+    """The big-cluster path on clusters spanning many 65536-row blocks, starting at
+    unaligned rows, with ties and constant runs, against the oracle."""
+    rng = np.random.default_rng(11)
+    parts = [
+        (0, rng.integers(0, 5, 1_234) + 100),                                    # unaligns the next group
+        (1, rng.lognormal(11, 1.0, 2_500_000)),                                  # heavy tail
+        (2, np.r_[np.full(400_000, 5000), np.full(700_001, 9000), rng.integers(20_000, 20_003, 300_000)]),
+        (3, rng.normal(50_000, 2_000, 1_100_000).clip(1)),                       # unimodal, wide plateau
+    ]
+    kid = np.concatenate([np.full(len(p), k, np.uint32) for k, p in parts])
+    t = np.concatenate([np.asarray(p) for _, p in parts]).astype(np.uint32)
+    perm = rng.permutation(len(t))
+    got, ref = _both(ctx, kid[perm], t[perm], 4, eps=0.01, seed=8)
+    assert_plans_equal(got, ref)
