@@ -678,12 +678,16 @@ __global__ void __launch_bounds__(256) big_seed_kernel(BigArgs a) {
 }
 constexpr int kBigChunks = (int)(kBigSeg / kChunk) + 2;
 constexpr int kBigRounds = (kBigChunks + kBigThreads - 1) / kBigThreads;
+constexpr size_t kBigSmem = (size_t)kBigChunks * (sizeof(double) + sizeof(uint64_t) + sizeof(uint2) + sizeof(float) +
+                                                  sizeof(uint16_t));
 
 __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
-    __shared__ double s_ub[kBigChunks];   // d2: the squared |D| bound of the chunk
-    __shared__ float s_pm[kBigChunks];    // min of k (n - k) over the chunk's cuts, rounded down (prunes less)
-    __shared__ uint64_t s_sl[kBigChunks];
-    __shared__ uint16_t s_list[kBigChunks];
+    extern __shared__ __align__(16) unsigned char s_big[];   // kBigSmem bytes
+    double *s_ub = reinterpret_cast<double *>(s_big);          // d2: the squared |D| bound of the chunk
+    uint64_t *s_sl = reinterpret_cast<uint64_t *>(s_ub + kBigChunks);   // PS1 at the chunk start, then S_L
+    uint2 *s_tb = reinterpret_cast<uint2 *>(s_sl + kBigChunks);         // TB pair at the chunk start
+    float *s_pm = reinterpret_cast<float *>(s_tb + kBigChunks);         // min k (n - k), rounded down (prunes less)
+    uint16_t *s_list = reinterpret_cast<uint16_t *>(s_pm + kBigChunks);
     __shared__ uint32_t s_nlist;
     __shared__ double s_thr[kBigThreads / 32];
     __shared__ Cand s_best[kBigThreads / 32];
@@ -708,18 +712,16 @@ __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
     const int nq = (int)(q1 - q0 + 1);
     const double up = 1.0 + 0x1p-44, dn = 1.0 - 0x1p-44;
     double lbm = 0.0;
-    // every round's sampled-prefix and boundary loads in flight first, with
-    // pref1(lo), the cluster's published threshold and the next descriptors
-    uint64_t pav[kBigRounds];
-    uint2 tbv[kBigRounds];
+    // every round's sampled-prefix and boundary loads in flight first (staged
+    // in shared memory, so the bound loop below stays rolled: a small kernel
+    // body, the unrolled one missed the instruction cache), with pref1(lo) and
+    // the next entry's descriptors
 #pragma unroll
     for (int r = 0; r < kBigRounds; r++) {
         const int i = tid + r * kBigThreads;
-        pav[r] = 0;
-        tbv[r] = make_uint2(0u, 0u);
         if (i < nq) {
-            pav[r] = a.PS1[q0 + i];
-            tbv[r] = reinterpret_cast<const uint2 *>(a.TB)[q0 + i];
+            s_sl[i] = a.PS1[q0 + i];
+            s_tb[i] = reinterpret_cast<const uint2 *>(a.TB)[q0 + i];
         }
     }
     if (w == 0) {   // pref1(lo) = PS1[lo/32] + partial chunk
@@ -743,19 +745,17 @@ __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
         Sn = a.f_S[en.c];
     }
     __syncthreads();
-#pragma unroll
-    for (int r = 0; r < kBigRounds; r++) {
-        const int i = tid + r * kBigThreads;
-        if (i >= nq) break;
+#pragma unroll 1
+    for (int i = tid; i < nq; i += kBigThreads) {
         const uint64_t q = q0 + i;
         const uint64_t ra = max(r0, q << kChunkLog), rb = min(r1, (q + 1) << kChunkLog);   // rows [ra, rb)
-        uint64_t pa = pav[r];
+        uint64_t pa = s_sl[i];
         const bool al = (ra & (kChunk - 1)) == 0;
         if (!al)   // only the block's first chunk can start unaligned
             for (uint64_t x = ra & ~(kChunk - 1); x < ra; x++) pa += a.t[x];
         const uint64_t SL = pa - s_base;       // S_L at k_a = ra - lo (exact)
         const uint32_t ka = (uint32_t)(ra - lo);
-        const uint2 tb = al ? tbv[r] : make_uint2(0u, 0u);
+        const uint2 tb = al ? s_tb[i] : make_uint2(0u, 0u);
         const uint32_t ta = al ? tb.y : a.t[ra];
         s_sl[i] = SL;
         const u128 ad = (u128)S * ka - (u128)n * SL;
@@ -1267,7 +1267,10 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             big_seed_kernel<<<(unsigned)min((max_ent + 7) / 8, (uint64_t)c.sms * 8), 256, 0, st>>>(ba);
             c.launches++;
         }
-        big_split_kernel<<<(unsigned)min(max_ent, (uint64_t)c.sms * 8), kBigThreads, 0, st>>>(ba);
+        static const cudaError_t big_attr =
+            cudaFuncSetAttribute(big_split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBigSmem);
+        CK(big_attr);
+        big_split_kernel<<<(unsigned)min(max_ent, (uint64_t)c.sms * 8), kBigThreads, kBigSmem, st>>>(ba);
         c.launches += 2;
         big_reduce_kernel<<<(unsigned)min(C, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, first_ent,
                                                       (const Cand *)c.big_part, c.cut, c.cut_SL);

@@ -319,6 +319,20 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
 
     uint64_t key[IT];
     uint32_t val[PK ? 1 : IT];
+    if (FIRST && PK && a.Bs16 && a.noalloc) {
+        // the common first pass (packed keys, 16-bit key-base table) as straight-line code
+        const uint32_t lm = (uint32_t)a.lomask;
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = wbase + (uint64_t)j * 32 + lane;
+            key[j] = ~0ull;
+            if (FULL || i < a.n) {
+                const uint32_t kd = ld_na(a.kid_in + i), tv = ld_na(a.t_in + i);
+                const uint64_t kk = ((uint64_t)__ldg(a.Bs16 + kd) << a.tsh) + tv;
+                key[j] = (kk << a.ks) | ((uint32_t)i & lm);
+            }
+        }
+    } else
 #pragma unroll
     for (int j = 0; j < IT; j++) {
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;

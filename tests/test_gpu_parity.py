@@ -337,3 +337,14 @@ def test_big_path_multi_segment(ctx):
     perm = rng.permutation(len(t))
     got, ref = _both(ctx, kid[perm], t[perm], 4, eps=0.01, seed=8)
     assert_plans_equal(got, ref)
+
+
+@pytest.mark.parametrize("n", [1, 31, 32, 33, 16352, 16353, 16384, 16385, 65536 * 2 + 7])
+def test_tile_boundaries(ctx, n):
+    """sizes at the 32-row chunk, the 16 384-row prefix-moment tile (the scan
+    element past the last chunk opening a tile of its own), the 65 536-row
+    leaf-bitmap tile and the 5120-row sort tile boundaries"""
+    rng = np.random.default_rng(n)
+    kid, t = _mixture(rng, n, 3 if n > 3 else 1, peaks=2, spread=0.2)
+    got, ref = _both(ctx, kid, t, 3 if n > 3 else 1, eps=0.02, seed=n)
+    assert_plans_equal(got, ref)
