@@ -365,7 +365,7 @@ __device__ __forceinline__ Cand warp_scan_cut(const uint32_t *__restrict__ t, ui
             tlast = __shfl_sync(0xffffffffu, tc, 31);
         }
     }
-#pragma unroll
+#pragma unroll 1   // one copy of better() (with its 256-bit tie path) in the kernel body
     for (int o = 16; o; o >>= 1) {
         const Cand v = shfl_cand_xor(best, o);
         if (better(v, best)) best = v;
@@ -515,19 +515,25 @@ __device__ __forceinline__ Cand warp_range_best(const uint32_t *__restrict__ t, 
         thr = fmax(thr, __longlong_as_double((long long)prev));   // positive doubles order as integers
     }
     Cand best = no_cand();
-#pragma unroll
+    // kept when d2 >= thr * pmin (d2 = RN(dub^2) (1 + 2^-43) covers the roundings).
+    // The round loop is rolled (per-round values picked by selects, not dynamic
+    // register indexing) so the row scan appears once in the kernel body.
+    // (Scanning the survivors four at a time with their rows loaded together
+    // spilled registers and measured slower.)
+#pragma unroll 1
     for (int r = 0; r < kMaxRounds; r++) {
-        // kept when d2 >= thr * pmin (d2 = RN(dub^2) (1 + 2^-43) covers the roundings).
-        // (Scanning the survivors four at a time with their rows loaded together
-        // spilled registers and measured slower.)
-        uint32_t live = __ballot_sync(0xffffffffu, d2[r] > 0.0 && d2[r] >= __dmul_rn(thr, pm[r]));
+        static_assert(kMaxRounds == 3, "the selects below cover three rounds");
+        const double rd2 = r == 0 ? d2[0] : r == 1 ? d2[1] : d2[2];
+        const double rpm = r == 0 ? pm[0] : r == 1 ? pm[1] : pm[2];
+        const uint64_t rsl = r == 0 ? sla[0] : r == 1 ? sla[1] : sla[2];
+        uint32_t live = __ballot_sync(0xffffffffu, rd2 > 0.0 && rd2 >= __dmul_rn(thr, rpm));
         while (live) {
             const int src = __ffs(live) - 1;
             live &= live - 1;
-            const double sd2 = __shfl_sync(0xffffffffu, d2[r], src), spm = __shfl_sync(0xffffffffu, pm[r], src);
+            const double sd2 = __shfl_sync(0xffffffffu, rd2, src), spm = __shfl_sync(0xffffffffu, rpm, src);
             if (sd2 < __dmul_rn(thr, spm)) continue;   // threshold raised meanwhile
             const uint64_t q = q0 + (uint64_t)r * 32 + src;
-            const uint64_t SLa = __shfl_sync(0xffffffffu, sla[r], src);
+            const uint64_t SLa = __shfl_sync(0xffffffffu, rsl, src);
             scan_chunk(t, lo, n, S, max(r0, q << kChunkLog), min(r1, (q + 1) << kChunkLog), SLa, best);
             double lb = best.k ? div_lower(best.x, best.dp) : 0.0;
 #pragma unroll
@@ -535,7 +541,7 @@ __device__ __forceinline__ Cand warp_range_best(const uint32_t *__restrict__ t, 
             thr = fmax(thr, __dmul_rn(lb, dn));
         }
     }
-#pragma unroll
+#pragma unroll 1   // one copy of better() (with its 256-bit tie path) in the kernel body
     for (int o = 16; o; o >>= 1) {
         const Cand v = shfl_cand_xor(best, o);
         if (better(v, best)) best = v;
@@ -852,7 +858,7 @@ __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
             if (in && k >= 1 && tp < tc) eval_cut(k, n, S, SLr, best);
         }
     }
-#pragma unroll
+#pragma unroll 1   // one copy of better() (with its 256-bit tie path) in the kernel body
     for (int o = 16; o; o >>= 1) {
         const Cand v = shfl_cand_xor(best, o);
         if (better(v, best)) best = v;
@@ -882,7 +888,7 @@ __global__ void big_reduce_kernel(const uint32_t *__restrict__ f_lo, const uint3
     Cand best = no_cand();
     for (uint32_t s = threadIdx.x; s < nb; s += 32)
         if (better(part[e0 + s], best)) best = part[e0 + s];
-#pragma unroll
+#pragma unroll 1   // one copy of better() (with its 256-bit tie path) in the kernel body
     for (int o = 16; o; o >>= 1) {
         const Cand v = shfl_cand_xor(best, o);
         if (better(v, best)) best = v;
