@@ -135,9 +135,24 @@ __device__ __forceinline__ bool better(const Cand &a, const Cand &b) {
 constexpr int kChunkLog = 5;
 constexpr uint64_t kChunk = 1ull << kChunkLog;
 
+// The partial chunk [32 (x / 32), x) lies in one 128-byte line: read with up to
+// eight independent uint4 loads (all in flight) when t is 16-byte aligned.
 __device__ __forceinline__ uint64_t pref1(const uint64_t *PS1, const uint32_t *t, uint64_t x) {
     uint64_t s = PS1[x >> kChunkLog];
-    for (uint64_t i = x & ~(kChunk - 1); i < x; i++) s += t[i];
+    const uint32_t r = (uint32_t)(x & (kChunk - 1));
+    const uint64_t b = x - r;
+    if (r && (reinterpret_cast<uintptr_t>(t) & 15) == 0) {
+        const uint4 *c = reinterpret_cast<const uint4 *>(t + b);
+#pragma unroll
+        for (uint32_t k = 0; k < kChunk / 4; k++)
+            if (4 * k < r) {
+                const uint4 v = c[k];
+                s += v.x + (4 * k + 1 < r ? (uint64_t)v.y : 0) + (4 * k + 2 < r ? (uint64_t)v.z : 0) +
+                     (4 * k + 3 < r ? (uint64_t)v.w : 0);
+            }
+        return s;
+    }
+    for (uint64_t i = b; i < x; i++) s += t[i];
     return s;
 }
 
@@ -145,7 +160,22 @@ __device__ __forceinline__ void pref12(const uint64_t *PS1, const u128 *PS2, con
                                        uint64_t &s, u128 &q) {
     s = PS1[x >> kChunkLog];
     q = PS2[x >> kChunkLog];
-    for (uint64_t i = x & ~(kChunk - 1); i < x; i++) {
+    const uint32_t r = (uint32_t)(x & (kChunk - 1));
+    const uint64_t b = x - r;
+    if (r && (reinterpret_cast<uintptr_t>(t) & 15) == 0) {
+        const uint4 *c = reinterpret_cast<const uint4 *>(t + b);
+#pragma unroll
+        for (uint32_t k = 0; k < kChunk / 4; k++)
+            if (4 * k < r) {
+                const uint4 v = c[k];
+                const uint64_t e0 = v.x, e1 = 4 * k + 1 < r ? v.y : 0u, e2 = 4 * k + 2 < r ? v.z : 0u,
+                               e3 = 4 * k + 3 < r ? v.w : 0u;
+                s += e0 + e1 + e2 + e3;
+                q += (u128)(e0 * e0) + (e1 * e1) + (u128)(e2 * e2) + (e3 * e3);
+            }
+        return;
+    }
+    for (uint64_t i = b; i < x; i++) {
         const uint64_t v = t[i];
         s += v;
         q += (u128)(v * v);

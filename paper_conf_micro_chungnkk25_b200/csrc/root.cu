@@ -1217,7 +1217,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(C) + 1) * sizeof(uint64_t)));
         const int nxt = cur ^ 1;
         CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
-        const int tk_l = c.stage_begin("root_local");
+        const int tk_l = local_rows() > 0 ? c.stage_begin("root_local") : -1;
         if (local_rows() > 0) {
             LocalArgs la{c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], (uint32_t)C, levels - 1, c.PS1, c.PS2,
                          c.t_sorted, c.TB, c.flags, eps, z, k2, clamp, &c.scalars->local_rows, &c.scalars->local_depth,
@@ -1226,7 +1226,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             local_root_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 64), 256, 0, st>>>(la);
             c.launches++;
         }
-        c.stage_end(tk_l, 4 * A);
+        if (tk_l >= 0) c.stage_end(tk_l, 4 * A);
         CK(cudaGetLastError());
         const int tk_s = c.stage_begin("root_split");
         // the small-cluster warps run on a side stream beside the big-cluster
