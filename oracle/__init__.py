@@ -34,7 +34,7 @@ def build(force: bool = False) -> str:
 
 class _Opts(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("z", C.c_double), ("scope", C.c_int), ("root", C.c_int),
-                ("clamp_in_split", C.c_int), ("census_cap", C.c_int)]
+                ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("split", C.c_int)]
 
 
 class _Plan(C.Structure):
@@ -70,6 +70,8 @@ def lib():
         _lib.or_philox4x32_10.argtypes = [u32p, u32p, u32p]
         _lib.or_best_cut.argtypes = [u32p, C.c_uint64]
         _lib.or_best_cut.restype = C.c_uint64
+        _lib.or_lloyd_cut.argtypes = [u32p, C.c_uint64, C.POINTER(C.c_uint32)]
+        _lib.or_lloyd_cut.restype = C.c_uint64
         _lib.or_eq3_m.argtypes = [C.c_uint64, C.c_uint64, C.c_uint64, C.c_uint64, C.c_double, C.c_double, C.c_int]
         _lib.or_eq3_m.restype = C.c_double
         _lib.or_eq6_m.argtypes = [C.c_uint32, dp, dp, C.c_double, C.c_double, C.c_double, dp]
@@ -99,7 +101,7 @@ class OracleError(RuntimeError):
 
 
 def plan(kernel_id, exec_ns, n_kernels, eps=0.05, z=1.959963984540054, seed=0, scope=0, root=1,
-         clamp_in_split=1, census_cap=0, metrics=None) -> dict:
+         clamp_in_split=1, census_cap=0, metrics=None, split=0) -> dict:
     """Full sampling plan (§3).  Returns numpy arrays + scalars."""
     kid = _u32(kernel_id)
     t = _u32(exec_ns)
@@ -110,7 +112,7 @@ def plan(kernel_id, exec_ns, n_kernels, eps=0.05, z=1.959963984540054, seed=0, s
         metp = _ptr(met, C.c_double)
     else:
         nm, metp = 0, None
-    o = _Opts(seed, z, scope, root, clamp_in_split, census_cap)
+    o = _Opts(seed, z, scope, root, clamp_in_split, census_cap, split)
     out = C.POINTER(_Plan)()
     st = lib().or_plan_build(n, n_kernels, _ptr(kid, C.c_uint32), _ptr(t, C.c_uint32), nm, metp, eps,
                              C.byref(o), C.byref(out))
@@ -143,6 +145,14 @@ def philox4x32_10(ctr, key):
     o = np.zeros(4, np.uint32)
     lib().or_philox4x32_10(_ptr(c, C.c_uint32), _ptr(k, C.c_uint32), _ptr(o, C.c_uint32))
     return [int(x) for x in o]
+
+
+def lloyd_cut(t_sorted):
+    """Lloyd's k-means (k = 2) cut of sorted times and its assignment steps (reading R26)."""
+    t = _u32(t_sorted)
+    it = C.c_uint32(0)
+    k = int(lib().or_lloyd_cut(_ptr(t, C.c_uint32), t.shape[0], C.byref(it)))
+    return k, int(it.value)
 
 
 def best_cut(t_sorted) -> int:

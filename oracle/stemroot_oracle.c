@@ -236,6 +236,51 @@ static uint64_t best_cut(const uint32_t *t, uint64_t lo, uint64_t hi, uint64_t S
     return best_k;
 }
 
+/* Lloyd's algorithm for k = 2 (reading R26), written as the
+ * textbook iteration on the cluster's values:
+ *   1. centroids c1 = min t, c2 = max t;
+ *   2. assignment: a value goes to cluster 1 iff it is not farther from c1 than
+ *      from c2, i.e. 2 t <= c1 + c2 (a tie at the midpoint goes to cluster 1);
+ *   3. update: c1, c2 = the means of the two clusters;
+ *   4. repeat 2-3 until the assignment no longer changes (at most
+ *      OR_LLOYD_MAX_ITERS assignment steps).
+ * Centroids are kept as exact fractions S_1/k and S_2/(n-k), so step 2 is the
+ * integer test 2 t k (n-k) <= S_1 (n-k) + S_2 k.  Sorted values make every
+ * assignment a cut: cluster 1 = t[lo .. lo+k).  Returns k (0: no cut, the
+ * cluster is constant or has < 2 rows). */
+#define OR_LLOYD_MAX_ITERS 1000
+static uint64_t lloyd_cut(const uint32_t *t, uint64_t lo, uint64_t hi, uint32_t *iters) {
+    uint64_t n = hi - lo;
+    if (iters) *iters = 0;
+    if (n < 2 || t[lo] == t[hi - 1]) return 0;
+    /* step 1 and the first assignment: 2 t <= min + max */
+    uint64_t mid2 = (uint64_t)t[lo] + t[hi - 1];
+    uint64_t k = 0;
+    for (uint64_t i = lo; i < hi; i++)
+        if (2 * (uint64_t)t[i] <= mid2) k++;
+    uint32_t it = 1;
+    for (; it < OR_LLOYD_MAX_ITERS; it++) {
+        /* step 3: exact centroid sums of the current assignment */
+        uint64_t S1 = 0, S2 = 0;
+        for (uint64_t i = lo; i < lo + k; i++) S1 += t[i];
+        for (uint64_t i = lo + k; i < hi; i++) S2 += t[i];
+        /* step 2 with the new centroids */
+        const u128 rhs = (u128)S1 * (n - k) + (u128)S2 * k;
+        const u128 f = (u128)2 * k * (n - k);
+        uint64_t k2 = 0;
+        for (uint64_t i = lo; i < hi; i++)
+            if ((u128)t[i] * f <= rhs) k2++;
+        if (k2 == k) break;
+        k = k2;
+    }
+    if (iters) *iters = it;
+    return k;
+}
+
+uint64_t or_lloyd_cut(const uint32_t *t_sorted, uint64_t n, uint32_t *iters) {
+    return lloyd_cut(t_sorted, 0, n, iters);
+}
+
 uint64_t or_best_cut(const uint32_t *t_sorted, uint64_t n) {
     if (n < 2) return 0;
     moments m = range_moments(t_sorted, 0, n);
@@ -288,12 +333,12 @@ void or_eq6_m(uint32_t k, const double *mu, const double *V, double T, double ep
 typedef struct { double tau_old, tau_new; uint64_t cut; int split; } decision;
 
 static decision root_decide(const uint32_t *t, uint64_t lo, uint64_t hi, double eps, double z,
-                            double k2, int clamp) {
+                            double k2, int clamp, int split) {
     decision d = {0.0, 0.0, 0, 0};
     uint64_t n = hi - lo;
     if (n < 2 || t[lo] == t[hi - 1]) return d;              /* R5: leaf */
     moments all = range_moments(t, lo, hi);
-    uint64_t k = best_cut(t, lo, hi, all.S);
+    uint64_t k = split == 1 ? lloyd_cut(t, lo, hi, NULL) : best_cut(t, lo, hi, all.S);
     d.cut = k;
     /* Eq. 7: tau_old = m * Xbar with m from Eq. 3 */
     double mu = rn64(all.S) / rn64(all.n);
@@ -317,7 +362,7 @@ static decision root_decide(const uint32_t *t, uint64_t lo, uint64_t hi, double 
 int or_root_decide(const uint32_t *t_sorted, uint64_t n, double eps, double z, int clamp,
                    double *tau_old, double *tau_new, uint64_t *cut) {
     double q = z / eps;
-    decision d = root_decide(t_sorted, 0, n, eps, z, q * q, clamp);
+    decision d = root_decide(t_sorted, 0, n, eps, z, q * q, clamp, 0);
     if (tau_old) *tau_old = d.tau_old;
     if (tau_new) *tau_new = d.tau_new;
     if (cut) *cut = d.cut;
@@ -384,6 +429,7 @@ int or_plan_build(uint64_t n, uint32_t n_kernels, const uint32_t *kernel_id,
     if (!(eps > 0.0 && eps < 1.0) || !(opts->z > 0.0) || !isfinite(opts->z)) return OR_E_INVAL;
     if (n_metrics > 64 || (n_metrics > 0 && !metrics)) return OR_E_INVAL;
     if (opts->scope < 0 || opts->scope > 2) return OR_E_INVAL;
+    if (opts->split < 0 || opts->split > 1) return OR_E_INVAL;
     if (n >= ((uint64_t)1 << 32)) return OR_E_RANGE;
     for (uint64_t i = 0; i < n; i++) if (kernel_id[i] >= n_kernels) return OR_E_RANGE;
 
@@ -421,7 +467,7 @@ int or_plan_build(uint64_t n, uint32_t n_kernels, const uint32_t *kernel_id,
             work_item w = work.v[--work.n];
             if (w.depth > max_depth) max_depth = w.depth;
             decision d = {0.0, 0.0, 0, 0};
-            if (opts->root) d = root_decide(t, w.lo, w.hi, eps, z, k2, clamp);
+            if (opts->root) d = root_decide(t, w.lo, w.hi, eps, z, k2, clamp, opts->split);
             if (d.split) {
                 /* push right then left: the left child is visited first */
                 if (work_push(&work, w.lo + d.cut, w.hi, w.depth + 1) ||

@@ -27,6 +27,8 @@ typedef struct {
     int      root;           /* 1 ROOT on, 0 STEM only                             */
     int      clamp_in_split; /* 1: m >= 1 inside Eq.7/8; 0: literal ceilings       */
     int      census_cap;     /* 1: m_i >= n_i => take all n_i rows                 */
+    int      split;          /* 0: exact optimal 2-means cut (R5); 1: Lloyd's k-means,
+                                k = 2, from the (min, max) centroids (R26)          */
 } or_opts;
 
 /* Structure-of-arrays plan.  Everything is malloc'ed; free with or_plan_free. */
@@ -61,6 +63,10 @@ void or_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out
 /* Optimal 2-means cut of sorted t[0..n): returns k* in [1,n-1]
  * or 0 when no cut exists (n < 2 or all equal). */
 uint64_t or_best_cut(const uint32_t *t_sorted, uint64_t n);
+/* Lloyd's k-means with k = 2 on sorted t[0..n) ("k-means", P:L258 k = 2;
+ * reading R26): returns the converged cut k in [1, n-1], 0 when no cut exists;
+ * *iters gets the number of assignment steps. */
+uint64_t or_lloyd_cut(const uint32_t *t_sorted, uint64_t n, uint32_t *iters);
 /* Eq. 3: m = ceil((V/S^2) * (z/eps)^2) for a cluster with moments. */
 double or_eq3_m(uint64_t n, uint64_t S, uint64_t Q_lo, uint64_t Q_hi, double eps, double z, int clamp);
 /* Eq. 6, corrected numerator: k clusters given a_i = mu_i, b_i = V_i

@@ -153,6 +153,39 @@ def test_split_is_optimal_two_means_brute_force():
         assert k == first
 
 
+def test_lloyd_variant_fixed_point_and_bounds():
+    """split=1 (reading R26): Lloyd's k-means with k = 2 from the (min, max)
+    centroids.  Pinned by what Lloyd's algorithm guarantees,
+    not by retyping it: the returned cut is a fixed point of the assignment
+    step (every value is on the side of its nearer centroid, ties to the left),
+    it never separates equal values, its SSE is no better than the brute-force
+    optimum and equals it on two well-separated groups, and on some inputs the
+    local optimum it stops at is strictly worse than the global one (so the
+    option really is a different split rule from the default)."""
+    rng = random.Random(23)
+    worse = 0
+    for _ in range(800):
+        n = rng.randint(2, 11)
+        t = sorted(rng.choice([rng.randint(0, 6), rng.randint(0, 60), rng.randint(0, 600)]) for _ in range(n))
+        k, iters = O.lloyd_cut(t)
+        if t[0] == t[-1]:
+            assert k == 0
+            continue
+        assert 1 <= k < n and t[k - 1] < t[k] and iters >= 1
+        c1, c2 = Fraction(sum(t[:k]), k), Fraction(sum(t[k:]), n - k)
+        assert all(2 * x <= c1 + c2 for x in t[:k]) and all(2 * x > c1 + c2 for x in t[k:])
+        best = min(_sse(t[:j]) + _sse(t[j:]) for j in range(1, n))   # contiguous cuts suffice (1-D)
+        mine = _sse(t[:k]) + _sse(t[k:])
+        assert mine >= best
+        worse += mine > best
+    assert worse > 0
+    for _ in range(50):   # two well-separated groups: the global optimum
+        a = [rng.randint(0, 50) for _ in range(rng.randint(1, 8))]
+        b = [10_000 + rng.randint(0, 50) for _ in range(rng.randint(1, 8))]
+        t = sorted(a + b)
+        assert O.lloyd_cut(t)[0] == len(a) == O.best_cut(t)
+
+
 def test_split_exact_tie(golden):
     for c in golden("split_tie.json")["cases"]:
         t = [c["s"] * x for x in c["base"]]
