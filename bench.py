@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--ref-sample-rows", type=int, default=8_000_000)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--split", type=int, default=0, help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26)")
     return ap.parse_args()
 
 
@@ -197,9 +198,9 @@ def run_ours(a):
     def step(timing=False):
         if comm is not None:
             return ctx.plan_dist(comm, kid, tt, sp.n_kernels, row0, eps=eps, conf=a.conf, metrics=met, seed=12345,
-                                 to_host=False, stream=stream.cuda_stream)
+                                 to_host=False, stream=stream.cuda_stream, split=a.split)
         return ctx.plan(kid, tt, sp.n_kernels, eps=eps, conf=a.conf, metrics=met, seed=12345, to_host=False,
-                        stream=stream.cuda_stream)
+                        stream=stream.cuda_stream, split=a.split)
 
     for _ in range(a.warmup):
         step()
@@ -260,6 +261,7 @@ def run_ours(a):
         "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded, on device)",
         "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n,
                    "kernels": sp.n_kernels, "eps": eps, "conf": a.conf, "metrics": nm,
+                   "split": "exact optimal 2-means (R5)" if a.split == 0 else "Lloyd k-means, k = 2 (R26)",
                    "parallelism": "single GPU" if world == 1 else
                    f"{world} GPUs: row shards, NCCL all-to-all by kernel id, exact allreduce",
                    "l2": "inputs 8 B/row x rows >> 126 MB L2 (no flush needed)" if n_local >= 50_000_000
@@ -292,9 +294,9 @@ def run_ours(a):
         def e2e_step():
             if comm is not None:
                 return ctx.plan_dist(comm, hk, ht, sp.n_kernels, row0, eps=eps, conf=a.conf, metrics=hm,
-                                     seed=12345, stream=stream.cuda_stream)
+                                     seed=12345, stream=stream.cuda_stream, split=a.split)
             return ctx.plan(hk, ht, sp.n_kernels, eps=eps, conf=a.conf, metrics=hm, seed=12345,
-                            stream=stream.cuda_stream)
+                            stream=stream.cuda_stream, split=a.split)
         p = e2e_step()
         torch.cuda.synchronize()
         if world > 1:

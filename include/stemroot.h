@@ -42,7 +42,7 @@
 extern "C" {
 #endif
 
-#define STEMROOT_ABI_VERSION 1
+#define STEMROOT_ABI_VERSION 2   /* 2: stem_opts.split */
 
 #if defined(__GNUC__)
 #define STEM_API __attribute__((visibility("default")))
@@ -83,6 +83,10 @@ typedef struct stem_opts {
                                 cluster per kernel                                               */
     int      clamp_in_split; /* 1 (default): m >= 1 inside Eq. 7/8; 0: literal ceilings (R7)     */
     int      census_cap;     /* 1: a leaf whose m_i >= n_i takes all its n_i rows once (exact)   */
+    int      split;          /* ROOT's sub-clustering ("a clustering method (e.g.,
+                                k-means)", P:L258 k = 2): 0 (default) the exact optimal 2-means
+                                cut (R5); 1 Lloyd's k-means, k = 2, from the (min, max)
+                                centroids to its fixed point (R26); other values: STEM_E_INVAL   */
     void    *stream;         /* cudaStream_t to run on; NULL = the legacy default stream         */
 } stem_opts;
 

@@ -69,7 +69,7 @@ class stem_trace(C.Structure):
 
 class stem_opts(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("z", C.c_double), ("scope", C.c_int), ("root", C.c_int),
-                ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("stream", C.c_void_p)]
+                ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("split", C.c_int), ("stream", C.c_void_p)]
 
 
 class stem_cluster(C.Structure):
@@ -272,7 +272,7 @@ class Context:
 
     def plan(self, kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, metrics=None,
              seed: int = 0, z: float = 0.0, scope: int = 0, root: bool = True, clamp_in_split: bool = True,
-             census_cap: bool = False, stream=None, to_host: bool = True):
+             census_cap: bool = False, stream=None, to_host: bool = True, split: int = 0):
         """stem_root_plan_ctx.  Returns the host plan as numpy arrays, or None when to_host=False
         (the plan then stays on the device: see device_plan())."""
         kp, kdev, k_keep = _arg(kernel_id, np.uint32)
@@ -291,7 +291,7 @@ class Context:
             import torch
             stream = torch.cuda.current_stream(kdev).cuda_stream
         o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
-                      stream or None)
+                      int(split), stream or None)
         out = C.POINTER(stem_plan)()
         st = lib().stem_root_plan_ctx(self._h, C.byref(tr), eps, conf, C.byref(o),
                                       C.byref(out) if to_host else None)
@@ -305,7 +305,7 @@ class Context:
 
     def plan_dist(self, comm: "Comm", kernel_id, exec_ns, n_kernels: int, global_row_base: int, eps: float = 0.05,
                   conf: float = 0.95, metrics=None, seed: int = 0, z: float = 0.0, scope: int = 0, root: bool = True,
-                  clamp_in_split: bool = True, census_cap: bool = False, stream=None, to_host: bool = True):
+                  clamp_in_split: bool = True, census_cap: bool = False, stream=None, to_host: bool = True, split: int = 0):
         """stem_root_plan_dist (collective).  Returns the global plan on rank 0, None elsewhere."""
         kp, kdev, k_keep = _arg(kernel_id, np.uint32)
         tp, tdev, t_keep = _arg(exec_ns, np.uint32)
@@ -319,7 +319,7 @@ class Context:
             stream = torch.cuda.current_stream(kdev).cuda_stream
         tr = stem_trace(n, n_kernels, kp if n else None, tp if n else None, nm, mp if n else None, kdev)
         o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
-                      stream or None)
+                      int(split), stream or None)
         out = C.POINTER(stem_plan)()
         st = lib().stem_root_plan_dist(self._h, comm._h, C.byref(tr), global_row_base, eps, conf, C.byref(o),
                                        C.byref(out) if to_host else None)
@@ -358,7 +358,7 @@ class Context:
 
 def plan(kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, metrics=None, seed: int = 0,
          z: float = 0.0, scope: int = 0, root: bool = True, clamp_in_split: bool = True, census_cap: bool = False,
-         stream=None) -> dict:
+         stream=None, split: int = 0) -> dict:
     """stem_root_plan: one-shot plan (temporary workspace), host plan out."""
     kp, kdev, k_keep = _arg(kernel_id, np.uint32)
     tp, tdev, t_keep = _arg(exec_ns, np.uint32)
@@ -374,7 +374,7 @@ def plan(kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.
         stream = torch.cuda.current_stream(kdev).cuda_stream
     tr = stem_trace(n, n_kernels, kp, tp, nm, mp, kdev)
     o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
-                  stream or None)
+                  int(split), stream or None)
     out = C.POINTER(stem_plan)()
     _check(lib().stem_root_plan(C.byref(tr), eps, conf, C.byref(o), C.byref(out)), "stem_root_plan")
     del k_keep, t_keep, m_keep

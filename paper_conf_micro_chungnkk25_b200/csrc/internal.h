@@ -227,7 +227,8 @@ int dist_metric_sums(Ctx &c, const double *metrics_local, uint32_t nm, uint64_t 
 int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *row_in, uint64_t n,
                uint32_t K, bool allow_pack);                                                   // a1
 int prefix_moments(Ctx &c, uint64_t n);                                                        // a2
-int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp);   // a3, a4
+int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp,
+                int split);   // a3, a4 (split: 0 exact 2-means, 1 Lloyd)
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,
                       uint32_t *tailh);   // pre-pass only

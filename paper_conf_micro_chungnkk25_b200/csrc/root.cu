@@ -594,6 +594,60 @@ __global__ void __launch_bounds__(256, MINB) small_split_kernel(const uint32_t *
     }
 }
 
+// ---------------------------------------------------------------- split variant: Lloyd (R26)
+// Lloyd's k-means with k = 2 ("k-means", P:L258 k = 2) from the (min, max)
+// centroids to its fixed point, one warp per cluster.  On sorted rows an
+// assignment is a cut: cluster 1 = the rows with 2 t <= c1 + c2, i.e. with the
+// exact fractional centroids c1 = S1/k, c2 = S2/(n-k), t * 2k(n-k) <= S1 (n-k)
+// + S2 k (integers < 2^97).  The cut is found by a 33-ary search (32 probes per
+// warp round trip), S1 from the sampled prefix; at most kLloydMaxIters
+// assignment steps (the bound DESIGN.md R26 states for both sides).
+constexpr uint32_t kLloydMaxIters = 1000;
+
+// first row in [a, b) whose t fails t * f <= rhs (rows sorted by t, so the
+// rows passing the test form a prefix); every lane returns it
+__device__ __forceinline__ uint64_t warp_cut_search(const uint32_t *__restrict__ t, uint64_t a, uint64_t b, uint64_t f,
+                                                    u128 rhs) {
+    const int lane = threadIdx.x & 31;
+    while (b - a > 32) {
+        const uint64_t p = a + ((uint64_t)(lane + 1) * (b - a)) / 33;
+        const uint32_t m = __ballot_sync(0xffffffffu, (u128)t[p] * f <= rhs);
+        const int c = __popc(m);   // a prefix of the probes passes
+        const uint64_t pa = __shfl_sync(0xffffffffu, p, c > 0 ? c - 1 : 0), pb = __shfl_sync(0xffffffffu, p, c < 32 ? c : 31);
+        if (c > 0) a = pa + 1;
+        if (c < 32) b = pb;
+    }
+    const uint32_t m = __ballot_sync(0xffffffffu, a + lane < b && (u128)t[a + lane] * f <= rhs);
+    return a + __popc(m);
+}
+
+__global__ void __launch_bounds__(256) lloyd_split_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
+                                                          const uint64_t *__restrict__ f_S, uint32_t C,
+                                                          const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
+                                                          uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
+        const uint64_t lo = f_lo[c], hi = f_hi[c], n = hi - lo, S = f_S[c];
+        const uint64_t base = pref1(PS1, t, lo);
+        // steps 1-2: centroids (min, max), first assignment 2 t <= min + max
+        uint64_t k = warp_cut_search(t, lo, hi, 2, (u128)t[lo] + t[hi - 1]) - lo;
+        uint64_t S1 = 0;
+        for (uint32_t it = 1;; it++) {
+            S1 = pref1(PS1, t, lo + k) - base;   // step 3: exact centroid sums
+            if (it >= kLloydMaxIters) break;
+            const u128 rhs = (u128)S1 * (n - k) + (u128)(S - S1) * k;
+            const uint64_t k2 = warp_cut_search(t, lo, hi, 2 * k * (n - k), rhs) - lo;
+            if (k2 == k) break;
+            k = k2;
+        }
+        if (lane == 0) {
+            cut[c] = (uint32_t)k;
+            cut_SL[c] = S1;
+        }
+    }
+}
+
 // ---------------------------------------------------------------- big clusters: chunk bounds
 // Clusters of >= kBig rows.  One block per kBigSeg rows.  For every 32-row chunk
 // (aligned to the sampled prefix PS1) the concavity bound of |D| gives an upper
@@ -1161,7 +1215,7 @@ static int ensure_frontier(Ctx &c, int b, uint64_t cap) {
     return STEM_OK;
 }
 
-int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp) {
+int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, int split) {
     cudaStream_t st = c.stream;
     {
         const uint64_t b = big_rows();
@@ -1229,6 +1283,11 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         if (tk_l >= 0) c.stage_end(tk_l, 4 * A);
         CK(cudaGetLastError());
         const int tk_s = c.stage_begin("root_split");
+        if (split == 1) {   // Lloyd variant: one warp per cluster, every size
+            lloyd_split_kernel<<<(unsigned)min((C + 7) / 8, (uint64_t)c.sms * 16), 256, 0, st>>>(
+                c.f_lo[cur], c.f_hi[cur], c.f_S[cur], (uint32_t)C, c.t_sorted, c.PS1, c.cut, c.cut_SL);
+            c.launches++;
+        } else {
         // the small-cluster warps run on a side stream beside the big-cluster
         // chain (both latency-bound; they read the same frontier and write
         // disjoint cuts), joined before the decision
@@ -1285,6 +1344,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             CK(cudaEventRecord(c.ev_join, c.side));
             CK(cudaStreamWaitEvent(st, c.ev_join, 0));
         }
+        }   // split == 0
         c.stage_end(tk_s, 4 * A + 20 * C);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");

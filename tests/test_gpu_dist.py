@@ -129,3 +129,12 @@ def test_packed_sort_candidate_rows_dist(sr, monkeypatch, world):
     ref = O.plan(kid, t, 5, eps=0.002, z=Z95, seed=8)
     got = _dist_plan(sr, kid, t, 5, world, eps=0.002, z=Z95, seed=8)
     assert_plans_equal(got, ref)
+
+
+def test_loopback_lloyd_split(sr):
+    """the Lloyd split variant (opts.split = 1) is independent of the rank count too"""
+    sp = G.spec("C2", n=120_000)
+    kid, t, _ = G.generate_np(sp)
+    ref = O.plan(kid, t, sp.n_kernels, eps=0.04, z=Z95, seed=6, split=1)
+    got = _dist_plan(sr, kid, t, sp.n_kernels, 3, eps=0.04, z=Z95, seed=6, split=1)
+    assert_plans_equal(got, ref)

@@ -348,3 +348,40 @@ def test_tile_boundaries(ctx, n):
     kid, t = _mixture(rng, n, 3 if n > 3 else 1, peaks=2, spread=0.2)
     got, ref = _both(ctx, kid, t, 3 if n > 3 else 1, eps=0.02, seed=n)
     assert_plans_equal(got, ref)
+
+
+# ------------------------------------------------------------------ split variant: Lloyd's k-means (R26)
+@pytest.mark.parametrize("case", ["mixture", "c2", "big", "ties"])
+def test_lloyd_split_variant(ctx, case):
+    """opts.split = 1 (Lloyd's k-means, k = 2, from (min, max), P:L192/P:L258,
+    reading R26): clusters, sizes and sample rows bit-exact against the oracle's
+    step-by-step Lloyd, on mixtures, a CASIO-shaped trace, multi-block clusters
+    and long runs of equal times."""
+    rng = np.random.default_rng(5)
+    if case == "mixture":
+        kid, t = _mixture(rng, 150_001, 97, peaks=4, spread=0.3)
+        K = 97
+    elif case == "c2":
+        sp = G.spec("C2", n=300_000)
+        kid, t, _ = G.generate_np(sp)
+        K = sp.n_kernels
+    elif case == "big":
+        t = np.concatenate([rng.lognormal(11, 1.0, 700_000), rng.normal(5e4, 3e3, 400_000).clip(1)]).astype(np.uint32)
+        kid = np.r_[np.zeros(700_000, np.uint32), np.ones(400_000, np.uint32)]
+        K = 2
+    else:
+        kid, t = _dup_heavy(200_003, 7, 3)
+        K = 7
+    got, ref = _both(ctx, kid, t, K, eps=0.03, seed=9, split=1)
+    assert_plans_equal(got, ref)
+    # the variant is a different rule: the default's leaves differ somewhere
+    if case in ("mixture", "c2"):
+        d = O.plan(kid, t, K, eps=0.03, z=Z95, seed=9)
+        assert len(d["n"]) != len(ref["n"]) or not np.array_equal(d["n"], ref["n"])
+
+
+def test_split_option_validation(ctx, sr):
+    kid = np.zeros(100, np.uint32)
+    t = np.arange(100, dtype=np.uint32)
+    with pytest.raises(sr.StemError):
+        ctx.plan(kid, t, 1, split=2)
