@@ -400,20 +400,34 @@ struct EstArgs {
 
 __global__ void __launch_bounds__(kThreads) estimate_kernel(EstArgs a) {
     __shared__ double sm[kThreads / 32];
+    __shared__ unsigned long long s_q[kThreads / 32];
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     double frac = 0.0, var = 0.0;
+    uint64_t q = 0;
     if (i < a.L) {
         const LeafView v = leaf_view(a.leaf_lo, a.L, a.n, a.PS1, a.PS2, a.t, i);
         const uint64_t m = a.m[i];
         const u128 num = (u128)v.n * a.U[i];
-        const uint64_t q = (uint64_t)(num / m), r = (uint64_t)(num % m);
-        atomicAdd((unsigned long long *)a.sum_q, (unsigned long long)q);
+        uint64_t r;
+        if ((uint64_t)(num >> 64) == 0) {   // the common case (m = 1: U < 2^32): 64-bit division
+            q = (uint64_t)num / m;
+            r = (uint64_t)num - q * m;
+        } else {
+            q = (uint64_t)(num / m);
+            r = (uint64_t)(num % m);
+        }
         frac = __ddiv_rn(rn64(r), rn64(m));
         var = __ddiv_rn(rn128(v.V), rn64(m));
     }
+    // sum_i q_i: one atomic per block (exact integer, any order)
+    for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+    if ((threadIdx.x & 31) == 0) s_q[threadIdx.x >> 5] = q;
     const double f = block_sum(frac, sm);
     const double vv = block_sum(var, sm);
     if (threadIdx.x == 0) {
+        unsigned long long bq = 0;
+        for (int w = 0; w < kThreads / 32; w++) bq += s_q[w];
+        if (bq) atomicAdd((unsigned long long *)a.sum_q, bq);
         a.part[2 * blockIdx.x] = f;
         a.part[2 * blockIdx.x + 1] = vv;
     }

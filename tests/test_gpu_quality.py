@@ -16,7 +16,7 @@ def test_quality_harness_c2():
     res = quality.run("C2", n=200_000, n_seeds=24, eps_list=(0.03, 0.25))
     m = res["methods"]
     eps = res["eps"]
-    for name in ("stem+root", "stem", "per-kernel", "per-leaf"):
+    for name in ("stem+root", "stem", "per-kernel", "per-leaf", "lloyd"):
         r = m[name]
         assert r["mean_error_pct"] < 100 * eps, (name, r)
         assert r["coverage_of_eps"] >= 0.9, (name, r)
