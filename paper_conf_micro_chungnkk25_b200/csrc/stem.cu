@@ -262,7 +262,10 @@ __device__ __forceinline__ uint32_t map_row(const SampleArgs &a, uint32_t r) {
 __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
     const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= a.S) return;
-    const uint64_t i = upper_bound(a.moff, a.L, s) - 1;
+    // leaf of sample s: s itself while every earlier leaf has m = 1 (the common
+    // case: one load), else a binary search over the sample offsets
+    uint64_t i = s;
+    if (!(s < a.L && a.moff[s] == s)) i = upper_bound(a.moff, a.L, s) - 1;
     const uint64_t j = s - a.moff[i];
     const uint32_t lo = a.leaf_lo[i];
     const uint32_t hi = (i + 1 < a.L) ? a.leaf_lo[i + 1] : (uint32_t)a.n;
@@ -288,9 +291,18 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
             // sorted run; the candidates (h << s) | low that hold (kernel, t)
             const uint32_t k = a.leaf_kid[i];
             uint64_t mask = 0;
-            for (uint32_t h = 0; h < a.pack_h; h++) {
-                const uint64_t r = ((uint64_t)h << a.pack_s) | low;
-                if (r < a.n && __ldg(a.kid_in + r) == k && __ldg(a.t_in + r) == tv) mask |= 1ull << h;
+            for (uint32_t h0 = 0; h0 < a.pack_h; h0 += 16) {   // 16 candidates' loads in flight
+                uint32_t kv[16], tw[16];
+#pragma unroll
+                for (int u = 0; u < 16; u++) {
+                    const uint64_t r = ((uint64_t)(h0 + u) << a.pack_s) | low;
+                    const bool ok = h0 + u < a.pack_h && r < a.n;
+                    kv[u] = ok ? __ldg(a.kid_in + r) : 0xFFFFFFFFu;   // never a kernel id (K <= 2^24)
+                    tw[u] = ok ? __ldg(a.t_in + r) : 0u;
+                }
+#pragma unroll
+                for (int u = 0; u < 16; u++)
+                    if (kv[u] == k && tw[u] == tv) mask |= 1ull << (h0 + u);
             }
             if (__popcll(mask) == 1) {
                 a.out_row[s] = map_row(a, (uint32_t)(((uint64_t)(__ffsll(mask) - 1) << a.pack_s) | low));
