@@ -50,6 +50,9 @@ void Ctx::release() {
     if (ev_fork) cudaEventDestroy(ev_fork);
     if (ev_join) cudaEventDestroy(ev_join);
     if (side) cudaStreamDestroy(side);
+    for (int i = 0; i < 4; i++)
+        if (ev_lvl[i]) { cudaEventDestroy(ev_lvl[i]); ev_lvl[i] = nullptr; }
+    if (h_lvl) { cudaFreeHost(h_lvl); h_lvl = nullptr; }
     ev_fork = ev_join = nullptr;
     side = nullptr;
     dfree(in_kid, cap_in_kid); dfree(in_t, cap_in_t); dfree(in_met, cap_in_met);

@@ -34,6 +34,7 @@ struct DevScalars {
     uint64_t scan_total64;        // generic scan total
     uint64_t scan_total64b;       // second scan total (coarse key bases)
     uint64_t frontier_total;      // packed (count << 32 | rows) of the next frontier
+    uint64_t ftot[2];             // ROOT levels: packed totals of the ping-pong frontiers
     uint64_t n_leaves;            // leaves after compaction
     uint64_t total_m;             // sum of m_i
     uint64_t sum_q;               // sum_i floor(n_i U_i / m_i)
@@ -104,6 +105,8 @@ struct Ctx {
     cudaStream_t stream = nullptr;
     cudaStream_t side = nullptr;                 // ROOT: the small-cluster split runs beside the big path
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    uint64_t *h_lvl = nullptr;                     // pinned: per-level frontier totals (ring of kLvlRing)
+    cudaEvent_t ev_lvl[4] = {nullptr, nullptr, nullptr, nullptr};
     uint32_t launches = 0;
     stem_stats stats{};
     Timing timing;

@@ -576,11 +576,12 @@ __device__ __forceinline__ Cand warp_best_cut(const uint32_t *__restrict__ t, co
 template <int MINB>
 __global__ void __launch_bounds__(256, MINB) small_split_kernel(const uint32_t *__restrict__ f_lo,
                                                           const uint32_t *__restrict__ f_hi,
-                                                          const uint64_t *__restrict__ f_S, uint32_t C,
+                                                          const uint64_t *__restrict__ f_S, const uint64_t *ctot,
                                                           const uint32_t *__restrict__ t,
                                                           const uint64_t *__restrict__ PS1,
                                                           const uint32_t *__restrict__ TB, uint32_t *__restrict__ cut,
                                                           uint64_t *__restrict__ cut_SL) {
+    const uint32_t C = (uint32_t)(*ctot >> 32);   // frontier size, read on the device (pipelined levels)
     const int lane = threadIdx.x & 31;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
@@ -622,9 +623,10 @@ __device__ __forceinline__ uint64_t warp_cut_search(const uint32_t *__restrict__
 }
 
 __global__ void __launch_bounds__(256) lloyd_split_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
-                                                          const uint64_t *__restrict__ f_S, uint32_t C,
+                                                          const uint64_t *__restrict__ f_S, const uint64_t *ctot,
                                                           const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
                                                           uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
+    const uint32_t C = (uint32_t)(*ctot >> 32);
     const int lane = threadIdx.x & 31;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
@@ -665,11 +667,12 @@ __device__ __forceinline__ uint32_t big_nseg(uint64_t lo, uint64_t hi) {
     return (uint32_t)((hi - lo + kBigSeg - 1) / kBigSeg);
 }
 
-__global__ void big_entries_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, uint32_t C,
-                                   BigEntry *__restrict__ ent, uint32_t *__restrict__ first_ent,
-                                   uint32_t *__restrict__ count) {
+__global__ void big_entries_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
+                                   const uint64_t *ctot, BigEntry *__restrict__ ent, uint32_t *__restrict__ first_ent,
+                                   uint32_t *__restrict__ count, unsigned long long *__restrict__ thr) {
     const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= C) return;
+    if (c >= (*ctot >> 32)) return;
+    thr[c] = 0;   // the cluster's pruning threshold (seeded and raised by the big-path kernels)
     const uint64_t n = f_hi[c] - f_lo[c];
     if (n < c_big) return;
     const uint32_t nb = big_nseg(f_lo[c], f_hi[c]);
@@ -932,9 +935,11 @@ __global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
 }
 
 // one block per big cluster: argmax over its entries
-__global__ void big_reduce_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi, uint32_t C,
-                                  const uint32_t *__restrict__ first_ent, const Cand *__restrict__ part,
-                                  uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
+__global__ void big_reduce_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
+                                  const uint64_t *ctot, const uint32_t *__restrict__ first_ent,
+                                  const Cand *__restrict__ part, uint32_t *__restrict__ cut,
+                                  uint64_t *__restrict__ cut_SL) {
+  const uint64_t C = *ctot >> 32;
   for (uint64_t c = blockIdx.x; c < C; c += gridDim.x) {
     const uint64_t n = f_hi[c] - f_lo[c];
     if (n < c_big) continue;
@@ -959,7 +964,7 @@ struct DecideArgs {
     const uint32_t *f_lo, *f_hi, *cut;
     const uint64_t *f_S, *cut_SL;
     const u128 *f_Q;
-    uint32_t C;
+    const uint64_t *ctot;   // packed (count << 32 | rows) of the current frontier
     const uint64_t *PS1;
     const u128 *PS2;
     const uint32_t *t;
@@ -1023,7 +1028,7 @@ __global__ void __launch_bounds__(256) decide_kernel(DecideArgs a) {
     uint64_t S = 0, SL = 0;
     u128 Q = 0, QL = 0;
     bool ntL = false, ntR = false;
-    if (c < a.C) {
+    if (c < (*a.ctot >> 32)) {
         lo = a.f_lo[c];
         hi = a.f_hi[c];
         const uint32_t k = a.cut[c];
@@ -1190,14 +1195,6 @@ __global__ void group_flags_kernel(const uint32_t *goff, uint32_t K, uint32_t *f
     if (g < K && goff[g] < goff[g + 1]) atomicOr(&flags[goff[g] >> 5], 1u << (goff[g] & 31));
 }
 
-static int read_frontier_total(Ctx &c, uint64_t &C, uint64_t &A) {
-    uint64_t tot = 0;
-    CK(cudaMemcpyAsync(&tot, &c.scalars->frontier_total, sizeof(uint64_t), cudaMemcpyDeviceToHost, c.stream));
-    CK(cudaStreamSynchronize(c.stream));
-    C = tot >> 32;
-    A = tot & 0xFFFFFFFFull;
-    return STEM_OK;
-}
 
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K) {
     CK(cudaMemsetAsync(c.flags, 0, sizeof(uint32_t) * (n / 32 + 1), c.stream));
@@ -1255,37 +1252,51 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                 nS[idx] = s1 - s0;
                 nQ[idx] = q1 - q0;
             },
-            (uint64_t)K, (uint64_t *)c.scan_scratch, &c.scalars->frontier_total, st, &c.launches);
+            (uint64_t)K, (uint64_t *)c.scan_scratch, &c.scalars->ftot[0], st, &c.launches);
         c.stage_end(tk, 64 * (uint64_t)K);
         CK(cudaGetLastError());
     }
-    uint64_t C = 0, A = 0;
-    CKS(read_frontier_total(c, C, A));
-    int cur = 0;
+    // Levels, pipelined: level L+1 is enqueued before level L's frontier size is
+    // known on the host.  Kernels read the size of the frontier they consume
+    // from HBM (ftot[cur]); the host sizes grids and buffers from upper bounds
+    // (a level at most doubles the cluster count and never adds rows) and reads
+    // each level's exact total one level later (pinned ring + event), so the GPU
+    // always has the next level queued.  The level after the last one runs on an
+    // empty frontier (its kernels exit at once).  STEMROOT_LEVEL_SYNC=1, the
+    // local-subtree option and STEMROOT_DEBUG_LEVELS use one host round trip per level.
+    const bool pipelined = local_rows() == 0 && !debug_levels() &&
+                           !(getenv("STEMROOT_LEVEL_SYNC") && getenv("STEMROOT_LEVEL_SYNC")[0] == '1');
+    if (!c.h_lvl) {
+        CK(cudaMallocHost((void **)&c.h_lvl, sizeof(uint64_t) * 4));
+        for (int i = 0; i < 4; i++) CK(cudaEventCreateWithFlags(&c.ev_lvl[i], cudaEventDisableTiming));
+    }
+    uint64_t t0 = 0;
+    CK(cudaMemcpyAsync(&t0, &c.scalars->ftot[0], sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
     uint32_t levels = 0;
-    while (C > 0) {
-        levels++;
-        c.stats.active_rows += A;
-        CKS(c.ensure(c.cut, c.cap_cut, sizeof(uint32_t) * C));
-        CKS(c.ensure(c.cut_SL, c.cap_cut_SL, sizeof(uint64_t) * C));
-        CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(C) + 1) * sizeof(uint64_t)));
+    // enqueue ROOT level `level` (1-based) consuming frontier cur, bounded by (Cub, Aub)
+    auto enqueue_level = [&](uint32_t level, int cur, uint64_t Cub, uint64_t Aub) -> int {
         const int nxt = cur ^ 1;
-        CKS(ensure_frontier(c, nxt, 2 * C));   // at most 2 children per cluster
+        const uint64_t *ctot = &c.scalars->ftot[cur];
+        uint64_t *ntot = &c.scalars->ftot[nxt];
+        CKS(c.ensure(c.cut, c.cap_cut, sizeof(uint32_t) * Cub));
+        CKS(c.ensure(c.cut_SL, c.cap_cut_SL, sizeof(uint64_t) * Cub));
+        CKS(ensure_frontier(c, nxt, 2 * Cub));   // at most 2 children per cluster
         const int tk_l = local_rows() > 0 ? c.stage_begin("root_local") : -1;
         if (local_rows() > 0) {
-            LocalArgs la{c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], (uint32_t)C, levels - 1, c.PS1, c.PS2,
+            LocalArgs la{c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], (uint32_t)Cub, level - 1, c.PS1, c.PS2,
                          c.t_sorted, c.TB, c.flags, eps, z, k2, clamp, &c.scalars->local_rows, &c.scalars->local_depth,
                          &c.scalars->err};
-            const uint64_t blocks = (C + 7) / 8;
+            const uint64_t blocks = (Cub + 7) / 8;
             local_root_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 64), 256, 0, st>>>(la);
             c.launches++;
         }
-        if (tk_l >= 0) c.stage_end(tk_l, 4 * A);
+        if (tk_l >= 0) c.stage_end(tk_l, 4 * Aub);
         CK(cudaGetLastError());
         const int tk_s = c.stage_begin("root_split");
         if (split == 1) {   // Lloyd variant: one warp per cluster, every size
-            lloyd_split_kernel<<<(unsigned)min((C + 7) / 8, (uint64_t)c.sms * 16), 256, 0, st>>>(
-                c.f_lo[cur], c.f_hi[cur], c.f_S[cur], (uint32_t)C, c.t_sorted, c.PS1, c.cut, c.cut_SL);
+            lloyd_split_kernel<<<(unsigned)min((Cub + 7) / 8, (uint64_t)c.sms * 16), 256, 0, st>>>(
+                c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.cut, c.cut_SL);
             c.launches++;
         } else {
         // the small-cluster warps run on a side stream beside the big-cluster
@@ -1303,28 +1314,28 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             CK(cudaStreamWaitEvent(c.side, c.ev_fork, 0));
         }
         if (local_rows() < big_rows()) {
-            const uint64_t blocks = (C + 7) / 8;
+            const uint64_t blocks = (Cub + 7) / 8;
             static int minb = -1;   // STEMROOT_SMALL_MINB: resident blocks per SM the registers are sized for
             if (minb < 0) minb = getenv("STEMROOT_SMALL_MINB") ? atoi(getenv("STEMROOT_SMALL_MINB")) : 4;
             if (minb == 3)
                 small_split_kernel<3><<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, sst>>>(
-                    c.f_lo[cur], c.f_hi[cur], c.f_S[cur], (uint32_t)C, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
+                    c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
             else
                 small_split_kernel<4><<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, sst>>>(
-                    c.f_lo[cur], c.f_hi[cur], c.f_S[cur], (uint32_t)C, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
+                    c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
             c.launches++;
         }
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
-        const uint64_t max_ent = A / kBigSeg + A / big_rows() + 1;
-        CKS(c.ensure(c.big_ent, c.cap_big_ent, sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (C + 1)));
+        const uint64_t max_ent = Aub / kBigSeg + Aub / big_rows() + 1;
+        CKS(c.ensure(c.big_ent, c.cap_big_ent, sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (Cub + 1)));
         CKS(c.ensure(c.big_part, c.cap_big_part, sizeof(Cand) * max_ent));
-        CKS(c.ensure(c.big_thr, c.cap_big_thr, sizeof(unsigned long long) * C));
+        CKS(c.ensure(c.big_thr, c.cap_big_thr, sizeof(unsigned long long) * Cub));
         BigEntry *ent = (BigEntry *)c.big_ent;
         uint32_t *first_ent = (uint32_t *)(ent + max_ent);
         CK(cudaMemsetAsync(&c.scalars->big_count, 0, sizeof(uint32_t), st));
-        CK(cudaMemsetAsync(c.big_thr, 0, sizeof(unsigned long long) * C, st));
-        big_entries_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, ent,
-                                                                       first_ent, &c.scalars->big_count);
+        big_entries_kernel<<<(unsigned)((Cub + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], ctot, ent, first_ent,
+                                                                         &c.scalars->big_count,
+                                                                         (unsigned long long *)c.big_thr);
         BigArgs ba{ent, &c.scalars->big_count, c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.PS1, c.t_sorted, c.TB,
                    (unsigned long long *)c.big_thr, (Cand *)c.big_part, &c.scalars->split_chunks,
                    &c.scalars->split_scanned};
@@ -1337,34 +1348,65 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CK(big_attr);
         big_split_kernel<<<(unsigned)min(max_ent, (uint64_t)c.sms * 8), kBigThreads, kBigSmem, st>>>(ba);
         c.launches += 2;
-        big_reduce_kernel<<<(unsigned)min(C, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], (uint32_t)C, first_ent,
-                                                      (const Cand *)c.big_part, c.cut, c.cut_SL);
+        big_reduce_kernel<<<(unsigned)min(Cub, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], ctot, first_ent,
+                                                                        (const Cand *)c.big_part, c.cut, c.cut_SL);
         c.launches += 2;
         if (overlap) {
             CK(cudaEventRecord(c.ev_join, c.side));
             CK(cudaStreamWaitEvent(st, c.ev_join, 0));
         }
         }   // split == 0
-        c.stage_end(tk_s, 4 * A + 20 * C);
+        c.stage_end(tk_s, 4 * Aub + 20 * Cub);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");
-        CK(cudaMemsetAsync(&c.scalars->frontier_total, 0, sizeof(uint64_t), st));
-        DecideArgs da{c.f_lo[cur], c.f_hi[cur], c.cut, c.f_S[cur], c.cut_SL, c.f_Q[cur], (uint32_t)C, c.PS1, c.PS2,
+        CK(cudaMemsetAsync(ntot, 0, sizeof(uint64_t), st));
+        DecideArgs da{c.f_lo[cur], c.f_hi[cur], c.cut, c.f_S[cur], c.cut_SL, c.f_Q[cur], ctot, c.PS1, c.PS2,
                       c.t_sorted, c.flags, c.f_lo[nxt], c.f_hi[nxt], c.f_S[nxt], c.f_Q[nxt],
-                      &c.scalars->frontier_total, eps, z, k2, clamp};
-        decide_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(da);
+                      ntot, eps, z, k2, clamp};
+        decide_kernel<<<(unsigned)((Cub + 255) / 256), 256, 0, st>>>(da);
         c.launches += 1;
-        c.stage_end(tk_d, 96 * C);
+        c.stage_end(tk_d, 96 * Cub);
         CK(cudaGetLastError());
         if (debug_levels()) {   // STEMROOT_DEBUG_LEVELS=1: per-level frontier and big-path stats on stderr
             DevScalars hs;
             CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
-            fprintf(stderr, "level %u: clusters %llu rows %llu big_entries %u chunks %llu scanned %llu\n", levels,
-                    (unsigned long long)C, (unsigned long long)A, hs.big_count, hs.split_chunks, hs.split_scanned);
+            fprintf(stderr, "level %u: clusters %llu rows %llu big_entries %u chunks %llu scanned %llu\n", level,
+                    (unsigned long long)(hs.ftot[cur] >> 32), (unsigned long long)(hs.ftot[cur] & 0xFFFFFFFFull),
+                    hs.big_count, hs.split_chunks, hs.split_scanned);
         }
-        CKS(read_frontier_total(c, C, A));
-        cur = nxt;
+        CK(cudaMemcpyAsync(&c.h_lvl[level & 3], ntot, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaEventRecord(c.ev_lvl[level & 3], st));
+        return STEM_OK;
+    };
+    uint64_t Cprev = t0 >> 32, Aprev = t0 & 0xFFFFFFFFull;   // the frontier level 1 consumes (exact)
+    if (Cprev > 0) {
+        if (!pipelined) {
+            int cur = 0;
+            for (uint32_t level = 1; Cprev > 0; level++) {
+                levels = level;
+                c.stats.active_rows += Aprev;
+                CKS(enqueue_level(level, cur, Cprev, Aprev));
+                CK(cudaEventSynchronize(c.ev_lvl[level & 3]));
+                Cprev = c.h_lvl[level & 3] >> 32;
+                Aprev = c.h_lvl[level & 3] & 0xFFFFFFFFull;
+                cur ^= 1;
+            }
+        } else {
+            // level 1 with the exact bound, then level L+1 queued while level L runs
+            CKS(enqueue_level(1, 0, Cprev, Aprev));
+            uint64_t Cl = Cprev, Al = Aprev;   // exact size of the frontier level `level` consumes
+            for (uint32_t level = 1;; level++) {
+                levels = level;
+                c.stats.active_rows += Al;
+                // level + 1 consumes level's output: at most 2 Cl clusters, Al rows
+                CKS(enqueue_level(level + 1, level & 1, 2 * Cl, Al));
+                CK(cudaEventSynchronize(c.ev_lvl[level & 3]));
+                Cl = c.h_lvl[level & 3] >> 32;
+                Al = c.h_lvl[level & 3] & 0xFFFFFFFFull;
+                if (Cl == 0) break;   // the queued level runs on an empty frontier
+            }
+        }
     }
     DevScalars hs;
     CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
