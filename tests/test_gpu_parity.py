@@ -385,3 +385,18 @@ def test_split_option_validation(ctx, sr):
     t = np.arange(100, dtype=np.uint32)
     with pytest.raises(sr.StemError):
         ctx.plan(kid, t, 1, split=2)
+
+
+@pytest.mark.parametrize("split", [0, 1])
+def test_pipelined_levels_match_synchronous(ctx, monkeypatch, split):
+    """the pipelined ROOT level loop (the next level queued before the host sees
+    the frontier size) gives the same plan as one host round trip per level"""
+    rng = np.random.default_rng(77)
+    kid, t = _mixture(rng, 120_011, 41, peaks=5, spread=0.4)
+    a = ctx.plan(kid, t, 41, eps=0.02, z=Z95, seed=2, split=split)
+    monkeypatch.setenv("STEMROOT_LEVEL_SYNC", "1")
+    b = ctx.plan(kid, t, 41, eps=0.02, z=Z95, seed=2, split=split)
+    for f in ("kernel_id", "ordinal", "lo_ns", "hi_ns", "n", "sum_ns", "m"):
+        assert np.array_equal(a["clusters"][f], b["clusters"][f]), f
+    assert np.array_equal(a["sample_row"], b["sample_row"])
+    assert a["est_total_ns"] == b["est_total_ns"]
