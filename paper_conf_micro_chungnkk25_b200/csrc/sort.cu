@@ -35,6 +35,20 @@
 namespace sr {
 
 constexpr uint64_t kFlagA = 1ull << 62, kFlagP = 2ull << 62, kValMask = (1ull << 62) - 1;
+
+// Look-back statuses are u32 (flag in bits 30-31, count in bits 0-29) when
+// n < 2^30, else u64 (flag in bits 62-63): half the status traffic and clear.
+__device__ __forceinline__ void put_status(uint64_t *st, bool s32, uint64_t idx, uint64_t flag, uint64_t val) {
+    if (s32) __stcg(reinterpret_cast<uint32_t *>(st) + idx, (uint32_t)(flag >> 32) | (uint32_t)val);
+    else __stcg(st + idx, flag | val);
+}
+__device__ __forceinline__ uint64_t get_status(const uint64_t *st, bool s32, uint64_t idx) {
+    if (s32) {
+        const uint32_t v = *(volatile const uint32_t *)(reinterpret_cast<const uint32_t *>(st) + idx);
+        return ((uint64_t)(v >> 30) << 62) | (v & 0x3FFFFFFFu);
+    }
+    return *(volatile const uint64_t *)(st + idx);
+}
 constexpr int kMaxPasses = 8;
 constexpr int kRB = 8, kR = 1 << kRB;       // byte digits
 constexpr int kHistR = 256;                 // histogram row stride
@@ -257,7 +271,8 @@ struct PassArgs {
     const uint32_t *ballot;             // [pass] 1: equal-digit lanes by 8 ballots, 0: match.any
     const uint64_t *gbase;              // [pass][kHistR] exclusive scan of the pass's digit counts
     uint64_t *hist;                     // [pass][kHistR] global digit counts
-    uint64_t *status;                   // [ntiles][R]
+    uint64_t *status;                   // [ntiles][R] (u32 words when s32)
+    bool s32;                           // n < 2^30: 32-bit look-back statuses
     uint32_t *tile_counter;
 };
 
@@ -267,8 +282,8 @@ struct PassArgs {
 // multi-split (match.any), global offsets found by decoupled look-back
 // (thread d < 256 owns digit d), then keys are staged in shared memory in
 // tile-sorted order and written out in digit runs (coalesced).
-template <int NT, int IT, bool FIRST, bool LAST, bool FULL, bool PK>
-__global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesweep_kernel(PassArgs a) {
+template <int NT, int IT, bool FIRST, bool LAST, bool FULL, bool PK, bool S32>
+__global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : 4) : 1) onesweep_kernel(PassArgs a) {   // (FULL = false: one ragged tile; a looser bound avoids a ptxas C7600 failure)
     constexpr int NW = NT / 32, TILE = NT * IT, R = kR;
     static_assert(NT >= R, "one thread per digit");
     static_assert(NT * IT <= 65536, "16-bit ranks");
@@ -372,7 +387,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             }
     }
     __syncthreads();
-    if (tid < R && !a.late) __stcg(a.status + (uint64_t)tile * R + tid, (tile == 0 ? kFlagP : kFlagA) | s_cnt[tid]);
+    if (tid < R && !a.late) put_status(a.status, S32, (uint64_t)tile * R + tid, tile == 0 ? kFlagP : kFlagA, s_cnt[tid]);
     if (FIRST && tid < R)
         for (int x = 0; x < a.nxh; x++)
             if (s_xh[x * R + tid])
@@ -415,7 +430,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
             s_whist[ww][d] = (uint16_t)cnt;
             cnt += c;
         }
-        if (a.late) __stcg(a.status + (uint64_t)tile * R + d, (tile == 0 ? kFlagP : kFlagA) | cnt);
+        if (a.late) put_status(a.status, S32, (uint64_t)tile * R + d, tile == 0 ? kFlagP : kFlagA, cnt);
         c_incl = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -458,7 +473,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
                 uint64_t sv[kLB];
 #pragma unroll
                 for (int q = 0; q < kLB; q++)
-                    sv[q] = (j - q >= 0) ? *(volatile uint64_t *)(a.status + (uint64_t)(j - q) * R + d) : (2ull << 62);
+                    sv[q] = (j - q >= 0) ? get_status(a.status, S32, (uint64_t)(j - q) * R + d) : kFlagP;
 #pragma unroll
                 for (int q = 0; q < kLB; q++) {
                     if (done) break;
@@ -468,7 +483,7 @@ __global__ void __launch_bounds__(NT, (NT >= 448 ? 2 : NT >= 320 ? 3 : 4)) onesw
                     else { if (a.nap) __nanosleep(a.nap); break; }   // not published yet: poll again from tile j
                 }
             }
-            __stcg(a.status + (uint64_t)tile * R + d, kFlagP | (excl + cnt));
+            put_status(a.status, S32, (uint64_t)tile * R + d, kFlagP, excl + cnt);
         }
         s_delta[d] = (uint32_t)(a.gbase[a.pass * kHistR + d] + excl) - s_lstart[d];
     }
@@ -507,7 +522,7 @@ static int first_blocks() {
 
 // full tiles in one launch (no bounds checks), the ragged last tile in a second
 // launch: its look-back finds every predecessor already inclusive
-template <int NT, int IT, bool FIRST, bool LAST, bool PK>
+template <int NT, int IT, bool FIRST, bool LAST, bool PK, bool S32>
 static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
     constexpr uint64_t TILE = (uint64_t)NT * IT;
     const uint64_t full = a.n / TILE, rag = a.n % TILE;
@@ -523,7 +538,8 @@ static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
         // FIRST gathers B[kid]: keep L1 beside first_blocks() blocks' shared memory
         const int carve = FIRST ? (int)((first_blocks() * (sbase + 12 * 1024) * 100 + 228 * 1024 - 1) / (228 * 1024)) : 100;
         for (int f = 0; f < 2; f++) {
-            auto fn = f ? onesweep_kernel<NT, IT, FIRST, LAST, true, PK> : onesweep_kernel<NT, IT, FIRST, LAST, false, PK>;
+            auto fn = f ? onesweep_kernel<NT, IT, FIRST, LAST, true, PK, S32>
+                        : onesweep_kernel<NT, IT, FIRST, LAST, false, PK, S32>;
             if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smax) != cudaSuccess ||
                 cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, carve > 100 ? 100 : carve) !=
                     cudaSuccess)
@@ -533,28 +549,31 @@ static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
     }();
     if (attr_status) return STEM_E_CUDA;
     if (full) {
-        onesweep_kernel<NT, IT, FIRST, LAST, true, PK><<<(unsigned)full, NT, smem, st>>>(a);
+        onesweep_kernel<NT, IT, FIRST, LAST, true, PK, S32><<<(unsigned)full, NT, smem, st>>>(a);
         (*launches)++;
     }
     if (rag) {
-        onesweep_kernel<NT, IT, FIRST, LAST, false, PK><<<1, NT, smem, st>>>(a);
+        onesweep_kernel<NT, IT, FIRST, LAST, false, PK, S32><<<1, NT, smem, st>>>(a);
         (*launches)++;
     }
     return STEM_OK;
 }
 
-template <int NT, int IT, bool PK>
+template <int NT, int IT, bool PK, bool S32>
 static int launch_pass_pk(const PassArgs &a, bool first, bool last, cudaStream_t st, uint32_t *launches) {
-    if (first && last) return launch_pass<NT, IT, true, true, PK>(a, st, launches);
-    if (first) return launch_pass<NT, IT, true, false, PK>(a, st, launches);
-    if (last) return launch_pass<NT, IT, false, true, PK>(a, st, launches);
-    return launch_pass<NT, IT, false, false, PK>(a, st, launches);
+    if (first && last) return launch_pass<NT, IT, true, true, PK, S32>(a, st, launches);
+    if (first) return launch_pass<NT, IT, true, false, PK, S32>(a, st, launches);
+    if (last) return launch_pass<NT, IT, false, true, PK, S32>(a, st, launches);
+    return launch_pass<NT, IT, false, false, PK, S32>(a, st, launches);
 }
 
 template <int NT, int IT>
 static int launch_pass_cfg(const PassArgs &a, bool first, bool last, cudaStream_t st, uint32_t *launches) {
-    return a.ks ? launch_pass_pk<NT, IT, true>(a, first, last, st, launches)
-                : launch_pass_pk<NT, IT, false>(a, first, last, st, launches);
+    // 32-bit look-back statuses only in the packed mode (the common one); the
+    // payload mode keeps 64-bit ones
+    if (!a.ks) return launch_pass_pk<NT, IT, false, false>(a, first, last, st, launches);
+    return a.s32 ? launch_pass_pk<NT, IT, true, true>(a, first, last, st, launches)
+                 : launch_pass_pk<NT, IT, true, false>(a, first, last, st, launches);
 }
 
 // tile shape (threads, keys per thread): 256 x 20 (4 blocks/SM) measured
@@ -722,11 +741,13 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     a.gbase = gbase;
     a.hist = c.hist;
     a.status = (uint64_t *)c.sort_status;
+    a.s32 = ks && n < (1ull << 30) && !(getenv("STEMROOT_SORT_S32") && getenv("STEMROOT_SORT_S32")[0] == '0');
+    const size_t status_bytes = ntiles * kR * (a.s32 ? sizeof(uint32_t) : sizeof(uint64_t));
     a.tile_counter = &c.scalars->tile_counter;
     uint64_t *kin = c.keys[0], *kout = c.keys[1];
     uint32_t *vin = c.vals[0], *vout = c.vals[1];
     for (int p = 0; p < npasses; p++) {
-        CK(cudaMemsetAsync(a.status, 0, ntiles * kR * sizeof(uint64_t), st));
+        CK(cudaMemsetAsync(a.status, 0, status_bytes, st));
         CK(cudaMemsetAsync(a.tile_counter, 0, sizeof(uint32_t), st));
         a.shift = ks + kRB * p;
         a.pass = p;

@@ -400,3 +400,14 @@ def test_pipelined_levels_match_synchronous(ctx, monkeypatch, split):
         assert np.array_equal(a["clusters"][f], b["clusters"][f]), f
     assert np.array_equal(a["sample_row"], b["sample_row"])
     assert a["est_total_ns"] == b["est_total_ns"]
+
+
+@pytest.mark.parametrize("s32", ["0", "1"])
+def test_sort_status_widths(ctx, monkeypatch, s32):
+    """32-bit look-back statuses (n < 2^30, the default) and the 64-bit ones
+    (larger traces) give the oracle's plan"""
+    monkeypatch.setenv("STEMROOT_SORT_S32", s32)
+    rng = np.random.default_rng(31)
+    kid, t = _mixture(rng, 400_009, 123, peaks=3, spread=0.3)
+    got, ref = _both(ctx, kid, t, 123, eps=0.03, seed=12)
+    assert_plans_equal(got, ref)
