@@ -72,6 +72,9 @@ def lib():
         _lib.or_best_cut.restype = C.c_uint64
         _lib.or_lloyd_cut.argtypes = [u32p, C.c_uint64, C.POINTER(C.c_uint32)]
         _lib.or_lloyd_cut.restype = C.c_uint64
+        _lib.or_kmpp_cut.argtypes = [u32p, C.c_uint64, C.c_uint64, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32),
+                                     C.POINTER(C.c_uint32)]
+        _lib.or_kmpp_cut.restype = C.c_uint64
         _lib.or_eq3_m.argtypes = [C.c_uint64, C.c_uint64, C.c_uint64, C.c_uint64, C.c_double, C.c_double, C.c_int]
         _lib.or_eq3_m.restype = C.c_double
         _lib.or_eq6_m.argtypes = [C.c_uint32, dp, dp, C.c_double, C.c_double, C.c_double, dp]
@@ -153,6 +156,15 @@ def lloyd_cut(t_sorted):
     it = C.c_uint32(0)
     k = int(lib().or_lloyd_cut(_ptr(t, C.c_uint32), t.shape[0], C.byref(it)))
     return k, int(it.value)
+
+
+def kmpp_cut(t_sorted, seed):
+    """Lloyd's k-means (k = 2) from k-means++ seeds (reading R27): (cut, c1, c2, steps)."""
+    t = _u32(t_sorted)
+    c1, c2, it = C.c_uint32(0), C.c_uint32(0), C.c_uint32(0)
+    k = int(lib().or_kmpp_cut(_ptr(t, C.c_uint32), t.shape[0], seed & 0xFFFFFFFFFFFFFFFF, C.byref(c1),
+                              C.byref(c2), C.byref(it)))
+    return k, int(c1.value), int(c2.value), int(it.value)
 
 
 def best_cut(t_sorted) -> int:

@@ -249,12 +249,59 @@ static uint64_t best_cut(const uint32_t *t, uint64_t lo, uint64_t hi, uint64_t S
  * assignment a cut: cluster 1 = t[lo .. lo+k).  Returns k (0: no cut, the
  * cluster is constant or has < 2 rows). */
 #define OR_LLOYD_MAX_ITERS 1000
+static uint64_t lloyd_from(const uint32_t *t, uint64_t lo, uint64_t hi, uint64_t mid2, uint32_t *iters);
+
 static uint64_t lloyd_cut(const uint32_t *t, uint64_t lo, uint64_t hi, uint32_t *iters) {
+    if (iters) *iters = 0;
+    if (hi - lo < 2 || t[lo] == t[hi - 1]) return 0;
+    /* step 1: centroids (min, max) */
+    return lloyd_from(t, lo, hi, (uint64_t)t[lo] + t[hi - 1], iters);
+}
+
+/* k-means++ seeding for k = 2 (Arthur & Vassilvitskii's D^2 weighting; the
+ * randomised initialisation of a library k-means, reading R27),
+ * with the random numbers drawn from Philox4x32-10 (P10) on the counter
+ * (min t, max t, n, 'KMPP') and the plan's seed as key:
+ *   1. c1 = t[lo + j1], j1 = floor(u * n), u = (x1:x0) / 2^64 (uniform row);
+ *   2. c2 = t[lo + j2], row j2 drawn with probability (t[lo+j2] - c1)^2 / W,
+ *      W = sum_i (t_i - c1)^2: j2 = the first row whose running sum of
+ *      (t_i - c1)^2 exceeds R = floor(W x2 / 2^32).
+ * Then Lloyd's steps 2-4 as above from the centroids (c1, c2).  Returns the cut
+ * k (0 for a constant cluster or < 2 rows); c1, c2 are reported when asked. */
+static uint64_t kmpp_cut(const uint32_t *t, uint64_t lo, uint64_t hi, uint64_t seed, uint32_t *c1o,
+                         uint32_t *c2o, uint32_t *iters) {
     uint64_t n = hi - lo;
     if (iters) *iters = 0;
     if (n < 2 || t[lo] == t[hi - 1]) return 0;
-    /* step 1 and the first assignment: 2 t <= min + max */
-    uint64_t mid2 = (uint64_t)t[lo] + t[hi - 1];
+    const uint32_t ctr[4] = {t[lo], t[hi - 1], (uint32_t)n, 0x4B4D5050u};
+    const uint32_t key[2] = {(uint32_t)seed, (uint32_t)(seed >> 32)};
+    uint32_t x[4];
+    or_philox4x32_10(ctr, key, x);
+    uint64_t j1 = (uint64_t)(((u128)((((uint64_t)x[1]) << 32) | x[0]) * n) >> 64);
+    uint32_t c1 = t[lo + j1];
+    u128 W = 0;
+    for (uint64_t i = lo; i < hi; i++) {
+        uint64_t d = t[i] > c1 ? (uint64_t)t[i] - c1 : (uint64_t)c1 - t[i];
+        W += (u128)d * d;
+    }
+    u128 R = (W * x[2]) >> 32;
+    u128 run = 0;
+    uint64_t j2 = 0;
+    for (uint64_t i = lo; i < hi; i++) {
+        uint64_t d = t[i] > c1 ? (uint64_t)t[i] - c1 : (uint64_t)c1 - t[i];
+        run += (u128)d * d;
+        if (run > R) { j2 = i - lo; break; }
+    }
+    uint32_t c2 = t[lo + j2];
+    if (c1o) *c1o = c1;
+    if (c2o) *c2o = c2;
+    return lloyd_from(t, lo, hi, (uint64_t)c1 + c2, iters);
+}
+
+/* Lloyd's steps 2-4 from centroids whose sum is mid2 (both centroids are
+ * values of the cluster, distinct, so the first cut is in [1, n)). */
+static uint64_t lloyd_from(const uint32_t *t, uint64_t lo, uint64_t hi, uint64_t mid2, uint32_t *iters) {
+    uint64_t n = hi - lo;
     uint64_t k = 0;
     for (uint64_t i = lo; i < hi; i++)
         if (2 * (uint64_t)t[i] <= mid2) k++;
@@ -279,6 +326,11 @@ static uint64_t lloyd_cut(const uint32_t *t, uint64_t lo, uint64_t hi, uint32_t 
 
 uint64_t or_lloyd_cut(const uint32_t *t_sorted, uint64_t n, uint32_t *iters) {
     return lloyd_cut(t_sorted, 0, n, iters);
+}
+
+uint64_t or_kmpp_cut(const uint32_t *t_sorted, uint64_t n, uint64_t seed, uint32_t *c1, uint32_t *c2,
+                     uint32_t *iters) {
+    return kmpp_cut(t_sorted, 0, n, seed, c1, c2, iters);
 }
 
 uint64_t or_best_cut(const uint32_t *t_sorted, uint64_t n) {
@@ -333,12 +385,14 @@ void or_eq6_m(uint32_t k, const double *mu, const double *V, double T, double ep
 typedef struct { double tau_old, tau_new; uint64_t cut; int split; } decision;
 
 static decision root_decide(const uint32_t *t, uint64_t lo, uint64_t hi, double eps, double z,
-                            double k2, int clamp, int split) {
+                            double k2, int clamp, int split, uint64_t seed) {
     decision d = {0.0, 0.0, 0, 0};
     uint64_t n = hi - lo;
     if (n < 2 || t[lo] == t[hi - 1]) return d;              /* R5: leaf */
     moments all = range_moments(t, lo, hi);
-    uint64_t k = split == 1 ? lloyd_cut(t, lo, hi, NULL) : best_cut(t, lo, hi, all.S);
+    uint64_t k = split == 1   ? lloyd_cut(t, lo, hi, NULL)
+               : split == 2 ? kmpp_cut(t, lo, hi, seed, NULL, NULL, NULL)
+                            : best_cut(t, lo, hi, all.S);
     d.cut = k;
     /* Eq. 7: tau_old = m * Xbar with m from Eq. 3 */
     double mu = rn64(all.S) / rn64(all.n);
@@ -362,7 +416,7 @@ static decision root_decide(const uint32_t *t, uint64_t lo, uint64_t hi, double 
 int or_root_decide(const uint32_t *t_sorted, uint64_t n, double eps, double z, int clamp,
                    double *tau_old, double *tau_new, uint64_t *cut) {
     double q = z / eps;
-    decision d = root_decide(t_sorted, 0, n, eps, z, q * q, clamp, 0);
+    decision d = root_decide(t_sorted, 0, n, eps, z, q * q, clamp, 0, 0);
     if (tau_old) *tau_old = d.tau_old;
     if (tau_new) *tau_new = d.tau_new;
     if (cut) *cut = d.cut;
@@ -429,7 +483,7 @@ int or_plan_build(uint64_t n, uint32_t n_kernels, const uint32_t *kernel_id,
     if (!(eps > 0.0 && eps < 1.0) || !(opts->z > 0.0) || !isfinite(opts->z)) return OR_E_INVAL;
     if (n_metrics > 64 || (n_metrics > 0 && !metrics)) return OR_E_INVAL;
     if (opts->scope < 0 || opts->scope > 2) return OR_E_INVAL;
-    if (opts->split < 0 || opts->split > 1) return OR_E_INVAL;
+    if (opts->split < 0 || opts->split > 2) return OR_E_INVAL;
     if (n >= ((uint64_t)1 << 32)) return OR_E_RANGE;
     for (uint64_t i = 0; i < n; i++) if (kernel_id[i] >= n_kernels) return OR_E_RANGE;
 
@@ -467,7 +521,7 @@ int or_plan_build(uint64_t n, uint32_t n_kernels, const uint32_t *kernel_id,
             work_item w = work.v[--work.n];
             if (w.depth > max_depth) max_depth = w.depth;
             decision d = {0.0, 0.0, 0, 0};
-            if (opts->root) d = root_decide(t, w.lo, w.hi, eps, z, k2, clamp, opts->split);
+            if (opts->root) d = root_decide(t, w.lo, w.hi, eps, z, k2, clamp, opts->split, opts->seed);
             if (d.split) {
                 /* push right then left: the left child is visited first */
                 if (work_push(&work, w.lo + d.cut, w.hi, w.depth + 1) ||

@@ -28,7 +28,8 @@ typedef struct {
     int      clamp_in_split; /* 1: m >= 1 inside Eq.7/8; 0: literal ceilings       */
     int      census_cap;     /* 1: m_i >= n_i => take all n_i rows                 */
     int      split;          /* 0: exact optimal 2-means cut (R5); 1: Lloyd's k-means,
-                                k = 2, from the (min, max) centroids (R26)          */
+                                k = 2, from the (min, max) centroids (R26); 2: the
+                                same from k-means++ seeds drawn with seed (R27)     */
 } or_opts;
 
 /* Structure-of-arrays plan.  Everything is malloc'ed; free with or_plan_free. */
@@ -67,6 +68,12 @@ uint64_t or_best_cut(const uint32_t *t_sorted, uint64_t n);
  * reading R26): returns the converged cut k in [1, n-1], 0 when no cut exists;
  * *iters gets the number of assignment steps. */
 uint64_t or_lloyd_cut(const uint32_t *t_sorted, uint64_t n, uint32_t *iters);
+/* Lloyd's k-means with k = 2 from k-means++ seeds (reading R27): c1 a uniform
+ * row, c2 a row drawn with D^2 weights, both from Philox4x32-10 on the counter
+ * (t[0], t[n-1], n, 0x4B4D5050) and key seed; returns the cut (0: none) and
+ * the seeds *c1, *c2 (either pointer may be NULL). */
+uint64_t or_kmpp_cut(const uint32_t *t_sorted, uint64_t n, uint64_t seed, uint32_t *c1, uint32_t *c2,
+                     uint32_t *iters);
 /* Eq. 3: m = ceil((V/S^2) * (z/eps)^2) for a cluster with moments. */
 double or_eq3_m(uint64_t n, uint64_t S, uint64_t Q_lo, uint64_t Q_hi, double eps, double z, int clamp);
 /* Eq. 6, corrected numerator: k clusters given a_i = mu_i, b_i = V_i

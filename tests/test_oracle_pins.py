@@ -186,6 +186,77 @@ def test_lloyd_variant_fixed_point_and_bounds():
         assert O.lloyd_cut(t)[0] == len(a) == O.best_cut(t)
 
 
+def test_kmpp_seeds_follow_d2_weighting():
+    """split=2 (reading R27): the k-means++ seeds.  Pinned by the definition of
+    D^2 seeding (Arthur & Vassilvitskii): c1 is a uniform row, and given c1 the
+    second seed is row j with probability (t_j - c1)^2 / sum_i (t_i - c1)^2.
+    Over 24 000 seeds the joint frequency of (c1, c2) values must match those
+    exact probabilities (each cell within 5 binomial standard deviations) and
+    a zero-probability pair (c2 == c1) must never occur."""
+    t = [3, 3, 5, 9, 9, 9, 14, 20]
+    n = len(t)
+    vals = sorted(set(t))
+    cnt = {v: t.count(v) for v in vals}
+    prob = {}
+    for a in vals:
+        W = sum((x - a) ** 2 for x in t)
+        for b in vals:
+            prob[(a, b)] = Fraction(cnt[a], n) * Fraction(cnt[b] * (b - a) ** 2, W)
+    R = 24_000
+    seen = {}
+    for s in range(R):
+        k, c1, c2, it = O.kmpp_cut(t, 0x9E3779B97F4A7C15 * (s + 1))
+        assert c1 in cnt and c2 in cnt and c1 != c2 and 1 <= k < n and t[k - 1] < t[k] and it >= 1
+        seen[(c1, c2)] = seen.get((c1, c2), 0) + 1
+    for key, p in prob.items():
+        e = float(p) * R
+        sd = math.sqrt(max(e * (1 - float(p)), 1e-9))
+        assert abs(seen.get(key, 0) - e) <= 5 * sd + 1e-9, (key, seen.get(key, 0), e)
+
+
+def test_kmpp_variant_fixed_point_and_bounds():
+    """split=2 (R27): whatever the seeds, the result is a Lloyd fixed point on
+    the exact fractional centroids (ties to the left), never separates equal
+    values, never beats the brute-force optimum, finds it on two well-separated
+    groups, is a pure function of (values, seed), and different seeds reach
+    different local optima on some inputs (the seeding is really random)."""
+    rng = random.Random(31)
+    differ = 0
+    for case in range(600):
+        n = rng.randint(2, 11)
+        t = sorted(rng.choice([rng.randint(0, 6), rng.randint(0, 60), rng.randint(0, 600)]) for _ in range(n))
+        k, c1, c2, it = O.kmpp_cut(t, case)
+        assert O.kmpp_cut(t, case) == (k, c1, c2, it)
+        if t[0] == t[-1]:
+            assert k == 0
+            continue
+        assert 1 <= k < n and t[k - 1] < t[k] and it >= 1 and c1 != c2 and c1 in t and c2 in t
+        m1, m2 = Fraction(sum(t[:k]), k), Fraction(sum(t[k:]), n - k)
+        assert all(2 * x <= m1 + m2 for x in t[:k]) and all(2 * x > m1 + m2 for x in t[k:])
+        best = min(_sse(t[:j]) + _sse(t[j:]) for j in range(1, n))
+        assert _sse(t[:k]) + _sse(t[k:]) >= best
+        differ += len({O.kmpp_cut(t, s)[0] for s in range(40)}) > 1
+    assert differ > 0
+    for _ in range(50):
+        a = [rng.randint(0, 50) for _ in range(rng.randint(1, 8))]
+        b = [10_000 + rng.randint(0, 50) for _ in range(rng.randint(1, 8))]
+        tt = sorted(a + b)
+        assert O.kmpp_cut(tt, rng.getrandbits(64))[0] == len(a) == O.best_cut(tt)
+
+
+def test_kmpp_plan_option():
+    """or_opts.split = 2 builds a valid partition, depends on the seed only
+    through the split, and the oracle rejects split = 3"""
+    rng = np.random.default_rng(4)
+    kid = rng.integers(0, 5, 4000).astype(np.uint32)
+    t = (rng.lognormal(8, 0.6, 4000) + 1000 * (rng.random(4000) < 0.3)).astype(np.uint32)
+    p = O.plan(kid, t, 5, eps=0.03, z=Z95, seed=1, split=2)
+    assert int(np.sum(p["n"])) == 4000
+    assert O.plan(kid, t, 5, eps=0.03, z=Z95, seed=1, split=2)["n"].tolist() == p["n"].tolist()
+    with pytest.raises(Exception):
+        O.plan(kid, t, 5, eps=0.03, z=Z95, seed=1, split=3)
+
+
 def test_split_exact_tie(golden):
     for c in golden("split_tie.json")["cases"]:
         t = [c["s"] * x for x in c["base"]]
