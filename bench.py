@@ -49,7 +49,7 @@ def parse():
     ap.add_argument("--ref-sample-rows", type=int, default=8_000_000)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--split", type=int, default=0, help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26)")
+    ap.add_argument("--split", type=int, default=0, help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26), 2 k-means++ seeded Lloyd (R27)")
     return ap.parse_args()
 
 
@@ -261,7 +261,8 @@ def run_ours(a):
         "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded, on device)",
         "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n,
                    "kernels": sp.n_kernels, "eps": eps, "conf": a.conf, "metrics": nm,
-                   "split": "exact optimal 2-means (R5)" if a.split == 0 else "Lloyd k-means, k = 2 (R26)",
+                   "split": ["exact optimal 2-means (R5)", "Lloyd k-means, k = 2 (R26)",
+                             "k-means++ seeded Lloyd, k = 2 (R27)"][a.split],
                    "parallelism": "single GPU" if world == 1 else
                    f"{world} GPUs: row shards, NCCL all-to-all by kernel id, exact allreduce",
                    "l2": "inputs 8 B/row x rows >> 126 MB L2 (no flush needed)" if n_local >= 50_000_000

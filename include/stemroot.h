@@ -42,7 +42,7 @@
 extern "C" {
 #endif
 
-#define STEMROOT_ABI_VERSION 2   /* 2: stem_opts.split */
+#define STEMROOT_ABI_VERSION 3   /* 2: stem_opts.split; 3: split = 2 (k-means++ seeds) */
 
 #if defined(__GNUC__)
 #define STEM_API __attribute__((visibility("default")))
@@ -86,7 +86,10 @@ typedef struct stem_opts {
     int      split;          /* ROOT's sub-clustering ("a clustering method (e.g.,
                                 k-means)", P:L258 k = 2): 0 (default) the exact optimal 2-means
                                 cut (R5); 1 Lloyd's k-means, k = 2, from the (min, max)
-                                centroids to its fixed point (R26); other values: STEM_E_INVAL   */
+                                centroids to its fixed point (R26); 2 the same Lloyd iteration
+                                from k-means++ seeds (uniform c1, D^2-weighted c2) drawn with
+                                Philox4x32-10 keyed by seed on (min t, max t, n) (R27), so the
+                                tree depends on seed; other values: STEM_E_INVAL                 */
     void    *stream;         /* cudaStream_t to run on; NULL = the legacy default stream         */
 } stem_opts;
 

@@ -115,7 +115,7 @@ static int validate(const stem_trace *tr, double eps, double conf, const stem_op
     if (!(o.z > 0.0) && !(conf > 0.0 && conf < 1.0)) return STEM_E_INVAL;
     if (o.z < 0.0 || std::isnan(o.z) || std::isinf(o.z)) return STEM_E_INVAL;
     if (o.scope < 0 || o.scope > 2) return STEM_E_INVAL;
-    if (o.split < 0 || o.split > 1) return STEM_E_INVAL;
+    if (o.split < 0 || o.split > 2) return STEM_E_INVAL;
     if (tr->n == 0 || !tr->kernel_id || !tr->exec_ns) return STEM_E_INVAL;
     if (tr->n_metrics > 64 || (tr->n_metrics > 0 && !tr->metrics)) return STEM_E_INVAL;
     if (tr->n >= (1ull << 32)) return STEM_E_RANGE;
@@ -160,7 +160,7 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
     CKS(sort_trace(c, kid, t, nullptr, n, K, !o.census_cap));   // a1
     CKS(prefix_moments(c, n));                        // a2
     if (o.root) {
-        CKS(root_levels(c, n, K, eps, z, k2, o.clamp_in_split ? 1 : 0, o.split));   // a3, a4
+        CKS(root_levels(c, n, K, eps, z, k2, o.clamp_in_split ? 1 : 0, o.split, o.seed));   // a3, a4
     } else {
         CKS(stem_only_leaves(c, n, K));
     }
@@ -302,7 +302,7 @@ int stem_root_plan_dist(stem_ctx *ctx, stem_comm *comm, const stem_trace *local_
     const stem_trace *tr = local_shard;
     // validation identical on every rank (a local shard may be empty)
     if (!(eps > 0.0 && eps < 1.0) || (!(o.z > 0.0) && !(conf > 0.0 && conf < 1.0)) || o.z < 0.0 ||
-        std::isnan(o.z) || std::isinf(o.z) || o.scope < 0 || o.scope > 2 || o.split < 0 || o.split > 1 ||
+        std::isnan(o.z) || std::isinf(o.z) || o.scope < 0 || o.scope > 2 || o.split < 0 || o.split > 2 ||
         tr->n_metrics > 64 ||
         (tr->n && (!tr->kernel_id || !tr->exec_ns)) || (tr->n && tr->n_metrics && !tr->metrics))
         return STEM_E_INVAL;

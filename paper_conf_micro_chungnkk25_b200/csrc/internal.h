@@ -231,7 +231,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
                uint32_t K, bool allow_pack);                                                   // a1
 int prefix_moments(Ctx &c, uint64_t n);                                                        // a2
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp,
-                int split);   // a3, a4 (split: 0 exact 2-means, 1 Lloyd)
+                int split, uint64_t seed);   // a3, a4 (split: 0 exact 2-means, 1 Lloyd, 2 k-means++ Lloyd)
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,
                       uint32_t *tailh);   // pre-pass only

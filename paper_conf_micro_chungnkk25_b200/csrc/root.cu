@@ -622,18 +622,64 @@ __device__ __forceinline__ uint64_t warp_cut_search(const uint32_t *__restrict__
     return a + __popc(m);
 }
 
+// k-means++ seeds (split = 2, reading R27): the D^2 draw of the second seed is
+// the first prefix p of the cluster whose running sum W(p) = sum_{i < p}
+// (t_i - c1)^2 = Q(p) + p c1^2 - 2 c1 S(p) exceeds R; W is monotone in p, so a
+// warp 33-ary search over p in [a, b) with exact prefix moments (PS1/PS2 plus
+// the partial chunk) finds it.  Returns the first failing p (b if none).
+__device__ __forceinline__ uint64_t warp_d2_search(const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
+                                                   const u128 *__restrict__ PS2, uint64_t lo, uint64_t s0, u128 q0,
+                                                   uint32_t c1, u128 R, uint64_t a, uint64_t b) {
+    const int lane = threadIdx.x & 31;
+    const u128 cc = (u128)((uint64_t)c1 * c1);
+    auto ok = [&](uint64_t p) {   // W(p) <= R
+        uint64_t s;
+        u128 q;
+        pref12(PS1, PS2, t, lo + p, s, q);
+        return (q - q0) + cc * p - (u128)(2 * (uint64_t)c1) * (s - s0) <= R;
+    };
+    while (b - a > 32) {
+        const uint64_t p = a + ((uint64_t)(lane + 1) * (b - a)) / 33;
+        const uint32_t m = __ballot_sync(0xffffffffu, ok(p));
+        const int c = __popc(m);
+        const uint64_t pa = __shfl_sync(0xffffffffu, p, c > 0 ? c - 1 : 0), pb = __shfl_sync(0xffffffffu, p, c < 32 ? c : 31);
+        if (c > 0) a = pa + 1;
+        if (c < 32) b = pb;
+    }
+    const uint32_t m = __ballot_sync(0xffffffffu, a + lane < b && ok(a + lane));
+    return a + __popc(m);
+}
+
+template <bool PP>
 __global__ void __launch_bounds__(256) lloyd_split_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
-                                                          const uint64_t *__restrict__ f_S, const uint64_t *ctot,
-                                                          const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
-                                                          uint32_t *__restrict__ cut, uint64_t *__restrict__ cut_SL) {
+                                                          const uint64_t *__restrict__ f_S, const u128 *__restrict__ f_Q,
+                                                          const uint64_t *ctot, const uint32_t *__restrict__ t,
+                                                          const uint64_t *__restrict__ PS1, const u128 *__restrict__ PS2,
+                                                          uint32_t k0, uint32_t k1, uint32_t *__restrict__ cut,
+                                                          uint64_t *__restrict__ cut_SL) {
     const uint32_t C = (uint32_t)(*ctot >> 32);
     const int lane = threadIdx.x & 31;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
         const uint64_t lo = f_lo[c], hi = f_hi[c], n = hi - lo, S = f_S[c];
-        const uint64_t base = pref1(PS1, t, lo);
-        // steps 1-2: centroids (min, max), first assignment 2 t <= min + max
-        uint64_t k = warp_cut_search(t, lo, hi, 2, (u128)t[lo] + t[hi - 1]) - lo;
+        uint64_t base;
+        u128 mid2;
+        if (PP) {   // R27: c1 a uniform row, c2 by D^2 weight (one Philox draw per cluster)
+            const U4 x = philox4x32_10(U4{t[lo], t[hi - 1], (uint32_t)n, 0x4B4D5050u}, k0, k1);
+            const uint64_t j1 = (uint64_t)(((u128)(((uint64_t)x.y << 32) | x.x) * n) >> 64);
+            const uint32_t c1 = t[lo + j1];
+            const u128 W = (f_Q[c] + (u128)((uint64_t)c1 * c1) * n) - (u128)(2 * (uint64_t)c1) * S;
+            const u128 R = (W * x.z) >> 32;
+            u128 q0;
+            pref12(PS1, PS2, t, lo, base, q0);
+            const uint64_t j2 = warp_d2_search(t, PS1, PS2, lo, base, q0, c1, R, 1, n + 1) - 1;
+            mid2 = (u128)c1 + t[lo + j2];
+        } else {    // R26: centroids (min, max)
+            base = pref1(PS1, t, lo);
+            mid2 = (u128)t[lo] + t[hi - 1];
+        }
+        // first assignment 2 t <= c1 + c2
+        uint64_t k = warp_cut_search(t, lo, hi, 2, mid2) - lo;
         uint64_t S1 = 0;
         for (uint32_t it = 1;; it++) {
             S1 = pref1(PS1, t, lo + k) - base;   // step 3: exact centroid sums
@@ -1212,7 +1258,8 @@ static int ensure_frontier(Ctx &c, int b, uint64_t cap) {
     return STEM_OK;
 }
 
-int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, int split) {
+int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, int split,
+                uint64_t seed) {
     cudaStream_t st = c.stream;
     {
         const uint64_t b = big_rows();
@@ -1294,9 +1341,15 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         if (tk_l >= 0) c.stage_end(tk_l, 4 * Aub);
         CK(cudaGetLastError());
         const int tk_s = c.stage_begin("root_split");
-        if (split == 1) {   // Lloyd variant: one warp per cluster, every size
-            lloyd_split_kernel<<<(unsigned)min((Cub + 7) / 8, (uint64_t)c.sms * 16), 256, 0, st>>>(
-                c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.cut, c.cut_SL);
+        if (split != 0) {   // Lloyd variants: one warp per cluster, every size
+            const unsigned g = (unsigned)min((Cub + 7) / 8, (uint64_t)c.sms * 16);
+            const uint32_t k0 = (uint32_t)seed, k1 = (uint32_t)(seed >> 32);
+            if (split == 2)
+                lloyd_split_kernel<true><<<g, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], ctot,
+                                                            c.t_sorted, c.PS1, c.PS2, k0, k1, c.cut, c.cut_SL);
+            else
+                lloyd_split_kernel<false><<<g, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], ctot,
+                                                             c.t_sorted, c.PS1, c.PS2, k0, k1, c.cut, c.cut_SL);
             c.launches++;
         } else {
         // the small-cluster warps run on a side stream beside the big-cluster

@@ -138,3 +138,14 @@ def test_loopback_lloyd_split(sr):
     ref = O.plan(kid, t, sp.n_kernels, eps=0.04, z=Z95, seed=6, split=1)
     got = _dist_plan(sr, kid, t, sp.n_kernels, 3, eps=0.04, z=Z95, seed=6, split=1)
     assert_plans_equal(got, ref)
+
+
+def test_loopback_kmpp_split(sr):
+    """the k-means++ split variant (opts.split = 2, R27) draws its seeds from the
+    cluster's values only, so the plan is independent of the rank count"""
+    sp = G.spec("C2", n=120_000)
+    kid, t, _ = G.generate_np(sp)
+    ref = O.plan(kid, t, sp.n_kernels, eps=0.04, z=Z95, seed=77, split=2)
+    for world in (2, 3):
+        got = _dist_plan(sr, kid, t, sp.n_kernels, world, eps=0.04, z=Z95, seed=77, split=2)
+        assert_plans_equal(got, ref)

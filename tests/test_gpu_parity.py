@@ -380,14 +380,48 @@ def test_lloyd_split_variant(ctx, case):
         assert len(d["n"]) != len(ref["n"]) or not np.array_equal(d["n"], ref["n"])
 
 
+# ------------------------------------------------------------------ split variant: k-means++ seeded Lloyd (R27)
+@pytest.mark.parametrize("case", ["mixture", "c2", "big", "ties"])
+def test_kmpp_split_variant(ctx, case):
+    """opts.split = 2 (Lloyd's k-means, k = 2, from k-means++ seeds drawn with
+    Philox on (min t, max t, n) keyed by the seed, reading R27): clusters,
+    sizes and sample rows bit-exact against the oracle's step-by-step seeding
+    and Lloyd iteration, for two seeds (the trees differ between them)."""
+    rng = np.random.default_rng(6)
+    if case == "mixture":
+        kid, t = _mixture(rng, 150_001, 97, peaks=4, spread=0.3)
+        K = 97
+    elif case == "c2":
+        sp = G.spec("C2", n=300_000)
+        kid, t, _ = G.generate_np(sp)
+        K = sp.n_kernels
+    elif case == "big":
+        t = np.concatenate([rng.lognormal(11, 1.0, 700_000), rng.normal(5e4, 3e3, 400_000).clip(1)]).astype(np.uint32)
+        kid = np.r_[np.zeros(700_000, np.uint32), np.ones(400_000, np.uint32)]
+        K = 2
+    else:
+        kid, t = _dup_heavy(200_003, 7, 3)
+        K = 7
+    refs = []
+    for seed in (9, 0xDEADBEEFCAFEF00D):
+        got, ref = _both(ctx, kid, t, K, eps=0.03, seed=seed, split=2)
+        assert_plans_equal(got, ref)
+        refs.append(ref)
+    if case in ("mixture", "c2"):
+        a, b = refs
+        assert len(a["n"]) != len(b["n"]) or not np.array_equal(a["n"], b["n"])
+
+
 def test_split_option_validation(ctx, sr):
     kid = np.zeros(100, np.uint32)
     t = np.arange(100, dtype=np.uint32)
     with pytest.raises(sr.StemError):
-        ctx.plan(kid, t, 1, split=2)
+        ctx.plan(kid, t, 1, split=3)
+    with pytest.raises(sr.StemError):
+        ctx.plan(kid, t, 1, split=-1)
 
 
-@pytest.mark.parametrize("split", [0, 1])
+@pytest.mark.parametrize("split", [0, 1, 2])
 def test_pipelined_levels_match_synchronous(ctx, monkeypatch, split):
     """the pipelined ROOT level loop (the next level queued before the host sees
     the frontier size) gives the same plan as one host round trip per level"""
