@@ -18,6 +18,8 @@ Methods:
   per-leaf    ROOT on, Eq. 3 per leaf (scope 2)
   lloyd       ROOT with Lloyd's k-means (k = 2) instead of the exact 2-means cut
               (opts.split = 1, R26: the paper's "k-means")
+  kmeans++    the same from k-means++ seeds (opts.split = 2, R27; the tree changes
+              with every sampling seed, like a randomly seeded library k-means)
   random-p    uniform random sampling, each invocation kept with probability p,
               estimate sum(t)/p (the paper's baseline)
 and an eps sweep of stem+root (Fig. 11).
@@ -110,6 +112,7 @@ def run(config="C2", n=None, n_seeds=20, eps_list=(0.03, 0.05, 0.1, 0.25), z=0.0
     res["methods"]["per-kernel"] = plan_quality(ctx, kid, t, sp.n_kernels, t64, total, eps, seeds, scope=1, **kw)
     res["methods"]["per-leaf"] = plan_quality(ctx, kid, t, sp.n_kernels, t64, total, eps, seeds, scope=2, **kw)
     res["methods"]["lloyd"] = plan_quality(ctx, kid, t, sp.n_kernels, t64, total, eps, seeds, split=1, **kw)
+    res["methods"]["kmeans++"] = plan_quality(ctx, kid, t, sp.n_kernels, t64, total, eps, seeds, split=2, **kw)
     for prob in (0.001, 0.1):
         res["methods"][f"random-{prob:g}"] = random_quality(t64, total, prob, seeds)
     for e in eps_list:
