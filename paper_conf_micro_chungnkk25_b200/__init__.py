@@ -55,7 +55,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and os.path.exists(LIB_PATH) and os.path.getmtime(LIB_PATH) >= max(map(os.path.getmtime, deps)):
         return LIB_PATH
     os.makedirs(os.path.dirname(LIB_PATH), exist_ok=True)
-    cmd = ["nvcc"] + NVCC_FLAGS + ["-I", _nccl_include()] + (["-Xptxas", "-v"] if verbose else []) + \
+    extra = os.environ.get("SR_EXTRA_NVCC", "").split()   # A/B builds only (tools/ab_build.sh)
+    cmd = ["nvcc"] + NVCC_FLAGS + extra + ["-I", _nccl_include()] + (["-Xptxas", "-v"] if verbose else []) + \
         ["-o", LIB_PATH] + srcs + ["-ldl"]
     subprocess.check_call(cmd, cwd=_CSRC)
     return LIB_PATH

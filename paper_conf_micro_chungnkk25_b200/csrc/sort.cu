@@ -54,7 +54,13 @@ constexpr int kRB = 8, kR = 1 << kRB;       // byte digits
 constexpr int kHistR = 256;                 // histogram row stride
 constexpr int kBaseShift = 16;              // B[k] is a multiple of 2^16
 constexpr uint64_t kMaxTable = 1ull << 27;  // kid-table entries (512 MB) before binary search
-constexpr int kLB = 4;                      // look-back: predecessor statuses read per round trip
+#ifndef SR_SORT_LB
+#define SR_SORT_LB 4
+#endif
+#ifndef SR_SORT_MINB
+#define SR_SORT_MINB 4
+#endif
+constexpr int kLB = SR_SORT_LB;             // look-back: predecessor statuses read per round trip
 constexpr int kCoarseShift = 24;            // coarse bases: B[k] a multiple of 2^24
 constexpr uint32_t kMaxTailK = 1u << 16;    // coarse bases need a [K][256] tail histogram
 constexpr int kHistT2 = kMaxPasses;         // hist row of t byte 2 (pre-pass)
@@ -283,7 +289,7 @@ struct PassArgs {
 // (thread d < 256 owns digit d), then keys are staged in shared memory in
 // tile-sorted order and written out in digit runs (coalesced).
 template <int NT, int IT, bool FIRST, bool LAST, bool FULL, bool PK, bool S32>
-__global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : 4) : 1) onesweep_kernel(PassArgs a) {   // (FULL = false: one ragged tile; a looser bound avoids a ptxas C7600 failure)
+__global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR_SORT_MINB) : 1) onesweep_kernel(PassArgs a) {   // (FULL = false: one ragged tile; a looser bound avoids a ptxas C7600 failure)
     constexpr int NW = NT / 32, TILE = NT * IT, R = kR;
     static_assert(NT >= R, "one thread per digit");
     static_assert(NT * IT <= 65536, "16-bit ranks");

@@ -202,9 +202,11 @@ def test_config_c3_full_size_with_metrics(ctx):
 
 
 @pytest.mark.slow
-def test_config_c5_full_size_sampled(ctx):
+@pytest.mark.parametrize("split", [0, 1, 2])
+def test_config_c5_full_size_sampled(ctx, split):
     """configs[4] (1e9 rows, 10k kernels) in the launch configuration bench.py times:
-    device-resident trace, default options.  The oracle recomputes the ROOT leaves of
+    device-resident trace, default options (and the two Lloyd split rules, R26/R27,
+    as `bench.py --split` runs them).  The oracle recomputes the ROOT leaves of
     sampled kernels one by one (leaves of a kernel depend only on its rows, P:L176-200);
     global outputs are checked through properties that hold at any size."""
     import torch
@@ -213,7 +215,7 @@ def test_config_c5_full_size_sampled(ctx):
     kid = torch.empty(sp.n, dtype=torch.int32, device="cuda")
     tt = torch.empty(sp.n, dtype=torch.int32, device="cuda")
     G.generate_cuda(ds, kid, tt)
-    p = ctx.plan(kid, tt, sp.n_kernels, eps=sp.eps, z=Z95, seed=12345)
+    p = ctx.plan(kid, tt, sp.n_kernels, eps=sp.eps, z=Z95, seed=12345, split=split)
     cl = p["clusters"]
     # properties: partition, exact total, ordering, bound, samples inside their clusters
     counts = torch.bincount(kid, minlength=sp.n_kernels).cpu().numpy()
@@ -235,7 +237,7 @@ def test_config_c5_full_size_sampled(ctx):
     for k in list(rng.choice(cand, 6, replace=False)) + [int(np.argmin(np.where(counts > 0, counts, 1 << 40)))]:
         sel = torch.nonzero(kid == int(k)).flatten()
         sub_t = (tt[sel].to(torch.int64) & 0xFFFFFFFF).cpu().numpy().astype(np.uint32)
-        ref = O.plan(np.zeros(len(sub_t), np.uint32), sub_t, 1, eps=sp.eps, z=Z95)
+        ref = O.plan(np.zeros(len(sub_t), np.uint32), sub_t, 1, eps=sp.eps, z=Z95, seed=12345, split=split)
         mine = cl[cl["kernel_id"] == k]
         for f in ("ordinal", "lo_ns", "hi_ns", "n", "sum_ns"):
             assert np.array_equal(mine[f].astype(np.int64), ref[f].astype(np.int64)), (k, f)
