@@ -74,10 +74,16 @@ __global__ void __launch_bounds__(kPreThreads, 2) prepass_kernel(const uint32_t 
                                                       uint64_t n, uint32_t K, int smem_kid,
                                                       uint32_t *__restrict__ kid_count, uint32_t *__restrict__ kid_max,
                                                       uint64_t *__restrict__ hist, uint32_t *__restrict__ max_t,
-                                                      uint32_t *__restrict__ err, uint32_t *__restrict__ tailh) {
-    extern __shared__ uint32_t sh[];   // [3][256] byte histograms, then [K] counts, [K] max
-    uint32_t *h0 = sh, *hk = sh + 3 * kR, *hm = hk + (smem_kid ? K : 0);
-    for (int i = threadIdx.x; i < 3 * kR; i += blockDim.x) h0[i] = 0;
+                                                      uint32_t *__restrict__ err, uint32_t *__restrict__ tailh,
+                                                      int nc) {
+    // [nc][3][256] byte histograms (copy = lane mod nc, stride 3*256+1 words so
+    // a bin's copies sit in different banks: equal bytes within a warp collide
+    // on one address nc times less often), then [K] counts, [K] max
+    extern __shared__ uint32_t sh[];
+    constexpr int HS = 3 * kR + 1;
+    uint32_t *hk = sh + nc * HS, *hm = hk + (smem_kid ? K : 0);
+    uint32_t *h0 = sh + (threadIdx.x & (nc - 1)) * HS;
+    for (int i = threadIdx.x; i < nc * HS; i += blockDim.x) sh[i] = 0;
     if (smem_kid)
         for (uint32_t i = threadIdx.x; i < 2 * K; i += blockDim.x) hk[i] = 0;
     __syncthreads();
@@ -128,9 +134,12 @@ __global__ void __launch_bounds__(kPreThreads, 2) prepass_kernel(const uint32_t 
         if (bad) atomicOr(err, 1u);
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < 3 * kR; i += blockDim.x)
-        if (h0[i]) atomicAdd((unsigned long long *)&hist[((i >> kRB) == 2 ? kHistT2 : (i >> kRB)) * kHistR + (i & (kR - 1))],
-                             (unsigned long long)h0[i]);
+    for (int i = threadIdx.x; i < 3 * kR; i += blockDim.x) {
+        uint32_t v = 0;
+        for (int cp = 0; cp < nc; cp++) v += sh[cp * HS + i];
+        if (v) atomicAdd((unsigned long long *)&hist[((i >> kRB) == 2 ? kHistT2 : (i >> kRB)) * kHistR + (i & (kR - 1))],
+                         (unsigned long long)v);
+    }
     if (smem_kid)
         for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
             if (hk[i]) {
@@ -601,15 +610,25 @@ int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n
     CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
     CK(cudaMemsetAsync(c.kid_max, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
     const int smem_kid = (K <= 24000) ? 1 : 0;
-    const size_t sm_bytes = sizeof(uint32_t) * (3 * kR + (smem_kid ? 2 * (size_t)K : 0));
+    constexpr int kMaxNC = 8;
+    auto bytes = [&](int nc) { return sizeof(uint32_t) * (nc * (3 * kR + 1) + (smem_kid ? 2 * (size_t)K : 0)); };
+    // histogram copies (env STEMROOT_PRE_NC, <= 8, capped to keep two blocks per SM).
+    // Default 1: on C5 the pre-pass takes 1.98 / 2.08 / 2.16 ms with 1 / 2 / 4 copies
+    // (the extra shared memory and final reduction cost more than the rarer collisions)
+    int nc = 1;
+    if (const char *e = getenv("STEMROOT_PRE_NC")) nc = atoi(e);
+    nc = nc < 1 ? 1 : nc > kMaxNC ? kMaxNC : nc;
+    while (nc > 1 && ((nc & (nc - 1)) || 2 * (bytes(nc) + 1024) > 200 * 1024)) nc--;
+    const size_t sm_bytes = bytes(nc);
     // once, for the largest request (thread-safe: loopback ranks are host threads)
     static const cudaError_t pre_attr = cudaFuncSetAttribute(
-        prepass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(uint32_t) * (3 * kR + 2 * 24000)));
+        prepass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        (int)(sizeof(uint32_t) * (kMaxNC * (3 * kR + 1) + 2 * 24000)));
     CK(pre_attr);
     int per_sm = (int)((200 * 1024) / (sm_bytes + 1024));
     per_sm = per_sm < 1 ? 1 : per_sm > 2 ? 2 : per_sm;
     prepass_kernel<<<c.sms * per_sm, kPreThreads, sm_bytes, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.kid_max, c.hist,
-                                                          &c.scalars->max_t, &c.scalars->err, tailh);
+                                                          &c.scalars->max_t, &c.scalars->err, tailh, nc);
     c.launches++;
     CK(cudaGetLastError());
     return STEM_OK;
