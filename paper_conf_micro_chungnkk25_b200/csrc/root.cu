@@ -1261,10 +1261,13 @@ static int ensure_frontier(Ctx &c, int b, uint64_t cap) {
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, int split,
                 uint64_t seed) {
     cudaStream_t st = c.stream;
+    // the local subtree kernel implements the exact split only: the Lloyd rules
+    // (split != 0) keep every cluster on the level path
+    const uint64_t loc_rows = split != 0 ? 0 : local_rows();
     {
         const uint64_t b = big_rows();
         CK(cudaMemcpyToSymbolAsync(c_big, &b, sizeof(b), 0, cudaMemcpyHostToDevice, st));
-        const uint64_t l = local_rows() < b ? local_rows() : b;
+        const uint64_t l = loc_rows < b ? loc_rows : b;
         CK(cudaMemcpyToSymbolAsync(c_loc, &l, sizeof(l), 0, cudaMemcpyHostToDevice, st));
         int b2 = 0;
         if (const char *e = getenv("STEMROOT_SPLIT_BOUND")) b2 = atoi(e) ? 1 : 0;
@@ -1311,7 +1314,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
     // always has the next level queued.  The level after the last one runs on an
     // empty frontier (its kernels exit at once).  STEMROOT_LEVEL_SYNC=1, the
     // local-subtree option and STEMROOT_DEBUG_LEVELS use one host round trip per level.
-    const bool pipelined = local_rows() == 0 && !debug_levels() &&
+    const bool pipelined = loc_rows == 0 && !debug_levels() &&
                            !(getenv("STEMROOT_LEVEL_SYNC") && getenv("STEMROOT_LEVEL_SYNC")[0] == '1');
     if (!c.h_lvl) {
         CK(cudaMallocHost((void **)&c.h_lvl, sizeof(uint64_t) * 4));
@@ -1329,8 +1332,8 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CKS(c.ensure(c.cut, c.cap_cut, sizeof(uint32_t) * Cub));
         CKS(c.ensure(c.cut_SL, c.cap_cut_SL, sizeof(uint64_t) * Cub));
         CKS(ensure_frontier(c, nxt, 2 * Cub));   // at most 2 children per cluster
-        const int tk_l = local_rows() > 0 ? c.stage_begin("root_local") : -1;
-        if (local_rows() > 0) {
+        const int tk_l = loc_rows > 0 ? c.stage_begin("root_local") : -1;
+        if (loc_rows > 0) {
             LocalArgs la{c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], (uint32_t)Cub, level - 1, c.PS1, c.PS2,
                          c.t_sorted, c.TB, c.flags, eps, z, k2, clamp, &c.scalars->local_rows, &c.scalars->local_depth,
                          &c.scalars->err};
@@ -1366,7 +1369,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             CK(cudaEventRecord(c.ev_fork, st));
             CK(cudaStreamWaitEvent(c.side, c.ev_fork, 0));
         }
-        if (local_rows() < big_rows()) {
+        if (loc_rows < big_rows()) {
             const uint64_t blocks = (Cub + 7) / 8;
             static int minb = -1;   // STEMROOT_SMALL_MINB: resident blocks per SM the registers are sized for
             if (minb < 0) minb = getenv("STEMROOT_SMALL_MINB") ? atoi(getenv("STEMROOT_SMALL_MINB")) : 4;

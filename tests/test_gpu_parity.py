@@ -447,3 +447,35 @@ def test_sort_status_widths(ctx, monkeypatch, s32):
     kid, t = _mixture(rng, 400_009, 123, peaks=3, spread=0.3)
     got, ref = _both(ctx, kid, t, 123, eps=0.03, seed=12)
     assert_plans_equal(got, ref)
+
+
+def test_local_subtree_path_all_split_rules(tmp_path):
+    """STEMROOT_LOCAL_ROWS (the optional local subtree kernel, exact split only;
+    read once per process, hence the subprocess) gives the oracle's plan with
+    every split rule: the Lloyd rules keep all clusters on the level path."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    root = os.path.dirname(here)
+    script = tmp_path / "local.py"
+    script.write_text(f"""
+import sys
+sys.path[:0] = [{root!r}, {here!r}]
+import numpy as np, torch
+import oracle as O, tracegen as G
+import paper_conf_micro_chungnkk25_b200 as sr
+from parity_util import Z95, assert_plans_equal
+sp = G.spec("C2", n=200_000)
+kid, t, _ = G.generate_np(sp)
+ctx = sr.Context(0)
+for split in (0, 1, 2):
+    got = ctx.plan(torch.from_numpy(kid.view(np.int32)).cuda(), torch.from_numpy(t.view(np.int32)).cuda(),
+                   sp.n_kernels, eps=0.03, z=Z95, seed=5, split=split)
+    ref = O.plan(kid, t, sp.n_kernels, eps=0.03, z=Z95, seed=5, split=split)
+    assert_plans_equal(got, ref)
+print("ok")
+""")
+    env = dict(os.environ, STEMROOT_LOCAL_ROWS="1024")
+    out = subprocess.run([sys.executable, str(script)], env=env, capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0 and out.stdout.strip().endswith("ok"), out.stdout[-2000:] + out.stderr[-2000:]
