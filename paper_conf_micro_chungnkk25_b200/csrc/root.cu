@@ -36,7 +36,10 @@ static uint64_t big_rows() {
     }
     return v;
 }
-constexpr uint64_t kBigSeg = 65536;                    // rows per block on the big-cluster path
+#ifndef SR_BIG_SEG
+#define SR_BIG_SEG 65536
+#endif
+constexpr uint64_t kBigSeg = SR_BIG_SEG;               // rows per block on the big-cluster path
 // clusters of < local_rows() rows are finished by local_root_kernel
 // (STEMROOT_LOCAL_ROWS, default 0 = off: measured slower than the level loop
 // on C5)
@@ -790,7 +793,10 @@ constexpr int kBigRounds = (kBigChunks + kBigThreads - 1) / kBigThreads;
 constexpr size_t kBigSmem = (size_t)kBigChunks * (sizeof(double) + sizeof(uint64_t) + sizeof(uint2) + sizeof(float) +
                                                   sizeof(uint16_t));
 
-__global__ void __launch_bounds__(kBigThreads, 3) big_split_kernel(BigArgs a) {
+#ifndef SR_BIG_MINB
+#define SR_BIG_MINB 3
+#endif
+__global__ void __launch_bounds__(kBigThreads, SR_BIG_MINB) big_split_kernel(BigArgs a) {
     extern __shared__ __align__(16) unsigned char s_big[];   // kBigSmem bytes
     double *s_ub = reinterpret_cast<double *>(s_big);          // d2: the squared |D| bound of the chunk
     uint64_t *s_sl = reinterpret_cast<uint64_t *>(s_ub + kBigChunks);   // PS1 at the chunk start, then S_L
