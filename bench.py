@@ -49,7 +49,7 @@ def parse():
     ap.add_argument("--ref-sample-rows", type=int, default=8_000_000)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--split", type=int, default=0, help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26), 2 k-means++ seeded Lloyd (R27)")
+    ap.add_argument("--split", type=int, default=0, choices=[0, 1, 2], help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26), 2 k-means++ seeded Lloyd (R27)")
     return ap.parse_args()
 
 
@@ -117,6 +117,9 @@ def dist_env():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
 
+SPLIT_NAMES = ["exact optimal 2-means (R5)", "Lloyd k-means, k = 2 (R26)", "k-means++ seeded Lloyd, k = 2 (R27)"]
+
+
 def run_reference(a):
     """--impl reference: the oracle (plain single-threaded C, oracle/) as it stands, on the
     host cores, on a bounded sample of the same workload; rank 0 only."""
@@ -135,7 +138,7 @@ def run_reference(a):
     times = []
     for i in range(a.warmup + a.steps):
         t0 = time.perf_counter()
-        oracle.plan(kid, t, sp.n_kernels, eps=eps, z=z, seed=i, metrics=met)
+        oracle.plan(kid, t, sp.n_kernels, eps=eps, z=z, seed=i, metrics=met, split=a.split)
         dt = time.perf_counter() - t0
         if i >= a.warmup:
             times.append(dt)
@@ -147,7 +150,7 @@ def run_reference(a):
         "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded)",
         "impl": "reference",
         "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n, "kernels": sp.n_kernels,
-                   "eps": eps, "conf": a.conf, "sample_rows": m},
+                   "eps": eps, "conf": a.conf, "split": SPLIT_NAMES[a.split], "sample_rows": m},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
                          "sample": f"first {m} rows of {a.config} (oracle single-threaded C, -O2)"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -261,8 +264,7 @@ def run_ours(a):
         "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded, on device)",
         "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n,
                    "kernels": sp.n_kernels, "eps": eps, "conf": a.conf, "metrics": nm,
-                   "split": ["exact optimal 2-means (R5)", "Lloyd k-means, k = 2 (R26)",
-                             "k-means++ seeded Lloyd, k = 2 (R27)"][a.split],
+                   "split": SPLIT_NAMES[a.split],
                    "parallelism": "single GPU" if world == 1 else
                    f"{world} GPUs: row shards, NCCL all-to-all by kernel id, exact allreduce",
                    "l2": "inputs 8 B/row x rows >> 126 MB L2 (no flush needed)" if n_local >= 50_000_000
@@ -325,7 +327,7 @@ def run_ours(a):
         t_np = tt[:m].cpu().numpy().view(np.uint32)
         m_np = met[:, :m].cpu().numpy() if nm else None
         t0 = time.perf_counter()
-        oracle.plan(k_np, t_np, sp.n_kernels, eps=eps, z=dplan["z"], seed=12345, metrics=m_np)
+        oracle.plan(k_np, t_np, sp.n_kernels, eps=eps, z=dplan["z"], seed=12345, metrics=m_np, split=a.split)
         cs = time.perf_counter() - t0
         line["cpu_baseline"] = {"value": m / cs, "unit": UNIT, "cores": 1, "kind": "oracle",
                                 "sample": f"first {m} rows of {a.config} ({cs:.1f} s, single-threaded C oracle)",

@@ -20,3 +20,12 @@ def test_reference_arm_json_line():
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
     assert "workload" in d["config"]
+
+
+def test_reference_arm_split_rule():
+    """--split reaches the reference arm: the oracle runs the same split rule (R26/R27)"""
+    out = subprocess.check_output([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--config",
+                                   "C1", "--steps", "1", "--warmup", "0", "--ref-sample-rows", "10000", "--split", "2"],
+                                  cwd=ROOT, timeout=300).decode().strip().splitlines()
+    d = json.loads(out[-1])
+    assert d["config"]["split"].startswith("k-means++") and d["value"] > 0
