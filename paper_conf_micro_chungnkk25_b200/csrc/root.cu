@@ -626,31 +626,58 @@ __device__ __forceinline__ uint64_t warp_cut_search(const uint32_t *__restrict__
 }
 
 // k-means++ seeds (split = 2, reading R27): the D^2 draw of the second seed is
-// the first prefix p of the cluster whose running sum W(p) = sum_{i < p}
-// (t_i - c1)^2 = Q(p) + p c1^2 - 2 c1 S(p) exceeds R; W is monotone in p, so a
-// warp 33-ary search over p in [a, b) with exact prefix moments (PS1/PS2 plus
-// the partial chunk) finds it.  Returns the first failing p (b if none).
+// the first row r of the cluster whose running sum W(r + 1 - lo), W(p) =
+// sum_{i < p} (t_i - c1)^2 = Q(p) + p c1^2 - 2 c1 S(p), exceeds R.  W is
+// monotone, so a warp 33-ary search over the 32-row chunk boundaries inside the
+// cluster (exact W from PS1/PS2 alone, two loads per probe) finds the chunk
+// holding r, and one warp scan of that chunk's (t - c1)^2 finds r.  Returns r
+// relative to lo.
 __device__ __forceinline__ uint64_t warp_d2_search(const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
-                                                   const u128 *__restrict__ PS2, uint64_t lo, uint64_t s0, u128 q0,
-                                                   uint32_t c1, u128 R, uint64_t a, uint64_t b) {
+                                                   const u128 *__restrict__ PS2, uint64_t lo, uint64_t hi,
+                                                   uint64_t s0, u128 q0, uint32_t c1, u128 R) {
     const int lane = threadIdx.x & 31;
     const u128 cc = (u128)((uint64_t)c1 * c1);
-    auto ok = [&](uint64_t p) {   // W(p) <= R
-        uint64_t s;
-        u128 q;
-        pref12(PS1, PS2, t, lo + p, s, q);
-        return (q - q0) + cc * p - (u128)(2 * (uint64_t)c1) * (s - s0) <= R;
+    const u128 c2x = (u128)(2 * (uint64_t)c1);
+    auto W_at = [&](uint64_t j) {   // W at the chunk boundary 32 j (lo < 32 j <= hi)
+        return (PS2[j] - q0) + cc * ((j << kChunkLog) - lo) - c2x * (PS1[j] - s0);
     };
+    // boundaries 32 j with lo < 32 j <= hi: j in [jlo, jhi]; first j with W > R
+    const uint64_t jlo = (lo >> kChunkLog) + 1, jhi = hi >> kChunkLog;
+    uint64_t a = jlo, b = jhi + 1;
     while (b - a > 32) {
         const uint64_t p = a + ((uint64_t)(lane + 1) * (b - a)) / 33;
-        const uint32_t m = __ballot_sync(0xffffffffu, ok(p));
+        const uint32_t m = __ballot_sync(0xffffffffu, W_at(p) <= R);
         const int c = __popc(m);
         const uint64_t pa = __shfl_sync(0xffffffffu, p, c > 0 ? c - 1 : 0), pb = __shfl_sync(0xffffffffu, p, c < 32 ? c : 31);
         if (c > 0) a = pa + 1;
         if (c < 32) b = pb;
     }
-    const uint32_t m = __ballot_sync(0xffffffffu, a + lane < b && ok(a + lane));
-    return a + __popc(m);
+    const uint32_t m = __ballot_sync(0xffffffffu, a + lane < b && W_at(a + lane) <= R);
+    const uint64_t jf = a + __popc(m);
+    // r lies in the rows [ra, rb) between the last boundary at or below R and the first above it
+    const uint64_t ra = jf > jlo ? (jf - 1) << kChunkLog : lo, rb = jf <= jhi ? jf << kChunkLog : hi;
+    const u128 Wa = jf > jlo ? W_at(jf - 1) : (u128)0;
+    const uint64_t row = ra + lane;
+    const bool in = row < rb;
+    uint64_t d = 0;
+    if (in) {
+        const uint32_t x = t[row];
+        d = x > c1 ? (uint64_t)(x - c1) : (uint64_t)(c1 - x);
+    }
+    // inclusive warp scan of d^2 (< 2^64 each) in 128 bits
+    uint64_t slo = d * d, shi = 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t vlo = __shfl_up_sync(0xffffffffu, slo, o), vhi = __shfl_up_sync(0xffffffffu, shi, o);
+        if (lane >= o) {
+            const uint64_t nlo = slo + vlo;
+            shi += vhi + (nlo < slo ? 1 : 0);
+            slo = nlo;
+        }
+    }
+    const u128 run = Wa + (((u128)shi << 64) | slo);
+    const uint32_t over = __ballot_sync(0xffffffffu, in && run > R);
+    return ra + (uint64_t)(__ffs(over) - 1) - lo;
 }
 
 template <bool PP>
@@ -675,7 +702,7 @@ __global__ void __launch_bounds__(256) lloyd_split_kernel(const uint32_t *__rest
             const u128 R = (W * x.z) >> 32;
             u128 q0;
             pref12(PS1, PS2, t, lo, base, q0);
-            const uint64_t j2 = warp_d2_search(t, PS1, PS2, lo, base, q0, c1, R, 1, n + 1) - 1;
+            const uint64_t j2 = warp_d2_search(t, PS1, PS2, lo, hi, base, q0, c1, R);
             mid2 = (u128)c1 + t[lo + j2];
         } else {    // R26: centroids (min, max)
             base = pref1(PS1, t, lo);
