@@ -464,3 +464,88 @@ def test_monte_carlo_unbiased_and_coverage():
     errs = np.array(errs)
     assert abs(errs.mean()) < 4 * errs.std() / math.sqrt(R)
     assert 0.89 <= cover / R <= 0.995
+
+
+# ----------------------------------------------------------------- leaf statistics (R3)
+def test_std_ns_population_hand_vectors(golden):
+    """std_ns is the population sigma of the leaf (reading R3), pinned by
+    hand vectors (tests/golden/std_hand.json), not by the oracle's own formula."""
+    g = golden("std_hand.json")
+    kid, t = [], []
+    for k, kern in enumerate(g["kernels"]):
+        kid += [k] * len(kern["t"])
+        t += kern["t"]
+    p = O.plan(kid, t, len(g["kernels"]), eps=0.05, z=1.96, root=0)
+    for k, kern in enumerate(g["kernels"]):
+        assert p["mean_ns"][k] == kern["mean_ns"]
+        assert p["std_ns"][k] == pytest.approx(kern["std_ns"], rel=1e-15)
+        assert abs(p["std_ns"][k] - kern["sample_std"]) > 1.0   # not the n-1 form
+
+
+def test_std_ns_against_numpy_on_random_leaves():
+    """Every leaf's (mean_ns, std_ns) equals numpy's mean / std(ddof=0) of the
+    leaf's member times (numpy is independent of the oracle's integer moments)."""
+    rng = np.random.default_rng(59)
+    kid, t = _random_trace(rng, 5000, 6)
+    p = O.plan(kid, t, 6, eps=0.02, z=Z95, seed=1)
+    for i in range(len(p["n"])):
+        mem = t[(kid == p["kernel_id"][i]) & (t >= p["lo_ns"][i]) & (t <= p["hi_ns"][i])].astype(np.float64)
+        assert len(mem) == p["n"][i]
+        assert p["mean_ns"][i] == pytest.approx(mem.mean(), rel=1e-13)
+        assert p["std_ns"][i] == pytest.approx(mem.std(), rel=1e-9, abs=1e-9 * mem.mean())
+
+
+# ----------------------------------------------------------------- metric estimator (R18, P:L371, P:L107)
+def _estimator_cases():
+    for scope in (0, 1, 2):
+        for root in (0, 1):
+            for seed in (0, 5, 0xDEADBEEF):
+                yield scope, root, seed
+
+
+def _hash_metric(rows):
+    x = rows.astype(np.uint64) * np.uint64(0x9E3779B97F4A7C15)
+    x ^= x >> np.uint64(29)
+    return (x % np.uint64(1_000_003)).astype(np.float64) / 7.0
+
+
+def test_metric_estimator_weighted_sum_invariants():
+    """The metric estimate is the weighted sum sum_i (n_i/m_i) sum_j metric[row_ij]
+    (P:L371 'weighted sum', P:L107 weights; reading R18), pinned outside census
+    mode (m_i > 1, samples with replacement) by three facts that a plausible
+    mistake breaks:
+      * a constant-1 column estimates N exactly (up to rounding): a swapped
+        weight m_i/n_i gives sum m_i^2/n_i instead;
+      * a column equal to t estimates est_total_ns: gathering metric[sorted
+        position] instead of metric[trace row] reads other rows' values;
+      * a column f(row) (a hash of the trace row) equals sum_s w_s f(row_s)
+        over the plan's own sample rows and weights."""
+    rng = np.random.default_rng(61)
+    kid, t = _random_trace(rng, 6000, 5)
+    rows = np.arange(len(t))
+    met = np.vstack([np.ones(len(t)), t.astype(np.float64), _hash_metric(rows)])
+    multi = 0
+    for scope, root, seed in _estimator_cases():
+        p = O.plan(kid, t, 5, eps=0.01, z=Z95, seed=seed, scope=scope, root=root, metrics=met)
+        assert not p["census"].any()
+        multi += int((p["m"] > 1).sum())
+        assert p["est_metric"][0] == pytest.approx(len(t), rel=1e-12)
+        assert p["est_metric"][1] == pytest.approx(p["est_total_ns"], rel=1e-12)
+        direct = float(np.sum(p["sample_weight"] * _hash_metric(p["sample_row"])))
+        assert p["est_metric"][2] == pytest.approx(direct, rel=1e-12)
+    assert multi > 100   # the pins run where weights differ from 1
+
+
+# ----------------------------------------------------------------- Lloyd trajectory (R26)
+def test_lloyd_hand_traced_trajectory(golden):
+    """split = 1 (reading R26): hand-traced Lloyd iterations from the (min, max)
+    centroids (tests/golden/lloyd_trace.json, every step written out).  The
+    oracle's cut and number of centroid updates must match the trace; a
+    different initialisation (e.g. the two smallest values, or k-means++)
+    takes a different number of steps or stops elsewhere."""
+    for c in golden("lloyd_trace.json")["cases"]:
+        k, updates = O.lloyd_cut(c["t"])
+        assert (k, updates) == (c["cut"], c["updates"])
+        assert O.best_cut(c["t"]) == c["best_cut"]
+        # the trace's first step starts from (min, max): pin the reading, not just the result
+        assert c["steps"][0][:2] == [str(min(c["t"])), str(max(c["t"]))]
