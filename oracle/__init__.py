@@ -34,7 +34,8 @@ def build(force: bool = False) -> str:
 
 class _Opts(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("z", C.c_double), ("scope", C.c_int), ("root", C.c_int),
-                ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("split", C.c_int)]
+                ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("split", C.c_int),
+                ("metric_bounds", C.c_int)]
 
 
 class _Plan(C.Structure):
@@ -52,6 +53,7 @@ class _Plan(C.Structure):
         ("bound", C.c_double), ("eps", C.c_double), ("z", C.c_double),
         ("n_metrics", C.c_uint32), ("est_metric", C.POINTER(C.c_double)),
         ("ssum", C.c_double), ("max_depth", C.c_uint32),
+        ("true_metric", C.POINTER(C.c_double)), ("bound_metric", C.POINTER(C.c_double)),
     ]
 
 
@@ -82,6 +84,8 @@ def lib():
         _lib.or_root_decide.restype = C.c_int
         _lib.or_exact_sum.argtypes = [dp, C.c_uint64]
         _lib.or_exact_sum.restype = C.c_double
+        _lib.or_exact_sum_signed.argtypes = [dp, C.c_uint64]
+        _lib.or_exact_sum_signed.restype = C.c_double
         _lib.or_u128_to_double.argtypes = [C.c_uint64, C.c_uint64]
         _lib.or_u128_to_double.restype = C.c_double
         _lib.or_z_from_conf.argtypes = [C.c_double]
@@ -104,7 +108,7 @@ class OracleError(RuntimeError):
 
 
 def plan(kernel_id, exec_ns, n_kernels, eps=0.05, z=1.959963984540054, seed=0, scope=0, root=1,
-         clamp_in_split=1, census_cap=0, metrics=None, split=0) -> dict:
+         clamp_in_split=1, census_cap=0, metrics=None, split=0, metric_bounds=0) -> dict:
     """Full sampling plan (§3).  Returns numpy arrays + scalars."""
     kid = _u32(kernel_id)
     t = _u32(exec_ns)
@@ -115,7 +119,7 @@ def plan(kernel_id, exec_ns, n_kernels, eps=0.05, z=1.959963984540054, seed=0, s
         metp = _ptr(met, C.c_double)
     else:
         nm, metp = 0, None
-    o = _Opts(seed, z, scope, root, clamp_in_split, census_cap, split)
+    o = _Opts(seed, z, scope, root, clamp_in_split, census_cap, split, int(metric_bounds))
     out = C.POINTER(_Plan)()
     st = lib().or_plan_build(n, n_kernels, _ptr(kid, C.c_uint32), _ptr(t, C.c_uint32), nm, metp, eps,
                              C.byref(o), C.byref(out))
@@ -137,6 +141,8 @@ def plan(kernel_id, exec_ns, n_kernels, eps=0.05, z=1.959963984540054, seed=0, s
         sample_weight=arr(p.sample_weight, S, np.float64),
         est_total_ns=p.est_total_ns, true_total_ns=int(p.true_total_ns), bound=p.bound, eps=p.eps, z=p.z,
         est_metric=arr(p.est_metric, p.n_metrics, np.float64), ssum=p.ssum, max_depth=int(p.max_depth),
+        true_metric=arr(p.true_metric, p.n_metrics, np.float64) if p.true_metric else None,
+        bound_metric=arr(p.bound_metric, p.n_metrics, np.float64) if p.bound_metric else None,
     )
     lib().or_plan_free(out)
     return res
@@ -196,6 +202,11 @@ def root_decide(t_sorted, eps, z, clamp=1):
 def exact_sum(x) -> float:
     a = np.ascontiguousarray(x, dtype=np.float64)
     return lib().or_exact_sum(_ptr(a, C.c_double), a.shape[0])
+
+
+def exact_sum_signed(x) -> float:
+    a = np.ascontiguousarray(x, dtype=np.float64)
+    return lib().or_exact_sum_signed(_ptr(a, C.c_double), a.shape[0])
 
 
 def u128_to_double(v: int) -> float:

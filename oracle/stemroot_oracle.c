@@ -127,6 +127,41 @@ double or_exact_sum(const double *x, uint64_t n) {
     return r;
 }
 
+/* Signed exact sum: positive and negative terms in two accumulators, the exact
+ * difference |pos - neg| formed digit by digit, rounded once. */
+typedef struct { fixacc pos, neg; } sfixacc;
+
+static void sfix_add(sfixacc *a, double x) {
+    if (x > 0.0) fix_add(&a->pos, x);
+    else if (x < 0.0) fix_add(&a->neg, -x);
+}
+
+static double sfix_round(const sfixacc *a) {
+    int cmp = 0;
+    for (int i = OR_FIX_DIGITS - 1; i >= 0 && !cmp; i--)
+        if (a->pos.d[i] != a->neg.d[i]) cmp = a->pos.d[i] > a->neg.d[i] ? 1 : -1;
+    if (cmp == 0) return 0.0;
+    const fixacc *big = cmp > 0 ? &a->pos : &a->neg, *small = cmp > 0 ? &a->neg : &a->pos;
+    fixacc diff;
+    int64_t borrow = 0;
+    for (int i = 0; i < OR_FIX_DIGITS; i++) {
+        int64_t d = (int64_t)big->d[i] - (int64_t)small->d[i] - borrow;
+        borrow = d < 0;
+        diff.d[i] = (uint32_t)(d + (borrow ? ((int64_t)1 << 32) : 0));
+    }
+    double r = fix_round(&diff);
+    return cmp > 0 ? r : -r;
+}
+
+double or_exact_sum_signed(const double *x, uint64_t n) {
+    sfixacc *acc = calloc(1, sizeof(sfixacc));
+    if (!acc) return NAN;
+    for (uint64_t i = 0; i < n; i++) sfix_add(acc, x[i]);
+    double r = sfix_round(acc);
+    free(acc);
+    return r;
+}
+
 /* ------------------------------------------------------------------------ */
 /* Philox4x32-10 (Random123), used for sampling with replacement    */
 /* ------------------------------------------------------------------------ */
@@ -470,7 +505,7 @@ void or_plan_free(or_plan *p) {
     free(p->kernel_id); free(p->ordinal); free(p->lo_ns); free(p->hi_ns);
     free(p->n); free(p->sum_ns); free(p->m); free(p->mean_ns); free(p->std_ns);
     free(p->census); free(p->sample_row); free(p->sample_cluster); free(p->sample_weight);
-    free(p->est_metric);
+    free(p->est_metric); free(p->true_metric); free(p->bound_metric);
     free(p);
 }
 
@@ -651,6 +686,39 @@ int or_plan_build(uint64_t n, uint32_t n_kernels, const uint32_t *kernel_id,
     p->bound = (T == 0) ? 0.0 : z * sqrt(sum_var) / rn64(T);
     p->eps = eps;
     p->z = z;
+
+    /* Step 6 (metric_bounds, reading R28): the true total of each metric column
+     * and its predicted relative error, Eq. 5 with the metric in place of the
+     * time: bound_c = z sqrt(sum_i V_ic / m_i) / |true_c|,
+     * V_ic = n_i^2 sigma_ic^2 = n_i * sum_j (x_j - xbar_ic)^2 over the leaf's rows
+     * (population variance, R3), xbar_ic = (exact sum_j x_j) / n_i. */
+    if (opts->metric_bounds && n_metrics) {
+        p->true_metric = calloc(n_metrics, 8);
+        p->bound_metric = calloc(n_metrics, 8);
+        sfixacc *acc = malloc(sizeof(sfixacc));
+        if (!p->true_metric || !p->bound_metric || !acc) { free(acc); status = OR_E_NOMEM; goto fail_leaves; }
+        for (uint32_t c = 0; c < n_metrics; c++) {
+            const double *col = metrics + (uint64_t)c * n;
+            p->true_metric[c] = or_exact_sum_signed(col, n);
+            double var_c = 0.0;
+            for (uint64_t i = 0; i < L; i++) {
+                leaf lf = leaves.v[i];
+                memset(acc, 0, sizeof(sfixacc));
+                for (uint64_t pos = lf.lo; pos < lf.hi; pos++) sfix_add(acc, col[row_of[pos]]);
+                const double xbar = sfix_round(acc) / rn64(p->n[i]);
+                memset(acc, 0, sizeof(sfixacc));
+                for (uint64_t pos = lf.lo; pos < lf.hi; pos++) {
+                    const double d = col[row_of[pos]] - xbar;
+                    fix_add(&acc->pos, d * d);
+                }
+                const double Vc = rn64(p->n[i]) * fix_round(&acc->pos);
+                var_c += Vc / rn64(p->m[i]);
+            }
+            const double tc = fabs(p->true_metric[c]);
+            p->bound_metric[c] = tc > 0.0 ? z * sqrt(var_c) / tc : (var_c > 0.0 ? INFINITY : 0.0);
+        }
+        free(acc);
+    }
 
     free(V); free(mu); free(mreal); free(terms);
     free(work.v); free(leaves.v); free(rows); free(t); free(row_of);

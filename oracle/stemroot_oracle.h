@@ -30,6 +30,7 @@ typedef struct {
     int      split;          /* 0: exact optimal 2-means cut (R5); 1: Lloyd's k-means,
                                 k = 2, from the (min, max) centroids (R26); 2: the
                                 same from k-means++ seeds drawn with seed (R27)     */
+    int      metric_bounds;  /* 1: also true_metric and bound_metric (reading R28)   */
 } or_opts;
 
 /* Structure-of-arrays plan.  Everything is malloc'ed; free with or_plan_free. */
@@ -49,6 +50,8 @@ typedef struct {
     double   *est_metric;        /* [n_metrics]                              */
     double    ssum;              /* RN(exact sum sqrt(mu_i V_i)), global     */
     uint32_t  max_depth;         /* deepest ROOT level reached (root = 0)    */
+    double   *true_metric;       /* [n_metrics] exact column sums (metric_bounds), else NULL */
+    double   *bound_metric;      /* [n_metrics] predicted relative error (R28), else NULL   */
 } or_plan;
 
 /* Whole plan (§3, Fig. 5).  kernel_id/exec_ns: [n];
@@ -85,6 +88,8 @@ int  or_root_decide(const uint32_t *t_sorted, uint64_t n, double eps, double z, 
                     double *tau_old, double *tau_new, uint64_t *cut);
 /* Exact sum of non-negative doubles, rounded once to nearest. */
 double or_exact_sum(const double *x, uint64_t n);
+/* Exact sum of finite doubles of either sign, rounded once to nearest. */
+double or_exact_sum_signed(const double *x, uint64_t n);
 /* Correctly rounded u128 -> double. */
 double or_u128_to_double(uint64_t lo, uint64_t hi);
 /* Inverse standard normal (AS241 PPND16); z for two-sided confidence conf. */

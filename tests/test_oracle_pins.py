@@ -549,3 +549,80 @@ def test_lloyd_hand_traced_trajectory(golden):
         assert O.best_cut(c["t"]) == c["best_cut"]
         # the trace's first step starts from (min, max): pin the reading, not just the result
         assert c["steps"][0][:2] == [str(min(c["t"])), str(max(c["t"]))]
+
+
+# ----------------------------------------------------------------- metric totals and bounds (R28)
+def test_exact_sum_signed_against_fsum():
+    rng = np.random.default_rng(67)
+    for n in (0, 1, 7, 1000, 20000):
+        x = rng.standard_normal(n) * 10.0 ** rng.integers(-30, 30, n)
+        assert O.exact_sum_signed(x) == math.fsum(x)
+    x = np.array([1e300, 1.0, -1e300, 2.0 ** -1000, -3.0])
+    assert O.exact_sum_signed(x) == math.fsum(x)
+
+
+def test_metric_bounds_invariants():
+    """metric_bounds (reading R28: Eq. 5 with the metric in place of the time,
+    P:L150-159), pinned by what holds whatever the implementation:
+      * true_metric is the column's exact sum (math.fsum, correctly rounded);
+      * a metric equal to t reproduces the time bound (the oracle computes the
+        time variance from exact integer moments and the metric variance by a
+        separate fp64 two-pass, so a dropped n_i, a sample variance or a
+        missing mean subtraction shows up);
+      * an affine metric a t + b has bound |a| bound T / |a T + b N| (a shift
+        leaves the variance alone, a scale multiplies it by a^2);
+      * a constant column has bound 0; the other outputs are unchanged."""
+    rng = np.random.default_rng(71)
+    kid, t = _random_trace(rng, 5000, 5)
+    N = len(t)
+    tf = t.astype(np.float64)
+    met = np.vstack([tf, 3.0 * tf + 1e6, -0.5 * tf, np.full(N, 7.25), rng.random(N) - 0.3])
+    for scope, root, seed in [(0, 1, 0), (0, 0, 3), (1, 1, 9), (2, 1, 4), (0, 1, 77)]:
+        p = O.plan(kid, t, 5, eps=0.01, z=Z95, seed=seed, scope=scope, root=root, metrics=met, metric_bounds=1)
+        q = O.plan(kid, t, 5, eps=0.01, z=Z95, seed=seed, scope=scope, root=root, metrics=met)
+        assert q["true_metric"] is None and q["bound_metric"] is None
+        assert np.array_equal(p["m"], q["m"]) and np.array_equal(p["est_metric"], q["est_metric"])
+        for c in range(met.shape[0]):
+            assert p["true_metric"][c] == math.fsum(met[c])
+        T, b = p["true_total_ns"], p["bound"]
+        assert b > 0
+        assert p["bound_metric"][0] == pytest.approx(b, rel=1e-10)
+        assert p["bound_metric"][1] == pytest.approx(3.0 * b * T / (3.0 * T + 1e6 * N), rel=1e-10)
+        assert p["bound_metric"][2] == pytest.approx(b, rel=1e-10)
+        assert p["bound_metric"][3] == 0.0
+        assert p["bound_metric"][4] > 0
+
+
+def test_metric_bounds_census_exact():
+    """census leaves (every row once): each metric estimate equals its true total."""
+    rng = np.random.default_rng(73)
+    kid, t = _random_trace(rng, 1500, 3)
+    met = np.vstack([rng.random(len(t)), t.astype(np.float64) ** 0.5])
+    p = O.plan(kid, t, 3, eps=1e-6, census_cap=1, root=0, metrics=met, metric_bounds=1)
+    assert p["census"].all()
+    for c in range(2):
+        assert p["est_metric"][c] == pytest.approx(p["true_metric"][c], rel=1e-12)
+
+
+@pytest.mark.slow
+def test_metric_bound_monte_carlo_coverage():
+    """bound_c is a z-level confidence bound of the metric estimate's relative
+    error (CLT over the leaves' with-replacement samples): over 300
+    seeds in the m_i > 1 regime the realised error is inside it about 95 % of
+    the time, and the estimate is unbiased."""
+    rng = np.random.default_rng(79)
+    kid, t = _random_trace(rng, 3000, 6)
+    met = np.vstack([t.astype(np.float64) * rng.uniform(0.5, 1.5, len(t)), rng.gamma(2.0, 3.0, len(t))])
+    R = 300
+    cover = np.zeros(2)
+    errs = [[], []]
+    for seed in range(R):
+        p = O.plan(kid, t, 6, eps=0.02, root=0, seed=seed, metrics=met, metric_bounds=1)
+        for c in range(2):
+            e = (p["est_metric"][c] - p["true_metric"][c]) / p["true_metric"][c]
+            errs[c].append(e)
+            cover[c] += abs(e) <= p["bound_metric"][c]
+    for c in range(2):
+        e = np.array(errs[c])
+        assert abs(e.mean()) < 4 * e.std() / math.sqrt(R)
+        assert 0.89 <= cover[c] / R <= 0.995, cover
