@@ -31,7 +31,8 @@
  *    distinct host threads; one stem_ctx must not be used concurrently.
  *  - Reproducibility: the plan is a pure function of (trace bytes, eps, z,
  *    seed, opts): integer outputs and sample rows are bit-identical to the
- *    test oracle; fp64 outputs agree with it to 1e-9 relative.
+ *    test oracle; fp64 outputs agree with it to 1e-9 relative (all of them
+ *    bit-identical run to run except true_metric / bound_metric).
  */
 #ifndef STEMROOT_H
 #define STEMROOT_H
@@ -42,7 +43,8 @@
 extern "C" {
 #endif
 
-#define STEMROOT_ABI_VERSION 3   /* 2: stem_opts.split; 3: split = 2 (k-means++ seeds) */
+#define STEMROOT_ABI_VERSION 4   /* 2: stem_opts.split; 3: split = 2 (k-means++ seeds);
+                                    4: metric_bounds, true_metric, bound_metric */
 
 #if defined(__GNUC__)
 #define STEM_API __attribute__((visibility("default")))
@@ -90,6 +92,10 @@ typedef struct stem_opts {
                                 from k-means++ seeds (uniform c1, D^2-weighted c2) drawn with
                                 Philox4x32-10 keyed by seed on (min t, max t, n) (R27), so the
                                 tree depends on seed; other values: STEM_E_INVAL                 */
+    int      metric_bounds;  /* 1: also the exact total and the predicted relative error of each
+                                metric column (Eq. 5 with the metric in place of t, P:L150-159,
+                                P:L371; R28): stem_plan.true_metric / bound_metric.
+                                0 (default): point estimates only, those two pointers are NULL  */
     void    *stream;         /* cudaStream_t to run on; NULL = the legacy default stream         */
 } stem_opts;
 
@@ -120,6 +126,12 @@ typedef struct stem_plan {
     double        eps, z;
     uint32_t      n_metrics;
     double       *est_metric;     /* [n_metrics] weighted-sum estimate of each metric total       */
+    double       *true_metric;    /* [n_metrics] exact column sum (metric_bounds = 1), else NULL  */
+    double       *bound_metric;   /* [n_metrics] z sqrt(sum_i V_ic/m_i)/|true_c| with V_ic =
+                                     n_i^2 sigma_ic^2 of the metric over leaf i (R28); 0 for a
+                                     zero-variance column, +inf when true_c = 0 and the variance
+                                     is not (metric_bounds = 1), else NULL.  These two come from
+                                     fp64 atomics: within 1e-12 relative run to run, not bitwise */
 } stem_plan;
 
 /* Device-resident view of the last plan built on a ctx (pointers owned by the
@@ -134,6 +146,8 @@ typedef struct stem_device_plan {
     uint64_t            true_total_ns;
     uint32_t            n_metrics;
     const double       *est_metric;     /* host [n_metrics]                                     */
+    const double       *true_metric;    /* host [n_metrics], NULL unless metric_bounds          */
+    const double       *bound_metric;   /* host [n_metrics], NULL unless metric_bounds          */
 } stem_device_plan;
 
 /* Counters of the last plan built on a ctx (for benchmarks and tests). */
@@ -166,7 +180,7 @@ typedef struct stem_stage_time {
 typedef struct stem_ctx stem_ctx;
 
 /* Fill *o with the defaults: seed 0, z 0, scope 0, root 1, clamp_in_split 1,
- * census_cap 0, stream NULL. */
+ * census_cap 0, split 0, metric_bounds 0, stream NULL. */
 STEM_API int stem_default_opts(stem_opts *o);
 
 /* A workspace bound to one CUDA device; keeps device scratch between calls. */

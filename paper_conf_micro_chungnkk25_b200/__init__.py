@@ -10,8 +10,10 @@ cannot find a GPU, every call raises.
     plan = ctx.plan(kernel_id, exec_ns, n_kernels, eps=0.05, conf=0.95)
 
 ``kernel_id`` / ``exec_ns`` are uint32 data either as CUDA tensors (int32 or
-uint32 dtype, bytes reinterpreted) on the context's device, or as host numpy
-arrays (then the library copies them in).  PAPER.md citations: see
+uint32 dtype, bytes reinterpreted; other dtypes raise TypeError) on the
+context's device, or as host arrays (4-byte integers viewed, other integer
+arrays range-checked and converted; the library copies them in).  ``metrics``
+is float64, shape (n_metrics, n) or (n,).  PAPER.md citations: see
 include/stemroot.h.
 """
 from __future__ import annotations
@@ -27,7 +29,7 @@ _ROOT = os.path.dirname(_HERE)
 _CSRC = os.path.join(_HERE, "csrc")
 LIB_PATH = os.path.join(_HERE, "lib", "libstemroot.so")
 HEADER = os.path.join(_ROOT, "include", "stemroot.h")
-SOURCES = ["capi.cu", "sort.cu", "root.cu", "stem.cu", "dist.cu"]
+SOURCES = ["capi.cu", "sort.cu", "root.cu", "stem.cu", "dist.cu", "metric.cu"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "--fmad=false",
               "--extended-lambda", "-Xcompiler", "-fPIC,-fvisibility=hidden", "-shared"]
 
@@ -70,7 +72,8 @@ class stem_trace(C.Structure):
 
 class stem_opts(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("z", C.c_double), ("scope", C.c_int), ("root", C.c_int),
-                ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("split", C.c_int), ("stream", C.c_void_p)]
+                ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("split", C.c_int),
+                ("metric_bounds", C.c_int), ("stream", C.c_void_p)]
 
 
 class stem_cluster(C.Structure):
@@ -90,14 +93,16 @@ class stem_plan(C.Structure):
                 ("sample_row", C.POINTER(C.c_uint32)), ("sample_cluster", C.POINTER(C.c_uint32)),
                 ("sample_weight", C.POINTER(C.c_double)), ("est_total_ns", C.c_double),
                 ("true_total_ns", C.c_uint64), ("bound", C.c_double), ("eps", C.c_double), ("z", C.c_double),
-                ("n_metrics", C.c_uint32), ("est_metric", C.POINTER(C.c_double))]
+                ("n_metrics", C.c_uint32), ("est_metric", C.POINTER(C.c_double)),
+                ("true_metric", C.POINTER(C.c_double)), ("bound_metric", C.POINTER(C.c_double))]
 
 
 class stem_device_plan(C.Structure):
     _fields_ = [("n_clusters", C.c_uint64), ("n_samples", C.c_uint64), ("clusters", C.c_void_p),
                 ("sample_row", C.c_void_p), ("sample_cluster", C.c_void_p), ("sample_weight", C.c_void_p),
                 ("est_total_ns", C.c_double), ("bound", C.c_double), ("eps", C.c_double), ("z", C.c_double),
-                ("true_total_ns", C.c_uint64), ("n_metrics", C.c_uint32), ("est_metric", C.POINTER(C.c_double))]
+                ("true_total_ns", C.c_uint64), ("n_metrics", C.c_uint32), ("est_metric", C.POINTER(C.c_double)),
+                ("true_metric", C.POINTER(C.c_double)), ("bound_metric", C.POINTER(C.c_double))]
 
 
 class stem_stats(C.Structure):
@@ -178,19 +183,74 @@ def z_from_conf(conf: float) -> float:
     return z.value
 
 
-def _arg(x, dtype):
-    """(pointer, device, keepalive) for a torch tensor or numpy array."""
+def _arg(x, kind: str, n: int = -1):
+    """(pointer, device, keepalive, shape) for a torch tensor or numpy array.
+
+    kind "u32": kernel_id / exec_ns -- torch int32/uint32 (bytes reinterpreted
+    as uint32); numpy 4-byte integers are viewed, other integer arrays are
+    converted after a range check; anything else raises.  kind "f64": metrics
+    -- torch float64 only; numpy arrays are converted to float64.  n >= 0
+    checks the trailing dimension (rows)."""
     try:
         import torch
         if isinstance(x, torch.Tensor):
+            ok = {"u32": (torch.int32, getattr(torch, "uint32", torch.int32)), "f64": (torch.float64,)}[kind]
+            if x.dtype not in ok:
+                raise TypeError(f"{'kernel_id/exec_ns' if kind == 'u32' else 'metrics'} tensor must be "
+                                f"{' or '.join(str(d) for d in ok)}, got {x.dtype}")
             if not x.is_contiguous():
                 raise ValueError("tensor must be contiguous")
-            return x.data_ptr(), (x.device.index if x.is_cuda else -1), x
+            if n >= 0 and (x.dim() == 0 or x.shape[-1] != n):
+                raise ValueError(f"expected {n} rows in the last dimension, got shape {tuple(x.shape)}")
+            return x.data_ptr(), (x.device.index if x.is_cuda else -1), x, tuple(x.shape)
     except ImportError:
         pass
-    a = np.ascontiguousarray(x).view(dtype) if np.asarray(x).dtype.itemsize == np.dtype(dtype).itemsize \
-        else np.ascontiguousarray(x, dtype=dtype)
-    return a.ctypes.data, -1, a
+    a = np.asarray(x)
+    if kind == "u32":
+        if a.dtype.kind not in "iu":
+            raise TypeError(f"kernel_id/exec_ns must be integer arrays, got {a.dtype}")
+        if a.dtype.itemsize == 4:
+            a = np.ascontiguousarray(a).view(np.uint32)
+        else:
+            if a.size and (int(a.min()) < 0 or int(a.max()) >= 1 << 32):
+                raise ValueError("kernel_id/exec_ns values must fit in uint32")
+            a = np.ascontiguousarray(a, dtype=np.uint32)
+    else:
+        a = np.ascontiguousarray(a, dtype=np.float64)
+    if n >= 0 and (a.ndim == 0 or a.shape[-1] != n):
+        raise ValueError(f"expected {n} rows in the last dimension, got shape {a.shape}")
+    return a.ctypes.data, -1, a, a.shape
+
+
+def _trace(kernel_id, exec_ns, n_kernels, metrics, allow_empty=False):
+    """stem_trace + keepalives from the user's arrays (argument marshalling only)."""
+    kp, kdev, k_keep, kshape = _arg(kernel_id, "u32")
+    if len(kshape) != 1:
+        raise ValueError("kernel_id must be one-dimensional")
+    n = int(kshape[0])
+    tp, tdev, t_keep, _ = _arg(exec_ns, "u32", n)
+    if kdev != tdev:
+        raise ValueError("kernel_id and exec_ns must live on the same device")
+    nm, mp, m_keep = 0, None, None
+    if metrics is not None:
+        mp, mdev, m_keep, mshape = _arg(metrics, "f64", n)
+        if mdev != kdev:
+            raise ValueError("metrics must live with the trace")
+        if len(mshape) not in (1, 2):
+            raise ValueError("metrics must be (n_metrics, n) or (n,)")
+        nm = int(mshape[0]) if len(mshape) == 2 else 1
+    if n == 0 and allow_empty:
+        kp = tp = mp = None
+    tr = stem_trace(n, n_kernels, kp, tp, nm, mp, kdev)
+    return tr, kdev, (k_keep, t_keep, m_keep)
+
+
+def _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev):
+    if stream is None and dev >= 0:
+        import torch
+        stream = torch.cuda.current_stream(dev).cuda_stream
+    return stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
+                     int(split), int(metric_bounds), stream or None)
 
 
 def _plan_to_numpy(p: stem_plan) -> dict:
@@ -203,7 +263,9 @@ def _plan_to_numpy(p: stem_plan) -> dict:
     return dict(clusters=cl, sample_row=arr(p.sample_row, S, np.uint32),
                 sample_cluster=arr(p.sample_cluster, S, np.uint32), sample_weight=arr(p.sample_weight, S, np.float64),
                 est_total_ns=p.est_total_ns, true_total_ns=int(p.true_total_ns), bound=p.bound, eps=p.eps, z=p.z,
-                est_metric=arr(p.est_metric, p.n_metrics, np.float64))
+                est_metric=arr(p.est_metric, p.n_metrics, np.float64),
+                true_metric=arr(p.true_metric, p.n_metrics, np.float64) if p.true_metric else None,
+                bound_metric=arr(p.bound_metric, p.n_metrics, np.float64) if p.bound_metric else None)
 
 
 def owner_ranges(counts, world: int) -> np.ndarray:
@@ -273,31 +335,17 @@ class Context:
 
     def plan(self, kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, metrics=None,
              seed: int = 0, z: float = 0.0, scope: int = 0, root: bool = True, clamp_in_split: bool = True,
-             census_cap: bool = False, stream=None, to_host: bool = True, split: int = 0):
+             census_cap: bool = False, stream=None, to_host: bool = True, split: int = 0,
+             metric_bounds: bool = False):
         """stem_root_plan_ctx.  Returns the host plan as numpy arrays, or None when to_host=False
         (the plan then stays on the device: see device_plan())."""
-        kp, kdev, k_keep = _arg(kernel_id, np.uint32)
-        tp, tdev, t_keep = _arg(exec_ns, np.uint32)
-        n = int(np.prod(getattr(k_keep, "shape", (0,))))
-        if kdev != tdev:
-            raise ValueError("kernel_id and exec_ns must live on the same device")
-        nm, mp, m_keep = 0, None, None
-        if metrics is not None:
-            mp, mdev, m_keep = _arg(metrics, np.float64)
-            if mdev != kdev:
-                raise ValueError("metrics must live with the trace")
-            nm = int(m_keep.shape[0]) if len(m_keep.shape) == 2 else 1
-        tr = stem_trace(n, n_kernels, kp, tp, nm, mp, kdev)
-        if stream is None and kdev >= 0:
-            import torch
-            stream = torch.cuda.current_stream(kdev).cuda_stream
-        o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
-                      int(split), stream or None)
+        tr, dev, keep = _trace(kernel_id, exec_ns, n_kernels, metrics)
+        o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev)
         out = C.POINTER(stem_plan)()
         st = lib().stem_root_plan_ctx(self._h, C.byref(tr), eps, conf, C.byref(o),
                                       C.byref(out) if to_host else None)
         _check(st, "stem_root_plan_ctx")
-        del k_keep, t_keep, m_keep
+        del keep
         if not to_host:
             return None
         res = _plan_to_numpy(out.contents)
@@ -306,26 +354,16 @@ class Context:
 
     def plan_dist(self, comm: "Comm", kernel_id, exec_ns, n_kernels: int, global_row_base: int, eps: float = 0.05,
                   conf: float = 0.95, metrics=None, seed: int = 0, z: float = 0.0, scope: int = 0, root: bool = True,
-                  clamp_in_split: bool = True, census_cap: bool = False, stream=None, to_host: bool = True, split: int = 0):
+                  clamp_in_split: bool = True, census_cap: bool = False, stream=None, to_host: bool = True,
+                  split: int = 0, metric_bounds: bool = False):
         """stem_root_plan_dist (collective).  Returns the global plan on rank 0, None elsewhere."""
-        kp, kdev, k_keep = _arg(kernel_id, np.uint32)
-        tp, tdev, t_keep = _arg(exec_ns, np.uint32)
-        n = int(np.prod(getattr(k_keep, "shape", (0,))))
-        nm, mp, m_keep = 0, None, None
-        if metrics is not None:
-            mp, _, m_keep = _arg(metrics, np.float64)
-            nm = int(m_keep.shape[0]) if len(m_keep.shape) == 2 else 1
-        if stream is None and kdev >= 0:
-            import torch
-            stream = torch.cuda.current_stream(kdev).cuda_stream
-        tr = stem_trace(n, n_kernels, kp if n else None, tp if n else None, nm, mp if n else None, kdev)
-        o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
-                      int(split), stream or None)
+        tr, dev, keep = _trace(kernel_id, exec_ns, n_kernels, metrics, allow_empty=True)
+        o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev)
         out = C.POINTER(stem_plan)()
         st = lib().stem_root_plan_dist(self._h, comm._h, C.byref(tr), global_row_base, eps, conf, C.byref(o),
                                        C.byref(out) if to_host else None)
         _check(st, "stem_root_plan_dist")
-        del k_keep, t_keep, m_keep
+        del keep
         if not to_host or not out:
             return None
         res = _plan_to_numpy(out.contents)
@@ -338,7 +376,9 @@ class Context:
         return dict(n_clusters=v.n_clusters, n_samples=v.n_samples, clusters=v.clusters, sample_row=v.sample_row,
                     sample_cluster=v.sample_cluster, sample_weight=v.sample_weight, est_total_ns=v.est_total_ns,
                     bound=v.bound, eps=v.eps, z=v.z, true_total_ns=int(v.true_total_ns),
-                    est_metric=[v.est_metric[i] for i in range(v.n_metrics)])
+                    est_metric=[v.est_metric[i] for i in range(v.n_metrics)],
+                    true_metric=[v.true_metric[i] for i in range(v.n_metrics)] if v.true_metric else None,
+                    bound_metric=[v.bound_metric[i] for i in range(v.n_metrics)] if v.bound_metric else None)
 
     def enable_timing(self, on: bool = True):
         _check(lib().stem_ctx_enable_timing(self._h, int(on)), "stem_ctx_enable_timing")
@@ -359,26 +399,13 @@ class Context:
 
 def plan(kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, metrics=None, seed: int = 0,
          z: float = 0.0, scope: int = 0, root: bool = True, clamp_in_split: bool = True, census_cap: bool = False,
-         stream=None, split: int = 0) -> dict:
+         stream=None, split: int = 0, metric_bounds: bool = False) -> dict:
     """stem_root_plan: one-shot plan (temporary workspace), host plan out."""
-    kp, kdev, k_keep = _arg(kernel_id, np.uint32)
-    tp, tdev, t_keep = _arg(exec_ns, np.uint32)
-    if kdev != tdev:
-        raise ValueError("kernel_id and exec_ns must live on the same device")
-    n = int(np.prod(getattr(k_keep, "shape", (0,))))
-    nm, mp, m_keep = 0, None, None
-    if metrics is not None:
-        mp, _, m_keep = _arg(metrics, np.float64)
-        nm = int(m_keep.shape[0]) if len(m_keep.shape) == 2 else 1
-    if stream is None and kdev >= 0:
-        import torch
-        stream = torch.cuda.current_stream(kdev).cuda_stream
-    tr = stem_trace(n, n_kernels, kp, tp, nm, mp, kdev)
-    o = stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
-                  int(split), stream or None)
+    tr, dev, keep = _trace(kernel_id, exec_ns, n_kernels, metrics)
+    o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev)
     out = C.POINTER(stem_plan)()
     _check(lib().stem_root_plan(C.byref(tr), eps, conf, C.byref(o), C.byref(out)), "stem_root_plan")
-    del k_keep, t_keep, m_keep
+    del keep
     res = _plan_to_numpy(out.contents)
     lib().stem_plan_free(out)
     return res

@@ -77,6 +77,10 @@ void Ctx::release() {
     dfree(xfer_f64, cap_xfer_f64); dfree(xfer_f64b, cap_xfer_f64b); dfree(red_part2, cap_red2);
     dfree(g_clusters, cap_g_clusters); dfree(g_row, cap_g_row); dfree(g_cluster, cap_g_cluster);
     dfree(g_weight, cap_g_weight);
+    dfree(mb_first, cap_mb_first); dfree(mb_lo, cap_mb_lo); dfree(mb_gkid, cap_mb_gkid);
+    dfree(mb_leaf_of, cap_mb_leaf_of); dfree(mb_n, cap_mb_n); dfree(mb_gm, cap_mb_gm);
+    dfree(mb_acc, cap_mb_acc); dfree(mb_part, cap_mb_part); dfree(mb_rec, cap_mb_rec);
+    mb_m = nullptr;
 }
 
 // z = Phi^-1(1 - q), q = (1-conf)/2: Acklam's rational initial guess for the
@@ -116,6 +120,7 @@ static int validate(const stem_trace *tr, double eps, double conf, const stem_op
     if (o.z < 0.0 || std::isnan(o.z) || std::isinf(o.z)) return STEM_E_INVAL;
     if (o.scope < 0 || o.scope > 2) return STEM_E_INVAL;
     if (o.split < 0 || o.split > 2) return STEM_E_INVAL;
+    if (o.metric_bounds < 0 || o.metric_bounds > 1) return STEM_E_INVAL;
     if (tr->n == 0 || !tr->kernel_id || !tr->exec_ns) return STEM_E_INVAL;
     if (tr->n_metrics > 64 || (tr->n_metrics > 0 && !tr->metrics)) return STEM_E_INVAL;
     if (tr->n >= (1ull << 32)) return STEM_E_RANGE;
@@ -164,7 +169,7 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
     } else {
         CKS(stem_only_leaves(c, n, K));
     }
-    CKS(leaves_and_plan(c, n, K, met, nm, eps, z, k2, o));   // a5 - a8
+    CKS(leaves_and_plan(c, n, K, met, nm, eps, z, k2, o, kid, t, n));   // a5 - a8
     c.n = n;
     c.K = K;
     c.n_metrics = nm;
@@ -191,7 +196,12 @@ static int to_host(Ctx &c, stem_plan **out) {
     p->sample_weight = (double *)malloc(sizeof(double) * (S ? S : 1));
     p->n_metrics = c.n_metrics;
     p->est_metric = (double *)calloc(c.n_metrics ? c.n_metrics : 1, sizeof(double));
-    if (!p->clusters || !p->sample_row || !p->sample_cluster || !p->sample_weight || !p->est_metric) {
+    if (c.have_mbounds) {
+        p->true_metric = (double *)calloc(c.n_metrics, sizeof(double));
+        p->bound_metric = (double *)calloc(c.n_metrics, sizeof(double));
+    }
+    if (!p->clusters || !p->sample_row || !p->sample_cluster || !p->sample_weight || !p->est_metric ||
+        (c.have_mbounds && (!p->true_metric || !p->bound_metric))) {
         stem_plan_free(p);
         return STEM_E_NOMEM;
     }
@@ -216,6 +226,10 @@ static int to_host(Ctx &c, stem_plan **out) {
     p->eps = c.eps;
     p->z = c.z;
     memcpy(p->est_metric, c.host_est_metric, sizeof(double) * c.n_metrics);
+    if (c.have_mbounds) {
+        memcpy(p->true_metric, c.host_true_metric, sizeof(double) * c.n_metrics);
+        memcpy(p->bound_metric, c.host_bound_metric, sizeof(double) * c.n_metrics);
+    }
     *out = p;
     return STEM_OK;
 }
@@ -240,6 +254,7 @@ int stem_default_opts(stem_opts *o) {
     o->clamp_in_split = 1;
     o->census_cap = 0;
     o->split = 0;
+    o->metric_bounds = 0;
     o->stream = nullptr;
     return STEM_OK;
 }
@@ -291,7 +306,7 @@ int stem_root_plan_dist(stem_ctx *ctx, stem_comm *comm, const stem_trace *local_
                         double eps, double conf, const stem_opts *opts, stem_plan **out) {
     if (out) *out = nullptr;
     sr::Comm *cm = stem_comm_impl(comm);
-    if (!ctx || !cm || !local_shard) return STEM_E_INVAL;
+    if (!ctx || !cm) return STEM_E_INVAL;   // no communicator: nothing to agree with
     stem_opts o;
     if (opts) o = *opts; else stem_default_opts(&o);
     sr::Ctx &c = ctx->c;
@@ -299,27 +314,33 @@ int stem_root_plan_dist(stem_ctx *ctx, stem_comm *comm, const stem_trace *local_
     c.launches = 0;
     c.stats = stem_stats{};
     c.timing.reset();
-    const stem_trace *tr = local_shard;
-    // validation identical on every rank (a local shard may be empty)
-    if (!(eps > 0.0 && eps < 1.0) || (!(o.z > 0.0) && !(conf > 0.0 && conf < 1.0)) || o.z < 0.0 ||
+    static const stem_trace empty{};
+    const stem_trace *tr = local_shard ? local_shard : &empty;
+    // argument checks are rank-local (a shard may be empty or bad on one rank
+    // only): the status is agreed across ranks inside run_plan_dist, so every
+    // rank returns the same error instead of leaving its peers in a collective
+    int local = STEM_OK;
+    if (!local_shard || !(eps > 0.0 && eps < 1.0) || (!(o.z > 0.0) && !(conf > 0.0 && conf < 1.0)) || o.z < 0.0 ||
         std::isnan(o.z) || std::isinf(o.z) || o.scope < 0 || o.scope > 2 || o.split < 0 || o.split > 2 ||
-        tr->n_metrics > 64 ||
+        o.metric_bounds < 0 || o.metric_bounds > 1 || tr->n_metrics > 64 ||
         (tr->n && (!tr->kernel_id || !tr->exec_ns)) || (tr->n && tr->n_metrics && !tr->metrics))
-        return STEM_E_INVAL;
-    if (tr->n >= (1ull << 32)) return STEM_E_RANGE;
-    if (tr->n_kernels == 0 || tr->n_kernels > (1u << 24)) return STEM_E_RANGE;
-    if (cudaSetDevice(c.device) != cudaSuccess) return STEM_E_CUDA;
-    if (tr->device >= 0 && tr->device != c.device) return STEM_E_INVAL;
+        local = STEM_E_INVAL;
+    else if (tr->n >= (1ull << 32) || tr->n_kernels == 0 || tr->n_kernels > (1u << 24))
+        local = STEM_E_RANGE;
+    else if (tr->device >= 0 && tr->device != c.device)
+        local = STEM_E_INVAL;
+    if (cudaSetDevice(c.device) != cudaSuccess) local = STEM_E_CUDA;
     c.stream = (cudaStream_t)o.stream;
     double z = o.z;
-    if (!(z > 0.0)) z = sr::z_two_sided(conf);
+    if (local == STEM_OK && !(z > 0.0)) z = sr::z_two_sided(conf);
     c.z = z;
     c.eps = eps;
     c.comm = cm;
-    int s = sr::run_plan_dist(c, *cm, tr, global_row_base, eps, conf, o);
+    int s = sr::run_plan_dist(c, *cm, tr, global_row_base, eps, conf, o, local);
     c.comm = nullptr;
     c.kid_base = 0;
     if (s != STEM_OK) return s;
+    c.n = tr->n;
     c.n_metrics = tr->n_metrics;
     c.stats.kernel_launches = c.launches;
     if (c.timing.on) {
@@ -359,6 +380,8 @@ int stem_ctx_device_plan(const stem_ctx *ctx, stem_device_plan *v) {
     v->true_total_ns = c.T;
     v->n_metrics = c.n_metrics;
     v->est_metric = c.host_est_metric;
+    v->true_metric = c.have_mbounds ? c.host_true_metric : nullptr;
+    v->bound_metric = c.have_mbounds ? c.host_bound_metric : nullptr;
     return STEM_OK;
 }
 
@@ -396,6 +419,8 @@ void stem_plan_free(stem_plan *p) {
     free(p->sample_cluster);
     free(p->sample_weight);
     free(p->est_metric);
+    free(p->true_metric);
+    free(p->bound_metric);
     free(p);
 }
 

@@ -12,8 +12,11 @@
 // GPU (single-GPU tests of the multi-rank logic).
 #include <dlfcn.h>
 
+#include <chrono>
 #include <condition_variable>
+#include <cstdlib>
 #include <cstring>
+#include <thread>
 #include <memory>
 #include <mutex>
 #include <vector>
@@ -24,10 +27,30 @@
 namespace sr {
 
 // ---------------------------------------------------------------- communicators
+// Seconds a rank waits for its peers (a collective, a barrier) before giving up
+// with STEM_E_NCCL: STEMROOT_COMM_TIMEOUT_S, default 600.
+static double comm_timeout_s() {
+    static double v = -1.0;
+    if (v < 0.0) {
+        const char *e = getenv("STEMROOT_COMM_TIMEOUT_S");
+        v = e ? atof(e) : 600.0;
+        if (!(v > 0.0)) v = 600.0;
+    }
+    return v;
+}
+
 class Comm {
   public:
     int rank = 0, world = 1, device = 0;
+    bool broken = false;   // a peer failed or timed out: every later call returns STEM_E_NCCL
     virtual ~Comm() {}
+    // wait for everything queued on st, collectives included; STEM_E_NCCL on a
+    // communicator error or after comm_timeout_s() (the communicator is then unusable)
+    virtual int wait(cudaStream_t st) {
+        if (broken) return STEM_E_NCCL;
+        CK(cudaStreamSynchronize(st));
+        return STEM_OK;
+    }
     // in-place sum over ranks of a device buffer (u64 or f64)
     virtual int allreduce(void *buf, size_t count, bool f64, cudaStream_t st) = 0;
     // host arrays: all[r * count + i] = rank r's mine[i]
@@ -49,6 +72,8 @@ struct NcclApi {
     ncclResult_t (*recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*groupStart)() = nullptr;
     ncclResult_t (*groupEnd)() = nullptr;
+    ncclResult_t (*getAsyncError)(ncclComm_t, ncclResult_t *) = nullptr;   // optional
+    ncclResult_t (*commAbort)(ncclComm_t) = nullptr;                         // optional
 };
 
 static NcclApi &nccl() {
@@ -66,6 +91,8 @@ static NcclApi &nccl() {
         a.recv = (decltype(a.recv))dlsym(h, "ncclRecv");
         a.groupStart = (decltype(a.groupStart))dlsym(h, "ncclGroupStart");
         a.groupEnd = (decltype(a.groupEnd))dlsym(h, "ncclGroupEnd");
+        a.getAsyncError = (decltype(a.getAsyncError))dlsym(h, "ncclCommGetAsyncError");
+        a.commAbort = (decltype(a.commAbort))dlsym(h, "ncclCommAbort");
         a.ok = a.getUniqueId && a.commInitRank && a.commDestroy && a.allReduce && a.allGather && a.send &&
                a.recv && a.groupStart && a.groupEnd;
         return a;
@@ -73,9 +100,10 @@ static NcclApi &nccl() {
     return api;
 }
 
-#define NK(x)                                      \
-    do {                                           \
-        if ((x) != ncclSuccess) return STEM_E_NCCL; \
+#define NK(x)                                                  \
+    do {                                                       \
+        if (broken) return STEM_E_NCCL;                        \
+        if ((x) != ncclSuccess) { fail(); return STEM_E_NCCL; } \
     } while (0)
 
 class NcclComm : public Comm {
@@ -86,6 +114,39 @@ class NcclComm : public Comm {
     ~NcclComm() override {
         if (comm) nccl().commDestroy(comm);
         if (stage) cudaFree(stage);
+    }
+    void fail() {   // abort the communicator: queued NCCL kernels terminate, later calls fail fast
+        if (comm && nccl().commAbort) nccl().commAbort(comm);
+        else if (comm) nccl().commDestroy(comm);
+        comm = nullptr;
+        broken = true;
+    }
+    // Poll the stream and the communicator's asynchronous error state instead
+    // of blocking in cudaStreamSynchronize: a lost or failed peer turns into
+    // STEM_E_NCCL within comm_timeout_s() instead of a hang.
+    int wait(cudaStream_t st) override {
+        if (broken) return STEM_E_NCCL;
+        const auto t0 = std::chrono::steady_clock::now();
+        for (uint64_t it = 0;; it++) {
+            const cudaError_t e = cudaStreamQuery(st);
+            if (e == cudaSuccess) return STEM_OK;
+            if (e != cudaErrorNotReady) {
+                last_cuda_error() = e;
+                return STEM_E_CUDA;
+            }
+            ncclResult_t ae = ncclSuccess;
+            if (nccl().getAsyncError && nccl().getAsyncError(comm, &ae) == ncclSuccess && ae != ncclSuccess &&
+                ae != ncclInProgress) {
+                fail();
+                return STEM_E_NCCL;
+            }
+            const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+            if (el > comm_timeout_s()) {
+                fail();
+                return STEM_E_NCCL;
+            }
+            if (el > 2e-3) std::this_thread::sleep_for(std::chrono::microseconds(50));
+        }
     }
     int allreduce(void *buf, size_t count, bool f64, cudaStream_t st) override {
         NK(nccl().allReduce(buf, buf, count, f64 ? ncclFloat64 : ncclUint64, ncclSum, comm, st));
@@ -103,8 +164,7 @@ class NcclComm : public Comm {
         CK(cudaMemcpyAsync(send, mine, count * sizeof(uint64_t), cudaMemcpyHostToDevice, st));
         NK(nccl().allGather(send, stage, count, ncclUint64, comm, st));
         CK(cudaMemcpyAsync(all, stage, count * world * sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        return STEM_OK;
+        return wait(st);
     }
     int alltoallv(const void *send, const uint64_t *scnt, const uint64_t *sdsp, void *recv, const uint64_t *rcnt,
                   const uint64_t *rdsp, size_t elem, cudaStream_t st) override {
@@ -129,17 +189,28 @@ struct LoopGroup {
     uint64_t gen = 0;
     std::vector<const void *> ptr;
     std::vector<const uint64_t *> h0, h1;
+    bool broken = false;
     explicit LoopGroup(int w) : world(w), ptr(w), h0(w), h1(w) {}
-    void barrier() {
+    // false when a member did not arrive within comm_timeout_s() (the group is then broken)
+    bool barrier() {
         std::unique_lock<std::mutex> l(m);
+        if (broken) return false;
         const uint64_t g = gen;
         if (++arrived == world) {
             arrived = 0;
             gen++;
             cv.notify_all();
-        } else {
-            cv.wait(l, [&] { return gen != g; });
+            return true;
         }
+        const auto dl = std::chrono::steady_clock::now() +
+                        std::chrono::duration_cast<std::chrono::steady_clock::duration>(
+                            std::chrono::duration<double>(comm_timeout_s()));
+        if (!cv.wait_until(l, dl, [&] { return gen != g || broken; }) || broken) {
+            broken = true;
+            cv.notify_all();
+            return false;
+        }
+        return true;
     }
 };
 
@@ -177,12 +248,12 @@ class LoopComm : public Comm {
         }
         CK(cudaStreamSynchronize(st));
         g->ptr[rank] = buf;
-        g->barrier();
+        if (!g->barrier()) return STEM_E_NCCL;
         PtrSet ps{};
         for (int r = 0; r < world; r++) ps.p[r] = g->ptr[r];
         if (count) sum_buffers_kernel<<<(unsigned)((count + 255) / 256), 256, 0, st>>>(ps, world, count, f64, tmp);
         cudaError_t e = cudaStreamSynchronize(st);
-        g->barrier();   // every rank has read every buffer
+        if (!g->barrier()) return STEM_E_NCCL;   // every rank has read every buffer
         if (e != cudaSuccess) return STEM_E_CUDA;
         CK(cudaMemcpyAsync(buf, tmp, count * 8, cudaMemcpyDeviceToDevice, st));
         CK(cudaStreamSynchronize(st));
@@ -190,9 +261,9 @@ class LoopComm : public Comm {
     }
     int allgather_host(const uint64_t *mine, size_t count, uint64_t *all, cudaStream_t) override {
         g->h0[rank] = mine;
-        g->barrier();
+        if (!g->barrier()) return STEM_E_NCCL;
         for (int r = 0; r < world; r++) memcpy(all + (size_t)r * count, g->h0[r], count * sizeof(uint64_t));
-        g->barrier();
+        if (!g->barrier()) return STEM_E_NCCL;
         return STEM_OK;
     }
     int alltoallv(const void *send, const uint64_t *scnt, const uint64_t *sdsp, void *recv, const uint64_t *rcnt,
@@ -202,7 +273,7 @@ class LoopComm : public Comm {
         g->ptr[rank] = send;
         g->h0[rank] = scnt;
         g->h1[rank] = sdsp;
-        g->barrier();
+        if (!g->barrier()) return STEM_E_NCCL;
         cudaError_t e = cudaSuccess;
         for (int r = 0; r < world && e == cudaSuccess; r++) {
             const uint64_t cnt = g->h0[r][rank];
@@ -211,13 +282,42 @@ class LoopComm : public Comm {
                                     cnt * elem, cudaMemcpyDeviceToDevice, st);
         }
         if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-        g->barrier();   // senders may reuse their buffers
+        if (!g->barrier()) return STEM_E_NCCL;   // senders may reuse their buffers
         if (e != cudaSuccess) return STEM_E_CUDA;
         return STEM_OK;
     }
 };
 
+int sync_stream(Ctx &c) {
+    if (c.comm) return c.comm->wait(c.stream);
+    CK(cudaStreamSynchronize(c.stream));
+    return STEM_OK;
+}
+
+// Every rank contributes its local status; all return the first non-OK status
+// in rank order (or OK).  Called between stretches of local work and the next
+// collective, so no rank is left waiting for a peer that already returned.
+int dist_checkpoint(Ctx &c, int status) {
+    if (!c.comm) return status;
+    const int W = c.comm->world;
+    uint64_t mine = (uint64_t)(int64_t)status;
+    std::vector<uint64_t> all((size_t)W);
+    const int e = c.comm->allgather_host(&mine, 1, all.data(), c.stream);
+    if (e != STEM_OK) return e;
+    for (int r = 0; r < W; r++)
+        if ((int64_t)all[r] != STEM_OK) return (int)(int64_t)all[r];
+    return STEM_OK;
+}
+
 int comm_rank(const Comm *c) { return c->rank; }
+int comm_world(const Comm *c) { return c->world; }
+int comm_allgather_host(Ctx &c, const uint64_t *mine, size_t count, uint64_t *all) {
+    return c.comm->allgather_host(mine, count, all, c.stream);
+}
+int comm_alltoallv(Ctx &c, const void *send, const uint64_t *scnt, const uint64_t *sdsp, void *recv,
+                   const uint64_t *rcnt, const uint64_t *rdsp, size_t elem) {
+    return c.comm->alltoallv(send, scnt, sdsp, recv, rcnt, rdsp, elem, c.stream);
+}
 int dist_allreduce_u64(Ctx &c, uint64_t *buf, size_t count) { return c.comm->allreduce(buf, count, false, c.stream); }
 int dist_allreduce_f64(Ctx &c, double *buf, size_t count) { return c.comm->allreduce(buf, count, true, c.stream); }
 
@@ -353,7 +453,7 @@ static int partition(Ctx &c, PartArgs &a, uint64_t *scnt, uint64_t *sdsp) {
     CK(cudaGetLastError());
     uint64_t h[kMaxWorld + 1];
     CK(cudaMemcpyAsync(h, displs, sizeof(uint64_t) * (W + 1), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
+    CKS(sync_stream(c));
     for (int d = 0; d < W; d++) {
         sdsp[d] = h[d];
         scnt[d] = h[d + 1] - h[d];
@@ -361,14 +461,22 @@ static int partition(Ctx &c, PartArgs &a, uint64_t *scnt, uint64_t *sdsp) {
     return STEM_OK;
 }
 
-// receive layout from everyone's send counts: rcnt[s] = counts s sends to me
-static int exchange_counts(Ctx &c, const uint64_t *scnt, uint64_t *rcnt, uint64_t *rdsp, uint64_t &total) {
+// receive layout from everyone's send counts: rcnt[s] = counts s sends to me.
+// The allgather also carries every rank's local status (the partition before
+// it is local work): all ranks return the first failure in rank order.
+static int exchange_counts(Ctx &c, int local_status, const uint64_t *scnt, uint64_t *rcnt, uint64_t *rdsp,
+                           uint64_t &total) {
     const int W = c.comm->world, me = c.comm->rank;
-    std::vector<uint64_t> all((size_t)W * W);
-    CKS(c.comm->allgather_host(scnt, W, all.data(), c.stream));
+    std::vector<uint64_t> mine((size_t)W + 1, 0), all((size_t)W * (W + 1));
+    if (local_status == STEM_OK)
+        for (int d = 0; d < W; d++) mine[d] = scnt[d];
+    mine[W] = (uint64_t)(int64_t)local_status;
+    CKS(c.comm->allgather_host(mine.data(), W + 1, all.data(), c.stream));
+    for (int r = 0; r < W; r++)
+        if ((int64_t)all[(size_t)r * (W + 1) + W] != STEM_OK) return (int)(int64_t)all[(size_t)r * (W + 1) + W];
     total = 0;
     for (int s = 0; s < W; s++) {
-        rcnt[s] = all[(size_t)s * W + me];
+        rcnt[s] = all[(size_t)s * (W + 1) + me];
         rdsp[s] = total;
         total += rcnt[s];
     }
@@ -416,27 +524,36 @@ int dist_metric_sums(Ctx &c, const double *metrics_local, uint32_t nm, uint64_t 
     a.n = S;
     a.in0 = c.out_row;
     a.inw = c.out_weight;
-    CKS(c.ensure(c.xfer_u32[0], c.cap_xfer_u32[0], sizeof(uint32_t) * (S + 1)));
-    CKS(c.ensure(c.xfer_f64, c.cap_xfer_f64, sizeof(double) * (S + 1)));
-    a.out0 = c.xfer_u32[0];
-    a.outw = c.xfer_f64;
     uint64_t scnt[kMaxWorld], sdsp[kMaxWorld], rcnt[kMaxWorld], rdsp[kMaxWorld], R = 0;
-    CKS(partition(c, a, scnt, sdsp));
-    CKS(exchange_counts(c, scnt, rcnt, rdsp, R));
-    CKS(c.ensure(c.xfer_u32[1], c.cap_xfer_u32[1], sizeof(uint32_t) * (R + 1)));
-    CKS(c.ensure(c.xfer_f64b, c.cap_xfer_f64b, sizeof(double) * (R + 1)));
+    const int ls = [&]() -> int {
+        CKS(c.ensure(c.xfer_u32[0], c.cap_xfer_u32[0], sizeof(uint32_t) * (S + 1)));
+        CKS(c.ensure(c.xfer_f64, c.cap_xfer_f64, sizeof(double) * (S + 1)));
+        a.out0 = c.xfer_u32[0];
+        a.outw = c.xfer_f64;
+        return partition(c, a, scnt, sdsp);
+    }();
+    CKS(exchange_counts(c, ls, scnt, rcnt, rdsp, R));
+    const uint64_t blocks = (R + 255) / 256;
+    CKS(dist_checkpoint(c, [&]() -> int {
+        CKS(c.ensure(c.xfer_u32[1], c.cap_xfer_u32[1], sizeof(uint32_t) * (R + 1)));
+        CKS(c.ensure(c.xfer_f64b, c.cap_xfer_f64b, sizeof(double) * (R + 1)));
+        CKS(c.ensure(c.red_part2, c.cap_red2, sizeof(double) * (blocks * nm + nm + 1)));
+        return STEM_OK;
+    }()));
     CKS(c.comm->alltoallv(c.xfer_u32[0], scnt, sdsp, c.xfer_u32[1], rcnt, rdsp, sizeof(uint32_t), st));
     CKS(c.comm->alltoallv(c.xfer_f64, scnt, sdsp, c.xfer_f64b, rcnt, rdsp, sizeof(double), st));
-    const uint64_t blocks = (R + 255) / 256;
-    CKS(c.ensure(c.red_part2, c.cap_red2, sizeof(double) * (blocks * nm + nm + 1)));
-    if (R) {
-        metric_req_kernel<<<(unsigned)blocks, 256, 0, st>>>(c.xfer_u32[1], c.xfer_f64b, R, c.row_bases[c.comm->rank],
-                                                            metrics_local, c.n_local_rows, nm, c.red_part2);
+    CKS(dist_checkpoint(c, [&]() -> int {
+        if (R) {
+            metric_req_kernel<<<(unsigned)blocks, 256, 0, st>>>(c.xfer_u32[1], c.xfer_f64b, R,
+                                                                c.row_bases[c.comm->rank], metrics_local,
+                                                                c.n_local_rows, nm, c.red_part2);
+            c.launches++;
+        }
+        cols_sum_kernel<<<1, 64, 0, st>>>(c.red_part2, blocks, nm, out);
         c.launches++;
-    }
-    cols_sum_kernel<<<1, 64, 0, st>>>(c.red_part2, blocks, nm, out);
-    c.launches++;
-    CK(cudaGetLastError());
+        CK(cudaGetLastError());
+        return STEM_OK;
+    }()));
     return c.comm->allreduce(out, nm, true, st);
 }
 
@@ -457,29 +574,44 @@ __global__ void add_kernel_u32(uint32_t *x, uint64_t n, uint32_t v) {
     if (i < n) x[i] += v;
 }
 
-
+// local_status: the rank's own argument checks (stem_root_plan_dist), agreed
+// across ranks first.  Every later stretch of local work ends in a checkpoint
+// (or in exchange_counts, which carries the status) before the next
+// collective, so all ranks return the same status together.
 int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
-                  const stem_opts &o) {
+                  const stem_opts &o, int local_status) {
     const int W = comm.world, me = comm.rank;
     const uint64_t n = tr->n;
     const uint32_t K = tr->n_kernels, nm = tr->n_metrics;
     cudaStream_t st = c.stream;
     const uint32_t *kid = tr->kernel_id, *t = tr->exec_ns;
     const double *met = tr->metrics;
-    if (tr->device < 0 && n) {   // host shard: copy in on the stream
-        CKS(c.ensure(c.in_kid, c.cap_in_kid, sizeof(uint32_t) * n));
-        CKS(c.ensure(c.in_t, c.cap_in_t, sizeof(uint32_t) * n));
-        CK(cudaMemcpyAsync(c.in_kid, kid, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
-        CK(cudaMemcpyAsync(c.in_t, t, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
-        kid = c.in_kid;
-        t = c.in_t;
-        if (nm) {
-            CKS(c.ensure(c.in_met, c.cap_in_met, sizeof(double) * n * nm));
-            CK(cudaMemcpyAsync(c.in_met, met, sizeof(double) * n * nm, cudaMemcpyHostToDevice, st));
-            met = c.in_met;
+    (void)conf;
+    // ---- arguments, input copy-in, histogram buffers
+    CKS(dist_checkpoint(c, [&]() -> int {
+        CKS(local_status);
+        if (tr->device < 0 && n) {   // host shard: copy in on the stream
+            CKS(c.ensure(c.in_kid, c.cap_in_kid, sizeof(uint32_t) * n));
+            CKS(c.ensure(c.in_t, c.cap_in_t, sizeof(uint32_t) * n));
+            CK(cudaMemcpyAsync(c.in_kid, kid, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
+            CK(cudaMemcpyAsync(c.in_t, t, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
+            kid = c.in_kid;
+            t = c.in_t;
+            if (nm) {
+                CKS(c.ensure(c.in_met, c.cap_in_met, sizeof(double) * n * nm));
+                CK(cudaMemcpyAsync(c.in_met, met, sizeof(double) * n * nm, cudaMemcpyHostToDevice, st));
+                met = c.in_met;
+            }
         }
-    }
-    // row shards of every rank (metric requests are routed by row)
+        CKS(c.ensure(c.kid_count, c.cap_kc, sizeof(uint32_t) * ((uint64_t)K + 1)));
+        CKS(c.ensure(c.dist_cnt, c.cap_dist_cnt, sizeof(uint64_t) * ((uint64_t)K + 2)));
+        CKS(c.ensure(c.scalars, c.cap_scalars, sizeof(DevScalars)));
+        CKS(c.ensure(c.kid_max, c.cap_kmax, sizeof(uint32_t) * ((uint64_t)K + 1)));
+        CKS(c.ensure(c.hist, c.cap_hist, sizeof(uint64_t) * 9 * 256));
+        return STEM_OK;
+    }()));
+    // row shards of every rank (metric requests are routed by row); the checks
+    // run on the same gathered data everywhere, so every rank agrees
     {
         uint64_t mine[2] = {row_base, n};
         std::vector<uint64_t> all(2 * (size_t)W);
@@ -493,22 +625,22 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
         c.n_local_rows = n;
     }
     // 1. global kernel histogram (+ range errors) -> owner ranges
-    CKS(c.ensure(c.kid_count, c.cap_kc, sizeof(uint32_t) * ((uint64_t)K + 1)));
-    CKS(c.ensure(c.dist_cnt, c.cap_dist_cnt, sizeof(uint64_t) * ((uint64_t)K + 2)));
-    CKS(c.ensure(c.scalars, c.cap_scalars, sizeof(DevScalars)));
-    CKS(c.ensure(c.kid_max, c.cap_kmax, sizeof(uint32_t) * ((uint64_t)K + 1)));
-    CKS(c.ensure(c.hist, c.cap_hist, sizeof(uint64_t) * 9 * 256));
-    CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
-    CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
     const int tk_x = c.stage_begin("dist_exchange");
-    if (n) CKS(histogram_kernels(c, kid, t, n, K, nullptr));
-    kid_counts_u64_kernel<<<(unsigned)((K + 256) / 256), 256, 0, st>>>(c.kid_count, K, &c.scalars->err, c.dist_cnt);
-    c.launches++;
+    CKS(dist_checkpoint(c, [&]() -> int {
+        CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
+        CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
+        if (n) CKS(histogram_kernels(c, kid, t, n, K, nullptr));
+        kid_counts_u64_kernel<<<(unsigned)((K + 256) / 256), 256, 0, st>>>(c.kid_count, K, &c.scalars->err,
+                                                                           c.dist_cnt);
+        c.launches++;
+        CK(cudaGetLastError());
+        return STEM_OK;
+    }()));
     CKS(comm.allreduce(c.dist_cnt, (size_t)K + 1, false, st));
     std::vector<uint64_t> gcnt((size_t)K + 1);
     CK(cudaMemcpyAsync(gcnt.data(), c.dist_cnt, sizeof(uint64_t) * ((uint64_t)K + 1), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    if (gcnt[K]) return STEM_E_RANGE;
+    CKS(sync_stream(c));
+    if (gcnt[K]) return STEM_E_RANGE;   // the same reduced flag on every rank
     std::vector<uint32_t> bounds(W + 1);
     owner_ranges(gcnt.data(), K, W, bounds.data());
     const uint32_t kb = bounds[me], ke = bounds[me + 1];
@@ -521,22 +653,29 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
     pa.in0 = kid;
     pa.in1 = t;
     pa.in2_add = row_base;
-    for (int i = 0; i < 3; i++) CKS(c.ensure(c.xfer_u32[i], c.cap_xfer_u32[i], sizeof(uint32_t) * (n + 1)));
-    pa.out0 = c.xfer_u32[0];
-    pa.out1 = c.xfer_u32[1];
-    pa.out2 = c.xfer_u32[2];
     uint64_t scnt[kMaxWorld], sdsp[kMaxWorld], rcnt[kMaxWorld], rdsp[kMaxWorld], R = 0;
-    CKS(partition(c, pa, scnt, sdsp));
-    CKS(exchange_counts(c, scnt, rcnt, rdsp, R));
-    if (R >= (1ull << 32)) return STEM_E_RANGE;
-    for (int i = 0; i < 3; i++) CKS(c.ensure(c.recv_u32[i], c.cap_recv_u32[i], sizeof(uint32_t) * (R + 1)));
+    const int ls = [&]() -> int {
+        for (int i = 0; i < 3; i++) CKS(c.ensure(c.xfer_u32[i], c.cap_xfer_u32[i], sizeof(uint32_t) * (n + 1)));
+        pa.out0 = c.xfer_u32[0];
+        pa.out1 = c.xfer_u32[1];
+        pa.out2 = c.xfer_u32[2];
+        return partition(c, pa, scnt, sdsp);
+    }();
+    CKS(exchange_counts(c, ls, scnt, rcnt, rdsp, R));
+    CKS(dist_checkpoint(c, [&]() -> int {
+        if (R >= (1ull << 32)) return STEM_E_RANGE;
+        for (int i = 0; i < 3; i++) CKS(c.ensure(c.recv_u32[i], c.cap_recv_u32[i], sizeof(uint32_t) * (R + 1)));
+        return STEM_OK;
+    }()));
     for (int i = 0; i < 3; i++)
         CKS(comm.alltoallv(c.xfer_u32[i], scnt, sdsp, c.recv_u32[i], rcnt, rdsp, sizeof(uint32_t), st));
+    CKS(sync_stream(c));   // the exchange is complete (or failed) before the local pipeline
     c.stage_end(tk_x, 24 * n + 12 * R);
     // 3. the local pipeline on my kernel range (kernel ids rebased to 0)
     const uint32_t KL = ke - kb;
     c.kid_base = kb;
-    if (R) {
+    CKS(dist_checkpoint(c, [&]() -> int {
+        if (!R) return STEM_OK;
         sub_kernel_u32<<<(unsigned)((R + 255) / 256), 256, 0, st>>>(c.recv_u32[0], R, kb);
         c.launches++;
         CKS(c.ensure_all(R, KL, nm));
@@ -548,10 +687,17 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
         } else {
             CKS(stem_only_leaves(c, R, KL));
         }
-    }
+        return STEM_OK;
+    }()));
     const double q = c.z / eps;
     CKS(leaves_and_plan(c, R, KL, met, nm, eps, c.z, q * q, o));
-    (void)conf;
+    c.have_mbounds = false;
+    if (o.metric_bounds && nm) {   // every rank's leaves gathered; each rank reads its home rows' metrics
+        const int tk_mb = c.stage_begin("metric_bounds");
+        CKS(metric_bounds_dist(c, c.n_leaves, R, K, kid, t, met, n, nm, c.z));
+        c.stage_end(tk_mb, (16 + 16 * (uint64_t)nm) * n);
+        c.have_mbounds = true;
+    }
     // 4. gather the plan on rank 0, canonical order = rank order (kernel ranges ascend)
     uint64_t mine[2] = {c.n_leaves, c.n_samples};
     std::vector<uint64_t> all(2 * (size_t)W);
@@ -562,30 +708,46 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
         Lg += all[2 * r];
         Sg += all[2 * r + 1];
     }
-    if (c.n_samples && Loff) {
-        add_kernel_u32<<<(unsigned)((c.n_samples + 255) / 256), 256, 0, st>>>(c.out_cluster, c.n_samples,
-                                                                             (uint32_t)Loff);
-        c.launches++;
-    }
     std::vector<uint64_t> s_c(W, 0), s_d(W, 0), r_c(W, 0), r_d(W, 0);
-    auto gather = [&](void *src, void *&dst, size_t &cap, size_t elem, int which) -> int {
-        s_c[0] = all[2 * me + which];
-        if (me == 0) {
-            uint64_t off = 0;
-            for (int r = 0; r < W; r++) {
-                r_c[r] = all[2 * r + which];
-                r_d[r] = off;
-                off += r_c[r];
-            }
-            CKS(c.ensure(dst, cap, elem * (off + 1)));
+    std::vector<uint64_t> rc_all[2];
+    for (int which = 0; which < 2; which++) {
+        rc_all[which].assign(2 * (size_t)W, 0);
+        uint64_t off = 0;
+        for (int r = 0; r < W; r++) {
+            rc_all[which][r] = all[2 * r + which];
+            rc_all[which][W + r] = off;
+            off += all[2 * r + which];
         }
+    }
+    CKS(dist_checkpoint(c, [&]() -> int {
+        if (c.n_samples && Loff) {
+            add_kernel_u32<<<(unsigned)((c.n_samples + 255) / 256), 256, 0, st>>>(c.out_cluster, c.n_samples,
+                                                                                 (uint32_t)Loff);
+            c.launches++;
+        }
+        if (me == 0) {
+            CKS(c.ensure(c.g_clusters, c.cap_g_clusters, sizeof(stem_cluster) * (Lg + 1)));
+            CKS(c.ensure(c.g_row, c.cap_g_row, sizeof(uint32_t) * (Sg + 1)));
+            CKS(c.ensure(c.g_cluster, c.cap_g_cluster, sizeof(uint32_t) * (Sg + 1)));
+            CKS(c.ensure(c.g_weight, c.cap_g_weight, sizeof(double) * (Sg + 1)));
+        }
+        CK(cudaGetLastError());
+        return STEM_OK;
+    }()));
+    auto gather = [&](void *src, void *dst, size_t elem, int which) -> int {
+        s_c[0] = all[2 * me + which];
+        if (me == 0)
+            for (int r = 0; r < W; r++) {
+                r_c[r] = rc_all[which][r];
+                r_d[r] = rc_all[which][W + r];
+            }
         return comm.alltoallv(src, s_c.data(), s_d.data(), dst, r_c.data(), r_d.data(), elem, st);
     };
-    CKS(gather(c.out_clusters, c.g_clusters, c.cap_g_clusters, sizeof(stem_cluster), 0));
-    CKS(gather(c.out_row, c.g_row, c.cap_g_row, sizeof(uint32_t), 1));
-    CKS(gather(c.out_cluster, c.g_cluster, c.cap_g_cluster, sizeof(uint32_t), 1));
-    CKS(gather(c.out_weight, c.g_weight, c.cap_g_weight, sizeof(double), 1));
-    CK(cudaStreamSynchronize(st));
+    CKS(gather(c.out_clusters, c.g_clusters, sizeof(stem_cluster), 0));
+    CKS(gather(c.out_row, c.g_row, sizeof(uint32_t), 1));
+    CKS(gather(c.out_cluster, c.g_cluster, sizeof(uint32_t), 1));
+    CKS(gather(c.out_weight, c.g_weight, sizeof(double), 1));
+    CKS(sync_stream(c));
     if (me == 0) {   // the global plan becomes this ctx's output
         std::swap(c.out_clusters, *(stem_cluster **)&c.g_clusters);
         std::swap(c.cap_out_cl, c.cap_g_clusters);
@@ -595,9 +757,11 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
         std::swap(c.cap_out_cluster, c.cap_g_cluster);
         std::swap(c.out_weight, *(double **)&c.g_weight);
         std::swap(c.cap_out_weight, c.cap_g_weight);
+        c.n_leaves = Lg;
+        c.n_samples = Sg;
     }
-    c.n_leaves = Lg;
-    c.n_samples = Sg;
+    // other ranks keep their own part (its clusters, its samples with global
+    // cluster indices): stem_ctx_device_plan then describes exactly the buffers it holds
     c.stats.n_clusters = Lg;
     c.stats.n_samples = Sg;
     return STEM_OK;

@@ -211,6 +211,15 @@ struct Ctx {
     size_t cap_g_clusters = 0, cap_g_row = 0, cap_g_cluster = 0, cap_g_weight = 0;
     uint64_t row_bases[65] = {0};
     uint64_t n_local_rows = 0;
+    // metric_bounds (metric.cu): leaf table (first leaf per kernel, lo_ns, n, m), per-leaf sums
+    uint32_t *mb_first = nullptr, *mb_lo = nullptr, *mb_gkid = nullptr, *mb_leaf_of = nullptr;
+    size_t cap_mb_first = 0, cap_mb_lo = 0, cap_mb_gkid = 0, cap_mb_leaf_of = 0;
+    uint64_t *mb_n = nullptr, *mb_gm = nullptr; size_t cap_mb_n = 0, cap_mb_gm = 0;
+    const uint64_t *mb_m = nullptr;                  // leaf_m (single GPU) or mb_gm (gathered)
+    double *mb_acc = nullptr, *mb_part = nullptr; size_t cap_mb_acc = 0, cap_mb_part = 0;
+    void *mb_rec = nullptr; size_t cap_mb_rec = 0;
+    bool have_mbounds = false;
+    double host_true_metric[64], host_bound_metric[64];
 
     // last plan
     bool have_plan = false;
@@ -220,8 +229,17 @@ struct Ctx {
     double est_total = 0, bound = 0, eps = 0, z = 0;
 };
 
+// host wait for c.stream: with a communicator, polls for peer failures and the
+// comm timeout (STEM_E_NCCL) instead of blocking forever (dist.cu)
+int sync_stream(Ctx &c);
+// multi-GPU: agree on a local status across ranks (identity without a communicator)
+int dist_checkpoint(Ctx &c, int status);
 // multi-GPU collectives on c.comm (dist.cu); device buffers, in place, sums
 int comm_rank(const Comm *c);
+int comm_world(const Comm *c);
+int comm_allgather_host(Ctx &c, const uint64_t *mine, size_t count, uint64_t *all);
+int comm_alltoallv(Ctx &c, const void *send, const uint64_t *scnt, const uint64_t *sdsp, void *recv,
+                   const uint64_t *rcnt, const uint64_t *rdsp, size_t elem);
 int dist_allreduce_u64(Ctx &c, uint64_t *buf, size_t count);
 int dist_allreduce_f64(Ctx &c, double *buf, size_t count);
 int dist_metric_sums(Ctx &c, const double *metrics_local, uint32_t nm, uint64_t S, double *out);
@@ -236,8 +254,14 @@ int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,
                       uint32_t *tailh);   // pre-pass only
 int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
-                  const stem_opts &o);
+                  const stem_opts &o, int local_status);
 int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint32_t n_metrics, double eps,
-                    double z, double k2, const stem_opts &o);                                  // a5..a8
+                    double z, double k2, const stem_opts &o, const uint32_t *tr_kid = nullptr,
+                    const uint32_t *tr_t = nullptr, uint64_t tr_n = 0);                        // a5..a8
+// a8 option metric_bounds (metric.cu): true totals and bounds into host_true/bound_metric
+int metric_bounds_local(Ctx &c, uint64_t L, uint32_t K, uint64_t n_sorted, const uint32_t *kid, const uint32_t *t,
+                        const double *met, uint64_t n_trace, uint32_t nm, double z);
+int metric_bounds_dist(Ctx &c, uint64_t L_local, uint64_t n_sorted, uint32_t K_global, const uint32_t *kid,
+                       const uint32_t *t, const double *met, uint64_t n_home, uint32_t nm, double z);
 
 }  // namespace sr

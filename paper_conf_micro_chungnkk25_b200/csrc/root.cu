@@ -1362,9 +1362,27 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         const int nxt = cur ^ 1;
         const uint64_t *ctot = &c.scalars->ftot[cur];
         uint64_t *ntot = &c.scalars->ftot[nxt];
-        CKS(c.ensure(c.cut, c.cap_cut, sizeof(uint32_t) * Cub));
-        CKS(c.ensure(c.cut_SL, c.cap_cut_SL, sizeof(uint64_t) * Cub));
-        CKS(ensure_frontier(c, nxt, 2 * Cub));   // at most 2 children per cluster
+        // Growing a buffer frees the old one, which the levels already queued
+        // may still read (nxt is the input of the level queued before this
+        // one): drain the stream first, then grow with 2x headroom so this
+        // happens only O(log) times per ctx.
+        const uint64_t max_ent = Aub / kBigSeg + Aub / big_rows() + 1;
+        const bool grow = sizeof(uint32_t) * Cub > c.cap_cut || sizeof(uint64_t) * Cub > c.cap_cut_SL ||
+                          sizeof(u128) * 2 * Cub > c.cap_fQ[nxt] ||
+                          (split == 0 && (sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (Cub + 1) > c.cap_big_ent ||
+                                          sizeof(Cand) * max_ent > c.cap_big_part ||
+                                          sizeof(unsigned long long) * Cub > c.cap_big_thr));
+        if (grow) {
+            CK(cudaStreamSynchronize(st));
+            CKS(c.ensure(c.cut, c.cap_cut, 2 * sizeof(uint32_t) * Cub));
+            CKS(c.ensure(c.cut_SL, c.cap_cut_SL, 2 * sizeof(uint64_t) * Cub));
+            CKS(ensure_frontier(c, nxt, 4 * Cub));   // at most 2 children per cluster
+            if (split == 0) {
+                CKS(c.ensure(c.big_ent, c.cap_big_ent, 2 * (sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (Cub + 1))));
+                CKS(c.ensure(c.big_part, c.cap_big_part, 2 * sizeof(Cand) * max_ent));
+                CKS(c.ensure(c.big_thr, c.cap_big_thr, 2 * sizeof(unsigned long long) * Cub));
+            }
+        }
         const int tk_l = loc_rows > 0 ? c.stage_begin("root_local") : -1;
         if (loc_rows > 0) {
             LocalArgs la{c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], (uint32_t)Cub, level - 1, c.PS1, c.PS2,
@@ -1415,10 +1433,6 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             c.launches++;
         }
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
-        const uint64_t max_ent = Aub / kBigSeg + Aub / big_rows() + 1;
-        CKS(c.ensure(c.big_ent, c.cap_big_ent, sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (Cub + 1)));
-        CKS(c.ensure(c.big_part, c.cap_big_part, sizeof(Cand) * max_ent));
-        CKS(c.ensure(c.big_thr, c.cap_big_thr, sizeof(unsigned long long) * Cub));
         BigEntry *ent = (BigEntry *)c.big_ent;
         uint32_t *first_ent = (uint32_t *)(ent + max_ent);
         CK(cudaMemsetAsync(&c.scalars->big_count, 0, sizeof(uint32_t), st));

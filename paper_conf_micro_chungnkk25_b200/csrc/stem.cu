@@ -508,57 +508,68 @@ __global__ void pack_kernel(const uint32_t *leaf_lo, const uint32_t *leaf_kid, c
 // ---------------------------------------------------------------- driver
 static unsigned blocks_for(uint64_t n) { return (unsigned)((n + kThreads - 1) / kThreads); }
 
+// In multi-GPU runs every stretch of local work between two collectives is one
+// segment: its status is agreed across ranks (dist_checkpoint) before the next
+// collective, so a rank-local failure (allocation, CUDA) makes every rank
+// return the same error instead of leaving peers blocked in a collective.
 int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint32_t nm, double eps, double z,
-                    double k2, const stem_opts &o) {
+                    double k2, const stem_opts &o, const uint32_t *tr_kid, const uint32_t *tr_t, uint64_t tr_n) {
     cudaStream_t st = c.stream;
-    // a5: leaf starts = group starts U accepted cuts, in row order = canonical (kernel, lo) order
-    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(n) + 1) * sizeof(uint64_t)));
-    CKS(c.ensure(c.leaf_lo, c.cap_leaf_lo, sizeof(uint32_t) * (n + 1)));
-    const int tk_leaf = c.stage_begin("leaf_table");
-    {
-        const uint64_t nw = (n + 31) / 32, nt = (nw + kFlagTileW - 1) / kFlagTileW;   // bits >= n are never set
-        CKS(c.ensure(c.leaf_moff, c.cap_leaf_moff, sizeof(uint64_t) * (nt + 1)));   // tile counts (scratch)
-        uint64_t *tcnt = c.leaf_moff;
-        if (nt) flag_count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, nw, tcnt);
-        exclusive_scan<uint64_t>([tcnt] __device__(uint64_t i) -> uint64_t { return tcnt[i]; },
-                                 [tcnt] __device__(uint64_t i, uint64_t pre, uint64_t) { tcnt[i] = pre; }, nt,
-                                 (uint64_t *)c.scan_scratch, &c.scalars->n_leaves, st, &c.launches);
-        if (nt) flag_compact_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, nw, tcnt, c.leaf_lo);
-        c.launches += 2;
-        CK(cudaGetLastError());
-    }
-    c.stage_end(tk_leaf, 2 * 4 * (n / 32 + 1));
     uint64_t L = 0;
-    CK(cudaMemcpyAsync(&L, &c.scalars->n_leaves, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    c.n_leaves = L;
-    // per-leaf arrays (leaf_kid/ord live in the two halves of one allocation)
-    CKS(c.ensure(c.leaf_m, c.cap_leaf_m, sizeof(uint64_t) * (L + 1)));
-    CKS(c.ensure(c.leaf_moff, c.cap_leaf_moff, sizeof(uint64_t) * (L + 1)));
-    CKS(c.ensure(c.leaf_U, c.cap_leaf_U, sizeof(uint64_t) * (L + 1)));
-    CKS(c.ensure(c.leaf_census, c.cap_leaf_census, L + 1));
-    CKS(c.ensure(c.leaf_kid, c.cap_leaf_kid, sizeof(uint32_t) * (L + 1)));
-    CKS(c.ensure(c.leaf_ord, c.cap_leaf_ord, sizeof(uint32_t) * (L + 1)));
-    uint32_t *leaf_kid = c.leaf_kid, *leaf_ord = c.leaf_ord;
     const uint32_t nsets = o.scope == 1 ? K : 1;
-    CKS(c.ensure(c.fix_acc, c.cap_fix, sizeof(uint64_t) * kFixDigits * nsets));
-    CKS(c.ensure(c.kern_T, c.cap_kern_T, sizeof(uint64_t) * nsets));
-    CKS(c.ensure(c.kern_g, c.cap_kern_g, sizeof(double) * nsets));
-    CK(cudaMemsetAsync(c.fix_acc, 0, sizeof(uint64_t) * kFixDigits * nsets, st));
-    CK(cudaMemsetAsync(c.kern_T, 0, sizeof(uint64_t) * nsets, st));
-    CK(cudaMemsetAsync(c.leaf_U, 0, sizeof(uint64_t) * (L + 1), st));
+    // ---- segment 1: leaf table (a5) and the exact KKT partials (a6)
+    CKS(dist_checkpoint(c, [&]() -> int {
+        // a5: leaf starts = group starts U accepted cuts, in row order = canonical (kernel, lo) order
+        CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(n) + 1) * sizeof(uint64_t)));
+        CKS(c.ensure(c.leaf_lo, c.cap_leaf_lo, sizeof(uint32_t) * (n + 1)));
+        const int tk_leaf = c.stage_begin("leaf_table");
+        {
+            const uint64_t nw = (n + 31) / 32, nt = (nw + kFlagTileW - 1) / kFlagTileW;   // bits >= n are never set
+            CKS(c.ensure(c.leaf_moff, c.cap_leaf_moff, sizeof(uint64_t) * (nt + 1)));   // tile counts (scratch)
+            uint64_t *tcnt = c.leaf_moff;
+            if (nt) flag_count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, nw, tcnt);
+            exclusive_scan<uint64_t>([tcnt] __device__(uint64_t i) -> uint64_t { return tcnt[i]; },
+                                     [tcnt] __device__(uint64_t i, uint64_t pre, uint64_t) { tcnt[i] = pre; }, nt,
+                                     (uint64_t *)c.scan_scratch, &c.scalars->n_leaves, st, &c.launches);
+            if (nt) flag_compact_kernel<<<(unsigned)nt, kThreads, 0, st>>>(c.flags, nw, tcnt, c.leaf_lo);
+            c.launches += 2;
+            CK(cudaGetLastError());
+        }
+        c.stage_end(tk_leaf, 2 * 4 * (n / 32 + 1));
+        CK(cudaMemcpyAsync(&L, &c.scalars->n_leaves, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CKS(sync_stream(c));
+        c.n_leaves = L;
+        CKS(c.ensure(c.leaf_m, c.cap_leaf_m, sizeof(uint64_t) * (L + 1)));
+        CKS(c.ensure(c.leaf_moff, c.cap_leaf_moff, sizeof(uint64_t) * (L + 1)));
+        CKS(c.ensure(c.leaf_U, c.cap_leaf_U, sizeof(uint64_t) * (L + 1)));
+        CKS(c.ensure(c.leaf_census, c.cap_leaf_census, L + 1));
+        CKS(c.ensure(c.leaf_kid, c.cap_leaf_kid, sizeof(uint32_t) * (L + 1)));
+        CKS(c.ensure(c.leaf_ord, c.cap_leaf_ord, sizeof(uint32_t) * (L + 1)));
+        CKS(c.ensure(c.fix_acc, c.cap_fix, sizeof(uint64_t) * kFixDigits * nsets));
+        CKS(c.ensure(c.kern_T, c.cap_kern_T, sizeof(uint64_t) * nsets));
+        CKS(c.ensure(c.kern_g, c.cap_kern_g, sizeof(double) * nsets));
+        CK(cudaMemsetAsync(c.fix_acc, 0, sizeof(uint64_t) * kFixDigits * nsets, st));
+        CK(cudaMemsetAsync(c.kern_T, 0, sizeof(uint64_t) * nsets, st));
+        CK(cudaMemsetAsync(c.leaf_U, 0, sizeof(uint64_t) * (L + 1), st));
+        return STEM_OK;
+    }()));
+    uint32_t *leaf_kid = c.leaf_kid, *leaf_ord = c.leaf_ord;
 
     const int tk_kkt = c.stage_begin("stem_sizes");
-    if (n) {
-        total_kernel<<<1, 32, 0, st>>>(c.PS1, c.t_sorted, n, &c.scalars->T);
+    CKS(dist_checkpoint(c, [&]() -> int {
+        if (n) {
+            total_kernel<<<1, 32, 0, st>>>(c.PS1, c.t_sorted, n, &c.scalars->T);
+            c.launches++;
+        } else {
+            CK(cudaMemsetAsync(&c.scalars->T, 0, sizeof(uint64_t), st));
+        }
+        LeafArgs la{c.leaf_lo, c.goff, c.t_sorted, c.PS1, c.PS2, L, n, K, o.scope, leaf_kid, leaf_ord,
+                    c.fix_acc, c.kern_T, &c.scalars->err};
+        if (L) leaf_kkt_kernel<<<blocks_for(L), kThreads, 0, st>>>(la);
         c.launches++;
-    } else {
-        CK(cudaMemsetAsync(&c.scalars->T, 0, sizeof(uint64_t), st));
-    }
-    LeafArgs la{c.leaf_lo, c.goff, c.t_sorted, c.PS1, c.PS2, L, n, K, o.scope, leaf_kid, leaf_ord,
-                c.fix_acc, c.kern_T, &c.scalars->err};
-    if (L) leaf_kkt_kernel<<<blocks_for(L), kThreads, 0, st>>>(la);
-    c.launches++;
+        CK(cudaGetLastError());
+        return STEM_OK;
+    }()));
     if (c.comm) {   // multi-GPU: T and the exact Ssum digits are sums over every rank's leaves
         uint64_t *r7 = c.scalars->red7;
         CK(cudaMemcpyAsync(r7, &c.scalars->T, sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
@@ -568,26 +579,28 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         if (o.scope == 0)
             CK(cudaMemcpyAsync(c.fix_acc, r7 + 1, sizeof(uint64_t) * kFixDigits, cudaMemcpyDeviceToDevice, st));
     }
-    // g per set (T = total_kernel above, exact)
-    if (o.scope == 0)
-        kkt_finalize_kernel<<<1, 32, 0, st>>>(c.fix_acc, nullptr, &c.scalars->T, 1, eps, z, c.kern_g, &c.scalars->ssum);
-    else if (o.scope == 1 && K)
-        kkt_finalize_kernel<<<blocks_for(K), kThreads, 0, st>>>(c.fix_acc, c.kern_T, nullptr, K, eps, z, c.kern_g,
-                                                               nullptr);
-    if (o.scope != 2) c.launches++;
-    MArgs ma{c.leaf_lo, leaf_kid, c.t_sorted, c.PS1, c.PS2, L, n, o.scope, o.census_cap, k2, c.kern_g, c.leaf_m,
-             c.leaf_census, &c.scalars->limit_err};
-    if (L) leaf_m_kernel<<<blocks_for(L), kThreads, 0, st>>>(ma);
-    c.launches++;
-    CK(cudaGetLastError());
-    {
+    // ---- segment 2: g per set, m_i, sample offsets
+    CKS(dist_checkpoint(c, [&]() -> int {
+        if (o.scope == 0)
+            kkt_finalize_kernel<<<1, 32, 0, st>>>(c.fix_acc, nullptr, &c.scalars->T, 1, eps, z, c.kern_g,
+                                                  &c.scalars->ssum);
+        else if (o.scope == 1 && K)
+            kkt_finalize_kernel<<<blocks_for(K), kThreads, 0, st>>>(c.fix_acc, c.kern_T, nullptr, K, eps, z, c.kern_g,
+                                                                   nullptr);
+        if (o.scope != 2) c.launches++;
+        MArgs ma{c.leaf_lo, leaf_kid, c.t_sorted, c.PS1, c.PS2, L, n, o.scope, o.census_cap, k2, c.kern_g,
+                 c.leaf_m, c.leaf_census, &c.scalars->limit_err};
+        if (L) leaf_m_kernel<<<blocks_for(L), kThreads, 0, st>>>(ma);
+        c.launches++;
+        CK(cudaGetLastError());
         const uint64_t *m = c.leaf_m;
         uint64_t *moff = c.leaf_moff;
         exclusive_scan<uint64_t>([m] __device__(uint64_t i) -> uint64_t { return m[i]; },
                                  [moff] __device__(uint64_t i, uint64_t pre, uint64_t) { moff[i] = pre; }, L,
                                  (uint64_t *)c.scan_scratch, &c.scalars->total_m, st, &c.launches);
         CK(cudaGetLastError());
-    }
+        return STEM_OK;
+    }()));
     c.stage_end(tk_kkt, 64 * L);
     uint64_t S_global = 0;
     if (c.comm) {
@@ -598,68 +611,78 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         CKS(dist_allreduce_u64(c, r7, 2));
         uint64_t h2[2];
         CK(cudaMemcpyAsync(h2, r7, sizeof(h2), cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        if (h2[1] || h2[0] >= (1ull << 32)) return STEM_E_LIMIT;
+        CKS(sync_stream(c));
+        if (h2[1] || h2[0] >= (1ull << 32)) return STEM_E_LIMIT;   // identical on every rank
         S_global = h2[0];
     }
-    DevScalars hs;
-    CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    if (hs.err & 2) return STEM_E_CUDA;
-    if (hs.limit_err || hs.total_m >= (1ull << 32)) return STEM_E_LIMIT;
-    const uint64_t S = hs.total_m;
-    const uint64_t T = hs.T;
-    c.n_samples = S;
-    c.T = T;
-    c.stats.ssum = o.scope == 0 ? hs.ssum : 0.0;
-    c.n_samples_global = c.comm ? S_global : S;
-
-    // a7: samples
-    CKS(c.ensure(c.out_row, c.cap_out_row, sizeof(uint32_t) * (S + 1)));
-    CKS(c.ensure(c.out_cluster, c.cap_out_cluster, sizeof(uint32_t) * (S + 1)));
-    CKS(c.ensure(c.out_weight, c.cap_out_weight, sizeof(double) * (S + 1)));
-    // packed sort: ambiguous-sample entries, their chunk counts/offsets, scan scratch
-    const size_t amb_bytes = sizeof(Amb) * (S + 1), nch_bytes = sizeof(uint64_t) * (S + 1);
-    if (c.pack_h > 1) CKS(c.ensure(c.amb, c.cap_amb, amb_bytes + 2 * nch_bytes + (scan_tiles(S + 1) + 2) * 16));
-    SampleArgs sa{c.leaf_lo, leaf_kid, leaf_ord, c.leaf_moff, c.leaf_m, c.leaf_census, c.t_sorted, c.row_sorted,
-                  L, n, S, (uint32_t)o.seed, (uint32_t)(o.seed >> 32), c.kid_base, c.out_row, c.out_cluster,
-                  c.out_weight, c.leaf_U, c.pack_s, c.pack_h, c.sort_kid, c.sort_t, c.sort_row_in,
-                  (Amb *)c.amb, &c.scalars->amb_count};
-    const int tk_smp = c.stage_begin("samples");
-    CK(cudaMemsetAsync(&c.scalars->amb_count, 0, sizeof(uint32_t), st));
-    if (S) sample_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa);
-    c.launches += S ? 1 : 0;
+    // ---- segment 3: samples (a7) and the local estimate partials (a8)
+    uint64_t S = 0;
     uint32_t n_amb = 0;
-    if (S && c.pack_h > 1) {
-        CK(cudaMemcpyAsync(&n_amb, &c.scalars->amb_count, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-    }
-    if (n_amb) {
-        uint64_t *nch = (uint64_t *)((char *)c.amb + amb_bytes), *choff = nch + (S + 1), *scr = choff + (S + 1);
-        uint64_t *tot = &c.scalars->scan_total64;
-        resolve_locate_kernel<<<blocks_for(n_amb), kThreads, 0, st>>>(sa, n_amb, nch);
-        exclusive_scan<uint64_t>([nch] __device__(uint64_t i) -> uint64_t { return nch[i]; },
-                                 [choff] __device__(uint64_t i, uint64_t pre, uint64_t) { choff[i] = pre; },
-                                 (uint64_t)n_amb, scr, tot, st, &c.launches);
-        resolve_count_kernel<<<4 * c.sms, kThreads, 0, st>>>(sa, n_amb, choff, tot);
-        resolve_final_kernel<<<blocks_for(n_amb), kThreads, 0, st>>>(sa, n_amb);
-        c.launches += 3;
-    }
-    c.stage_end(tk_smp, 40 * S);
-    CK(cudaGetLastError());
+    const uint64_t eb = blocks_for(L);
+    double *part_est = nullptr, *part_met = nullptr, *red_out = nullptr;
+    uint64_t mb = 0;
+    int tk_est = -1;
+    CKS(dist_checkpoint(c, [&]() -> int {
+        DevScalars hs;
+        CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
+        CKS(sync_stream(c));
+        if (hs.err & 2) return STEM_E_CUDA;
+        if (hs.limit_err || hs.total_m >= (1ull << 32)) return STEM_E_LIMIT;
+        S = hs.total_m;
+        c.n_samples = S;
+        c.T = hs.T;
+        c.stats.ssum = o.scope == 0 ? hs.ssum : 0.0;
+        c.n_samples_global = c.comm ? S_global : S;
 
-    // a8: estimate, bound, metrics (deterministic block partials)
-    const uint64_t eb = blocks_for(L), mb = blocks_for(S);
-    const uint64_t part_cols = 2 + (uint64_t)nm;
-    const uint64_t part_doubles = 2 * eb + mb * (nm ? nm : 1) + part_cols + 16;
-    CKS(c.ensure(c.red_part, c.cap_red, sizeof(double) * part_doubles));
-    double *part_est = c.red_part, *part_met = c.red_part + 2 * eb, *red_out = part_met + mb * (nm ? nm : 1);
-    CK(cudaMemsetAsync(&c.scalars->sum_q, 0, sizeof(uint64_t), st));
-    const int tk_est = c.stage_begin("estimate");
-    EstArgs ea{c.leaf_lo, c.t_sorted, c.PS1, c.PS2, c.leaf_m, c.leaf_U, L, n, &c.scalars->sum_q, part_est};
-    if (eb) estimate_kernel<<<(unsigned)eb, kThreads, 0, st>>>(ea);
-    reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_est, eb, 2, red_out);
-    c.launches += 2;
+        CKS(c.ensure(c.out_row, c.cap_out_row, sizeof(uint32_t) * (S + 1)));
+        CKS(c.ensure(c.out_cluster, c.cap_out_cluster, sizeof(uint32_t) * (S + 1)));
+        CKS(c.ensure(c.out_weight, c.cap_out_weight, sizeof(double) * (S + 1)));
+        // packed sort: ambiguous-sample entries, their chunk counts/offsets, scan scratch
+        const size_t amb_bytes = sizeof(Amb) * (S + 1), nch_bytes = sizeof(uint64_t) * (S + 1);
+        if (c.pack_h > 1) CKS(c.ensure(c.amb, c.cap_amb, amb_bytes + 2 * nch_bytes + (scan_tiles(S + 1) + 2) * 16));
+        SampleArgs sa{c.leaf_lo, leaf_kid, leaf_ord, c.leaf_moff, c.leaf_m, c.leaf_census, c.t_sorted,
+                      c.row_sorted, L, n, S, (uint32_t)o.seed, (uint32_t)(o.seed >> 32), c.kid_base, c.out_row,
+                      c.out_cluster, c.out_weight, c.leaf_U, c.pack_s, c.pack_h, c.sort_kid, c.sort_t,
+                      c.sort_row_in, (Amb *)c.amb, &c.scalars->amb_count};
+        const int tk_smp = c.stage_begin("samples");
+        CK(cudaMemsetAsync(&c.scalars->amb_count, 0, sizeof(uint32_t), st));
+        if (S) sample_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa);
+        c.launches += S ? 1 : 0;
+        if (S && c.pack_h > 1) {
+            CK(cudaMemcpyAsync(&n_amb, &c.scalars->amb_count, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+            CKS(sync_stream(c));
+        }
+        if (n_amb) {
+            uint64_t *nch = (uint64_t *)((char *)c.amb + amb_bytes), *choff = nch + (S + 1), *scr = choff + (S + 1);
+            uint64_t *tot = &c.scalars->scan_total64;
+            resolve_locate_kernel<<<blocks_for(n_amb), kThreads, 0, st>>>(sa, n_amb, nch);
+            exclusive_scan<uint64_t>([nch] __device__(uint64_t i) -> uint64_t { return nch[i]; },
+                                     [choff] __device__(uint64_t i, uint64_t pre, uint64_t) { choff[i] = pre; },
+                                     (uint64_t)n_amb, scr, tot, st, &c.launches);
+            resolve_count_kernel<<<4 * c.sms, kThreads, 0, st>>>(sa, n_amb, choff, tot);
+            resolve_final_kernel<<<blocks_for(n_amb), kThreads, 0, st>>>(sa, n_amb);
+            c.launches += 3;
+        }
+        c.stage_end(tk_smp, 40 * S);
+        CK(cudaGetLastError());
+
+        // a8: estimate, bound, metrics (deterministic block partials)
+        mb = blocks_for(S);
+        const uint64_t part_cols = 2 + (uint64_t)nm;
+        const uint64_t part_doubles = 2 * eb + mb * (nm ? nm : 1) + part_cols + 16;
+        CKS(c.ensure(c.red_part, c.cap_red, sizeof(double) * part_doubles));
+        part_est = c.red_part;
+        part_met = c.red_part + 2 * eb;
+        red_out = part_met + mb * (nm ? nm : 1);
+        CK(cudaMemsetAsync(&c.scalars->sum_q, 0, sizeof(uint64_t), st));
+        tk_est = c.stage_begin("estimate");
+        EstArgs ea{c.leaf_lo, c.t_sorted, c.PS1, c.PS2, c.leaf_m, c.leaf_U, L, n, &c.scalars->sum_q, part_est};
+        if (eb) estimate_kernel<<<(unsigned)eb, kThreads, 0, st>>>(ea);
+        reduce_cols_kernel<<<1, kThreads, 0, st>>>(part_est, eb, 2, red_out);
+        c.launches += 2;
+        CK(cudaGetLastError());
+        return STEM_OK;
+    }()));
     if (c.comm) {
         CKS(dist_allreduce_u64(c, &c.scalars->sum_q, 1));
         CKS(dist_allreduce_f64(c, red_out, 2));
@@ -671,27 +694,39 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         c.launches += 2;
     }
     c.stage_end(tk_est, 56 * L + 12 * S * nm);
-    // a5 output records
-    CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
-    const int tk_pack = c.stage_begin("pack");
-    if (L) pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.PS1, c.PS2, c.t_sorted, c.leaf_m,
-                                                   c.leaf_census, L, n, c.kid_base, c.out_clusters);
-    c.launches++;
-    c.stage_end(tk_pack, 88 * L);
-    CK(cudaGetLastError());
-    double *est_out = red_out + 2 + nm;
-    est_finalize_kernel<<<1, 1, 0, st>>>(&c.scalars->sum_q, red_out, &c.scalars->T, z, est_out);
-    c.launches++;
-    CK(cudaGetLastError());
-    double red[2 + 64 + 2];
-    CK(cudaMemcpyAsync(red, red_out, sizeof(double) * (2 + nm + 2), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    c.est_total = red[2 + nm];
-    c.bound = red[2 + nm + 1];
-    for (uint32_t k = 0; k < nm; k++) c.host_est_metric[k] = (S || c.comm) ? red[2 + k] : 0.0;
-    c.stats.n_clusters = L;
-    c.stats.n_samples = S;
-    c.stats.ambiguous_samples = n_amb;
+    // ---- segment 4: cluster records, final scalars
+    CKS(dist_checkpoint(c, [&]() -> int {
+        CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
+        const int tk_pack = c.stage_begin("pack");
+        if (L)
+            pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.PS1, c.PS2, c.t_sorted,
+                                                            c.leaf_m, c.leaf_census, L, n, c.kid_base,
+                                                            c.out_clusters);
+        c.launches++;
+        c.stage_end(tk_pack, 88 * L);
+        CK(cudaGetLastError());
+        double *est_out = red_out + 2 + nm;
+        est_finalize_kernel<<<1, 1, 0, st>>>(&c.scalars->sum_q, red_out, &c.scalars->T, z, est_out);
+        c.launches++;
+        CK(cudaGetLastError());
+        double red[2 + 64 + 2];
+        CK(cudaMemcpyAsync(red, red_out, sizeof(double) * (2 + nm + 2), cudaMemcpyDeviceToHost, st));
+        CKS(sync_stream(c));
+        c.est_total = red[2 + nm];
+        c.bound = red[2 + nm + 1];
+        for (uint32_t k = 0; k < nm; k++) c.host_est_metric[k] = (S || c.comm) ? red[2 + k] : 0.0;
+        c.stats.n_clusters = L;
+        c.stats.n_samples = S;
+        c.stats.ambiguous_samples = n_amb;
+        c.have_mbounds = false;
+        if (o.metric_bounds && nm && !c.comm) {   // multi-GPU: metric_bounds_dist after the plan is gathered
+            const int tk_mb = c.stage_begin("metric_bounds");
+            CKS(metric_bounds_local(c, L, K, n, tr_kid, tr_t, metrics, tr_n, nm, z));
+            c.stage_end(tk_mb, (16 + 16 * (uint64_t)nm) * tr_n);
+            c.have_mbounds = true;
+        }
+        return STEM_OK;
+    }()));
     return STEM_OK;
 }
 

@@ -36,3 +36,12 @@ def assert_plans_equal(got: dict, ref: dict, metrics: bool = False):
     assert got["z"] == ref["z"] and got["eps"] == ref["eps"]
     if metrics:
         assert rel_close(got["est_metric"], ref["est_metric"])
+    if ref.get("true_metric") is not None:   # metric_bounds (R28)
+        assert got["true_metric"] is not None and got["bound_metric"] is not None
+        assert rel_close(got["true_metric"], ref["true_metric"])
+        gb, rb = np.asarray(got["bound_metric"]), np.asarray(ref["bound_metric"])
+        assert np.array_equal(np.isinf(gb), np.isinf(rb)) and np.array_equal(gb == 0, rb == 0)
+        fin = np.isfinite(rb) & (rb != 0)
+        assert rel_close(gb[fin], rb[fin])
+    elif "true_metric" in ref:
+        assert got.get("true_metric") is None

@@ -73,3 +73,34 @@ def test_product_path_has_no_oracle_dependency():
                 text = open(os.path.join(dirpath, fn)).read()
                 for pat in ("import oracle", "from oracle", "liboracle", "stemroot_oracle", "or_plan"):
                     assert pat not in text, (fn, pat)
+
+
+def test_binding_rejects_wrong_dtypes_and_shapes():
+    """the binding must not reinterpret a wrong dtype's bytes
+    (torch's default int64 ids, float32 times or metrics) -- it raises before
+    any library call; numpy integer arrays of other widths are range-checked
+    and converted, 4-byte ones viewed."""
+    import numpy as np
+    import torch
+    k = np.zeros(8, np.uint32)
+    t = np.arange(8, dtype=np.uint32)
+    with pytest.raises(TypeError):
+        sr._trace(torch.zeros(8, dtype=torch.int64), torch.zeros(8, dtype=torch.int32), 1, None)
+    with pytest.raises(TypeError):
+        sr._trace(torch.zeros(8, dtype=torch.int32), torch.zeros(8, dtype=torch.float32), 1, None)
+    with pytest.raises(TypeError):
+        sr._trace(torch.zeros(8, dtype=torch.int32), torch.zeros(8, dtype=torch.int32), 1,
+                  torch.zeros((2, 8), dtype=torch.float32))
+    with pytest.raises(TypeError):
+        sr._trace(k, t.astype(np.float64), 1, None)
+    with pytest.raises(ValueError):
+        sr._trace(k, t[:7], 1, None)
+    with pytest.raises(ValueError):
+        sr._trace(k, t, 1, np.zeros((2, 7)))
+    with pytest.raises(ValueError):
+        sr._trace(k.astype(np.int64) - 1, t, 1, None)
+    tr, dev, keep = sr._trace(k.astype(np.int64), t.astype(np.uint16), 1, np.ones((3, 8), np.float32))
+    assert (tr.n, tr.n_metrics, dev) == (8, 3, -1)
+    assert keep[0].dtype == np.uint32 and keep[1].dtype == np.uint32 and keep[2].dtype == np.float64
+    tr, _, keep = sr._trace(k.view(np.int32), t, 1, np.ones(8))
+    assert tr.n_metrics == 1 and keep[0].dtype == np.uint32

@@ -3,6 +3,7 @@ sharing cuda:0 through the loopback communicator (the same C++ SPMD code the
 NCCL communicator drives), and a real one-rank NCCL communicator.  The
 gathered plan must equal the single-GPU plan: integers bit-exact, fp64 sums
 within 1e-9 relative (their summation order depends on the rank count)."""
+import os
 import threading
 
 import numpy as np
@@ -13,6 +14,7 @@ import tracegen as G
 from parity_util import Z95, assert_plans_equal
 
 pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 @pytest.fixture(scope="module")
@@ -99,6 +101,18 @@ def test_loopback_metrics_and_empty_ranks(sr):
     assert_plans_equal(got, ref)
 
 
+@pytest.mark.parametrize("world", [2, 4])
+def test_loopback_metric_bounds(sr, world):
+    """metric_bounds (R28) across ranks: every rank's leaves are gathered, each
+    rank reads its home rows' metrics, the per-leaf sums are allreduced; the
+    totals and bounds match the single-trace oracle"""
+    sp = G.spec("C3", n=150_000)
+    kid, t, met = G.generate_np(sp)
+    ref = O.plan(kid, t, sp.n_kernels, eps=0.03, z=Z95, seed=5, metrics=met, metric_bounds=1)
+    got = _dist_plan(sr, kid, t, sp.n_kernels, world, metrics=met, eps=0.03, z=Z95, seed=5, metric_bounds=True)
+    assert_plans_equal(got, ref, metrics=True)
+
+
 def test_nccl_single_rank(sr):
     import torch
     sp = G.spec("C1")
@@ -149,3 +163,63 @@ def test_loopback_kmpp_split(sr):
     for world in (2, 3):
         got = _dist_plan(sr, kid, t, sp.n_kernels, world, eps=0.04, z=Z95, seed=77, split=2)
         assert_plans_equal(got, ref)
+
+
+def test_loopback_rank_local_error_is_agreed(sr):
+    """a failure on one rank only (here rank 1 passes n_kernels = 0,
+    STEM_E_RANGE) makes every rank return that status, instead of the healthy
+    ranks blocking in a collective."""
+    import torch
+    world = 3
+    rng = np.random.default_rng(3)
+    kid = rng.integers(0, 4, 9000).astype(np.uint32)
+    t = rng.integers(100, 5000, 9000).astype(np.uint32)
+    comms = sr.Comm.loopback(world, 0)
+    ctxs = [sr.Context(0) for _ in range(world)]
+    streams = [torch.cuda.Stream() for _ in range(world)]
+    res = [None] * world
+
+    def run(r):
+        a, b = 3000 * r, 3000 * (r + 1)
+        dk = torch.from_numpy(kid[a:b].view(np.int32)).cuda()
+        dt = torch.from_numpy(t[a:b].view(np.int32)).cuda()
+        try:
+            ctxs[r].plan_dist(comms[r], dk, dt, 0 if r == 1 else 4, a, z=Z95, stream=streams[r].cuda_stream)
+            res[r] = 0
+        except sr.StemError as e:
+            res[r] = e.status
+    th = [threading.Thread(target=run, args=(r,)) for r in range(world)]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join(timeout=120)
+    assert not any(x.is_alive() for x in th), "a rank hung"
+    assert res == [sr.STEM_E_RANGE] * world, res
+    for c in ctxs:
+        c.close()
+    for c in comms:
+        c.close()
+
+
+def test_loopback_missing_peer_times_out(tmp_path):
+    """A peer that never joins: the others give up after STEMROOT_COMM_TIMEOUT_S
+    with STEM_E_NCCL (the NCCL communicator polls ncclCommGetAsyncError with the
+    same timeout) instead of hanging."""
+    import subprocess
+    import sys
+    prog = tmp_path / "miss.py"
+    prog.write_text(
+        "import sys, threading, numpy as np, torch\n"
+        f"sys.path.insert(0, {ROOT!r})\n"
+        "import paper_conf_micro_chungnkk25_b200 as sr\n"
+        "comms = sr.Comm.loopback(2, 0)\n"
+        "ctx = sr.Context(0)\n"
+        "k = torch.zeros(100, dtype=torch.int32, device='cuda'); t = torch.arange(100, dtype=torch.int32, device='cuda')\n"
+        "try:\n"
+        "    ctx.plan_dist(comms[0], k, t, 1, 0)\n"
+        "    print('NO-ERROR')\n"
+        "except sr.StemError as e:\n"
+        "    print('STATUS', e.status)\n")
+    env = dict(os.environ, STEMROOT_COMM_TIMEOUT_S="3")
+    out = subprocess.run([sys.executable, str(prog)], env=env, capture_output=True, text=True, timeout=300)
+    assert "STATUS -5" in out.stdout, out.stdout + out.stderr

@@ -134,6 +134,27 @@ def test_host_pointers_and_metrics(ctx):
     assert_plans_equal(got, ref, metrics=True)
 
 
+@pytest.mark.parametrize("host", [False, True])
+@pytest.mark.parametrize("opts", [dict(), dict(root=False), dict(scope=2), dict(census_cap=True, eps=1e-5)])
+def test_metric_bounds(ctx, host, opts):
+    """metric_bounds (R28): true totals and bounds element by element against the
+    oracle, on columns that pin the arithmetic (t itself, an affine map, a
+    constant, an all-zero column, noise, a signed column)."""
+    rng = np.random.default_rng(17)
+    n = 50000
+    kid, t = _mixture(rng, n, 30, peaks=3, spread=0.1)
+    tf = t.astype(np.float64)
+    met = np.vstack([tf, 2.5 * tf + 1e5, np.full(n, 3.0), np.zeros(n), rng.random(n), rng.standard_normal(n)])
+    kw = dict(opts)
+    kw.setdefault("eps", 0.02)
+    got, ref = _both(ctx, kid, t, 30, metrics=met, host=host, metric_bounds=True, seed=8, **kw)
+    assert_plans_equal(got, ref, metrics=True)
+    assert got["bound_metric"][0] == pytest.approx(got["bound"], rel=1e-9)
+    assert got["bound_metric"][2] == 0.0 and got["bound_metric"][3] == 0.0 and got["true_metric"][3] == 0.0
+    off, _ = _both(ctx, kid, t, 30, metrics=met, host=host, seed=8, **kw)
+    assert off["true_metric"] is None and off["bound_metric"] is None
+
+
 def test_determinism(ctx):
     rng = np.random.default_rng(13)
     kid, t = _mixture(rng, 200000, 64)
@@ -162,7 +183,7 @@ def test_configs(ctx, name, n):
 def test_config_c3_with_metrics(ctx):
     sp = G.spec("C3", n=2_000_000)
     kid, t, met = G.generate_np(sp)
-    got, ref = _both(ctx, kid, t, sp.n_kernels, metrics=met, eps=sp.eps, seed=2)
+    got, ref = _both(ctx, kid, t, sp.n_kernels, metrics=met, eps=sp.eps, seed=2, metric_bounds=True)
     assert_plans_equal(got, ref, metrics=True)
 
 
@@ -197,7 +218,7 @@ def test_config_c3_full_size_with_metrics(ctx):
     (the e2e launch), element by element against the oracle."""
     sp = G.spec("C3")
     kid, t, met = G.generate_np(sp)
-    got, ref = _both(ctx, kid, t, sp.n_kernels, metrics=met, host=True, eps=sp.eps, seed=12345)
+    got, ref = _both(ctx, kid, t, sp.n_kernels, metrics=met, host=True, eps=sp.eps, seed=12345, metric_bounds=True)
     assert_plans_equal(got, ref, metrics=True)
 
 
