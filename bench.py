@@ -50,7 +50,42 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--split", type=int, default=0, choices=[0, 1, 2], help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26), 2 k-means++ seeded Lloyd (R27)")
+    ap.add_argument("--metric-bounds", action="store_true", help="also true totals and bounds of the metric columns (R28)")
+    ap.add_argument("--dry-launch", action="store_true", help="print the torchrun command --gpus N would run, and exit")
     return ap.parse_args()
+
+
+def launch(a):
+    """--gpus N without a torchrun environment: re-exec this script under torchrun
+    with N ranks (one per GPU, rendezvous on 127.0.0.1).  Under torchrun the rank
+    count must equal --gpus.  Our arm needs N visible CUDA devices and fails
+    loudly otherwise (never a silent 1-GPU run)."""
+    ws = os.environ.get("WORLD_SIZE")
+    if ws is not None:
+        if int(ws) != a.gpus:
+            print(json.dumps({"metric": METRIC, "error": f"WORLD_SIZE={ws} but --gpus {a.gpus}"}), flush=True)
+            sys.exit(2)
+        return
+    if a.gpus <= 1:
+        return
+    if a.impl == "ours" and not a.dry_launch:
+        import torch
+        have = torch.cuda.device_count()
+        if have < a.gpus:
+            print(json.dumps({"metric": METRIC, "error": f"--gpus {a.gpus} requested but {have} CUDA devices are "
+                              "visible"}), flush=True)
+            sys.exit(2)
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + \
+        [x for x in sys.argv[1:] if x != "--dry-launch"]
+    if a.dry_launch:
+        print(json.dumps({"launch": cmd}), flush=True)
+        sys.exit(0)
+    sys.exit(subprocess.call(cmd))
 
 
 def load_peaks():
@@ -138,7 +173,8 @@ def run_reference(a):
     times = []
     for i in range(a.warmup + a.steps):
         t0 = time.perf_counter()
-        oracle.plan(kid, t, sp.n_kernels, eps=eps, z=z, seed=i, metrics=met, split=a.split)
+        oracle.plan(kid, t, sp.n_kernels, eps=eps, z=z, seed=i, metrics=met, split=a.split,
+                    metric_bounds=int(a.metric_bounds))
         dt = time.perf_counter() - t0
         if i >= a.warmup:
             times.append(dt)
@@ -198,12 +234,15 @@ def run_ours(a):
     ctx = sr.Context(local)
     stream = torch.cuda.current_stream(dev)
 
-    def step(timing=False):
-        if comm is not None:
-            return ctx.plan_dist(comm, kid, tt, sp.n_kernels, row0, eps=eps, conf=a.conf, metrics=met, seed=12345,
-                                 to_host=False, stream=stream.cuda_stream, split=a.split)
-        return ctx.plan(kid, tt, sp.n_kernels, eps=eps, conf=a.conf, metrics=met, seed=12345, to_host=False,
-                        stream=stream.cuda_stream, split=a.split)
+    def step():
+        # one whole plan through the C ABI, ending with the plan in host memory
+        # (rows/s up to "the plan on host"); rank 0 gets the plan
+        hp = ctx.plan_host_raw(kid, tt, sp.n_kernels, eps=eps, conf=a.conf, metrics=met, comm=comm,
+                               global_row_base=row0, seed=12345, stream=stream.cuda_stream, split=a.split,
+                               metric_bounds=a.metric_bounds)
+        nb = hp.nbytes()
+        hp.close()
+        return nb
 
     for _ in range(a.warmup):
         step()
@@ -220,8 +259,9 @@ def run_ours(a):
     ev1 = torch.cuda.Event(enable_timing=True)
     ev0.record(stream)
     launches = 0
+    plan_bytes = 0
     for _ in range(a.steps):
-        step()
+        plan_bytes = step()
         for s in ctx.stage_times():
             g = stages.setdefault(s["name"], {"ms": 0.0, "bytes": 0, "launches": 0, "count": 0})
             for k in ("ms", "bytes", "launches", "count"):
@@ -241,6 +281,13 @@ def run_ours(a):
     st = ctx.stats()
     dplan = ctx.device_plan()
     ms_per_step = elapsed_ms / a.steps
+    # rows each rank grouped and clustered after the kernel-id exchange (SURVEY §8(e) skew caveat)
+    owned = [int(st["owned_rows"])]
+    if world > 1:
+        owned = [None] * world
+        torch.distributed.all_gather_object(owned, int(st["owned_rows"]))
+    balance = {"rows_per_rank": owned, "max_over_mean": max(owned) / (sum(owned) / len(owned)) if sum(owned) else 1.0,
+               "comm_ranks": int(st["world"])}
     value = sp.n * a.steps / (elapsed_ms / 1e3)
 
     # roofline of the dominant kernel (largest share of the step)
@@ -272,8 +319,10 @@ def run_ours(a):
                    "sort_key_bits": st["key_bits"], "sort_passes": st["sort_passes"],
                    "sort_row_bits_in_key": st["pack_bits"], "ambiguous_samples": st["ambiguous_samples"],
                    "split_chunks": st["split_chunks"], "split_scanned": st["split_scanned"],
-                   "root_levels": st["levels"], "clusters": dplan["n_clusters"], "samples": dplan["n_samples"],
-                   "active_rows_over_levels": st["active_rows"]},
+                   "root_levels": st["levels"], "clusters": st["n_clusters"], "samples": st["n_samples"],
+                   "active_rows_over_levels": st["active_rows"], "plan_to_host": True,
+                   "plan_bytes_d2h": plan_bytes, "metric_bounds": bool(a.metric_bounds)},
+        "balance": balance,
         "clocks": ck,
         "gpu_launches": launches,
         "roofline": roofline,
@@ -297,9 +346,10 @@ def run_ours(a):
         def e2e_step():
             if comm is not None:
                 return ctx.plan_dist(comm, hk, ht, sp.n_kernels, row0, eps=eps, conf=a.conf, metrics=hm,
-                                     seed=12345, stream=stream.cuda_stream, split=a.split)
+                                     seed=12345, stream=stream.cuda_stream, split=a.split,
+                                     metric_bounds=a.metric_bounds)
             return ctx.plan(hk, ht, sp.n_kernels, eps=eps, conf=a.conf, metrics=hm, seed=12345,
-                            stream=stream.cuda_stream, split=a.split)
+                            stream=stream.cuda_stream, split=a.split, metric_bounds=a.metric_bounds)
         p = e2e_step()
         torch.cuda.synchronize()
         if world > 1:
@@ -313,7 +363,7 @@ def run_ours(a):
             torch.distributed.all_reduce(tm, op=torch.distributed.ReduceOp.MAX)
             e2e_s = float(tm.item())
         d2h = 0 if p is None else p["clusters"].nbytes + p["sample_row"].nbytes + p["sample_cluster"].nbytes + \
-            p["sample_weight"].nbytes + 8 * (6 + nm)
+            p["sample_weight"].nbytes + 8 * (6 + (3 if a.metric_bounds else 1) * nm)
         line["e2e"] = {"value": sp.n / e2e_s, "unit": UNIT,
                        "h2d_bytes_per_step": sp.n * (8 + 8 * nm), "d2h_bytes_per_step": int(d2h),
                        "ms_per_step": e2e_s * 1e3, "steps": e2e_steps}
@@ -327,7 +377,8 @@ def run_ours(a):
         t_np = tt[:m].cpu().numpy().view(np.uint32)
         m_np = met[:, :m].cpu().numpy() if nm else None
         t0 = time.perf_counter()
-        oracle.plan(k_np, t_np, sp.n_kernels, eps=eps, z=dplan["z"], seed=12345, metrics=m_np, split=a.split)
+        oracle.plan(k_np, t_np, sp.n_kernels, eps=eps, z=dplan["z"], seed=12345, metrics=m_np, split=a.split,
+                    metric_bounds=int(a.metric_bounds))
         cs = time.perf_counter() - t0
         line["cpu_baseline"] = {"value": m / cs, "unit": UNIT, "cores": 1, "kind": "oracle",
                                 "sample": f"first {m} rows of {a.config} ({cs:.1f} s, single-threaded C oracle)",
@@ -343,6 +394,7 @@ def run_ours(a):
 
 def main():
     a = parse()
+    launch(a)
     if a.impl == "reference":
         run_reference(a)
     else:

@@ -165,6 +165,11 @@ typedef struct stem_stats {
     uint32_t reserved0;
     uint64_t split_chunks;     /* 32-row chunks of big clusters bounded, summed over ROOT levels   */
     uint64_t split_scanned;    /* of those, chunks scanned row by row (the rest pruned exactly)   */
+    uint64_t owned_rows;       /* rows this ctx grouped and clustered: n on one GPU; in
+                                  stem_root_plan_dist the rows of the kernels this rank owns
+                                  after the exchange (max/mean over ranks = the imbalance)     */
+    uint32_t world;            /* ranks of the communicator of the last plan (1 on one GPU)    */
+    uint32_t reserved1;
 } stem_stats;
 
 /* Per-stage device time of the last plan (stem_ctx_enable_timing).  bytes is

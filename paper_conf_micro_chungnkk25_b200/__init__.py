@@ -110,7 +110,8 @@ class stem_stats(C.Structure):
                 ("kernel_launches", C.c_uint32), ("active_rows", C.c_uint64), ("n_clusters", C.c_uint64),
                 ("n_samples", C.c_uint64), ("ssum", C.c_double), ("pack_bits", C.c_uint32),
                 ("ambiguous_samples", C.c_uint32), ("coarse_bases", C.c_uint32), ("reserved0", C.c_uint32),
-                ("split_chunks", C.c_uint64), ("split_scanned", C.c_uint64)]
+                ("split_chunks", C.c_uint64), ("split_scanned", C.c_uint64), ("owned_rows", C.c_uint64),
+                ("world", C.c_uint32), ("reserved1", C.c_uint32)]
 
 
 class stem_stage_time(C.Structure):
@@ -314,6 +315,40 @@ class Comm:
             pass
 
 
+class HostPlan:
+    """A library-allocated stem_plan (host memory), freed by close() / stem_plan_free."""
+
+    def __init__(self, ptr):
+        self._p = ptr
+
+    @property
+    def plan(self):
+        return self._p.contents if self._p else None
+
+    def nbytes(self) -> int:
+        """bytes of the plan's arrays (what the library copied to the host)"""
+        p = self.plan
+        if p is None:
+            return 0
+        nmb = 3 if p.true_metric else 1
+        return (int(p.n_clusters) * CLUSTER_DTYPE.itemsize + int(p.n_samples) * (4 + 4 + 8) +
+                8 * nmb * int(p.n_metrics) + 8 * 6)
+
+    def to_numpy(self) -> dict:
+        return _plan_to_numpy(self.plan)
+
+    def close(self):
+        if self._p:
+            lib().stem_plan_free(self._p)
+            self._p = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 class Context:
     """A stem_ctx: device workspace reused across plans (stem_ctx_create)."""
 
@@ -369,6 +404,29 @@ class Context:
         res = _plan_to_numpy(out.contents)
         lib().stem_plan_free(out)
         return res
+
+    def plan_host_raw(self, kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95,
+                      metrics=None, comm: "Comm" = None, global_row_base: int = 0, **kw) -> "HostPlan":
+        """stem_root_plan_ctx (or _dist with comm) with the host plan kept as the
+        library allocated it (no numpy conversion): a HostPlan whose close()
+        calls stem_plan_free.  On ranks other than 0 of a dist plan it is empty."""
+        opt = {k: kw.pop(k) for k in list(kw) if k in ("seed", "z", "scope", "root", "clamp_in_split",
+                                                          "census_cap", "split", "metric_bounds", "stream")}
+        if kw:
+            raise TypeError(f"unknown options {sorted(kw)}")
+        tr, dev, keep = _trace(kernel_id, exec_ns, n_kernels, metrics, allow_empty=comm is not None)
+        o = _opts(opt.get("seed", 0), opt.get("z", 0.0), opt.get("scope", 0), opt.get("root", True),
+                  opt.get("clamp_in_split", True), opt.get("census_cap", False), opt.get("split", 0),
+                  opt.get("metric_bounds", False), opt.get("stream"), dev)
+        out = C.POINTER(stem_plan)()
+        if comm is None:
+            st = lib().stem_root_plan_ctx(self._h, C.byref(tr), eps, conf, C.byref(o), C.byref(out))
+        else:
+            st = lib().stem_root_plan_dist(self._h, comm._h, C.byref(tr), global_row_base, eps, conf, C.byref(o),
+                                           C.byref(out))
+        _check(st, "stem_root_plan_ctx" if comm is None else "stem_root_plan_dist")
+        del keep
+        return HostPlan(out)
 
     def device_plan(self) -> dict:
         v = stem_device_plan()

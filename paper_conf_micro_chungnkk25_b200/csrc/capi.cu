@@ -176,6 +176,8 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
     c.eps = eps;
     c.z = z;
     c.stats.kernel_launches = c.launches;
+    c.stats.owned_rows = n;
+    c.stats.world = 1;
     if (c.timing.on) {
         CK(cudaStreamSynchronize(c.stream));
         c.timing.finish();

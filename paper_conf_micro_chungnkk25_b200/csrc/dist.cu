@@ -764,6 +764,8 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
     // cluster indices): stem_ctx_device_plan then describes exactly the buffers it holds
     c.stats.n_clusters = Lg;
     c.stats.n_samples = Sg;
+    c.stats.owned_rows = R;
+    c.stats.world = (uint32_t)W;
     return STEM_OK;
 }
 

@@ -29,3 +29,41 @@ def test_reference_arm_split_rule():
                                   cwd=ROOT, timeout=300).decode().strip().splitlines()
     d = json.loads(out[-1])
     assert d["config"]["split"].startswith("k-means++") and d["value"] > 0
+
+
+def test_gpus_flag_launches_ranks_reference_arm():
+    """--gpus N without a torchrun environment re-execs bench.py under torchrun
+    with N ranks (127.0.0.1 rendezvous); rank 0 alone prints the reference line,
+    which reports the rank count (CPU-only: the reference arm needs no GPU)."""
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--config", "C1",
+                          "--gpus", "2", "--steps", "1", "--warmup", "0", "--ref-sample-rows", "5000"],
+                         cwd=ROOT, timeout=600, capture_output=True, text=True)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.strip().splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["impl"] == "reference"
+
+
+def test_gpus_flag_fails_loudly_without_devices():
+    """our arm never silently runs on fewer GPUs than --gpus asks for"""
+    import torch
+    if torch.cuda.device_count() >= 2:
+        import pytest
+        pytest.skip("enough GPUs here")
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "1"], cwd=ROOT,
+                         timeout=300, capture_output=True, text=True)
+    assert out.returncode != 0
+    assert "CUDA devices" in out.stdout
+
+
+def test_gpus_flag_dry_launch_and_world_mismatch():
+    out = subprocess.check_output([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "8", "--dry-launch"],
+                                  cwd=ROOT, timeout=300).decode()
+    cmd = json.loads(out.strip().splitlines()[-1])["launch"]
+    assert "torch.distributed.run" in cmd and "--nproc-per-node=8" in cmd and "--master-addr=127.0.0.1" in cmd
+    assert cmd[-4:] == ["--gpus", "8"] or "--gpus" in cmd
+    env = dict(os.environ, WORLD_SIZE="2", RANK="0", LOCAL_RANK="0")
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--impl", "reference"],
+                         cwd=ROOT, timeout=300, capture_output=True, text=True, env=env)
+    assert out.returncode != 0 and "WORLD_SIZE=2" in out.stdout
