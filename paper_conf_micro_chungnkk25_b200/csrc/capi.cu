@@ -72,6 +72,7 @@ void Ctx::release() {
     dfree(red_part, cap_red); dfree(out_clusters, cap_out_cl); dfree(out_row, cap_out_row);
     dfree(out_cluster, cap_out_cluster); dfree(out_weight, cap_out_weight);
     dfree(big_ent, cap_big_ent); dfree(big_part, cap_big_part); dfree(big_thr, cap_big_thr);
+    dfree(big_base, cap_big_base);
     dfree(part_cnt, cap_part_cnt); dfree(dist_cnt, cap_dist_cnt);
     for (int i = 0; i < 3; i++) { dfree(xfer_u32[i], cap_xfer_u32[i]); dfree(recv_u32[i], cap_recv_u32[i]); }
     dfree(xfer_f64, cap_xfer_f64); dfree(xfer_f64b, cap_xfer_f64b); dfree(red_part2, cap_red2);

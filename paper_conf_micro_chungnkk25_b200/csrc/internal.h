@@ -182,6 +182,7 @@ struct Ctx {
     uint64_t *cut_SL = nullptr; size_t cap_cut_SL = 0;
     u128 *cut_QL = nullptr; size_t cap_cut_QL = 0;
     void *big_ent = nullptr, *big_part = nullptr, *big_thr = nullptr;
+    uint64_t *big_base = nullptr; size_t cap_big_base = 0;   // v2: per-cluster sum of t before lo
     size_t cap_big_ent = 0, cap_big_part = 0, cap_big_thr = 0;
     uint64_t *cnt_sz = nullptr; size_t cap_cntsz = 0;
     uint32_t *flags = nullptr; size_t cap_flags = 0;   // leaf-start bitmap: bit i & 31 of word i >> 5
