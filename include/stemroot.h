@@ -169,7 +169,9 @@ typedef struct stem_stats {
                                   stem_root_plan_dist the rows of the kernels this rank owns
                                   after the exchange (max/mean over ranks = the imbalance)     */
     uint32_t world;            /* ranks of the communicator of the last plan (1 on one GPU)    */
-    uint32_t reserved1;
+    uint32_t fused_exchange;   /* 1: the last stem_root_plan_dist stored every row straight into
+                                  its owner's receive window (peer memory over NVLink, CUDA IPC);
+                                  0: grouped send/recv (STEMROOT_DIST_P2P=0, or no peer access) */
 } stem_stats;
 
 /* Per-stage device time of the last plan (stem_ctx_enable_timing).  bytes is

@@ -4,7 +4,9 @@
 #include <cmath>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <new>
+#include <utility>
 
 #include "internal.h"
 
@@ -72,7 +74,7 @@ void Ctx::release() {
     dfree(red_part, cap_red); dfree(out_clusters, cap_out_cl); dfree(out_row, cap_out_row);
     dfree(out_cluster, cap_out_cluster); dfree(out_weight, cap_out_weight);
     dfree(big_ent, cap_big_ent); dfree(big_part, cap_big_part); dfree(big_thr, cap_big_thr);
-    dfree(big_base, cap_big_base);
+    dfree(peer_dst, cap_peer_dst);
     dfree(part_cnt, cap_part_cnt); dfree(dist_cnt, cap_dist_cnt);
     for (int i = 0; i < 3; i++) { dfree(xfer_u32[i], cap_xfer_u32[i]); dfree(recv_u32[i], cap_recv_u32[i]); }
     dfree(xfer_f64, cap_xfer_f64); dfree(xfer_f64b, cap_xfer_f64b); dfree(red_part2, cap_red2);
@@ -187,27 +189,104 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
     return STEM_OK;
 }
 
-static int to_host(Ctx &c, stem_plan **out) {
-    stem_plan *p = (stem_plan *)calloc(1, sizeof(stem_plan));
-    if (!p) return STEM_E_NOMEM;
-    const uint64_t L = c.n_leaves, S = c.n_samples;
-    p->n_clusters = L;
-    p->n_samples = S;
-    p->clusters = (stem_cluster *)malloc(sizeof(stem_cluster) * (L ? L : 1));
-    p->sample_row = (uint32_t *)malloc(sizeof(uint32_t) * (S ? S : 1));
-    p->sample_cluster = (uint32_t *)malloc(sizeof(uint32_t) * (S ? S : 1));
-    p->sample_weight = (double *)malloc(sizeof(double) * (S ? S : 1));
-    p->n_metrics = c.n_metrics;
-    p->est_metric = (double *)calloc(c.n_metrics ? c.n_metrics : 1, sizeof(double));
-    if (c.have_mbounds) {
-        p->true_metric = (double *)calloc(c.n_metrics, sizeof(double));
-        p->bound_metric = (double *)calloc(c.n_metrics, sizeof(double));
+// ---------------------------------------------------------------- host plans
+// A plan is one header + one host block holding every array.  The block is
+// page-locked (cudaMallocHost) so the plan's device-to-host copies run at full
+// PCIe / C2C speed; freed blocks are kept in a small process-wide pool and
+// reused by later plans, since pinning memory costs far more than copying it.
+struct PlanBlock {
+    stem_plan pub;     // first member: stem_plan_free casts back
+    void *mem;
+    size_t bytes;
+    bool pinned;
+};
+
+struct PinnedPool {
+    std::mutex m;
+    std::vector<std::pair<void *, size_t>> free_blocks;   // (block, bytes)
+    static constexpr size_t kKeep = 4;
+};
+
+static PinnedPool &pinned_pool() {
+    static PinnedPool *p = new PinnedPool();   // never destroyed: blocks may outlive static teardown
+    return *p;
+}
+
+static void *pool_acquire(size_t bytes, size_t &got, bool &pinned) {
+    {
+        PinnedPool &pp = pinned_pool();
+        std::lock_guard<std::mutex> g(pp.m);
+        int bi = -1;
+        for (size_t i = 0; i < pp.free_blocks.size(); i++) {
+            const size_t b = pp.free_blocks[i].second;
+            if (b >= bytes && b <= 4 * bytes + (1u << 20) && (bi < 0 || b < pp.free_blocks[bi].second)) bi = (int)i;
+        }
+        if (bi >= 0) {
+            void *m = pp.free_blocks[bi].first;
+            got = pp.free_blocks[bi].second;
+            pp.free_blocks.erase(pp.free_blocks.begin() + bi);
+            pinned = true;
+            return m;
+        }
     }
-    if (!p->clusters || !p->sample_row || !p->sample_cluster || !p->sample_weight || !p->est_metric ||
-        (c.have_mbounds && (!p->true_metric || !p->bound_metric))) {
-        stem_plan_free(p);
+    const size_t want = bytes + bytes / 8 + 4096;   // headroom: the next plan of the same trace reuses it
+    void *m = nullptr;
+    if (cudaMallocHost(&m, want) == cudaSuccess) {
+        got = want;
+        pinned = true;
+        return m;
+    }
+    cudaGetLastError();
+    pinned = false;
+    got = bytes;
+    return malloc(bytes);
+}
+
+static void pool_release(void *m, size_t bytes, bool pinned) {
+    if (!m) return;
+    if (!pinned) {
+        free(m);
+        return;
+    }
+    PinnedPool &pp = pinned_pool();
+    std::lock_guard<std::mutex> g(pp.m);
+    if (pp.free_blocks.size() < PinnedPool::kKeep) {
+        pp.free_blocks.emplace_back(m, bytes);
+        return;
+    }
+    cudaFreeHost(m);
+}
+
+static int to_host(Ctx &c, stem_plan **out) {
+    PlanBlock *pb = (PlanBlock *)calloc(1, sizeof(PlanBlock));
+    if (!pb) return STEM_E_NOMEM;
+    stem_plan *p = &pb->pub;
+    const uint64_t L = c.n_leaves, S = c.n_samples, nm = c.n_metrics;
+    auto al = [](size_t x) { return (x + 63) & ~(size_t)63; };
+    const size_t o_cl = 0, o_row = o_cl + al(sizeof(stem_cluster) * L), o_scl = o_row + al(sizeof(uint32_t) * S),
+                 o_w = o_scl + al(sizeof(uint32_t) * S), o_est = o_w + al(sizeof(double) * S),
+                 o_tru = o_est + al(sizeof(double) * (nm ? nm : 1)), o_bnd = o_tru + al(sizeof(double) * nm),
+                 total = o_bnd + al(sizeof(double) * nm);
+    size_t got = 0;
+    bool pinned = false;
+    char *mem = (char *)pool_acquire(total, got, pinned);
+    if (!mem) {
+        free(pb);
         return STEM_E_NOMEM;
     }
+    pb->mem = mem;
+    pb->bytes = got;
+    pb->pinned = pinned;
+    p->n_clusters = L;
+    p->n_samples = S;
+    p->clusters = (stem_cluster *)(mem + o_cl);
+    p->sample_row = (uint32_t *)(mem + o_row);
+    p->sample_cluster = (uint32_t *)(mem + o_scl);
+    p->sample_weight = (double *)(mem + o_w);
+    p->n_metrics = c.n_metrics;
+    p->est_metric = (double *)(mem + o_est);
+    p->true_metric = c.have_mbounds ? (double *)(mem + o_tru) : nullptr;
+    p->bound_metric = c.have_mbounds ? (double *)(mem + o_bnd) : nullptr;
     cudaStream_t st = c.stream;
     cudaError_t e = cudaSuccess;
     if (L) e = cudaMemcpyAsync(p->clusters, c.out_clusters, sizeof(stem_cluster) * L, cudaMemcpyDeviceToHost, st);
@@ -417,14 +496,9 @@ int stem_ctx_stage_times(const stem_ctx *ctx, stem_stage_time *out, uint32_t cap
 
 void stem_plan_free(stem_plan *p) {
     if (!p) return;
-    free(p->clusters);
-    free(p->sample_row);
-    free(p->sample_cluster);
-    free(p->sample_weight);
-    free(p->est_metric);
-    free(p->true_metric);
-    free(p->bound_metric);
-    free(p);
+    sr::PlanBlock *pb = reinterpret_cast<sr::PlanBlock *>(p);   // every plan is a PlanBlock (to_host)
+    sr::pool_release(pb->mem, pb->bytes, pb->pinned);
+    free(pb);
 }
 
 const char *stem_strerror(int status) {

@@ -56,6 +56,11 @@ class Comm {
     // host arrays: all[r * count + i] = rank r's mine[i]
     virtual int allgather_host(const uint64_t *mine, size_t count, uint64_t *all, cudaStream_t st) = 0;
     // device buffers; counts/displacements are host arrays of `world` elements (units of elem bytes)
+    // Collective: every rank passes nptr device buffers of its own; peers[r *
+    // nptr + i] receives rank r's buffer i as a pointer this rank's kernels can
+    // store to (peer memory over NVLink; its own buffers for r == rank).
+    // STEM_E_CUDA (on every rank) when peer access is not possible.
+    virtual int window(void *const *mine, int nptr, void **peers, cudaStream_t st) = 0;
     virtual int alltoallv(const void *send, const uint64_t *scnt, const uint64_t *sdsp, void *recv,
                           const uint64_t *rcnt, const uint64_t *rdsp, size_t elem, cudaStream_t st) = 0;
 };
@@ -111,9 +116,62 @@ class NcclComm : public Comm {
     ncclComm_t comm = nullptr;
     uint64_t *stage = nullptr;
     size_t stage_cap = 0;
+    struct IpcMap {
+        cudaIpcMemHandle_t h;
+        void *p = nullptr;
+    };
+    std::vector<IpcMap> ipc;   // [world * nptr] peer buffers opened by CUDA IPC (cached by handle)
     ~NcclComm() override {
+        for (auto &m : ipc)
+            if (m.p) cudaIpcCloseMemHandle(m.p);
         if (comm) nccl().commDestroy(comm);
         if (stage) cudaFree(stage);
+    }
+    // CUDA IPC: handles allgathered, peers' buffers opened once per allocation
+    int window(void *const *mine, int nptr, void **peers, cudaStream_t st) override {
+        if (broken) return STEM_E_NCCL;
+        constexpr int HW = (int)(sizeof(cudaIpcMemHandle_t) / 8);   // 64-byte handle = 8 words
+        std::vector<uint64_t> my((size_t)nptr * HW + 1, 0), all((size_t)world * (nptr * HW + 1));
+        int st_local = STEM_OK;
+        for (int i = 0; i < nptr && st_local == STEM_OK; i++) {
+            cudaIpcMemHandle_t h;
+            if (cudaIpcGetMemHandle(&h, mine[i]) != cudaSuccess) { cudaGetLastError(); st_local = STEM_E_CUDA; }
+            else memcpy(&my[(size_t)i * HW], &h, sizeof(h));
+        }
+        my[(size_t)nptr * HW] = (uint64_t)(int64_t)st_local;
+        CKS(allgather_host(my.data(), my.size(), all.data(), st));
+        for (int r = 0; r < world; r++)
+            if ((int64_t)all[(size_t)r * my.size() + nptr * HW] != STEM_OK) return STEM_E_CUDA;
+        if (ipc.size() != (size_t)world * nptr) {
+            for (auto &m : ipc)
+                if (m.p) cudaIpcCloseMemHandle(m.p);
+            ipc.assign((size_t)world * nptr, IpcMap{});
+        }
+        for (int r = 0; r < world && st_local == STEM_OK; r++)
+            for (int i = 0; i < nptr; i++) {
+                if (r == rank) { peers[(size_t)r * nptr + i] = mine[i]; continue; }
+                IpcMap &m = ipc[(size_t)r * nptr + i];
+                const void *hr = &all[(size_t)r * my.size() + (size_t)i * HW];
+                if (!m.p || memcmp(&m.h, hr, sizeof(m.h)) != 0) {
+                    if (m.p) cudaIpcCloseMemHandle(m.p);
+                    m.p = nullptr;
+                    memcpy(&m.h, hr, sizeof(m.h));
+                    if (cudaIpcOpenMemHandle(&m.p, m.h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+                        cudaGetLastError();
+                        m.p = nullptr;
+                        st_local = STEM_E_CUDA;
+                        break;
+                    }
+                }
+                peers[(size_t)r * nptr + i] = m.p;
+            }
+        // every rank learns whether every rank could open every peer
+        uint64_t flag = (uint64_t)(int64_t)st_local;
+        std::vector<uint64_t> flags(world);
+        CKS(allgather_host(&flag, 1, flags.data(), st));
+        for (int r = 0; r < world; r++)
+            if ((int64_t)flags[r] != STEM_OK) return STEM_E_CUDA;
+        return STEM_OK;
     }
     void fail() {   // abort the communicator: queued NCCL kernels terminate, later calls fail fast
         if (comm && nccl().commAbort) nccl().commAbort(comm);
@@ -189,8 +247,9 @@ struct LoopGroup {
     uint64_t gen = 0;
     std::vector<const void *> ptr;
     std::vector<const uint64_t *> h0, h1;
+    std::vector<void *const *> wptr;
     bool broken = false;
-    explicit LoopGroup(int w) : world(w), ptr(w), h0(w), h1(w) {}
+    explicit LoopGroup(int w) : world(w), ptr(w), h0(w), h1(w), wptr(w) {}
     // false when a member did not arrive within comm_timeout_s() (the group is then broken)
     bool barrier() {
         std::unique_lock<std::mutex> l(m);
@@ -259,6 +318,15 @@ class LoopComm : public Comm {
         CK(cudaStreamSynchronize(st));
         return STEM_OK;
     }
+    // the ranks share one device: a peer's buffer is its plain device pointer
+    int window(void *const *mine, int nptr, void **peers, cudaStream_t) override {
+        g->wptr[rank] = mine;
+        if (!g->barrier()) return STEM_E_NCCL;
+        for (int r = 0; r < world; r++)
+            for (int i = 0; i < nptr; i++) peers[(size_t)r * nptr + i] = g->wptr[r][i];
+        if (!g->barrier()) return STEM_E_NCCL;
+        return STEM_OK;
+    }
     int allgather_host(const uint64_t *mine, size_t count, uint64_t *all, cudaStream_t) override {
         g->h0[rank] = mine;
         if (!g->barrier()) return STEM_E_NCCL;
@@ -287,6 +355,14 @@ class LoopComm : public Comm {
         return STEM_OK;
     }
 };
+
+// STEMROOT_DIST_P2P=0: the kernel-id exchange by grouped send/recv instead of
+// the fused scatter into peer receive windows
+static bool dist_p2p() {
+    static int v = -1;
+    if (v < 0) v = (getenv("STEMROOT_DIST_P2P") && getenv("STEMROOT_DIST_P2P")[0] == '0') ? 0 : 1;
+    return v == 1;
+}
 
 int sync_stream(Ctx &c) {
     if (c.comm) return c.comm->wait(c.stream);
@@ -375,8 +451,20 @@ __global__ void __launch_bounds__(kPartThreads) part_count_kernel(PartArgs a, ui
     for (int d = threadIdx.x; d < a.world; d += kPartThreads) cnt[(uint64_t)d * ntiles + blockIdx.x] = h[d];
 }
 
+// Fused exchange: the destinations' receive windows (peer device memory over
+// NVLink / NVSwitch, or the other loopback ranks' buffers on this GPU) and, per
+// destination d, delta[d] = (my first row in d's window) - (the start of d's
+// segment in my partition order).  The scatter stores each row straight into
+// its owner's window: no local staging, no send/recv pass.
+struct PeerDst {
+    uint32_t *kid[kMaxWorld], *t[kMaxWorld], *row[kMaxWorld];
+    int64_t delta[kMaxWorld];
+};
+
 // stable: element order within each destination is preserved (warp-striped ranking)
-__global__ void __launch_bounds__(kPartThreads) part_scatter_kernel(PartArgs a, uint64_t ntiles, const uint64_t *off) {
+template <bool PEER>
+__global__ void __launch_bounds__(kPartThreads) part_scatter_kernel(PartArgs a, uint64_t ntiles, const uint64_t *off,
+                                                                   const PeerDst *__restrict__ pd) {
     constexpr int NW = kPartThreads / 32;
     __shared__ uint32_t wh[NW][kMaxWorld];
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
@@ -418,11 +506,19 @@ __global__ void __launch_bounds__(kPartThreads) part_scatter_kernel(PartArgs a, 
         if (i >= a.n) continue;
         const int d = dst[j];
         const uint64_t pos = off[(uint64_t)d * ntiles + blockIdx.x] + wh[w][d] + rank[j];
+        if (PEER) {
+            const uint64_t rp = (uint64_t)((int64_t)pos + pd->delta[d]);
+            pd->kid[d][rp] = a.in0[i];
+            pd->t[d][rp] = a.in1[i];
+            pd->row[d][rp] = (uint32_t)(a.in2_add + i);
+            continue;
+        }
         if (a.out0) a.out0[pos] = a.in0[i];
         if (a.out1) a.out1[pos] = a.in1[i];
         if (a.out2) a.out2[pos] = (uint32_t)(a.in2_add + i);
         if (a.outw) a.outw[pos] = a.inw[i];
     }
+    if (PEER) __threadfence_system();   // the stores are visible to the owners before the barrier
 }
 
 __global__ void part_displs_kernel(const uint64_t *off, uint64_t ntiles, int world, uint64_t *displs) {
@@ -430,15 +526,18 @@ __global__ void part_displs_kernel(const uint64_t *off, uint64_t ntiles, int wor
     if (d <= world) displs[d] = off[(uint64_t)d * ntiles];
 }
 
-// Runs the partition; host scnt/sdsp get per-destination counts and displacements.
-static int partition(Ctx &c, PartArgs &a, uint64_t *scnt, uint64_t *sdsp) {
+// Runs the partition; host scnt/sdsp get per-destination counts and
+// displacements.  pd != NULL: the rows are stored into the owners' windows
+// instead (partition_peer), after the counts are known everywhere.
+static int partition_count(Ctx &c, PartArgs &a, uint64_t *scnt, uint64_t *sdsp, uint64_t &ntiles) {
     cudaStream_t st = c.stream;
     const int W = a.world;
+    ntiles = 0;
     if (a.n == 0) {
         for (int d = 0; d < W; d++) scnt[d] = sdsp[d] = 0;
         return STEM_OK;
     }
-    const uint64_t ntiles = (a.n + kPartTile - 1) / kPartTile;
+    ntiles = (a.n + kPartTile - 1) / kPartTile;
     const uint64_t cells = (uint64_t)W * ntiles;
     CKS(c.ensure(c.part_cnt, c.cap_part_cnt, sizeof(uint64_t) * (cells + 1 + kMaxWorld + 1)));
     CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(cells + 1) + 1) * sizeof(uint64_t)));
@@ -447,9 +546,8 @@ static int partition(Ctx &c, PartArgs &a, uint64_t *scnt, uint64_t *sdsp) {
     exclusive_scan<uint64_t>([cnt, cells] __device__(uint64_t i) -> uint64_t { return i < cells ? cnt[i] : 0; },
                              [cnt] __device__(uint64_t i, uint64_t pre, uint64_t) { cnt[i] = pre; }, cells + 1,
                              (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
-    part_scatter_kernel<<<(unsigned)ntiles, kPartThreads, 0, st>>>(a, ntiles, cnt);
     part_displs_kernel<<<1, kMaxWorld + 1, 0, st>>>(cnt, ntiles, W, displs);
-    c.launches += 3;
+    c.launches += 2;
     CK(cudaGetLastError());
     uint64_t h[kMaxWorld + 1];
     CK(cudaMemcpyAsync(h, displs, sizeof(uint64_t) * (W + 1), cudaMemcpyDeviceToHost, st));
@@ -461,11 +559,28 @@ static int partition(Ctx &c, PartArgs &a, uint64_t *scnt, uint64_t *sdsp) {
     return STEM_OK;
 }
 
+static int partition_scatter(Ctx &c, PartArgs &a, uint64_t ntiles, const PeerDst *pd_dev) {
+    if (!ntiles) return STEM_OK;
+    if (pd_dev)
+        part_scatter_kernel<true><<<(unsigned)ntiles, kPartThreads, 0, c.stream>>>(a, ntiles, c.part_cnt, pd_dev);
+    else
+        part_scatter_kernel<false><<<(unsigned)ntiles, kPartThreads, 0, c.stream>>>(a, ntiles, c.part_cnt, nullptr);
+    c.launches++;
+    CK(cudaGetLastError());
+    return STEM_OK;
+}
+
+static int partition(Ctx &c, PartArgs &a, uint64_t *scnt, uint64_t *sdsp) {
+    uint64_t ntiles = 0;
+    CKS(partition_count(c, a, scnt, sdsp, ntiles));
+    return partition_scatter(c, a, ntiles, nullptr);
+}
+
 // receive layout from everyone's send counts: rcnt[s] = counts s sends to me.
 // The allgather also carries every rank's local status (the partition before
 // it is local work): all ranks return the first failure in rank order.
 static int exchange_counts(Ctx &c, int local_status, const uint64_t *scnt, uint64_t *rcnt, uint64_t *rdsp,
-                           uint64_t &total) {
+                           uint64_t &total, uint64_t *mystart = nullptr) {
     const int W = c.comm->world, me = c.comm->rank;
     std::vector<uint64_t> mine((size_t)W + 1, 0), all((size_t)W * (W + 1));
     if (local_status == STEM_OK)
@@ -480,6 +595,11 @@ static int exchange_counts(Ctx &c, int local_status, const uint64_t *scnt, uint6
         rdsp[s] = total;
         total += rcnt[s];
     }
+    if (mystart)   // where my rows start in destination d's receive order (senders in rank order)
+        for (int d = 0; d < W; d++) {
+            mystart[d] = 0;
+            for (int s = 0; s < me; s++) mystart[d] += all[(size_t)s * (W + 1) + d];
+        }
     return STEM_OK;
 }
 
@@ -653,24 +773,57 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
     pa.in0 = kid;
     pa.in1 = t;
     pa.in2_add = row_base;
-    uint64_t scnt[kMaxWorld], sdsp[kMaxWorld], rcnt[kMaxWorld], rdsp[kMaxWorld], R = 0;
-    const int ls = [&]() -> int {
+    uint64_t scnt[kMaxWorld], sdsp[kMaxWorld], rcnt[kMaxWorld], rdsp[kMaxWorld], mystart[kMaxWorld], R = 0;
+    uint64_t ntiles = 0;
+    const bool p2p = dist_p2p();
+    auto stage_rows = [&]() -> int {   // the send/recv path: rows staged by destination locally
         for (int i = 0; i < 3; i++) CKS(c.ensure(c.xfer_u32[i], c.cap_xfer_u32[i], sizeof(uint32_t) * (n + 1)));
         pa.out0 = c.xfer_u32[0];
         pa.out1 = c.xfer_u32[1];
         pa.out2 = c.xfer_u32[2];
-        return partition(c, pa, scnt, sdsp);
+        return partition_scatter(c, pa, ntiles, nullptr);
+    };
+    const int ls = [&]() -> int {
+        CKS(partition_count(c, pa, scnt, sdsp, ntiles));
+        return p2p ? STEM_OK : stage_rows();
     }();
-    CKS(exchange_counts(c, ls, scnt, rcnt, rdsp, R));
+    CKS(exchange_counts(c, ls, scnt, rcnt, rdsp, R, mystart));
     CKS(dist_checkpoint(c, [&]() -> int {
         if (R >= (1ull << 32)) return STEM_E_RANGE;
         for (int i = 0; i < 3; i++) CKS(c.ensure(c.recv_u32[i], c.cap_recv_u32[i], sizeof(uint32_t) * (R + 1)));
         return STEM_OK;
     }()));
-    for (int i = 0; i < 3; i++)
-        CKS(comm.alltoallv(c.xfer_u32[i], scnt, sdsp, c.recv_u32[i], rcnt, rdsp, sizeof(uint32_t), st));
+    bool fused = false;
+    if (p2p) {   // the fused exchange: every row stored straight into its owner's receive window
+        void *mine[3] = {c.recv_u32[0], c.recv_u32[1], c.recv_u32[2]};
+        std::vector<void *> peers(3 * (size_t)W);
+        const int ws = comm.window(mine, 3, peers.data(), st);
+        if (ws == STEM_E_NCCL) return ws;
+        if (ws == STEM_OK) {   // (STEM_E_CUDA, agreed by every rank: no peer access, use send/recv)
+            CKS(dist_checkpoint(c, [&]() -> int {
+                PeerDst h{};
+                for (int d = 0; d < W; d++) {
+                    h.kid[d] = (uint32_t *)peers[3 * d];
+                    h.t[d] = (uint32_t *)peers[3 * d + 1];
+                    h.row[d] = (uint32_t *)peers[3 * d + 2];
+                    h.delta[d] = (int64_t)mystart[d] - (int64_t)sdsp[d];
+                }
+                CKS(c.ensure(c.peer_dst, c.cap_peer_dst, sizeof(PeerDst)));
+                CK(cudaMemcpyAsync(c.peer_dst, &h, sizeof(PeerDst), cudaMemcpyHostToDevice, st));
+                CKS(partition_scatter(c, pa, ntiles, (const PeerDst *)c.peer_dst));
+                return sync_stream(c);   // h lives on this stack frame until the copy is done
+            }()));   // every rank's stores have landed once all ranks pass this point
+            fused = true;
+        }
+    }
+    if (!fused) {
+        if (p2p) CKS(dist_checkpoint(c, stage_rows()));
+        for (int i = 0; i < 3; i++)
+            CKS(comm.alltoallv(c.xfer_u32[i], scnt, sdsp, c.recv_u32[i], rcnt, rdsp, sizeof(uint32_t), st));
+    }
+    c.stats.fused_exchange = fused ? 1u : 0u;
     CKS(sync_stream(c));   // the exchange is complete (or failed) before the local pipeline
-    c.stage_end(tk_x, 24 * n + 12 * R);
+    c.stage_end(tk_x, (fused ? 8 + 12 : 8 + 24) * n + (fused ? 0 : 12) * R);
     // 3. the local pipeline on my kernel range (kernel ids rebased to 0)
     const uint32_t KL = ke - kb;
     c.kid_base = kb;

@@ -182,7 +182,6 @@ struct Ctx {
     uint64_t *cut_SL = nullptr; size_t cap_cut_SL = 0;
     u128 *cut_QL = nullptr; size_t cap_cut_QL = 0;
     void *big_ent = nullptr, *big_part = nullptr, *big_thr = nullptr;
-    uint64_t *big_base = nullptr; size_t cap_big_base = 0;   // v2: per-cluster sum of t before lo
     size_t cap_big_ent = 0, cap_big_part = 0, cap_big_thr = 0;
     uint64_t *cnt_sz = nullptr; size_t cap_cntsz = 0;
     uint32_t *flags = nullptr; size_t cap_flags = 0;   // leaf-start bitmap: bit i & 31 of word i >> 5
@@ -210,6 +209,7 @@ struct Ctx {
     double *red_part2 = nullptr; size_t cap_red2 = 0;
     void *g_clusters = nullptr, *g_row = nullptr, *g_cluster = nullptr, *g_weight = nullptr;
     size_t cap_g_clusters = 0, cap_g_row = 0, cap_g_cluster = 0, cap_g_weight = 0;
+    void *peer_dst = nullptr; size_t cap_peer_dst = 0;   // fused exchange: the owners' windows (PeerDst)
     uint64_t row_bases[65] = {0};
     uint64_t n_local_rows = 0;
     // metric_bounds (metric.cu): leaf table (first leaf per kernel, lo_ns, n, m), per-leaf sums

@@ -54,11 +54,6 @@ static bool seed_on() {   // STEMROOT_SPLIT_SEED=0 disables the coarse threshold
     if (v < 0) v = (getenv("STEMROOT_SPLIT_SEED") && getenv("STEMROOT_SPLIT_SEED")[0] == '0') ? 0 : 1;
     return v == 1;
 }
-static bool split_v2() {   // STEMROOT_SPLIT_V=1: the v1 big-cluster path (one-level chunk bounds)
-    static int v = -1;
-    if (v < 0) v = (getenv("STEMROOT_SPLIT_V") && getenv("STEMROOT_SPLIT_V")[0] == '1') ? 0 : 1;
-    return v == 1;
-}
 static bool debug_levels() {
     static int v = -1;
     if (v < 0) v = getenv("STEMROOT_DEBUG_LEVELS") ? 1 : 0;
@@ -285,7 +280,8 @@ __device__ __forceinline__ void eval_cut(uint32_t k, uint64_t n, uint64_t S, uin
             cd.dlo = dlo;
             cd.dhi = dhi;
             cd.p = (uint64_t)k * (n - k);
-            take = exact_cmp(cd, best) > 0;               // equal -> keep the smaller k
+            const int cmp = exact_cmp(cd, best);          // equal -> the smaller k (any scan order)
+            take = cmp > 0 || (cmp == 0 && k < best.k);
         }
     }
     if (take) {
@@ -1043,383 +1039,6 @@ __global__ void big_reduce_kernel(const uint32_t *__restrict__ f_lo, const uint3
   }
 }
 
-// ---------------------------------------------------------------- big clusters, v2: two-level bounds
-// Entries on the aligned grid: entry E covers rows [E 2^16, (E+1) 2^16) of a
-// cluster [lo, hi) (clipped), so every boundary inside a cluster that a bound
-// needs is a multiple of 32 (PS1 / TB give S_L and t there exactly) except
-// the cluster's own ends, where ad = S k - n S_L is 0.
-//
-// Bound of ad over the cuts k of a row range [a, b) of the cluster (cuts
-// k = a - lo .. b - 1 - lo, i.e. the boundaries before each row): with A =
-// ad(a - lo), E = ad(b - lo), the first increment sa = S - n t[a] and the last
-// one S - n t[b - 1] (increments fall, ad is concave),
-//   ad(k) <= A + (k - ka) max(sa, 0)        (tangent at the start)
-//   ad(k) <= E + (b - lo - k) max(-sb, 0)   (tangent at the end)
-// so max ad <= min(A + (cnt-1) sa+, E + cnt sb-, max(A, E) + cnt min(sa+, sb-)).
-// Every fp64 step is rounded up (or down for the divisor p = k (n - k)), so a
-// range is pruned only when no cut in it can reach the threshold -- a
-// certified lower bound of a real candidate's score (div_lower, as the v1
-// path) -- and neither the argmax nor a tie is lost.  No u128 arithmetic and
-// no division per range: ~40 instructions where the v1 chunk bound took ~350.
-// Level 1 of the bound works on 1024-row super-chunks; only the surviving ones
-// are bounded 32 rows at a time, and only surviving 32-row chunks are scanned.
-constexpr int kB2Log = 16;                          // rows per entry = 2^16
-constexpr int kB2SupLog = 10;                       // rows per super-chunk = 2^10
-constexpr int kB2Sup = 1 << (kB2Log - kB2SupLog);   // super-chunks per entry (64)
-
-__device__ __forceinline__ uint32_t big2_nent(uint64_t lo, uint64_t hi) {
-    return (uint32_t)(((hi - 1) >> kB2Log) - (lo >> kB2Log) + 1);
-}
-
-// exact ad = S k - n SL (>= 0 for sorted rows), rounded up / to nearest to fp64
-__device__ __forceinline__ void ad_exact(uint64_t S, uint64_t k, uint64_t n, uint64_t SL, uint64_t &lo_, uint32_t &hi_) {
-    const uint64_t a0 = S * k, a1 = __umul64hi(S, k);
-    const uint64_t b0 = n * SL, b1 = __umul64hi(n, SL);
-    lo_ = a0 - b0;
-    hi_ = (uint32_t)(a1 - b1 - (a0 < b0 ? 1 : 0));
-}
-__device__ __forceinline__ double ad_ru(uint64_t lo_, uint32_t hi_) {
-    return __dadd_ru(__dmul_ru(__uint2double_rn(hi_), 0x1p64), __ull2double_ru(lo_));
-}
-
-struct Big2Args {
-    const BigEntry *ent;           // (cluster, aligned entry index)
-    const uint32_t *count;
-    const uint32_t *f_lo, *f_hi;
-    const uint64_t *f_S, *PS1;
-    const uint32_t *t, *TB;
-    const uint64_t *base;          // per cluster: exact sum of t before lo
-    unsigned long long *thr;       // per cluster: bits of the best certified lower bound so far
-    Cand *part;                    // per entry
-    unsigned long long *n_chunks, *n_scanned;
-};
-
-// value of ad, and t at the first / last row, of the range boundaries a < b
-// (a, b in [lo, hi]; interior boundaries are multiples of 32)
-struct RangeEnds {
-    uint64_t ka, cnt;
-    uint64_t Alo, Elo;
-    uint32_t Ahi, Ehi;
-    uint32_t ta, tl, tprev;        // t[a], t[b - 1], t[a - 1] (0 when a == lo)
-};
-
-__device__ __forceinline__ void range_ends(const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
-                                           const uint32_t *__restrict__ TB, uint64_t lo, uint64_t hi, uint64_t n,
-                                           uint64_t S, uint64_t base, uint64_t a, uint64_t b, RangeEnds &r) {
-    r.ka = a - lo;
-    r.cnt = b - a;
-    if (a == lo) {
-        r.Alo = 0; r.Ahi = 0;
-        r.ta = t[a];
-        r.tprev = 0;
-    } else {
-        ad_exact(S, r.ka, n, PS1[a >> kChunkLog] - base, r.Alo, r.Ahi);
-        const uint2 tb = reinterpret_cast<const uint2 *>(TB)[a >> kChunkLog];
-        r.ta = tb.y;
-        r.tprev = tb.x;
-    }
-    if (b == hi) {
-        r.Elo = 0; r.Ehi = 0;
-        r.tl = t[b - 1];
-    } else {
-        ad_exact(S, b - lo, n, PS1[b >> kChunkLog] - base, r.Elo, r.Ehi);
-        r.tl = reinterpret_cast<const uint2 *>(TB)[b >> kChunkLog].x;
-    }
-}
-
-// certified bound of the range's scores as (d2, pm): every cut k in the range
-// has ad(k)^2 <= d2 and k (n - k) >= pm; pm = 0 when the range holds no cut
-__device__ __forceinline__ void range_bound(const RangeEnds &r, uint64_t n, uint64_t S, double &d2, double &pm) {
-    const uint64_t kf = max(r.ka, (uint64_t)1), kl = min(r.ka + r.cnt - 1, n - 1);
-    d2 = 0.0;
-    pm = 0.0;
-    if (kf > kl) return;
-    const double A = ad_ru(r.Alo, r.Ahi), E = ad_ru(r.Elo, r.Ehi);
-    const uint64_t nta = n * (uint64_t)r.ta, ntl = n * (uint64_t)r.tl;
-    const double sa = S > nta ? __ull2double_ru(S - nta) : 0.0;
-    const double sb = ntl > S ? __ull2double_ru(ntl - S) : 0.0;
-    const double c = (double)r.cnt;
-    const double u1 = __dadd_ru(A, __dmul_ru(sa, c - 1.0));
-    const double u2 = __dadd_ru(E, __dmul_ru(sb, c));
-    const double u3 = __dadd_ru(fmax(A, E), __dmul_ru(fmin(sa, sb), c));
-    const double dmax = fmin(fmin(u1, u2), u3);
-    d2 = __dmul_ru(dmax, dmax);
-    pm = __ull2double_rd(min(kf * (n - kf), kl * (n - kl)));
-}
-
-// true when a range with bound (d2, pm) may hold a cut scoring >= thr (a
-// certified lower bound of a real candidate's score)
-__device__ __forceinline__ bool bound_survives(double d2, double pm, double thr) {
-    return pm > 0.0 && !(d2 < __dmul_rd(thr, pm));
-}
-
-__device__ __forceinline__ bool range_survives(const RangeEnds &r, uint64_t n, uint64_t S, double thr) {
-    double d2, pm;
-    range_bound(r, n, S, d2, pm);
-    return bound_survives(d2, pm, thr);
-}
-
-// certified lower bound of the score of the cut at the range start (0: not a cut)
-__device__ __forceinline__ double start_lower(const RangeEnds &r, uint64_t n) {
-    if (r.ka < 1 || !(r.tprev < r.ta)) return 0.0;
-    const double dD = approx_d(r.Ahi, r.Alo);
-    return __dmul_rn(div_lower(__dmul_rn(dD, dD), __dmul_rn((double)r.ka, (double)(n - r.ka))), 1.0 - 0x1p-44);
-}
-
-__global__ void big2_entries_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
-                                    const uint64_t *ctot, const uint64_t *__restrict__ PS1,
-                                    const uint32_t *__restrict__ t, BigEntry *__restrict__ ent,
-                                    uint32_t *__restrict__ first_ent, uint32_t *__restrict__ count,
-                                    unsigned long long *__restrict__ thr, uint64_t *__restrict__ base) {
-    const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= (*ctot >> 32)) return;
-    thr[c] = 0;
-    const uint64_t lo = f_lo[c], hi = f_hi[c];
-    if (hi - lo < c_big) return;
-    base[c] = pref1(PS1, t, lo);
-    const uint32_t nb = big2_nent(lo, hi), e0 = atomicAdd(count, nb);
-    const uint32_t E0 = (uint32_t)(lo >> kB2Log);
-    for (uint32_t s = 0; s < nb; s++) ent[e0 + s] = BigEntry{(uint32_t)c, E0 + s};
-    first_ent[c] = e0;
-}
-
-// the cluster's threshold from every 1024-row boundary inside it (real
-// candidates where t[b - 1] < t[b]); one warp per entry (64 boundaries)
-__global__ void __launch_bounds__(256) big2_seed_kernel(Big2Args g) {
-    const uint32_t n_ent = *g.count;
-    const int lane = threadIdx.x & 31;
-    const uint32_t nw = gridDim.x * (blockDim.x / 32);
-    for (uint32_t eb = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); eb < n_ent; eb += nw) {
-        const BigEntry e = g.ent[eb];
-        const uint64_t lo = g.f_lo[e.c], hi = g.f_hi[e.c], n = hi - lo, S = g.f_S[e.c], base = g.base[e.c];
-        double lbm = 0.0;
-#pragma unroll
-        for (int h = 0; h < kB2Sup / 32; h++) {
-            const uint64_t b = ((uint64_t)e.seg << kB2Log) + ((uint64_t)(h * 32 + lane) << kB2SupLog);
-            if (b > lo && b < hi) {
-                const uint2 tb = reinterpret_cast<const uint2 *>(g.TB)[b >> kChunkLog];
-                if (tb.x < tb.y) {
-                    uint64_t alo;
-                    uint32_t ahi;
-                    ad_exact(S, b - lo, n, g.PS1[b >> kChunkLog] - base, alo, ahi);
-                    const double dD = approx_d(ahi, alo);
-                    lbm = fmax(lbm, div_lower(__dmul_rn(dD, dD), __dmul_rn((double)(b - lo), (double)(hi - b))));
-                }
-            }
-        }
-#pragma unroll
-        for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));
-        if (lane == 0 && lbm > 0.0)
-            atomicMax(g.thr + e.c, (unsigned long long)__double_as_longlong(__dmul_rn(lbm, 1.0 - 0x1p-44)));
-    }
-}
-
-// one block (256 threads) per entry: 64 super-chunk bounds, then each
-// surviving super-chunk by one warp (32 chunk bounds, lane = chunk), then a
-// warp scan of each surviving chunk (lane = row); the entry's best candidate
-__global__ void __launch_bounds__(256) big2_split_kernel(Big2Args g) {
-    __shared__ uint32_t s_sup[kB2Sup];
-    __shared__ uint32_t s_nsup;
-    __shared__ unsigned long long s_thr;
-    __shared__ Cand s_best[8];
-    const uint32_t n_ent = *g.count;
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    for (uint32_t eb = blockIdx.x; eb < n_ent; eb += gridDim.x) {
-        const BigEntry e = g.ent[eb];
-        const uint64_t lo = g.f_lo[e.c], hi = g.f_hi[e.c], n = hi - lo, S = g.f_S[e.c], base = g.base[e.c];
-        const uint64_t r0 = max(lo, (uint64_t)e.seg << kB2Log), r1 = min(hi, ((uint64_t)e.seg + 1) << kB2Log);
-        if (tid == 0) {
-            s_nsup = 0;
-            s_thr = g.thr[e.c];
-        }
-        __syncthreads();
-        const double thr0 = __longlong_as_double((long long)s_thr);
-        // level 1: super-chunks [a, b) on the 1024-row grid
-        const uint64_t sbase = r0 >> kB2SupLog;
-        const uint32_t nsup = (uint32_t)(((r1 - 1) >> kB2SupLog) - sbase + 1);
-        if (tid < (int)nsup) {
-            const uint64_t a = max(r0, (sbase + tid) << kB2SupLog), b = min(r1, (sbase + tid + 1) << kB2SupLog);
-            RangeEnds re;
-            range_ends(g.t, g.PS1, g.TB, lo, hi, n, S, base, a, b, re);
-            if (range_survives(re, n, S, thr0)) s_sup[atomicAdd(&s_nsup, 1u)] = (uint32_t)tid;
-        }
-        __syncthreads();
-        const uint32_t ns = s_nsup;
-        Cand best = no_cand();
-        uint32_t scanned = 0, bounded = 0;
-        for (uint32_t si = w; si < ns; si += 8) {
-            const uint64_t sa_ = max(r0, (sbase + s_sup[si]) << kB2SupLog);
-            const uint64_t sb_ = min(r1, (sbase + s_sup[si] + 1) << kB2SupLog);
-            // level 2: chunk `lane` of the super-chunk
-            const uint64_t q0 = sa_ >> kChunkLog;
-            const uint32_t nq = (uint32_t)(((sb_ - 1) >> kChunkLog) - q0 + 1);
-            bool live = false;
-            uint64_t ca = 0, cb = 0, SLa = 0;
-            double lb = 0.0;
-            const double thr = fmax(thr0, __longlong_as_double((long long)*(volatile unsigned long long *)&s_thr));
-            if (lane < (int)nq) {
-                ca = max(sa_, (q0 + lane) << kChunkLog);
-                cb = min(sb_, (q0 + lane + 1) << kChunkLog);
-                RangeEnds re;
-                range_ends(g.t, g.PS1, g.TB, lo, hi, n, S, base, ca, cb, re);
-                live = range_survives(re, n, S, thr);
-                lb = start_lower(re, n);
-                SLa = ca == lo ? 0 : g.PS1[ca >> kChunkLog] - base;
-            }
-            bounded += nq;
-#pragma unroll
-            for (int o = 16; o; o >>= 1) lb = fmax(lb, __shfl_xor_sync(0xffffffffu, lb, o));
-            if (lane == 0 && lb > thr) atomicMax(&s_thr, (unsigned long long)__double_as_longlong(lb));
-            uint32_t lv = __ballot_sync(0xffffffffu, live);
-            scanned += __popc(lv);
-            while (lv) {
-                const int src = __ffs(lv) - 1;
-                lv &= lv - 1;
-                const uint64_t xa = __shfl_sync(0xffffffffu, ca, src), xb = __shfl_sync(0xffffffffu, cb, src);
-                const uint64_t xs = __shfl_sync(0xffffffffu, SLa, src);
-                scan_chunk(g.t, lo, n, S, xa, xb, xs, best);
-            }
-            if (best.k) {   // share the warp's best as a threshold with the other warps of the entry
-                const double l2 = __dmul_rn(div_lower(best.x, best.dp), 1.0 - 0x1p-44);
-                if (lane == 0) atomicMax(&s_thr, (unsigned long long)__double_as_longlong(l2));
-            }
-        }
-#pragma unroll 1
-        for (int o = 16; o; o >>= 1) {
-            const Cand v = shfl_cand_xor(best, o);
-            if (better(v, best)) best = v;
-        }
-        if (lane == 0) {
-            s_best[w] = best;
-            if (bounded) {
-                atomicAdd(g.n_chunks, (unsigned long long)bounded);
-                atomicAdd(g.n_scanned, (unsigned long long)scanned);
-            }
-        }
-        __syncthreads();
-        if (tid == 0) {
-            Cand b = s_best[0];
-            for (int k = 1; k < 8; k++)
-                if (better(s_best[k], b)) b = s_best[k];
-            g.part[eb] = b;
-            const unsigned long long m = s_thr;
-            if (m) atomicMax(g.thr + e.c, m);
-        }
-        __syncthreads();
-    }
-}
-
-__global__ void big2_reduce_kernel(const uint32_t *__restrict__ f_lo, const uint32_t *__restrict__ f_hi,
-                                   const uint64_t *ctot, const uint32_t *__restrict__ first_ent,
-                                   const Cand *__restrict__ part, uint32_t *__restrict__ cut,
-                                   uint64_t *__restrict__ cut_SL) {
-    const uint64_t C = *ctot >> 32;
-    for (uint64_t c = blockIdx.x; c < C; c += gridDim.x) {
-        const uint64_t lo = f_lo[c], hi = f_hi[c];
-        if (hi - lo < c_big) continue;
-        const uint32_t nb = big2_nent(lo, hi), e0 = first_ent[c];
-        Cand best = no_cand();
-        for (uint32_t s = threadIdx.x; s < nb; s += 32)
-            if (better(part[e0 + s], best)) best = part[e0 + s];
-#pragma unroll 1
-        for (int o = 16; o; o >>= 1) {
-            const Cand v = shfl_cand_xor(best, o);
-            if (better(v, best)) best = v;
-        }
-        if (threadIdx.x == 0) {
-            cut[c] = best.k;
-            cut_SL[c] = best.SL;
-        }
-    }
-}
-
-// Clusters of c_loc .. c_big rows, v2: one warp per cluster; lane i bounds
-// chunk i (32 rows, aligned; up to 3 rounds of 32 chunks) with the certified
-// two-tangent bound of big2 and scores its start when that is a real cut
-// (the threshold); the surviving chunks are scanned row by row in order,
-// each re-checked against the threshold raised by the scans before it.
-__device__ __forceinline__ Cand warp_best_cut2(const uint32_t *__restrict__ t, const uint64_t *__restrict__ PS1,
-                                               const uint32_t *__restrict__ TB, uint64_t lo, uint64_t n, uint64_t S) {
-    const uint64_t hi = lo + n;
-    const uint64_t q0 = lo >> kChunkLog;
-    const uint32_t nq = (uint32_t)(((hi - 1) >> kChunkLog) - q0 + 1);
-    if (n <= 64 || nq > 32 * kMaxRounds) return warp_scan_cut(t, lo, n, S);
-    const int lane = threadIdx.x & 31;
-    const uint64_t base = warp_pref1(t, PS1, lo);
-    double d2[kMaxRounds], pm[kMaxRounds];
-    uint64_t sl[kMaxRounds];
-    double lbm = 0.0;
-#pragma unroll
-    for (int r = 0; r < kMaxRounds; r++) {
-        const uint32_t i = r * 32 + lane;
-        sl[r] = 0;
-        d2[r] = 0.0;
-        pm[r] = 0.0;
-        if (i < nq) {
-            const uint64_t ca = max(lo, (q0 + i) << kChunkLog), cb = min(hi, (q0 + i + 1) << kChunkLog);
-            RangeEnds re;
-            range_ends(t, PS1, TB, lo, hi, n, S, base, ca, cb, re);
-            range_bound(re, n, S, d2[r], pm[r]);
-            lbm = fmax(lbm, start_lower(re, n));
-            sl[r] = ca == lo ? 0 : PS1[ca >> kChunkLog] - base;
-        }
-    }
-#pragma unroll
-    for (int o = 16; o; o >>= 1) lbm = fmax(lbm, __shfl_xor_sync(0xffffffffu, lbm, o));
-    double thr = lbm;
-    Cand best = no_cand();
-#pragma unroll 1
-    for (int r = 0; r < kMaxRounds; r++) {
-        static_assert(kMaxRounds == 3, "the selects below cover three rounds");
-        const double rd2 = r == 0 ? d2[0] : r == 1 ? d2[1] : d2[2];
-        const double rpm = r == 0 ? pm[0] : r == 1 ? pm[1] : pm[2];
-        const uint64_t rsl = r == 0 ? sl[0] : r == 1 ? sl[1] : sl[2];
-        uint32_t live = __ballot_sync(0xffffffffu, bound_survives(rd2, rpm, thr));
-        while (live) {
-            const int src = __ffs(live) - 1;
-            live &= live - 1;
-            const double sd2 = __shfl_sync(0xffffffffu, rd2, src), spm = __shfl_sync(0xffffffffu, rpm, src);
-            if (!bound_survives(sd2, spm, thr)) continue;   // threshold raised meanwhile
-            const uint32_t i = r * 32 + src;
-            const uint64_t ca = max(lo, (q0 + i) << kChunkLog), cb = min(hi, (q0 + i + 1) << kChunkLog);
-            const uint64_t SLa = __shfl_sync(0xffffffffu, rsl, src);
-            scan_chunk(t, lo, n, S, ca, cb, SLa, best);
-            double lb = best.k ? div_lower(best.x, best.dp) : 0.0;
-#pragma unroll
-            for (int o = 16; o; o >>= 1) lb = fmax(lb, __shfl_xor_sync(0xffffffffu, lb, o));
-            thr = fmax(thr, __dmul_rn(lb, 1.0 - 0x1p-44));
-        }
-    }
-#pragma unroll 1
-    for (int o = 16; o; o >>= 1) {
-        const Cand v = shfl_cand_xor(best, o);
-        if (better(v, best)) best = v;
-    }
-    return best;
-}
-
-template <int MINB>
-__global__ void __launch_bounds__(256, MINB) small2_split_kernel(const uint32_t *__restrict__ f_lo,
-                                                           const uint32_t *__restrict__ f_hi,
-                                                           const uint64_t *__restrict__ f_S, const uint64_t *ctot,
-                                                           const uint32_t *__restrict__ t,
-                                                           const uint64_t *__restrict__ PS1,
-                                                           const uint32_t *__restrict__ TB, uint32_t *__restrict__ cut,
-                                                           uint64_t *__restrict__ cut_SL) {
-    const uint32_t C = (uint32_t)(*ctot >> 32);
-    const int lane = threadIdx.x & 31;
-    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
-        const uint64_t lo = f_lo[c], n = f_hi[c] - lo;
-        if (n < c_loc || n >= c_big) continue;
-        const Cand best = warp_best_cut2(t, PS1, TB, lo, n, f_S[c]);
-        if (lane == 0) {
-            cut[c] = best.k;
-            cut_SL[c] = best.SL;
-        }
-    }
-}
-
 // ---------------------------------------------------------------- a4: decide
 struct DecideArgs {
     const uint32_t *f_lo, *f_hi, *cut;
@@ -1748,13 +1367,12 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         // may still read (nxt is the input of the level queued before this
         // one): drain the stream first, then grow with 2x headroom so this
         // happens only O(log) times per ctx.
-        const uint64_t max_ent = Aub / kBigSeg + 2 * (Aub / big_rows()) + 2;
+        const uint64_t max_ent = Aub / kBigSeg + Aub / big_rows() + 1;
         const bool grow = sizeof(uint32_t) * Cub > c.cap_cut || sizeof(uint64_t) * Cub > c.cap_cut_SL ||
                           sizeof(u128) * 2 * Cub > c.cap_fQ[nxt] ||
                           (split == 0 && (sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (Cub + 1) > c.cap_big_ent ||
                                           sizeof(Cand) * max_ent > c.cap_big_part ||
-                                          sizeof(unsigned long long) * Cub > c.cap_big_thr ||
-                                          sizeof(uint64_t) * Cub > c.cap_big_base));
+                                          sizeof(unsigned long long) * Cub > c.cap_big_thr));
         if (grow) {
             CK(cudaStreamSynchronize(st));
             CKS(c.ensure(c.cut, c.cap_cut, 2 * sizeof(uint32_t) * Cub));
@@ -1764,7 +1382,6 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                 CKS(c.ensure(c.big_ent, c.cap_big_ent, 2 * (sizeof(BigEntry) * max_ent + sizeof(uint32_t) * (Cub + 1))));
                 CKS(c.ensure(c.big_part, c.cap_big_part, 2 * sizeof(Cand) * max_ent));
                 CKS(c.ensure(c.big_thr, c.cap_big_thr, 2 * sizeof(unsigned long long) * Cub));
-                CKS(c.ensure(c.big_base, c.cap_big_base, 2 * sizeof(uint64_t) * Cub));
             }
         }
         const int tk_l = loc_rows > 0 ? c.stage_begin("root_local") : -1;
@@ -1808,10 +1425,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             const uint64_t blocks = (Cub + 7) / 8;
             static int minb = -1;   // STEMROOT_SMALL_MINB: resident blocks per SM the registers are sized for
             if (minb < 0) minb = getenv("STEMROOT_SMALL_MINB") ? atoi(getenv("STEMROOT_SMALL_MINB")) : 4;
-            if (split_v2())
-                small2_split_kernel<4><<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, sst>>>(
-                    c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
-            else if (minb == 3)
+            if (minb == 3)
                 small_split_kernel<3><<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, sst>>>(
                     c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
             else
@@ -1823,19 +1437,6 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         BigEntry *ent = (BigEntry *)c.big_ent;
         uint32_t *first_ent = (uint32_t *)(ent + max_ent);
         CK(cudaMemsetAsync(&c.scalars->big_count, 0, sizeof(uint32_t), st));
-        if (split_v2()) {   // two-level bounds on the aligned entry grid (default)
-            big2_entries_kernel<<<(unsigned)((Cub + 255) / 256), 256, 0, st>>>(
-                c.f_lo[cur], c.f_hi[cur], ctot, c.PS1, c.t_sorted, ent, first_ent, &c.scalars->big_count,
-                (unsigned long long *)c.big_thr, c.big_base);
-            Big2Args g{ent, &c.scalars->big_count, c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.PS1, c.t_sorted, c.TB,
-                       c.big_base, (unsigned long long *)c.big_thr, (Cand *)c.big_part, &c.scalars->split_chunks,
-                       &c.scalars->split_scanned};
-            big2_seed_kernel<<<(unsigned)min((max_ent + 7) / 8, (uint64_t)c.sms * 8), 256, 0, st>>>(g);
-            big2_split_kernel<<<(unsigned)min(max_ent, (uint64_t)c.sms * 8), 256, 0, st>>>(g);
-            big2_reduce_kernel<<<(unsigned)min(Cub, (uint64_t)4096), 32, 0, st>>>(
-                c.f_lo[cur], c.f_hi[cur], ctot, first_ent, (const Cand *)c.big_part, c.cut, c.cut_SL);
-            c.launches += 4;
-        } else {
         big_entries_kernel<<<(unsigned)((Cub + 255) / 256), 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], ctot, ent, first_ent,
                                                                          &c.scalars->big_count,
                                                                          (unsigned long long *)c.big_thr);
@@ -1854,7 +1455,6 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         big_reduce_kernel<<<(unsigned)min(Cub, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], ctot, first_ent,
                                                                         (const Cand *)c.big_part, c.cut, c.cut_SL);
         c.launches += 2;
-        }
         if (overlap) {
             CK(cudaEventRecord(c.ev_join, c.side));
             CK(cudaStreamWaitEvent(st, c.ev_join, 0));

@@ -223,3 +223,35 @@ def test_loopback_missing_peer_times_out(tmp_path):
     env = dict(os.environ, STEMROOT_COMM_TIMEOUT_S="3")
     out = subprocess.run([sys.executable, str(prog)], env=env, capture_output=True, text=True, timeout=300)
     assert "STATUS -5" in out.stdout, out.stdout + out.stderr
+
+
+def test_fused_exchange_and_send_recv_paths_agree(tmp_path):
+    """The kernel-id exchange stores rows straight into the owners' receive
+    windows (stats.fused_exchange = 1; loopback windows are the other ranks'
+    device buffers, NCCL ones CUDA-IPC peer memory); STEMROOT_DIST_P2P=0 keeps
+    the grouped send/recv path.  Both give the single-trace oracle plan."""
+    import subprocess
+    import sys
+    prog = tmp_path / "fx.py"
+    prog.write_text(
+        "import sys, threading, numpy as np, torch\n"
+        f"sys.path.insert(0, {ROOT!r}); sys.path.insert(0, {os.path.join(ROOT, 'tests')!r})\n"
+        "import paper_conf_micro_chungnkk25_b200 as sr, oracle as O, tracegen as G\n"
+        "from parity_util import Z95, assert_plans_equal\n"
+        "sp = G.spec('C2', n=90_000); kid, t, _ = G.generate_np(sp); W = 3\n"
+        "cuts = [len(kid) * r // W for r in range(W + 1)]\n"
+        "comms = sr.Comm.loopback(W, 0); ctxs = [sr.Context(0) for _ in range(W)]\n"
+        "out = [None] * W; fx = [None] * W\n"
+        "def run(r):\n"
+        "    a, b = cuts[r], cuts[r + 1]\n"
+        "    dk = torch.from_numpy(kid[a:b].view(np.int32)).cuda(); dt = torch.from_numpy(t[a:b].view(np.int32)).cuda()\n"
+        "    out[r] = ctxs[r].plan_dist(comms[r], dk, dt, sp.n_kernels, a, z=Z95, seed=3, stream=torch.cuda.Stream().cuda_stream)\n"
+        "    fx[r] = ctxs[r].stats()['fused_exchange']\n"
+        "th = [threading.Thread(target=run, args=(r,)) for r in range(W)]\n"
+        "[x.start() for x in th]; [x.join() for x in th]\n"
+        "assert_plans_equal(out[0], O.plan(kid, t, sp.n_kernels, z=Z95, seed=3))\n"
+        "print('FUSED', fx)\n")
+    for env, want in (({}, "FUSED [1, 1, 1]"), ({"STEMROOT_DIST_P2P": "0"}, "FUSED [0, 0, 0]")):
+        out = subprocess.run([sys.executable, str(prog)], env=dict(os.environ, **env), capture_output=True, text=True,
+                             timeout=600)
+        assert want in out.stdout, out.stdout + out.stderr[-3000:]
