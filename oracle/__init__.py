@@ -35,7 +35,7 @@ def build(force: bool = False) -> str:
 class _Opts(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("z", C.c_double), ("scope", C.c_int), ("root", C.c_int),
                 ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("split", C.c_int),
-                ("metric_bounds", C.c_int)]
+                ("metric_bounds", C.c_int), ("kmeans_k", C.c_int)]
 
 
 class _Plan(C.Structure):
@@ -77,6 +77,8 @@ def lib():
         _lib.or_kmpp_cut.argtypes = [u32p, C.c_uint64, C.c_uint64, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32),
                                      C.POINTER(C.c_uint32)]
         _lib.or_kmpp_cut.restype = C.c_uint64
+        _lib.or_kmeans_cuts.argtypes = [u32p, C.c_uint64, C.c_uint32, u64p]
+        _lib.or_kmeans_cuts.restype = C.c_uint32
         _lib.or_eq3_m.argtypes = [C.c_uint64, C.c_uint64, C.c_uint64, C.c_uint64, C.c_double, C.c_double, C.c_int]
         _lib.or_eq3_m.restype = C.c_double
         _lib.or_eq6_m.argtypes = [C.c_uint32, dp, dp, C.c_double, C.c_double, C.c_double, dp]
@@ -108,7 +110,7 @@ class OracleError(RuntimeError):
 
 
 def plan(kernel_id, exec_ns, n_kernels, eps=0.05, z=1.959963984540054, seed=0, scope=0, root=1,
-         clamp_in_split=1, census_cap=0, metrics=None, split=0, metric_bounds=0) -> dict:
+         clamp_in_split=1, census_cap=0, metrics=None, split=0, metric_bounds=0, kmeans_k=3) -> dict:
     """Full sampling plan (§3).  Returns numpy arrays + scalars."""
     kid = _u32(kernel_id)
     t = _u32(exec_ns)
@@ -119,7 +121,7 @@ def plan(kernel_id, exec_ns, n_kernels, eps=0.05, z=1.959963984540054, seed=0, s
         metp = _ptr(met, C.c_double)
     else:
         nm, metp = 0, None
-    o = _Opts(seed, z, scope, root, clamp_in_split, census_cap, split, int(metric_bounds))
+    o = _Opts(seed, z, scope, root, clamp_in_split, census_cap, split, int(metric_bounds), int(kmeans_k))
     out = C.POINTER(_Plan)()
     st = lib().or_plan_build(n, n_kernels, _ptr(kid, C.c_uint32), _ptr(t, C.c_uint32), nm, metp, eps,
                              C.byref(o), C.byref(out))
@@ -171,6 +173,14 @@ def kmpp_cut(t_sorted, seed):
     k = int(lib().or_kmpp_cut(_ptr(t, C.c_uint32), t.shape[0], seed & 0xFFFFFFFFFFFFFFFF, C.byref(c1),
                               C.byref(c2), C.byref(it)))
     return k, int(c1.value), int(c2.value), int(it.value)
+
+
+def kmeans_cuts(t_sorted, k):
+    """Exact optimal 1-D k-means cuts of sorted times (reading R29): list of row cuts."""
+    t = _u32(t_sorted)
+    out = np.zeros(16, np.uint64)
+    g = int(lib().or_kmeans_cuts(_ptr(t, C.c_uint32), t.shape[0], k, _ptr(out, C.c_uint64)))
+    return [int(x) for x in out[:max(g - 1, 0)]]
 
 
 def best_cut(t_sorted) -> int:

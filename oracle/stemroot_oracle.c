@@ -375,6 +375,110 @@ uint64_t or_best_cut(const uint32_t *t_sorted, uint64_t n) {
 }
 
 /* ------------------------------------------------------------------------ */
+/* Exact optimal 1-D k-means (split = 3; "k-means ... any number above */
+/* 2 works well"; reading R29)                                                */
+/* ------------------------------------------------------------------------ */
+/* Total SSE of a partition = Q - sum_g S_g^2 / n_g, so the optimal partition
+ * maximises sum_g S_g^2 / n_g.  In 1-D some optimal partition consists of
+ * consecutive sorted values and never separates equal values, so the groups
+ * are runs of consecutive distinct values and the textbook dynamic program
+ *   F[1][b] = S(0,b)^2 / n(0,b),
+ *   F[j][b] = max_{a < b} F[j-1][a] + S(a,b)^2 / n(a,b)
+ * over the distinct values is exact.  Every F is kept as an exact fraction of
+ * big integers (num / den, den = product of the group sizes), so comparisons
+ * are exact; ties take the smallest a, i.e. among optimal partitions the one
+ * whose last cut is smallest, then the one before it, and so on. */
+#define OR_BIG 12          /* 768-bit: num * den' < 2^(96 + 64 k + 3) for k <= 8 */
+typedef struct { uint64_t w[OR_BIG]; } bigint;
+typedef struct { bigint num, den; } fraction;
+
+static bigint big_mul(const bigint *a, const bigint *b) {
+    uint64_t out[2 * OR_BIG];
+    limb_mul(a->w, OR_BIG, b->w, OR_BIG, out);
+    bigint r;
+    memcpy(r.w, out, sizeof(r.w));   /* the high half is zero for k <= 8 */
+    return r;
+}
+
+static bigint big_add(const bigint *a, const bigint *b) {
+    bigint r;
+    u128 carry = 0;
+    for (int i = 0; i < OR_BIG; i++) {
+        u128 s = (u128)a->w[i] + b->w[i] + carry;
+        r.w[i] = (uint64_t)s;
+        carry = s >> 64;
+    }
+    return r;
+}
+
+static bigint big_u128(u128 v) {
+    bigint r;
+    memset(&r, 0, sizeof(r));
+    r.w[0] = (uint64_t)v;
+    r.w[1] = (uint64_t)(v >> 64);
+    return r;
+}
+
+/* f + S^2 / n */
+static fraction frac_add_group(const fraction *f, uint64_t S, uint64_t n) {
+    bigint bn = big_u128(n), s2 = big_u128((u128)S * S);
+    bigint a = big_mul(&f->num, &bn), b = big_mul(&s2, &f->den);
+    fraction r;
+    r.num = big_add(&a, &b);
+    r.den = big_mul(&f->den, &bn);
+    return r;
+}
+
+static int frac_cmp(const fraction *a, const fraction *b) {
+    bigint l = big_mul(&a->num, &b->den), r = big_mul(&b->num, &a->den);
+    return limb_cmp(l.w, r.w, OR_BIG);
+}
+
+uint32_t or_kmeans_cuts(const uint32_t *t, uint64_t n, uint32_t k, uint64_t *cuts) {
+    if (n < 2 || t[0] == t[n - 1] || k < 2) return 0;
+    /* run starts of the distinct values: pos[0] = 0 < ... < pos[d-1], pos[d] = n */
+    uint64_t d = 1;
+    for (uint64_t i = 1; i < n; i++) d += t[i - 1] < t[i];
+    uint64_t *pos = malloc((d + 1) * sizeof(uint64_t)), *P = malloc((d + 1) * sizeof(uint64_t));
+    uint32_t K = k < d ? k : (uint32_t)d;
+    fraction *F = malloc((size_t)(K + 1) * (d + 1) * sizeof(fraction));
+    uint64_t *arg = malloc((size_t)(K + 1) * (d + 1) * sizeof(uint64_t));
+    if (!pos || !P || !F || !arg) { free(pos); free(P); free(F); free(arg); return 0; }
+    uint64_t r = 0, run = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        if (i == 0 || t[i - 1] < t[i]) { pos[r] = i; P[r] = run; r++; }
+        run += t[i];
+    }
+    pos[d] = n;
+    P[d] = run;
+#define FF(j, b) F[(size_t)(j) * (d + 1) + (b)]
+#define ARG(j, b) arg[(size_t)(j) * (d + 1) + (b)]
+    fraction zero;
+    memset(&zero, 0, sizeof(zero));
+    zero.den.w[0] = 1;
+    for (uint64_t b = 1; b <= d; b++) FF(1, b) = frac_add_group(&zero, P[b], pos[b]);
+    for (uint32_t j = 2; j <= K; j++)
+        for (uint64_t b = j; b <= d; b++) {
+            for (uint64_t a = j - 1; a < b; a++) {
+                fraction c = frac_add_group(&FF(j - 1, a), P[b] - P[a], pos[b] - pos[a]);
+                if (a == j - 1 || frac_cmp(&c, &FF(j, b)) > 0) {   /* strict: ties keep the smaller a */
+                    FF(j, b) = c;
+                    ARG(j, b) = a;
+                }
+            }
+        }
+    uint64_t b = d;
+    for (uint32_t j = K; j >= 2; j--) {
+        b = ARG(j, b);
+        cuts[j - 2] = pos[b];
+    }
+#undef FF
+#undef ARG
+    free(pos); free(P); free(F); free(arg);
+    return K;
+}
+
+/* ------------------------------------------------------------------------ */
 /* STEM sample sizes                                                          */
 /* ------------------------------------------------------------------------ */
 /* Eq. 3 in the fixed order of R9: x = (rn(V)/(rn(S)*rn(S))) * k2,
@@ -417,33 +521,64 @@ void or_eq6_m(uint32_t k, const double *mu, const double *V, double T, double ep
 /* ------------------------------------------------------------------------ */
 /* ROOT decision (Eq. 7 vs Eq. 8; readings R6-R9)                */
 /* ------------------------------------------------------------------------ */
-typedef struct { double tau_old, tau_new; uint64_t cut; int split; } decision;
+#define OR_KMAX 8
+typedef struct {
+    double tau_old, tau_new;
+    uint64_t cut;                 /* 2-way rules: the cut */
+    uint32_t ngroups;             /* children if split (2, or 2..kmeans_k for split = 3) */
+    uint64_t cuts[OR_KMAX - 1];   /* their boundaries, relative to lo, ascending */
+    int split;
+} decision;
+
+/* Eq. 8 for the children [lo + b_{g-1}, lo + b_g) of a cluster, b_0 = 0 and
+ * b_G = n, Eq. 6 (corrected numerator) over them with c from the parent's
+ * total, summed left to right (for two children exactly the 2-way formula). */
+static double tau_children(const uint32_t *t, uint64_t lo, uint64_t hi, const uint64_t *cuts, uint32_t G,
+                           double eps, double z, int clamp, uint64_t S_parent) {
+    double mu[OR_KMAX], V[OR_KMAX];
+    for (uint32_t g = 0; g < G; g++) {
+        uint64_t a = g == 0 ? lo : lo + cuts[g - 1], b = g + 1 == G ? hi : lo + cuts[g];
+        moments m = range_moments(t, a, b);
+        mu[g] = rn64(m.S) / rn64(m.n);
+        V[g] = rn128(moments_V(m));
+    }
+    double w = (eps * rn64(S_parent)) / z;
+    double c = w * w;
+    double ssum = 0.0;
+    for (uint32_t g = 0; g < G; g++) ssum = g == 0 ? sqrt(mu[0] * V[0]) : ssum + sqrt(mu[g] * V[g]);
+    double gg = ssum / c;
+    double tau = 0.0;
+    for (uint32_t g = 0; g < G; g++) {
+        double m = eq6_one(gg, mu[g], V[g], clamp);
+        tau = g == 0 ? m * mu[0] : tau + m * mu[g];
+    }
+    return tau;
+}
 
 static decision root_decide(const uint32_t *t, uint64_t lo, uint64_t hi, double eps, double z,
-                            double k2, int clamp, int split, uint64_t seed) {
-    decision d = {0.0, 0.0, 0, 0};
+                            double k2, int clamp, int split, uint64_t seed, uint32_t kk) {
+    decision d;
+    memset(&d, 0, sizeof(d));
     uint64_t n = hi - lo;
     if (n < 2 || t[lo] == t[hi - 1]) return d;              /* R5: leaf */
     moments all = range_moments(t, lo, hi);
-    uint64_t k = split == 1   ? lloyd_cut(t, lo, hi, NULL)
-               : split == 2 ? kmpp_cut(t, lo, hi, seed, NULL, NULL, NULL)
-                            : best_cut(t, lo, hi, all.S);
-    d.cut = k;
+    if (split == 3) {                                       /* R29: k groups at once */
+        d.ngroups = or_kmeans_cuts(t + lo, n, kk, d.cuts);
+        d.cut = d.cuts[0];
+    } else {
+        uint64_t k = split == 1   ? lloyd_cut(t, lo, hi, NULL)
+                   : split == 2 ? kmpp_cut(t, lo, hi, seed, NULL, NULL, NULL)
+                                : best_cut(t, lo, hi, all.S);
+        d.cut = k;
+        d.cuts[0] = k;
+        d.ngroups = 2;
+    }
     /* Eq. 7: tau_old = m * Xbar with m from Eq. 3 */
     double mu = rn64(all.S) / rn64(all.n);
     double m_old = eq3_m(moments_V(all), all.S, k2, clamp);
     d.tau_old = m_old * mu;
-    /* Eq. 8: tau_new = sum_i m_i Xbar_i with m_i from Eq. 6 over {L, R} */
-    moments L = range_moments(t, lo, lo + k), R = range_moments(t, lo + k, hi);
-    u128 VL = moments_V(L), VR = moments_V(R);
-    double muL = rn64(L.S) / rn64(L.n), muR = rn64(R.S) / rn64(R.n);
-    double w = (eps * rn64(all.S)) / z;
-    double c = w * w;
-    double ssum = sqrt(muL * rn128(VL)) + sqrt(muR * rn128(VR));
-    double g = ssum / c;
-    double mL = eq6_one(g, muL, rn128(VL), clamp);
-    double mR = eq6_one(g, muR, rn128(VR), clamp);
-    d.tau_new = mL * muL + mR * muR;
+    /* Eq. 8: tau_new = sum_i m_i Xbar_i with m_i from Eq. 6 over the children */
+    d.tau_new = tau_children(t, lo, hi, d.cuts, d.ngroups, eps, z, clamp, all.S);
     d.split = d.tau_new < d.tau_old;                        /* strict */
     return d;
 }
@@ -451,7 +586,7 @@ static decision root_decide(const uint32_t *t, uint64_t lo, uint64_t hi, double 
 int or_root_decide(const uint32_t *t_sorted, uint64_t n, double eps, double z, int clamp,
                    double *tau_old, double *tau_new, uint64_t *cut) {
     double q = z / eps;
-    decision d = root_decide(t_sorted, 0, n, eps, z, q * q, clamp, 0, 0);
+    decision d = root_decide(t_sorted, 0, n, eps, z, q * q, clamp, 0, 0, 2);
     if (tau_old) *tau_old = d.tau_old;
     if (tau_new) *tau_new = d.tau_new;
     if (cut) *cut = d.cut;
@@ -518,7 +653,8 @@ int or_plan_build(uint64_t n, uint32_t n_kernels, const uint32_t *kernel_id,
     if (!(eps > 0.0 && eps < 1.0) || !(opts->z > 0.0) || !isfinite(opts->z)) return OR_E_INVAL;
     if (n_metrics > 64 || (n_metrics > 0 && !metrics)) return OR_E_INVAL;
     if (opts->scope < 0 || opts->scope > 2) return OR_E_INVAL;
-    if (opts->split < 0 || opts->split > 2) return OR_E_INVAL;
+    if (opts->split < 0 || opts->split > 3) return OR_E_INVAL;
+    if (opts->split == 3 && (opts->kmeans_k < 2 || opts->kmeans_k > OR_KMAX)) return OR_E_INVAL;
     if (n >= ((uint64_t)1 << 32)) return OR_E_RANGE;
     for (uint64_t i = 0; i < n; i++) if (kernel_id[i] >= n_kernels) return OR_E_RANGE;
 
@@ -555,12 +691,16 @@ int or_plan_build(uint64_t n, uint32_t n_kernels, const uint32_t *kernel_id,
         while (work.n > 0) {
             work_item w = work.v[--work.n];
             if (w.depth > max_depth) max_depth = w.depth;
-            decision d = {0.0, 0.0, 0, 0};
-            if (opts->root) d = root_decide(t, w.lo, w.hi, eps, z, k2, clamp, opts->split, opts->seed);
+            decision d;
+            memset(&d, 0, sizeof(d));
+            if (opts->root)
+                d = root_decide(t, w.lo, w.hi, eps, z, k2, clamp, opts->split, opts->seed, (uint32_t)opts->kmeans_k);
             if (d.split) {
-                /* push right then left: the left child is visited first */
-                if (work_push(&work, w.lo + d.cut, w.hi, w.depth + 1) ||
-                    work_push(&work, w.lo, w.lo + d.cut, w.depth + 1)) { status = OR_E_NOMEM; goto fail; }
+                /* push the children right to left: the leftmost is visited first */
+                for (uint32_t g = d.ngroups; g-- > 0;) {
+                    uint64_t a = g == 0 ? w.lo : w.lo + d.cuts[g - 1], b = g + 1 == d.ngroups ? w.hi : w.lo + d.cuts[g];
+                    if (work_push(&work, a, b, w.depth + 1)) { status = OR_E_NOMEM; goto fail; }
+                }
             } else {
                 leaf lf = {kid, w.lo, w.hi};
                 if (leaf_push(&leaves, lf)) { status = OR_E_NOMEM; goto fail; }

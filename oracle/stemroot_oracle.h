@@ -29,8 +29,10 @@ typedef struct {
     int      census_cap;     /* 1: m_i >= n_i => take all n_i rows                 */
     int      split;          /* 0: exact optimal 2-means cut (R5); 1: Lloyd's k-means,
                                 k = 2, from the (min, max) centroids (R26); 2: the
-                                same from k-means++ seeds drawn with seed (R27)     */
+                                same from k-means++ seeds drawn with seed (R27); 3:
+                                exact optimal 1-D k-means, k = kmeans_k (R29)       */
     int      metric_bounds;  /* 1: also true_metric and bound_metric (reading R28)   */
+    int      kmeans_k;       /* split = 3: groups per ROOT split, 2..8               */
 } or_opts;
 
 /* Structure-of-arrays plan.  Everything is malloc'ed; free with or_plan_free. */
@@ -77,6 +79,13 @@ uint64_t or_lloyd_cut(const uint32_t *t_sorted, uint64_t n, uint32_t *iters);
  * the seeds *c1, *c2 (either pointer may be NULL). */
 uint64_t or_kmpp_cut(const uint32_t *t_sorted, uint64_t n, uint64_t seed, uint32_t *c1, uint32_t *c2,
                      uint32_t *iters);
+/* Exact optimal 1-D k-means of sorted t[0..n) ("k-means ... any number
+ * above 2", reading R29): the partition into min(k, #distinct values) groups of
+ * consecutive distinct values with the least total SSE; among optimal ones the
+ * one whose last cut is smallest, then the cut before it, and so on.  Writes
+ * the cuts (row indices, ascending) to cuts[0 .. groups-2] and returns the
+ * number of groups (0 when n < 2 or all values are equal). */
+uint32_t or_kmeans_cuts(const uint32_t *t_sorted, uint64_t n, uint32_t k, uint64_t *cuts);
 /* Eq. 3: m = ceil((V/S^2) * (z/eps)^2) for a cluster with moments. */
 double or_eq3_m(uint64_t n, uint64_t S, uint64_t Q_lo, uint64_t Q_hi, double eps, double z, int clamp);
 /* Eq. 6, corrected numerator: k clusters given a_i = mu_i, b_i = V_i

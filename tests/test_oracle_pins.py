@@ -246,7 +246,7 @@ def test_kmpp_variant_fixed_point_and_bounds():
 
 def test_kmpp_plan_option():
     """or_opts.split = 2 builds a valid partition, depends on the seed only
-    through the split, and the oracle rejects split = 3"""
+    through the split, and the oracle rejects split = 4"""
     rng = np.random.default_rng(4)
     kid = rng.integers(0, 5, 4000).astype(np.uint32)
     t = (rng.lognormal(8, 0.6, 4000) + 1000 * (rng.random(4000) < 0.3)).astype(np.uint32)
@@ -254,7 +254,7 @@ def test_kmpp_plan_option():
     assert int(np.sum(p["n"])) == 4000
     assert O.plan(kid, t, 5, eps=0.03, z=Z95, seed=1, split=2)["n"].tolist() == p["n"].tolist()
     with pytest.raises(Exception):
-        O.plan(kid, t, 5, eps=0.03, z=Z95, seed=1, split=3)
+        O.plan(kid, t, 5, eps=0.03, z=Z95, seed=1, split=4)
 
 
 def test_split_exact_tie(golden):
@@ -626,3 +626,115 @@ def test_metric_bound_monte_carlo_coverage():
         e = np.array(errs[c])
         assert abs(e.mean()) < 4 * e.std() / math.sqrt(R)
         assert 0.89 <= cover[c] / R <= 0.995, cover
+
+
+# ----------------------------------------------------------------- exact k-means, k > 2 (R29)
+def _set_partitions(items, k):
+    """every partition of the list into exactly k nonempty blocks"""
+    if k == 1:
+        yield [items]
+        return
+    if len(items) < k:
+        return
+    first, rest = items[0], items[1:]
+    for p in _set_partitions(rest, k - 1):   # first alone
+        yield [[first]] + p
+    for p in _set_partitions(rest, k):       # first joins a block
+        for i in range(len(p)):
+            yield p[:i] + [[first] + p[i]] + p[i + 1:]
+
+
+def _groups_from_cuts(t, cuts):
+    b = [0] + list(cuts) + [len(t)]
+    return [t[b[i]:b[i + 1]] for i in range(len(b) - 1)]
+
+
+def test_kmeans_hand_vectors(golden):
+    g = golden("kmeans_hand.json")
+    for c in g["cuts"]:
+        assert O.kmeans_cuts(c["t"], c["k"]) == c["cuts"], c
+    tr = g["tree"]
+    p = O.plan([0] * len(tr["t"]), tr["t"], 1, eps=tr["eps"], z=tr["z"], split=3, kmeans_k=tr["k"])
+    assert [[int(a), int(b)] for a, b in zip(p["lo_ns"], p["hi_ns"])] == tr["leaves_lo_hi"]
+
+
+def test_kmeans_is_the_global_optimum_brute_force():
+    """R29: the DP's partition has the least SSE among ALL partitions of the
+    multiset into min(k, #distinct) nonempty groups (not only contiguous ones),
+    is contiguous in sorted order and never separates equal values."""
+    rng = random.Random(83)
+    for _ in range(300):
+        n = rng.randint(2, 8)
+        t = sorted(rng.choice([rng.randint(0, 5), rng.randint(0, 40)]) for _ in range(n))
+        if t[0] == t[-1]:
+            continue
+        k = rng.randint(2, 4)
+        d = len(set(t))
+        K = min(k, d)
+        cuts = O.kmeans_cuts(t, k)
+        assert len(cuts) == K - 1 and all(t[c - 1] < t[c] for c in cuts) and cuts == sorted(cuts)
+        mine = sum(_sse(g) for g in _groups_from_cuts(t, cuts))
+        best = min(sum(_sse(g) for g in p) for p in _set_partitions(list(t), K))
+        assert mine == best, (t, k, cuts)
+
+
+def test_kmeans_tie_rule_brute_force():
+    """Among the optimal contiguous distinct-value partitions the DP returns the
+    one with the smallest last cut, then the smallest cut before it (R29)."""
+    rng = random.Random(89)
+    ties = 0
+    for _ in range(400):
+        n = rng.randint(3, 10)
+        t = sorted(rng.choice([rng.randint(0, 3) * 10, rng.randint(0, 6) * 10]) for _ in range(n))
+        if t[0] == t[-1]:
+            continue
+        k = rng.randint(2, 4)
+        valid = [i for i in range(1, n) if t[i - 1] < t[i]]
+        K = min(k, len(valid) + 1)
+        cands = []
+        for cut in itertools.combinations(valid, K - 1):
+            cands.append((sum(_sse(g) for g in _groups_from_cuts(t, cut)), tuple(reversed(cut)), list(cut)))
+        best = min(c[0] for c in cands)
+        opt = [c for c in cands if c[0] == best]
+        ties += len(opt) > 1
+        assert O.kmeans_cuts(t, k) == min(opt, key=lambda c: c[1])[2], (t, k)
+    assert ties > 20
+
+
+def test_kmeans_k2_is_the_exact_two_means(golden):
+    """k = 2 reduces to the exact 2-means cut of R5 (same objective, same tie rule)"""
+    rng = random.Random(97)
+    for _ in range(1500):
+        n = rng.randint(2, 30)
+        t = sorted(rng.choice([rng.randint(0, 4), rng.randint(0, 100), rng.randint(0, 5000)]) for _ in range(n))
+        if t[0] == t[-1]:
+            continue
+        assert O.kmeans_cuts(t, 2) == [O.best_cut(t)]
+    for c in golden("split_tie.json")["cases"]:
+        t = [c["s"] * x for x in c["base"]]
+        assert O.kmeans_cuts(t, 2) == [c["cut"]]
+
+
+def test_kmeans_plan_k2_equals_default_split():
+    rng = np.random.default_rng(101)
+    kid, t = _random_trace(rng, 3000, 5)
+    a = O.plan(kid, t, 5, eps=0.02, z=Z95, seed=3)
+    b = O.plan(kid, t, 5, eps=0.02, z=Z95, seed=3, split=3, kmeans_k=2)
+    for key in ("kernel_id", "ordinal", "lo_ns", "hi_ns", "n", "sum_ns", "m", "sample_row"):
+        assert np.array_equal(a[key], b[key]), key
+    assert a["est_total_ns"] == b["est_total_ns"] and a["bound"] == b["bound"]
+
+
+@pytest.mark.parametrize("k", [3, 4, 8])
+def test_kmeans_plan_invariants(k):
+    rng = np.random.default_rng(103 + k)
+    kid = rng.integers(0, 4, 2500).astype(np.uint32)
+    t = (rng.integers(1, 60, 2500) * 37 + kid * 1000).astype(np.uint32)   # few distinct values per kernel
+    p = O.plan(kid, t, 4, eps=0.02, z=Z95, seed=5, split=3, kmeans_k=k)
+    assert int(p["n"].sum()) == len(t) and p["true_total_ns"] == int(t.astype(np.uint64).sum())
+    for kk in range(4):
+        idx = np.nonzero(p["kernel_id"] == kk)[0]
+        assert np.all(p["hi_ns"][idx][:-1] < p["lo_ns"][idx][1:])
+    assert p["bound"] <= 0.02 and np.all(p["m"] >= 1)
+    with pytest.raises(O.OracleError):
+        O.plan(kid, t, 4, split=3, kmeans_k=1)
