@@ -44,7 +44,8 @@ extern "C" {
 #endif
 
 #define STEMROOT_ABI_VERSION 4   /* 2: stem_opts.split; 3: split = 2 (k-means++ seeds);
-                                    4: metric_bounds, true_metric, bound_metric */
+                                    4: metric_bounds, true_metric, bound_metric; split = 3 and
+                                    kmeans_k; stem_stats.owned_rows/world/fused_exchange */
 
 #if defined(__GNUC__)
 #define STEM_API __attribute__((visibility("default")))
@@ -91,11 +92,17 @@ typedef struct stem_opts {
                                 centroids to its fixed point (R26); 2 the same Lloyd iteration
                                 from k-means++ seeds (uniform c1, D^2-weighted c2) drawn with
                                 Philox4x32-10 keyed by seed on (min t, max t, n) (R27), so the
-                                tree depends on seed; other values: STEM_E_INVAL                 */
+                                tree depends on seed; 3 the exact optimal 1-D k-means with
+                                kmeans_k groups per split (R29); other values: STEM_E_INVAL     */
     int      metric_bounds;  /* 1: also the exact total and the predicted relative error of each
                                 metric column (Eq. 5 with the metric in place of t, P:L150-159,
                                 P:L371; R28): stem_plan.true_metric / bound_metric.
                                 0 (default): point estimates only, those two pointers are NULL  */
+    int      kmeans_k;       /* split = 3: ROOT divides each cluster into min(kmeans_k, #distinct
+                                values) groups by the exact optimal 1-D k-means ("any
+                                number above 2 works well"; R29) and keeps them iff
+                                Eq. 8 over the groups beats Eq. 7; 2..8 (default 3), ignored for
+                                the other split rules                                            */
     void    *stream;         /* cudaStream_t to run on; NULL = the legacy default stream         */
 } stem_opts;
 
@@ -187,7 +194,7 @@ typedef struct stem_stage_time {
 typedef struct stem_ctx stem_ctx;
 
 /* Fill *o with the defaults: seed 0, z 0, scope 0, root 1, clamp_in_split 1,
- * census_cap 0, split 0, metric_bounds 0, stream NULL. */
+ * census_cap 0, split 0, metric_bounds 0, kmeans_k 3, stream NULL. */
 STEM_API int stem_default_opts(stem_opts *o);
 
 /* A workspace bound to one CUDA device; keeps device scratch between calls. */

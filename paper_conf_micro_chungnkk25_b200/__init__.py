@@ -29,7 +29,7 @@ _ROOT = os.path.dirname(_HERE)
 _CSRC = os.path.join(_HERE, "csrc")
 LIB_PATH = os.path.join(_HERE, "lib", "libstemroot.so")
 HEADER = os.path.join(_ROOT, "include", "stemroot.h")
-SOURCES = ["capi.cu", "sort.cu", "root.cu", "stem.cu", "dist.cu", "metric.cu"]
+SOURCES = ["capi.cu", "sort.cu", "root.cu", "stem.cu", "dist.cu", "metric.cu", "kmeans.cu"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "--fmad=false",
               "--extended-lambda", "-Xcompiler", "-fPIC,-fvisibility=hidden", "-shared"]
 
@@ -73,7 +73,7 @@ class stem_trace(C.Structure):
 class stem_opts(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("z", C.c_double), ("scope", C.c_int), ("root", C.c_int),
                 ("clamp_in_split", C.c_int), ("census_cap", C.c_int), ("split", C.c_int),
-                ("metric_bounds", C.c_int), ("stream", C.c_void_p)]
+                ("metric_bounds", C.c_int), ("kmeans_k", C.c_int), ("stream", C.c_void_p)]
 
 
 class stem_cluster(C.Structure):
@@ -246,12 +246,12 @@ def _trace(kernel_id, exec_ns, n_kernels, metrics, allow_empty=False):
     return tr, kdev, (k_keep, t_keep, m_keep)
 
 
-def _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev):
+def _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev, kmeans_k=3):
     if stream is None and dev >= 0:
         import torch
         stream = torch.cuda.current_stream(dev).cuda_stream
     return stem_opts(seed & 0xFFFFFFFFFFFFFFFF, z, scope, int(root), int(clamp_in_split), int(census_cap),
-                     int(split), int(metric_bounds), stream or None)
+                     int(split), int(metric_bounds), int(kmeans_k), stream or None)
 
 
 def _plan_to_numpy(p: stem_plan) -> dict:
@@ -371,11 +371,11 @@ class Context:
     def plan(self, kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, metrics=None,
              seed: int = 0, z: float = 0.0, scope: int = 0, root: bool = True, clamp_in_split: bool = True,
              census_cap: bool = False, stream=None, to_host: bool = True, split: int = 0,
-             metric_bounds: bool = False):
+             metric_bounds: bool = False, kmeans_k: int = 3):
         """stem_root_plan_ctx.  Returns the host plan as numpy arrays, or None when to_host=False
         (the plan then stays on the device: see device_plan())."""
         tr, dev, keep = _trace(kernel_id, exec_ns, n_kernels, metrics)
-        o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev)
+        o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev, kmeans_k)
         out = C.POINTER(stem_plan)()
         st = lib().stem_root_plan_ctx(self._h, C.byref(tr), eps, conf, C.byref(o),
                                       C.byref(out) if to_host else None)
@@ -390,10 +390,10 @@ class Context:
     def plan_dist(self, comm: "Comm", kernel_id, exec_ns, n_kernels: int, global_row_base: int, eps: float = 0.05,
                   conf: float = 0.95, metrics=None, seed: int = 0, z: float = 0.0, scope: int = 0, root: bool = True,
                   clamp_in_split: bool = True, census_cap: bool = False, stream=None, to_host: bool = True,
-                  split: int = 0, metric_bounds: bool = False):
+                  split: int = 0, metric_bounds: bool = False, kmeans_k: int = 3):
         """stem_root_plan_dist (collective).  Returns the global plan on rank 0, None elsewhere."""
         tr, dev, keep = _trace(kernel_id, exec_ns, n_kernels, metrics, allow_empty=True)
-        o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev)
+        o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev, kmeans_k)
         out = C.POINTER(stem_plan)()
         st = lib().stem_root_plan_dist(self._h, comm._h, C.byref(tr), global_row_base, eps, conf, C.byref(o),
                                        C.byref(out) if to_host else None)
@@ -411,13 +411,14 @@ class Context:
         library allocated it (no numpy conversion): a HostPlan whose close()
         calls stem_plan_free.  On ranks other than 0 of a dist plan it is empty."""
         opt = {k: kw.pop(k) for k in list(kw) if k in ("seed", "z", "scope", "root", "clamp_in_split",
-                                                          "census_cap", "split", "metric_bounds", "stream")}
+                                                          "census_cap", "split", "metric_bounds", "stream",
+                                                          "kmeans_k")}
         if kw:
             raise TypeError(f"unknown options {sorted(kw)}")
         tr, dev, keep = _trace(kernel_id, exec_ns, n_kernels, metrics, allow_empty=comm is not None)
         o = _opts(opt.get("seed", 0), opt.get("z", 0.0), opt.get("scope", 0), opt.get("root", True),
                   opt.get("clamp_in_split", True), opt.get("census_cap", False), opt.get("split", 0),
-                  opt.get("metric_bounds", False), opt.get("stream"), dev)
+                  opt.get("metric_bounds", False), opt.get("stream"), dev, opt.get("kmeans_k", 3))
         out = C.POINTER(stem_plan)()
         if comm is None:
             st = lib().stem_root_plan_ctx(self._h, C.byref(tr), eps, conf, C.byref(o), C.byref(out))
@@ -457,10 +458,10 @@ class Context:
 
 def plan(kernel_id, exec_ns, n_kernels: int, eps: float = 0.05, conf: float = 0.95, metrics=None, seed: int = 0,
          z: float = 0.0, scope: int = 0, root: bool = True, clamp_in_split: bool = True, census_cap: bool = False,
-         stream=None, split: int = 0, metric_bounds: bool = False) -> dict:
+         stream=None, split: int = 0, metric_bounds: bool = False, kmeans_k: int = 3) -> dict:
     """stem_root_plan: one-shot plan (temporary workspace), host plan out."""
     tr, dev, keep = _trace(kernel_id, exec_ns, n_kernels, metrics)
-    o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev)
+    o = _opts(seed, z, scope, root, clamp_in_split, census_cap, split, metric_bounds, stream, dev, kmeans_k)
     out = C.POINTER(stem_plan)()
     _check(lib().stem_root_plan(C.byref(tr), eps, conf, C.byref(o), C.byref(out)), "stem_root_plan")
     del keep

@@ -75,6 +75,8 @@ void Ctx::release() {
     dfree(out_cluster, cap_out_cluster); dfree(out_weight, cap_out_weight);
     dfree(big_ent, cap_big_ent); dfree(big_part, cap_big_part); dfree(big_thr, cap_big_thr);
     dfree(peer_dst, cap_peer_dst);
+    dfree(km_dpos, cap_km_dpos); dfree(km_arg, cap_km_arg); dfree(km_ngrp, cap_km_ngrp);
+    dfree(km_dP, cap_km_dP); dfree(km_F, cap_km_F);
     dfree(part_cnt, cap_part_cnt); dfree(dist_cnt, cap_dist_cnt);
     for (int i = 0; i < 3; i++) { dfree(xfer_u32[i], cap_xfer_u32[i]); dfree(recv_u32[i], cap_recv_u32[i]); }
     dfree(xfer_f64, cap_xfer_f64); dfree(xfer_f64b, cap_xfer_f64b); dfree(red_part2, cap_red2);
@@ -122,7 +124,8 @@ static int validate(const stem_trace *tr, double eps, double conf, const stem_op
     if (!(o.z > 0.0) && !(conf > 0.0 && conf < 1.0)) return STEM_E_INVAL;
     if (o.z < 0.0 || std::isnan(o.z) || std::isinf(o.z)) return STEM_E_INVAL;
     if (o.scope < 0 || o.scope > 2) return STEM_E_INVAL;
-    if (o.split < 0 || o.split > 2) return STEM_E_INVAL;
+    if (o.split < 0 || o.split > 3) return STEM_E_INVAL;
+    if (o.split == 3 && (o.kmeans_k < 2 || o.kmeans_k > 8)) return STEM_E_INVAL;
     if (o.metric_bounds < 0 || o.metric_bounds > 1) return STEM_E_INVAL;
     if (tr->n == 0 || !tr->kernel_id || !tr->exec_ns) return STEM_E_INVAL;
     if (tr->n_metrics > 64 || (tr->n_metrics > 0 && !tr->metrics)) return STEM_E_INVAL;
@@ -167,7 +170,9 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
     }
     CKS(sort_trace(c, kid, t, nullptr, n, K, !o.census_cap));   // a1
     CKS(prefix_moments(c, n));                        // a2
-    if (o.root) {
+    if (o.root && o.split == 3) {
+        CKS(root_levels_kmeans(c, n, K, eps, z, k2, o.clamp_in_split ? 1 : 0, (uint32_t)o.kmeans_k));   // a3, a4
+    } else if (o.root) {
         CKS(root_levels(c, n, K, eps, z, k2, o.clamp_in_split ? 1 : 0, o.split, o.seed));   // a3, a4
     } else {
         CKS(stem_only_leaves(c, n, K));
@@ -337,6 +342,7 @@ int stem_default_opts(stem_opts *o) {
     o->census_cap = 0;
     o->split = 0;
     o->metric_bounds = 0;
+    o->kmeans_k = 3;
     o->stream = nullptr;
     return STEM_OK;
 }
@@ -403,7 +409,8 @@ int stem_root_plan_dist(stem_ctx *ctx, stem_comm *comm, const stem_trace *local_
     // rank returns the same error instead of leaving its peers in a collective
     int local = STEM_OK;
     if (!local_shard || !(eps > 0.0 && eps < 1.0) || (!(o.z > 0.0) && !(conf > 0.0 && conf < 1.0)) || o.z < 0.0 ||
-        std::isnan(o.z) || std::isinf(o.z) || o.scope < 0 || o.scope > 2 || o.split < 0 || o.split > 2 ||
+        std::isnan(o.z) || std::isinf(o.z) || o.scope < 0 || o.scope > 2 || o.split < 0 || o.split > 3 ||
+        (o.split == 3 && (o.kmeans_k < 2 || o.kmeans_k > 8)) ||
         o.metric_bounds < 0 || o.metric_bounds > 1 || tr->n_metrics > 64 ||
         (tr->n && (!tr->kernel_id || !tr->exec_ns)) || (tr->n && tr->n_metrics && !tr->metrics))
         local = STEM_E_INVAL;

@@ -834,7 +834,10 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
         CKS(c.ensure_all(R, KL, nm));
         CKS(sort_trace(c, c.recv_u32[0], c.recv_u32[1], c.recv_u32[2], R, KL, !o.census_cap));
         CKS(prefix_moments(c, R));
-        if (o.root) {
+        if (o.root && o.split == 3) {
+            CKS(root_levels_kmeans(c, R, KL, eps, c.z, c.z / eps * (c.z / eps), o.clamp_in_split ? 1 : 0,
+                                   (uint32_t)o.kmeans_k));
+        } else if (o.root) {
             CKS(root_levels(c, R, KL, eps, c.z, c.z / eps * (c.z / eps), o.clamp_in_split ? 1 : 0, o.split,
                             o.seed));
         } else {

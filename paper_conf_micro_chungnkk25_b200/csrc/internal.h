@@ -209,6 +209,11 @@ struct Ctx {
     double *red_part2 = nullptr; size_t cap_red2 = 0;
     void *g_clusters = nullptr, *g_row = nullptr, *g_cluster = nullptr, *g_weight = nullptr;
     size_t cap_g_clusters = 0, cap_g_row = 0, cap_g_cluster = 0, cap_g_weight = 0;
+    // split = 3 (kmeans.cu): distinct-value starts, DP tables, groups per cluster
+    uint32_t *km_dpos = nullptr, *km_arg = nullptr, *km_ngrp = nullptr;
+    size_t cap_km_dpos = 0, cap_km_arg = 0, cap_km_ngrp = 0;
+    uint64_t *km_dP = nullptr; size_t cap_km_dP = 0;
+    double *km_F = nullptr; size_t cap_km_F = 0;
     void *peer_dst = nullptr; size_t cap_peer_dst = 0;   // fused exchange: the owners' windows (PeerDst)
     uint64_t row_bases[65] = {0};
     uint64_t n_local_rows = 0;
@@ -252,6 +257,8 @@ int prefix_moments(Ctx &c, uint64_t n);                                         
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp,
                 int split, uint64_t seed);   // a3, a4 (split: 0 exact 2-means, 1 Lloyd, 2 k-means++ Lloyd)
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
+// split = 3: ROOT with exact optimal 1-D k-means splits into kk groups (kmeans.cu, R29)
+int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, uint32_t kk);
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,
                       uint32_t *tailh);   // pre-pass only
 int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,

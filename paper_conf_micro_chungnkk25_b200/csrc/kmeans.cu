@@ -1,0 +1,457 @@
+// kmeans.cu -- ROOT with k-ary splits, split = 3 (R29): each
+// frontier cluster is divided by the exact optimal 1-D k-means ("a
+// clustering method (e.g., k-means) ... any number above 2 works well") into
+// min(k, #distinct values) groups of consecutive distinct values, and the
+// split is kept iff Eq. 8 over the groups beats Eq. 7.
+//
+// The k-means is the dynamic program over the cluster's distinct values
+//   F[1][b] = S(0,b)^2 / n(0,b),  F[j][b] = max_a F[j-1][a] + S(a,b)^2 / n(a,b)
+// (maximising sum_g S_g^2 / n_g = minimising the SSE).  The group cost obeys
+// the quadrangle inequality, so the smallest optimal a is non-decreasing in b
+// and each layer is solved by divide and conquer in O(d log d): one warp per
+// cluster, 32 candidate a per step.  Values are fp64; candidates within 2^-40
+// of the best are compared EXACTLY (the prefix partitions rebuilt from the
+// argmax table, sums of fractions in 768-bit integers), and ties keep the
+// smaller a -- the oracle's rule (smallest last cut, then the one before).
+//
+// Distinct values: row i starts one when it starts a kernel group or
+// t[i-1] < t[i]; their positions and exact prefix sums are built once per
+// plan for the whole trace, so a cluster's distinct values are the contiguous
+// slice of that list between its bounds (a cut never separates equal times).
+#include "internal.h"
+
+namespace sr {
+
+constexpr int kKmMax = 8;              // largest kmeans_k
+constexpr int kKmLimbs = 12;           // 768-bit integers (sums of <= 8 fractions, cross-multiplied)
+
+// ---------------------------------------------------------------- exact fractions (rare near-tie path)
+struct KBig { uint64_t w[kKmLimbs]; };
+
+__device__ __noinline__ void kbig_mul(const KBig &a, const KBig &b, KBig &r) {
+    uint64_t o[kKmLimbs];
+    for (int i = 0; i < kKmLimbs; i++) o[i] = 0;
+    for (int i = 0; i < kKmLimbs; i++) {
+        if (!a.w[i]) continue;
+        uint64_t carry = 0;
+        for (int j = 0; i + j < kKmLimbs; j++) {
+            const uint64_t lo = a.w[i] * b.w[j], hi = __umul64hi(a.w[i], b.w[j]);
+            uint64_t s = o[i + j] + lo;
+            uint64_t c1 = s < lo;
+            s += carry;
+            c1 += s < carry;
+            o[i + j] = s;
+            carry = hi + c1;
+        }
+    }
+    for (int i = 0; i < kKmLimbs; i++) r.w[i] = o[i];
+}
+
+__device__ __forceinline__ void kbig_add(KBig &a, const KBig &b) {
+    uint64_t carry = 0;
+    for (int i = 0; i < kKmLimbs; i++) {
+        uint64_t s = a.w[i] + b.w[i];
+        const uint64_t c1 = s < a.w[i];
+        s += carry;
+        carry = c1 + (s < carry);
+        a.w[i] = s;
+    }
+}
+
+__device__ __forceinline__ int kbig_cmp(const KBig &a, const KBig &b) {
+    for (int i = kKmLimbs - 1; i >= 0; i--)
+        if (a.w[i] != b.w[i]) return a.w[i] < b.w[i] ? -1 : 1;
+    return 0;
+}
+
+struct KFrac { KBig num, den; };
+
+// f + S^2 / n
+__device__ __noinline__ void kfrac_add(KFrac &f, uint64_t S, uint64_t n) {
+    KBig bn{}, s2{}, a, b;
+    bn.w[0] = n;
+    s2.w[0] = S * S;
+    s2.w[1] = __umul64hi(S, S);
+    kbig_mul(f.num, bn, a);
+    kbig_mul(s2, f.den, b);
+    kbig_add(a, b);
+    f.num = a;
+    kbig_mul(f.den, bn, b);
+    f.den = b;
+}
+
+__device__ __noinline__ int kfrac_cmp(const KFrac &x, const KFrac &y) {
+    KBig l, r;
+    kbig_mul(x.num, y.den, l);
+    kbig_mul(y.num, x.den, r);
+    return kbig_cmp(l, r);
+}
+
+struct KmArgs {
+    const uint32_t *f_lo, *f_hi;
+    const uint64_t *ctot;          // packed (count << 32 | rows) of the frontier
+    const uint32_t *dpos;          // [D + 1] rows starting a distinct value (dpos[D] = n)
+    const uint64_t *dP;            // [D + 1] exact sum of t before them
+    uint64_t D;
+    double *F;                     // [kKmMax + 1][D + 1] fp64 DP values
+    uint32_t *arg;                 // [kKmMax + 1][D + 1] argmax (distinct index relative to the cluster)
+    uint32_t k;
+    uint32_t *cutk;                // [cluster][kKmMax - 1] cuts relative to lo
+    uint32_t *ngrp;                // [cluster] groups (0: leaf)
+};
+
+struct KmCluster {
+    uint64_t D0, lo;
+    uint32_t d;
+};
+
+__device__ __forceinline__ uint64_t km_pos(const KmArgs &a, const KmCluster &c, uint32_t u) {
+    return (uint64_t)a.dpos[c.D0 + u] - c.lo;
+}
+__device__ __forceinline__ uint64_t km_P(const KmArgs &a, const KmCluster &c, uint32_t u) {
+    return a.dP[c.D0 + u] - a.dP[c.D0];
+}
+
+// exact value of F[j-1][a] + S(a,b)^2/n(a,b): the prefix partition of the first
+// a distinct values into j - 1 groups rebuilt from the argmax table
+__device__ __noinline__ void km_exact(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t a, uint32_t b,
+                                      KFrac &out) {
+    for (int i = 0; i < kKmLimbs; i++) out.num.w[i] = out.den.w[i] = 0;
+    out.den.w[0] = 1;
+    const size_t L = g.D + 1;
+    uint32_t hi = a;
+    for (uint32_t l = j - 1; l >= 1; l--) {
+        const uint32_t lo = l == 1 ? 0u : g.arg[(size_t)l * L + c.D0 + hi];
+        kfrac_add(out, km_P(g, c, hi) - km_P(g, c, lo), km_pos(g, c, hi) - km_pos(g, c, lo));
+        hi = lo;
+        if (l == 1) break;
+    }
+    kfrac_add(out, km_P(g, c, b) - km_P(g, c, a), km_pos(g, c, b) - km_pos(g, c, a));
+}
+
+__device__ __forceinline__ double km_score(const KmArgs &g, const KmCluster &c, uint32_t a, uint32_t b) {
+    const double s = rn64(km_P(g, c, b) - km_P(g, c, a));
+    return __ddiv_rn(__dmul_rn(s, s), rn64(km_pos(g, c, b) - km_pos(g, c, a)));
+}
+
+// best a in [a0, a1] for F[j][b] (warp-uniform result); exact among near-ties
+__device__ void km_argmax(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t b, uint32_t a0, uint32_t a1,
+                          double &vbest, uint32_t &abest) {
+    const int lane = threadIdx.x & 31;
+    const size_t L = g.D + 1;
+    const double win = 1.0 - 0x1p-40;
+    bool have = false;
+    vbest = 0.0;
+    abest = a0;
+    for (uint32_t base = a0; base <= a1; base += 32) {
+        const uint32_t a = base + lane;
+        const bool ok = a <= a1;
+        const double v = ok ? __dadd_rn(g.F[(size_t)(j - 1) * L + c.D0 + a], km_score(g, c, a, b)) : -1.0;
+        double vr = v;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) vr = fmax(vr, __shfl_xor_sync(0xffffffffu, vr, o));
+        if (have && vr < __dmul_rn(vbest, win)) continue;        // nothing here comes close
+        const double top = have ? fmax(vr, vbest) : vr;
+        const double thr = __dmul_rn(top, win);
+        const uint32_t cm = __ballot_sync(0xffffffffu, ok && v >= thr);
+        const bool prev_in = have && vbest >= thr;
+        if (__popc(cm) == 1 && !prev_in) {
+            const int src = __ffs(cm) - 1;
+            vbest = __shfl_sync(0xffffffffu, v, src);
+            abest = base + src;
+            have = true;
+            continue;
+        }
+        // near tie: exact comparison, candidates in ascending a (ties keep the smaller)
+        KFrac bf, cf;
+        bool bset = false;
+        if (prev_in) {
+            km_exact(g, c, j, abest, b, bf);
+            bset = true;
+        }
+        uint32_t m = cm;
+        while (m) {
+            const int src = __ffs(m) - 1;
+            m &= m - 1;
+            km_exact(g, c, j, base + src, b, cf);
+            if (!bset || kfrac_cmp(cf, bf) > 0) {
+                bf = cf;
+                bset = true;
+                abest = base + src;
+                vbest = __shfl_sync(0xffffffffu, v, src);
+            }
+        }
+        have = true;
+    }
+}
+
+// one warp per cluster: the DP layers by divide and conquer, then the cuts
+__global__ void __launch_bounds__(128) kmeans_cut_kernel(KmArgs g) {
+    const uint32_t C = (uint32_t)(*g.ctot >> 32);
+    const int lane = threadIdx.x & 31;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const size_t L = g.D + 1;
+    for (uint64_t ci = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; ci < C; ci += nwarps) {
+        KmCluster c;
+        c.lo = g.f_lo[ci];
+        const uint64_t hi = g.f_hi[ci];
+        c.D0 = lower_bound(g.dpos, g.D + 1, (uint32_t)c.lo);
+        c.d = (uint32_t)(lower_bound(g.dpos, g.D + 1, (uint32_t)hi) - c.D0);
+        const uint32_t K = min(g.k, c.d);
+        if (K < 2) {
+            if (lane == 0) g.ngrp[ci] = 0;
+            continue;
+        }
+        for (uint32_t b = 1 + lane; b <= c.d; b += 32) g.F[1 * L + c.D0 + b] = km_score(g, c, 0, b);
+        __syncwarp();
+        for (uint32_t j = 2; j <= K; j++) {
+            // divide and conquer over b in [j, d], a in [j - 1, b - 1]; explicit stack (warp-uniform)
+            uint32_t st[4 * 40];
+            int sp = 0;
+            st[0] = j; st[1] = c.d; st[2] = j - 1; st[3] = c.d - 1;
+            sp = 1;
+            while (sp) {
+                sp--;
+                const uint32_t blo = st[4 * sp], bhi = st[4 * sp + 1], alo = st[4 * sp + 2], ahi = st[4 * sp + 3];
+                if (blo > bhi) continue;
+                const uint32_t mid = blo + (bhi - blo) / 2;
+                double v;
+                uint32_t a;
+                km_argmax(g, c, j, mid, alo, min(ahi, mid - 1), v, a);
+                if (lane == 0) {
+                    g.F[(size_t)j * L + c.D0 + mid] = v;
+                    g.arg[(size_t)j * L + c.D0 + mid] = a;
+                }
+                if (mid < bhi) { st[4 * sp] = mid + 1; st[4 * sp + 1] = bhi; st[4 * sp + 2] = a; st[4 * sp + 3] = ahi; sp++; }
+                if (mid > blo) { st[4 * sp] = blo; st[4 * sp + 1] = mid - 1; st[4 * sp + 2] = alo; st[4 * sp + 3] = a; sp++; }
+            }
+            __syncwarp();
+        }
+        if (lane == 0) {
+            uint32_t b = c.d;
+            for (uint32_t j = K; j >= 2; j--) {
+                b = g.arg[(size_t)j * L + c.D0 + b];
+                g.cutk[ci * (kKmMax - 1) + (j - 2)] = (uint32_t)km_pos(g, c, b);
+            }
+            g.ngrp[ci] = K;
+        }
+        __syncwarp();
+    }
+}
+
+// ---------------------------------------------------------------- decision and children (Eq. 7 vs Eq. 8)
+struct KdArgs {
+    const uint32_t *f_lo, *f_hi;
+    const uint64_t *f_S;
+    const u128 *f_Q;
+    const uint64_t *ctot;
+    const uint32_t *cutk, *ngrp;
+    const uint64_t *PS1;
+    const u128 *PS2;
+    const uint32_t *t;
+    uint32_t *flags;
+    uint32_t *nlo, *nhi;
+    uint64_t *nS;
+    u128 *nQ;
+    uint64_t *total;
+    double eps, z, k2;
+    int clamp;
+};
+
+__device__ __forceinline__ double km_eq6(double g, double mu, double V, int clamp) {
+    if (V == 0.0) return clamp ? 1.0 : 0.0;
+    double m = ceil(__dmul_rn(g, __dsqrt_rn(__ddiv_rn(V, mu))));
+    if (clamp && m < 1.0) m = 1.0;
+    return m;
+}
+
+__global__ void __launch_bounds__(128) kmeans_decide_kernel(KdArgs a) {
+    const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= (*a.ctot >> 32)) return;
+    const uint32_t G = a.ngrp[c];
+    if (G < 2) return;
+    const uint64_t lo = a.f_lo[c], hi = a.f_hi[c], n = hi - lo, S = a.f_S[c];
+    const u128 Q = a.f_Q[c];
+    // group boundaries and moments
+    uint64_t bnd[kKmMax + 1], gS[kKmMax];
+    u128 gQ[kKmMax];
+    bnd[0] = lo;
+    for (uint32_t i = 1; i < G; i++) bnd[i] = lo + a.cutk[c * (kKmMax - 1) + (i - 1)];
+    bnd[G] = hi;
+    uint64_t s0, sp;
+    u128 q0, qp;
+    pref12(a.PS1, a.PS2, a.t, lo, s0, q0);
+    sp = s0;
+    qp = q0;
+    for (uint32_t i = 0; i < G; i++) {
+        uint64_t s1;
+        u128 q1;
+        if (i + 1 == G) { s1 = s0 + S; q1 = q0 + Q; }
+        else pref12(a.PS1, a.PS2, a.t, bnd[i + 1], s1, q1);
+        gS[i] = s1 - sp;
+        gQ[i] = q1 - qp;
+        sp = s1;
+        qp = q1;
+    }
+    // Eq. 7: tau_old = m * Xbar, m from Eq. 3
+    const u128 V = (u128)n * Q - (u128)S * S;
+    const double mu = __ddiv_rn(rn64(S), rn64(n));
+    double m_old;
+    if (V == 0) m_old = a.clamp ? 1.0 : 0.0;
+    else {
+        const double dS = rn64(S);
+        m_old = ceil(__dmul_rn(__ddiv_rn(rn128(V), __dmul_rn(dS, dS)), a.k2));
+        if (a.clamp && m_old < 1.0) m_old = 1.0;
+    }
+    const double tau_old = __dmul_rn(m_old, mu);
+    // Eq. 8 over the G children, Eq. 6 with c from the parent's total, left to right
+    double gmu[kKmMax], gV[kKmMax];
+    for (uint32_t i = 0; i < G; i++) {
+        const uint64_t ni = bnd[i + 1] - bnd[i];
+        gmu[i] = __ddiv_rn(rn64(gS[i]), rn64(ni));
+        gV[i] = rn128((u128)ni * gQ[i] - (u128)gS[i] * gS[i]);
+    }
+    const double w = __ddiv_rn(__dmul_rn(a.eps, rn64(S)), a.z);
+    const double cc = __dmul_rn(w, w);
+    double ssum = 0.0;
+    for (uint32_t i = 0; i < G; i++) {
+        const double term = __dsqrt_rn(__dmul_rn(gmu[i], gV[i]));
+        ssum = i == 0 ? term : __dadd_rn(ssum, term);
+    }
+    const double gg = __ddiv_rn(ssum, cc);
+    double tau_new = 0.0;
+    for (uint32_t i = 0; i < G; i++) {
+        const double term = __dmul_rn(km_eq6(gg, gmu[i], gV[i], a.clamp), gmu[i]);
+        tau_new = i == 0 ? term : __dadd_rn(tau_new, term);
+    }
+    if (!(tau_new < tau_old)) return;   // strict: a leaf
+    for (uint32_t i = 0; i < G; i++) {
+        if (i > 0) atomicOr(&a.flags[bnd[i] >> 5], 1u << (bnd[i] & 31));
+        const uint64_t x0 = bnd[i], x1 = bnd[i + 1];
+        if (x1 - x0 >= 2 && a.t[x0] != a.t[x1 - 1]) {
+            const uint64_t slot = atomicAdd((unsigned long long *)a.total,
+                                            (unsigned long long)((1ull << 32) | (x1 - x0))) >> 32;
+            a.nlo[slot] = (uint32_t)x0;
+            a.nhi[slot] = (uint32_t)x1;
+            a.nS[slot] = gS[i];
+            a.nQ[slot] = gQ[i];
+        }
+    }
+}
+
+// ---------------------------------------------------------------- setup kernels
+// initial frontier: the non-trivial kernel groups (order immaterial)
+__global__ void kmeans_init_kernel(const uint32_t *goff, uint32_t K, const uint32_t *t, const uint64_t *PS1,
+                                   const u128 *PS2, uint32_t *nlo, uint32_t *nhi, uint64_t *nS, u128 *nQ,
+                                   uint64_t *total) {
+    const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (g >= K) return;
+    const uint32_t lo = goff[g], hi = goff[g + 1];
+    if (hi - lo < 2 || t[lo] == t[hi - 1]) return;
+    uint64_t s0, s1;
+    u128 q0, q1;
+    pref12(PS1, PS2, t, lo, s0, q0);
+    pref12(PS1, PS2, t, hi, s1, q1);
+    const uint64_t slot = atomicAdd((unsigned long long *)total, (unsigned long long)((1ull << 32) | (hi - lo))) >> 32;
+    nlo[slot] = lo;
+    nhi[slot] = hi;
+    nS[slot] = s1 - s0;
+    nQ[slot] = q1 - q0;
+}
+
+__global__ void kmeans_sentinel_kernel(const uint64_t *PS1, const uint32_t *t, uint64_t n, uint32_t *dpos,
+                                       uint64_t *dP) {
+    if (threadIdx.x == 0) {
+        *dpos = (uint32_t)n;
+        *dP = pref1(PS1, t, n);
+    }
+}
+
+int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, uint32_t kk) {
+    cudaStream_t st = c.stream;
+    if (kk < 2 || kk > (uint32_t)kKmMax) return STEM_E_INVAL;
+    CKS(stem_only_leaves(c, n, K));   // group starts in the leaf bitmap
+    // distinct-value starts of the whole trace: positions and exact prefix sums
+    CKS(c.ensure(c.km_dpos, c.cap_km_dpos, sizeof(uint32_t) * (n + 2)));
+    CKS(c.ensure(c.km_dP, c.cap_km_dP, sizeof(uint64_t) * (n + 2)));
+    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(n) + 1) * sizeof(uint64_t)));
+    {
+        const uint32_t *t = c.t_sorted, *fl = c.flags;
+        const uint64_t *PS1 = c.PS1;
+        uint32_t *dpos = c.km_dpos;
+        uint64_t *dP = c.km_dP;
+        exclusive_scan<uint64_t>(
+            [t, fl] __device__(uint64_t i) -> uint64_t {
+                return (i == 0 || ((fl[i >> 5] >> (i & 31)) & 1u) || t[i - 1] < t[i]) ? 1ull : 0ull;
+            },
+            [t, dpos, dP, PS1] __device__(uint64_t i, uint64_t pre, uint64_t v) {
+                if (!v) return;
+                dpos[pre] = (uint32_t)i;
+                dP[pre] = pref1(PS1, t, i);
+            },
+            n, (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
+    }
+    uint64_t D = 0;
+    CK(cudaMemcpyAsync(&D, &c.scalars->scan_total64, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    kmeans_sentinel_kernel<<<1, 32, 0, st>>>(c.PS1, c.t_sorted, n, c.km_dpos + D, c.km_dP + D);   // dpos[D] = n
+    c.launches++;
+    CKS(c.ensure(c.km_F, c.cap_km_F, sizeof(double) * (size_t)(kKmMax + 1) * (D + 1)));
+    CKS(c.ensure(c.km_arg, c.cap_km_arg, sizeof(uint32_t) * (size_t)(kKmMax + 1) * (D + 1)));
+    // initial frontier
+    uint64_t Cmax = (uint64_t)K + 1;
+    for (int b = 0; b < 2; b++) {
+        CKS(c.ensure(c.f_lo[b], c.cap_flo[b], sizeof(uint32_t) * Cmax));
+        CKS(c.ensure(c.f_hi[b], c.cap_fhi[b], sizeof(uint32_t) * Cmax));
+        CKS(c.ensure(c.f_S[b], c.cap_fS[b], sizeof(uint64_t) * Cmax));
+        CKS(c.ensure(c.f_Q[b], c.cap_fQ[b], sizeof(u128) * Cmax));
+    }
+    CK(cudaMemsetAsync(&c.scalars->ftot[0], 0, sizeof(uint64_t), st));
+    if (K) {
+        kmeans_init_kernel<<<(unsigned)((K + 255) / 256), 256, 0, st>>>(c.goff, K, c.t_sorted, c.PS1, c.PS2, c.f_lo[0],
+                                                                       c.f_hi[0], c.f_S[0], c.f_Q[0],
+                                                                       &c.scalars->ftot[0]);
+        c.launches++;
+    }
+    uint64_t tot = 0;
+    CK(cudaMemcpyAsync(&tot, &c.scalars->ftot[0], sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    int cur = 0;
+    uint32_t levels = 0;
+    while (tot >> 32) {
+        const uint64_t C = tot >> 32;
+        levels++;
+        c.stats.active_rows += tot & 0xFFFFFFFFull;
+        const int nxt = cur ^ 1;
+        CKS(c.ensure(c.cut, c.cap_cut, sizeof(uint32_t) * C * (kKmMax - 1)));
+        CKS(c.ensure(c.km_ngrp, c.cap_km_ngrp, sizeof(uint32_t) * C));
+        const uint64_t cap = kk * C;   // at most kk children per cluster
+        CKS(c.ensure(c.f_lo[nxt], c.cap_flo[nxt], sizeof(uint32_t) * cap));
+        CKS(c.ensure(c.f_hi[nxt], c.cap_fhi[nxt], sizeof(uint32_t) * cap));
+        CKS(c.ensure(c.f_S[nxt], c.cap_fS[nxt], sizeof(uint64_t) * cap));
+        CKS(c.ensure(c.f_Q[nxt], c.cap_fQ[nxt], sizeof(u128) * cap));
+        const int tk_s = c.stage_begin("root_split");
+        KmArgs ka{c.f_lo[cur], c.f_hi[cur], &c.scalars->ftot[cur], c.km_dpos, c.km_dP, D, c.km_F, c.km_arg, kk,
+                  c.cut, c.km_ngrp};
+        kmeans_cut_kernel<<<(unsigned)min((C + 3) / 4, (uint64_t)c.sms * 16), 128, 0, st>>>(ka);
+        c.launches++;
+        c.stage_end(tk_s, 12 * (tot & 0xFFFFFFFFull));
+        CK(cudaGetLastError());
+        const int tk_d = c.stage_begin("root_decide");
+        CK(cudaMemsetAsync(&c.scalars->ftot[nxt], 0, sizeof(uint64_t), st));
+        KdArgs da{c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], &c.scalars->ftot[cur], c.cut, c.km_ngrp, c.PS1,
+                  c.PS2, c.t_sorted, c.flags, c.f_lo[nxt], c.f_hi[nxt], c.f_S[nxt], c.f_Q[nxt],
+                  &c.scalars->ftot[nxt], eps, z, k2, clamp};
+        kmeans_decide_kernel<<<(unsigned)((C + 127) / 128), 128, 0, st>>>(da);
+        c.launches++;
+        c.stage_end(tk_d, 96 * C);
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(&tot, &c.scalars->ftot[nxt], sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        cur = nxt;
+    }
+    c.stats.levels = levels;
+    return STEM_OK;
+}
+
+}  // namespace sr

@@ -154,6 +154,17 @@ def test_loopback_lloyd_split(sr):
     assert_plans_equal(got, ref)
 
 
+def test_loopback_kmeans_split(sr):
+    """the k-means split (split = 3, R29) decides on each cluster's own rows: independent of the rank count"""
+    rng = np.random.default_rng(31)
+    kid = rng.integers(0, 9, 30_000).astype(np.uint32)
+    t = (rng.integers(0, 80, 30_000) * 53 + 2000 + kid * 9000).astype(np.uint32)
+    ref = O.plan(kid, t, 9, eps=0.02, z=Z95, seed=2, split=3, kmeans_k=4)
+    for world in (2, 3):
+        got = _dist_plan(sr, kid, t, 9, world, eps=0.02, z=Z95, seed=2, split=3, kmeans_k=4)
+        assert_plans_equal(got, ref)
+
+
 def test_loopback_kmpp_split(sr):
     """the k-means++ split variant (opts.split = 2, R27) draws its seeds from the
     cluster's values only, so the plan is independent of the rank count"""

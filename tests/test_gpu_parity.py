@@ -439,9 +439,48 @@ def test_split_option_validation(ctx, sr):
     kid = np.zeros(100, np.uint32)
     t = np.arange(100, dtype=np.uint32)
     with pytest.raises(sr.StemError):
-        ctx.plan(kid, t, 1, split=3)
+        ctx.plan(kid, t, 1, split=4)
     with pytest.raises(sr.StemError):
         ctx.plan(kid, t, 1, split=-1)
+    for k in (0, 1, 9):
+        with pytest.raises(sr.StemError):
+            ctx.plan(kid, t, 1, split=3, kmeans_k=k)
+
+
+# ------------------------------------------------------------------ split variant: exact k-means, k > 2 (R29)
+def _few_values(rng, n, K, vals=150):
+    """mixtures whose kernels have at most `vals` distinct times (the oracle's
+    exact DP is O(k d^2) in the distinct values d)"""
+    kid = rng.integers(0, K, n).astype(np.uint32)
+    base = rng.integers(2000, 200_000, (K, 3))
+    peak = rng.integers(0, 3, n)
+    q = rng.integers(0, vals // 3, n)
+    t = base[kid, peak] + q * (base[kid, 0] // 400 + 1)
+    return kid, t.astype(np.uint32)
+
+
+@pytest.mark.parametrize("k", [2, 3, 4, 8])
+@pytest.mark.parametrize("case", ["mixture", "ties", "big"])
+def test_kmeans_split_variant(ctx, k, case):
+    rng = np.random.default_rng(k * 7 + len(case))
+    if case == "mixture":
+        kid, t = _few_values(rng, 40_000, 12)
+        K = 12
+    elif case == "ties":   # evenly spaced values: many optimal partitions, the tie rule decides
+        kid = rng.integers(0, 3, 9000).astype(np.uint32)
+        t = (rng.integers(0, 12, 9000) * 100 + 1000 + kid * 5000).astype(np.uint32)
+        K = 3
+    else:                  # one kernel, 300k rows over ~300 values (many D&C rounds, big frontier clusters)
+        kid = np.zeros(300_000, np.uint32)
+        t = (np.round(rng.lognormal(5, 0.4, 300_000)) * 3).astype(np.uint32)
+        K = 1
+    for eps in (0.01, 0.05):
+        got, ref = _both(ctx, kid, t, K, eps=eps, seed=9, split=3, kmeans_k=k)
+        assert_plans_equal(got, ref)
+    if k == 2:   # k = 2 is the default exact 2-means (R5)
+        a = ctx.plan(_dev(kid), _dev(t), K, z=Z95, seed=9, split=3, kmeans_k=2)
+        b = ctx.plan(_dev(kid), _dev(t), K, z=Z95, seed=9)
+        assert a["clusters"].tobytes() == b["clusters"].tobytes()
 
 
 @pytest.mark.parametrize("split", [0, 1, 2])
