@@ -49,7 +49,8 @@ def parse():
     ap.add_argument("--ref-sample-rows", type=int, default=8_000_000)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--split", type=int, default=0, choices=[0, 1, 2], help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26), 2 k-means++ seeded Lloyd (R27)")
+    ap.add_argument("--split", type=int, default=0, choices=[0, 1, 2, 3], help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26), 2 k-means++ seeded Lloyd (R27), 3 exact k-means with --kmeans-k groups (R29)")
+    ap.add_argument("--kmeans-k", type=int, default=3, help="groups per ROOT split with --split 3 (2..8)")
     ap.add_argument("--metric-bounds", action="store_true", help="also true totals and bounds of the metric columns (R28)")
     ap.add_argument("--dry-launch", action="store_true", help="print the torchrun command --gpus N would run, and exit")
     return ap.parse_args()
@@ -152,7 +153,12 @@ def dist_env():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
 
-SPLIT_NAMES = ["exact optimal 2-means (R5)", "Lloyd k-means, k = 2 (R26)", "k-means++ seeded Lloyd, k = 2 (R27)"]
+SPLIT_NAMES = ["exact optimal 2-means (R5)", "Lloyd k-means, k = 2 (R26)", "k-means++ seeded Lloyd, k = 2 (R27)",
+               "exact optimal k-means, k = {k} (R29)"]
+
+
+def split_name(a):
+    return SPLIT_NAMES[a.split].format(k=a.kmeans_k)
 
 
 def run_reference(a):
@@ -174,7 +180,7 @@ def run_reference(a):
     for i in range(a.warmup + a.steps):
         t0 = time.perf_counter()
         oracle.plan(kid, t, sp.n_kernels, eps=eps, z=z, seed=i, metrics=met, split=a.split,
-                    metric_bounds=int(a.metric_bounds))
+                    metric_bounds=int(a.metric_bounds), kmeans_k=a.kmeans_k)
         dt = time.perf_counter() - t0
         if i >= a.warmup:
             times.append(dt)
@@ -186,7 +192,7 @@ def run_reference(a):
         "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded)",
         "impl": "reference",
         "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n, "kernels": sp.n_kernels,
-                   "eps": eps, "conf": a.conf, "split": SPLIT_NAMES[a.split], "sample_rows": m},
+                   "eps": eps, "conf": a.conf, "split": split_name(a), "sample_rows": m},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
                          "sample": f"first {m} rows of {a.config} (oracle single-threaded C, -O2)"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -239,7 +245,7 @@ def run_ours(a):
         # (rows/s up to "the plan on host"); rank 0 gets the plan
         hp = ctx.plan_host_raw(kid, tt, sp.n_kernels, eps=eps, conf=a.conf, metrics=met, comm=comm,
                                global_row_base=row0, seed=12345, stream=stream.cuda_stream, split=a.split,
-                               metric_bounds=a.metric_bounds)
+                               metric_bounds=a.metric_bounds, kmeans_k=a.kmeans_k)
         nb = hp.nbytes()
         hp.close()
         return nb
@@ -311,7 +317,7 @@ def run_ours(a):
         "dtype": "u32 keys, exact int64/int128 moments, f64", "data": "synthetic (tracegen, seeded, on device)",
         "config": {"workload": WORKLOADS.get(a.config, a.config), "rows": sp.n,
                    "kernels": sp.n_kernels, "eps": eps, "conf": a.conf, "metrics": nm,
-                   "split": SPLIT_NAMES[a.split],
+                   "split": split_name(a),
                    "parallelism": "single GPU" if world == 1 else
                    f"{world} GPUs: row shards, NCCL all-to-all by kernel id, exact allreduce",
                    "l2": "inputs 8 B/row x rows >> 126 MB L2 (no flush needed)" if n_local >= 50_000_000
@@ -347,9 +353,10 @@ def run_ours(a):
             if comm is not None:
                 return ctx.plan_dist(comm, hk, ht, sp.n_kernels, row0, eps=eps, conf=a.conf, metrics=hm,
                                      seed=12345, stream=stream.cuda_stream, split=a.split,
-                                     metric_bounds=a.metric_bounds)
+                                     metric_bounds=a.metric_bounds, kmeans_k=a.kmeans_k)
             return ctx.plan(hk, ht, sp.n_kernels, eps=eps, conf=a.conf, metrics=hm, seed=12345,
-                            stream=stream.cuda_stream, split=a.split, metric_bounds=a.metric_bounds)
+                            stream=stream.cuda_stream, split=a.split, metric_bounds=a.metric_bounds,
+                            kmeans_k=a.kmeans_k)
         p = e2e_step()
         torch.cuda.synchronize()
         if world > 1:
@@ -378,7 +385,7 @@ def run_ours(a):
         m_np = met[:, :m].cpu().numpy() if nm else None
         t0 = time.perf_counter()
         oracle.plan(k_np, t_np, sp.n_kernels, eps=eps, z=dplan["z"], seed=12345, metrics=m_np, split=a.split,
-                    metric_bounds=int(a.metric_bounds))
+                    metric_bounds=int(a.metric_bounds), kmeans_k=a.kmeans_k)
         cs = time.perf_counter() - t0
         line["cpu_baseline"] = {"value": m / cs, "unit": UNIT, "cores": 1, "kind": "oracle",
                                 "sample": f"first {m} rows of {a.config} ({cs:.1f} s, single-threaded C oracle)",

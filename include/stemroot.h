@@ -60,7 +60,8 @@ typedef enum stem_status {
     STEM_E_NOMEM = -3,  /* host or device allocation failed                                       */
     STEM_E_CUDA = -4,   /* a CUDA runtime call or kernel failed (no device, bad pointer, ...)     */
     STEM_E_NCCL = -5,   /* reserved for the multi-GPU entry point                                 */
-    STEM_E_LIMIT = -6,  /* total sample count would reach 2^32, or some m_i >= 2^32               */
+    STEM_E_LIMIT = -6,  /* total sample count would reach 2^32, or some m_i >= 2^32; split = 3:
+                           more than 256 exactly tied candidates in one k-means DP cell          */
     STEM_E_STATE = -7   /* stem_ctx_device_plan called before any successful plan on that ctx     */
 } stem_status;
 

@@ -76,7 +76,7 @@ void Ctx::release() {
     dfree(big_ent, cap_big_ent); dfree(big_part, cap_big_part); dfree(big_thr, cap_big_thr);
     dfree(peer_dst, cap_peer_dst);
     dfree(km_dpos, cap_km_dpos); dfree(km_arg, cap_km_arg); dfree(km_ngrp, cap_km_ngrp);
-    dfree(km_dP, cap_km_dP); dfree(km_F, cap_km_F);
+    dfree(km_dP, cap_km_dP); dfree(km_F, cap_km_F); dfree(km_meta, cap_km_meta); dfree(km_sub, cap_km_sub);
     dfree(part_cnt, cap_part_cnt); dfree(dist_cnt, cap_dist_cnt);
     for (int i = 0; i < 3; i++) { dfree(xfer_u32[i], cap_xfer_u32[i]); dfree(recv_u32[i], cap_recv_u32[i]); }
     dfree(xfer_f64, cap_xfer_f64); dfree(xfer_f64b, cap_xfer_f64b); dfree(red_part2, cap_red2);

@@ -49,6 +49,7 @@ struct DevScalars {
     unsigned long long local_rows;        // rows scanned below the frontier (local subtrees)
     unsigned long long split_chunks, split_scanned;   // big-cluster chunks bounded / scanned row by row
     uint32_t local_depth, amb_count;      // deepest ROOT level of a local subtree; ambiguous samples
+    uint32_t km_nsub[2];                  // split = 3: subproblems of the current / next D&C round
 };
 
 constexpr int kMaxCand = 64;     // packed sort: most candidate rows per sample (one u64 mask)
@@ -214,6 +215,7 @@ struct Ctx {
     size_t cap_km_dpos = 0, cap_km_arg = 0, cap_km_ngrp = 0;
     uint64_t *km_dP = nullptr; size_t cap_km_dP = 0;
     double *km_F = nullptr; size_t cap_km_F = 0;
+    void *km_meta = nullptr, *km_sub = nullptr; size_t cap_km_meta = 0, cap_km_sub = 0;
     void *peer_dst = nullptr; size_t cap_peer_dst = 0;   // fused exchange: the owners' windows (PeerDst)
     uint64_t row_bases[65] = {0};
     uint64_t n_local_rows = 0;

@@ -134,109 +134,207 @@ __device__ __forceinline__ double km_score(const KmArgs &g, const KmCluster &c, 
     return __ddiv_rn(__dmul_rn(s, s), rn64(km_pos(g, c, b) - km_pos(g, c, a)));
 }
 
-// best a in [a0, a1] for F[j][b] (warp-uniform result); exact among near-ties
-__device__ void km_argmax(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t b, uint32_t a0, uint32_t a1,
-                          double &vbest, uint32_t &abest) {
-    const int lane = threadIdx.x & 31;
-    const size_t L = g.D + 1;
-    const double win = 1.0 - 0x1p-40;
-    bool have = false;
-    vbest = 0.0;
-    abest = a0;
-    for (uint32_t base = a0; base <= a1; base += 32) {
-        const uint32_t a = base + lane;
-        const bool ok = a <= a1;
-        const double v = ok ? __dadd_rn(g.F[(size_t)(j - 1) * L + c.D0 + a], km_score(g, c, a, b)) : -1.0;
-        double vr = v;
-#pragma unroll
-        for (int o = 16; o; o >>= 1) vr = fmax(vr, __shfl_xor_sync(0xffffffffu, vr, o));
-        if (have && vr < __dmul_rn(vbest, win)) continue;        // nothing here comes close
-        const double top = have ? fmax(vr, vbest) : vr;
-        const double thr = __dmul_rn(top, win);
-        const uint32_t cm = __ballot_sync(0xffffffffu, ok && v >= thr);
-        const bool prev_in = have && vbest >= thr;
-        if (__popc(cm) == 1 && !prev_in) {
-            const int src = __ffs(cm) - 1;
-            vbest = __shfl_sync(0xffffffffu, v, src);
-            abest = base + src;
-            have = true;
-            continue;
+// ---------------------------------------------------------------- the DP, level-synchronous divide and conquer
+// Layer j of every active cluster at once: a subproblem (cluster, b range,
+// a range) takes b = mid of its range, finds the best a for it and hands the
+// two halves (with the narrowed a ranges) to the next round.  One round per
+// recursion depth for all clusters together (about log2 of the largest d);
+// long a ranges get a block, short ones a warp.
+struct KmSub {
+    uint32_t c, blo, bhi, alo, ahi, pad;
+};
+
+struct KmMeta {          // per frontier cluster
+    uint64_t D0, lo;
+    uint32_t d, K;
+};
+
+__device__ __forceinline__ double km_value(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t a, uint32_t b) {
+    return __dadd_rn(g.F[(size_t)(j - 1) * (g.D + 1) + c.D0 + a], km_score(g, c, a, b));
+}
+
+// exact winner among the candidates a in list[0..m) (ascending), any thread
+__device__ __noinline__ uint32_t km_exact_best(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t b,
+                                               const uint32_t *list, uint32_t m) {
+    KFrac bf, cf;
+    uint32_t best = list[0];
+    km_exact(g, c, j, best, b, bf);
+    for (uint32_t i = 1; i < m; i++) {
+        km_exact(g, c, j, list[i], b, cf);
+        if (kfrac_cmp(cf, bf) > 0) {
+            bf = cf;
+            best = list[i];
         }
-        // near tie: exact comparison, candidates in ascending a (ties keep the smaller)
-        KFrac bf, cf;
-        bool bset = false;
-        if (prev_in) {
-            km_exact(g, c, j, abest, b, bf);
-            bset = true;
-        }
-        uint32_t m = cm;
-        while (m) {
-            const int src = __ffs(m) - 1;
-            m &= m - 1;
-            km_exact(g, c, j, base + src, b, cf);
-            if (!bset || kfrac_cmp(cf, bf) > 0) {
-                bf = cf;
-                bset = true;
-                abest = base + src;
-                vbest = __shfl_sync(0xffffffffu, v, src);
-            }
-        }
-        have = true;
+    }
+    return best;
+}
+
+struct KmStep {
+    KmArgs g;
+    const KmMeta *meta;
+    const KmSub *cur;
+    const uint32_t *ncur;
+    KmSub *nxt;
+    uint32_t *nnxt;
+    uint32_t j;
+};
+
+constexpr uint32_t kKmLong = 512;   // a ranges longer than this get a block
+constexpr int kKmNear = 256;        // near-tie candidates resolved exactly per subproblem
+
+__device__ __forceinline__ void km_emit(const KmStep &s, const KmSub &x, uint32_t mid, uint32_t a) {
+    KmSub ch[2];
+    int nc = 0;
+    if (mid > x.blo) ch[nc++] = KmSub{x.c, x.blo, mid - 1, x.alo, a, 0};
+    if (mid < x.bhi) ch[nc++] = KmSub{x.c, mid + 1, x.bhi, a, x.ahi, 0};
+    if (nc) {
+        const uint32_t o = atomicAdd(s.nnxt, (uint32_t)nc);
+        for (int i = 0; i < nc; i++) s.nxt[o + i] = ch[i];
     }
 }
 
-// one warp per cluster: the DP layers by divide and conquer, then the cuts
-__global__ void __launch_bounds__(128) kmeans_cut_kernel(KmArgs g) {
-    const uint32_t C = (uint32_t)(*g.ctot >> 32);
-    const int lane = threadIdx.x & 31;
-    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    const size_t L = g.D + 1;
-    for (uint64_t ci = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; ci < C; ci += nwarps) {
-        KmCluster c;
-        c.lo = g.f_lo[ci];
-        const uint64_t hi = g.f_hi[ci];
-        c.D0 = lower_bound(g.dpos, g.D + 1, (uint32_t)c.lo);
-        c.d = (uint32_t)(lower_bound(g.dpos, g.D + 1, (uint32_t)hi) - c.D0);
-        const uint32_t K = min(g.k, c.d);
-        if (K < 2) {
-            if (lane == 0) g.ngrp[ci] = 0;
-            continue;
-        }
-        for (uint32_t b = 1 + lane; b <= c.d; b += 32) g.F[1 * L + c.D0 + b] = km_score(g, c, 0, b);
-        __syncwarp();
-        for (uint32_t j = 2; j <= K; j++) {
-            // divide and conquer over b in [j, d], a in [j - 1, b - 1]; explicit stack (warp-uniform)
-            uint32_t st[4 * 40];
-            int sp = 0;
-            st[0] = j; st[1] = c.d; st[2] = j - 1; st[3] = c.d - 1;
-            sp = 1;
-            while (sp) {
-                sp--;
-                const uint32_t blo = st[4 * sp], bhi = st[4 * sp + 1], alo = st[4 * sp + 2], ahi = st[4 * sp + 3];
-                if (blo > bhi) continue;
-                const uint32_t mid = blo + (bhi - blo) / 2;
-                double v;
-                uint32_t a;
-                km_argmax(g, c, j, mid, alo, min(ahi, mid - 1), v, a);
-                if (lane == 0) {
-                    g.F[(size_t)j * L + c.D0 + mid] = v;
-                    g.arg[(size_t)j * L + c.D0 + mid] = a;
+__device__ __forceinline__ KmCluster km_cluster(const KmMeta &m) {
+    KmCluster c;
+    c.D0 = m.D0;
+    c.lo = m.lo;
+    c.d = m.d;
+    return c;
+}
+
+// subproblems with long a ranges: one block each
+__global__ void __launch_bounds__(256) km_step_block_kernel(KmStep s) {
+    __shared__ double s_v[8];
+    __shared__ uint32_t s_list[kKmNear];
+    __shared__ uint32_t s_m;
+    const uint32_t n = *s.ncur;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    for (uint32_t i = blockIdx.x; i < n; i += gridDim.x) {
+        const KmSub x = s.cur[i];
+        const uint32_t mid = x.blo + (x.bhi - x.blo) / 2;
+        const uint32_t a0 = x.alo, a1 = min(x.ahi, mid - 1);
+        if (a1 - a0 + 1 <= kKmLong) continue;   // the warp kernel's
+        const KmCluster c = km_cluster(s.meta[x.c]);
+        double vm = -1.0;
+        for (uint32_t a = a0 + tid; a <= a1; a += 256) vm = fmax(vm, km_value(s.g, c, s.j, a, mid));
+#pragma unroll
+        for (int o = 16; o; o >>= 1) vm = fmax(vm, __shfl_xor_sync(0xffffffffu, vm, o));
+        if (lane == 0) s_v[w] = vm;
+        if (tid == 0) s_m = 0;
+        __syncthreads();
+        double top = s_v[0];
+        for (int k = 1; k < 8; k++) top = fmax(top, s_v[k]);
+        const double thr = __dmul_rn(top, 1.0 - 0x1p-40);
+        for (uint32_t a = a0 + tid; a <= a1; a += 256)
+            if (km_value(s.g, c, s.j, a, mid) >= thr) {
+                const uint32_t q = atomicAdd(&s_m, 1u);
+                if (q < (uint32_t)kKmNear) s_list[q] = a;
+            }
+        __syncthreads();
+        if (tid == 0) {
+            uint32_t m = min(s_m, (uint32_t)kKmNear), best;
+            for (uint32_t p = 1; p < m; p++)   // ascending a (insertion sort of a few entries)
+                for (uint32_t q = p; q > 0 && s_list[q - 1] > s_list[q]; q--) {
+                    const uint32_t t = s_list[q]; s_list[q] = s_list[q - 1]; s_list[q - 1] = t;
                 }
-                if (mid < bhi) { st[4 * sp] = mid + 1; st[4 * sp + 1] = bhi; st[4 * sp + 2] = a; st[4 * sp + 3] = ahi; sp++; }
-                if (mid > blo) { st[4 * sp] = blo; st[4 * sp + 1] = mid - 1; st[4 * sp + 2] = alo; st[4 * sp + 3] = a; sp++; }
-            }
-            __syncwarp();
+            best = m == 1 ? s_list[0] : km_exact_best(s.g, c, s.j, mid, s_list, m);
+            const size_t L = s.g.D + 1;
+            s.g.F[(size_t)s.j * L + c.D0 + mid] = km_value(s.g, c, s.j, best, mid);
+            s.g.arg[(size_t)s.j * L + c.D0 + mid] = best;
+            km_emit(s, x, mid, best);
+            if (s_m > (uint32_t)kKmNear) atomicOr(s.g.ngrp + x.c, 0x80000000u);   // flagged: too many near ties
         }
-        if (lane == 0) {
-            uint32_t b = c.d;
-            for (uint32_t j = K; j >= 2; j--) {
-                b = g.arg[(size_t)j * L + c.D0 + b];
-                g.cutk[ci * (kKmMax - 1) + (j - 2)] = (uint32_t)km_pos(g, c, b);
+        __syncthreads();
+    }
+}
+
+// subproblems with short a ranges: one warp each
+__global__ void __launch_bounds__(256) km_step_warp_kernel(KmStep s) {
+    __shared__ uint32_t s_list[8][kKmNear];   // 8 KB
+    const uint32_t n = *s.ncur;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t i = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += nwarps) {
+        const KmSub x = s.cur[i];
+        const uint32_t mid = x.blo + (x.bhi - x.blo) / 2;
+        const uint32_t a0 = x.alo, a1 = min(x.ahi, mid - 1);
+        if (a1 - a0 + 1 > kKmLong) continue;    // the block kernel's
+        const KmCluster c = km_cluster(s.meta[x.c]);
+        double vm = -1.0;
+        for (uint32_t a = a0 + lane; a <= a1; a += 32) vm = fmax(vm, km_value(s.g, c, s.j, a, mid));
+#pragma unroll
+        for (int o = 16; o; o >>= 1) vm = fmax(vm, __shfl_xor_sync(0xffffffffu, vm, o));
+        const double thr = __dmul_rn(vm, 1.0 - 0x1p-40);
+        uint32_t m = 0;
+        for (uint32_t base = a0; base <= a1; base += 32) {   // near-tie candidates, ascending
+            const uint32_t a = base + lane;
+            const bool near = a <= a1 && km_value(s.g, c, s.j, a, mid) >= thr;
+            const uint32_t bm = __ballot_sync(0xffffffffu, near);
+            if (near) {
+                const uint32_t q = m + __popc(bm & ((1u << lane) - 1));
+                if (q < (uint32_t)kKmNear) s_list[w][q] = a;
             }
-            g.ngrp[ci] = K;
+            m += __popc(bm);
+        }
+        __syncwarp();
+        if (lane == 0) {
+            const uint32_t mm = min(m, (uint32_t)kKmNear);
+            const uint32_t best = mm == 1 ? s_list[w][0] : km_exact_best(s.g, c, s.j, mid, s_list[w], mm);
+            const size_t L = s.g.D + 1;
+            s.g.F[(size_t)s.j * L + c.D0 + mid] = km_value(s.g, c, s.j, best, mid);
+            s.g.arg[(size_t)s.j * L + c.D0 + mid] = best;
+            km_emit(s, x, mid, best);
+            if (m > (uint32_t)kKmNear) atomicOr(s.g.ngrp + x.c, 0x80000000u);
         }
         __syncwarp();
     }
+}
+
+// per cluster: its distinct-value slice, K = min(k, d), layer 1, and the
+// layer-2 subproblem; one warp per cluster
+__global__ void __launch_bounds__(256) km_prep_kernel(KmArgs g, KmMeta *meta, KmSub *sub, uint32_t *nsub) {
+    const uint32_t C = (uint32_t)(*g.ctot >> 32);
+    const int lane = threadIdx.x & 31;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t ci = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; ci < C; ci += nwarps) {
+        const uint64_t lo = g.f_lo[ci], hi = g.f_hi[ci];
+        KmMeta m;
+        m.lo = lo;
+        m.D0 = lower_bound(g.dpos, g.D + 1, (uint32_t)lo);
+        m.d = (uint32_t)(lower_bound(g.dpos, g.D + 1, (uint32_t)hi) - m.D0);
+        m.K = min(g.k, m.d);
+        const KmCluster c = km_cluster(m);
+        for (uint32_t b = 1 + lane; b <= m.d; b += 32) g.F[(g.D + 1) + c.D0 + b] = km_score(g, c, 0, b);
+        if (lane == 0) {
+            meta[ci] = m;
+            g.ngrp[ci] = 0;
+            if (m.K >= 2) sub[atomicAdd(nsub, 1u)] = KmSub{(uint32_t)ci, 2, m.d, 1, m.d - 1, 0};
+        }
+    }
+}
+
+// the next layer's root subproblems
+__global__ void km_layer_kernel(const uint64_t *ctot, const KmMeta *meta, uint32_t j, KmSub *sub, uint32_t *nsub) {
+    const uint64_t ci = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (ci >= (*ctot >> 32)) return;
+    const KmMeta m = meta[ci];
+    if (m.K >= j) sub[atomicAdd(nsub, 1u)] = KmSub{(uint32_t)ci, j, m.d, j - 1, m.d - 1, 0};
+}
+
+// backtrack the cuts
+__global__ void km_finish_kernel(KmArgs g, const KmMeta *meta) {
+    const uint64_t ci = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (ci >= (*g.ctot >> 32)) return;
+    const KmMeta m = meta[ci];
+    if (g.ngrp[ci] & 0x80000000u) return;   // too many near ties for the exact list: reported as an error
+    if (m.K < 2) { g.ngrp[ci] = 0; return; }
+    const KmCluster c = km_cluster(m);
+    const size_t L = g.D + 1;
+    uint32_t b = m.d;
+    for (uint32_t j = m.K; j >= 2; j--) {
+        b = g.arg[(size_t)j * L + c.D0 + b];
+        g.cutk[ci * (kKmMax - 1) + (j - 2)] = (uint32_t)km_pos(g, c, b);
+    }
+    g.ngrp[ci] = m.K;
 }
 
 // ---------------------------------------------------------------- decision and children (Eq. 7 vs Eq. 8)
@@ -256,6 +354,7 @@ struct KdArgs {
     uint64_t *total;
     double eps, z, k2;
     int clamp;
+    uint32_t *err;
 };
 
 __device__ __forceinline__ double km_eq6(double g, double mu, double V, int clamp) {
@@ -269,6 +368,10 @@ __global__ void __launch_bounds__(128) kmeans_decide_kernel(KdArgs a) {
     const uint64_t c = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= (*a.ctot >> 32)) return;
     const uint32_t G = a.ngrp[c];
+    if (G & 0x80000000u) {   // more than kKmNear exact-tie candidates in one DP cell
+        atomicOr(a.err, 8u);
+        return;
+    }
     if (G < 2) return;
     const uint64_t lo = a.f_lo[c], hi = a.f_hi[c], n = hi - lo, S = a.f_S[c];
     const u128 Q = a.f_Q[c];
@@ -433,15 +536,43 @@ int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, dou
         const int tk_s = c.stage_begin("root_split");
         KmArgs ka{c.f_lo[cur], c.f_hi[cur], &c.scalars->ftot[cur], c.km_dpos, c.km_dP, D, c.km_F, c.km_arg, kk,
                   c.cut, c.km_ngrp};
-        kmeans_cut_kernel<<<(unsigned)min((C + 3) / 4, (uint64_t)c.sms * 16), 128, 0, st>>>(ka);
+        // subproblem lists: at most one per distinct value in flight per round
+        const uint64_t rows_l = tot & 0xFFFFFFFFull;
+        CKS(c.ensure(c.km_meta, c.cap_km_meta, sizeof(KmMeta) * C));
+        CKS(c.ensure(c.km_sub, c.cap_km_sub, sizeof(KmSub) * 2 * (rows_l + C + 2)));
+        KmMeta *meta = (KmMeta *)c.km_meta;
+        KmSub *sub[2] = {(KmSub *)c.km_sub, (KmSub *)c.km_sub + (rows_l + C + 2)};
+        uint32_t *nsub = c.scalars->km_nsub;
+        CK(cudaMemsetAsync(nsub, 0, 2 * sizeof(uint32_t), st));
+        km_prep_kernel<<<(unsigned)min((C + 7) / 8, (uint64_t)c.sms * 16), 256, 0, st>>>(ka, meta, sub[0], nsub);
         c.launches++;
-        c.stage_end(tk_s, 12 * (tot & 0xFFFFFFFFull));
+        const int depth = 2 + (int)(64 - __builtin_clzll(rows_l + 1));   // rounds: > log2 of the largest d
+        for (uint32_t j = 2; j <= kk; j++) {
+            if (j > 2) {
+                CK(cudaMemsetAsync(nsub, 0, sizeof(uint32_t), st));
+                km_layer_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(&c.scalars->ftot[cur], meta, j, sub[0],
+                                                                            nsub);
+                c.launches++;
+            }
+            int sc = 0;
+            for (int r = 0; r < depth; r++) {   // empty rounds exit at once (counts read on the device)
+                CK(cudaMemsetAsync(nsub + (sc ^ 1), 0, sizeof(uint32_t), st));
+                KmStep ks{ka, meta, sub[sc], nsub + sc, sub[sc ^ 1], nsub + (sc ^ 1), j};
+                km_step_block_kernel<<<(unsigned)c.sms * 2, 256, 0, st>>>(ks);
+                km_step_warp_kernel<<<(unsigned)c.sms * 16, 256, 0, st>>>(ks);
+                c.launches += 2;
+                sc ^= 1;
+            }
+        }
+        km_finish_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(ka, meta);
+        c.launches++;
+        c.stage_end(tk_s, 12 * rows_l);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");
         CK(cudaMemsetAsync(&c.scalars->ftot[nxt], 0, sizeof(uint64_t), st));
         KdArgs da{c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], &c.scalars->ftot[cur], c.cut, c.km_ngrp, c.PS1,
                   c.PS2, c.t_sorted, c.flags, c.f_lo[nxt], c.f_hi[nxt], c.f_S[nxt], c.f_Q[nxt],
-                  &c.scalars->ftot[nxt], eps, z, k2, clamp};
+                  &c.scalars->ftot[nxt], eps, z, k2, clamp, &c.scalars->err};
         kmeans_decide_kernel<<<(unsigned)((C + 127) / 128), 128, 0, st>>>(da);
         c.launches++;
         c.stage_end(tk_d, 96 * C);
@@ -451,6 +582,10 @@ int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, dou
         cur = nxt;
     }
     c.stats.levels = levels;
+    uint32_t err = 0;
+    CK(cudaMemcpyAsync(&err, &c.scalars->err, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (err & 8u) return STEM_E_LIMIT;
     return STEM_OK;
 }
 
