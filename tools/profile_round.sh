@@ -22,4 +22,10 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:ones
 timeout 900 ncu --set full --clock-control none --import-source on \
     -k regex:"prepass|pm_sums|pm_apply|big_split|small_split|decide|flag_c|sample_kernel|estimate|onesweep" -c 24 \
     -o gpurun_out/${R}_prof_other_c5 python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > /dev/null 2>&1
-ls -la gpurun_out
+# summaries here; only the small reports travel back (gpurun_out must stay under 64 MiB)
+python tools/ncu_summary.py gpurun_out/${R}_prof_sort_mid_c5.ncu-rep --traffic-json gpurun_out/ncu_traffic.json --config C5 --stage sort_pass_mid > gpurun_out/${R}_ncu_sort_mid_c5.txt 2>&1
+python tools/sass_hot.py gpurun_out/${R}_prof_sort_mid_c5.ncu-rep 25 >> gpurun_out/${R}_ncu_sort_mid_c5.txt 2>&1
+python tools/ncu_summary.py gpurun_out/${R}_prof_other_c5.ncu-rep > gpurun_out/${R}_ncu_other_c5.txt 2>&1
+python tools/sass_hot.py gpurun_out/${R}_prof_other_c5.ncu-rep 15 big_split >> gpurun_out/${R}_ncu_other_c5.txt 2>&1
+rm -f gpurun_out/${R}_prof_other_c5.ncu-rep
+du -sh gpurun_out; ls -la gpurun_out
