@@ -12,6 +12,8 @@
 // kernel's leaf lower bounds.  Two passes (sums, then squared deviations from
 // the leaf mean) accumulate per-leaf fp64 sums with warp-aggregated atomics;
 // the column totals use deterministic per-warp / per-block partials.
+#include <cstdlib>
+
 #include "internal.h"
 
 namespace sr {
@@ -232,6 +234,173 @@ static int metric_bounds_table_run(Ctx &c, uint64_t L, const uint32_t *kid, cons
     return STEM_OK;
 }
 
+// ---------------------------------------------------------------- sorted-order path (single GPU)
+// When every sorted position's trace row is known (row payload, or a packed
+// key whose low bits hold the whole row), the rows are walked in SORTED order:
+// a leaf is then a contiguous run, so sums need no per-row atomics -- each
+// warp walks a segment of kMbSeg positions, reduces runs of equal leaf with a
+// segmented warp scan and carries the open run across its iterations; only a
+// run's end (a leaf boundary, or the segment's end) is added atomically.  The
+// metric values are gathered by row (random 8-byte reads).
+constexpr int kMbSeg = 2048;   // sorted positions per warp
+
+struct MbSorted {
+    const uint32_t *row;        // row_sorted: the trace row of each sorted position
+    const uint32_t *flags;      // leaf-start bitmap (bit p: a leaf starts at sorted position p)
+    const uint32_t *leaf_lo;    // [L] leaf starts
+    uint64_t L, n;
+    const double *met;          // [nm][n] trace order
+    uint32_t nm;
+    const double *mean;         // pass 2: [L][nm] leaf means, NULL in pass 1
+    double *acc;                // [L][nm]
+    double *part;               // pass 1: [warps][nm] column partials (deterministic)
+};
+
+template <bool DEV>
+__global__ void __launch_bounds__(kMbThreads) mb_sorted_kernel(MbSorted a) {
+    __shared__ double s_carry[kMbWarps][64];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint64_t s0 = gw * kMbSeg;
+    if (s0 >= a.n) return;
+    const uint64_t s1 = min(a.n, s0 + kMbSeg);
+    // leaf of the segment's first position (the last leaf start <= s0)
+    uint64_t base_leaf = upper_bound(a.leaf_lo, a.L, (uint32_t)s0) - 1;
+    const uint64_t nwords = (a.n + 31) / 32;
+    uint64_t carry_leaf = ~0ull;
+    for (uint32_t c = lane; c < a.nm; c += 32) s_carry[w][c] = 0.0;
+    double colsum = 0.0;   // pass 1: lane c's column total over the segment (c < 32), in position order
+    __syncwarp();
+    for (uint64_t p0 = s0; p0 < s1; p0 += 32) {
+        const uint64_t pos = p0 + lane;
+        const bool in = pos < s1;
+        // leaf starts at positions p0 .. p0 + 63 (bit i = position p0 + i)
+        const uint64_t w0 = p0 >> 5;
+        const uint64_t bits = ((uint64_t)(w0 + 1 < nwords ? a.flags[w0 + 1] : 0u) << 32 | a.flags[w0]) >> (p0 & 31);
+        const uint64_t upto = bits & ((2ull << lane) - 1);
+        const uint64_t leaf = base_leaf + __popcll(upto & ~1ull);   // + starts in (p0, pos]
+        const uint32_t head = __ballot_sync(0xffffffffu, in && (lane == 0 || ((bits >> lane) & 1ull)));
+        const uint32_t inm = __ballot_sync(0xffffffffu, in);
+        const int last_in = 31 - __clz(inm);
+        const int seg = 31 - __clz(head & (0xFFFFFFFFu >> (31 - lane)));   // first lane of my run
+        const bool tail = in && (lane == last_in || ((head >> (lane + 1)) & 1u));
+        const uint64_t leaf_first = base_leaf;
+        const bool last_iter = p0 + 32 >= s1;
+        const uint32_t r = in ? a.row[pos] : 0u;
+        constexpr int kG = 4;   // metric columns whose gathers are in flight together
+        for (uint32_t c0 = 0; c0 < a.nm; c0 += kG) {
+          double xs[kG];
+#pragma unroll
+          for (int u = 0; u < kG; u++)
+              xs[u] = (in && c0 + u < a.nm) ? __ldg(a.met + (uint64_t)(c0 + u) * a.n + r) : 0.0;
+#pragma unroll 1
+          for (int u = 0; u < kG && c0 + u < a.nm; u++) {
+            const uint32_t c = c0 + u;
+            double x = u == 0 ? xs[0] : u == 1 ? xs[1] : u == 2 ? xs[2] : xs[3];
+            if (!DEV && c < 32) {   // column total (pass 1), deterministic butterfly then in order
+                double tsum = x;
+#pragma unroll
+                for (int o = 16; o; o >>= 1) tsum = __dadd_rn(tsum, __shfl_xor_sync(0xffffffffu, tsum, o));
+                if (lane == (int)c) colsum = __dadd_rn(colsum, tsum);
+            }
+            if (DEV && in) {
+                const double d = __dsub_rn(x, a.mean[leaf * a.nm + c]);
+                x = __dmul_rn(d, d);
+            }
+            // segmented inclusive scan over runs of equal leaf
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const double u = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane - o >= seg) x = __dadd_rn(x, u);
+            }
+            const double carry = s_carry[w][c];
+            __syncwarp();
+            // the open run of the previous iteration ended at its last position
+            if (lane == 0 && carry_leaf != ~0ull && carry_leaf != leaf_first)
+                atomicAdd(a.acc + carry_leaf * a.nm + c, carry);
+            if (tail) {
+                double v = x;
+                if (seg == 0 && leaf == carry_leaf) v = __dadd_rn(v, carry);   // the open run continues
+                if (lane == last_in && !last_iter) s_carry[w][c] = v;          // still open
+                else atomicAdd(a.acc + leaf * a.nm + c, v);
+            }
+            __syncwarp();
+          }
+        }
+        carry_leaf = __shfl_sync(0xffffffffu, leaf, last_in);
+        base_leaf += __popcll((bits >> 1) & 0xFFFFFFFFull);   // leaf of position p0 + 32
+    }
+    if (!DEV) {   // column partials of this warp: lane c holds column c (c < 32), others by a second sweep
+        for (uint32_t c = lane; c < a.nm && c < 32; c += 32) a.part[gw * a.nm + c] = colsum;
+    }
+}
+
+// columns 32..63 of pass 1's totals (rare: more than 32 metrics), per warp in position order
+__global__ void __launch_bounds__(kMbThreads) mb_sorted_cols_hi_kernel(MbSorted a) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint64_t s0 = gw * kMbSeg;
+    if (s0 >= a.n) return;
+    const uint64_t s1 = min(a.n, s0 + kMbSeg);
+    for (uint32_t c = 32; c < a.nm; c++) {
+        double colsum = 0.0;
+        for (uint64_t p0 = s0; p0 < s1; p0 += 32) {
+            const uint64_t pos = p0 + lane;
+            double x = pos < s1 ? __ldg(a.met + (uint64_t)c * a.n + a.row[pos]) : 0.0;
+#pragma unroll
+            for (int o = 16; o; o >>= 1) x = __dadd_rn(x, __shfl_xor_sync(0xffffffffu, x, o));
+            colsum = __dadd_rn(colsum, x);
+        }
+        if (lane == 0) a.part[gw * a.nm + c] = colsum;
+    }
+}
+
+static int metric_bounds_sorted(Ctx &c, uint64_t L, uint64_t n, const double *met, uint32_t nm, double z) {
+    cudaStream_t st = c.stream;
+    const uint64_t cells = L * nm;
+    const uint64_t warps = (n + kMbSeg - 1) / kMbSeg;
+    const unsigned grid = (unsigned)((warps + kMbWarps - 1) / kMbWarps);
+    const uint64_t vblocks = (L + kMbThreads - 1) / kMbThreads;
+    CKS(c.ensure(c.mb_acc, c.cap_mb_acc, sizeof(double) * (2 * cells + 1)));
+    CKS(c.ensure(c.mb_part, c.cap_mb_part, sizeof(double) * ((warps + vblocks) * nm + 4 * 64)));
+    double *acc1 = c.mb_acc, *acc2 = c.mb_acc + cells;
+    double *partA = c.mb_part, *partV = partA + warps * nm, *red = partV + vblocks * nm;
+    double *tru = red, *var = red + 64, *bnd = red + 128;
+    CK(cudaMemsetAsync(c.mb_acc, 0, sizeof(double) * 2 * cells, st));
+    MbSorted a{c.row_sorted, c.flags, c.leaf_lo, L, n, met, nm, nullptr, acc1, partA};
+    if (n) {
+        mb_sorted_kernel<false><<<grid, kMbThreads, 0, st>>>(a);
+        if (nm > 32) mb_sorted_cols_hi_kernel<<<grid, kMbThreads, 0, st>>>(a);
+        mb_cols_kernel<<<1, 64, 0, st>>>(partA, warps, nm, tru);
+        c.launches += nm > 32 ? 3 : 2;
+    } else {
+        CK(cudaMemsetAsync(tru, 0, sizeof(double) * nm, st));
+    }
+    if (cells) {
+        mb_mean_kernel<<<(unsigned)((cells + 255) / 256), 256, 0, st>>>(acc1, c.mb_n, L, nm);
+        c.launches++;
+    }
+    if (n) {
+        MbSorted b{c.row_sorted, c.flags, c.leaf_lo, L, n, met, nm, acc1, acc2, nullptr};
+        mb_sorted_kernel<true><<<grid, kMbThreads, 0, st>>>(b);
+        c.launches++;
+    }
+    if (L) {
+        mb_var_kernel<<<(unsigned)vblocks, kMbThreads, 0, st>>>(acc2, c.mb_n, c.mb_m, L, nm, partV);
+        mb_cols_kernel<<<1, 64, 0, st>>>(partV, vblocks, nm, var);
+        c.launches += 2;
+    } else {
+        CK(cudaMemsetAsync(var, 0, sizeof(double) * nm, st));
+    }
+    mb_final_kernel<<<1, 64, 0, st>>>(tru, var, nm, z, bnd);
+    c.launches++;
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(c.host_true_metric, tru, sizeof(double) * nm, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(c.host_bound_metric, bnd, sizeof(double) * nm, cudaMemcpyDeviceToHost, st));
+    CKS(sync_stream(c));
+    return STEM_OK;
+}
+
 // single GPU: the plan's own leaves are the table
 int metric_bounds_local(Ctx &c, uint64_t L, uint32_t K, uint64_t n_sorted, const uint32_t *kid, const uint32_t *t,
                         const double *met, uint64_t n_trace, uint32_t nm, double z) {
@@ -244,6 +413,9 @@ int metric_bounds_local(Ctx &c, uint64_t L, uint32_t K, uint64_t n_sorted, const
                                                                                 c.mb_n);
     c.launches += 2;
     c.mb_m = c.leaf_m;
+    // every sorted position's row known (payload, or packed low bits = the whole row): sorted order
+    if ((c.pack_h <= 1 && !c.sort_row_in) && !(getenv("STEMROOT_MB_TRACE_ORDER")))
+        return metric_bounds_sorted(c, L, n_sorted, met, nm, z);
     return metric_bounds_table_run(c, L, kid, t, met, n_trace, nm, z, c.host_true_metric, c.host_bound_metric);
 }
 
