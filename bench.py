@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--eps", type=float, default=None)
     ap.add_argument("--conf", type=float, default=0.95)
     ap.add_argument("--cpu-sample-rows", type=int, default=30_000_000)
-    ap.add_argument("--ref-sample-rows", type=int, default=8_000_000)
+    ap.add_argument("--ref-sample-rows", type=int, default=30_000_000)   # the same sample as cpu_baseline
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--split", type=int, default=0, choices=[0, 1, 2, 3], help="ROOT split rule: 0 exact 2-means (default), 1 Lloyd (R26), 2 k-means++ seeded Lloyd (R27), 3 exact k-means with --kmeans-k groups (R29)")
