@@ -539,3 +539,39 @@ print("ok")
     env = dict(os.environ, STEMROOT_LOCAL_ROWS="1024")
     out = subprocess.run([sys.executable, str(script)], env=env, capture_output=True, text=True, timeout=300)
     assert out.returncode == 0 and out.stdout.strip().endswith("ok"), out.stdout[-2000:] + out.stderr[-2000:]
+
+
+def test_metric_bounds_trace_order_path(tmp_path):
+    """metric_bounds has two GPU paths: sorted order (one GPU, every sorted
+    position's row known: the default above) and trace order with per-leaf
+    atomics (multi-GPU and multi-candidate packed keys); STEMROOT_MB_TRACE_ORDER
+    forces the latter on one GPU.  Both match the oracle."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    prog = tmp_path / "mb.py"
+    prog.write_text(
+        "import sys, numpy as np, torch\n"
+        f"sys.path.insert(0, {root!r}); sys.path.insert(0, {os.path.join(root, 'tests')!r})\n"
+        "import paper_conf_micro_chungnkk25_b200 as sr, oracle as O, tracegen as G\n"
+        "from parity_util import Z95, assert_plans_equal\n"
+        "sp = G.spec('C3', n=300_000); kid, t, met = G.generate_np(sp)\n"
+        "ctx = sr.Context(0)\n"
+        "got = ctx.plan(kid, t, sp.n_kernels, metrics=met, eps=0.02, z=Z95, seed=3, metric_bounds=True)\n"
+        "ref = O.plan(kid, t, sp.n_kernels, metrics=met, eps=0.02, z=Z95, seed=3, metric_bounds=1)\n"
+        "assert_plans_equal(got, ref, metrics=True); print('MB_OK')\n")
+    out = subprocess.run([sys.executable, str(prog)], env=dict(os.environ, STEMROOT_MB_TRACE_ORDER="1"),
+                         capture_output=True, text=True, timeout=600)
+    assert "MB_OK" in out.stdout, out.stdout + out.stderr[-3000:]
+
+
+@pytest.mark.parametrize("opts", [dict(scope=1), dict(scope=2), dict(census_cap=True, eps=1e-4),
+                                  dict(clamp_in_split=False)])
+def test_kmeans_option_matrix(ctx, opts):
+    rng = np.random.default_rng(71)
+    kid, t = _few_values(rng, 20_000, 6)
+    kw = dict(opts)
+    kw.setdefault("eps", 0.02)
+    got, ref = _both(ctx, kid, t, 6, seed=5, split=3, kmeans_k=3, **kw)
+    assert_plans_equal(got, ref)
