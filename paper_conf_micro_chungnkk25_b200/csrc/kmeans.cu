@@ -93,8 +93,8 @@ struct KmArgs {
     const uint32_t *dpos;          // [D + 1] rows starting a distinct value (dpos[D] = n)
     const uint64_t *dP;            // [D + 1] exact sum of t before them
     uint64_t D;
-    double *F;                     // [kKmMax + 1][D + 1] fp64 DP values
-    uint32_t *arg;                 // [kKmMax + 1][D + 1] argmax (distinct index relative to the cluster)
+    double *F;                     // [k + 1][D + 1] fp64 DP values (layers 1..k)
+    uint32_t *arg;                 // [k + 1][D + 1] argmax (distinct index relative to the cluster)
     uint32_t k;
     uint32_t *cutk;                // [cluster][kKmMax - 1] cuts relative to lo
     uint32_t *ngrp;                // [cluster] groups (0: leaf)
@@ -499,8 +499,8 @@ int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, dou
     CK(cudaStreamSynchronize(st));
     kmeans_sentinel_kernel<<<1, 32, 0, st>>>(c.PS1, c.t_sorted, n, c.km_dpos + D, c.km_dP + D);   // dpos[D] = n
     c.launches++;
-    CKS(c.ensure(c.km_F, c.cap_km_F, sizeof(double) * (size_t)(kKmMax + 1) * (D + 1)));
-    CKS(c.ensure(c.km_arg, c.cap_km_arg, sizeof(uint32_t) * (size_t)(kKmMax + 1) * (D + 1)));
+    CKS(c.ensure(c.km_F, c.cap_km_F, sizeof(double) * (size_t)(kk + 1) * (D + 1)));
+    CKS(c.ensure(c.km_arg, c.cap_km_arg, sizeof(uint32_t) * (size_t)(kk + 1) * (D + 1)));
     // initial frontier
     uint64_t Cmax = (uint64_t)K + 1;
     for (int b = 0; b < 2; b++) {
