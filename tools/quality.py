@@ -20,9 +20,14 @@ Methods:
               (opts.split = 1, R26: the paper's "k-means")
   kmeans++    the same from k-means++ seeds (opts.split = 2, R27; the tree changes
               with every sampling seed, like a randomly seeded library k-means)
+  kmeans-3/4  ROOT splitting each cluster into 3 / 4 groups by the exact k-means
+              (opts.split = 3, R29: "any number above 2 works well", P:L192)
   random-p    uniform random sampling, each invocation kept with probability p,
               estimate sum(t)/p (the paper's baseline)
-and an eps sweep of stem+root (Fig. 11).
+and an eps sweep of stem+root (Fig. 11).  Configs with metric columns
+(C3) add the metric estimates: per column the relative error of the
+weighted sum against the exact total, and how often it lies inside the
+predicted metric bound (metric_bounds, R28).
 
     python tools/quality.py [--config C2] [--n ROWS] [--seeds 20] [--eps 0.03,0.05,0.1,0.25]
                             [--out profiles/r01_quality_C2.json]
@@ -74,6 +79,25 @@ def plan_quality(ctx, kid, t, n_kernels, t64, total, eps, seeds, **opts):
     return _summary(err, spd, bnd, eps, ns)
 
 
+def metric_quality(ctx, kid, t, sp, eps, seeds, kw):
+    """Per metric column: mean / max relative error of the weighted-sum estimate
+     against the exact total, the mean predicted bound and its coverage."""
+    import torch
+    import tracegen as G
+    _, _, met_np = G.generate_np(sp)
+    met = torch.from_numpy(met_np).cuda()
+    errs, bnds = [], []
+    for s in seeds:
+        p = ctx.plan(kid, t, sp.n_kernels, eps=eps, seed=int(s), metrics=met, metric_bounds=True, **kw)
+        tru = np.asarray(p["true_metric"])
+        errs.append(100.0 * np.abs(np.asarray(p["est_metric"]) - tru) / np.abs(tru))
+        bnds.append(100.0 * np.asarray(p["bound_metric"]))
+    e, b = np.array(errs), np.array(bnds)
+    return {"columns": int(e.shape[1]), "mean_error_pct": e.mean(axis=0).tolist(),
+            "max_error_pct": e.max(axis=0).tolist(), "mean_bound_pct": b.mean(axis=0).tolist(),
+            "coverage_of_bound": (e <= b).mean(axis=0).tolist(), "coverage_all": float((e <= b).mean())}
+
+
 def random_quality(t64, total, prob, seeds):
     """Uniform random sampling baseline: Bernoulli(prob) per invocation,
     Horvitz-Thompson estimate sum(t) / prob."""
@@ -113,6 +137,11 @@ def run(config="C2", n=None, n_seeds=20, eps_list=(0.03, 0.05, 0.1, 0.25), z=0.0
     res["methods"]["per-leaf"] = plan_quality(ctx, kid, t, sp.n_kernels, t64, total, eps, seeds, scope=2, **kw)
     res["methods"]["lloyd"] = plan_quality(ctx, kid, t, sp.n_kernels, t64, total, eps, seeds, split=1, **kw)
     res["methods"]["kmeans++"] = plan_quality(ctx, kid, t, sp.n_kernels, t64, total, eps, seeds, split=2, **kw)
+    for k in (3, 4):
+        res["methods"][f"kmeans-{k}"] = plan_quality(ctx, kid, t, sp.n_kernels, t64, total, eps, seeds, split=3,
+                                                     kmeans_k=k, **kw)
+    if sp.n_metrics:
+        res["metrics"] = metric_quality(ctx, kid, t, sp, eps, seeds, kw)
     for prob in (0.001, 0.1):
         res["methods"][f"random-{prob:g}"] = random_quality(t64, total, prob, seeds)
     for e in eps_list:
@@ -123,6 +152,11 @@ def run(config="C2", n=None, n_seeds=20, eps_list=(0.03, 0.05, 0.1, 0.25), z=0.0
 
 def _print(res):
     print(f"{res['config']}: {res['rows']} rows, {res['kernels']} kernels, eps {res['eps']}, {res['seeds']} seeds")
+    if "metrics" in res:
+        m = res["metrics"]
+        print(f"metrics: {m['columns']} columns, mean error % " + " ".join(f"{x:.3f}" for x in m["mean_error_pct"]) +
+              f"; mean bound % " + " ".join(f"{x:.3f}" for x in m["mean_bound_pct"]) +
+              f"; coverage {m['coverage_all']:.2f}")
     print(f"{'method':<14} {'mean err %':>10} {'max err %':>10} {'hmean speedup':>14} {'bound %':>8} "
           f"{'cov(bound)':>10} {'samples':>9}")
     rows = list(res["methods"].items()) + [(f"eps={k}", v) for k, v in res["eps_sweep"].items()]
