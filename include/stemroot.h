@@ -230,14 +230,28 @@ STEM_API const char *stem_strerror(int status);     /* static string, never NULL
 /* ---- multi-GPU (one process or thread per GPU) ---------------------------
  * The trace is sharded by contiguous row ranges: rank r holds rows
  * [global_row_base_r, global_row_base_r + local_shard->n) (shards in rank
- * order, no gaps).  stem_root_plan_dist exchanges rows so that every rank
- * owns whole kernel groups (contiguous kernel-id ranges of ~N/world rows,
- * stem_owner_ranges), runs steps a1-a5 locally, reduces T and the exact KKT
- * sum as integers across ranks, samples locally, and gathers the plan on rank
- * 0 (*out is set on rank 0 only; other ranks get NULL).  The plan is
- * identical to stem_root_plan on the unsharded trace for every world size
- * (integers bit-exact, fp64 sums within 1e-9 relative).  All ranks must call
- * it collectively with the same eps, conf, opts and n_kernels. */
+ * order, no gaps; a shard may be empty).  stem_root_plan_dist exchanges rows so
+ * that every rank owns whole kernel groups (contiguous kernel-id ranges of
+ * ~N/world rows, stem_owner_ranges) -- by default each row is stored straight
+ * into its owner's receive window (CUDA-IPC peer memory over NVLink/NVSwitch;
+ * STEMROOT_DIST_P2P=0, or peers without access, use grouped ncclSend/Recv) --
+ * runs steps a1-a5 locally, reduces T and the exact KKT sum as integers
+ * across ranks, samples locally, and gathers the plan on rank 0 (*out is set
+ * on rank 0 only; other ranks get NULL and keep their own part, which
+ * stem_ctx_device_plan then describes).  The plan is identical to
+ * stem_root_plan on the unsharded trace for every world size (integers
+ * bit-exact, fp64 sums within 1e-9 relative).  All ranks must call it
+ * collectively with the same eps, conf, opts and n_kernels.
+ * Failure semantics: rank-local errors (a bad shard, an allocation, a CUDA
+ * error) are agreed across ranks before the next collective, so every rank
+ * returns the same status; a peer that fails or disappears makes the others
+ * return STEM_E_NCCL after STEMROOT_COMM_TIMEOUT_S seconds (default 600: the
+ * NCCL communicator polls ncclCommGetAsyncError and aborts itself), after which
+ * the communicator is unusable.
+ * Entry point shape (a recorded choice): the communicator and
+ * the workspace are objects created once and reused across plans; the
+ * one-shot form (unique id, rank, world per call) is stem_comm_init_nccl +
+ * stem_ctx_create + stem_root_plan_dist + the destroys. */
 typedef struct stem_comm stem_comm;
 
 /* 128 opaque bytes created by one rank and shared with all (e.g. broadcast
