@@ -75,6 +75,8 @@ void Ctx::release() {
     dfree(out_cluster, cap_out_cluster); dfree(out_weight, cap_out_weight);
     dfree(big_ent, cap_big_ent); dfree(big_part, cap_big_part); dfree(big_thr, cap_big_thr);
     dfree(peer_dst, cap_peer_dst);
+    dfree(vr_P, cap_vr_P); dfree(vr_work, cap_vr_work); dfree(gi_buf, cap_gi_buf);
+    dfree(gi_tab, cap_gi_tab); dfree(gi_rec, cap_gi_rec); dfree(gi_all, cap_gi_all); dfree(gi_val, cap_gi_val);
     dfree(km_dpos, cap_km_dpos); dfree(km_arg, cap_km_arg); dfree(km_ngrp, cap_km_ngrp);
     dfree(km_dP, cap_km_dP); dfree(km_F, cap_km_F); dfree(km_meta, cap_km_meta); dfree(km_sub, cap_km_sub);
     dfree(part_cnt, cap_part_cnt); dfree(dist_cnt, cap_dist_cnt);

@@ -429,10 +429,18 @@ struct PartArgs {
     const double *inw;              // payload f64 column
     uint32_t *out0, *out1, *out2;
     double *outw;
+    // unit mode (kernels larger than a rank's share): the key is the row's unit,
+    // kunit[kid] + (its leaf among the kernel's gl_n[kid] value-tree leaves, by t)
+    const uint32_t *kunit, *gl_first, *gl_n, *gl_t;
 };
 
 __device__ __forceinline__ int part_dest(const PartArgs &a, uint64_t i) {
-    const uint64_t k = a.key ? (uint64_t)a.key[i] + a.key_add : a.key_add + i;
+    uint64_t k = a.key ? (uint64_t)a.key[i] + a.key_add : a.key_add + i;
+    if (a.kunit) {
+        const uint32_t kid = (uint32_t)k, m = a.gl_n[kid];
+        k = a.kunit[kid];
+        if (m) k += upper_bound(a.gl_t + a.gl_first[kid], (uint64_t)m, a.in1[i]) - 1;
+    }
     int d = 0;
     for (int r = 1; r < a.world; r++) d += a.bounds[r] <= k;
     return d;
@@ -694,6 +702,270 @@ __global__ void add_kernel_u32(uint32_t *x, uint64_t n, uint32_t v) {
     if (i < n) x[i] += v;
 }
 
+// ---------------------------------------------------------------- kernels larger than a rank's share
+// A kernel with more than factor * N / P rows (STEMROOT_DIST_GIANT, default
+// 1.25; 0 disables) would overload the rank owning it.  Its ROOT tree is built
+// instead from its value histogram (root.cu root_values: the decisions depend
+// only on the multiset of times, so the tree is the row tree): every rank
+// histograms its rows of the kernel, the histograms are merged on every rank,
+// every rank builds the same value tree, and the kernel's LEAVES become units of
+// ownership next to the whole ordinary kernels.  Units are dealt to ranks in
+// (kernel, value) order, so the gathered plan is still in (kernel, ordinal)
+// order; a rank keeps the leaves it owns fixed (no ROOT on them) and numbers
+// them from the kernel's global ordinal.  Used with the exact 2-means split and
+// the global or per-leaf scopes (the Lloyd rules and the per-kernel solve keep
+// whole kernels).
+struct GiantPlan {
+    bool on = false;
+    std::vector<uint32_t> ubounds;          // [W + 1] first unit of each rank
+    uint32_t kb = 0, ke = 0;                // my kernel range [kb, ke)
+    uint32_t *kunit = nullptr, *gl_first = nullptr, *gl_n = nullptr, *gl_t = nullptr;   // device tables
+    uint8_t *fixed = nullptr;               // device [ke - kb]
+    uint32_t *ord_off = nullptr;            // device [ke - kb]
+    uint32_t *cuts = nullptr;               // device pairs (local kernel, rows from the local group start)
+    uint64_t ncuts = 0;
+};
+
+static double giant_factor() {
+    static double v = -1.0;
+    if (v < 0.0) {
+        const char *e = getenv("STEMROOT_DIST_GIANT");
+        v = e ? atof(e) : 1.25;
+        if (!(v >= 0.0)) v = 1.25;
+    }
+    return v;
+}
+
+__global__ void gi_group_kernel(const uint32_t *goff, uint32_t G, uint64_t m, uint32_t *grp) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < m) grp[i] = (uint32_t)(upper_bound(goff, (uint64_t)G + 1, (uint32_t)i) - 1);
+}
+
+__global__ void gi_counts_kernel(const uint32_t *start, uint64_t nrec, uint64_t total, uint32_t *cnt) {
+    const uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r < nrec) cnt[r] = (uint32_t)((r + 1 < nrec ? start[r + 1] : total) - start[r]);
+}
+
+__global__ void gi_vcnt_kernel(const uint32_t *vstart, uint64_t D, uint64_t total, const uint64_t *cp, uint64_t *vcnt) {
+    const uint64_t u = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (u < D) vcnt[u] = cp[u + 1 < D ? vstart[u + 1] : total] - cp[vstart[u]];
+}
+
+__global__ void gi_goffv_kernel(const uint32_t *goff, uint32_t G, const uint32_t *vstart, uint64_t D, uint32_t *goffv) {
+    const uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
+    if (g <= G) goffv[g] = (uint32_t)lower_bound(vstart, D, goff[g]);
+}
+
+template <class T>
+static int up(Ctx &c, T *dst, const std::vector<T> &v) {
+    if (!v.empty()) CK(cudaMemcpyAsync(dst, v.data(), sizeof(T) * v.size(), cudaMemcpyHostToDevice, c.stream));
+    return STEM_OK;
+}
+
+// Builds the value trees of the giant kernels and the unit owner map.  Collective.
+static int giant_plan(Ctx &c, Comm &comm, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,
+                      const std::vector<uint64_t> &gcnt, const std::vector<uint32_t> &giant, double eps, double z,
+                      int clamp, GiantPlan &gp) {
+    cudaStream_t st = c.stream;
+    const int W = comm.world, me = comm.rank;
+    const uint32_t G = (uint32_t)giant.size();
+    const double k2 = (z / eps) * (z / eps);
+    std::vector<uint32_t> gidx_h(K, 0xFFFFFFFFu);
+    for (uint32_t g = 0; g < G; g++) gidx_h[giant[g]] = g;
+    // 1. this rank's rows of the giant kernels, sorted by (giant, t), run-length encoded
+    uint64_t ng = 0, nrec = 0;
+    uint32_t *rec = nullptr;   // [3][nrec]: giant, t, count
+    CKS(dist_checkpoint(c, [&]() -> int {
+        CKS(c.ensure(c.gi_tab, c.cap_gi_tab, sizeof(uint32_t) * ((uint64_t)K + 1)));
+        uint32_t *gidx = (uint32_t *)c.gi_tab;
+        CKS(up(c, gidx, gidx_h));
+        for (int i = 0; i < 2; i++) CKS(c.ensure(c.xfer_u32[i], c.cap_xfer_u32[i], sizeof(uint32_t) * (n + 1)));
+        CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(n + 1) + 1) * sizeof(uint64_t)));
+        uint32_t *ga = c.xfer_u32[0], *ta = c.xfer_u32[1];
+        exclusive_scan<uint64_t>(
+            [kid, gidx] __device__(uint64_t i) -> uint64_t { return gidx[kid[i]] != 0xFFFFFFFFu ? 1ull : 0ull; },
+            [kid, t, gidx, ga, ta] __device__(uint64_t i, uint64_t pre, uint64_t v) {
+                if (v) { ga[pre] = gidx[kid[i]]; ta[pre] = t[i]; }
+            },
+            n, (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
+        CK(cudaMemcpyAsync(&ng, &c.scalars->scan_total64, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CKS(sync_stream(c));
+        CKS(c.ensure(c.gi_rec, c.cap_gi_rec, sizeof(uint32_t) * 4 * (ng + 1)));
+        rec = (uint32_t *)c.gi_rec;
+        if (!ng) return STEM_OK;
+        CKS(c.ensure_all(ng, G, 0));
+        CKS(sort_trace(c, ga, ta, nullptr, ng, G, false));
+        uint32_t *grp = rec + 3 * (ng + 1);   // scratch: giant of each sorted position
+        gi_group_kernel<<<(unsigned)((ng + 255) / 256), 256, 0, st>>>(c.goff, G, ng, grp);
+        const uint32_t *ts = c.t_sorted;
+        uint32_t *rg = rec, *rt = rec + (ng + 1), *rs = rec + 2 * (ng + 1);
+        exclusive_scan<uint64_t>(
+            [ts, grp] __device__(uint64_t i) -> uint64_t {
+                return (i == 0 || grp[i] != grp[i - 1] || ts[i] != ts[i - 1]) ? 1ull : 0ull;
+            },
+            [ts, grp, rg, rt, rs] __device__(uint64_t i, uint64_t pre, uint64_t v) {
+                if (v) { rg[pre] = grp[i]; rt[pre] = ts[i]; rs[pre] = (uint32_t)i; }
+            },
+            ng, (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
+        CK(cudaMemcpyAsync(&nrec, &c.scalars->scan_total64, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CKS(sync_stream(c));
+        gi_counts_kernel<<<(unsigned)((nrec + 255) / 256), 256, 0, st>>>(rs, nrec, ng, grp);
+        CK(cudaMemcpyAsync(rs, grp, sizeof(uint32_t) * nrec, cudaMemcpyDeviceToDevice, st));   // starts -> counts
+        c.launches += 2;
+        CK(cudaGetLastError());
+        return STEM_OK;
+    }()));
+    // 2. every rank's records, on every rank (rank order)
+    std::vector<uint64_t> cnts((size_t)W);
+    CKS(comm.allgather_host(&nrec, 1, cnts.data(), st));
+    uint64_t Rall = 0;
+    std::vector<uint64_t> scnt(W, nrec), sdsp(W, 0), rcnt(W), rdsp(W);
+    for (int r = 0; r < W; r++) { rcnt[r] = cnts[r]; rdsp[r] = Rall; Rall += cnts[r]; }
+    uint32_t *all = nullptr;
+    CKS(dist_checkpoint(c, [&]() -> int {
+        CKS(c.ensure(c.gi_all, c.cap_gi_all, sizeof(uint32_t) * 3 * (Rall + 1)));
+        all = (uint32_t *)c.gi_all;
+        return STEM_OK;
+    }()));
+    const uint32_t *rsrc = (const uint32_t *)c.gi_rec;
+    for (int f = 0; f < 3; f++)
+        CKS(comm.alltoallv(rsrc + f * (ng + 1), scnt.data(), sdsp.data(), all + f * (Rall + 1), rcnt.data(),
+                           rdsp.data(), sizeof(uint32_t), st));
+    CKS(sync_stream(c));
+    // 3. merged histogram (identical on every rank), the value trees, the leaves
+    std::vector<uint32_t> l_g, l_t;
+    std::vector<uint64_t> l_rows;
+    CKS(dist_checkpoint(c, [&]() -> int {
+        if (!Rall) return STEM_OK;
+        uint32_t *ag = all, *at = all + (Rall + 1), *ac = all + 2 * (Rall + 1);
+        CKS(c.ensure_all(Rall, G, 0));
+        CKS(sort_trace(c, ag, at, ac, Rall, G, false));   // payload = the counts
+        const uint32_t *ts = c.t_sorted, *cs = c.row_sorted, *goff = c.goff;
+        CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(Rall + 1) + 1) * sizeof(uint64_t)));
+        const uint64_t R2 = (Rall + 2 + 1) & ~1ull, G2 = (G + 2 + 1) & ~1ull;   // even: 8-byte aligned after
+        CKS(c.ensure(c.gi_val, c.cap_gi_val, sizeof(uint32_t) * (3 * R2 + G2) + sizeof(uint64_t) * 2 * R2 + R2));
+        uint32_t *grp = (uint32_t *)c.gi_val, *vt = grp + R2, *vstart = vt + R2, *goffv = vstart + R2;
+        uint64_t *cp = (uint64_t *)(goffv + G2), *vcnt = cp + R2;
+        uint8_t *vflag = (uint8_t *)(vcnt + R2);
+        gi_group_kernel<<<(unsigned)((Rall + 255) / 256), 256, 0, st>>>(goff, G, Rall, grp);
+        exclusive_scan<uint64_t>([cs] __device__(uint64_t i) -> uint64_t { return cs[i]; },
+                                 [cp] __device__(uint64_t i, uint64_t pre, uint64_t) { cp[i] = pre; }, Rall,
+                                 (uint64_t *)c.scan_scratch, &c.scalars->scan_total64, st, &c.launches);
+        uint64_t D = 0;
+        exclusive_scan<uint64_t>(
+            [ts, grp] __device__(uint64_t i) -> uint64_t {
+                return (i == 0 || grp[i] != grp[i - 1] || ts[i] != ts[i - 1]) ? 1ull : 0ull;
+            },
+            [ts, vt, vstart] __device__(uint64_t i, uint64_t pre, uint64_t v) {
+                if (v) { vt[pre] = ts[i]; vstart[pre] = (uint32_t)i; }
+            },
+            Rall, (uint64_t *)c.scan_scratch, &c.scalars->scan_total64b, st, &c.launches);
+        uint64_t tot_rows = 0;
+        CK(cudaMemcpyAsync(&D, &c.scalars->scan_total64b, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(&tot_rows, &c.scalars->scan_total64, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CKS(sync_stream(c));
+        CK(cudaMemcpyAsync(cp + Rall, &tot_rows, sizeof(uint64_t), cudaMemcpyHostToDevice, st));
+        gi_vcnt_kernel<<<(unsigned)((D + 255) / 256), 256, 0, st>>>(vstart, D, Rall, cp, vcnt);
+        gi_goffv_kernel<<<(unsigned)((G + 256) / 256), 256, 0, st>>>(goff, G, vstart, D, goffv);
+        c.launches += 3;
+        CK(cudaGetLastError());
+        CKS(root_values(c, vt, vcnt, goffv, G, D, eps, z, k2, clamp, vflag));
+        // leaves: value starts with vflag set, their giant, lowest t and rows (from the prefix counts)
+        std::vector<uint8_t> vf(D);
+        std::vector<uint32_t> vt_h(D), goffv_h(G + 1);
+        std::vector<uint64_t> vcnt_h(D);
+        CK(cudaMemcpyAsync(vf.data(), vflag, D, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(vt_h.data(), vt, sizeof(uint32_t) * D, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(vcnt_h.data(), vcnt, sizeof(uint64_t) * D, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(goffv_h.data(), goffv, sizeof(uint32_t) * (G + 1), cudaMemcpyDeviceToHost, st));
+        CKS(sync_stream(c));
+        for (uint32_t g = 0; g < G; g++)   // (host bookkeeping of the tree's leaves: list building only)
+            for (uint32_t u = goffv_h[g]; u < goffv_h[g + 1]; u++) {
+                if (vf[u] || u == goffv_h[g]) {
+                    l_g.push_back(g);
+                    l_t.push_back(vt_h[u]);
+                    l_rows.push_back(0);
+                }
+                l_rows.back() += vcnt_h[u];
+            }
+        return STEM_OK;
+    }()));
+    // 4. units in (kernel, value) order and the owner map over them
+    std::vector<uint64_t> urows;
+    std::vector<uint32_t> ukid, uleaf, kunit_h(K + 1), gl_first_h(K, 0), gl_n_h(K, 0), gl_t_h;
+    {
+        std::vector<uint32_t> gfirst(G + 1, 0);
+        for (size_t i = 0; i < l_g.size(); i++) gfirst[l_g[i] + 1]++;
+        for (uint32_t g = 0; g < G; g++) gfirst[g + 1] += gfirst[g];
+        for (uint32_t k = 0; k < K; k++) {
+            kunit_h[k] = (uint32_t)urows.size();
+            const uint32_t g = gidx_h[k];
+            if (g == 0xFFFFFFFFu || gfirst[g + 1] == gfirst[g]) {
+                urows.push_back(gcnt[k]);
+                ukid.push_back(k);
+                uleaf.push_back(0);
+                continue;
+            }
+            gl_first_h[k] = (uint32_t)gl_t_h.size();
+            gl_n_h[k] = gfirst[g + 1] - gfirst[g];
+            for (uint32_t j = gfirst[g]; j < gfirst[g + 1]; j++) {
+                urows.push_back(l_rows[j]);
+                ukid.push_back(k);
+                uleaf.push_back(j - gfirst[g]);
+                gl_t_h.push_back(l_t[j]);
+            }
+        }
+        kunit_h[K] = (uint32_t)urows.size();
+    }
+    const uint32_t U = (uint32_t)urows.size();
+    gp.ubounds.assign(W + 1, 0);
+    owner_ranges(urows.data(), U, W, gp.ubounds.data());
+    const uint32_t u0 = gp.ubounds[me], u1 = gp.ubounds[me + 1];
+    gp.kb = u0 < u1 ? ukid[u0] : 0;
+    gp.ke = u0 < u1 ? ukid[u1 - 1] + 1 : 0;
+    const uint32_t KL = gp.ke - gp.kb;
+    std::vector<uint8_t> fixed_h(KL + 1, 0);
+    std::vector<uint32_t> ord_h(KL + 1, 0), cuts_h;
+    for (uint32_t u = u0; u < u1; u++) {
+        const uint32_t kl = ukid[u] - gp.kb;
+        if (gl_n_h[ukid[u]] == 0) continue;
+        if (!fixed_h[kl]) {   // the first leaf of this kernel on this rank
+            fixed_h[kl] = 1;
+            ord_h[kl] = uleaf[u];
+            continue;
+        }
+        uint64_t rel = 0;     // rows of this kernel's earlier local leaves
+        for (uint32_t v = u; v-- > u0 && ukid[v] == ukid[u];) rel += urows[v];
+        cuts_h.push_back(kl);
+        cuts_h.push_back((uint32_t)rel);
+    }
+    gp.ncuts = cuts_h.size() / 2;
+    CKS(dist_checkpoint(c, [&]() -> int {
+        const size_t words = (size_t)3 * (K + 1) + gl_t_h.size() + 2 * (KL + 1) + cuts_h.size() + 8;
+        CKS(c.ensure(c.gi_tab, c.cap_gi_tab, sizeof(uint32_t) * words));
+        uint32_t *w = (uint32_t *)c.gi_tab;
+        gp.kunit = w; w += K + 1;
+        gp.gl_first = w; w += K + 1;
+        gp.gl_n = w; w += K + 1;
+        gp.gl_t = w; w += gl_t_h.size() + 1;
+        gp.ord_off = w; w += KL + 1;
+        gp.cuts = w; w += cuts_h.size() + 1;
+        gp.fixed = (uint8_t *)w;
+        CKS(up(c, gp.kunit, kunit_h));
+        gl_first_h.push_back(0);
+        gl_n_h.push_back(0);
+        CKS(up(c, gp.gl_first, gl_first_h));
+        CKS(up(c, gp.gl_n, gl_n_h));
+        CKS(up(c, gp.gl_t, gl_t_h));
+        CKS(up(c, gp.ord_off, ord_h));
+        CKS(up(c, gp.cuts, cuts_h));
+        CKS(up(c, gp.fixed, fixed_h));
+        return sync_stream(c);   // the host vectors are this frame's
+    }()));
+    gp.on = true;
+    return STEM_OK;
+}
+
 // local_status: the rank's own argument checks (stem_root_plan_dist), agreed
 // across ranks first.  Every later stretch of local work ends in a checkpoint
 // (or in exchange_counts, which carries the status) before the next
@@ -763,11 +1035,33 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
     if (gcnt[K]) return STEM_E_RANGE;   // the same reduced flag on every rank
     std::vector<uint32_t> bounds(W + 1);
     owner_ranges(gcnt.data(), K, W, bounds.data());
-    const uint32_t kb = bounds[me], ke = bounds[me + 1];
+    uint32_t kb = bounds[me], ke = bounds[me + 1];
+    // kernels larger than a rank's share: value trees and unit ownership (identical decision on every rank)
+    GiantPlan gp;
+    {
+        std::vector<uint32_t> giant;
+        uint64_t N = 0;
+        for (uint32_t k = 0; k < K; k++) N += gcnt[k];
+        const double f = giant_factor();
+        if (W > 1 && f > 0.0 && o.root && o.split == 0 && o.scope != 1)
+            for (uint32_t k = 0; k < K; k++)
+                if ((double)gcnt[k] * W > f * (double)N) giant.push_back(k);
+        if (!giant.empty()) {
+            CKS(giant_plan(c, comm, kid, t, n, K, gcnt, giant, eps, c.z, o.clamp_in_split ? 1 : 0, gp));
+            kb = gp.kb;
+            ke = gp.ke;
+        }
+    }
     // 2. all-to-all keyed on kernel id: (kernel_id, t, global row) to the owner of the kernel
     PartArgs pa{};
     pa.key = kid;
-    for (int r = 0; r <= W; r++) pa.bounds[r] = bounds[r];
+    for (int r = 0; r <= W; r++) pa.bounds[r] = gp.on ? gp.ubounds[r] : bounds[r];
+    if (gp.on) {
+        pa.kunit = gp.kunit;
+        pa.gl_first = gp.gl_first;
+        pa.gl_n = gp.gl_n;
+        pa.gl_t = gp.gl_t;
+    }
     pa.world = W;
     pa.n = n;
     pa.in0 = kid;
@@ -827,6 +1121,16 @@ int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, d
     // 3. the local pipeline on my kernel range (kernel ids rebased to 0)
     const uint32_t KL = ke - kb;
     c.kid_base = kb;
+    if (gp.on) {   // this rank's leaves of split kernels are given: no ROOT on them, ordinals from the tree
+        c.fixed_kernel = gp.fixed;
+        c.fixed_cuts = gp.cuts;
+        c.n_fixed_cuts = gp.ncuts;
+        c.ord_off = gp.ord_off;
+    }
+    struct Unfix {
+        Ctx &c;
+        ~Unfix() { c.fixed_kernel = nullptr; c.fixed_cuts = nullptr; c.n_fixed_cuts = 0; c.ord_off = nullptr; }
+    } unfix{c};
     CKS(dist_checkpoint(c, [&]() -> int {
         if (!R) return STEM_OK;
         sub_kernel_u32<<<(unsigned)((R + 255) / 256), 256, 0, st>>>(c.recv_u32[0], R, kb);

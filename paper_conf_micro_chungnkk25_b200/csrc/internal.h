@@ -216,7 +216,15 @@ struct Ctx {
     uint64_t *km_dP = nullptr; size_t cap_km_dP = 0;
     double *km_F = nullptr; size_t cap_km_F = 0;
     void *km_meta = nullptr, *km_sub = nullptr; size_t cap_km_meta = 0, cap_km_sub = 0;
-    void *peer_dst = nullptr; size_t cap_peer_dst = 0;   // fused exchange: the owners' windows (PeerDst)
+    void *peer_dst = nullptr; size_t cap_peer_dst = 0;
+    // multi-GPU kernels larger than a rank's share (root.cu root_values, dist.cu)
+    void *vr_P = nullptr, *vr_work = nullptr; size_t cap_vr_P = 0, cap_vr_work = 0;
+    void *gi_buf = nullptr; size_t cap_gi_buf = 0;
+    void *gi_tab = nullptr, *gi_rec = nullptr, *gi_all = nullptr, *gi_val = nullptr;   // histograms, tables
+    size_t cap_gi_tab = 0, cap_gi_rec = 0, cap_gi_all = 0, cap_gi_val = 0;
+    const uint8_t *fixed_kernel = nullptr;                  // local kernels whose leaves are given (no ROOT)
+    const uint32_t *fixed_cuts = nullptr; uint64_t n_fixed_cuts = 0;   // their inner leaf starts: (local kernel, row in group)
+    const uint32_t *ord_off = nullptr;                      // per local kernel: ordinal of its first local leaf   // fused exchange: the owners' windows (PeerDst)
     uint64_t row_bases[65] = {0};
     uint64_t n_local_rows = 0;
     // metric_bounds (metric.cu): leaf table (first leaf per kernel, lo_ns, n, m), per-leaf sums
@@ -259,6 +267,9 @@ int prefix_moments(Ctx &c, uint64_t n);                                         
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp,
                 int split, uint64_t seed);   // a3, a4 (split: 0 exact 2-means, 1 Lloyd, 2 k-means++ Lloyd)
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
+// ROOT over a histogram of distinct values per group (root.cu): vflag[u] = 1 where a leaf starts
+int root_values(Ctx &c, const uint32_t *vt, const uint64_t *vcnt, const uint32_t *goffv, uint32_t G, uint64_t D,
+                double eps, double z, double k2, int clamp, uint8_t *vflag);
 // split = 3: ROOT with exact optimal 1-D k-means splits into kk groups (kmeans.cu, R29)
 int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, uint32_t kk);
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,

@@ -1276,6 +1276,15 @@ __global__ void group_flags_kernel(const uint32_t *goff, uint32_t K, uint32_t *f
 }
 
 
+// leaf starts given from outside (multi-GPU: the leaves of a kernel split across
+// ranks): entry i = (local kernel, rows from the kernel's local group start)
+__global__ void fixed_flags_kernel(const uint32_t *cut, uint64_t m, const uint32_t *goff, uint32_t *flags) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= m) return;
+    const uint32_t p = goff[cut[2 * i]] + cut[2 * i + 1];
+    atomicOr(&flags[p >> 5], 1u << (p & 31));
+}
+
 int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K) {
     CK(cudaMemsetAsync(c.flags, 0, sizeof(uint32_t) * (n / 32 + 1), c.stream));
     group_flags_kernel<<<(unsigned)((K + 255) / 256), 256, 0, c.stream>>>(c.goff, K, c.flags);
@@ -1318,11 +1327,17 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         uint32_t *nlo = c.f_lo[0], *nhi = c.f_hi[0];
         uint64_t *nS = c.f_S[0];
         u128 *nQ = c.f_Q[0];
+        const uint8_t *fixed = c.fixed_kernel;   // multi-GPU: kernels whose leaves were decided on the value tree
+        if (c.fixed_cuts && c.n_fixed_cuts) {
+            fixed_flags_kernel<<<(unsigned)((c.n_fixed_cuts + 255) / 256), 256, 0, st>>>(c.fixed_cuts, c.n_fixed_cuts,
+                                                                                      c.goff, c.flags);
+            c.launches++;
+        }
         const int tk = c.stage_begin("root_init");
         exclusive_scan<uint64_t>(
-            [goff, t] __device__(uint64_t g) -> uint64_t {
+            [goff, t, fixed] __device__(uint64_t g) -> uint64_t {
                 const uint32_t lo = goff[g], hi = goff[g + 1];
-                return nontrivial(t, lo, hi) ? ((1ull << 32) | (hi - lo)) : 0ull;
+                return (nontrivial(t, lo, hi) && !(fixed && fixed[g])) ? ((1ull << 32) | (hi - lo)) : 0ull;
             },
             [nlo, nhi, nS, nQ, goff, t, PS1, PS2] __device__(uint64_t g, uint64_t pre, uint64_t v) {
                 if (!v) return;
@@ -1520,6 +1535,167 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
     c.stats.active_rows += hs.local_rows;
     c.stats.split_chunks = hs.split_chunks;
     c.stats.split_scanned = hs.split_scanned;
+    return STEM_OK;
+}
+
+
+// ---------------------------------------------------------------- ROOT over a value histogram
+// ROOT's decisions depend only on the multiset of a cluster's times: a cut
+// lies between two distinct values, D_k = n S_L - S k and the Eq. 7/8 test use
+// the counts and sums below it.  So the tree of a kernel can be built from its
+// distinct values and their counts alone -- exactly the tree the row levels
+// build -- which is how the multi-GPU plan splits a kernel larger than a
+// rank's share (dist.cu): every rank builds the value tree of the merged
+// histogram, then the kernel's leaves are dealt to ranks whole.
+struct VH {
+    uint64_t c, s;
+    u128 q;
+};
+__host__ __device__ __forceinline__ VH operator+(const VH &a, const VH &b) { return VH{a.c + b.c, a.s + b.s, a.q + b.q}; }
+__host__ __device__ __forceinline__ VH operator-(const VH &a, const VH &b) { return VH{a.c - b.c, a.s - b.s, a.q - b.q}; }
+
+struct VrArgs {
+    const VH *P;               // [D + 1] exclusive prefix of (count, sum t, sum t^2) over the values
+    const uint32_t *vlo, *vhi; // frontier: value ranges [vlo, vhi)
+    const uint64_t *ctot;      // packed (count << 32 | values) of the frontier
+    uint32_t *cutv;            // per cluster: value index of the cut (0: none)
+    uint64_t *cutk;            // per cluster: rows left of the cut
+    uint64_t *cutSL;
+};
+
+// one block per cluster: the exact best cut over the cluster's distinct-value boundaries
+__global__ void __launch_bounds__(256) vroot_cut_kernel(VrArgs a) {
+    __shared__ Cand s_best[8];
+    const uint32_t C = (uint32_t)(*a.ctot >> 32);
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (uint32_t ci = blockIdx.x; ci < C; ci += gridDim.x) {
+        const uint32_t v0 = a.vlo[ci], v1 = a.vhi[ci];
+        const VH p0 = a.P[v0], tot = a.P[v1] - p0;
+        const uint64_t n = tot.c, S = tot.s;
+        Cand best = no_cand();
+        for (uint32_t u = v0 + 1 + threadIdx.x; u < v1; u += blockDim.x) {
+            const VH pu = a.P[u] - p0;
+            eval_cut((uint32_t)pu.c, n, S, pu.s, best);
+        }
+#pragma unroll 1
+        for (int o = 16; o; o >>= 1) {
+            const Cand v = shfl_cand_xor(best, o);
+            if (better(v, best)) best = v;
+        }
+        if (lane == 0) s_best[w] = best;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            Cand b = s_best[0];
+            for (int k = 1; k < 8; k++)
+                if (better(s_best[k], b)) b = s_best[k];
+            uint32_t cu = 0;
+            if (b.k) {   // the value index whose prefix count is k
+                uint32_t lo = v0 + 1, hi = v1;
+                while (lo < hi) {
+                    const uint32_t mid = lo + (hi - lo) / 2;
+                    if (a.P[mid].c - p0.c < b.k) lo = mid + 1; else hi = mid;
+                }
+                cu = lo;
+            }
+            a.cutv[ci] = cu;
+            a.cutk[ci] = b.k;
+            a.cutSL[ci] = b.SL;
+        }
+        __syncthreads();
+    }
+}
+
+struct VdArgs {
+    const VH *P;
+    const uint32_t *vlo, *vhi;
+    const uint64_t *ctot;
+    const uint32_t *cutv;
+    const uint64_t *cutk, *cutSL;
+    uint8_t *vflag;            // 1 at the first value of every leaf
+    uint32_t *nlo, *nhi;
+    uint64_t *total;
+    double eps, z, k2;
+    int clamp;
+};
+
+__global__ void vroot_decide_kernel(VdArgs a) {
+    const uint64_t ci = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (ci >= (*a.ctot >> 32)) return;
+    const uint32_t v0 = a.vlo[ci], v1 = a.vhi[ci], u = a.cutv[ci];
+    if (!u) return;
+    const VH p0 = a.P[v0], tot = a.P[v1] - p0, left = a.P[u] - p0;
+    if (!split_pays(tot.c, tot.s, tot.q, a.cutk[ci], a.cutSL[ci], left.q, a.eps, a.z, a.k2, a.clamp)) return;
+    a.vflag[u] = 1;
+    const uint32_t kids[2][2] = {{v0, u}, {u, v1}};
+    for (int h = 0; h < 2; h++)
+        if (kids[h][1] - kids[h][0] >= 2) {   // at least two distinct values
+            const uint64_t slot = atomicAdd((unsigned long long *)a.total,
+                                            (unsigned long long)((1ull << 32) | (kids[h][1] - kids[h][0]))) >> 32;
+            a.nlo[slot] = kids[h][0];
+            a.nhi[slot] = kids[h][1];
+        }
+}
+
+__global__ void vroot_init_kernel(const uint32_t *goffv, uint32_t G, uint8_t *vflag, uint32_t *nlo, uint32_t *nhi,
+                                  uint64_t *total) {
+    const uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
+    if (g >= G) return;
+    const uint32_t v0 = goffv[g], v1 = goffv[g + 1];
+    if (v1 > v0) vflag[v0] = 1;
+    if (v1 - v0 >= 2) {
+        const uint64_t slot = atomicAdd((unsigned long long *)total, (unsigned long long)((1ull << 32) | (v1 - v0))) >> 32;
+        nlo[slot] = v0;
+        nhi[slot] = v1;
+    }
+}
+
+int root_values(Ctx &c, const uint32_t *vt, const uint64_t *vcnt, const uint32_t *goffv, uint32_t G, uint64_t D,
+                double eps, double z, double k2, int clamp, uint8_t *vflag) {
+    cudaStream_t st = c.stream;
+    CKS(c.ensure(c.vr_P, c.cap_vr_P, sizeof(VH) * (D + 2)));
+    CKS(c.ensure(c.vr_work, c.cap_vr_work, (sizeof(uint32_t) * 5 + sizeof(uint64_t) * 2) * (D + 3) + 8));
+    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(D + 1) + 1) * sizeof(VH)));
+    VH *P = (VH *)c.vr_P;
+    {
+        exclusive_scan<VH>(
+            [vt, vcnt, D] __device__(uint64_t i) -> VH {
+                if (i >= D) return VH{0, 0, 0};
+                const uint64_t cn = vcnt[i], tv = vt[i];
+                return VH{cn, cn * tv, (u128)cn * ((u128)tv * tv)};
+            },
+            [P] __device__(uint64_t i, VH pre, VH) { P[i] = pre; }, D + 1, (VH *)c.scan_scratch,
+            (VH *)c.scalars->wide_total, st, &c.launches);
+    }
+    uint32_t *w32 = (uint32_t *)c.vr_work;
+    const uint64_t D2 = (D + 2 + 1) & ~1ull;   // even: the u64 arrays after the u32 ones stay aligned
+    uint32_t *lo[2] = {w32, w32 + D2}, *hi[2] = {w32 + 2 * D2, w32 + 3 * D2};
+    uint32_t *cutv = w32 + 4 * D2;
+    uint64_t *cutk = (uint64_t *)(w32 + 5 * D2 + (5 * D2 & 1)), *cutSL = cutk + D2;
+    CK(cudaMemsetAsync(vflag, 0, D + 1, st));
+    CK(cudaMemsetAsync(&c.scalars->ftot[0], 0, 2 * sizeof(uint64_t), st));
+    if (G) {
+        vroot_init_kernel<<<(G + 255) / 256, 256, 0, st>>>(goffv, G, vflag, lo[0], hi[0], &c.scalars->ftot[0]);
+        c.launches++;
+    }
+    uint64_t tot = 0;
+    CK(cudaMemcpyAsync(&tot, &c.scalars->ftot[0], sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    int cur = 0;
+    while (tot >> 32) {
+        const uint64_t C = tot >> 32;
+        const int nxt = cur ^ 1;
+        VrArgs va{P, lo[cur], hi[cur], &c.scalars->ftot[cur], cutv, cutk, cutSL};
+        vroot_cut_kernel<<<(unsigned)min(C, (uint64_t)c.sms * 8), 256, 0, st>>>(va);
+        CK(cudaMemsetAsync(&c.scalars->ftot[nxt], 0, sizeof(uint64_t), st));
+        VdArgs vd{P, lo[cur], hi[cur], &c.scalars->ftot[cur], cutv, cutk, cutSL, vflag, lo[nxt], hi[nxt],
+                  &c.scalars->ftot[nxt], eps, z, k2, clamp};
+        vroot_decide_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(vd);
+        c.launches += 2;
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(&tot, &c.scalars->ftot[nxt], sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        cur = nxt;
+    }
     return STEM_OK;
 }
 

@@ -115,6 +115,7 @@ struct LeafArgs {
     uint64_t *fix_acc;   // [scope==1 ? K : 1][kFixDigits]
     uint64_t *kern_T;    // scope 1
     uint32_t *err;
+    const uint32_t *ord_off;   // multi-GPU: ordinal of the kernel's first local leaf (NULL: 0)
 };
 
 struct LeafView {
@@ -155,7 +156,7 @@ __global__ void __launch_bounds__(kThreads) leaf_kkt_kernel(LeafArgs a) {
         const uint32_t g = (uint32_t)upper_bound(a.goff, (uint64_t)a.K + 1, v.lo) - 1;
         const uint64_t first = lower_bound(a.leaf_lo, a.L, a.goff[g]);
         a.leaf_kid[i] = g;
-        a.leaf_ord[i] = (uint32_t)(i - first);
+        a.leaf_ord[i] = (uint32_t)(i - first) + (a.ord_off ? a.ord_off[g] : 0u);
         if (a.scope != 2) {
             const double mu = __ddiv_rn(rn64(v.S), rn64(v.n));
             const double term = __dsqrt_rn(__dmul_rn(mu, rn128(v.V)));
@@ -564,7 +565,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
             CK(cudaMemsetAsync(&c.scalars->T, 0, sizeof(uint64_t), st));
         }
         LeafArgs la{c.leaf_lo, c.goff, c.t_sorted, c.PS1, c.PS2, L, n, K, o.scope, leaf_kid, leaf_ord,
-                    c.fix_acc, c.kern_T, &c.scalars->err};
+                    c.fix_acc, c.kern_T, &c.scalars->err, c.ord_off};
         if (L) leaf_kkt_kernel<<<blocks_for(L), kThreads, 0, st>>>(la);
         c.launches++;
         CK(cudaGetLastError());

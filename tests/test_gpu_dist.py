@@ -24,7 +24,7 @@ def sr():
     return m
 
 
-def _dist_plan(sr, kid, t, K, world, metrics=None, **kw):
+def _dist_plan(sr, kid, t, K, world, metrics=None, stats_out=None, **kw):
     import torch
     n = len(kid)
     cuts = [n * r // world for r in range(world + 1)]
@@ -57,6 +57,8 @@ def _dist_plan(sr, kid, t, K, world, metrics=None, **kw):
         if e is not None:
             raise e
     assert all(o is None for o in out[1:])
+    if stats_out is not None:
+        stats_out.extend(c.stats() for c in ctxs)
     for c in ctxs:
         c.close()
     for c in comms:
@@ -111,6 +113,73 @@ def test_loopback_metric_bounds(sr, world):
     ref = O.plan(kid, t, sp.n_kernels, eps=0.03, z=Z95, seed=5, metrics=met, metric_bounds=1)
     got = _dist_plan(sr, kid, t, sp.n_kernels, world, metrics=met, eps=0.03, z=Z95, seed=5, metric_bounds=True)
     assert_plans_equal(got, ref, metrics=True)
+
+
+def _giant_trace(n, K, share, seed):
+    """one kernel holding `share` of the rows (a multi-modal time mix, so its
+    ROOT tree is deep), the rest spread over K - 1 small kernels"""
+    rng = np.random.default_rng(seed)
+    kid = np.where(rng.random(n) < share, 0, rng.integers(1, K, n)).astype(np.uint32)
+    modes = np.array([20_000, 55_000, 140_000, 400_000])
+    t = np.where(kid == 0, modes[rng.integers(0, 4, n)] * rng.lognormal(0, 0.15, n),
+                 (kid * 3000 + 5000) * rng.lognormal(0, 0.3, n)).astype(np.uint32)
+    return kid, t
+
+
+@pytest.mark.parametrize("world", [2, 3, 4, 8])
+def test_loopback_giant_kernel_is_split_across_ranks(sr, world):
+    """A kernel larger than a rank's share (70 % of the rows): its ROOT tree is
+    built on the merged value histogram and its leaves are dealt to ranks as
+    units (dist.cu giant_plan).  The plan equals the single-trace oracle's
+    bit-for-bit on integers, and the busiest rank owns far fewer rows than the
+    70 % it would own with whole kernels."""
+    n, K = 240_000, 41
+    kid, t = _giant_trace(n, K, 0.7, 11 + world)
+    ref = O.plan(kid, t, K, eps=0.02, z=Z95, seed=3)
+    st = []
+    got = _dist_plan(sr, kid, t, K, world, stats_out=st, eps=0.02, z=Z95, seed=3)
+    assert_plans_equal(got, ref)
+    owned = [s["owned_rows"] for s in st]
+    assert sum(owned) == n
+    assert max(owned) < 0.7 * n * 0.9, owned
+
+
+@pytest.mark.parametrize("opts", [dict(scope=2), dict(census_cap=True, eps=0.005), dict(clamp_in_split=False)])
+def test_loopback_giant_kernel_options(sr, opts):
+    n, K = 120_000, 9
+    kid, t = _giant_trace(n, K, 0.8, 5)
+    kw = dict(z=Z95, seed=4)
+    kw.update(opts)
+    eps = kw.pop("eps", 0.03)
+    ref = O.plan(kid, t, K, eps=eps, **kw)
+    got = _dist_plan(sr, kid, t, K, 3, eps=eps, **kw)
+    assert_plans_equal(got, ref)
+
+
+def test_loopback_giant_kernel_with_metrics(sr):
+    n, K = 100_000, 13
+    kid, t = _giant_trace(n, K, 0.6, 8)
+    met = np.random.default_rng(2).normal(5, 1, (2, n))
+    ref = O.plan(kid, t, K, eps=0.03, z=Z95, seed=6, metrics=met, metric_bounds=1)
+    got = _dist_plan(sr, kid, t, K, 4, metrics=met, eps=0.03, z=Z95, seed=6, metric_bounds=True)
+    assert_plans_equal(got, ref, metrics=True)
+
+
+def test_loopback_giant_kernel_disabled_by_env(sr, monkeypatch):
+    """STEMROOT_DIST_GIANT=0 keeps whole kernels (the value is read once per
+    process, so this runs in a child)"""
+    import subprocess
+    import sys
+    code = (
+        "import sys; sys.path.insert(0, 'tests'); sys.path.insert(0, '.')\n"
+        "import numpy as np, test_gpu_dist as T, paper_conf_micro_chungnkk25_b200 as sr, oracle as O\n"
+        "kid, t = T._giant_trace(60000, 7, 0.7, 1); st = []\n"
+        "got = T._dist_plan(sr, kid, t, 7, 2, stats_out=st, z=T.Z95)\n"
+        "T.assert_plans_equal(got, O.plan(kid, t, 7, z=T.Z95))\n"
+        "assert max(s['owned_rows'] for s in st) >= 0.69 * 60000, st\n")
+    env = dict(os.environ, STEMROOT_DIST_GIANT="0")
+    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-3000:]
 
 
 def test_nccl_single_rank(sr):
