@@ -43,9 +43,10 @@
 extern "C" {
 #endif
 
-#define STEMROOT_ABI_VERSION 4   /* 2: stem_opts.split; 3: split = 2 (k-means++ seeds);
+#define STEMROOT_ABI_VERSION 5   /* 2: stem_opts.split; 3: split = 2 (k-means++ seeds);
                                     4: metric_bounds, true_metric, bound_metric; split = 3 and
-                                    kmeans_k; stem_stats.owned_rows/world/fused_exchange */
+                                    kmeans_k; stem_stats.owned_rows/world/fused_exchange;
+                                    5: stem_stats.value_groups/value_count/value_levels */
 
 #if defined(__GNUC__)
 #define STEM_API __attribute__((visibility("default")))
@@ -180,6 +181,12 @@ typedef struct stem_stats {
     uint32_t fused_exchange;   /* 1: the last stem_root_plan_dist stored every row straight into
                                   its owner's receive window (peer memory over NVLink, CUDA IPC);
                                   0: grouped send/recv (STEMROOT_DIST_P2P=0, or no peer access) */
+    uint32_t value_levels;     /* ROOT levels of the value-histogram path (0: not used)         */
+    uint64_t value_groups;     /* kernel groups whose ROOT tree was built over their distinct
+                                  values instead of their rows (split = 0: groups of
+                                  >= STEMROOT_VALUE_ROWS rows whose times repeat; the tree is
+                                  the same)                                    */
+    uint64_t value_count;      /* distinct values of those groups                               */
 } stem_stats;
 
 /* Per-stage device time of the last plan (stem_ctx_enable_timing).  bytes is

@@ -111,7 +111,8 @@ class stem_stats(C.Structure):
                 ("n_samples", C.c_uint64), ("ssum", C.c_double), ("pack_bits", C.c_uint32),
                 ("ambiguous_samples", C.c_uint32), ("coarse_bases", C.c_uint32), ("reserved0", C.c_uint32),
                 ("split_chunks", C.c_uint64), ("split_scanned", C.c_uint64), ("owned_rows", C.c_uint64),
-                ("world", C.c_uint32), ("fused_exchange", C.c_uint32)]
+                ("world", C.c_uint32), ("fused_exchange", C.c_uint32), ("value_levels", C.c_uint32),
+                ("value_groups", C.c_uint64), ("value_count", C.c_uint64)]
 
 
 class stem_stage_time(C.Structure):

@@ -23,7 +23,7 @@ int Ctx::ensure_all(uint64_t n, uint32_t K, uint32_t n_metrics) {
     CKS(ensure(keys[1], cap_keys[1], sizeof(uint64_t) * n));
     CKS(ensure(vals[0], cap_vals[0], sizeof(uint32_t) * n));
     CKS(ensure(vals[1], cap_vals[1], sizeof(uint32_t) * n));
-    CKS(ensure(t_sorted, cap_ts, sizeof(uint32_t) * (n + 1)));
+    CKS(ensure(t_sorted, cap_ts, sizeof(uint32_t) * (n + 4)));   // + slack: uint4 reads of the last rows
     CKS(ensure(row_sorted, cap_rs, sizeof(uint32_t) * (n + 1)));
     CKS(ensure(kid_count, cap_kc, sizeof(uint32_t) * ((uint64_t)K + 1)));
     CKS(ensure(goff, cap_goff, sizeof(uint32_t) * ((uint64_t)K + 2)));
@@ -55,6 +55,16 @@ void Ctx::release() {
     for (int i = 0; i < 4; i++)
         if (ev_lvl[i]) { cudaEventDestroy(ev_lvl[i]); ev_lvl[i] = nullptr; }
     if (h_lvl) { cudaFreeHost(h_lvl); h_lvl = nullptr; }
+    for (int i = 0; i < 8; i++)
+        if (ev_vr[i]) { cudaEventDestroy(ev_vr[i]); ev_vr[i] = nullptr; }
+    if (h_vr) { cudaFreeHost(h_vr); h_vr = nullptr; }
+    if (h_vcount) { cudaFreeHost(h_vcount); h_vcount = nullptr; }
+    if (ev_vcount) { cudaEventDestroy(ev_vcount); ev_vcount = nullptr; }
+    if (ev_vfork) cudaEventDestroy(ev_vfork);
+    if (ev_vjoin) cudaEventDestroy(ev_vjoin);
+    if (vside) cudaStreamDestroy(vside);
+    ev_vfork = ev_vjoin = nullptr;
+    vside = nullptr;
     ev_fork = ev_join = nullptr;
     side = nullptr;
     dfree(in_kid, cap_in_kid); dfree(in_t, cap_in_t); dfree(in_met, cap_in_met);
@@ -76,6 +86,7 @@ void Ctx::release() {
     dfree(big_ent, cap_big_ent); dfree(big_part, cap_big_part); dfree(big_thr, cap_big_thr);
     dfree(peer_dst, cap_peer_dst);
     dfree(vr_P, cap_vr_P); dfree(vr_work, cap_vr_work); dfree(gi_buf, cap_gi_buf);
+    dfree(dn_sel, cap_dn_sel); dfree(dn_meta, cap_dn_meta); dfree(dn_val, cap_dn_val);
     dfree(gi_tab, cap_gi_tab); dfree(gi_rec, cap_gi_rec); dfree(gi_all, cap_gi_all); dfree(gi_val, cap_gi_val);
     dfree(km_dpos, cap_km_dpos); dfree(km_arg, cap_km_arg); dfree(km_ngrp, cap_km_ngrp);
     dfree(km_dP, cap_km_dP); dfree(km_F, cap_km_F); dfree(km_meta, cap_km_meta); dfree(km_sub, cap_km_sub);

@@ -106,6 +106,12 @@ struct Ctx {
     cudaStream_t stream = nullptr;
     cudaStream_t side = nullptr;                 // ROOT: the small-cluster split runs beside the big path
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    cudaStream_t vside = nullptr;                // ROOT: the value-histogram levels run beside the row levels
+    cudaEvent_t ev_vfork = nullptr, ev_vjoin = nullptr;
+    uint64_t *h_vr = nullptr;                    // pinned: value-level frontier totals (ring)
+    uint64_t *h_vcount = nullptr;                // pinned: distinct values of the dense groups
+    cudaEvent_t ev_vcount = nullptr;
+    cudaEvent_t ev_vr[8] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     uint64_t *h_lvl = nullptr;                     // pinned: per-level frontier totals (ring of kLvlRing)
     cudaEvent_t ev_lvl[4] = {nullptr, nullptr, nullptr, nullptr};
     uint32_t launches = 0;
@@ -220,6 +226,8 @@ struct Ctx {
     // multi-GPU kernels larger than a rank's share (root.cu root_values, dist.cu)
     void *vr_P = nullptr, *vr_work = nullptr; size_t cap_vr_P = 0, cap_vr_work = 0;
     void *gi_buf = nullptr; size_t cap_gi_buf = 0;
+    void *dn_sel = nullptr, *dn_meta = nullptr, *dn_val = nullptr;   // value path of repeated-time groups
+    size_t cap_dn_sel = 0, cap_dn_meta = 0, cap_dn_val = 0;
     void *gi_tab = nullptr, *gi_rec = nullptr, *gi_all = nullptr, *gi_val = nullptr;   // histograms, tables
     size_t cap_gi_tab = 0, cap_gi_rec = 0, cap_gi_all = 0, cap_gi_val = 0;
     const uint8_t *fixed_kernel = nullptr;                  // local kernels whose leaves are given (no ROOT)
@@ -270,6 +278,56 @@ int stem_only_leaves(Ctx &c, uint64_t n, uint32_t K);
 // ROOT over a histogram of distinct values per group (root.cu): vflag[u] = 1 where a leaf starts
 int root_values(Ctx &c, const uint32_t *vt, const uint64_t *vcnt, const uint32_t *goffv, uint32_t G, uint64_t D,
                 double eps, double z, double k2, int clamp, uint8_t *vflag);
+// One pipelined run of the value-histogram ROOT (root.cu): setup enqueues the
+// first frontier on stream s, pump advances the levels (block = false: never
+// waits), finish completes them.
+struct VrSource {
+    const uint32_t *kc = nullptr;      // [D] rows before value u
+    const uint64_t *Ps = nullptr;      // [D] sum of t before value u
+    const u128 *Pq = nullptr;          // [D] sum of t^2 before value u (histogram input; nullptr: from the rows)
+    const uint32_t *goffv = nullptr;   // [G + 1] first value of each group
+    const uint32_t *dgrp = nullptr;    // dense path: group j's kernel group (rows from goff, PS1/PS2)
+    const uint32_t *goff = nullptr;
+    uint32_t G = 0;
+};
+struct VrRun {
+    Ctx &c;
+    cudaStream_t st = nullptr;
+    uint64_t D = 0;
+    uint64_t enq = 0, done = 0;
+    bool finished = false;
+    uint32_t launches = 0, levels = 0;
+    struct VrDevStore { alignas(16) unsigned char b[256]; } devs;
+    int setup(const VrSource &src, uint64_t D, double eps, double z, double k2, int clamp, uint8_t *vflag,
+              cudaStream_t s);
+    int enqueue_one();
+    int pump(bool block);
+    int finish(uint64_t *active_rows);
+};
+// Kernel groups with many repeated times take the value path (root.cu)
+struct DensePath {
+    Ctx &c;
+    VrRun run{c};
+    bool on = false;
+    int phase = 0;                   // 1: distinct count queued, 2: levels running
+    const uint8_t *sel_ = nullptr;   // per group: 0 row path, 1 fixed leaves, 2 value path
+    uint32_t *dgrp = nullptr, *dsegf = nullptr, *goffv = nullptr, *segcnt = nullptr, *segoff = nullptr;
+    uint32_t *vpos = nullptr;
+    uint8_t *vflag = nullptr;
+    uint64_t D_ = 0;
+    uint32_t Gd = 0, NS = 0;         // dense groups, their windows (kWinRows rows, one warp each)
+    uint64_t n_ = 0;
+    unsigned grid = 0;
+    bool sync_mode = false;
+    cudaStream_t vs_ = nullptr;
+    uint64_t act_ = 0;
+    double eps_ = 0, z_ = 0, k2_ = 0;
+    int clamp_ = 0;
+    int start(uint64_t n, uint32_t K, double eps, double z, double k2, int clamp);
+    int build();
+    int pump();
+    int finish(uint32_t *flags);
+};
 // split = 3: ROOT with exact optimal 1-D k-means splits into kk groups (kmeans.cu, R29)
 int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, uint32_t kk);
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,

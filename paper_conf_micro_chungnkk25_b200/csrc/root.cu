@@ -1317,6 +1317,9 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         CK(cudaMemcpyToSymbolAsync(c_bound2, &b2, sizeof(b2), 0, cudaMemcpyHostToDevice, st));
     }
     CKS(stem_only_leaves(c, n, K));
+    // groups with many repeated times: their trees are built over values, beside the row levels
+    DensePath dense{c};
+    if (split == 0) CKS(dense.start(n, K, eps, z, k2, clamp));
     // initial frontier: non-trivial kernel groups, in kernel order, with exact S and Q
     {
         CKS(ensure_frontier(c, 0, (uint64_t)K + 1));
@@ -1327,7 +1330,8 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         uint32_t *nlo = c.f_lo[0], *nhi = c.f_hi[0];
         uint64_t *nS = c.f_S[0];
         u128 *nQ = c.f_Q[0];
-        const uint8_t *fixed = c.fixed_kernel;   // multi-GPU: kernels whose leaves were decided on the value tree
+        // skipped: kernels whose leaves are given (multi-GPU) or built on the value path
+        const uint8_t *fixed = dense.on ? dense.sel_ : c.fixed_kernel;
         if (c.fixed_cuts && c.n_fixed_cuts) {
             fixed_flags_kernel<<<(unsigned)((c.n_fixed_cuts + 255) / 256), 256, 0, st>>>(c.fixed_cuts, c.n_fixed_cuts,
                                                                                       c.goff, c.flags);
@@ -1506,6 +1510,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                 levels = level;
                 c.stats.active_rows += Aprev;
                 CKS(enqueue_level(level, cur, Cprev, Aprev));
+                CKS(dense.pump());
                 CK(cudaEventSynchronize(c.ev_lvl[level & 3]));
                 Cprev = c.h_lvl[level & 3] >> 32;
                 Aprev = c.h_lvl[level & 3] & 0xFFFFFFFFull;
@@ -1520,6 +1525,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                 c.stats.active_rows += Al;
                 // level + 1 consumes level's output: at most 2 Cl clusters, Al rows
                 CKS(enqueue_level(level + 1, level & 1, 2 * Cl, Al));
+                CKS(dense.pump());
                 CK(cudaEventSynchronize(c.ev_lvl[level & 3]));
                 Cl = c.h_lvl[level & 3] >> 32;
                 Al = c.h_lvl[level & 3] & 0xFFFFFFFFull;
@@ -1527,6 +1533,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             }
         }
     }
+    CKS(dense.finish(c.flags));
     DevScalars hs;
     CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -1544,9 +1551,21 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
 // lies between two distinct values, D_k = n S_L - S k and the Eq. 7/8 test use
 // the counts and sums below it.  So the tree of a kernel can be built from its
 // distinct values and their counts alone -- exactly the tree the row levels
-// build -- which is how the multi-GPU plan splits a kernel larger than a
-// rank's share (dist.cu): every rank builds the value tree of the merged
-// histogram, then the kernel's leaves are dealt to ranks whole.
+// build.  Two users: the single-GPU plan hands kernels with many repeated
+// times (C5's large kernels: 532 M rows, 23.5 M distinct values) to this path,
+// which scans values instead of rows; the multi-GPU plan builds the tree of a
+// kernel larger than a rank's share from the merged histogram (dist.cu).
+//
+// A value u (interior of its group) is described by kc[u], the rows before it
+// (dense path: its first row; histogram: the prefix count), Ps[u], the sum of
+// t before it, and the sum of t^2 before it (histogram: Pq[u]; dense path:
+// from the row prefix PS2 at that row, needed only at accepted cuts).  A
+// cluster carries its value range, rows, and exact S, Q (and the prefixes at
+// its start), like the row frontier.  Levels are pipelined like the row
+// levels: every kernel reads the size of the frontier it consumes from device
+// memory, the grids are persistent, and the host learns a level's output size
+// later (pinned ring + events), so the run can advance on a side stream from
+// the row loop without blocking it (VrRun::pump).
 struct VH {
     uint64_t c, s;
     u128 q;
@@ -1554,148 +1573,652 @@ struct VH {
 __host__ __device__ __forceinline__ VH operator+(const VH &a, const VH &b) { return VH{a.c + b.c, a.s + b.s, a.q + b.q}; }
 __host__ __device__ __forceinline__ VH operator-(const VH &a, const VH &b) { return VH{a.c - b.c, a.s - b.s, a.q - b.q}; }
 
-struct VrArgs {
-    const VH *P;               // [D + 1] exclusive prefix of (count, sum t, sum t^2) over the values
-    const uint32_t *vlo, *vhi; // frontier: value ranges [vlo, vhi)
-    const uint64_t *ctot;      // packed (count << 32 | values) of the frontier
-    uint32_t *cutv;            // per cluster: value index of the cut (0: none)
-    uint64_t *cutk;            // per cluster: rows left of the cut
-    uint64_t *cutSL;
+constexpr uint32_t kVrEV = 1024;                 // values per entry (one warp)
+constexpr unsigned long long kVrMask = (1ull << 40) - 1;
+constexpr int kVrRing = 8;
+
+struct VrClu {          // a frontier cluster
+    uint32_t lo, hi;    // value range [lo, hi)
+    uint32_t k0, n;     // rows before it (kc at lo), its rows
+    uint64_t s0, S;     // sum t before it, its sum
+    u128 q0, Q;         // sum t^2 before it, its sum
+    uint32_t ef, pad;   // first entry
 };
 
-// one block per cluster: the exact best cut over the cluster's distinct-value boundaries
-__global__ void __launch_bounds__(256) vroot_cut_kernel(VrArgs a) {
-    __shared__ Cand s_best[8];
-    const uint32_t C = (uint32_t)(*a.ctot >> 32);
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    for (uint32_t ci = blockIdx.x; ci < C; ci += gridDim.x) {
-        const uint32_t v0 = a.vlo[ci], v1 = a.vhi[ci];
-        const VH p0 = a.P[v0], tot = a.P[v1] - p0;
-        const uint64_t n = tot.c, S = tot.s;
+struct VrDev {
+    const uint32_t *kc;                          // [D] rows before value u
+    const uint64_t *Ps;                          // [D] sum t before value u
+    const u128 *Pq;                              // [D] sum t^2 before value u (nullptr: from the rows)
+    const uint64_t *PS1;                         // dense path: row prefixes and times
+    const u128 *PS2;
+    const uint32_t *t;
+    VrClu *clu[2];                               // frontier f
+    uint32_t *eclu, *ea, *eb;                    // entries of the level being cut
+    Cand *cand;                                  // best cut per entry
+    unsigned long long *cnt;                     // [2] (clusters << 40) | entries, per frontier
+    unsigned long long *active;                  // rows of the clusters decided (ROOT active rows)
+    uint8_t *vflag;                              // 1 at the first value of every leaf
+    double eps, z, k2;
+    int clamp;
+};
+
+static VrDev &vdev(VrRun &r) {
+    static_assert(sizeof(VrDev) <= sizeof(r.devs.b), "VrRun::devs too small");
+    return *reinterpret_cast<VrDev *>(r.devs.b);
+}
+
+__device__ __forceinline__ uint32_t vr_nent(uint32_t nv) { return (nv + kVrEV - 1) / kVrEV; }
+
+__device__ __forceinline__ u128 vr_q(const VrDev &a, uint32_t u) {
+    if (a.Pq) return a.Pq[u];
+    uint64_t s;
+    u128 q;
+    pref12(a.PS1, a.PS2, a.t, a.kc[u], s, q);
+    return q;
+}
+
+__device__ __forceinline__ void vr_push(const VrDev &a, int f, const VrClu &x) {
+    const unsigned long long p = atomicAdd(&a.cnt[f], (1ull << 40) | vr_nent(x.hi - x.lo));
+    VrClu y = x;
+    y.ef = (uint32_t)(p & kVrMask);
+    a.clu[f][p >> 40] = y;
+}
+
+// first frontier from prefix arrays over [0, D] (histogram input)
+__global__ void vr_init_hist_kernel(VrDev a, const uint32_t *goffv, uint32_t G) {
+    const uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
+    if (g >= G) return;
+    const uint32_t v0 = goffv[g], v1 = goffv[g + 1];
+    if (v1 > v0) a.vflag[v0] = 1;
+    if (v1 - v0 < 2) return;   // at least two distinct values
+    VrClu x{};
+    x.lo = v0;
+    x.hi = v1;
+    x.k0 = a.kc[v0];
+    x.n = a.kc[v1] - x.k0;
+    x.s0 = a.Ps[v0];
+    x.S = a.Ps[v1] - x.s0;
+    x.q0 = a.Pq[v0];
+    x.Q = a.Pq[v1] - x.q0;
+    vr_push(a, 0, x);
+}
+
+// first frontier of the dense groups: rows and moments from the row prefixes
+__global__ void vr_init_rows_kernel(VrDev a, const uint32_t *goffv, const uint32_t *dgrp, uint32_t G,
+                                    const uint32_t *goff) {
+    const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j >= G) return;
+    const uint32_t v0 = goffv[j], v1 = goffv[j + 1], g = dgrp[j];
+    if (v1 > v0) a.vflag[v0] = 1;
+    if (v1 - v0 < 2) return;
+    VrClu x{};
+    x.lo = v0;
+    x.hi = v1;
+    x.k0 = goff[g];
+    x.n = goff[g + 1] - goff[g];
+    uint64_t s1;
+    u128 q1;
+    pref12(a.PS1, a.PS2, a.t, goff[g], x.s0, x.q0);
+    pref12(a.PS1, a.PS2, a.t, goff[g + 1], s1, q1);
+    x.S = s1 - x.s0;
+    x.Q = q1 - x.q0;
+    vr_push(a, 0, x);
+}
+
+// one warp per cluster of frontier f: its entry records
+__global__ void vr_expand_kernel(VrDev a, int f) {
+    const uint64_t C = a.cnt[f] >> 40;
+    const int lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
+    for (uint64_t ci = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); ci < C; ci += nw) {
+        const uint32_t lo = a.clu[f][ci].lo, hi = a.clu[f][ci].hi, e0 = a.clu[f][ci].ef, ne = vr_nent(hi - lo);
+        for (uint32_t j = lane; j < ne; j += 32) {
+            a.eclu[e0 + j] = (uint32_t)ci;
+            a.ea[e0 + j] = lo + j * kVrEV;
+            a.eb[e0 + j] = min(lo + (j + 1) * kVrEV, hi);
+        }
+    }
+}
+
+// one warp per entry: the exact best cut over its distinct-value boundaries
+// u (left = values [lo, u)), eval_cut as on the row path
+__global__ void __launch_bounds__(256) vr_cut_kernel(VrDev a, int f) {
+    const uint64_t E = a.cnt[f] & kVrMask;
+    const int lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
+    for (uint64_t e = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); e < E; e += nw) {
+        const VrClu &x = a.clu[f][a.eclu[e]];
+        const uint32_t k0 = x.k0, n = x.n, ua = max(a.ea[e], x.lo + 1), ub = a.eb[e];
+        const uint64_t s0 = x.s0, S = x.S;
         Cand best = no_cand();
-        for (uint32_t u = v0 + 1 + threadIdx.x; u < v1; u += blockDim.x) {
-            const VH pu = a.P[u] - p0;
-            eval_cut((uint32_t)pu.c, n, S, pu.s, best);
+        for (uint32_t u = ua + lane; u < ub; u += 32) eval_cut(a.kc[u] - k0, n, S, a.Ps[u] - s0, best);
+#pragma unroll 1
+        for (int o = 16; o; o >>= 1) {
+            const Cand v = shfl_cand_xor(best, o);
+            if (better(v, best)) best = v;
+        }
+        if (lane == 0) a.cand[e] = best;
+    }
+}
+
+// one warp per cluster: the best of its entries, the Eq. 7/8 decision, the children
+__global__ void __launch_bounds__(256) vr_decide_kernel(VrDev a, int f) {
+    const uint64_t C = a.cnt[f] >> 40;
+    const int lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
+    for (uint64_t ci = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); ci < C; ci += nw) {
+        const VrClu x = a.clu[f][ci];
+        const uint32_t ne = vr_nent(x.hi - x.lo);
+        Cand best = no_cand();
+        for (uint32_t j = lane; j < ne; j += 32) {
+            const Cand v = a.cand[x.ef + j];
+            if (better(v, best)) best = v;
         }
 #pragma unroll 1
         for (int o = 16; o; o >>= 1) {
             const Cand v = shfl_cand_xor(best, o);
             if (better(v, best)) best = v;
         }
-        if (lane == 0) s_best[w] = best;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            Cand b = s_best[0];
-            for (int k = 1; k < 8; k++)
-                if (better(s_best[k], b)) b = s_best[k];
-            uint32_t cu = 0;
-            if (b.k) {   // the value index whose prefix count is k
-                uint32_t lo = v0 + 1, hi = v1;
-                while (lo < hi) {
-                    const uint32_t mid = lo + (hi - lo) / 2;
-                    if (a.P[mid].c - p0.c < b.k) lo = mid + 1; else hi = mid;
+        if (lane != 0) continue;
+        atomicAdd(a.active, (unsigned long long)x.n);
+        if (!best.k) continue;
+        uint32_t l = x.lo + 1, h = x.hi;   // the value index with best.k rows before it
+        while (l < h) {
+            const uint32_t mid = l + (h - l) / 2;
+            if (a.kc[mid] - x.k0 < best.k) l = mid + 1; else h = mid;
+        }
+        const uint32_t u = l;
+        const u128 QL = vr_q(a, u) - x.q0;
+        if (!split_pays(x.n, x.S, x.Q, best.k, best.SL, QL, a.eps, a.z, a.k2, a.clamp)) continue;
+        a.vflag[u] = 1;
+        if (u - x.lo >= 2) {
+            VrClu L = x;
+            L.hi = u;
+            L.n = best.k;
+            L.S = best.SL;
+            L.Q = QL;
+            vr_push(a, f ^ 1, L);
+        }
+        if (x.hi - u >= 2) {
+            VrClu R = x;
+            R.lo = u;
+            R.k0 = x.k0 + best.k;
+            R.n = x.n - best.k;
+            R.s0 = x.s0 + best.SL;
+            R.S = x.S - best.SL;
+            R.q0 = x.q0 + QL;
+            R.Q = x.Q - QL;
+            vr_push(a, f ^ 1, R);
+        }
+    }
+}
+
+size_t vr_work_bytes(uint64_t D) {
+    const uint64_t Ccap = D / 2 + 2, Ecap = Ccap + D / kVrEV + 2;
+    return 16 * 8 + 2 * sizeof(VrClu) * Ccap + sizeof(uint32_t) * 3 * Ecap + sizeof(Cand) * Ecap + 512;
+}
+
+// Lays out one run in c.vr_work (sized by the caller with vr_work_bytes(D)).
+int VrRun::setup(const VrSource &src, uint64_t Dv, double eps, double z, double k2, int clamp, uint8_t *vflag,
+                 cudaStream_t s) {
+    st = s;
+    D = Dv;
+    enq = done = 0;
+    finished = false;
+    const uint64_t Ccap = D / 2 + 2, Ecap = Ccap + D / kVrEV + 2;
+    VrDev d{};
+    d.kc = src.kc;
+    d.Ps = src.Ps;
+    d.Pq = src.Pq;
+    d.PS1 = c.PS1;
+    d.PS2 = c.PS2;
+    d.t = c.t_sorted;
+    char *w = (char *)c.vr_work;
+    auto take = [&](size_t bytes) {
+        char *p = w;
+        w += (bytes + 15) & ~(size_t)15;
+        return (void *)p;
+    };
+    d.cnt = (unsigned long long *)take(16 * 8);
+    d.active = d.cnt + 2;
+    for (int f = 0; f < 2; f++) d.clu[f] = (VrClu *)take(sizeof(VrClu) * Ccap);
+    d.eclu = (uint32_t *)take(sizeof(uint32_t) * Ecap);
+    d.ea = (uint32_t *)take(sizeof(uint32_t) * Ecap);
+    d.eb = (uint32_t *)take(sizeof(uint32_t) * Ecap);
+    d.cand = (Cand *)take(sizeof(Cand) * Ecap);
+    d.vflag = vflag;
+    d.eps = eps;
+    d.z = z;
+    d.k2 = k2;
+    d.clamp = clamp;
+    vdev(*this) = d;
+    if (!c.h_vr) {
+        CK(cudaMallocHost((void **)&c.h_vr, sizeof(uint64_t) * (kVrRing + 1)));
+        for (int i = 0; i < kVrRing; i++) CK(cudaEventCreateWithFlags(&c.ev_vr[i], cudaEventDisableTiming));
+    }
+    CK(cudaMemsetAsync(d.cnt, 0, 16 * 8, st));
+    CK(cudaMemsetAsync(vflag, 0, D + 1, st));
+    if (src.G) {
+        if (src.dgrp)
+            vr_init_rows_kernel<<<(src.G + 255) / 256, 256, 0, st>>>(d, src.goffv, src.dgrp, src.G, src.goff);
+        else
+            vr_init_hist_kernel<<<(src.G + 255) / 256, 256, 0, st>>>(d, src.goffv, src.G);
+        launches++;
+    }
+    CK(cudaGetLastError());
+    return STEM_OK;
+}
+
+int VrRun::enqueue_one() {
+    const int f = (int)(enq & 1);
+    const unsigned g = (unsigned)c.sms * 8;
+    const VrDev &dev = vdev(*this);
+    vr_expand_kernel<<<g, 256, 0, st>>>(dev, f);
+    vr_cut_kernel<<<g, 256, 0, st>>>(dev, f);
+    CK(cudaMemsetAsync(&dev.cnt[f ^ 1], 0, sizeof(unsigned long long), st));
+    vr_decide_kernel<<<g, 256, 0, st>>>(dev, f);
+    launches += 3;
+    const int r = (int)(enq % kVrRing);
+    CK(cudaMemcpyAsync(&c.h_vr[r], &dev.cnt[f ^ 1], sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaEventRecord(c.ev_vr[r], st));
+    CK(cudaGetLastError());
+    enq++;
+    return STEM_OK;
+}
+
+// Advances the run: reads finished levels, keeps up to 3 levels queued.
+// block = false never waits on the GPU (called from the row loop).
+int VrRun::pump(bool block) {
+    while (!finished) {
+        while (done < enq) {
+            const int r = (int)(done % kVrRing);
+            if (block) {
+                CK(cudaEventSynchronize(c.ev_vr[r]));
+            } else {
+                const cudaError_t q = cudaEventQuery(c.ev_vr[r]);
+                if (q == cudaErrorNotReady) {
+                    (void)cudaGetLastError();
+                    break;
                 }
-                cu = lo;
+                CK(q);
             }
-            a.cutv[ci] = cu;
-            a.cutk[ci] = b.k;
-            a.cutSL[ci] = b.SL;
+            done++;
+            if ((c.h_vr[r] >> 40) == 0) {   // no cluster left: the levels queued after it are empty
+                finished = true;
+                break;
+            }
         }
-        __syncthreads();
+        if (finished) break;
+        if (enq - done < 3) CKS(enqueue_one());
+        else if (!block) break;
     }
+    return STEM_OK;
 }
 
-struct VdArgs {
-    const VH *P;
-    const uint32_t *vlo, *vhi;
-    const uint64_t *ctot;
-    const uint32_t *cutv;
-    const uint64_t *cutk, *cutSL;
-    uint8_t *vflag;            // 1 at the first value of every leaf
-    uint32_t *nlo, *nhi;
-    uint64_t *total;
-    double eps, z, k2;
-    int clamp;
-};
-
-__global__ void vroot_decide_kernel(VdArgs a) {
-    const uint64_t ci = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (ci >= (*a.ctot >> 32)) return;
-    const uint32_t v0 = a.vlo[ci], v1 = a.vhi[ci], u = a.cutv[ci];
-    if (!u) return;
-    const VH p0 = a.P[v0], tot = a.P[v1] - p0, left = a.P[u] - p0;
-    if (!split_pays(tot.c, tot.s, tot.q, a.cutk[ci], a.cutSL[ci], left.q, a.eps, a.z, a.k2, a.clamp)) return;
-    a.vflag[u] = 1;
-    const uint32_t kids[2][2] = {{v0, u}, {u, v1}};
-    for (int h = 0; h < 2; h++)
-        if (kids[h][1] - kids[h][0] >= 2) {   // at least two distinct values
-            const uint64_t slot = atomicAdd((unsigned long long *)a.total,
-                                            (unsigned long long)((1ull << 32) | (kids[h][1] - kids[h][0]))) >> 32;
-            a.nlo[slot] = kids[h][0];
-            a.nhi[slot] = kids[h][1];
-        }
-}
-
-__global__ void vroot_init_kernel(const uint32_t *goffv, uint32_t G, uint8_t *vflag, uint32_t *nlo, uint32_t *nhi,
-                                  uint64_t *total) {
-    const uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
-    if (g >= G) return;
-    const uint32_t v0 = goffv[g], v1 = goffv[g + 1];
-    if (v1 > v0) vflag[v0] = 1;
-    if (v1 - v0 >= 2) {
-        const uint64_t slot = atomicAdd((unsigned long long *)total, (unsigned long long)((1ull << 32) | (v1 - v0))) >> 32;
-        nlo[slot] = v0;
-        nhi[slot] = v1;
-    }
+int VrRun::finish(uint64_t *active_rows) {
+    CKS(pump(true));
+    uint64_t act = 0;
+    CK(cudaMemcpyAsync(&act, vdev(*this).active, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (active_rows) *active_rows = act;
+    levels = (uint32_t)done;
+    return STEM_OK;
 }
 
 int root_values(Ctx &c, const uint32_t *vt, const uint64_t *vcnt, const uint32_t *goffv, uint32_t G, uint64_t D,
                 double eps, double z, double k2, int clamp, uint8_t *vflag) {
     cudaStream_t st = c.stream;
-    CKS(c.ensure(c.vr_P, c.cap_vr_P, sizeof(VH) * (D + 2)));
-    CKS(c.ensure(c.vr_work, c.cap_vr_work, (sizeof(uint32_t) * 5 + sizeof(uint64_t) * 2) * (D + 3) + 8));
-    CKS(c.ensure(c.scan_scratch, c.cap_scan, (scan_tiles(D + 1) + 1) * sizeof(VH)));
-    VH *P = (VH *)c.vr_P;
-    {
-        exclusive_scan<VH>(
-            [vt, vcnt, D] __device__(uint64_t i) -> VH {
-                if (i >= D) return VH{0, 0, 0};
-                const uint64_t cn = vcnt[i], tv = vt[i];
-                return VH{cn, cn * tv, (u128)cn * ((u128)tv * tv)};
-            },
-            [P] __device__(uint64_t i, VH pre, VH) { P[i] = pre; }, D + 1, (VH *)c.scan_scratch,
-            (VH *)c.scalars->wide_total, st, &c.launches);
+    // prefix arrays over the values (D + 1 entries: the last is the total)
+    CKS(c.ensure(c.vr_P, c.cap_vr_P, (sizeof(uint32_t) + sizeof(uint64_t) + sizeof(u128)) * (D + 2) + 64 +
+                                     (scan_tiles(D + 1) + 2) * sizeof(VH)));
+    u128 *Pq = (u128 *)c.vr_P;
+    uint64_t *Ps = (uint64_t *)(Pq + (D + 2));
+    uint32_t *Pc = (uint32_t *)(Ps + (D + 2));
+    VH *scratch = (VH *)(((uintptr_t)(Pc + (D + 2)) + 63) & ~(uintptr_t)63);
+    CKS(c.ensure(c.vr_work, c.cap_vr_work, vr_work_bytes(D)));
+    exclusive_scan<VH>(
+        [vt, vcnt, D] __device__(uint64_t u) -> VH {
+            if (u >= D) return VH{0, 0, 0};
+            const uint64_t cn = vcnt[u], tv = vt[u];
+            return VH{cn, cn * tv, (u128)cn * ((u128)tv * tv)};
+        },
+        [Pc, Ps, Pq] __device__(uint64_t u, VH pre, VH) {
+            Pc[u] = (uint32_t)pre.c;
+            Ps[u] = pre.s;
+            Pq[u] = pre.q;
+        },
+        D + 1, scratch, (VH *)c.scalars->wide_total, st, &c.launches);
+    VrRun run{c};
+    VrSource src{};
+    src.kc = Pc;
+    src.Ps = Ps;
+    src.Pq = Pq;
+    src.goffv = goffv;
+    src.G = G;
+    CKS(run.setup(src, D, eps, z, k2, clamp, vflag, st));
+    CKS(run.finish(nullptr));
+    c.launches += run.launches;
+    return STEM_OK;
+}
+
+// ---------------------------------------------------------------- kernels with many repeated times
+// A kernel group of >= STEMROOT_VALUE_ROWS rows (default 2^18; 0 = off) whose
+// times repeat (a 1024-point sample finds t[i] == t[i-1] at >= 1 - 1/R of the
+// points, R = STEMROOT_VALUE_RATIO, default 4) is handed to the value path:
+// its distinct values are listed once (first row, sum of t before it), its
+// tree is built by VrRun on a side stream while the row levels handle the
+// other groups, and its leaf starts are set in the row flags.  The tree is the
+// one the row levels would build (same cuts, same decisions), so this only
+// changes the cost: C5's 79 largest kernels hold 53 % of the rows but 2.4 % of
+// the distinct values.
+constexpr uint32_t kWinRows = 2048;   // one warp's window of a dense group (64 aligned 32-row chunks)
+
+static uint32_t value_rows() {   // read per plan (tests switch it)
+    const char *e = getenv("STEMROOT_VALUE_ROWS");
+    const long v = e ? atol(e) : (1l << 18);
+    return v < 0 ? 0u : (uint32_t)v;
+}
+
+static uint32_t value_ratio() {
+    const char *e = getenv("STEMROOT_VALUE_RATIO");
+    const long v = e ? atol(e) : 4;
+    return v < 2 ? 2u : (uint32_t)v;
+}
+
+// one warp per group: sel[g] = 1 fixed (given leaves), 2 dense, 0 row path
+__global__ void dense_select_kernel(const uint32_t *goff, const uint32_t *t, uint32_t K, const uint8_t *fixed,
+                                    uint32_t min_rows, uint32_t ratio, uint8_t *sel, unsigned long long *acc) {
+    const uint32_t g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (g >= K) return;
+    const uint32_t lo = goff[g], n = goff[g + 1] - lo;
+    uint8_t v = fixed && fixed[g] ? 1 : 0;
+    if (!v && min_rows && n >= min_rows && n >= 2) {
+        uint32_t rep = 0;
+        for (uint32_t j = lane; j < 1024; j += 32) {
+            const uint32_t i = lo + 1 + (uint32_t)(((uint64_t)j * (n - 1)) >> 10);
+            rep += t[i] == t[i - 1];
+        }
+        for (int o = 16; o; o >>= 1) rep += __shfl_xor_sync(0xffffffffu, rep, o);
+        if ((uint64_t)rep * ratio >= 1024ull * (ratio - 1)) v = 2;
     }
-    uint32_t *w32 = (uint32_t *)c.vr_work;
-    const uint64_t D2 = (D + 2 + 1) & ~1ull;   // even: the u64 arrays after the u32 ones stay aligned
-    uint32_t *lo[2] = {w32, w32 + D2}, *hi[2] = {w32 + 2 * D2, w32 + 3 * D2};
-    uint32_t *cutv = w32 + 4 * D2;
-    uint64_t *cutk = (uint64_t *)(w32 + 5 * D2 + (5 * D2 & 1)), *cutSL = cutk + D2;
-    CK(cudaMemsetAsync(vflag, 0, D + 1, st));
-    CK(cudaMemsetAsync(&c.scalars->ftot[0], 0, 2 * sizeof(uint64_t), st));
-    if (G) {
-        vroot_init_kernel<<<(G + 255) / 256, 256, 0, st>>>(goffv, G, vflag, lo[0], hi[0], &c.scalars->ftot[0]);
-        c.launches++;
+    if (lane == 0) {
+        sel[g] = v;
+        if (v == 2) {
+            atomicAdd(&acc[0], 1ull);
+            atomicAdd(&acc[1], (unsigned long long)((n + (lo & 31u) + kWinRows - 1) / kWinRows));
+        }
     }
-    uint64_t tot = 0;
-    CK(cudaMemcpyAsync(&tot, &c.scalars->ftot[0], sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+}
+
+struct DenseWin {   // window w of the dense groups -> group rows [glo, ghi), window rows [a, b), a 32-aligned
+    const uint32_t *dgrp, *dwinf, *goff;
+    uint32_t Gd;
+    __device__ void operator()(uint32_t w, uint32_t &glo, uint32_t &ghi, uint32_t &a, uint32_t &b) const {
+        const uint32_t j = (uint32_t)upper_bound(dwinf, (uint64_t)Gd + 1, w) - 1, g = dgrp[j];
+        glo = goff[g];
+        ghi = goff[g + 1];
+        a = (glo & ~31u) + (w - dwinf[j]) * kWinRows;
+        b = min(a + kWinRows, ghi);
+    }
+};
+
+// Value starts among the rows [c, c + 128) of a window, 4 per lane (c is
+// 32-aligned, so the uint4 loads are aligned; t_sorted has 4 rows of slack):
+// bit r of the result = row c + 4 lane + r starts a value of the group.
+// v = the 4 times (0 where the lane's first row is at or after b).
+__device__ __forceinline__ uint32_t win_starts4(const uint32_t *t, uint32_t c, uint32_t glo, uint32_t b, uint4 &v) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t i0 = c + 4 * lane;
+    v = i0 < b ? *reinterpret_cast<const uint4 *>(t + i0) : make_uint4(0, 0, 0, 0);
+    uint32_t prev = __shfl_up_sync(0xffffffffu, v.w, 1);
+    if (lane == 0) prev = c > glo ? t[c - 1] : 0u;
+    const uint32_t e[4] = {v.x, v.y, v.z, v.w};
+    uint32_t f = 0;
+#pragma unroll
+    for (int r = 0; r < 4; r++) {
+        const uint32_t i = i0 + r;
+        const uint32_t p = r ? e[r - 1] : prev;
+        if (i >= glo && i < b && (i == glo || e[r] != p)) f |= 1u << r;
+    }
+    return f;
+}
+
+// one warp per window: distinct values (value starts) in it
+__global__ void __launch_bounds__(256) dense_count_kernel(DenseWin dw, const uint32_t *t, uint32_t NW,
+                                                          uint32_t *wcnt) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t nw = gridDim.x * (blockDim.x >> 5);
+    for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < NW; w += nw) {
+        uint32_t glo, ghi, a, b;
+        dw(w, glo, ghi, a, b);
+        uint32_t cnt = 0;
+#pragma unroll 4
+        for (uint32_t c = a; c < b; c += 128) {
+            uint4 v;
+            cnt += __popc(win_starts4(t, c, glo, b, v));
+        }
+        for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+        if (lane == 0) wcnt[w] = cnt;
+    }
+}
+
+// one warp per window: the value list in row order, vpos[u] = first row of
+// value u, Ps[u] = sum of t before it (PS1 at the 32-row chunk c + a warp scan)
+__global__ void __launch_bounds__(256) dense_write_kernel(DenseWin dw, const uint32_t *t, const uint64_t *PS1,
+                                                          uint32_t NW, const uint32_t *woff, uint32_t *vpos,
+                                                          uint64_t *Ps) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t nw = gridDim.x * (blockDim.x >> 5);
+    for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < NW; w += nw) {
+        uint32_t glo, ghi, a, b;
+        dw(w, glo, ghi, a, b);
+        uint32_t off = woff[w];
+#pragma unroll 2
+        for (uint32_t c = a; c < b; c += 128) {
+            uint4 v;
+            const uint32_t f = win_starts4(t, c, glo, b, v);
+            const uint32_t nf = __popc(f);
+            if (!__any_sync(0xffffffffu, nf != 0)) continue;
+            // Ps: rows of [c, c + 128) before i, whatever their group (PS1 is the global prefix;
+            // v holds every row below b, and rows at or after b follow every start)
+            const uint32_t i0 = c + 4 * lane;
+            const uint4 x = v;
+            const uint64_t lsum = (uint64_t)x.x + x.y + x.z + x.w;
+            const uint64_t lexcl = warp_incl_scan(lsum) - lsum;
+            const uint32_t cexcl = warp_incl_scan(nf) - nf;
+            if (f) {
+                const uint64_t base = PS1[c >> kChunkLog] + lexcl;
+                const uint32_t e[4] = {x.x, x.y, x.z, x.w};
+                uint64_t run = 0;
+                uint32_t k = off + cexcl;
+#pragma unroll
+                for (int r = 0; r < 4; r++) {
+                    if ((f >> r) & 1u) {
+                        vpos[k] = i0 + r;
+                        Ps[k] = base + run;
+                        k++;
+                    }
+                    run += e[r];
+                }
+            }
+            off += __shfl_sync(0xffffffffu, cexcl + nf, 31);
+        }
+    }
+}
+
+__global__ void dense_goffv_kernel(const uint32_t *segoff, const uint32_t *dsegf, uint32_t Gd, uint32_t NS,
+                                   uint32_t D, uint32_t *goffv) {
+    const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j <= Gd) goffv[j] = dsegf[j] < NS ? segoff[dsegf[j]] : D;
+}
+
+__global__ void fill_kernel_u32(uint32_t *p, uint32_t n, uint32_t v) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) p[i] = v;
+}
+
+__global__ void dense_flags_kernel(const uint8_t *vflag, const uint32_t *vpos, uint64_t D, uint32_t *flags) {
+    const uint64_t u = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (u < D && vflag[u]) atomicOr(&flags[vpos[u] >> 5], 1u << (vpos[u] & 31));
+}
+
+// Selects the dense groups (main stream, one small round trip) and queues the
+// count of their distinct values on c.vside; the rest follows from pump().
+int DensePath::start(uint64_t n, uint32_t K, double eps, double z, double k2, int clamp) {
+    on = false;
+    n_ = n;
+    phase = 0;
+    eps_ = eps;
+    z_ = z;
+    k2_ = k2;
+    clamp_ = clamp;
+    if (!value_rows() || K == 0) return STEM_OK;
+    cudaStream_t st = c.stream;
+    CKS(c.ensure(c.dn_sel, c.cap_dn_sel, (uint64_t)K + 16 * 8));
+    uint8_t *sel = (uint8_t *)c.dn_sel;
+    unsigned long long *acc = (unsigned long long *)(sel + (((uint64_t)K + 15) & ~15ull));
+    CK(cudaMemsetAsync(acc, 0, 16, st));
+    dense_select_kernel<<<(unsigned)((K + 7) / 8), 256, 0, st>>>(c.goff, c.t_sorted, K, c.fixed_kernel, value_rows(),
+                                                                 value_ratio(), sel, acc);
+    c.launches++;
+    unsigned long long h[2];
+    CK(cudaMemcpyAsync(h, acc, sizeof(h), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
-    int cur = 0;
-    while (tot >> 32) {
-        const uint64_t C = tot >> 32;
-        const int nxt = cur ^ 1;
-        VrArgs va{P, lo[cur], hi[cur], &c.scalars->ftot[cur], cutv, cutk, cutSL};
-        vroot_cut_kernel<<<(unsigned)min(C, (uint64_t)c.sms * 8), 256, 0, st>>>(va);
-        CK(cudaMemsetAsync(&c.scalars->ftot[nxt], 0, sizeof(uint64_t), st));
-        VdArgs vd{P, lo[cur], hi[cur], &c.scalars->ftot[cur], cutv, cutk, cutSL, vflag, lo[nxt], hi[nxt],
-                  &c.scalars->ftot[nxt], eps, z, k2, clamp};
-        vroot_decide_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(vd);
-        c.launches += 2;
-        CK(cudaGetLastError());
-        CK(cudaMemcpyAsync(&tot, &c.scalars->ftot[nxt], sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        cur = nxt;
+    if (h[0] == 0) return STEM_OK;
+    Gd = (uint32_t)h[0];
+    NS = (uint32_t)h[1];
+    CKS(c.ensure(c.dn_meta, c.cap_dn_meta, sizeof(uint32_t) * (3 * (Gd + 2) + 2 * (NS + 2)) + 64 +
+                                           (scan_tiles((uint64_t)K + NS + 2) + 2) * sizeof(uint64_t)));
+    dgrp = (uint32_t *)c.dn_meta;
+    dsegf = dgrp + (Gd + 2);
+    goffv = dsegf + (Gd + 2);
+    segcnt = goffv + (Gd + 2);
+    segoff = segcnt + (NS + 2);
+    uint64_t *scr = (uint64_t *)(((uintptr_t)(segoff + NS + 2) + 63) & ~(uintptr_t)63);
+    if (!c.vside) {
+        CK(cudaStreamCreateWithFlags(&c.vside, cudaStreamNonBlocking));
+        CK(cudaEventCreateWithFlags(&c.ev_vfork, cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&c.ev_vjoin, cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&c.ev_vcount, cudaEventDisableTiming));
+        CK(cudaMallocHost((void **)&c.h_vcount, sizeof(uint64_t) * 2));
     }
+    // STEMROOT_VALUE_SYNC=1: the whole value path on the main stream, before the row levels (a timed stage)
+    sync_mode = getenv("STEMROOT_VALUE_SYNC") && getenv("STEMROOT_VALUE_SYNC")[0] == '1';
+    vs_ = sync_mode ? st : c.vside;
+    cudaStream_t vs = vs_;
+    const int tk = sync_mode ? c.stage_begin("root_value") : -1;
+    if (!sync_mode) {
+        CK(cudaEventRecord(c.ev_vfork, st));
+        CK(cudaStreamWaitEvent(vs, c.ev_vfork, 0));
+    }
+    unsigned long long *tot = acc + 2;
+    const uint32_t *goff = c.goff;
+    uint32_t *dg = dgrp, *ds = dsegf;
+    exclusive_scan<uint64_t>(
+        [sel, goff] __device__(uint64_t g) -> uint64_t {
+            return sel[g] == 2 ? ((1ull << 32) | ((goff[g + 1] - goff[g] + (goff[g] & 31u) + kWinRows - 1) / kWinRows))
+                               : 0ull;
+        },
+        [dg, ds] __device__(uint64_t g, uint64_t pre, uint64_t v) {
+            if (v) {
+                dg[pre >> 32] = (uint32_t)g;
+                ds[pre >> 32] = (uint32_t)pre;
+            }
+        },
+        K, scr, (uint64_t *)tot, vs, &c.launches);
+    const uint32_t ns = NS;
+    uint32_t *dsend = dsegf + Gd;
+    fill_kernel_u32<<<1, 32, 0, vs>>>(dsend, 1, ns);
+    const DenseWin dw{dgrp, dsegf, goff, Gd};
+    grid = (unsigned)min((uint64_t)(NS + 7) / 8, (uint64_t)c.sms * 8);
+    dense_count_kernel<<<grid, 256, 0, vs>>>(dw, c.t_sorted, NS, segcnt);
+    uint32_t *sc = segcnt, *so = segoff;
+    exclusive_scan<uint64_t>([sc] __device__(uint64_t s) -> uint64_t { return sc[s]; },
+                             [so] __device__(uint64_t s, uint64_t pre, uint64_t) { so[s] = (uint32_t)pre; },
+                             NS, scr, (uint64_t *)tot, vs, &c.launches);
+    CK(cudaMemcpyAsync(c.h_vcount, tot, sizeof(uint64_t), cudaMemcpyDeviceToHost, vs));
+    CK(cudaEventRecord(c.ev_vcount, vs));
+    c.launches += 2;
+    CK(cudaGetLastError());
+    sel_ = sel;
+    on = true;
+    phase = 1;
+    if (sync_mode) {
+        CK(cudaEventSynchronize(c.ev_vcount));
+        CKS(build());
+        uint64_t act = 0;
+        CKS(run.finish(&act));
+        act_ = act;
+        c.stage_end(tk, 12 * act);
+    }
+    return STEM_OK;
+}
+
+// phase 1 -> 2: the distinct count is known: buffers, the value list, the first frontier
+int DensePath::build() {
+    const uint64_t D = *c.h_vcount;
+    D_ = D;
+    // growing a buffer frees the old one (an implicit device synchronisation): rare, sizes persist per ctx
+    CKS(c.ensure(c.dn_val, c.cap_dn_val, (sizeof(uint32_t) + sizeof(uint64_t) + 1) * (D + 4) + 64));
+    vpos = (uint32_t *)c.dn_val;
+    uint64_t *Ps = (uint64_t *)(((uintptr_t)(vpos + D + 4) + 15) & ~(uintptr_t)15);
+    vflag = (uint8_t *)(Ps + D + 4);
+    CKS(c.ensure(c.vr_work, c.cap_vr_work, vr_work_bytes(D)));
+    cudaStream_t vs = vs_;
+    dense_goffv_kernel<<<(Gd + 256) / 256, 256, 0, vs>>>(segoff, dsegf, Gd, NS, (uint32_t)D, goffv);
+    const DenseWin dw{dgrp, dsegf, c.goff, Gd};
+    dense_write_kernel<<<grid, 256, 0, vs>>>(dw, c.t_sorted, c.PS1, NS, segoff, vpos, Ps);
+    c.launches += 2;
+    CK(cudaGetLastError());
+    VrSource src{};
+    src.kc = vpos;
+    src.Ps = Ps;
+    src.goffv = goffv;
+    src.dgrp = dgrp;
+    src.goff = c.goff;
+    src.G = Gd;
+    CKS(run.setup(src, D, eps_, z_, k2_, clamp_, vflag, vs));
+    phase = 2;
+    return STEM_OK;
+}
+
+int DensePath::pump() {
+    if (!on || sync_mode) return STEM_OK;
+    if (phase == 1) {
+        const cudaError_t q = cudaEventQuery(c.ev_vcount);
+        if (q == cudaErrorNotReady) {
+            (void)cudaGetLastError();
+            return STEM_OK;
+        }
+        CK(q);
+        CKS(build());
+    }
+    return run.pump(false);
+}
+
+// Completes the value tree, sets its leaf starts in the row flags and joins the streams.
+int DensePath::finish(uint32_t *flags) {
+    if (!on) return STEM_OK;
+    if (phase == 1) {
+        CK(cudaEventSynchronize(c.ev_vcount));
+        CKS(build());
+    }
+    uint64_t act = act_;
+    if (!sync_mode) CKS(run.finish(&act));
+    cudaStream_t vs = vs_;
+    if (D_) dense_flags_kernel<<<(unsigned)((D_ + 255) / 256), 256, 0, vs>>>(vflag, vpos, D_, flags);
+    c.launches += 1 + run.launches;
+    if (!sync_mode) {
+        CK(cudaEventRecord(c.ev_vjoin, vs));
+        CK(cudaStreamWaitEvent(c.stream, c.ev_vjoin, 0));
+    }
+    CK(cudaGetLastError());
+    c.stats.active_rows += act;
+    c.stats.value_groups += Gd;
+    c.stats.value_count += D_;
+    if (run.levels > c.stats.value_levels) c.stats.value_levels = run.levels;
+    on = false;
     return STEM_OK;
 }
 

@@ -575,3 +575,68 @@ def test_kmeans_option_matrix(ctx, opts):
     kw.setdefault("eps", 0.02)
     got, ref = _both(ctx, kid, t, 6, seed=5, split=3, kmeans_k=3, **kw)
     assert_plans_equal(got, ref)
+
+
+# ------------------------------------------------------------------ value-histogram ROOT (root.cu DensePath, VrRun)
+def _value_case(case, seed):
+    rng = np.random.default_rng(seed)
+    if case == "dup_heavy":
+        return _dup_heavy(400_000, 37, seed) + (37,)
+    K = 23
+    kid, t = _mixture(rng, 300_001, K, peaks=4, spread=0.3, max_t=2 ** 22)
+    if case == "quantised":     # microsecond timer: long runs of equal times
+        t = (t // 1000 * 1000 + 1000).astype(np.uint32)
+    elif case == "mixed":       # even kernels quantised, odd ones continuous
+        q = kid % 2 == 0
+        t[q] = t[q] // 5000 * 5000 + 7
+    elif case == "two_values":  # one kernel of two times and an outlier, the rest continuous
+        t[kid == 0] = np.where(rng.random(int((kid == 0).sum())) < 0.6, 4000, 4001)
+        t[np.flatnonzero(kid == 0)[:1]] = 900_000
+    return kid, t.astype(np.uint32), K
+
+
+@pytest.mark.parametrize("min_rows", ["64", "4096", "0"])
+@pytest.mark.parametrize("case", ["dup_heavy", "quantised", "mixed", "two_values"])
+def test_value_path_matches_oracle(ctx, monkeypatch, min_rows, case):
+    """Groups whose times repeat take the value-histogram ROOT (their tree built
+    over distinct values on a side stream, beside the row levels);
+    STEMROOT_VALUE_ROWS is the group size from which a group is tested, 0 turns
+    the path off.  The plan equals the oracle's either way."""
+    kid, t, K = _value_case(case, 3)
+    monkeypatch.setenv("STEMROOT_VALUE_ROWS", min_rows)
+    got, ref = _both(ctx, kid, t, K, eps=0.01, seed=6)
+    assert_plans_equal(got, ref)
+    st = ctx.stats()
+    if min_rows == "0":
+        assert st["value_groups"] == 0 and st["value_levels"] == 0
+    elif case in ("dup_heavy", "quantised"):
+        assert st["value_groups"] > 0 and 0 < st["value_count"] < len(t) // 4
+        assert st["value_levels"] > 0
+
+
+@pytest.mark.parametrize("ratio", ["2", "64"])
+@pytest.mark.parametrize("opts", [dict(), dict(scope=2), dict(census_cap=True, eps=0.002), dict(clamp_in_split=False)])
+def test_value_path_options(ctx, monkeypatch, ratio, opts):
+    kid, t, K = _value_case("mixed", 9)
+    monkeypatch.setenv("STEMROOT_VALUE_ROWS", "256")
+    monkeypatch.setenv("STEMROOT_VALUE_RATIO", ratio)
+    kw = dict(seed=2)
+    kw.update(opts)
+    eps = kw.pop("eps", 0.02)
+    got, ref = _both(ctx, kid, t, K, eps=eps, **kw)
+    assert_plans_equal(got, ref)
+
+
+def test_value_path_active_rows_and_levels(ctx, monkeypatch):
+    """the value path reports the same ROOT work as the row levels: the rows of
+    every cluster it decides (active_rows) and the tree depth"""
+    kid, t, K = _value_case("quantised", 4)
+    monkeypatch.setenv("STEMROOT_VALUE_ROWS", "0")
+    ctx.plan(_dev(kid), _dev(t), K, eps=0.01, z=Z95, seed=1)
+    rows_path = ctx.stats()
+    monkeypatch.setenv("STEMROOT_VALUE_ROWS", "64")
+    ctx.plan(_dev(kid), _dev(t), K, eps=0.01, z=Z95, seed=1)
+    val_path = ctx.stats()
+    assert val_path["value_groups"] > 0
+    assert val_path["active_rows"] == rows_path["active_rows"]
+    assert max(val_path["levels"], val_path["value_levels"]) == rows_path["levels"]
