@@ -1691,7 +1691,19 @@ __global__ void __launch_bounds__(256) vr_cut_kernel(VrDev a, int f) {
         const uint32_t k0 = x.k0, n = x.n, ua = max(a.ea[e], x.lo + 1), ub = a.eb[e];
         const uint64_t s0 = x.s0, S = x.S;
         Cand best = no_cand();
-        for (uint32_t u = ua + lane; u < ub; u += 32) eval_cut(a.kc[u] - k0, n, S, a.Ps[u] - s0, best);
+        for (uint32_t b0 = ua; b0 < ub; b0 += 8 * 32) {   // 8 loads in flight per lane, then the scores
+            uint32_t kk[8];
+            uint64_t ss[8];
+#pragma unroll
+            for (int q = 0; q < 8; q++) {
+                const uint32_t u = b0 + lane + 32 * q;
+                kk[q] = u < ub ? a.kc[u] : 0u;
+                ss[q] = u < ub ? a.Ps[u] : 0ull;
+            }
+#pragma unroll 1
+            for (int q = 0; q < 8; q++)
+                if (b0 + lane + 32 * q < ub) eval_cut(kk[q] - k0, n, S, ss[q] - s0, best);
+        }
 #pragma unroll 1
         for (int o = 16; o; o >>= 1) {
             const Cand v = shfl_cand_xor(best, o);
@@ -1967,12 +1979,11 @@ struct DenseWin {   // window w of the dense groups -> group rows [glo, ghi), wi
 // 32-aligned, so the uint4 loads are aligned; t_sorted has 4 rows of slack):
 // bit r of the result = row c + 4 lane + r starts a value of the group.
 // v = the 4 times (0 where the lane's first row is at or after b).
-__device__ __forceinline__ uint32_t win_starts4(const uint32_t *t, uint32_t c, uint32_t glo, uint32_t b, uint4 &v) {
+__device__ __forceinline__ uint32_t win_starts4(uint4 v, uint32_t c, uint32_t glo, uint32_t b, uint32_t tprev) {
     const int lane = threadIdx.x & 31;
     const uint32_t i0 = c + 4 * lane;
-    v = i0 < b ? *reinterpret_cast<const uint4 *>(t + i0) : make_uint4(0, 0, 0, 0);
     uint32_t prev = __shfl_up_sync(0xffffffffu, v.w, 1);
-    if (lane == 0) prev = c > glo ? t[c - 1] : 0u;
+    if (lane == 0) prev = tprev;   // t[c - 1] (any value when c <= glo)
     const uint32_t e[4] = {v.x, v.y, v.z, v.w};
     uint32_t f = 0;
 #pragma unroll
@@ -1984,6 +1995,11 @@ __device__ __forceinline__ uint32_t win_starts4(const uint32_t *t, uint32_t c, u
     return f;
 }
 
+__device__ __forceinline__ uint4 win_load(const uint32_t *t, uint32_t c, uint32_t b) {
+    const uint32_t i0 = c + 4 * (threadIdx.x & 31);
+    return i0 < b ? *reinterpret_cast<const uint4 *>(t + i0) : make_uint4(0, 0, 0, 0);
+}
+
 // one warp per window: distinct values (value starts) in it
 __global__ void __launch_bounds__(256) dense_count_kernel(DenseWin dw, const uint32_t *t, uint32_t NW,
                                                           uint32_t *wcnt) {
@@ -1993,10 +2009,13 @@ __global__ void __launch_bounds__(256) dense_count_kernel(DenseWin dw, const uin
         uint32_t glo, ghi, a, b;
         dw(w, glo, ghi, a, b);
         uint32_t cnt = 0;
-#pragma unroll 4
+        uint32_t tprev = a > glo ? t[a - 1] : 0u;
+        uint4 v = win_load(t, a, b);
         for (uint32_t c = a; c < b; c += 128) {
-            uint4 v;
-            cnt += __popc(win_starts4(t, c, glo, b, v));
+            const uint4 vn = c + 128 < b ? win_load(t, c + 128, b) : make_uint4(0, 0, 0, 0);   // next, in flight
+            cnt += __popc(win_starts4(v, c, glo, b, tprev));
+            tprev = __shfl_sync(0xffffffffu, v.w, 31);
+            v = vn;
         }
         for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
         if (lane == 0) wcnt[w] = cnt;
@@ -2014,16 +2033,20 @@ __global__ void __launch_bounds__(256) dense_write_kernel(DenseWin dw, const uin
         uint32_t glo, ghi, a, b;
         dw(w, glo, ghi, a, b);
         uint32_t off = woff[w];
-#pragma unroll 2
+        uint32_t tprev = a > glo ? t[a - 1] : 0u;
+        uint4 v = win_load(t, a, b);
         for (uint32_t c = a; c < b; c += 128) {
-            uint4 v;
-            const uint32_t f = win_starts4(t, c, glo, b, v);
+            const uint4 vn = c + 128 < b ? win_load(t, c + 128, b) : make_uint4(0, 0, 0, 0);   // next, in flight
+            const uint32_t f = win_starts4(v, c, glo, b, tprev);
+            tprev = __shfl_sync(0xffffffffu, v.w, 31);
+            const uint4 vc = v;
+            v = vn;
             const uint32_t nf = __popc(f);
             if (!__any_sync(0xffffffffu, nf != 0)) continue;
             // Ps: rows of [c, c + 128) before i, whatever their group (PS1 is the global prefix;
             // v holds every row below b, and rows at or after b follow every start)
             const uint32_t i0 = c + 4 * lane;
-            const uint4 x = v;
+            const uint4 x = vc;
             const uint64_t lsum = (uint64_t)x.x + x.y + x.z + x.w;
             const uint64_t lexcl = warp_incl_scan(lsum) - lsum;
             const uint32_t cexcl = warp_incl_scan(nf) - nf;
