@@ -42,6 +42,8 @@ def test_compute_sanitizer(tool, cfg):
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     with open(os.path.join(ROOT, "gpurun_out", f"sanitizer_{tool}_{cfg}.log"), "w") as f:
         f.write(log)
+    if "closed on this pool" in log:   # the GPU pool's operators disabled the tool (it left GPUs needing a reset)
+        pytest.skip("compute-sanitizer disabled on this GPU pool: " + log.strip().splitlines()[0][:200])
     assert "SANITIZE_RUN_OK" in log, log[-4000:]
     assert out.returncode == 0, log[-6000:]
     if tool == "racecheck":
