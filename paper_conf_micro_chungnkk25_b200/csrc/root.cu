@@ -49,6 +49,14 @@ static bool split_overlap() {   // STEMROOT_SPLIT_OVERLAP=0: small and big split
     if (v < 0) v = (getenv("STEMROOT_SPLIT_OVERLAP") && getenv("STEMROOT_SPLIT_OVERLAP")[0] == '0') ? 0 : 1;
     return v == 1;
 }
+// exact split rule's kernels: 2 (default) the nearest-centre descent for every
+// cluster; 1 the descent for big clusters, chunk bounds for the small ones; 0
+// chunk bounds for all (small-cluster warps + big-cluster blocks, the round-1/2
+// design).  STEMROOT_SPLIT_NC, read per plan.  C5: root_split 6.5 ms (0), 3.6 (1), 2.2 (2).
+static int nc_mode() {
+    const char *e = getenv("STEMROOT_SPLIT_NC");
+    return e ? atoi(e) : 2;
+}
 static bool seed_on() {   // STEMROOT_SPLIT_SEED=0 disables the coarse threshold seed
     static int v = -1;
     if (v < 0) v = (getenv("STEMROOT_SPLIT_SEED") && getenv("STEMROOT_SPLIT_SEED")[0] == '0') ? 0 : 1;
@@ -596,6 +604,136 @@ __global__ void __launch_bounds__(256, MINB) small_split_kernel(const uint32_t *
             cut[c] = best.k;
             cut_SL[c] = best.SL;
         }
+    }
+}
+
+// ---------------------------------------------------------------- nearest-centre descent (exact, any size)
+// The optimal cut k* of a cluster satisfies the nearest-centre condition of
+// 2-means: t[k*-1] <= m(k*) <= t[k*], m(k) = (mu_L(k) + mu_R(k)) / 2.  (If
+// t[k*-1] > m, the run of rows equal to t[k*-1] is strictly closer to mu_R:
+// moving it to R is a valid cut with a strictly smaller within-cluster sum of
+// squares, i.e. a strictly larger D^2 / (k (n - k)); symmetrically for t[k*].)
+// Every maximiser, so every tie, satisfies it.  For sorted rows mu_L and mu_R,
+// hence m, are non-decreasing in k, so a range of cuts [a, b] can hold a
+// maximiser only if m(b) >= t[a-1] and m(a) <= t[b], and only if it holds a
+// valid cut (t[a-1] < t[b]).  With cuts at 32-row chunk starts S_L is exact
+// from the sampled prefix PS1 and t[a-1], t[b] come from the chunk-boundary
+// pairs TB, so a warp tests 32 sub-ranges per step: a 32-ary descent from the
+// whole cluster to the surviving 32-row chunks, which are scanned row by row
+// (eval_cut, exact, ties -> smallest k).  All comparisons are exact integers:
+// m(k) >= v  <=>  S_L (n - k) + (S - S_L) k >= 2 v k (n - k)  (both < 2^97).
+__device__ __forceinline__ bool mid_ge(uint64_t SL, uint64_t k, uint64_t n, uint64_t S, uint32_t v) {
+    const uint64_t nk = n - k;
+    const u128 F = (u128)SL * nk + (u128)(S - SL) * k;
+    const u128 G = (u128)(k * nk) * (2ull * v);
+    return F >= G;
+}
+__device__ __forceinline__ bool mid_le(uint64_t SL, uint64_t k, uint64_t n, uint64_t S, uint32_t v) {
+    const uint64_t nk = n - k;
+    const u128 F = (u128)SL * nk + (u128)(S - SL) * k;
+    const u128 G = (u128)(k * nk) * (2ull * v);
+    return F <= G;
+}
+
+constexpr int kNcStack = 256;   // per warp: 1 + 31 x (descent depth <= 6) entries suffice
+struct NcStats {
+    unsigned long long *n_nodes, *n_scanned;
+};
+__global__ void __launch_bounds__(256) nc_split_kernel(const uint32_t *__restrict__ f_lo,
+                                                       const uint32_t *__restrict__ f_hi,
+                                                       const uint64_t *__restrict__ f_S, const uint64_t *ctot,
+                                                       const uint32_t *__restrict__ t,
+                                                       const uint64_t *__restrict__ PS1,
+                                                       const uint32_t *__restrict__ TB, uint32_t *__restrict__ cut,
+                                                       uint64_t *__restrict__ cut_SL, uint64_t nmin, NcStats st) {
+    __shared__ uint2 s_stack[256 / 32][kNcStack];
+    const uint32_t C = (uint32_t)(*ctot >> 32);
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    uint2 *stk = s_stack[w];
+    const uint2 *TB2 = reinterpret_cast<const uint2 *>(TB);
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    uint32_t my_nodes = 0, my_scanned = 0;
+    for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
+        const uint64_t lo = f_lo[c], hi = f_hi[c], n = hi - lo;
+        if (n < nmin) continue;
+        const uint64_t S = f_S[c];
+        const uint64_t base = warp_pref1(t, PS1, lo);
+        Cand best = no_cand();
+        // aligned chunks [C0, C1]: cut positions 32 C0 .. 32 C1 + 31 within [lo + 1, hi - 2],
+        // and the next chunk start 32 (C1 + 1) <= hi - 1 (so m is defined there)
+        const uint64_t C0 = (lo + 1 + kChunk - 1) >> kChunkLog;
+        const int64_t C1s = ((int64_t)hi - 33) >> kChunkLog;
+        if (hi < 33 || (int64_t)C0 > C1s) {   // short: scan every cut
+            uint64_t SLa = 0;
+            for (uint64_t ra = lo; ra < hi; ra += 32) {
+                const uint64_t rb = min(ra + 32, hi);
+                scan_chunk(t, lo, n, S, ra, rb, SLa, best);
+                uint64_t v = ra + lane < rb ? t[ra + lane] : 0u;
+#pragma unroll
+                for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+                SLa += v;
+            }
+            my_scanned += (uint32_t)((n + 31) / 32);
+        } else {
+            const uint64_t C1 = (uint64_t)C1s;
+            // head cuts [lo + 1, 32 C0) and tail cuts [32 (C1 + 1), hi)
+            scan_chunk(t, lo, n, S, lo, C0 << kChunkLog, 0, best);
+            scan_chunk(t, lo, n, S, (C1 + 1) << kChunkLog, hi, PS1[C1 + 1] - base, best);
+            int sp = 0;
+            if (lane == 0) stk[0] = make_uint2((uint32_t)C0, (uint32_t)C1);
+            sp = 1;
+            __syncwarp();
+            while (sp > 0) {
+                const uint2 nd = stk[--sp];
+                __syncwarp();
+                const uint64_t c0 = nd.x, c1 = nd.y, L = c1 - c0 + 1;
+                const uint64_t wd = (L + 31) / 32;                 // chunks per sub-range
+                const uint64_t s0 = c0 + (uint64_t)lane * wd;
+                const bool in = s0 <= c1;
+                const uint64_t s1 = min(s0 + wd - 1, c1);
+                bool keep = false;
+                uint64_t SLs = 0;
+                if (in) {
+                    const uint64_t pa = PS1[s0], pb = PS1[s1 + 1];
+                    const uint32_t tam1 = TB2[s0].x, tb = TB2[s1 + 1].x;   // t[32 s0 - 1], t[32 s1 + 31]
+                    SLs = pa - base;
+                    const uint64_t ka = (s0 << kChunkLog) - lo, kb = ((s1 + 1) << kChunkLog) - lo;
+                    keep = tam1 < tb && mid_ge(pb - base, kb, n, S, tam1) && mid_le(SLs, ka, n, S, tb);
+                }
+                my_nodes += in ? 1u : 0u;
+                uint32_t live = __ballot_sync(0xffffffffu, keep);
+                if (wd == 1) {   // single chunks: scan the survivors now
+                    while (live) {
+                        const int src = __ffs(live) - 1;
+                        live &= live - 1;
+                        const uint64_t q = c0 + (uint64_t)src;
+                        const uint64_t SLa = __shfl_sync(0xffffffffu, SLs, src);
+                        scan_chunk(t, lo, n, S, q << kChunkLog, (q + 1) << kChunkLog, SLa, best);
+                        my_scanned++;
+                    }
+                } else {
+                    const int below = __popc(live & ((1u << lane) - 1));
+                    if (keep) stk[sp + __popc(live) - 1 - below] = make_uint2((uint32_t)s0, (uint32_t)s1);   // leftmost on top
+                    sp += __popc(live);
+                    __syncwarp();
+                }
+            }
+        }
+#pragma unroll 1   // one copy of better() (with its 256-bit tie path) in the kernel body
+        for (int o = 16; o; o >>= 1) {
+            const Cand v = shfl_cand_xor(best, o);
+            if (better(v, best)) best = v;
+        }
+        if (lane == 0) {
+            cut[c] = best.k;
+            cut_SL[c] = best.SL;
+        }
+    }
+    // stats (lane sums; scanned is warp-uniform)
+    for (int o = 16; o; o >>= 1) my_nodes += __shfl_xor_sync(0xffffffffu, my_nodes, o);
+    if (lane == 0 && my_nodes) {
+        atomicAdd(st.n_nodes, (unsigned long long)my_nodes);
+        atomicAdd(st.n_scanned, (unsigned long long)my_scanned);
     }
 }
 
@@ -1440,6 +1578,14 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             CK(cudaEventRecord(c.ev_fork, st));
             CK(cudaStreamWaitEvent(c.side, c.ev_fork, 0));
         }
+        const int ncm = nc_mode();
+        if (ncm == 2) {   // every cluster by the nearest-centre descent
+            const uint64_t blocks = (Cub + 7) / 8;
+            nc_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, st>>>(
+                c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL, 0,
+                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned});
+            c.launches++;
+        } else {
         if (loc_rows < big_rows()) {
             const uint64_t blocks = (Cub + 7) / 8;
             static int minb = -1;   // STEMROOT_SMALL_MINB: resident blocks per SM the registers are sized for
@@ -1452,6 +1598,13 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
                     c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL);
             c.launches++;
         }
+        if (ncm == 1) {   // big clusters by the nearest-centre descent, beside the small-cluster warps
+            const uint64_t blocks = (Cub + 7) / 8;
+            nc_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, st>>>(
+                c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL, big_rows(),
+                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned});
+            c.launches++;
+        } else {
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
         BigEntry *ent = (BigEntry *)c.big_ent;
         uint32_t *first_ent = (uint32_t *)(ent + max_ent);
@@ -1474,10 +1627,12 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         big_reduce_kernel<<<(unsigned)min(Cub, (uint64_t)4096), 32, 0, st>>>(c.f_lo[cur], c.f_hi[cur], ctot, first_ent,
                                                                         (const Cand *)c.big_part, c.cut, c.cut_SL);
         c.launches += 2;
+        }   // ncm != 1
         if (overlap) {
             CK(cudaEventRecord(c.ev_join, c.side));
             CK(cudaStreamWaitEvent(st, c.ev_join, 0));
         }
+        }   // ncm != 2
         }   // split == 0
         c.stage_end(tk_s, 4 * Aub + 20 * Cub);
         CK(cudaGetLastError());
@@ -1914,7 +2069,7 @@ int root_values(Ctx &c, const uint32_t *vt, const uint64_t *vcnt, const uint32_t
 }
 
 // ---------------------------------------------------------------- kernels with many repeated times
-// A kernel group of >= STEMROOT_VALUE_ROWS rows (default 2^18; 0 = off) whose
+// A kernel group of >= STEMROOT_VALUE_ROWS rows (default 0 = off; 2^18 was the round-2 default) whose
 // times repeat (a 1024-point sample finds t[i] == t[i-1] at >= 1 - 1/R of the
 // points, R = STEMROOT_VALUE_RATIO, default 4) is handed to the value path:
 // its distinct values are listed once (first row, sum of t before it), its
@@ -1922,12 +2077,15 @@ int root_values(Ctx &c, const uint32_t *vt, const uint64_t *vcnt, const uint32_t
 // other groups, and its leaf starts are set in the row flags.  The tree is the
 // one the row levels would build (same cuts, same decisions), so this only
 // changes the cost: C5's 79 largest kernels hold 53 % of the rows but 2.4 % of
-// the distinct values.
+// the distinct values.  Off by default since the nearest-centre descent: the
+// row levels then decide those groups in less time than this path's listing.
 constexpr uint32_t kWinRows = 2048;   // one warp's window of a dense group (64 aligned 32-row chunks)
 
 static uint32_t value_rows() {   // read per plan (tests switch it)
     const char *e = getenv("STEMROOT_VALUE_ROWS");
-    const long v = e ? atol(e) : (1l << 18);
+    // default 0 (off): with the nearest-centre descent the row levels decide such
+    // groups faster than the value path's own preparation (C5: 31.7 vs 33.0 ms per plan)
+    const long v = e ? atol(e) : 0;
     return v < 0 ? 0u : (uint32_t)v;
 }
 

@@ -419,8 +419,13 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
         if (valid) {
             const uint32_t d = (uint32_t)(key[j] >> a.shift) & (R - 1);
             uint32_t peers;
+#ifdef SR_SORT_FAKE_RANK   // timing experiment only: no multi-split (wrong ranks)
+            if (true) {
+                peers = 1u << lane;
+#else
             if (ballot) {
                 peers = vmask & ~ballot_diff8(d, vmask);
+#endif
             } else {
                 peers = __match_any_sync(vmask, d);
             }
@@ -481,7 +486,12 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
     // round trip; global offset = pass digit base + predecessors' counts
     if (d < R) {
         uint64_t excl = 0;
+#ifdef SR_SORT_FAKE_LB   // timing experiment only (tools/sortbench): no look-back, approximate offsets, wrong output
+        excl = (uint64_t)((double)a.hist[a.pass * kHistR + d] * tile / (double)((a.n + TILE - 1) / TILE));
+        if (false) {
+#else
         if (tile != 0) {
+#endif
             int64_t j = (int64_t)tile - 1;
             bool done = false;
             while (!done) {
@@ -508,7 +518,10 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
     for (uint32_t i = tid; i < nvalid; i += NT) {
         const uint64_t k = s_keys[i];
         const uint32_t dd = (uint32_t)(k >> a.shift) & (R - 1);
-        const uint32_t gp = s_delta[dd] + i;
+        uint32_t gp = s_delta[dd] + i;
+#ifdef SR_SORT_FAKE_LB
+        if (gp >= a.n) gp = (uint32_t)(a.n - 1);
+#endif
         if (LAST) {
             const uint64_t kk = PK ? k >> a.ks : k;
             const uint32_t g = a.tab ? __ldg(a.tab + (kk >> a.tsh))

@@ -640,3 +640,45 @@ def test_value_path_active_rows_and_levels(ctx, monkeypatch):
     assert val_path["value_groups"] > 0
     assert val_path["active_rows"] == rows_path["active_rows"]
     assert max(val_path["levels"], val_path["value_levels"]) == rows_path["levels"]
+
+
+# ------------------------------------------------------------------ nearest-centre descent (root.cu nc_split_kernel)
+def _nc_case(case):
+    if case in BIG:
+        t = BIG[case]()
+        perm = np.random.default_rng(len(t)).permutation(len(t))
+        return np.zeros(len(t), np.uint32), t[perm], 1, 0.02
+    if case in EDGE:
+        kid, t, K = EDGE[case]
+        return kid, t, K, 0.05
+    if case == "mixture":
+        kid, t = _mixture(np.random.default_rng(11), 250_000, 19, peaks=5, spread=0.1)
+        return kid, t, 19, 0.01
+    if case == "dup_heavy":
+        return _dup_heavy(300_000, 29, 5) + (29, 0.005)
+    if case in ("quantised", "two_values"):
+        return _value_case(case, 7) + (0.01,)
+    sp = G.spec(case, n=1_500_000 if case == "C3" else None)
+    kid, t, _ = G.generate_np(sp)
+    return kid, t, sp.n_kernels, sp.eps
+
+
+@pytest.mark.parametrize("nc", ["0", "1", "2"])
+@pytest.mark.parametrize("case", sorted(BIG) + ["two_values", "one_off_short_call", "max_t", "mixture", "dup_heavy",
+                                                "quantised", "C2", "C3"])
+def test_nearest_centre_descent(ctx, monkeypatch, nc, case):
+    """The exact split by the nearest-centre descent (STEMROOT_SPLIT_NC=2, the
+    default: every cluster; 1: big clusters, chunk bounds for the rest; 0: the
+    chunk-bound kernels alone) equals the oracle's tree, samples and estimate
+    (the value path off, so every group takes the row levels)."""
+    kid, t, K, eps = _nc_case(case)
+    monkeypatch.setenv("STEMROOT_SPLIT_NC", nc)
+    monkeypatch.setenv("STEMROOT_VALUE_ROWS", "0")
+    got, ref = _both(ctx, kid, t, K, eps=eps, seed=3)
+    assert_plans_equal(got, ref)
+
+
+def test_nearest_centre_descent_ties(ctx, monkeypatch, golden):
+    monkeypatch.setenv("STEMROOT_SPLIT_NC", "2")
+    test_exact_tie_split(ctx, golden)
+    test_worked_trees(ctx, golden)
