@@ -1,6 +1,8 @@
 // internal.h -- host-side context and stage entry points of libstemroot.
 #pragma once
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 #include <cuda_runtime.h>
@@ -83,6 +85,18 @@ struct Timing {
     }
     void reset() { used = 0; pend.clear(); agg.clear(); }
     void finish() {   // stream already synchronised
+        if (getenv("STEMROOT_GAPS")) {   // analysis: device idle before each stage (stderr)
+            double tot = 0.0;
+            for (size_t i = 1; i < pend.size(); i++) {
+                float g = 0.f;
+                cudaEventElapsedTime(&g, pend[i - 1].b, pend[i].a);
+                if (g > 0.f) tot += g;
+                if (g > 0.02f) fprintf(stderr, "gap %.3f ms before %s\n", g, pend[i].name);
+            }
+            float span = 0.f;
+            if (!pend.empty()) cudaEventElapsedTime(&span, pend.front().a, pend.back().b);
+            fprintf(stderr, "gaps total %.3f ms, stage span %.3f ms\n", tot, span);
+        }
         for (auto &p : pend) {
             float ms = 0.f;
             cudaEventElapsedTime(&ms, p.a, p.b);

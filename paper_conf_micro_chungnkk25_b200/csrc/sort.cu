@@ -57,6 +57,9 @@ constexpr uint64_t kMaxTable = 1ull << 27;  // kid-table entries (512 MB) before
 #ifndef SR_SORT_LB
 #define SR_SORT_LB 4
 #endif
+#ifndef SR_SORT_LSMERGE
+#define SR_SORT_LSMERGE 1
+#endif
 #ifndef SR_SORT_MINB
 #define SR_SORT_MINB 4
 #endif
@@ -466,6 +469,11 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
         const uint32_t c_excl = coff + c_incl - cnt;
         s_lstart[d] = c_excl;
         if (d == R - 1) s_lstart[R] = c_excl + cnt;
+#if SR_SORT_LSMERGE
+        // fold the tile offset into every warp's base: one lookup per key in the scatter
+#pragma unroll
+        for (int ww = 0; ww < NW; ww++) s_whist[ww][d] = (uint16_t)(s_whist[ww][d] + c_excl);
+#endif
     }
     __syncthreads();
 
@@ -476,7 +484,11 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
         const uint64_t i = wbase + (uint64_t)j * 32 + lane;
         if (FULL || i < a.n) {
             const uint32_t dd = (uint32_t)(key[j] >> a.shift) & (R - 1);
+#if SR_SORT_LSMERGE
+            const uint32_t lp = s_whist[w][dd] + ((rank2[j / 2] >> (16 * (j & 1))) & 0xffffu);
+#else
             const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + ((rank2[j / 2] >> (16 * (j & 1))) & 0xffffu);
+#endif
             s_keys[lp] = key[j];
             if (!PK) s_vals[lp] = val[PK ? 0 : j];
         }

@@ -14,11 +14,11 @@ starts = [i for i, (k, _) in enumerate(seq) if k.startswith("prepass")]
 step = seq[starts[-1]:]
 levels, cur = [], {}
 for k, v in step:
-    if "entries" in k:
+    if "entries" in k or k.startswith("nc_split"):
         if cur:
             levels.append(cur)
         cur = {}
-    if any(x in k for x in ("big", "small", "decide", "lloyd")):
+    if any(x in k for x in ("big", "small", "decide", "lloyd", "nc_split")):
         cur[k] = cur.get(k, 0.0) + v
 levels.append(cur)
 tot = {}
