@@ -635,38 +635,53 @@ __device__ __forceinline__ bool mid_le(uint64_t SL, uint64_t k, uint64_t n, uint
     return F <= G;
 }
 
+#ifndef SR_NC_MINB
+#define SR_NC_MINB 4
+#endif
+#ifndef SR_NC_QUEUE
+#define SR_NC_QUEUE 1
+#endif
 constexpr int kNcStack = 256;   // per warp: 1 + 31 x (descent depth <= 6) entries suffice
 struct NcStats {
     unsigned long long *n_nodes, *n_scanned;
 };
-__global__ void __launch_bounds__(256) nc_split_kernel(const uint32_t *__restrict__ f_lo,
+__global__ void __launch_bounds__(256, SR_NC_MINB) nc_split_kernel(const uint32_t *__restrict__ f_lo,
                                                        const uint32_t *__restrict__ f_hi,
                                                        const uint64_t *__restrict__ f_S, const uint64_t *ctot,
                                                        const uint32_t *__restrict__ t,
                                                        const uint64_t *__restrict__ PS1,
                                                        const uint32_t *__restrict__ TB, uint32_t *__restrict__ cut,
-                                                       uint64_t *__restrict__ cut_SL, uint64_t nmin, NcStats st) {
+                                                       uint64_t *__restrict__ cut_SL, uint64_t nmin, NcStats st,
+                                                       uint32_t *__restrict__ queue) {
     __shared__ uint2 s_stack[256 / 32][kNcStack];
     const uint32_t C = (uint32_t)(*ctot >> 32);
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     uint2 *stk = s_stack[w];
     const uint2 *TB2 = reinterpret_cast<const uint2 *>(TB);
-    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
     uint32_t my_nodes = 0, my_scanned = 0;
-    for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
-        const uint64_t lo = f_lo[c], hi = f_hi[c], n = hi - lo;
-        if (n < nmin) continue;
+    // clusters by a work queue (the next index fetched while this one is split:
+    // cluster sizes vary by orders of magnitude) or grid-stride
+    uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    for (; c < C;) {
+        uint32_t cn = 0;
+        if (SR_NC_QUEUE && lane == 0) cn = nwarps + atomicAdd(queue, 1u);
+        const uint32_t lo = f_lo[c], hi = f_hi[c], n = hi - lo;
+        if (n < nmin) {
+            c = SR_NC_QUEUE ? __shfl_sync(0xffffffffu, cn, 0) : c + nwarps;
+            continue;
+        }
         const uint64_t S = f_S[c];
         const uint64_t base = warp_pref1(t, PS1, lo);
         Cand best = no_cand();
         // aligned chunks [C0, C1]: cut positions 32 C0 .. 32 C1 + 31 within [lo + 1, hi - 2],
         // and the next chunk start 32 (C1 + 1) <= hi - 1 (so m is defined there)
-        const uint64_t C0 = (lo + 1 + kChunk - 1) >> kChunkLog;
+        const uint32_t C0 = (uint32_t)(((uint64_t)lo + kChunk) >> kChunkLog);
         const int64_t C1s = ((int64_t)hi - 33) >> kChunkLog;
         if (hi < 33 || (int64_t)C0 > C1s) {   // short: scan every cut
             uint64_t SLa = 0;
             for (uint64_t ra = lo; ra < hi; ra += 32) {
-                const uint64_t rb = min(ra + 32, hi);
+                const uint64_t rb = min(ra + 32, (uint64_t)hi);
                 scan_chunk(t, lo, n, S, ra, rb, SLa, best);
                 uint64_t v = ra + lane < rb ? t[ra + lane] : 0u;
 #pragma unroll
@@ -675,29 +690,29 @@ __global__ void __launch_bounds__(256) nc_split_kernel(const uint32_t *__restric
             }
             my_scanned += (uint32_t)((n + 31) / 32);
         } else {
-            const uint64_t C1 = (uint64_t)C1s;
+            const uint32_t C1 = (uint32_t)C1s;
             // head cuts [lo + 1, 32 C0) and tail cuts [32 (C1 + 1), hi)
-            scan_chunk(t, lo, n, S, lo, C0 << kChunkLog, 0, best);
-            scan_chunk(t, lo, n, S, (C1 + 1) << kChunkLog, hi, PS1[C1 + 1] - base, best);
+            scan_chunk(t, lo, n, S, lo, (uint64_t)C0 << kChunkLog, 0, best);
+            scan_chunk(t, lo, n, S, (uint64_t)(C1 + 1) << kChunkLog, hi, PS1[C1 + 1] - base, best);
             int sp = 0;
-            if (lane == 0) stk[0] = make_uint2((uint32_t)C0, (uint32_t)C1);
+            if (lane == 0) stk[0] = make_uint2(C0, C1);
             sp = 1;
             __syncwarp();
             while (sp > 0) {
                 const uint2 nd = stk[--sp];
                 __syncwarp();
-                const uint64_t c0 = nd.x, c1 = nd.y, L = c1 - c0 + 1;
-                const uint64_t wd = (L + 31) / 32;                 // chunks per sub-range
-                const uint64_t s0 = c0 + (uint64_t)lane * wd;
+                const uint32_t c0 = nd.x, c1 = nd.y;
+                const uint32_t wd = (c1 - c0 + 32) / 32;          // chunks per sub-range
+                const uint32_t s0 = c0 + (uint32_t)lane * wd;
                 const bool in = s0 <= c1;
-                const uint64_t s1 = min(s0 + wd - 1, c1);
+                const uint32_t s1 = min(s0 + wd - 1, c1);
                 bool keep = false;
                 uint64_t SLs = 0;
                 if (in) {
                     const uint64_t pa = PS1[s0], pb = PS1[s1 + 1];
                     const uint32_t tam1 = TB2[s0].x, tb = TB2[s1 + 1].x;   // t[32 s0 - 1], t[32 s1 + 31]
                     SLs = pa - base;
-                    const uint64_t ka = (s0 << kChunkLog) - lo, kb = ((s1 + 1) << kChunkLog) - lo;
+                    const uint64_t ka = ((uint64_t)s0 << kChunkLog) - lo, kb = ((uint64_t)(s1 + 1) << kChunkLog) - lo;
                     keep = tam1 < tb && mid_ge(pb - base, kb, n, S, tam1) && mid_le(SLs, ka, n, S, tb);
                 }
                 my_nodes += in ? 1u : 0u;
@@ -713,7 +728,7 @@ __global__ void __launch_bounds__(256) nc_split_kernel(const uint32_t *__restric
                     }
                 } else {
                     const int below = __popc(live & ((1u << lane) - 1));
-                    if (keep) stk[sp + __popc(live) - 1 - below] = make_uint2((uint32_t)s0, (uint32_t)s1);   // leftmost on top
+                    if (keep) stk[sp + __popc(live) - 1 - below] = make_uint2(s0, s1);   // leftmost on top
                     sp += __popc(live);
                     __syncwarp();
                 }
@@ -728,6 +743,7 @@ __global__ void __launch_bounds__(256) nc_split_kernel(const uint32_t *__restric
             cut[c] = best.k;
             cut_SL[c] = best.SL;
         }
+        c = SR_NC_QUEUE ? __shfl_sync(0xffffffffu, cn, 0) : c + nwarps;
     }
     // stats (lane sums; scanned is warp-uniform)
     for (int o = 16; o; o >>= 1) my_nodes += __shfl_xor_sync(0xffffffffu, my_nodes, o);
@@ -1579,11 +1595,12 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             CK(cudaStreamWaitEvent(c.side, c.ev_fork, 0));
         }
         const int ncm = nc_mode();
+        if (ncm) CK(cudaMemsetAsync(&c.scalars->nc_queue, 0, sizeof(uint32_t), st));
         if (ncm == 2) {   // every cluster by the nearest-centre descent
             const uint64_t blocks = (Cub + 7) / 8;
             nc_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, st>>>(
                 c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL, 0,
-                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned});
+                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned}, &c.scalars->nc_queue);
             c.launches++;
         } else {
         if (loc_rows < big_rows()) {
@@ -1602,7 +1619,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             const uint64_t blocks = (Cub + 7) / 8;
             nc_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, st>>>(
                 c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL, big_rows(),
-                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned});
+                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned}, &c.scalars->nc_queue);
             c.launches++;
         } else {
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
