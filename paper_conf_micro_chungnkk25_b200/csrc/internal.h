@@ -52,7 +52,7 @@ struct DevScalars {
     unsigned long long split_chunks, split_scanned;   // big-cluster chunks bounded / scanned row by row
     uint32_t local_depth, amb_count;      // deepest ROOT level of a local subtree; ambiguous samples
     uint32_t km_nsub[2];                  // split = 3: subproblems of the current / next D&C round
-    uint32_t nc_queue, pad3;              // nearest-centre descent: next cluster of the level's work queue
+    uint32_t nc_queue[2];                 // nearest-centre descent: next cluster of the level's work queue (by level parity)
 };
 
 constexpr int kMaxCand = 64;     // packed sort: most candidate rows per sample (one u64 mask)

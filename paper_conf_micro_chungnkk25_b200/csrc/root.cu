@@ -638,6 +638,12 @@ __device__ __forceinline__ bool mid_le(uint64_t SL, uint64_t k, uint64_t n, uint
 #ifndef SR_NC_MINB
 #define SR_NC_MINB 4
 #endif
+#ifndef SR_NC_THREADS
+#define SR_NC_THREADS 256
+#endif
+#ifndef SR_NC_SBEST
+#define SR_NC_SBEST 0
+#endif
 #ifndef SR_NC_QUEUE
 #define SR_NC_QUEUE 1
 #endif
@@ -645,17 +651,25 @@ constexpr int kNcStack = 256;   // per warp: 1 + 31 x (descent depth <= 6) entri
 struct NcStats {
     unsigned long long *n_nodes, *n_scanned;
 };
-__global__ void __launch_bounds__(256, SR_NC_MINB) nc_split_kernel(const uint32_t *__restrict__ f_lo,
+__global__ void __launch_bounds__(SR_NC_THREADS, SR_NC_MINB) nc_split_kernel(const uint32_t *__restrict__ f_lo,
                                                        const uint32_t *__restrict__ f_hi,
                                                        const uint64_t *__restrict__ f_S, const uint64_t *ctot,
                                                        const uint32_t *__restrict__ t,
                                                        const uint64_t *__restrict__ PS1,
                                                        const uint32_t *__restrict__ TB, uint32_t *__restrict__ cut,
                                                        uint64_t *__restrict__ cut_SL, uint64_t nmin, NcStats st,
-                                                       uint32_t *__restrict__ queue) {
-    __shared__ uint2 s_stack[256 / 32][kNcStack];
+                                                       uint32_t *__restrict__ queue, uint32_t *__restrict__ queue_next,
+                                                       uint64_t *__restrict__ ntot) {
+    __shared__ uint2 s_stack[SR_NC_THREADS / 32][kNcStack];
+#if SR_NC_SBEST
+    __shared__ Cand s_best[SR_NC_THREADS / 32][32];   // each lane's best candidate lives in shared memory (registers for occupancy)
+#endif
     const uint32_t C = (uint32_t)(*ctot >> 32);
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {   // for the next kernels in stream order (no memset launches)
+        if (queue_next) *queue_next = 0u;    // the next level's work queue
+        if (ntot) *ntot = 0ull;              // the frontier this level's decision appends to
+    }
     uint2 *stk = s_stack[w];
     const uint2 *TB2 = reinterpret_cast<const uint2 *>(TB);
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -673,7 +687,12 @@ __global__ void __launch_bounds__(256, SR_NC_MINB) nc_split_kernel(const uint32_
         }
         const uint64_t S = f_S[c];
         const uint64_t base = warp_pref1(t, PS1, lo);
-        Cand best = no_cand();
+#if SR_NC_SBEST
+        Cand &best = s_best[w][lane];
+#else
+        Cand best;
+#endif
+        best = no_cand();
         // aligned chunks [C0, C1]: cut positions 32 C0 .. 32 C1 + 31 within [lo + 1, hi - 2],
         // and the next chunk start 32 (C1 + 1) <= hi - 1 (so m is defined there)
         const uint32_t C0 = (uint32_t)(((uint64_t)lo + kChunk) >> kChunkLog);
@@ -734,14 +753,15 @@ __global__ void __launch_bounds__(256, SR_NC_MINB) nc_split_kernel(const uint32_
                 }
             }
         }
+        Cand fin = best;
 #pragma unroll 1   // one copy of better() (with its 256-bit tie path) in the kernel body
         for (int o = 16; o; o >>= 1) {
-            const Cand v = shfl_cand_xor(best, o);
-            if (better(v, best)) best = v;
+            const Cand v = shfl_cand_xor(fin, o);
+            if (better(v, fin)) fin = v;
         }
         if (lane == 0) {
-            cut[c] = best.k;
-            cut_SL[c] = best.SL;
+            cut[c] = fin.k;
+            cut_SL[c] = fin.SL;
         }
         c = SR_NC_QUEUE ? __shfl_sync(0xffffffffu, cn, 0) : c + nwarps;
     }
@@ -1532,6 +1552,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
     CK(cudaStreamSynchronize(st));
     uint32_t levels = 0;
     // enqueue ROOT level `level` (1-based) consuming frontier cur, bounded by (Cub, Aub)
+    const int ncm_l = split == 0 ? nc_mode() : -1;   // the exact rule's split kernels (read once per plan)
     auto enqueue_level = [&](uint32_t level, int cur, uint64_t Cub, uint64_t Aub) -> int {
         const int nxt = cur ^ 1;
         const uint64_t *ctot = &c.scalars->ftot[cur];
@@ -1594,13 +1615,15 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             CK(cudaEventRecord(c.ev_fork, st));
             CK(cudaStreamWaitEvent(c.side, c.ev_fork, 0));
         }
-        const int ncm = nc_mode();
-        if (ncm) CK(cudaMemsetAsync(&c.scalars->nc_queue, 0, sizeof(uint32_t), st));
+        const int ncm = ncm_l;
+        uint32_t *q_cur = &c.scalars->nc_queue[level & 1], *q_next = &c.scalars->nc_queue[(level + 1) & 1];
+        if (ncm == 1 || (ncm == 2 && level == 1)) CK(cudaMemsetAsync(q_cur, 0, sizeof(uint32_t), st));
         if (ncm == 2) {   // every cluster by the nearest-centre descent
-            const uint64_t blocks = (Cub + 7) / 8;
-            nc_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, st>>>(
+            constexpr uint64_t wpb = SR_NC_THREADS / 32;
+            const uint64_t blocks = (Cub + wpb - 1) / wpb;
+            nc_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16 * (8 / wpb)), SR_NC_THREADS, 0, st>>>(
                 c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL, 0,
-                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned}, &c.scalars->nc_queue);
+                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned}, q_cur, q_next, ntot);
             c.launches++;
         } else {
         if (loc_rows < big_rows()) {
@@ -1616,10 +1639,11 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
             c.launches++;
         }
         if (ncm == 1) {   // big clusters by the nearest-centre descent, beside the small-cluster warps
-            const uint64_t blocks = (Cub + 7) / 8;
-            nc_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16), 256, 0, st>>>(
+            constexpr uint64_t wpb = SR_NC_THREADS / 32;
+            const uint64_t blocks = (Cub + wpb - 1) / wpb;
+            nc_split_kernel<<<(unsigned)min(blocks, (uint64_t)c.sms * 16 * (8 / wpb)), SR_NC_THREADS, 0, st>>>(
                 c.f_lo[cur], c.f_hi[cur], c.f_S[cur], ctot, c.t_sorted, c.PS1, c.TB, c.cut, c.cut_SL, big_rows(),
-                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned}, &c.scalars->nc_queue);
+                NcStats{&c.scalars->split_chunks, &c.scalars->split_scanned}, q_cur, nullptr, nullptr);
             c.launches++;
         } else {
         // big clusters: entries (cluster, segment), chunk-bound argmax, per-cluster reduce
@@ -1654,7 +1678,7 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         c.stage_end(tk_s, 4 * Aub + 20 * Cub);
         CK(cudaGetLastError());
         const int tk_d = c.stage_begin("root_decide");
-        CK(cudaMemsetAsync(ntot, 0, sizeof(uint64_t), st));
+        if (ncm_l != 2) CK(cudaMemsetAsync(ntot, 0, sizeof(uint64_t), st));   // else zeroed by nc_split
         DecideArgs da{c.f_lo[cur], c.f_hi[cur], c.cut, c.f_S[cur], c.cut_SL, c.f_Q[cur], ctot, c.PS1, c.PS2,
                       c.t_sorted, c.flags, c.f_lo[nxt], c.f_hi[nxt], c.f_S[nxt], c.f_Q[nxt],
                       ntot, eps, z, k2, clamp};

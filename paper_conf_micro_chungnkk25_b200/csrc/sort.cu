@@ -779,6 +779,9 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     a.noalloc = 1;
     if (const char *e = getenv("STEMROOT_SORT_NOALLOC")) a.noalloc = atoi(e) ? 1 : 0;
     if (const char *e = getenv("STEMROOT_SORT_LATE")) a.late = atoi(e) ? 1 : 0;
+    int late_first = a.late;   // STEMROOT_SORT_LATE_FIRST: the first pass's publication alone
+    if (const char *e = getenv("STEMROOT_SORT_LATE_FIRST")) late_first = atoi(e) ? 1 : 0;
+    const int late_rest = a.late;
     int rank_force = -1;   // STEMROOT_SORT_RANK=match|ballot forces one ranking mode
     double rank_thr = 24.0;   // STEMROOT_SORT_RANK_THR: ballots from this many expected distinct digits
     if (const char *e = getenv("STEMROOT_SORT_RANK_THR")) rank_thr = atof(e);
@@ -802,6 +805,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         a.shift = ks + kRB * p;
         a.pass = p;
         const bool first = p == 0, last = p == npasses - 1;
+        a.late = first ? late_first : late_rest;
         a.kid_in = kid;
         a.t_in = t;
         a.row_in = row_in;

@@ -292,18 +292,19 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
             // sorted run; the candidates (h << s) | low that hold (kernel, t)
             const uint32_t k = a.leaf_kid[i];
             uint64_t mask = 0;
-            for (uint32_t h0 = 0; h0 < a.pack_h; h0 += 16) {   // 16 candidates' loads in flight
-                uint32_t kv[16], tw[16];
+            for (uint32_t h0 = 0; h0 < a.pack_h; h0 += 16) {   // 16 candidates' times in flight
+                uint32_t tw[16];
 #pragma unroll
                 for (int u = 0; u < 16; u++) {
                     const uint64_t r = ((uint64_t)(h0 + u) << a.pack_s) | low;
                     const bool ok = h0 + u < a.pack_h && r < a.n;
-                    kv[u] = ok ? __ldg(a.kid_in + r) : 0xFFFFFFFFu;   // never a kernel id (K <= 2^24)
-                    tw[u] = ok ? __ldg(a.t_in + r) : 0u;
+                    tw[u] = ok ? __ldg(a.t_in + r) : ~tv;   // never equal to tv
                 }
+                // the kernel id only where the time matches (most candidates differ in t)
 #pragma unroll
                 for (int u = 0; u < 16; u++)
-                    if (kv[u] == k && tw[u] == tv) mask |= 1ull << (h0 + u);
+                    if (tw[u] == tv && __ldg(a.kid_in + (((uint64_t)(h0 + u) << a.pack_s) | low)) == k)
+                        mask |= 1ull << (h0 + u);
             }
             if (__popcll(mask) == 1) {
                 a.out_row[s] = map_row(a, (uint32_t)(((uint64_t)(__ffsll(mask) - 1) << a.pack_s) | low));

@@ -20,12 +20,12 @@ python tools/level_table.py gpurun_out/${R}_launches_c5.csv > gpurun_out/${R}_le
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:onesweep -s 2 -c 1 \
     -o gpurun_out/${R}_prof_sort_mid_c5 python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > /dev/null 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on \
-    -k regex:"prepass|pm_sums|pm_apply|big_split|small_split|decide|flag_c|sample_kernel|estimate|onesweep" -c 24 \
+    -k regex:"prepass|pm_sums|pm_apply|nc_split|decide|flag_c|sample_kernel|estimate|onesweep" -c 30 \
     -o gpurun_out/${R}_prof_other_c5 python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > /dev/null 2>&1
 # summaries here; only the small reports travel back (gpurun_out must stay under 64 MiB)
 python tools/ncu_summary.py gpurun_out/${R}_prof_sort_mid_c5.ncu-rep --traffic-json gpurun_out/ncu_traffic.json --config C5 --stage sort_pass_mid > gpurun_out/${R}_ncu_sort_mid_c5.txt 2>&1
 python tools/sass_hot.py gpurun_out/${R}_prof_sort_mid_c5.ncu-rep 25 >> gpurun_out/${R}_ncu_sort_mid_c5.txt 2>&1
 python tools/ncu_summary.py gpurun_out/${R}_prof_other_c5.ncu-rep > gpurun_out/${R}_ncu_other_c5.txt 2>&1
-python tools/sass_hot.py gpurun_out/${R}_prof_other_c5.ncu-rep 15 big_split >> gpurun_out/${R}_ncu_other_c5.txt 2>&1
+python tools/sass_hot.py gpurun_out/${R}_prof_other_c5.ncu-rep 15 nc_split >> gpurun_out/${R}_ncu_other_c5.txt 2>&1
 rm -f gpurun_out/${R}_prof_other_c5.ncu-rep
 du -sh gpurun_out; ls -la gpurun_out
