@@ -636,13 +636,13 @@ __device__ __forceinline__ bool mid_le(uint64_t SL, uint64_t k, uint64_t n, uint
 }
 
 #ifndef SR_NC_MINB
-#define SR_NC_MINB 4
+#define SR_NC_MINB 9
 #endif
 #ifndef SR_NC_THREADS
-#define SR_NC_THREADS 256
+#define SR_NC_THREADS 128
 #endif
 #ifndef SR_NC_SBEST
-#define SR_NC_SBEST 0
+#define SR_NC_SBEST 1
 #endif
 #ifndef SR_NC_QUEUE
 #define SR_NC_QUEUE 1
