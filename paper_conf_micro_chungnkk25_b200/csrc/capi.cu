@@ -49,6 +49,10 @@ static void dfree(T *&p, size_t &cap) {
 }
 
 void Ctx::release() {
+    plan_block_abort(*this);
+    if (dstream) { cudaStreamDestroy(dstream); dstream = nullptr; }
+    if (ev_pack) { cudaEventDestroy(ev_pack); ev_pack = nullptr; }
+    if (ev_d2h) { cudaEventDestroy(ev_d2h); ev_d2h = nullptr; }
     if (ev_fork) cudaEventDestroy(ev_fork);
     if (ev_join) cudaEventDestroy(ev_join);
     if (side) cudaStreamDestroy(side);
@@ -275,50 +279,102 @@ static void pool_release(void *m, size_t bytes, bool pinned) {
     cudaFreeHost(m);
 }
 
-static int to_host(Ctx &c, stem_plan **out) {
+// the plan block's layout for L clusters, S samples, nm metrics
+struct PlanLayout {
+    size_t o_cl, o_row, o_scl, o_w, o_est, o_tru, o_bnd, total;
+    PlanLayout(uint64_t L, uint64_t S, uint64_t nm) {
+        auto al = [](size_t x) { return (x + 63) & ~(size_t)63; };
+        o_cl = 0;
+        o_row = o_cl + al(sizeof(stem_cluster) * L);
+        o_scl = o_row + al(sizeof(uint32_t) * S);
+        o_w = o_scl + al(sizeof(uint32_t) * S);
+        o_est = o_w + al(sizeof(double) * S);
+        o_tru = o_est + al(sizeof(double) * (nm ? nm : 1));
+        o_bnd = o_tru + al(sizeof(double) * nm);
+        total = o_bnd + al(sizeof(double) * nm);
+    }
+};
+
+static PlanBlock *plan_block_new(uint64_t L, uint64_t S, uint32_t nm) {
     PlanBlock *pb = (PlanBlock *)calloc(1, sizeof(PlanBlock));
-    if (!pb) return STEM_E_NOMEM;
+    if (!pb) return nullptr;
     stem_plan *p = &pb->pub;
-    const uint64_t L = c.n_leaves, S = c.n_samples, nm = c.n_metrics;
-    auto al = [](size_t x) { return (x + 63) & ~(size_t)63; };
-    const size_t o_cl = 0, o_row = o_cl + al(sizeof(stem_cluster) * L), o_scl = o_row + al(sizeof(uint32_t) * S),
-                 o_w = o_scl + al(sizeof(uint32_t) * S), o_est = o_w + al(sizeof(double) * S),
-                 o_tru = o_est + al(sizeof(double) * (nm ? nm : 1)), o_bnd = o_tru + al(sizeof(double) * nm),
-                 total = o_bnd + al(sizeof(double) * nm);
+    const PlanLayout ly(L, S, nm);
     size_t got = 0;
     bool pinned = false;
-    char *mem = (char *)pool_acquire(total, got, pinned);
+    char *mem = (char *)pool_acquire(ly.total, got, pinned);
     if (!mem) {
         free(pb);
-        return STEM_E_NOMEM;
+        return nullptr;
     }
     pb->mem = mem;
     pb->bytes = got;
     pb->pinned = pinned;
     p->n_clusters = L;
     p->n_samples = S;
-    p->clusters = (stem_cluster *)(mem + o_cl);
-    p->sample_row = (uint32_t *)(mem + o_row);
-    p->sample_cluster = (uint32_t *)(mem + o_scl);
-    p->sample_weight = (double *)(mem + o_w);
-    p->n_metrics = c.n_metrics;
-    p->est_metric = (double *)(mem + o_est);
-    p->true_metric = c.have_mbounds ? (double *)(mem + o_tru) : nullptr;
-    p->bound_metric = c.have_mbounds ? (double *)(mem + o_bnd) : nullptr;
-    cudaStream_t st = c.stream;
+    p->clusters = (stem_cluster *)(mem + ly.o_cl);
+    p->sample_row = (uint32_t *)(mem + ly.o_row);
+    p->sample_cluster = (uint32_t *)(mem + ly.o_scl);
+    p->sample_weight = (double *)(mem + ly.o_w);
+    p->n_metrics = nm;
+    p->est_metric = (double *)(mem + ly.o_est);
+    p->true_metric = (double *)(mem + ly.o_tru);
+    p->bound_metric = (double *)(mem + ly.o_bnd);
+    return pb;
+}
+
+int plan_block_begin(Ctx &c, uint64_t L, uint64_t S, uint32_t nm, stem_cluster **clusters_dst, uint32_t **row_dst,
+                     uint32_t **cl_dst, double **w_dst) {
+    plan_block_abort(c);
+    PlanBlock *pb = plan_block_new(L, S, nm);
+    if (!pb) return STEM_E_NOMEM;
+    c.early_plan = pb;
+    *clusters_dst = pb->pub.clusters;
+    *row_dst = pb->pub.sample_row;
+    *cl_dst = pb->pub.sample_cluster;
+    *w_dst = pb->pub.sample_weight;
+    return STEM_OK;
+}
+
+void plan_block_abort(Ctx &c) {
+    if (!c.early_plan) return;
+    if (c.dstream) cudaStreamSynchronize(c.dstream);   // no copy may land in a released block
+    cudaStreamSynchronize(c.stream);
+    stem_plan_free(&((PlanBlock *)c.early_plan)->pub);
+    c.early_plan = nullptr;
+}
+
+static int to_host(Ctx &c, stem_plan **out) {
+    const uint64_t L = c.n_leaves, S = c.n_samples;
+    PlanBlock *pb = (PlanBlock *)c.early_plan;
+    c.early_plan = nullptr;
     cudaError_t e = cudaSuccess;
-    if (L) e = cudaMemcpyAsync(p->clusters, c.out_clusters, sizeof(stem_cluster) * L, cudaMemcpyDeviceToHost, st);
-    if (S && e == cudaSuccess)
-        e = cudaMemcpyAsync(p->sample_row, c.out_row, sizeof(uint32_t) * S, cudaMemcpyDeviceToHost, st);
-    if (S && e == cudaSuccess)
-        e = cudaMemcpyAsync(p->sample_cluster, c.out_cluster, sizeof(uint32_t) * S, cudaMemcpyDeviceToHost, st);
-    if (S && e == cudaSuccess)
-        e = cudaMemcpyAsync(p->sample_weight, c.out_weight, sizeof(double) * S, cudaMemcpyDeviceToHost, st);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (pb) {   // every copy already queued (leaves_and_plan): wait for them
+        if (c.dstream) e = cudaStreamSynchronize(c.dstream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(c.stream);
+    } else {
+        pb = plan_block_new(L, S, c.n_metrics);
+        if (!pb) return STEM_E_NOMEM;
+        stem_plan *p = &pb->pub;
+        cudaStream_t st = c.stream;
+        if (L) e = cudaMemcpyAsync(p->clusters, c.out_clusters, sizeof(stem_cluster) * L, cudaMemcpyDeviceToHost, st);
+        if (S && e == cudaSuccess)
+            e = cudaMemcpyAsync(p->sample_row, c.out_row, sizeof(uint32_t) * S, cudaMemcpyDeviceToHost, st);
+        if (S && e == cudaSuccess)
+            e = cudaMemcpyAsync(p->sample_cluster, c.out_cluster, sizeof(uint32_t) * S, cudaMemcpyDeviceToHost, st);
+        if (S && e == cudaSuccess)
+            e = cudaMemcpyAsync(p->sample_weight, c.out_weight, sizeof(double) * S, cudaMemcpyDeviceToHost, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    }
+    stem_plan *p = &pb->pub;
     if (e != cudaSuccess) {
         last_cuda_error() = e;
         stem_plan_free(p);
         return STEM_E_CUDA;
+    }
+    if (!c.have_mbounds) {
+        p->true_metric = nullptr;
+        p->bound_metric = nullptr;
     }
     p->est_total_ns = c.est_total;
     p->true_total_ns = c.T;
@@ -394,12 +450,16 @@ int stem_root_plan_ctx(stem_ctx *ctx, const stem_trace *trace, double eps, doubl
     if (!ctx) return STEM_E_INVAL;
     stem_opts o;
     if (opts) o = *opts; else stem_default_opts(&o);
+    ctx->c.want_host = out != nullptr;
     int s = sr::run_plan(ctx->c, trace, eps, conf, o);
+    ctx->c.want_host = false;
     if (s != STEM_OK) {
+        sr::plan_block_abort(ctx->c);
         ctx->c.have_plan = false;
         return s;
     }
     if (out) return sr::to_host(ctx->c, out);
+    sr::plan_block_abort(ctx->c);
     return STEM_OK;
 }
 

@@ -260,6 +260,15 @@ struct Ctx {
     bool have_mbounds = false;
     double host_true_metric[64], host_bound_metric[64];
 
+    // host plan: with want_host the single-GPU path allocates the caller's plan
+    // block as soon as its size is known and copies the cluster records into it
+    // on dstream while the samples are drawn (capi.cu plan_block_begin / to_host)
+    bool want_host = false;
+    void *early_plan = nullptr;                 // PlanBlock (capi.cu), or NULL
+    cudaStream_t dstream = nullptr;
+    cudaEvent_t ev_pack = nullptr, ev_d2h = nullptr;
+    bool early_packed = false;
+
     // last plan
     bool have_plan = false;
     uint64_t n = 0, n_leaves = 0, n_samples = 0, T = 0;
@@ -349,6 +358,11 @@ int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n
                       uint32_t *tailh);   // pre-pass only
 int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
                   const stem_opts &o, int local_status);
+// capi.cu: allocate the host plan block for L clusters, S samples (c.early_plan);
+// returns the device-to-host destination of the cluster records
+int plan_block_begin(Ctx &c, uint64_t L, uint64_t S, uint32_t nm, stem_cluster **clusters_dst, uint32_t **row_dst,
+                     uint32_t **cl_dst, double **w_dst);
+void plan_block_abort(Ctx &c);
 int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint32_t n_metrics, double eps,
                     double z, double k2, const stem_opts &o, const uint32_t *tr_kid = nullptr,
                     const uint32_t *tr_t = nullptr, uint64_t tr_n = 0);                        // a5..a8

@@ -624,6 +624,8 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     double *part_est = nullptr, *part_met = nullptr, *red_out = nullptr;
     uint64_t mb = 0;
     int tk_est = -1;
+    uint32_t *h_row = nullptr, *h_scl = nullptr;   // the early host plan's sample arrays
+    double *h_w = nullptr;
     CKS(dist_checkpoint(c, [&]() -> int {
         DevScalars hs;
         CK(cudaMemcpyAsync(&hs, c.scalars, sizeof(DevScalars), cudaMemcpyDeviceToHost, st));
@@ -642,6 +644,30 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         // packed sort: ambiguous-sample entries, their chunk counts/offsets, scan scratch
         const size_t amb_bytes = sizeof(Amb) * (S + 1), nch_bytes = sizeof(uint64_t) * (S + 1);
         if (c.pack_h > 1) CKS(c.ensure(c.amb, c.cap_amb, amb_bytes + 2 * nch_bytes + (scan_tiles(S + 1) + 2) * 16));
+        c.early_packed = false;
+        static const bool early_on = !(getenv("STEMROOT_EARLY_PLAN") && getenv("STEMROOT_EARLY_PLAN")[0] == '0');
+        if (c.want_host && !c.comm && L && S && early_on) {
+            // the caller's plan block now: the cluster records are packed here (they
+            // need only m) and copied to it on dstream while the samples are drawn
+            stem_cluster *h_cl = nullptr;
+            CKS(plan_block_begin(c, L, S, nm, &h_cl, &h_row, &h_scl, &h_w));
+            if (!c.dstream) {
+                CK(cudaStreamCreateWithFlags(&c.dstream, cudaStreamNonBlocking));
+                CK(cudaEventCreateWithFlags(&c.ev_pack, cudaEventDisableTiming));
+                CK(cudaEventCreateWithFlags(&c.ev_d2h, cudaEventDisableTiming));
+            }
+            CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
+            const int tk_pack = c.stage_begin("pack");
+            pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.PS1, c.PS2, c.t_sorted,
+                                                            c.leaf_m, c.leaf_census, L, n, c.kid_base, c.out_clusters);
+            c.launches++;
+            c.stage_end(tk_pack, 88 * L);
+            CK(cudaGetLastError());
+            CK(cudaEventRecord(c.ev_pack, st));
+            CK(cudaStreamWaitEvent(c.dstream, c.ev_pack, 0));
+            CK(cudaMemcpyAsync(h_cl, c.out_clusters, sizeof(stem_cluster) * L, cudaMemcpyDeviceToHost, c.dstream));
+            c.early_packed = true;
+        }
         SampleArgs sa{c.leaf_lo, leaf_kid, leaf_ord, c.leaf_moff, c.leaf_m, c.leaf_census, c.t_sorted,
                       c.row_sorted, L, n, S, (uint32_t)o.seed, (uint32_t)(o.seed >> 32), c.kid_base, c.out_row,
                       c.out_cluster, c.out_weight, c.leaf_U, c.pack_s, c.pack_h, c.sort_kid, c.sort_t,
@@ -667,6 +693,13 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         }
         c.stage_end(tk_smp, 40 * S);
         CK(cudaGetLastError());
+        if (c.early_plan) {   // the samples' host copies, beside the estimate
+            CK(cudaEventRecord(c.ev_d2h, st));
+            CK(cudaStreamWaitEvent(c.dstream, c.ev_d2h, 0));
+            CK(cudaMemcpyAsync(h_row, c.out_row, sizeof(uint32_t) * S, cudaMemcpyDeviceToHost, c.dstream));
+            CK(cudaMemcpyAsync(h_scl, c.out_cluster, sizeof(uint32_t) * S, cudaMemcpyDeviceToHost, c.dstream));
+            CK(cudaMemcpyAsync(h_w, c.out_weight, sizeof(double) * S, cudaMemcpyDeviceToHost, c.dstream));
+        }
 
         // a8: estimate, bound, metrics (deterministic block partials)
         mb = blocks_for(S);
@@ -698,15 +731,17 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
     c.stage_end(tk_est, 56 * L + 12 * S * nm);
     // ---- segment 4: cluster records, final scalars
     CKS(dist_checkpoint(c, [&]() -> int {
-        CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
-        const int tk_pack = c.stage_begin("pack");
-        if (L)
-            pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.PS1, c.PS2, c.t_sorted,
-                                                            c.leaf_m, c.leaf_census, L, n, c.kid_base,
-                                                            c.out_clusters);
-        c.launches++;
-        c.stage_end(tk_pack, 88 * L);
-        CK(cudaGetLastError());
+        if (!c.early_packed) {
+            CKS(c.ensure(c.out_clusters, c.cap_out_cl, sizeof(stem_cluster) * (L + 1)));
+            const int tk_pack = c.stage_begin("pack");
+            if (L)
+                pack_kernel<<<blocks_for(L), kThreads, 0, st>>>(c.leaf_lo, leaf_kid, leaf_ord, c.PS1, c.PS2,
+                                                                c.t_sorted, c.leaf_m, c.leaf_census, L, n, c.kid_base,
+                                                                c.out_clusters);
+            c.launches++;
+            c.stage_end(tk_pack, 88 * L);
+            CK(cudaGetLastError());
+        }
         double *est_out = red_out + 2 + nm;
         est_finalize_kernel<<<1, 1, 0, st>>>(&c.scalars->sum_q, red_out, &c.scalars->T, z, est_out);
         c.launches++;

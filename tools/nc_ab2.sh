@@ -1,5 +1,3 @@
-# descent-split variants (compile-time) and the sort's first-pass publication mode
-python -m pytest tests/test_gpu_parity.py tests/test_gpu_dist.py -x -q > gpurun_out/nc3_tests.txt 2>&1; echo rc=$? >> gpurun_out/nc3_tests.txt
-bash tools/ab_build.sh "-DSR_NC_SBEST=0" "-DSR_NC_SBEST=1" "-DSR_NC_SBEST=1 -DSR_NC_THREADS=128 -DSR_NC_MINB=9" > gpurun_out/nc3_ab.txt 2>&1
-python tools/sortbench/sortbench.py -- "" > gpurun_out/sb3.txt 2>&1
-STEMROOT_SORT_LATE_FIRST=0 python tools/sortbench/sortbench.py -- "" >> gpurun_out/sb3.txt 2>&1
+# descent-split variants (compile-time)
+python -m pytest tests/test_gpu_parity.py -x -q -k "nearest_centre or big_clusters or worked or tie or edge or configs or mixtures" > gpurun_out/nc4_tests.txt 2>&1; echo rc=$? >> gpurun_out/nc4_tests.txt
+bash tools/ab_build.sh "-DSR_NC_MINB=9" "-DSR_NC_MINB=8" "-DSR_NC_MINB=7" > gpurun_out/nc4_ab.txt 2>&1
