@@ -53,6 +53,9 @@ void Ctx::release() {
     if (dstream) { cudaStreamDestroy(dstream); dstream = nullptr; }
     if (ev_pack) { cudaEventDestroy(ev_pack); ev_pack = nullptr; }
     if (ev_d2h) { cudaEventDestroy(ev_d2h); ev_d2h = nullptr; }
+    for (auto &e : ev_h2d)
+        if (e) { cudaEventDestroy(e); e = nullptr; }
+    if (ev_pre) { cudaEventDestroy(ev_pre); ev_pre = nullptr; }
     if (ev_fork) cudaEventDestroy(ev_fork);
     if (ev_join) cudaEventDestroy(ev_join);
     if (side) cudaStreamDestroy(side);
@@ -172,11 +175,12 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
     CKS(c.ensure_all(n, K, nm));
     const uint32_t *kid = tr->kernel_id, *t = tr->exec_ns;
     const double *met = tr->metrics;
-    if (tr->device < 0) {   // host trace: copy in on the stream
+    const uint32_t *h_kid = nullptr, *h_t = nullptr;
+    if (tr->device < 0) {   // host trace: copied in by sort_trace, in chunks overlapped with its pre-pass
         CKS(c.ensure(c.in_kid, c.cap_in_kid, sizeof(uint32_t) * n));
         CKS(c.ensure(c.in_t, c.cap_in_t, sizeof(uint32_t) * n));
-        CK(cudaMemcpyAsync(c.in_kid, kid, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, c.stream));
-        CK(cudaMemcpyAsync(c.in_t, t, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, c.stream));
+        h_kid = kid;
+        h_t = t;
         kid = c.in_kid;
         t = c.in_t;
         if (nm) {
@@ -185,7 +189,7 @@ static int run_plan(Ctx &c, const stem_trace *tr, double eps, double conf, const
             met = c.in_met;
         }
     }
-    CKS(sort_trace(c, kid, t, nullptr, n, K, !o.census_cap));   // a1
+    CKS(sort_trace(c, kid, t, nullptr, n, K, !o.census_cap, h_kid, h_t));   // a1
     CKS(prefix_moments(c, n));                        // a2
     if (o.root && o.split == 3) {
         CKS(root_levels_kmeans(c, n, K, eps, z, k2, o.clamp_in_split ? 1 : 0, (uint32_t)o.kmeans_k));   // a3, a4

@@ -267,6 +267,8 @@ struct Ctx {
     void *early_plan = nullptr;                 // PlanBlock (capi.cu), or NULL
     cudaStream_t dstream = nullptr;
     cudaEvent_t ev_pack = nullptr, ev_d2h = nullptr;
+    cudaEvent_t ev_h2d[8] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    cudaEvent_t ev_pre = nullptr;
     bool early_packed = false;
 
     // last plan
@@ -293,8 +295,11 @@ int dist_allreduce_f64(Ctx &c, double *buf, size_t count);
 int dist_metric_sums(Ctx &c, const double *metrics_local, uint32_t nm, uint64_t S, double *out);
 
 // stages
+// h_kid/h_t (optional): the trace is in host memory and kid/t are its device
+// copies to fill; the copies go in chunks and the pre-pass consumes each chunk
+// as it lands (host-to-device traffic overlapped with the pre-pass)
 int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *row_in, uint64_t n,
-               uint32_t K, bool allow_pack);                                                   // a1
+               uint32_t K, bool allow_pack, const uint32_t *h_kid = nullptr, const uint32_t *h_t = nullptr);                                                   // a1
 int prefix_moments(Ctx &c, uint64_t n);                                                        // a2
 int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp,
                 int split, uint64_t seed);   // a3, a4 (split: 0 exact 2-means, 1 Lloyd, 2 k-means++ Lloyd)
@@ -355,7 +360,7 @@ struct DensePath {
 // split = 3: ROOT with exact optimal 1-D k-means splits into kk groups (kmeans.cu, R29)
 int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, uint32_t kk);
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,
-                      uint32_t *tailh);   // pre-pass only
+                      uint32_t *tailh, bool zero = true, cudaStream_t pst = nullptr);   // pre-pass only   // pre-pass only
 int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
                   const stem_opts &o, int local_status);
 // capi.cu: allocate the host plan block for L clusters, S samples (c.early_plan);

@@ -627,13 +627,18 @@ static int launch_sort_pass(const PassArgs &a, bool first, bool last, cudaStream
 }
 
 // the pre-pass alone (kernel-id counts and max t, range check): also the
-// multi-GPU histogram step.  Zeroes its outputs first.
-int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K, uint32_t *tailh) {
-    cudaStream_t st = c.stream;
-    CK(cudaMemsetAsync(c.hist, 0, sizeof(uint64_t) * (kMaxPasses + 1) * kHistR, st));
-    if (tailh) CK(cudaMemsetAsync(tailh, 0, sizeof(uint32_t) * kR * (uint64_t)K, st));
-    CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
-    CK(cudaMemsetAsync(c.kid_max, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
+// multi-GPU histogram step.  Zeroes its outputs first (zero = false: they
+// accumulate, for a trace handed over in chunks; pst = the launch stream).
+int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K, uint32_t *tailh,
+                      bool zero, cudaStream_t pst) {
+    cudaStream_t st = pst ? pst : c.stream;
+    if (zero) {
+        CK(cudaMemsetAsync(c.hist, 0, sizeof(uint64_t) * (kMaxPasses + 1) * kHistR, st));
+        if (tailh) CK(cudaMemsetAsync(tailh, 0, sizeof(uint32_t) * kR * (uint64_t)K, st));
+        CK(cudaMemsetAsync(c.kid_count, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
+        CK(cudaMemsetAsync(c.kid_max, 0, sizeof(uint32_t) * ((uint64_t)K + 1), st));
+    }
+    if (n == 0) return STEM_OK;
     const int smem_kid = (K <= 24000) ? 1 : 0;
     constexpr int kMaxNC = 8;
     auto bytes = [&](int nc) { return sizeof(uint32_t) * (nc * (3 * kR + 1) + (smem_kid ? 2 * (size_t)K : 0)); };
@@ -659,15 +664,56 @@ int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n
     return STEM_OK;
 }
 
+// chunks of a host trace's copy (pre-pass overlapped with the copy); STEMROOT_H2D_CHUNKS
+static int h2d_chunks(uint64_t n) {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("STEMROOT_H2D_CHUNKS");
+        v = e ? atoi(e) : 8;
+        v = v < 1 ? 1 : v > 8 ? 8 : v;
+    }
+    return n >= (1ull << 24) ? v : 1;
+}
+
 int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *row_in, uint64_t n, uint32_t K,
-               bool allow_pack) {
+               bool allow_pack, const uint32_t *h_kid, const uint32_t *h_t) {
     cudaStream_t st = c.stream;
     CK(cudaMemsetAsync(c.scalars, 0, sizeof(DevScalars), st));
-    const int tk_pre = c.stage_begin("prepass");
     // coarse bases are possible when the [K][256] tail histogram is small
     const bool coarse_ok = K <= kMaxTailK && !(getenv("STEMROOT_SORT_COARSE") && getenv("STEMROOT_SORT_COARSE")[0] == '0');
     if (coarse_ok) CKS(c.ensure(c.tailh, c.cap_tailh, sizeof(uint32_t) * kR * (uint64_t)K));
-    CKS(histogram_kernels(c, kid, t, n, K, coarse_ok ? c.tailh : nullptr));
+    uint32_t *tailh = coarse_ok ? c.tailh : nullptr;
+    const int nch = h_kid ? h2d_chunks(n) : 0;
+    if (nch > 1) {
+        // host trace: the copies run back to back on the plan's stream; the
+        // pre-pass of chunk i runs on dstream as soon as chunk i has landed
+        if (!c.dstream) {
+            CK(cudaStreamCreateWithFlags(&c.dstream, cudaStreamNonBlocking));
+            CK(cudaEventCreateWithFlags(&c.ev_pack, cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&c.ev_d2h, cudaEventDisableTiming));
+        }
+        for (int i = 0; i < nch; i++)
+            if (!c.ev_h2d[i]) CK(cudaEventCreateWithFlags(&c.ev_h2d[i], cudaEventDisableTiming));
+        if (!c.ev_pre) CK(cudaEventCreateWithFlags(&c.ev_pre, cudaEventDisableTiming));
+        CKS(histogram_kernels(c, nullptr, nullptr, 0, K, tailh, true, st));   // zero the outputs
+        const uint64_t step = ((n + nch - 1) / nch + 1023) & ~1023ull;
+        int used = 0;
+        for (uint64_t r0 = 0; r0 < n; r0 += step, used++) {
+            const uint64_t cnt = min(step, n - r0);
+            CK(cudaMemcpyAsync((void *)(kid + r0), h_kid + r0, sizeof(uint32_t) * cnt, cudaMemcpyHostToDevice, st));
+            CK(cudaMemcpyAsync((void *)(t + r0), h_t + r0, sizeof(uint32_t) * cnt, cudaMemcpyHostToDevice, st));
+            CK(cudaEventRecord(c.ev_h2d[used], st));
+            CK(cudaStreamWaitEvent(c.dstream, c.ev_h2d[used], 0));
+            CKS(histogram_kernels(c, kid + r0, t + r0, cnt, K, tailh, false, c.dstream));
+        }
+        CK(cudaEventRecord(c.ev_pre, c.dstream));
+        CK(cudaStreamWaitEvent(st, c.ev_pre, 0));
+    } else if (h_kid) {
+        CK(cudaMemcpyAsync((void *)kid, h_kid, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync((void *)t, h_t, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
+    }
+    const int tk_pre = c.stage_begin("prepass");
+    if (nch <= 1) CKS(histogram_kernels(c, kid, t, n, K, tailh, true, st));
     // key bases B = exclusive scan of W[k] = roundup(max_t[k] + 1, 2^16) (0 if
     // absent); Bc the same with 2^24
     const uint32_t *cnt = c.kid_count, *kmax = c.kid_max;

@@ -682,3 +682,12 @@ def test_nearest_centre_descent_ties(ctx, monkeypatch, golden):
     monkeypatch.setenv("STEMROOT_SPLIT_NC", "2")
     test_exact_tie_split(ctx, golden)
     test_worked_trees(ctx, golden)
+
+
+def test_host_trace_chunked_copy(ctx):
+    """A host trace of >= 2^24 rows is copied in chunks, each consumed by the
+    pre-pass as it lands (sort.cu h2d_chunks): the plan equals the oracle's."""
+    sp = G.spec("C4", n=(1 << 24) + 4099)
+    kid, t, _ = G.generate_np(sp)
+    got, ref = _both(ctx, kid, t, sp.n_kernels, host=True, eps=sp.eps, seed=5)
+    assert_plans_equal(got, ref)
