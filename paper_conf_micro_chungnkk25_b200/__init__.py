@@ -27,7 +27,9 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _ROOT = os.path.dirname(_HERE)
 _CSRC = os.path.join(_HERE, "csrc")
-LIB_PATH = os.path.join(_HERE, "lib", "libstemroot.so")
+# STEMROOT_LIB: another build of the same sources (the bounds-checked -DSR_CHECK
+# build of tests/test_gpu_checked.py); default the in-tree libstemroot.so
+LIB_PATH = os.environ.get("STEMROOT_LIB") or os.path.join(_HERE, "lib", "libstemroot.so")
 HEADER = os.path.join(_ROOT, "include", "stemroot.h")
 SOURCES = ["capi.cu", "sort.cu", "root.cu", "stem.cu", "dist.cu", "metric.cu", "kmeans.cu"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "--fmad=false",

@@ -8,6 +8,23 @@
 typedef unsigned __int128 u128;
 typedef __int128 i128;
 
+// Device-side bounds checks of the checked build (-DSR_CHECK: tests/test_gpu_checked.py,
+// the stand-in for compute-sanitizer's memcheck where the GPU pool disables it).
+// A failed check prints its site and traps (the context dies, the call fails loudly).
+#ifdef SR_CHECK
+#include <cstdio>
+#define SR_DCHECK(cond)                                                                  \
+    do {                                                                                 \
+        if (!(cond)) {                                                                   \
+            printf("SR_CHECK failed at %s:%d: %s (block %d thread %d)\n", __FILE__, __LINE__, #cond, \
+                   (int)blockIdx.x, (int)threadIdx.x);                                   \
+            __trap();                                                                    \
+        }                                                                                \
+    } while (0)
+#else
+#define SR_DCHECK(cond) do { } while (0)
+#endif
+
 namespace sr {
 
 constexpr int kWarp = 32;

@@ -6,7 +6,8 @@
 //
 // The k-means is the dynamic program over the cluster's distinct values
 //   F[1][b] = S(0,b)^2 / n(0,b),  F[j][b] = max_a F[j-1][a] + S(a,b)^2 / n(a,b)
-// (maximising sum_g S_g^2 / n_g = minimising the SSE).  The group cost obeys
+// (maximising sum_g S_g^2 / n_g = minimising the SSE), evaluated in fp64 in its
+// between-group form (km_between below) and only for b = d in the last layer.  The group cost obeys
 // the quadrangle inequality, so the smallest optimal a is non-decreasing in b
 // and each layer is solved by divide and conquer in O(d log d): one warp per
 // cluster, 32 candidate a per step.  Values are fp64; candidates within 2^-40
@@ -129,11 +130,6 @@ __device__ __noinline__ void km_exact(const KmArgs &g, const KmCluster &c, uint3
     kfrac_add(out, km_P(g, c, b) - km_P(g, c, a), km_pos(g, c, b) - km_pos(g, c, a));
 }
 
-__device__ __forceinline__ double km_score(const KmArgs &g, const KmCluster &c, uint32_t a, uint32_t b) {
-    const double s = rn64(km_P(g, c, b) - km_P(g, c, a));
-    return __ddiv_rn(__dmul_rn(s, s), rn64(km_pos(g, c, b) - km_pos(g, c, a)));
-}
-
 // ---------------------------------------------------------------- the DP, level-synchronous divide and conquer
 // Layer j of every active cluster at once: a subproblem (cluster, b range,
 // a range) takes b = mid of its range, finds the best a for it and hands the
@@ -149,8 +145,27 @@ struct KmMeta {          // per frontier cluster
     uint32_t d, K;
 };
 
+// Between-group form of the DP (the fp64 filter's values): G[j][b] = F[j][b] -
+// S(0,b)^2/n(0,b) = max_a G[j-1][a] + T(a,b), G[1][b] = 0, with
+// T(a,b) = S(0,a)^2/n(0,a) + S(a,b)^2/n(a,b) - S(0,b)^2/n(0,b)
+//        = (n(a,b) S(0,a) - n(0,a) S(a,b))^2 / (n(0,a) n(a,b) n(0,b)),
+// the numerator exact in 128 bits (<= 0 inside the difference for sorted
+// values).  For a fixed b the order of G[j-1][a] + T(a,b) is the order of
+// F[j-1][a] + S(a,b)^2/n(a,b) (they differ by a constant), so the exact
+// comparison of near ties is unchanged; but G has no large common part, so
+// the 2^-40 filter flags far fewer near ties than F = sum S^2/n did (C5: the
+// sums are ~1e20 while candidates differ by ~1e9).
+__device__ __forceinline__ double km_between(const KmArgs &g, const KmCluster &c, uint32_t a, uint32_t b) {
+    const uint64_t na = km_pos(g, c, a), nb = km_pos(g, c, b), nab = nb - na;
+    const uint64_t Sa = km_P(g, c, a), Sab = km_P(g, c, b) - Sa;
+    const u128 l = (u128)na * Sab, r = (u128)nab * Sa;   // n(0,a) S(a,b) >= n(a,b) S(0,a) for sorted values
+    const u128 D = l >= r ? l - r : r - l;
+    const double dD = rn128(D);
+    return __ddiv_rn(__dmul_rn(dD, dD), __dmul_rn(__dmul_rn(rn64(na), rn64(nab)), rn64(nb)));
+}
+
 __device__ __forceinline__ double km_value(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t a, uint32_t b) {
-    return __dadd_rn(g.F[(size_t)(j - 1) * (g.D + 1) + c.D0 + a], km_score(g, c, a, b));
+    return __dadd_rn(g.F[(size_t)(j - 1) * (g.D + 1) + c.D0 + a], km_between(g, c, a, b));
 }
 
 // exact winner among the candidates a in list[0..m) (ascending), any thread
@@ -201,9 +216,41 @@ __device__ __forceinline__ KmCluster km_cluster(const KmMeta &m) {
     return c;
 }
 
+// running (best value, its smallest a, second best value) of a candidate scan;
+// the second best counts an equal best value, so a unique winner is certain
+// when second < best (1 - 2^-40) and the near-tie pass can be skipped
+struct KmTop {
+    double v1, v2;
+    uint32_t a1;
+};
+__device__ __forceinline__ void km_top_add(KmTop &t, double v, uint32_t a) {
+    if (v > t.v1) { t.v2 = t.v1; t.v1 = v; t.a1 = a; }
+    else if (v == t.v1) { t.v2 = v; if (a < t.a1) t.a1 = a; }
+    else if (v > t.v2) t.v2 = v;
+}
+__device__ __forceinline__ KmTop km_top_merge(const KmTop &x, const KmTop &y) {
+    KmTop r;
+    if (x.v1 > y.v1) { r.v1 = x.v1; r.a1 = x.a1; r.v2 = fmax(x.v2, y.v1); }
+    else if (y.v1 > x.v1) { r.v1 = y.v1; r.a1 = y.a1; r.v2 = fmax(y.v2, x.v1); }
+    else { r.v1 = x.v1; r.a1 = min(x.a1, y.a1); r.v2 = x.v1; }
+    return r;
+}
+__device__ __forceinline__ KmTop km_top_warp(KmTop t) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        KmTop y;
+        y.v1 = __shfl_xor_sync(0xffffffffu, t.v1, o);
+        y.v2 = __shfl_xor_sync(0xffffffffu, t.v2, o);
+        y.a1 = __shfl_xor_sync(0xffffffffu, t.a1, o);
+        t = km_top_merge(t, y);
+    }
+    return t;
+}
+
 // subproblems with long a ranges: one block each
 __global__ void __launch_bounds__(256) km_step_block_kernel(KmStep s) {
-    __shared__ double s_v[8];
+    __shared__ double s_v[8], s_v2[8];
+    __shared__ uint32_t s_a[8];
     __shared__ uint32_t s_list[kKmNear];
     __shared__ uint32_t s_m;
     const uint32_t n = *s.ncur;
@@ -214,23 +261,25 @@ __global__ void __launch_bounds__(256) km_step_block_kernel(KmStep s) {
         const uint32_t a0 = x.alo, a1 = min(x.ahi, mid - 1);
         if (a1 - a0 + 1 <= kKmLong) continue;   // the warp kernel's
         const KmCluster c = km_cluster(s.meta[x.c]);
-        double vm = -1.0;
-        for (uint32_t a = a0 + tid; a <= a1; a += 256) vm = fmax(vm, km_value(s.g, c, s.j, a, mid));
-#pragma unroll
-        for (int o = 16; o; o >>= 1) vm = fmax(vm, __shfl_xor_sync(0xffffffffu, vm, o));
-        if (lane == 0) s_v[w] = vm;
+        KmTop tp{-1.0, -1.0, 0xFFFFFFFFu};
+        for (uint32_t a = a0 + tid; a <= a1; a += 256) km_top_add(tp, km_value(s.g, c, s.j, a, mid), a);
+        tp = km_top_warp(tp);
+        if (lane == 0) { s_v[w] = tp.v1; s_v2[w] = tp.v2; s_a[w] = tp.a1; }
         if (tid == 0) s_m = 0;
         __syncthreads();
-        double top = s_v[0];
-        for (int k = 1; k < 8; k++) top = fmax(top, s_v[k]);
-        const double thr = __dmul_rn(top, 1.0 - 0x1p-40);
-        for (uint32_t a = a0 + tid; a <= a1; a += 256)
-            if (km_value(s.g, c, s.j, a, mid) >= thr) {
-                const uint32_t q = atomicAdd(&s_m, 1u);
-                if (q < (uint32_t)kKmNear) s_list[q] = a;
-            }
+        KmTop top{s_v[0], s_v2[0], s_a[0]};
+        for (int k = 1; k < 8; k++) top = km_top_merge(top, KmTop{s_v[k], s_v2[k], s_a[k]});
+        const double thr = __dmul_rn(top.v1, 1.0 - 0x1p-40);
+        const bool unique = top.v2 < thr;   // every other candidate is below the near-tie band
+        if (!unique)
+            for (uint32_t a = a0 + tid; a <= a1; a += 256)
+                if (km_value(s.g, c, s.j, a, mid) >= thr) {
+                    const uint32_t q = atomicAdd(&s_m, 1u);
+                    if (q < (uint32_t)kKmNear) s_list[q] = a;
+                }
         __syncthreads();
         if (tid == 0) {
+            if (unique) { s_list[0] = top.a1; s_m = 1; }
             uint32_t m = min(s_m, (uint32_t)kKmNear), best;
             for (uint32_t p = 1; p < m; p++)   // ascending a (insertion sort of a few entries)
                 for (uint32_t q = p; q > 0 && s_list[q - 1] > s_list[q]; q--) {
@@ -259,12 +308,15 @@ __global__ void __launch_bounds__(256) km_step_warp_kernel(KmStep s) {
         const uint32_t a0 = x.alo, a1 = min(x.ahi, mid - 1);
         if (a1 - a0 + 1 > kKmLong) continue;    // the block kernel's
         const KmCluster c = km_cluster(s.meta[x.c]);
-        double vm = -1.0;
-        for (uint32_t a = a0 + lane; a <= a1; a += 32) vm = fmax(vm, km_value(s.g, c, s.j, a, mid));
-#pragma unroll
-        for (int o = 16; o; o >>= 1) vm = fmax(vm, __shfl_xor_sync(0xffffffffu, vm, o));
-        const double thr = __dmul_rn(vm, 1.0 - 0x1p-40);
+        KmTop tp{-1.0, -1.0, 0xFFFFFFFFu};
+        for (uint32_t a = a0 + lane; a <= a1; a += 32) km_top_add(tp, km_value(s.g, c, s.j, a, mid), a);
+        tp = km_top_warp(tp);
+        const double thr = __dmul_rn(tp.v1, 1.0 - 0x1p-40);
         uint32_t m = 0;
+        if (tp.v2 < thr) {   // a unique winner: no near-tie pass
+            if (lane == 0) s_list[w][0] = tp.a1;
+            m = 1;
+        } else
         for (uint32_t base = a0; base <= a1; base += 32) {   // near-tie candidates, ascending
             const uint32_t a = base + lane;
             const bool near = a <= a1 && km_value(s.g, c, s.j, a, mid) >= thr;
@@ -303,11 +355,12 @@ __global__ void __launch_bounds__(256) km_prep_kernel(KmArgs g, KmMeta *meta, Km
         m.d = (uint32_t)(lower_bound(g.dpos, g.D + 1, (uint32_t)hi) - m.D0);
         m.K = min(g.k, m.d);
         const KmCluster c = km_cluster(m);
-        for (uint32_t b = 1 + lane; b <= m.d; b += 32) g.F[(g.D + 1) + c.D0 + b] = km_score(g, c, 0, b);
+        for (uint32_t b = 1 + lane; b <= m.d; b += 32) g.F[(g.D + 1) + c.D0 + b] = 0.0;   // G[1][b] (one group)
         if (lane == 0) {
             meta[ci] = m;
             g.ngrp[ci] = 0;
-            if (m.K >= 2) sub[atomicAdd(nsub, 1u)] = KmSub{(uint32_t)ci, 2, m.d, 1, m.d - 1, 0};
+            // the last layer needs b = d only (the backtrack starts there)
+            if (m.K >= 2) sub[atomicAdd(nsub, 1u)] = KmSub{(uint32_t)ci, m.K == 2 ? m.d : 2, m.d, 1, m.d - 1, 0};
         }
     }
 }
@@ -317,7 +370,7 @@ __global__ void km_layer_kernel(const uint64_t *ctot, const KmMeta *meta, uint32
     const uint64_t ci = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (ci >= (*ctot >> 32)) return;
     const KmMeta m = meta[ci];
-    if (m.K >= j) sub[atomicAdd(nsub, 1u)] = KmSub{(uint32_t)ci, j, m.d, j - 1, m.d - 1, 0};
+    if (m.K >= j) sub[atomicAdd(nsub, 1u)] = KmSub{(uint32_t)ci, m.K == j ? m.d : j, m.d, j - 1, m.d - 1, 0};
 }
 
 // backtrack the cuts

@@ -435,6 +435,7 @@ __device__ __forceinline__ double chunk_ad_bound(double A, uint64_t n, uint64_t 
 __device__ __forceinline__ void scan_chunk(const uint32_t *__restrict__ t, uint64_t lo, uint64_t n, uint64_t S,
                                            uint64_t ra, uint64_t rb, uint64_t SLa, Cand &best) {
     const int lane = threadIdx.x & 31;
+    SR_DCHECK(ra >= lo && rb <= lo + n && rb - ra <= 32);
     const uint64_t row = ra + lane;
     const bool in = row < rb;
     const uint32_t tc = in ? t[row] : 0u;
@@ -728,6 +729,7 @@ __global__ void __launch_bounds__(SR_NC_THREADS, SR_NC_MINB) nc_split_kernel(con
                 bool keep = false;
                 uint64_t SLs = 0;
                 if (in) {
+                    SR_DCHECK(s0 >= C0 && s1 + 1 <= (uint32_t)C1s + 1 && ((uint64_t)(s1 + 1) << kChunkLog) < hi);
                     const uint64_t pa = PS1[s0], pb = PS1[s1 + 1];
                     const uint32_t tam1 = TB2[s0].x, tb = TB2[s1 + 1].x;   // t[32 s0 - 1], t[32 s1 + 31]
                     SLs = pa - base;
@@ -747,6 +749,7 @@ __global__ void __launch_bounds__(SR_NC_THREADS, SR_NC_MINB) nc_split_kernel(con
                     }
                 } else {
                     const int below = __popc(live & ((1u << lane) - 1));
+                    SR_DCHECK(sp + __popc(live) <= kNcStack);
                     if (keep) stk[sp + __popc(live) - 1 - below] = make_uint2(s0, s1);   // leftmost on top
                     sp += __popc(live);
                     __syncwarp();
@@ -1317,6 +1320,7 @@ __global__ void __launch_bounds__(256) decide_kernel(DecideArgs a) {
     if (lane == 31 && wtot) base = atomicAdd((unsigned long long *)a.total, (unsigned long long)wtot);
     base = __shfl_sync(0xffffffffu, base, 31);
     uint32_t idx = (uint32_t)((base + incl - mine) >> 32);
+    SR_DCHECK(!(ntL || ntR) || idx + (ntL ? 1u : 0u) + (ntR ? 1u : 0u) <= 2u * (uint32_t)(*a.ctot >> 32));
     if (ntL) {
         a.nlo[idx] = lo; a.nhi[idx] = mid;
         a.nS[idx] = SL; a.nQ[idx] = QL;

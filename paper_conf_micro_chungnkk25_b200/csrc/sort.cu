@@ -489,6 +489,7 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
 #else
             const uint32_t lp = s_lstart[dd] + s_whist[w][dd] + ((rank2[j / 2] >> (16 * (j & 1))) & 0xffffu);
 #endif
+            SR_DCHECK(lp < (uint32_t)TILE);
             s_keys[lp] = key[j];
             if (!PK) s_vals[lp] = val[PK ? 0 : j];
         }
@@ -531,6 +532,7 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
         const uint64_t k = s_keys[i];
         const uint32_t dd = (uint32_t)(k >> a.shift) & (R - 1);
         uint32_t gp = s_delta[dd] + i;
+        SR_DCHECK(gp < a.n);
 #ifdef SR_SORT_FAKE_LB
         if (gp >= a.n) gp = (uint32_t)(a.n - 1);
 #endif

@@ -280,6 +280,7 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
         const uint64_t r = (j & 1) ? (((uint64_t)x.w << 32) | x.z) : (((uint64_t)x.y << 32) | x.x);
         pos = lo + __umul64hi(r, n);
     }
+    SR_DCHECK(i < a.L && j < m && pos >= lo && pos < hi);
     const uint32_t tv = a.t[pos];
     if (a.pack_h == 0) {
         a.out_row[s] = a.row[pos];
@@ -310,6 +311,7 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
                 a.out_row[s] = map_row(a, (uint32_t)(((uint64_t)(__ffsll(mask) - 1) << a.pack_s) | low));
             } else {   // resolved by resolve_kernel: which of the matches sits at pos
                 const uint32_t e = atomicAdd(a.amb_count, 1u);
+                SR_DCHECK(e < a.S && __popcll(mask) >= 1);
                 a.amb[e] = Amb{mask, (uint32_t)s, (uint32_t)i, (uint32_t)pos, low};
             }
         }
