@@ -51,7 +51,7 @@ struct DevScalars {
     unsigned long long local_rows;        // rows scanned below the frontier (local subtrees)
     unsigned long long split_chunks, split_scanned;   // big-cluster chunks bounded / scanned row by row
     uint32_t local_depth, amb_count;      // deepest ROOT level of a local subtree; ambiguous samples
-    uint32_t km_nsub[2];                  // split = 3: subproblems of the current / next D&C round
+    uint32_t km_nsub[4];                  // split = 3: subproblems [short, long][current / next D&C round]
     uint32_t nc_queue[2];                 // nearest-centre descent: next cluster of the level's work queue (by level parity)
 };
 

@@ -94,7 +94,8 @@ struct KmArgs {
     const uint32_t *dpos;          // [D + 1] rows starting a distinct value (dpos[D] = n)
     const uint64_t *dP;            // [D + 1] exact sum of t before them
     uint64_t D;
-    double *F;                     // [k + 1][D + 1] fp64 DP values (layers 1..k)
+    double *F;                     // [k + 1][D + 1] fp64 DP values (layers 1..k): the high part of
+    double *Flo;                   // [k + 1][D + 1] their double-double low part
     uint32_t *arg;                 // [k + 1][D + 1] argmax (distinct index relative to the cluster)
     uint32_t k;
     uint32_t *cutk;                // [cluster][kKmMax - 1] cuts relative to lo
@@ -164,6 +165,82 @@ __device__ __forceinline__ double km_between(const KmArgs &g, const KmCluster &c
     return __ddiv_rn(__dmul_rn(dD, dD), __dmul_rn(__dmul_rn(rn64(na), rn64(nab)), rn64(nb)));
 }
 
+__device__ __noinline__ uint32_t km_exact_best(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t b,
+                                               const uint32_t *list, uint32_t m);
+
+// ---- double-double (~2^-100 relative) values: the second filter between the
+// fp64 scan (2^-40 band) and the exact 768-bit comparison
+struct KDD {
+    double hi, lo;
+};
+__device__ __forceinline__ KDD kdd_qsum(double a, double b) {
+    const double s = __dadd_rn(a, b);
+    return KDD{s, __dsub_rn(b, __dsub_rn(s, a))};
+}
+__device__ __forceinline__ KDD kdd_sum(double a, double b) {
+    const double s = __dadd_rn(a, b), bb = __dsub_rn(s, a);
+    return KDD{s, __dadd_rn(__dsub_rn(a, __dsub_rn(s, bb)), __dsub_rn(b, bb))};
+}
+__device__ __forceinline__ KDD kdd_add(KDD a, KDD b) {
+    KDD s = kdd_sum(a.hi, b.hi);
+    const KDD t = kdd_sum(a.lo, b.lo);
+    s = kdd_qsum(s.hi, __dadd_rn(s.lo, t.hi));
+    return kdd_qsum(s.hi, __dadd_rn(s.lo, t.lo));
+}
+__device__ __forceinline__ KDD kdd_mul(KDD a, KDD b) {
+    const double p = __dmul_rn(a.hi, b.hi);
+    double e = __fma_rn(a.hi, b.hi, -p);
+    e = __dadd_rn(e, __dadd_rn(__dmul_rn(a.hi, b.lo), __dmul_rn(a.lo, b.hi)));
+    return kdd_qsum(p, e);
+}
+__device__ __forceinline__ KDD kdd_mul_d(KDD a, double b) {
+    const double p = __dmul_rn(a.hi, b);
+    const double e = __dadd_rn(__fma_rn(a.hi, b, -p), __dmul_rn(a.lo, b));
+    return kdd_qsum(p, e);
+}
+__device__ __forceinline__ KDD kdd_div(KDD a, KDD b) {
+    const double q1 = __ddiv_rn(a.hi, b.hi);
+    KDD r = kdd_add(a, kdd_mul_d(b, -q1));
+    const double q2 = __ddiv_rn(r.hi, b.hi);
+    r = kdd_add(r, kdd_mul_d(b, -q2));
+    const double q3 = __ddiv_rn(r.hi, b.hi);
+    return kdd_add(kdd_qsum(q1, q2), KDD{q3, 0.0});
+}
+__device__ __forceinline__ KDD kdd_u128(u128 x) {   // exact for x < 2^106
+    const uint64_t h = (uint64_t)(x >> 53), l = (uint64_t)x & ((1ull << 53) - 1);
+    return kdd_sum(__dmul_rn((double)h, 0x1p53), (double)l);
+}
+__device__ __forceinline__ bool kdd_gt(KDD a, KDD b) { return a.hi > b.hi || (a.hi == b.hi && a.lo > b.lo); }
+
+// G[j-1][a] + T(a,b) in double-double
+__device__ __forceinline__ KDD km_value_dd(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t a, uint32_t b) {
+    const uint64_t na = km_pos(g, c, a), nb = km_pos(g, c, b), nab = nb - na;
+    const uint64_t Sa = km_P(g, c, a), Sab = km_P(g, c, b) - Sa;
+    const u128 l = (u128)na * Sab, r = (u128)nab * Sa;
+    const KDD D = kdd_u128(l >= r ? l - r : r - l);   // < 2^96
+    const KDD T = kdd_div(kdd_mul(D, D), kdd_u128((u128)(na * nab) * nb));
+    const size_t idx = (size_t)(j - 1) * (g.D + 1) + c.D0 + a;
+    return kdd_add(KDD{g.F[idx], g.Flo[idx]}, T);
+}
+
+// The winner among near-tie candidates (ascending): by double-double values
+// when one beats every other by more than 2^-90 relative (their errors are
+// below 2^-96), else by the exact comparison
+__device__ __noinline__ uint32_t km_near_best(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t b,
+                                              const uint32_t *list, uint32_t m) {
+    if (m == 1) return list[0];
+    KDD v1 = km_value_dd(g, c, j, list[0], b), v2{-1.0, 0.0};
+    uint32_t a1 = list[0];
+    for (uint32_t i = 1; i < m; i++) {
+        const KDD v = km_value_dd(g, c, j, list[i], b);
+        if (kdd_gt(v, v1)) { v2 = v1; v1 = v; a1 = list[i]; }
+        else if (kdd_gt(v, v2)) v2 = v;
+    }
+    const KDD thr = kdd_add(v1, KDD{__dmul_rn(-v1.hi, 0x1p-90), 0.0});
+    if (kdd_gt(thr, v2)) return a1;
+    return km_exact_best(g, c, j, b, list, m);
+}
+
 __device__ __forceinline__ double km_value(const KmArgs &g, const KmCluster &c, uint32_t j, uint32_t a, uint32_t b) {
     return __dadd_rn(g.F[(size_t)(j - 1) * (g.D + 1) + c.D0 + a], km_between(g, c, a, b));
 }
@@ -184,28 +261,34 @@ __device__ __noinline__ uint32_t km_exact_best(const KmArgs &g, const KmCluster 
     return best;
 }
 
+// Subproblems travel in two lists by the length of their a range (short: a
+// warp each, long: a block each), so neither kernel walks the other's entries.
 struct KmStep {
     KmArgs g;
     const KmMeta *meta;
-    const KmSub *cur;
-    const uint32_t *ncur;
-    KmSub *nxt;
-    uint32_t *nnxt;
+    const KmSub *cur[2];      // [short, long]
+    const uint32_t *ncur[2];
+    KmSub *nxt[2];
+    uint32_t *nnxt[2];
     uint32_t j;
 };
 
 constexpr uint32_t kKmLong = 512;   // a ranges longer than this get a block
 constexpr int kKmNear = 256;        // near-tie candidates resolved exactly per subproblem
 
+// the list a subproblem belongs to: 1 (long) when its b = mid scans more than kKmLong candidates
+__device__ __forceinline__ int km_cls(const KmSub &x) {
+    const uint32_t mid = x.blo + (x.bhi - x.blo) / 2;
+    return min(x.ahi, mid - 1) - x.alo + 1 > kKmLong ? 1 : 0;
+}
+__device__ __forceinline__ void km_push(KmSub *const *lst, uint32_t *const *cnt, const KmSub &x) {
+    const int k = km_cls(x);
+    lst[k][atomicAdd(cnt[k], 1u)] = x;
+}
+
 __device__ __forceinline__ void km_emit(const KmStep &s, const KmSub &x, uint32_t mid, uint32_t a) {
-    KmSub ch[2];
-    int nc = 0;
-    if (mid > x.blo) ch[nc++] = KmSub{x.c, x.blo, mid - 1, x.alo, a, 0};
-    if (mid < x.bhi) ch[nc++] = KmSub{x.c, mid + 1, x.bhi, a, x.ahi, 0};
-    if (nc) {
-        const uint32_t o = atomicAdd(s.nnxt, (uint32_t)nc);
-        for (int i = 0; i < nc; i++) s.nxt[o + i] = ch[i];
-    }
+    if (mid > x.blo) km_push(s.nxt, s.nnxt, KmSub{x.c, x.blo, mid - 1, x.alo, a, 0});
+    if (mid < x.bhi) km_push(s.nxt, s.nnxt, KmSub{x.c, mid + 1, x.bhi, a, x.ahi, 0});
 }
 
 __device__ __forceinline__ KmCluster km_cluster(const KmMeta &m) {
@@ -253,13 +336,12 @@ __global__ void __launch_bounds__(256) km_step_block_kernel(KmStep s) {
     __shared__ uint32_t s_a[8];
     __shared__ uint32_t s_list[kKmNear];
     __shared__ uint32_t s_m;
-    const uint32_t n = *s.ncur;
+    const uint32_t n = *s.ncur[1];
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     for (uint32_t i = blockIdx.x; i < n; i += gridDim.x) {
-        const KmSub x = s.cur[i];
+        const KmSub x = s.cur[1][i];
         const uint32_t mid = x.blo + (x.bhi - x.blo) / 2;
         const uint32_t a0 = x.alo, a1 = min(x.ahi, mid - 1);
-        if (a1 - a0 + 1 <= kKmLong) continue;   // the warp kernel's
         const KmCluster c = km_cluster(s.meta[x.c]);
         KmTop tp{-1.0, -1.0, 0xFFFFFFFFu};
         for (uint32_t a = a0 + tid; a <= a1; a += 256) km_top_add(tp, km_value(s.g, c, s.j, a, mid), a);
@@ -285,9 +367,11 @@ __global__ void __launch_bounds__(256) km_step_block_kernel(KmStep s) {
                 for (uint32_t q = p; q > 0 && s_list[q - 1] > s_list[q]; q--) {
                     const uint32_t t = s_list[q]; s_list[q] = s_list[q - 1]; s_list[q - 1] = t;
                 }
-            best = m == 1 ? s_list[0] : km_exact_best(s.g, c, s.j, mid, s_list, m);
+            best = km_near_best(s.g, c, s.j, mid, s_list, m);
             const size_t L = s.g.D + 1;
-            s.g.F[(size_t)s.j * L + c.D0 + mid] = km_value(s.g, c, s.j, best, mid);
+            const KDD vb = km_value_dd(s.g, c, s.j, best, mid);
+            s.g.F[(size_t)s.j * L + c.D0 + mid] = vb.hi;
+            s.g.Flo[(size_t)s.j * L + c.D0 + mid] = vb.lo;
             s.g.arg[(size_t)s.j * L + c.D0 + mid] = best;
             km_emit(s, x, mid, best);
             if (s_m > (uint32_t)kKmNear) atomicOr(s.g.ngrp + x.c, 0x80000000u);   // flagged: too many near ties
@@ -299,14 +383,13 @@ __global__ void __launch_bounds__(256) km_step_block_kernel(KmStep s) {
 // subproblems with short a ranges: one warp each
 __global__ void __launch_bounds__(256) km_step_warp_kernel(KmStep s) {
     __shared__ uint32_t s_list[8][kKmNear];   // 8 KB
-    const uint32_t n = *s.ncur;
+    const uint32_t n = *s.ncur[0];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t i = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += nwarps) {
-        const KmSub x = s.cur[i];
+        const KmSub x = s.cur[0][i];
         const uint32_t mid = x.blo + (x.bhi - x.blo) / 2;
         const uint32_t a0 = x.alo, a1 = min(x.ahi, mid - 1);
-        if (a1 - a0 + 1 > kKmLong) continue;    // the block kernel's
         const KmCluster c = km_cluster(s.meta[x.c]);
         KmTop tp{-1.0, -1.0, 0xFFFFFFFFu};
         for (uint32_t a = a0 + lane; a <= a1; a += 32) km_top_add(tp, km_value(s.g, c, s.j, a, mid), a);
@@ -330,9 +413,11 @@ __global__ void __launch_bounds__(256) km_step_warp_kernel(KmStep s) {
         __syncwarp();
         if (lane == 0) {
             const uint32_t mm = min(m, (uint32_t)kKmNear);
-            const uint32_t best = mm == 1 ? s_list[w][0] : km_exact_best(s.g, c, s.j, mid, s_list[w], mm);
+            const uint32_t best = km_near_best(s.g, c, s.j, mid, s_list[w], mm);
             const size_t L = s.g.D + 1;
-            s.g.F[(size_t)s.j * L + c.D0 + mid] = km_value(s.g, c, s.j, best, mid);
+            const KDD vb = km_value_dd(s.g, c, s.j, best, mid);
+            s.g.F[(size_t)s.j * L + c.D0 + mid] = vb.hi;
+            s.g.Flo[(size_t)s.j * L + c.D0 + mid] = vb.lo;
             s.g.arg[(size_t)s.j * L + c.D0 + mid] = best;
             km_emit(s, x, mid, best);
             if (m > (uint32_t)kKmNear) atomicOr(s.g.ngrp + x.c, 0x80000000u);
@@ -343,7 +428,11 @@ __global__ void __launch_bounds__(256) km_step_warp_kernel(KmStep s) {
 
 // per cluster: its distinct-value slice, K = min(k, d), layer 1, and the
 // layer-2 subproblem; one warp per cluster
-__global__ void __launch_bounds__(256) km_prep_kernel(KmArgs g, KmMeta *meta, KmSub *sub, uint32_t *nsub) {
+struct KmLists {
+    KmSub *lst[2];
+    uint32_t *cnt[2];
+};
+__global__ void __launch_bounds__(256) km_prep_kernel(KmArgs g, KmMeta *meta, KmLists L) {
     const uint32_t C = (uint32_t)(*g.ctot >> 32);
     const int lane = threadIdx.x & 31;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
@@ -355,22 +444,25 @@ __global__ void __launch_bounds__(256) km_prep_kernel(KmArgs g, KmMeta *meta, Km
         m.d = (uint32_t)(lower_bound(g.dpos, g.D + 1, (uint32_t)hi) - m.D0);
         m.K = min(g.k, m.d);
         const KmCluster c = km_cluster(m);
-        for (uint32_t b = 1 + lane; b <= m.d; b += 32) g.F[(g.D + 1) + c.D0 + b] = 0.0;   // G[1][b] (one group)
+        for (uint32_t b = 1 + lane; b <= m.d; b += 32) {   // G[1][b] = 0 (one group)
+            g.F[(g.D + 1) + c.D0 + b] = 0.0;
+            g.Flo[(g.D + 1) + c.D0 + b] = 0.0;
+        }
         if (lane == 0) {
             meta[ci] = m;
             g.ngrp[ci] = 0;
             // the last layer needs b = d only (the backtrack starts there)
-            if (m.K >= 2) sub[atomicAdd(nsub, 1u)] = KmSub{(uint32_t)ci, m.K == 2 ? m.d : 2, m.d, 1, m.d - 1, 0};
+            if (m.K >= 2) km_push(L.lst, L.cnt, KmSub{(uint32_t)ci, m.K == 2 ? m.d : 2, m.d, 1, m.d - 1, 0});
         }
     }
 }
 
 // the next layer's root subproblems
-__global__ void km_layer_kernel(const uint64_t *ctot, const KmMeta *meta, uint32_t j, KmSub *sub, uint32_t *nsub) {
+__global__ void km_layer_kernel(const uint64_t *ctot, const KmMeta *meta, uint32_t j, KmLists L) {
     const uint64_t ci = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (ci >= (*ctot >> 32)) return;
     const KmMeta m = meta[ci];
-    if (m.K >= j) sub[atomicAdd(nsub, 1u)] = KmSub{(uint32_t)ci, m.K == j ? m.d : j, m.d, j - 1, m.d - 1, 0};
+    if (m.K >= j) km_push(L.lst, L.cnt, KmSub{(uint32_t)ci, m.K == j ? m.d : j, m.d, j - 1, m.d - 1, 0});
 }
 
 // backtrack the cuts
@@ -552,7 +644,7 @@ int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, dou
     CK(cudaStreamSynchronize(st));
     kmeans_sentinel_kernel<<<1, 32, 0, st>>>(c.PS1, c.t_sorted, n, c.km_dpos + D, c.km_dP + D);   // dpos[D] = n
     c.launches++;
-    CKS(c.ensure(c.km_F, c.cap_km_F, sizeof(double) * (size_t)(kk + 1) * (D + 1)));
+    CKS(c.ensure(c.km_F, c.cap_km_F, 2 * sizeof(double) * (size_t)(kk + 1) * (D + 1)));   // high and low parts
     CKS(c.ensure(c.km_arg, c.cap_km_arg, sizeof(uint32_t) * (size_t)(kk + 1) * (D + 1)));
     // initial frontier
     uint64_t Cmax = (uint64_t)K + 1;
@@ -587,30 +679,38 @@ int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, dou
         CKS(c.ensure(c.f_S[nxt], c.cap_fS[nxt], sizeof(uint64_t) * cap));
         CKS(c.ensure(c.f_Q[nxt], c.cap_fQ[nxt], sizeof(u128) * cap));
         const int tk_s = c.stage_begin("root_split");
-        KmArgs ka{c.f_lo[cur], c.f_hi[cur], &c.scalars->ftot[cur], c.km_dpos, c.km_dP, D, c.km_F, c.km_arg, kk,
+        KmArgs ka{c.f_lo[cur], c.f_hi[cur], &c.scalars->ftot[cur], c.km_dpos, c.km_dP, D, c.km_F,
+                  c.km_F + (size_t)(kk + 1) * (D + 1), c.km_arg, kk,
                   c.cut, c.km_ngrp};
         // subproblem lists: at most one per distinct value in flight per round
         const uint64_t rows_l = tot & 0xFFFFFFFFull;
         CKS(c.ensure(c.km_meta, c.cap_km_meta, sizeof(KmMeta) * C));
-        CKS(c.ensure(c.km_sub, c.cap_km_sub, sizeof(KmSub) * 2 * (rows_l + C + 2)));
+        // short lists: at most one subproblem per distinct value in flight; long
+        // ones: their a ranges (> kKmLong each) overlap only at their ends
+        const uint64_t cap_s = rows_l + C + 2, cap_l = rows_l / kKmLong + 2 * C + 2;
+        CKS(c.ensure(c.km_sub, c.cap_km_sub, sizeof(KmSub) * 2 * (cap_s + cap_l)));
         KmMeta *meta = (KmMeta *)c.km_meta;
-        KmSub *sub[2] = {(KmSub *)c.km_sub, (KmSub *)c.km_sub + (rows_l + C + 2)};
-        uint32_t *nsub = c.scalars->km_nsub;
-        CK(cudaMemsetAsync(nsub, 0, 2 * sizeof(uint32_t), st));
-        km_prep_kernel<<<(unsigned)min((C + 7) / 8, (uint64_t)c.sms * 16), 256, 0, st>>>(ka, meta, sub[0], nsub);
+        KmSub *sb = (KmSub *)c.km_sub;
+        KmSub *sub[2][2] = {{sb, sb + cap_s}, {sb + 2 * cap_s, sb + 2 * cap_s + cap_l}};   // [class][parity]
+        uint32_t *nsub = c.scalars->km_nsub;   // [class * 2 + parity]
+        CK(cudaMemsetAsync(nsub, 0, 4 * sizeof(uint32_t), st));
+        km_prep_kernel<<<(unsigned)min((C + 7) / 8, (uint64_t)c.sms * 16), 256, 0, st>>>(
+            ka, meta, KmLists{{sub[0][0], sub[1][0]}, {nsub + 0, nsub + 2}});
         c.launches++;
         const int depth = 2 + (int)(64 - __builtin_clzll(rows_l + 1));   // rounds: > log2 of the largest d
         for (uint32_t j = 2; j <= kk; j++) {
             if (j > 2) {
-                CK(cudaMemsetAsync(nsub, 0, sizeof(uint32_t), st));
-                km_layer_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(&c.scalars->ftot[cur], meta, j, sub[0],
-                                                                            nsub);
+                CK(cudaMemsetAsync(nsub, 0, 4 * sizeof(uint32_t), st));
+                km_layer_kernel<<<(unsigned)((C + 255) / 256), 256, 0, st>>>(
+                    &c.scalars->ftot[cur], meta, j, KmLists{{sub[0][0], sub[1][0]}, {nsub + 0, nsub + 2}});
                 c.launches++;
             }
             int sc = 0;
             for (int r = 0; r < depth; r++) {   // empty rounds exit at once (counts read on the device)
                 CK(cudaMemsetAsync(nsub + (sc ^ 1), 0, sizeof(uint32_t), st));
-                KmStep ks{ka, meta, sub[sc], nsub + sc, sub[sc ^ 1], nsub + (sc ^ 1), j};
+                CK(cudaMemsetAsync(nsub + 2 + (sc ^ 1), 0, sizeof(uint32_t), st));
+                KmStep ks{ka, meta, {sub[0][sc], sub[1][sc]}, {nsub + sc, nsub + 2 + sc},
+                          {sub[0][sc ^ 1], sub[1][sc ^ 1]}, {nsub + (sc ^ 1), nsub + 2 + (sc ^ 1)}, j};
                 km_step_block_kernel<<<(unsigned)c.sms * 2, 256, 0, st>>>(ks);
                 km_step_warp_kernel<<<(unsigned)c.sms * 16, 256, 0, st>>>(ks);
                 c.launches += 2;
