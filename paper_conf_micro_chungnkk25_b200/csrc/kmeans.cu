@@ -274,6 +274,7 @@ struct KmStep {
 };
 
 constexpr uint32_t kKmLong = 512;   // a ranges longer than this get a block
+constexpr uint32_t kKmLeafA = 64;   // subproblems of <= 32 b and < this many a: solved whole by one warp
 constexpr int kKmNear = 256;        // near-tie candidates resolved exactly per subproblem
 
 // the list a subproblem belongs to: 1 (long) when its b = mid scans more than kKmLong candidates
@@ -388,9 +389,31 @@ __global__ void __launch_bounds__(256) km_step_warp_kernel(KmStep s) {
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t i = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += nwarps) {
         const KmSub x = s.cur[0][i];
+        const KmCluster c = km_cluster(s.meta[x.c]);
+        if (x.bhi - x.blo < 32 && x.ahi - x.alo < kKmLeafA && !x.pad) {
+            // the whole sub-tree at once: lane i solves b = blo + i over the
+            // subproblem's a range (it holds every b's smallest optimal a), one
+            // scan per lane; a lane whose best is not unique by 2^-40 goes back
+            // to the list as a single-b subproblem (near-tie path next round)
+            const uint32_t b = x.blo + lane;
+            if (b <= x.bhi) {
+                KmTop tp{-1.0, -1.0, 0xFFFFFFFFu};
+                const uint32_t ae = min(x.ahi, b - 1);
+                for (uint32_t a = x.alo; a <= ae; a++) km_top_add(tp, km_value(s.g, c, s.j, a, b), a);
+                if (tp.v2 < __dmul_rn(tp.v1, 1.0 - 0x1p-40)) {
+                    const size_t L = s.g.D + 1, idx = (size_t)s.j * L + c.D0 + b;
+                    const KDD vb = km_value_dd(s.g, c, s.j, tp.a1, b);
+                    s.g.F[idx] = vb.hi;
+                    s.g.Flo[idx] = vb.lo;
+                    s.g.arg[idx] = tp.a1;
+                } else {
+                    km_push(s.nxt, s.nnxt, KmSub{x.c, b, b, x.alo, x.ahi, 1});   // pad = 1: never a leaf again
+                }
+            }
+            continue;
+        }
         const uint32_t mid = x.blo + (x.bhi - x.blo) / 2;
         const uint32_t a0 = x.alo, a1 = min(x.ahi, mid - 1);
-        const KmCluster c = km_cluster(s.meta[x.c]);
         KmTop tp{-1.0, -1.0, 0xFFFFFFFFu};
         for (uint32_t a = a0 + lane; a <= a1; a += 32) km_top_add(tp, km_value(s.g, c, s.j, a, mid), a);
         tp = km_top_warp(tp);
