@@ -274,7 +274,10 @@ struct KmStep {
 };
 
 constexpr uint32_t kKmLong = 512;   // a ranges longer than this get a block
-constexpr uint32_t kKmLeafA = 64;   // subproblems of <= 32 b and < this many a: solved whole by one warp
+#ifndef SR_KM_LEAFA
+#define SR_KM_LEAFA 64
+#endif
+constexpr uint32_t kKmLeafA = SR_KM_LEAFA;   // subproblems of <= 32 b and < this many a: solved whole by one warp
 constexpr int kKmNear = 256;        // near-tie candidates resolved exactly per subproblem
 
 // the list a subproblem belongs to: 1 (long) when its b = mid scans more than kKmLong candidates
