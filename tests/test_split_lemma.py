@@ -89,3 +89,41 @@ def test_midpoint_is_monotone_and_range_pruning_is_safe():
                     continue
                 assert t[a - 1] < t[b]
                 assert ms[b - 1] >= t[a - 1] and ms[a - 1] <= t[b]
+
+
+def test_kmeans_between_group_form():
+    """The k-means option's fp64 filter (kmeans.cu km_between) evaluates the DP in
+    between-group form: for prefix sums S, counts n over sorted distinct values,
+    S(0,a)^2/n(0,a) + S(a,b)^2/n(a,b) - S(0,b)^2/n(0,b)
+        = (n(a,b) S(0,a) - n(0,a) S(a,b))^2 / (n(0,a) n(a,b) n(0,b)),
+    so G[j][b] = F[j][b] - S(0,b)^2/n(0,b) obeys G[j][b] = max_a G[j-1][a] + T(a,b)
+    with the same argmax as the F recurrence.  Checked with exact rationals."""
+    rng = np.random.default_rng(77)
+    for _ in range(40):
+        d = int(rng.integers(3, 14))
+        cnt = rng.integers(1, 50, d)
+        val = np.cumsum(rng.integers(1, 10_000, d))          # distinct sorted values
+        n = np.r_[0, np.cumsum(cnt)].astype(object)
+        S = np.r_[0, np.cumsum(cnt * val)].astype(object)
+
+        def T(a, b):
+            na, nab, nb = n[a], n[b] - n[a], n[b]
+            Sa, Sab = S[a], S[b] - S[a]
+            return Fraction((nab * Sa - na * Sab) ** 2, na * nab * nb)
+
+        for a in range(1, d):
+            for b in range(a + 1, d + 1):
+                lhs = Fraction(S[a] ** 2, n[a]) + Fraction((S[b] - S[a]) ** 2, n[b] - n[a]) - Fraction(S[b] ** 2, n[b])
+                assert lhs == T(a, b)
+        K = min(4, d)
+        F = {(1, b): Fraction(S[b] ** 2, n[b]) for b in range(1, d + 1)}
+        G = {(1, b): Fraction(0) for b in range(1, d + 1)}
+        for j in range(2, K + 1):
+            for b in range(j, d + 1):
+                fv = [(F[(j - 1, a)] + Fraction((S[b] - S[a]) ** 2, n[b] - n[a]), a) for a in range(j - 1, b)]
+                gv = [(G[(j - 1, a)] + T(a, b), a) for a in range(j - 1, b)]
+                fbest = max(v for v, _ in fv)
+                gbest = max(v for v, _ in gv)
+                assert [a for v, a in fv if v == fbest] == [a for v, a in gv if v == gbest]
+                F[(j, b)], G[(j, b)] = fbest, gbest
+                assert gbest == fbest - Fraction(S[b] ** 2, n[b])
