@@ -82,7 +82,7 @@ void Ctx::release() {
     }
     dfree(t_sorted, cap_ts); dfree(row_sorted, cap_rs); dfree(kid_count, cap_kc); dfree(goff, cap_goff);
     dfree(kid_max, cap_kmax); dfree(key_base, cap_kbase); dfree(key_base_c, cap_kbase_c); dfree(key_base_s, cap_kbase_s); dfree(tailh, cap_tailh); dfree(kid_tab, cap_kid_tab); dfree(sort_mode, cap_sort_mode); dfree(sort_gbase, cap_sort_gbase);
-    dfree(hist, cap_hist); dfree(sort_status, cap_status); dfree(scalars, cap_scalars);
+    dfree(hist, cap_hist); dfree(sort_status, cap_status); dfree(tile_hist, cap_tile_hist); dfree(scalars, cap_scalars);
     dfree(scan_scratch, cap_scan); dfree(PS1, cap_ps1); dfree(PS2, cap_ps2); dfree(TB, cap_TB); dfree(chunk_sq, cap_chunk_sq);
     dfree(cut, cap_cut); dfree(cut_SL, cap_cut_SL); dfree(cut_QL, cap_cut_QL); dfree(cnt_sz, cap_cntsz); dfree(flags, cap_flags);
     dfree(leaf_lo, cap_leaf_lo); dfree(leaf_m, cap_leaf_m); dfree(leaf_moff, cap_leaf_moff);

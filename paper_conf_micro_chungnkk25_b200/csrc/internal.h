@@ -188,6 +188,7 @@ struct Ctx {
     uint64_t *sort_gbase = nullptr; size_t cap_sort_gbase = 0; // [pass][256] digit bases
     uint64_t *hist = nullptr; size_t cap_hist = 0;
     void *sort_status = nullptr; size_t cap_status = 0;
+    void *tile_hist = nullptr; size_t cap_tile_hist = 0;   // first pass: per-tile digit counts, group sums, offsets
     DevScalars *scalars = nullptr; size_t cap_scalars = 0;
     void *scan_scratch = nullptr; size_t cap_scan = 0;
     // sampled prefix moments (a2): PS1/PS2 every kChunk rows
@@ -360,7 +361,8 @@ struct DensePath {
 // split = 3: ROOT with exact optimal 1-D k-means splits into kk groups (kmeans.cu, R29)
 int root_levels_kmeans(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2, int clamp, uint32_t kk);
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K,
-                      uint32_t *tailh, bool zero = true, cudaStream_t pst = nullptr);   // pre-pass only   // pre-pass only
+                      uint32_t *tailh, bool zero = true, cudaStream_t pst = nullptr, uint16_t *tileh = nullptr,
+                      uint64_t tile0 = 0);   // pre-pass only (tileh: the first sort pass's tile histograms too)   // pre-pass only
 int run_plan_dist(Ctx &c, Comm &comm, const stem_trace *tr, uint64_t row_base, double eps, double conf,
                   const stem_opts &o, int local_status);
 // capi.cu: allocate the host plan block for L clusters, S samples (c.early_plan);

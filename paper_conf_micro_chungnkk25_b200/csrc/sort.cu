@@ -151,6 +151,156 @@ __global__ void __launch_bounds__(kPreThreads, 2) prepass_kernel(const uint32_t 
             }
 }
 
+// The pre-pass over whole 5 120-row sort tiles (the first pass's tile shape):
+// besides everything prepass_kernel counts, each tile's histogram of t byte 0
+// (the first pass's digit) goes to tileh[tile][256] (u16).  Their column
+// prefix sums give every first-pass tile its global digit offsets, so the
+// first pass needs no decoupled look-back (tile_excl_*_kernel below).
+constexpr int kPreTThreads = 1024;   // 4 tiles per step = 5120 uint4 = five per thread
+constexpr int kPreTiles = 4;
+__global__ void __launch_bounds__(kPreTThreads) prepass_tile_kernel(
+    const uint32_t *__restrict__ kid, const uint32_t *__restrict__ t, uint64_t n, uint32_t K, int smem_kid,
+    uint32_t *__restrict__ kid_count, uint32_t *__restrict__ kid_max, uint64_t *__restrict__ hist,
+    uint32_t *__restrict__ max_t, uint32_t *__restrict__ err, uint32_t *__restrict__ tailh,
+    uint16_t *__restrict__ tileh, uint64_t tile0, uint32_t tile_rows) {
+    extern __shared__ uint32_t sh[];
+    // [3][256] block histograms of t bytes 0..2 (byte 0 from the tile histograms),
+    // [kPreTiles][256] the current tiles', [K] counts, [K] max
+    uint32_t *h0 = sh, *th = sh + 3 * kR, *hk = th + kPreTiles * kR, *hm = hk + (smem_kid ? K : 0);
+    for (int i = threadIdx.x; i < (3 + kPreTiles) * kR; i += blockDim.x) sh[i] = 0;
+    if (smem_kid)
+        for (uint32_t i = threadIdx.x; i < 2 * K; i += blockDim.x) hk[i] = 0;
+    __syncthreads();
+    uint32_t mx = 0, bad = 0;
+    auto one = [&](uint32_t *tq, uint32_t k, uint32_t x) {
+        mx = max(mx, x);
+        atomicAdd(&tq[x & (kR - 1)], 1u);
+        atomicAdd(&h0[kR + ((x >> kRB) & (kR - 1))], 1u);
+        if ((x >> (2 * kRB)) & (kR - 1)) atomicAdd(&h0[2 * kR + ((x >> (2 * kRB)) & (kR - 1))], 1u);
+        if (k >= K) { bad = 1; return; }
+        if (tailh && (x >> kCoarseShift)) atomicAdd(&tailh[(uint64_t)k * kR + (x >> kCoarseShift)], 1u);
+        if (smem_kid) {
+            atomicAdd(&hk[k], 1u);
+            if (x > hm[k]) atomicMax(&hm[k], x);
+        } else {
+            atomicAdd(&kid_count[k], 1u);
+            atomicMax(&kid_max[k], x);
+        }
+    };
+    const uint64_t ntiles = (n + tile_rows - 1) / tile_rows, nsteps = (ntiles + kPreTiles - 1) / kPreTiles;
+    const uint4 *kid4 = reinterpret_cast<const uint4 *>(kid), *t4 = reinterpret_cast<const uint4 *>(t);
+    const bool aligned = ((reinterpret_cast<uintptr_t>(kid) | reinterpret_cast<uintptr_t>(t)) & 15) == 0 &&
+                         tile_rows % 4 == 0;
+    const uint32_t q4 = tile_rows / 4;   // uint4 per tile
+    for (uint64_t sidx = blockIdx.x; sidx < nsteps; sidx += gridDim.x) {
+        const uint64_t q0 = sidx * kPreTiles, r0 = q0 * tile_rows;
+        const uint64_t cnt = min((uint64_t)kPreTiles * tile_rows, n - r0);
+        if (aligned && cnt == (uint64_t)kPreTiles * tile_rows && kPreTiles * q4 == 5 * kPreTThreads) {
+            uint4 a[5], b[5];
+#pragma unroll
+            for (int k = 0; k < 5; k++) {
+                a[k] = __ldg(kid4 + r0 / 4 + threadIdx.x + k * kPreTThreads);
+                b[k] = __ldg(t4 + r0 / 4 + threadIdx.x + k * kPreTThreads);
+            }
+#pragma unroll
+            for (int k = 0; k < 5; k++) {
+                uint32_t *tq = th + ((threadIdx.x + k * kPreTThreads) / q4) * kR;
+                one(tq, a[k].x, b[k].x); one(tq, a[k].y, b[k].y); one(tq, a[k].z, b[k].z); one(tq, a[k].w, b[k].w);
+            }
+        } else {
+            for (uint64_t i = threadIdx.x; i < cnt; i += blockDim.x)
+                one(th + (i / tile_rows) * kR, __ldg(kid + r0 + i), __ldg(t + r0 + i));
+        }
+        __syncthreads();
+        for (int i = threadIdx.x; i < kPreTiles * kR; i += blockDim.x) {
+            const uint64_t q = q0 + (i >> kRB);
+            const uint32_t v = th[i];
+            if (q < ntiles) {
+                tileh[(tile0 + q) * kR + (i & (kR - 1))] = (uint16_t)v;
+                atomicAdd(&h0[i & (kR - 1)], v);
+            }
+            th[i] = 0;
+        }
+        __syncthreads();
+    }
+    for (int o = 16; o; o >>= 1) {
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        bad |= __shfl_xor_sync(0xffffffffu, bad, o);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        if (mx) atomicMax(max_t, mx);
+        if (bad) atomicOr(err, 1u);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < 3 * kR; i += blockDim.x) {
+        const uint32_t v = sh[i];
+        if (v) atomicAdd((unsigned long long *)&hist[((i >> kRB) == 2 ? kHistT2 : (i >> kRB)) * kHistR + (i & (kR - 1))],
+                         (unsigned long long)v);
+    }
+    if (smem_kid)
+        for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
+            if (hk[i]) {
+                atomicAdd(&kid_count[i], hk[i]);
+                atomicMax(&kid_max[i], hm[i]);
+            }
+}
+
+// Global first-pass offsets per tile from the tile histograms: excl[q][d] =
+// the rows of digit d in tiles before q.  Groups of kExGrp tiles: their
+// column sums, a scan of those per digit, then the tiles of each group.
+constexpr int kExGrp = 64;
+__global__ void tile_grp_kernel(const uint16_t *__restrict__ tileh, uint64_t ntiles, uint32_t *__restrict__ grp) {
+    const uint64_t g = blockIdx.x, q0 = g * kExGrp, q1 = min(q0 + kExGrp, ntiles);
+    uint32_t s = 0;
+#pragma unroll 16
+    for (uint64_t q = q0; q < q1; q++) s += tileh[q * kR + threadIdx.x];
+    grp[g * kR + threadIdx.x] = s;
+}
+// one block per digit: exclusive scan of its column of group sums (in place)
+__global__ void __launch_bounds__(1024) grp_scan_kernel(uint32_t *__restrict__ grp, uint64_t ngrp) {
+    __shared__ uint32_t s_w[32];
+    const uint32_t d = blockIdx.x;
+    uint32_t carry = 0;
+    for (uint64_t b0 = 0; b0 < ngrp; b0 += 1024) {
+        const uint64_t g = b0 + threadIdx.x;
+        const uint32_t v = g < ngrp ? grp[g * kR + d] : 0u;
+        uint32_t incl = v;
+        const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += u;
+        }
+        if (lane == 31) s_w[w] = incl;
+        __syncthreads();
+        uint32_t off = 0;
+        for (int k = 0; k < w; k++) off += s_w[k];
+        uint32_t tot = 0;
+        for (int k = 0; k < 32; k++) tot += s_w[k];
+        if (g < ngrp) grp[g * kR + d] = carry + off + incl - v;
+        carry += tot;
+        __syncthreads();
+    }
+}
+__global__ void tile_excl_kernel(const uint16_t *__restrict__ tileh, uint64_t ntiles, const uint32_t *__restrict__ grp,
+                                 uint32_t *__restrict__ excl) {
+    const uint64_t g = blockIdx.x, q0 = g * kExGrp;
+    uint32_t run = grp[g * kR + threadIdx.x];
+    for (int h = 0; h < kExGrp; h += 16) {   // 16 loads in flight, then the running sums
+        uint32_t v[16];
+#pragma unroll
+        for (int u = 0; u < 16; u++) {
+            const uint64_t q = q0 + h + u;
+            v[u] = q < ntiles ? tileh[q * kR + threadIdx.x] : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < 16; u++) {
+            const uint64_t q = q0 + h + u;
+            if (q < ntiles) excl[q * kR + threadIdx.x] = run;
+            run += v[u];
+        }
+    }
+}
+
 // kid-table entry j -> the kernel whose key range holds j << tsh
 __global__ void kid_table_kernel(const uint64_t *__restrict__ B, uint32_t K, uint64_t entries, int tsh,
                                  uint32_t *__restrict__ tab) {
@@ -292,6 +442,8 @@ struct PassArgs {
     uint64_t *status;                   // [ntiles][R] (u32 words when s32)
     bool s32;                           // n < 2^30: 32-bit look-back statuses
     uint32_t *tile_counter;
+    const uint32_t *tile_excl;          // FIRST: [tile][R] global offsets from the pre-pass (no look-back), or NULL
+    uint64_t tile_base;                 // tile index of blockIdx.x 0 (with tile_excl)
 };
 
 // One LSD pass over digit (key >> shift) & 255.  NT threads, IT keys per
@@ -318,7 +470,8 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
     uint32_t *s_xh = reinterpret_cast<uint32_t *>(&s_whist[0][0] + NW * R);
 
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    if (tid == 0) s_tile = atomicAdd(a.tile_counter, 1u);
+    const bool nolb = FIRST && a.tile_excl;   // offsets known in advance: no look-back
+    if (tid == 0) s_tile = nolb ? (uint32_t)(a.tile_base + blockIdx.x) : atomicAdd(a.tile_counter, 1u);
     for (int i = tid; i < NW * R / 2; i += NT) reinterpret_cast<uint32_t *>(&s_whist[0][0])[i] = 0;
     for (int i = tid; i < R; i += NT) s_cnt[i] = 0;
     if (FIRST)
@@ -405,7 +558,7 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
             }
     }
     __syncthreads();
-    if (tid < R && !a.late) put_status(a.status, S32, (uint64_t)tile * R + tid, tile == 0 ? kFlagP : kFlagA, s_cnt[tid]);
+    if (tid < R && !a.late && !nolb) put_status(a.status, S32, (uint64_t)tile * R + tid, tile == 0 ? kFlagP : kFlagA, s_cnt[tid]);
     if (FIRST && tid < R)
         for (int x = 0; x < a.nxh; x++)
             if (s_xh[x * R + tid])
@@ -453,7 +606,7 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
             s_whist[ww][d] = (uint16_t)cnt;
             cnt += c;
         }
-        if (a.late) put_status(a.status, S32, (uint64_t)tile * R + d, tile == 0 ? kFlagP : kFlagA, cnt);
+        if (a.late && !nolb) put_status(a.status, S32, (uint64_t)tile * R + d, tile == 0 ? kFlagP : kFlagA, cnt);
         c_incl = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -503,7 +656,8 @@ __global__ void __launch_bounds__(NT, FULL ? (NT >= 448 ? 2 : NT >= 320 ? 3 : SR
         excl = (uint64_t)((double)a.hist[a.pass * kHistR + d] * tile / (double)((a.n + TILE - 1) / TILE));
         if (false) {
 #else
-        if (tile != 0) {
+        if (nolb) excl = a.tile_excl[(uint64_t)tile * R + d];
+        if (tile != 0 && !nolb) {
 #endif
             int64_t j = (int64_t)tile - 1;
             bool done = false;
@@ -595,7 +749,9 @@ static int launch_pass(const PassArgs &a, cudaStream_t st, uint32_t *launches) {
         (*launches)++;
     }
     if (rag) {
-        onesweep_kernel<NT, IT, FIRST, LAST, false, PK, S32><<<1, NT, smem, st>>>(a);
+        PassArgs ar = a;
+        ar.tile_base = full;   // (tile_excl: the ragged tile's index)
+        onesweep_kernel<NT, IT, FIRST, LAST, false, PK, S32><<<1, NT, smem, st>>>(ar);
         (*launches)++;
     }
     return STEM_OK;
@@ -632,7 +788,7 @@ static int launch_sort_pass(const PassArgs &a, bool first, bool last, cudaStream
 // multi-GPU histogram step.  Zeroes its outputs first (zero = false: they
 // accumulate, for a trace handed over in chunks; pst = the launch stream).
 int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n, uint32_t K, uint32_t *tailh,
-                      bool zero, cudaStream_t pst) {
+                      bool zero, cudaStream_t pst, uint16_t *tileh, uint64_t tile0) {
     cudaStream_t st = pst ? pst : c.stream;
     if (zero) {
         CK(cudaMemsetAsync(c.hist, 0, sizeof(uint64_t) * (kMaxPasses + 1) * kHistR, st));
@@ -642,6 +798,21 @@ int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n
     }
     if (n == 0) return STEM_OK;
     const int smem_kid = (K <= 24000) ? 1 : 0;
+    if (tileh) {   // whole sort tiles, with the first pass's per-tile digit histograms
+        const size_t tb = sizeof(uint32_t) * ((3 + kPreTiles) * kR + (smem_kid ? 2 * (size_t)K : 0));
+        static const cudaError_t pt_attr = cudaFuncSetAttribute(
+            prepass_tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            (int)(sizeof(uint32_t) * ((3 + kPreTiles) * kR + 2 * 24000)));
+        CK(pt_attr);
+        int per_sm = (int)((200 * 1024) / (tb + 1024));
+        per_sm = per_sm < 1 ? 1 : per_sm > 2 ? 2 : per_sm;
+        prepass_tile_kernel<<<c.sms * per_sm, kPreTThreads, tb, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.kid_max,
+                                                                      c.hist, &c.scalars->max_t, &c.scalars->err, tailh,
+                                                                      tileh, tile0, (uint32_t)tile_keys());
+        c.launches++;
+        CK(cudaGetLastError());
+        return STEM_OK;
+    }
     constexpr int kMaxNC = 8;
     auto bytes = [&](int nc) { return sizeof(uint32_t) * (nc * (3 * kR + 1) + (smem_kid ? 2 * (size_t)K : 0)); };
     // histogram copies (env STEMROOT_PRE_NC, <= 8, capped to keep two blocks per SM).
@@ -685,6 +856,22 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     const bool coarse_ok = K <= kMaxTailK && !(getenv("STEMROOT_SORT_COARSE") && getenv("STEMROOT_SORT_COARSE")[0] == '0');
     if (coarse_ok) CKS(c.ensure(c.tailh, c.cap_tailh, sizeof(uint32_t) * kR * (uint64_t)K));
     uint32_t *tailh = coarse_ok ? c.tailh : nullptr;
+    // the first pass without look-back: the pre-pass counts its digit per tile
+    // and three small kernels turn the counts into each tile's offsets
+    // (STEMROOT_SORT_NOLB=0: the look-back first pass)
+    const uint64_t ntiles = (n + tile_keys() - 1) / tile_keys();
+    const bool nolb = !(getenv("STEMROOT_SORT_NOLB") && getenv("STEMROOT_SORT_NOLB")[0] == '0') && n > 0;
+    const uint64_t ngrp = (ntiles + kExGrp - 1) / kExGrp;
+    uint16_t *tileh = nullptr;
+    uint32_t *tgrp = nullptr, *texcl = nullptr;
+    if (nolb) {
+        const size_t b_h = (sizeof(uint16_t) * ntiles * kR + 255) & ~(size_t)255;
+        const size_t b_g = (sizeof(uint32_t) * ngrp * kR + 255) & ~(size_t)255;
+        CKS(c.ensure(c.tile_hist, c.cap_tile_hist, b_h + b_g + sizeof(uint32_t) * ntiles * kR));
+        tileh = (uint16_t *)c.tile_hist;
+        tgrp = (uint32_t *)((char *)c.tile_hist + b_h);
+        texcl = (uint32_t *)((char *)c.tile_hist + b_h + b_g);
+    }
     const int nch = h_kid ? h2d_chunks(n) : 0;
     if (nch > 1) {
         // host trace: the copies run back to back on the plan's stream; the
@@ -698,7 +885,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
             if (!c.ev_h2d[i]) CK(cudaEventCreateWithFlags(&c.ev_h2d[i], cudaEventDisableTiming));
         if (!c.ev_pre) CK(cudaEventCreateWithFlags(&c.ev_pre, cudaEventDisableTiming));
         CKS(histogram_kernels(c, nullptr, nullptr, 0, K, tailh, true, st));   // zero the outputs
-        const uint64_t step = ((n + nch - 1) / nch + 1023) & ~1023ull;
+        const uint64_t step = ((n + nch - 1) / nch + tile_keys() - 1) / tile_keys() * tile_keys();   // whole tiles
         int used = 0;
         for (uint64_t r0 = 0; r0 < n; r0 += step, used++) {
             const uint64_t cnt = min(step, n - r0);
@@ -706,7 +893,7 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
             CK(cudaMemcpyAsync((void *)(t + r0), h_t + r0, sizeof(uint32_t) * cnt, cudaMemcpyHostToDevice, st));
             CK(cudaEventRecord(c.ev_h2d[used], st));
             CK(cudaStreamWaitEvent(c.dstream, c.ev_h2d[used], 0));
-            CKS(histogram_kernels(c, kid + r0, t + r0, cnt, K, tailh, false, c.dstream));
+            CKS(histogram_kernels(c, kid + r0, t + r0, cnt, K, tailh, false, c.dstream, tileh, r0 / tile_keys()));
         }
         CK(cudaEventRecord(c.ev_pre, c.dstream));
         CK(cudaStreamWaitEvent(st, c.ev_pre, 0));
@@ -715,7 +902,13 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         CK(cudaMemcpyAsync((void *)t, h_t, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, st));
     }
     const int tk_pre = c.stage_begin("prepass");
-    if (nch <= 1) CKS(histogram_kernels(c, kid, t, n, K, tailh, true, st));
+    if (nch <= 1) CKS(histogram_kernels(c, kid, t, n, K, tailh, true, st, tileh, 0));
+    if (nolb) {
+        tile_grp_kernel<<<(unsigned)ngrp, kR, 0, st>>>(tileh, ntiles, tgrp);
+        grp_scan_kernel<<<kR, 1024, 0, st>>>(tgrp, ngrp);
+        tile_excl_kernel<<<(unsigned)ngrp, kR, 0, st>>>(tileh, ntiles, tgrp, texcl);
+        c.launches += 3;
+    }
     // key bases B = exclusive scan of W[k] = roundup(max_t[k] + 1, 2^16) (0 if
     // absent); Bc the same with 2^24
     const uint32_t *cnt = c.kid_count, *kmax = c.kid_max;
@@ -789,7 +982,6 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
         tab = c.kid_tab;
     }
 
-    const uint64_t ntiles = (n + tile_keys() - 1) / tile_keys();
     CKS(c.ensure(c.sort_status, c.cap_status, ntiles * kR * sizeof(uint64_t)));
     PassArgs a{};
     a.n = n;
@@ -848,8 +1040,12 @@ int sort_trace(Ctx &c, const uint32_t *kid, const uint32_t *t, const uint32_t *r
     uint64_t *kin = c.keys[0], *kout = c.keys[1];
     uint32_t *vin = c.vals[0], *vout = c.vals[1];
     for (int p = 0; p < npasses; p++) {
-        CK(cudaMemsetAsync(a.status, 0, status_bytes, st));
-        CK(cudaMemsetAsync(a.tile_counter, 0, sizeof(uint32_t), st));
+        a.tile_excl = p == 0 && nolb ? texcl : nullptr;
+        a.tile_base = 0;
+        if (!a.tile_excl) {
+            CK(cudaMemsetAsync(a.status, 0, status_bytes, st));
+            CK(cudaMemsetAsync(a.tile_counter, 0, sizeof(uint32_t), st));
+        }
         a.shift = ks + kRB * p;
         a.pass = p;
         const bool first = p == 0, last = p == npasses - 1;
