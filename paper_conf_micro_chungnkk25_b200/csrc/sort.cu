@@ -156,9 +156,18 @@ __global__ void __launch_bounds__(kPreThreads, 2) prepass_kernel(const uint32_t 
 // (the first pass's digit) goes to tileh[tile][256] (u16).  Their column
 // prefix sums give every first-pass tile its global digit offsets, so the
 // first pass needs no decoupled look-back (tile_excl_*_kernel below).
-constexpr int kPreTThreads = 1024;   // 4 tiles per step = 5120 uint4 = five per thread
-constexpr int kPreTiles = 4;
-__global__ void __launch_bounds__(kPreTThreads) prepass_tile_kernel(
+#ifndef SR_PRET_THREADS
+#define SR_PRET_THREADS 1024
+#endif
+#ifndef SR_PRET_MINB
+#define SR_PRET_MINB 2
+#endif
+#ifndef SR_PRET_PAIRS
+#define SR_PRET_PAIRS 1
+#endif
+constexpr int kPreTThreads = SR_PRET_THREADS;              // kPreTiles tiles per step = five uint4 per thread
+constexpr int kPreTiles = kPreTThreads * 5 * 4 / 5120;     // 512 threads: 2 tiles, 1024: 4
+__global__ void __launch_bounds__(kPreTThreads, SR_PRET_MINB) prepass_tile_kernel(
     const uint32_t *__restrict__ kid, const uint32_t *__restrict__ t, uint64_t n, uint32_t K, int smem_kid,
     uint32_t *__restrict__ kid_count, uint32_t *__restrict__ kid_max, uint64_t *__restrict__ hist,
     uint32_t *__restrict__ max_t, uint32_t *__restrict__ err, uint32_t *__restrict__ tailh,
@@ -196,6 +205,7 @@ __global__ void __launch_bounds__(kPreTThreads) prepass_tile_kernel(
         const uint64_t q0 = sidx * kPreTiles, r0 = q0 * tile_rows;
         const uint64_t cnt = min((uint64_t)kPreTiles * tile_rows, n - r0);
         if (aligned && cnt == (uint64_t)kPreTiles * tile_rows && kPreTiles * q4 == 5 * kPreTThreads) {
+#if SR_PRET_PAIRS == 5
             uint4 a[5], b[5];
 #pragma unroll
             for (int k = 0; k < 5; k++) {
@@ -207,6 +217,25 @@ __global__ void __launch_bounds__(kPreTThreads) prepass_tile_kernel(
                 uint32_t *tq = th + ((threadIdx.x + k * kPreTThreads) / q4) * kR;
                 one(tq, a[k].x, b[k].x); one(tq, a[k].y, b[k].y); one(tq, a[k].z, b[k].z); one(tq, a[k].w, b[k].w);
             }
+#else   // SR_PRET_PAIRS uint4 pairs in flight per thread (fewer registers: more warps per SM)
+#pragma unroll 1
+            for (int k0 = 0; k0 < 5; k0 += SR_PRET_PAIRS) {
+                uint4 a[SR_PRET_PAIRS], b[SR_PRET_PAIRS];
+#pragma unroll
+                for (int k = 0; k < SR_PRET_PAIRS; k++)
+                    if (k0 + k < 5) {
+                        a[k] = __ldg(kid4 + r0 / 4 + threadIdx.x + (k0 + k) * kPreTThreads);
+                        b[k] = __ldg(t4 + r0 / 4 + threadIdx.x + (k0 + k) * kPreTThreads);
+                    }
+#pragma unroll
+                for (int k = 0; k < SR_PRET_PAIRS; k++)
+                    if (k0 + k < 5) {
+                        uint32_t *tq = th + ((threadIdx.x + (k0 + k) * kPreTThreads) / q4) * kR;
+                        one(tq, a[k].x, b[k].x); one(tq, a[k].y, b[k].y); one(tq, a[k].z, b[k].z);
+                        one(tq, a[k].w, b[k].w);
+                    }
+            }
+#endif
         } else {
             for (uint64_t i = threadIdx.x; i < cnt; i += blockDim.x)
                 one(th + (i / tile_rows) * kR, __ldg(kid + r0 + i), __ldg(t + r0 + i));
@@ -804,8 +833,8 @@ int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n
             prepass_tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
             (int)(sizeof(uint32_t) * ((3 + kPreTiles) * kR + 2 * 24000)));
         CK(pt_attr);
-        int per_sm = (int)((200 * 1024) / (tb + 1024));
-        per_sm = per_sm < 1 ? 1 : per_sm > 2 ? 2 : per_sm;
+        int per_sm = (int)((220 * 1024) / (tb + 1024));
+        per_sm = per_sm < 1 ? 1 : per_sm > SR_PRET_MINB ? SR_PRET_MINB : per_sm;   // the registers allow SR_PRET_MINB
         prepass_tile_kernel<<<c.sms * per_sm, kPreTThreads, tb, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.kid_max,
                                                                       c.hist, &c.scalars->max_t, &c.scalars->err, tailh,
                                                                       tileh, tile0, (uint32_t)tile_keys());
