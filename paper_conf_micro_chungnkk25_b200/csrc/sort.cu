@@ -274,6 +274,92 @@ __global__ void __launch_bounds__(kPreTThreads, SR_PRET_MINB) prepass_tile_kerne
             }
 }
 
+// The same pre-pass with the tiles dealt to WARPS: each warp keeps its tile's
+// digit histogram in shared memory (two u16 counts per word), so no block
+// barrier is needed between tiles and warps drift as in prepass_kernel.
+__global__ void __launch_bounds__(1024, 2) prepass_wtile_kernel(
+    const uint32_t *__restrict__ kid, const uint32_t *__restrict__ t, uint64_t n, uint32_t K, int smem_kid,
+    uint32_t *__restrict__ kid_count, uint32_t *__restrict__ kid_max, uint64_t *__restrict__ hist,
+    uint32_t *__restrict__ max_t, uint32_t *__restrict__ err, uint32_t *__restrict__ tailh,
+    uint16_t *__restrict__ tileh, uint64_t tile0, uint32_t tile_rows) {
+    extern __shared__ uint32_t sh[];
+    // [3][256] block histograms of t bytes 0..2, [32 warps][128] packed tile counts, [K] counts, [K] max
+    constexpr int NW = 1024 / 32, TW = kR / 2;
+    uint32_t *h0 = sh, *tw = sh + 3 * kR, *hk = tw + NW * TW, *hm = hk + (smem_kid ? K : 0);
+    for (int i = threadIdx.x; i < 3 * kR + NW * TW; i += blockDim.x) sh[i] = 0;
+    if (smem_kid)
+        for (uint32_t i = threadIdx.x; i < 2 * K; i += blockDim.x) hk[i] = 0;
+    __syncthreads();
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    uint32_t *th = tw + w * TW;
+    uint32_t mx = 0, bad = 0;
+    auto one = [&](uint32_t k, uint32_t x) {
+        mx = max(mx, x);
+        atomicAdd(&th[(x & (kR - 1)) >> 1], 1u << (16 * (x & 1)));
+        atomicAdd(&h0[kR + ((x >> kRB) & (kR - 1))], 1u);
+        if ((x >> (2 * kRB)) & (kR - 1)) atomicAdd(&h0[2 * kR + ((x >> (2 * kRB)) & (kR - 1))], 1u);
+        if (k >= K) { bad = 1; return; }
+        if (tailh && (x >> kCoarseShift)) atomicAdd(&tailh[(uint64_t)k * kR + (x >> kCoarseShift)], 1u);
+        if (smem_kid) {
+            atomicAdd(&hk[k], 1u);
+            if (x > hm[k]) atomicMax(&hm[k], x);
+        } else {
+            atomicAdd(&kid_count[k], 1u);
+            atomicMax(&kid_max[k], x);
+        }
+    };
+    const uint64_t ntiles = (n + tile_rows - 1) / tile_rows;
+    const uint64_t gw = (uint64_t)blockIdx.x * NW + w, nwarps = (uint64_t)gridDim.x * NW;
+    const uint4 *kid4 = reinterpret_cast<const uint4 *>(kid), *t4 = reinterpret_cast<const uint4 *>(t);
+    const bool aligned = ((reinterpret_cast<uintptr_t>(kid) | reinterpret_cast<uintptr_t>(t)) & 15) == 0 &&
+                         tile_rows % 128 == 0;
+    for (uint64_t q = gw; q < ntiles; q += nwarps) {
+        const uint64_t r0 = q * tile_rows, cnt = min((uint64_t)tile_rows, n - r0);
+        if (aligned && cnt == tile_rows) {
+            const uint64_t j0 = r0 / 4;
+            const uint32_t nj = tile_rows / 4;
+#pragma unroll 2
+            for (uint32_t j = lane; j < nj; j += 32) {
+                const uint4 a = __ldg(kid4 + j0 + j), b = __ldg(t4 + j0 + j);
+                one(a.x, b.x); one(a.y, b.y); one(a.z, b.z); one(a.w, b.w);
+            }
+        } else {
+            for (uint64_t i = lane; i < cnt; i += 32) one(__ldg(kid + r0 + i), __ldg(t + r0 + i));
+        }
+        __syncwarp();
+#pragma unroll
+        for (int u = 0; u < TW / 32; u++) {   // 4 words (8 digits) per lane: out, into the block's byte-0 counts, zero
+            const int wi = lane + 32 * u;
+            const uint32_t v = th[wi];
+            th[wi] = 0;
+            reinterpret_cast<uint32_t *>(tileh + (tile0 + q) * kR)[wi] = v;   // the two u16 counts, in place
+            if (v & 0xFFFFu) atomicAdd(&h0[2 * wi], v & 0xFFFFu);
+            if (v >> 16) atomicAdd(&h0[2 * wi + 1], v >> 16);
+        }
+        __syncwarp();
+    }
+    for (int o = 16; o; o >>= 1) {
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        bad |= __shfl_xor_sync(0xffffffffu, bad, o);
+    }
+    if (lane == 0) {
+        if (mx) atomicMax(max_t, mx);
+        if (bad) atomicOr(err, 1u);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < 3 * kR; i += blockDim.x) {
+        const uint32_t v = sh[i];
+        if (v) atomicAdd((unsigned long long *)&hist[((i >> kRB) == 2 ? kHistT2 : (i >> kRB)) * kHistR + (i & (kR - 1))],
+                         (unsigned long long)v);
+    }
+    if (smem_kid)
+        for (uint32_t i = threadIdx.x; i < K; i += blockDim.x)
+            if (hk[i]) {
+                atomicAdd(&kid_count[i], hk[i]);
+                atomicMax(&kid_max[i], hm[i]);
+            }
+}
+
 // Global first-pass offsets per tile from the tile histograms: excl[q][d] =
 // the rows of digit d in tiles before q.  Groups of kExGrp tiles: their
 // column sums, a scan of those per digit, then the tiles of each group.
@@ -827,6 +913,22 @@ int histogram_kernels(Ctx &c, const uint32_t *kid, const uint32_t *t, uint64_t n
     }
     if (n == 0) return STEM_OK;
     const int smem_kid = (K <= 24000) ? 1 : 0;
+    static const int wtile = !(getenv("STEMROOT_PRE_WTILE") && getenv("STEMROOT_PRE_WTILE")[0] == '0');
+    if (tileh && wtile) {   // tiles dealt to warps (default)
+        const size_t tb = sizeof(uint32_t) * (3 * kR + 32 * (kR / 2) + (smem_kid ? 2 * (size_t)K : 0));
+        static const cudaError_t pw_attr = cudaFuncSetAttribute(
+            prepass_wtile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            (int)(sizeof(uint32_t) * (3 * kR + 32 * (kR / 2) + 2 * 24000)));
+        CK(pw_attr);
+        int per_sm = (int)((220 * 1024) / (tb + 1024));
+        per_sm = per_sm < 1 ? 1 : per_sm > 2 ? 2 : per_sm;
+        prepass_wtile_kernel<<<c.sms * per_sm, 1024, tb, st>>>(kid, t, n, K, smem_kid, c.kid_count, c.kid_max, c.hist,
+                                                                &c.scalars->max_t, &c.scalars->err, tailh, tileh, tile0,
+                                                                (uint32_t)tile_keys());
+        c.launches++;
+        CK(cudaGetLastError());
+        return STEM_OK;
+    }
     if (tileh) {   // whole sort tiles, with the first pass's per-tile digit histograms
         const size_t tb = sizeof(uint32_t) * ((3 + kPreTiles) * kR + (smem_kid ? 2 * (size_t)K : 0));
         static const cudaError_t pt_attr = cudaFuncSetAttribute(
