@@ -864,11 +864,13 @@ __global__ void __launch_bounds__(256) lloyd_split_kernel(const uint32_t *__rest
                                                           const uint64_t *ctot, const uint32_t *__restrict__ t,
                                                           const uint64_t *__restrict__ PS1, const u128 *__restrict__ PS2,
                                                           uint32_t k0, uint32_t k1, uint32_t *__restrict__ cut,
-                                                          uint64_t *__restrict__ cut_SL) {
+                                                          uint64_t *__restrict__ cut_SL, uint32_t *__restrict__ queue) {
     const uint32_t C = (uint32_t)(*ctot >> 32);
     const int lane = threadIdx.x & 31;
-    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    for (uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nwarps) {
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    // clusters from a work queue (the next index fetched while this one is split)
+    for (uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, cn = 0; c < C; c = __shfl_sync(0xffffffffu, cn, 0)) {
+        if (lane == 0) cn = nwarps + atomicAdd(queue, 1u);
         const uint64_t lo = f_lo[c], hi = f_hi[c], n = hi - lo, S = f_S[c];
         uint64_t base;
         u128 mid2;
@@ -1597,12 +1599,14 @@ int root_levels(Ctx &c, uint64_t n, uint32_t K, double eps, double z, double k2,
         if (split != 0) {   // Lloyd variants: one warp per cluster, every size
             const unsigned g = (unsigned)min((Cub + 7) / 8, (uint64_t)c.sms * 16);
             const uint32_t k0 = (uint32_t)seed, k1 = (uint32_t)(seed >> 32);
+            uint32_t *q = &c.scalars->nc_queue[level & 1];
+            CK(cudaMemsetAsync(q, 0, sizeof(uint32_t), st));
             if (split == 2)
                 lloyd_split_kernel<true><<<g, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], ctot,
-                                                            c.t_sorted, c.PS1, c.PS2, k0, k1, c.cut, c.cut_SL);
+                                                            c.t_sorted, c.PS1, c.PS2, k0, k1, c.cut, c.cut_SL, q);
             else
                 lloyd_split_kernel<false><<<g, 256, 0, st>>>(c.f_lo[cur], c.f_hi[cur], c.f_S[cur], c.f_Q[cur], ctot,
-                                                             c.t_sorted, c.PS1, c.PS2, k0, k1, c.cut, c.cut_SL);
+                                                             c.t_sorted, c.PS1, c.PS2, k0, k1, c.cut, c.cut_SL, q);
             c.launches++;
         } else {
         // the small-cluster warps run on a side stream beside the big-cluster
