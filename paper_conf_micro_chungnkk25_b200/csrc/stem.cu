@@ -330,9 +330,12 @@ __global__ void __launch_bounds__(kThreads) sample_kernel(SampleArgs a) {
 // grid, pick the candidate.
 constexpr uint32_t kAmbChunk = 1u << 16;
 
-__global__ void __launch_bounds__(kThreads) resolve_locate_kernel(SampleArgs a, uint32_t na, uint64_t *nch) {
+// (the ambiguous-sample count na is read on the device: grids are sized for
+// every sample, entries past na get no chunks; no host round trip)
+__global__ void __launch_bounds__(kThreads) resolve_locate_kernel(SampleArgs a, const uint32_t *nap, uint64_t *nch) {
     const uint32_t e = blockIdx.x * blockDim.x + threadIdx.x;
-    if (e >= na) return;
+    if (e >= a.S) return;
+    if (e >= *nap) { nch[e] = 0; return; }
     Amb &en = a.amb[e];
     const uint32_t tv = a.t[en.pos];
     const uint32_t lo = a.leaf_lo[en.leaf];
@@ -378,9 +381,9 @@ __global__ void __launch_bounds__(kThreads) resolve_count_kernel(SampleArgs a, u
     }
 }
 
-__global__ void __launch_bounds__(kThreads) resolve_final_kernel(SampleArgs a, uint32_t na) {
+__global__ void __launch_bounds__(kThreads) resolve_final_kernel(SampleArgs a, const uint32_t *nap) {
     const uint32_t e = blockIdx.x * blockDim.x + threadIdx.x;
-    if (e >= na) return;
+    if (e >= *nap) return;
     const Amb en = a.amb[e];
     const uint32_t M = (uint32_t)__popcll(en.mask);
     uint32_t idx = en.side ? M - 1 - en.q : en.q;
@@ -678,19 +681,16 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         CK(cudaMemsetAsync(&c.scalars->amb_count, 0, sizeof(uint32_t), st));
         if (S) sample_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa);
         c.launches += S ? 1 : 0;
-        if (S && c.pack_h > 1) {
-            CK(cudaMemcpyAsync(&n_amb, &c.scalars->amb_count, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
-            CKS(sync_stream(c));
-        }
-        if (n_amb) {
+        if (S && c.pack_h > 1) {   // ambiguous samples, counted on the device (no host round trip)
+            const uint32_t *nap = &c.scalars->amb_count;
             uint64_t *nch = (uint64_t *)((char *)c.amb + amb_bytes), *choff = nch + (S + 1), *scr = choff + (S + 1);
             uint64_t *tot = &c.scalars->scan_total64;
-            resolve_locate_kernel<<<blocks_for(n_amb), kThreads, 0, st>>>(sa, n_amb, nch);
+            resolve_locate_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa, nap, nch);
             exclusive_scan<uint64_t>([nch] __device__(uint64_t i) -> uint64_t { return nch[i]; },
                                      [choff] __device__(uint64_t i, uint64_t pre, uint64_t) { choff[i] = pre; },
-                                     (uint64_t)n_amb, scr, tot, st, &c.launches);
-            resolve_count_kernel<<<4 * c.sms, kThreads, 0, st>>>(sa, n_amb, choff, tot);
-            resolve_final_kernel<<<blocks_for(n_amb), kThreads, 0, st>>>(sa, n_amb);
+                                     S, scr, tot, st, &c.launches);
+            resolve_count_kernel<<<4 * c.sms, kThreads, 0, st>>>(sa, (uint32_t)S, choff, tot);
+            resolve_final_kernel<<<blocks_for(S), kThreads, 0, st>>>(sa, nap);
             c.launches += 3;
         }
         c.stage_end(tk_smp, 40 * S);
@@ -750,6 +750,7 @@ int leaves_and_plan(Ctx &c, uint64_t n, uint32_t K, const double *metrics, uint3
         CK(cudaGetLastError());
         double red[2 + 64 + 2];
         CK(cudaMemcpyAsync(red, red_out, sizeof(double) * (2 + nm + 2), cudaMemcpyDeviceToHost, st));
+        if (c.pack_h > 1) CK(cudaMemcpyAsync(&n_amb, &c.scalars->amb_count, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
         CKS(sync_stream(c));
         c.est_total = red[2 + nm];
         c.bound = red[2 + nm + 1];
