@@ -691,3 +691,16 @@ def test_host_trace_chunked_copy(ctx):
     kid, t, _ = G.generate_np(sp)
     got, ref = _both(ctx, kid, t, sp.n_kernels, host=True, eps=sp.eps, seed=5)
     assert_plans_equal(got, ref)
+
+
+@pytest.mark.parametrize("K", [30_000, 100_000])
+def test_many_kernel_ids(ctx, K):
+    """More kernel ids than the pre-pass keeps in shared memory (> 24 000: global
+    count/max atomics) and than the coarse key bases allow (> 65 536); ids used
+    sparsely, several tiles and a ragged tail"""
+    rng = np.random.default_rng(K)
+    n = 400_003
+    kid = (rng.zipf(1.2, n) * 7919 % K).astype(np.uint32)
+    t = (rng.lognormal(9, 0.8, n) * (1 + kid % 13)).astype(np.uint32)
+    got, ref = _both(ctx, kid, t, K, eps=0.05, seed=8)
+    assert_plans_equal(got, ref)
