@@ -120,9 +120,14 @@ def run(config="C2", n=None, n_seeds=20, eps_list=(0.03, 0.05, 0.1, 0.25), z=0.0
     import tracegen as G
 
     sp = G.spec(config, n=n)
-    kid_np, t_np, _ = G.generate_np(sp)
-    kid = torch.from_numpy(kid_np.view(np.int32)).cuda()
-    t = torch.from_numpy(t_np.view(np.int32)).cuda()
+    if sp.n > 50_000_000 and not sp.n_metrics:   # bench-size traces: the byte-identical CUDA twin
+        kid = torch.empty(sp.n, dtype=torch.int32, device="cuda")
+        t = torch.empty(sp.n, dtype=torch.int32, device="cuda")
+        G.generate_cuda(G.DeviceSpec(sp, "cuda"), kid, t)
+    else:
+        kid_np, t_np, _ = G.generate_np(sp)
+        kid = torch.from_numpy(kid_np.view(np.int32)).cuda()
+        t = torch.from_numpy(t_np.view(np.int32)).cuda()
     t64 = t.to(torch.int64) & 0xFFFFFFFF
     total = int(t64.sum().item())
     seeds = [1000 + i for i in range(n_seeds)]
